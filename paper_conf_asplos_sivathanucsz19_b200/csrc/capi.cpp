@@ -1,0 +1,360 @@
+// L3: the C ABI (include/astra.h).  Every entry point converts C++ exceptions into status codes;
+// argument and state errors are raised before any device work is enqueued.
+#include <nccl.h>
+
+#include <cstring>
+#include <memory>
+#include <string>
+
+#include "common.h"
+#include "runtime/cell.h"
+#include "tuner/tuner.h"
+
+namespace astra {
+std::atomic<uint64_t> g_launches{0};
+static thread_local std::string t_err;
+void set_error(const std::string& s) { t_err = s; }
+}  // namespace astra
+
+using namespace astra;
+
+struct astra_cell_s {
+  std::unique_ptr<Cell> c;
+};
+struct astra_lm_s {
+  std::unique_ptr<LM> m;
+};
+
+template <class F>
+static astra_status guard(F&& f) {
+  try {
+    f();
+    return ASTRA_OK;
+  } catch (const Error& e) {
+    set_error(e.what());
+    return e.code;
+  } catch (const std::exception& e) {
+    set_error(e.what());
+    return ASTRA_E_ARG;
+  } catch (...) {
+    set_error("unknown error");
+    return ASTRA_E_ARG;
+  }
+}
+
+#define NEED(p) do { if (!(p)) throw Error(ASTRA_E_ARG, #p " is null"); } while (0)
+
+extern "C" {
+
+astra_status astra_cell_create_ex(astra_cell* out, const astra_cell_desc* d) {
+  return guard([&] {
+    NEED(out); NEED(d);
+    astra_cell_desc dd = *d;
+    if (dd.depth <= 0) dd.depth = 10;
+    if (dd.context <= 0) dd.context = dd.hidden;
+    if (dd.scrn_alpha == 0.f) dd.scrn_alpha = 0.95f;
+    if (dd.src_seq <= 0) dd.src_seq = dd.seq;
+    if (dd.attn_dim <= 0) dd.attn_dim = dd.hidden;
+    auto h = std::make_unique<astra_cell_s>();
+    h->c.reset(new Cell(dd));
+    *out = h.release();
+  });
+}
+
+astra_status astra_cell_create(astra_cell* out, int cell_type, int hidden, int input, int batch, int seq) {
+  astra_cell_desc d;
+  std::memset(&d, 0, sizeof(d));
+  d.cell_type = cell_type; d.hidden = hidden; d.input = input; d.batch = batch; d.seq = seq;
+  d.dtype = ASTRA_BF16;
+  return astra_cell_create_ex(out, &d);
+}
+
+astra_status astra_cell_destroy(astra_cell c) {
+  return guard([&] { delete c; });
+}
+
+astra_status astra_param_count(astra_cell c, size_t* n) {
+  return guard([&] { NEED(c); NEED(n); *n = c->c->n_params; });
+}
+
+astra_status astra_param_info(astra_cell c, int idx, const char** name, size_t* offset, int* rows, int* cols) {
+  return guard([&] {
+    NEED(c);
+    auto& ps = c->c->params;
+    if (idx < 0 || idx >= (int)ps.size()) throw Error(ASTRA_E_ARG, "param index out of range");
+    if (name) *name = ps[idx].name.c_str();
+    if (offset) *offset = ps[idx].offset;
+    if (rows) *rows = ps[idx].rows;
+    if (cols) *cols = ps[idx].cols;
+  });
+}
+
+astra_status astra_workspace_size(astra_cell c, size_t* saved, size_t* scratch) {
+  return guard([&] {
+    NEED(c);
+    if (saved) *saved = c->c->saved_bytes;
+    if (scratch) *scratch = c->c->scratch_bytes;
+  });
+}
+
+astra_status astra_bind(astra_cell c, float* params, float* grads, void* saved, void* scratch) {
+  return guard([&] { NEED(c); c->c->bind(params, grads, saved, scratch); });
+}
+
+astra_status astra_set_streams(astra_cell c, astra_stream main, const astra_stream* side, int n_side, astra_stream comm) {
+  return guard([&] {
+    NEED(c);
+    ASTRA_CHECK_ARG(n_side >= 0 && (n_side == 0 || side), "set_streams: bad side streams");
+    c->c->main_st = (cudaStream_t)main;
+    c->c->side.clear();
+    for (int i = 0; i < n_side; ++i) c->c->side.push_back((cudaStream_t)side[i]);
+    c->c->comm_st = (cudaStream_t)comm;
+  });
+}
+
+astra_status astra_step_fwd(astra_cell c, const void* x, const float* h0, const float* c0, void* y, float* hT,
+                            float* cT) {
+  return guard([&] {
+    NEED(c);
+    ASTRA_CHECK_STATE(!c->c->lm_mode, "step_fwd: cell is owned by an LM");
+    c->c->forward(x, h0, c0, y, hT, cT);
+  });
+}
+
+astra_status astra_step_bwd(astra_cell c, const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0,
+                            float* dc0) {
+  return guard([&] {
+    NEED(c);
+    ASTRA_CHECK_STATE(!c->c->lm_mode, "step_bwd: cell is owned by an LM");
+    c->c->backward(dy, dhT, dcT, dx, dh0, dc0);
+  });
+}
+
+astra_status astra_sgd(astra_cell c, float lr) {
+  return guard([&] { NEED(c); c->c->sgd_step(lr); });
+}
+
+astra_status astra_tune_next(astra_cell c, int* state) {
+  return guard([&] {
+    NEED(c);
+    int s = c->c->tune_next();
+    if (state) *state = s;
+  });
+}
+
+astra_status astra_tune_mode(astra_cell c, int mode, const char* forced) {
+  return guard([&] {
+    NEED(c);
+    Cell& cc = *c->c;
+    ASTRA_CHECK_ARG(mode == ASTRA_TUNE_OFF || mode == ASTRA_TUNE_ON || mode == ASTRA_TUNE_FROZEN, "tune_mode: bad mode");
+    if (mode == ASTRA_TUNE_OFF) {
+      cc.var = Variant();
+      cc.wirer.reset();
+    } else if (mode == ASTRA_TUNE_ON) {
+      cc.wirer.reset();
+      cc.var = Variant();
+    } else if (forced) {
+      Variant v;
+      std::string s(forced);
+      size_t p = 0;
+      while (p < s.size()) {
+        size_t q = s.find(',', p);
+        if (q == std::string::npos) q = s.size();
+        std::string kv = s.substr(p, q - p);
+        size_t eq = kv.find('=');
+        ASTRA_CHECK_ARG(eq != std::string::npos, "tune_mode: variant must be k=v,...");
+        std::string k = kv.substr(0, eq);
+        int val = std::stoi(kv.substr(eq + 1));
+        if (k == "bn_a1") v.bn_a1 = val;
+        else if (k == "bn_rec") v.bn_rec = val;
+        else if (k == "bn_bptt") v.bn_bptt = val;
+        else if (k == "bn_wg") v.bn_wg = val;
+        else if (k == "bn_dx") v.bn_dx = val;
+        else if (k == "bn_head") v.bn_head = val;
+        else if (k == "wg_side") v.wg_side = val;
+        else throw Error(ASTRA_E_ARG, "tune_mode: unknown variable " + k);
+        p = q + 1;
+      }
+      for (int bn : {v.bn_a1, v.bn_rec, v.bn_bptt, v.bn_wg, v.bn_dx, v.bn_head})
+        ASTRA_CHECK_ARG(bn == 64 || bn == 128 || bn == 256, "tune_mode: tile widths must be 64/128/256");
+      cc.var = v;
+    }
+    cc.tune_mode = mode;
+  });
+}
+
+astra_status astra_tune_report(astra_cell c, char* buf, size_t len, size_t* needed) {
+  return guard([&] {
+    NEED(c);
+    std::string r = c->c->report();
+    if (needed) *needed = r.size() + 1;
+    if (buf && len) {
+      size_t n = std::min(len - 1, r.size());
+      std::memcpy(buf, r.data(), n);
+      buf[n] = 0;
+    }
+  });
+}
+
+astra_status astra_comm_unique_id(void* out, size_t len) {
+  return guard([&] {
+    NEED(out);
+    ASTRA_CHECK_ARG(len >= sizeof(ncclUniqueId), "comm_unique_id: buffer too small");
+    ncclUniqueId id;
+    ncclResult_t r = ncclGetUniqueId(&id);
+    if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclGetUniqueId: ") + ncclGetErrorString(r));
+    std::memcpy(out, &id, sizeof(id));
+  });
+}
+
+astra_status astra_comm_init(astra_cell c, const void* uid, int rank, int world) {
+  return guard([&] {
+    NEED(c); NEED(uid);
+    ASTRA_CHECK_ARG(world >= 1 && rank >= 0 && rank < world, "comm_init: bad rank/world");
+    Cell& cc = *c->c;
+    CUDA_TRY(cudaSetDevice(cc.d.device));
+    ncclUniqueId id;
+    std::memcpy(&id, uid, sizeof(id));
+    ncclComm_t comm;
+    ncclResult_t r = ncclCommInitRank(&comm, world, id, rank);
+    if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+    if (cc.nccl_comm) ncclCommDestroy((ncclComm_t)cc.nccl_comm);
+    cc.nccl_comm = comm;
+    cc.rank = rank;
+    cc.world = world;
+  });
+}
+
+astra_status astra_lm_create(astra_lm* out, astra_cell c, int vocab) {
+  return guard([&] {
+    NEED(out); NEED(c);
+    auto h = std::make_unique<astra_lm_s>();
+    h->m.reset(new LM(c->c.get(), vocab));
+    *out = h.release();
+  });
+}
+
+astra_status astra_lm_destroy(astra_lm m) {
+  return guard([&] { delete m; });
+}
+
+astra_status astra_lm_param_count(astra_lm m, size_t* n) {
+  return guard([&] { NEED(m); NEED(n); *n = m->m->n_params; });
+}
+
+astra_status astra_lm_param_info(astra_lm m, int idx, const char** name, size_t* offset, int* rows, int* cols) {
+  return guard([&] {
+    NEED(m);
+    auto& ps = m->m->params;
+    if (idx < 0 || idx >= (int)ps.size()) throw Error(ASTRA_E_ARG, "param index out of range");
+    if (name) *name = ps[idx].name.c_str();
+    if (offset) *offset = ps[idx].offset;
+    if (rows) *rows = ps[idx].rows;
+    if (cols) *cols = ps[idx].cols;
+  });
+}
+
+astra_status astra_lm_workspace_size(astra_lm m, size_t* bytes) {
+  return guard([&] { NEED(m); NEED(bytes); *bytes = m->m->ws_bytes; });
+}
+
+astra_status astra_lm_bind(astra_lm m, float* params, float* grads, void* ws) {
+  return guard([&] { NEED(m); m->m->bind(params, grads, ws); });
+}
+
+astra_status astra_lm_set_state(astra_lm m, const float* h, const float* c) {
+  return guard([&] { NEED(m); m->m->set_state(h, c); });
+}
+
+astra_status astra_lm_train_step(astra_lm m, const int32_t* tokens, float lr, float* loss_dev) {
+  return guard([&] { NEED(m); m->m->step(tokens, lr, loss_dev, true); });
+}
+
+astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev) {
+  return guard([&] { NEED(m); m->m->step(tokens, 0.f, loss_dev, false); });
+}
+
+astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long lda, const void* Bp, int b_mn,
+                             long ldb, float* C, long ldc, int bn, astra_stream stream) {
+  return guard([&] {
+    NEED(A); NEED(Bp); NEED(C);
+    ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "gemm: sizes must be positive");
+    ASTRA_CHECK_ARG(ldc >= N, "gemm: ldc < N");
+    Mat2 a, b;
+    a.ptr = A; a.ld = lda;
+    if (a_mn) { a.inner = M; a.outer = K; } else { a.inner = K; a.outer = M; }
+    b.ptr = Bp; b.ld = ldb;
+    if (b_mn) { b.inner = N; b.outer = K; } else { b.inner = K; b.outer = N; }
+    ASTRA_CHECK_ARG(lda >= a.inner && ldb >= b.inner, "gemm: leading dimension too small");
+    TcGemm g;
+    tc_gemm_prepare(g, a, a_mn != 0, b, b_mn != 0, M, N, K, bn);
+    EpiStore e;
+    e.C = C; e.ldc = ldc; e.Mv = M; e.Nv = N; e.out_bf16 = 0; e.bias = nullptr; e.perm_u = 0; e.perm_H = 0;
+    tc_gemm_launch(g, e, 0, 0, (cudaStream_t)stream);
+  });
+}
+
+const char* astra_status_string(astra_status s) {
+  switch (s) {
+    case ASTRA_OK: return "ASTRA_OK";
+    case ASTRA_E_ARG: return "ASTRA_E_ARG";
+    case ASTRA_E_UNSUPPORTED: return "ASTRA_E_UNSUPPORTED";
+    case ASTRA_E_STATE: return "ASTRA_E_STATE";
+    case ASTRA_E_CUDA: return "ASTRA_E_CUDA";
+    case ASTRA_E_NCCL: return "ASTRA_E_NCCL";
+    case ASTRA_E_WORKSPACE: return "ASTRA_E_WORKSPACE";
+    default: return "ASTRA_E_UNKNOWN";
+  }
+}
+
+const char* astra_last_error(void) { return t_err.c_str(); }
+
+uint64_t astra_kernel_launch_count(void) { return g_launches.load(); }
+
+astra_status astra_region_times(astra_cell c, double* out, int cap, int* n) {
+  return guard([&] {
+    NEED(c); NEED(out);
+    Cell& cc = *c->c;
+    ASTRA_CHECK_STATE(cc.bound, "region_times: not bound");
+    CUDA_TRY(cudaEventSynchronize(cc.ev[R_STEP][1]));
+    int k = 0;
+    for (int r = 0; r < R_COUNT && k < cap; ++r, ++k) {
+      float ms = 0.f;
+      if (cc.region_used[r] && cudaEventElapsedTime(&ms, cc.ev[r][0], cc.ev[r][1]) != cudaSuccess) {
+        cudaGetLastError();
+        ms = 0.f;
+      }
+      out[k] = cc.region_used[r] ? ms : 0.0;
+    }
+    if (n) *n = k;
+  });
+}
+
+astra_status astra_tuner_selftest(const char* tree, astra_fake_cost_fn cost, void* user, int* trials_out,
+                                  int max_trials, int* n_trials, int* final_out, int* n_avs) {
+  return guard([&] {
+    NEED(tree); NEED(cost);
+    tuner::Tree t = tuner::parse(tree);
+    tuner::Wirer w(&t);
+    w.start();
+    tuner::Config c;
+    int k = 0;
+    const int na = (int)t.avs.size();
+    tuner::Metrics m(t.metrics.size(), 0.0);
+    while (w.propose(c)) {
+      if (trials_out && k < max_trials)
+        for (int i = 0; i < na; ++i) trials_out[k * na + i] = c[i];
+      cost(c.data(), na, m.data(), (int)m.size(), user);
+      w.feed(m);
+      ++k;
+    }
+    if (n_trials) *n_trials = k;
+    if (n_avs) *n_avs = na;
+    if (final_out) {
+      tuner::Config f = w.final_config();
+      for (int i = 0; i < na; ++i) final_out[i] = f[i];
+    }
+  });
+}
+
+}  // extern "C"

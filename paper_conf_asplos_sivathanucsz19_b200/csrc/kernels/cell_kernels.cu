@@ -1,0 +1,524 @@
+// Pointwise cell kernels (unfused halves of K2/K4), K5 fixed-order reductions, K6 embedding,
+// K7 cross-entropy, K9 SGD and operand mirrors.
+#include <cub/device/device_radix_sort.cuh>
+
+#include "cell_math.cuh"
+#include "kernels.h"
+
+namespace astra {
+
+// ============================================================================ mirrors
+template <typename T>
+__global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int H, int Hp, T* __restrict__ dst,
+                                      long ldd) {
+  // tile 32 (k) x 32 (internal rows r); dst[r][k] = src[k][ext(r)]
+  __shared__ float tile[32][33];
+  const int r0 = blockIdx.x * 32, k0 = blockIdx.y * 32;
+  const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
+  for (int i = ty; i < 32; i += 8) {
+    const int k = k0 + i, r = r0 + tx;
+    const int tileu = r / (4 * GATE_U), g = (r % (4 * GATE_U)) / GATE_U, j = tileu * GATE_U + r % GATE_U;
+    float v = 0.f;
+    if (k < K && j < H) v = src[(long)k * 4 * H + g * H + j];
+    tile[i][tx] = v;
+  }
+  __syncthreads();
+  for (int i = ty; i < 32; i += 8) {
+    const int r = r0 + i, k = k0 + tx;
+    if (r < 4 * Hp && k < ldd) dst[(long)r * ldd + k] = from_f<T>(tile[tx][i]);
+  }
+}
+
+void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st) {
+  dim3 grid(cdiv(4L * Hp, 32), cdiv(ldd, 32)), block(32, 8);
+  if (ot == OT::BF16)
+    mirror_gates_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd);
+  else
+    mirror_gates_T_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd);
+  LAUNCH_CHECK();
+}
+
+template <typename T>
+__global__ void mirror_T_kernel(const float* __restrict__ src, int K, int N, int Np, int Kp, T* __restrict__ dst,
+                                long ldd) {
+  __shared__ float tile[32][33];
+  const int n0 = blockIdx.x * 32, k0 = blockIdx.y * 32;
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  for (int i = ty; i < 32; i += 8) {
+    const int k = k0 + i, n = n0 + tx;
+    tile[i][tx] = (k < K && n < N) ? src[(long)k * N + n] : 0.f;
+  }
+  __syncthreads();
+  for (int i = ty; i < 32; i += 8) {
+    const int n = n0 + i, k = k0 + tx;
+    if (n < Np && k < Kp) dst[(long)n * ldd + k] = from_f<T>(tile[tx][i]);
+  }
+}
+
+void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, long ldd, cudaStream_t st) {
+  dim3 grid(cdiv(Np, 32), cdiv(Kp, 32)), block(32, 8);
+  if (ot == OT::BF16)
+    mirror_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, N, Np, Kp, (__nv_bfloat16*)dst, ldd);
+  else
+    mirror_T_kernel<float><<<grid, block, 0, st>>>(src, K, N, Np, Kp, (float*)dst, ldd);
+  LAUNCH_CHECK();
+}
+
+template <typename TD, typename TS>
+__global__ void copy_pad_kernel(const TS* __restrict__ src, long rows, int cols, long lds, TD* __restrict__ dst,
+                                long ldd) {
+  const long r = blockIdx.y;
+  for (long c = blockIdx.x * blockDim.x + threadIdx.x; c < ldd; c += (long)gridDim.x * blockDim.x) {
+    float v = (c < cols && src) ? to_f<TS>(src[r * lds + c]) : 0.f;
+    dst[r * ldd + c] = from_f<TD>(v);
+  }
+}
+
+void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, void* dst, long ldd, cudaStream_t st) {
+  if (rows == 0) return;
+  ASTRA_CHECK_ARG(rows < 65536L * 32768L, "copy_pad: too many rows");
+  // grid.y is limited to 65535: fold rows into chunks
+  const long ychunk = 65535;
+  for (long r0 = 0; r0 < rows; r0 += ychunk) {
+    const long nr = rows - r0 < ychunk ? rows - r0 : ychunk;
+    dim3 grid(cdiv(ldd, 256) < 8 ? cdiv(ldd, 256) : 8, (unsigned)nr);
+    const size_t es = ot_size(src_ot), ed = ot_size(ot);
+    const char* s = (const char*)src + (src ? r0 * lds * es : 0);
+    char* d = (char*)dst + r0 * ldd * ed;
+    if (ot == OT::BF16 && src_ot == OT::BF16)
+      copy_pad_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)(src ? s : nullptr), nr, cols, lds, (__nv_bfloat16*)d, ldd);
+    else if (ot == OT::BF16)
+      copy_pad_kernel<__nv_bfloat16, float><<<grid, 256, 0, st>>>((const float*)(src ? s : nullptr), nr, cols, lds, (__nv_bfloat16*)d, ldd);
+    else if (src_ot == OT::BF16)
+      copy_pad_kernel<float, __nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)(src ? s : nullptr), nr, cols, lds, (float*)d, ldd);
+    else
+      copy_pad_kernel<float, float><<<grid, 256, 0, st>>>((const float*)(src ? s : nullptr), nr, cols, lds, (float*)d, ldd);
+    LAUNCH_CHECK();
+  }
+}
+
+void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, long ldd, int dcols, cudaStream_t st) {
+  // dst has `dcols` used columns (≤ ldd); columns ≥ cols are zero
+  (void)dcols;
+  copy_pad(OT::F32, src, OT::F32, rows, cols, lds, dst, ldd, st);
+}
+
+// ============================================================================ LSTM-family pointwise
+template <int KIND, typename T, typename TY>
+__global__ void lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ WX, const float* __restrict__ UH,
+                                   GateParams gp, const float* __restrict__ c_prev, float* __restrict__ c_new,
+                                   T* __restrict__ h_op, TY* __restrict__ y, long ldy, float* __restrict__ hT,
+                                   float* __restrict__ cT) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  const int b = blockIdx.y;
+  if (j >= Hp) return;
+  const long rowg = (long)b * 4 * Hp, rowh = (long)b * Hp;
+  if (j >= H) {  // keep padding units exactly zero
+    c_new[rowh + j] = 0.f;
+    h_op[rowh + j] = from_f<T>(0.f);
+    return;
+  }
+  float a[4];
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    const int col = gcol(g, j), e = g * H + j;
+    const float wx = WX[rowg + col], uh = UH[rowg + col];
+    a[g] = preact<KIND>(wx, uh, gp.b[e], KIND == K_MILSTM ? gp.alpha[e] : 0.f, KIND == K_MILSTM ? gp.beta1[e] : 0.f,
+                        KIND == K_MILSTM ? gp.beta2[e] : 0.f);
+  }
+  float c, h;
+  cell_fwd<KIND>(a, c_prev[rowh + j], c, h);
+  c_new[rowh + j] = c;
+  h_op[rowh + j] = from_f<T>(h);
+  if (y) y[(long)b * ldy + j] = from_f<TY>(h);
+  if (hT) hT[(long)b * H + j] = h;
+  if (cT) cT[(long)b * H + j] = c;
+}
+
+template <int KIND, typename T>
+static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
+                          const float* c_prev, float* c_new, void* h_op, void* y, long ldy, float* hT, float* cT,
+                          cudaStream_t st) {
+  dim3 grid(cdiv(Hp, 128), B);
+  if (y_ot == OT::BF16)
+    lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
+                                                                     (__nv_bfloat16*)y, ldy, hT, cT);
+  else
+    lstm_fwd_pw_kernel<KIND, T, float><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
+                                                             (float*)y, ldy, hT, cT);
+  LAUNCH_CHECK();
+}
+
+void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
+                        const float* c_prev, float* c_new, void* h_op, void* y, long ldy, OT y_ot, float* hT,
+                        float* cT, cudaStream_t st) {
+#define FWD_CASE(K)                                                                                          \
+  if (kind == K) {                                                                                           \
+    if (ot == OT::BF16)                                                                                      \
+      fwd_pw_launch<K, __nv_bfloat16>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, y, ldy, hT, cT, st);  \
+    else                                                                                                     \
+      fwd_pw_launch<K, float>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, y, ldy, hT, cT, st);          \
+    return;                                                                                                  \
+  }
+  FWD_CASE(K_LSTM)
+  FWD_CASE(K_MILSTM)
+  FWD_CASE(K_SUBLSTM)
+#undef FWD_CASE
+  throw Error(ASTRA_E_UNSUPPORTED, "lstm_fwd_pointwise: kind");
+}
+
+constexpr int BWD_RB = 16;  // rows per CTA in the backward pointwise kernel
+int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
+
+// Thread = one hidden unit (all four gates), CTA row chunk of BWD_RB batch rows.  Column partial
+// sums (db, dα, dβ1, dβ2) are accumulated in registers over the chunk's rows in ascending order
+// and added to partials[chunk][q][col] — one owner per element, steps ordered on the stream, so
+// the reduction order is fixed (R5: no floating-point atomics).
+template <int KIND, typename T, typename TDY>
+__global__ void lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy,
+                                   const float* __restrict__ dh_rec, long ld_dh, float* __restrict__ dc,
+                                   const float* __restrict__ WX, const float* __restrict__ UH,
+                                   const float* __restrict__ c_new, const float* __restrict__ c_prev, GateParams gp,
+                                   T* __restrict__ D_uh, T* __restrict__ D_wx, float* __restrict__ partials, int nq,
+                                   int first) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  const int chunk = blockIdx.y;
+  if (j >= Hp) return;
+  const int NG = 4 * Hp;
+  const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
+  if (j >= H) {
+    for (int b = b0; b < b1; ++b) {
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        D_uh[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
+        if (KIND == K_MILSTM) D_wx[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
+      }
+      dc[(long)b * Hp + j] = 0.f;
+    }
+    return;
+  }
+  float s_b[4] = {0, 0, 0, 0}, s_al[4] = {0, 0, 0, 0}, s_b1[4] = {0, 0, 0, 0}, s_b2[4] = {0, 0, 0, 0};
+  float al[4], be1[4], be2[4], bb[4];
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    const int e = g * H + j;
+    bb[g] = gp.b[e];
+    al[g] = KIND == K_MILSTM ? gp.alpha[e] : 0.f;
+    be1[g] = KIND == K_MILSTM ? gp.beta1[e] : 0.f;
+    be2[g] = KIND == K_MILSTM ? gp.beta2[e] : 0.f;
+  }
+  for (int b = b0; b < b1; ++b) {
+    const long rg = (long)b * NG;
+    float wx[4], uh[4], a[4];
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      wx[g] = WX[rg + gcol(g, j)];
+      uh[g] = UH[rg + gcol(g, j)];
+      a[g] = preact<KIND>(wx[g], uh[g], bb[g], al[g], be1[g], be2[g]);
+    }
+    float dh = to_f<TDY>(dy[(long)b * ldy + j]);
+    if (dh_rec) dh = __fadd_rn(dh, dh_rec[(long)b * ld_dh + j]);
+    float dcv = dc[(long)b * Hp + j];
+    float da[4];
+    cell_bwd<KIND>(a, c_prev[(long)b * Hp + j], c_new[(long)b * Hp + j], dh, dcv, da);
+    dc[(long)b * Hp + j] = dcv;
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      s_b[g] = __fadd_rn(s_b[g], da[g]);
+      if (KIND == K_MILSTM) {
+        const float duh = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], wx[g]), be1[g]));
+        const float dwx = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], uh[g]), be2[g]));
+        D_uh[rg + gcol(g, j)] = from_f<T>(duh);
+        D_wx[rg + gcol(g, j)] = from_f<T>(dwx);
+        s_al[g] = __fadd_rn(s_al[g], __fmul_rn(__fmul_rn(da[g], wx[g]), uh[g]));
+        s_b1[g] = __fadd_rn(s_b1[g], __fmul_rn(da[g], uh[g]));
+        s_b2[g] = __fadd_rn(s_b2[g], __fmul_rn(da[g], wx[g]));
+      } else {
+        D_uh[rg + gcol(g, j)] = from_f<T>(da[g]);
+      }
+    }
+  }
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    const long base = (long)chunk * nq * NG + gcol(g, j);
+    float* p0 = partials + base;
+    *p0 = first ? s_b[g] : __fadd_rn(*p0, s_b[g]);
+    if (KIND == K_MILSTM) {
+      float* p1 = partials + base + NG;
+      float* p2 = partials + base + 2L * NG;
+      float* p3 = partials + base + 3L * NG;
+      *p1 = first ? s_al[g] : __fadd_rn(*p1, s_al[g]);
+      *p2 = first ? s_b1[g] : __fadd_rn(*p2, s_b1[g]);
+      *p3 = first ? s_b2[g] : __fadd_rn(*p3, s_b2[g]);
+    }
+  }
+}
+
+template <int KIND, typename T>
+static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32, const float* dh_rec,
+                          long ld_dh, float* dc, const float* WX, const float* UH, const float* c_new,
+                          const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
+                          bool first, cudaStream_t st) {
+  dim3 grid(cdiv(Hp, 128), lstm_bwd_row_chunks(B));
+  if (dy_f32 || dy_ot == OT::F32)
+    lstm_bwd_pw_kernel<KIND, T, float><<<grid, 128, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, dc, WX,
+                                                             UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials,
+                                                             nq, first);
+  else
+    lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, 128, 0, st>>>(B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec,
+                                                                     ld_dh, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh,
+                                                                     (T*)D_wx, partials, nq, first);
+  LAUNCH_CHECK();
+}
+
+void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
+                        const float* dh_rec, long ld_dh, float* dc, const float* WX, const float* UH,
+                        const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
+                        float* partials, int nq, bool first, cudaStream_t st) {
+#define BWD_CASE(K)                                                                                            \
+  if (kind == K) {                                                                                             \
+    if (ot == OT::BF16)                                                                                        \
+      bwd_pw_launch<K, __nv_bfloat16>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, dc, WX, UH, c_new, c_prev, \
+                                      gp, D_uh, D_wx, partials, nq, first, st);                                \
+    else                                                                                                       \
+      bwd_pw_launch<K, float>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, dc, WX, UH, c_new, c_prev, gp,  \
+                              D_uh, D_wx, partials, nq, first, st);                                            \
+    return;                                                                                                    \
+  }
+  BWD_CASE(K_LSTM)
+  BWD_CASE(K_MILSTM)
+  BWD_CASE(K_SUBLSTM)
+#undef BWD_CASE
+  throw Error(ASTRA_E_UNSUPPORTED, "lstm_bwd_pointwise: kind");
+}
+
+struct GradPtrs { float* p[4]; };
+
+__global__ void reduce_gate_partials_kernel(const float* __restrict__ partials, int nchunk, int nq, int H, int Hp,
+                                            GradPtrs out) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  const int q = blockIdx.y;
+  if (e >= 4 * H) return;
+  const int g = e / H, j = e % H;
+  const long NG = 4L * Hp;
+  const int col = gcol(g, j);
+  float s = 0.f;
+  for (int c = 0; c < nchunk; ++c) s = __fadd_rn(s, partials[((long)c * nq + q) * NG + col]);
+  out.p[q][e] = s;
+}
+
+void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,
+                          cudaStream_t st) {
+  GradPtrs gp{};
+  for (int q = 0; q < nq; ++q) gp.p[q] = grads_q[q];
+  dim3 grid(cdiv(4L * H, 256), nq);
+  reduce_gate_partials_kernel<<<grid, 256, 0, st>>>(partials, nchunk, nq, H, Hp, gp);
+  LAUNCH_CHECK();
+}
+
+// ============================================================================ LM pieces
+template <typename T>
+__global__ void embed_gather_kernel(const int32_t* __restrict__ tok, long n, const float* __restrict__ E, int I,
+                                    T* __restrict__ X, long ldx) {
+  const long r = blockIdx.x;
+  const long src = (long)tok[r] * I;
+  for (int c = threadIdx.x; c < ldx; c += blockDim.x) X[r * ldx + c] = from_f<T>(c < I ? E[src + c] : 0.f);
+}
+
+void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st) {
+  if (ot == OT::BF16)
+    embed_gather_kernel<__nv_bfloat16><<<(unsigned)n, 256, 0, st>>>(tok, n, E, I, (__nv_bfloat16*)X, ldx);
+  else
+    embed_gather_kernel<float><<<(unsigned)n, 256, 0, st>>>(tok, n, E, I, (float*)X, ldx);
+  LAUNCH_CHECK();
+}
+
+// one warp per row; fixed-order warp-shuffle trees
+template <typename T>
+__global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, const int32_t* __restrict__ targets,
+                          long n, float inv_n, float* __restrict__ rowloss, T* __restrict__ dlog, long ldd,
+                          float* __restrict__ dlog32) {
+  const long r = (long)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
+  const int lane = threadIdx.x % 32;
+  if (r >= n) return;
+  const float* row = logits + r * ldl;
+  float m = -INFINITY;
+  for (int c = lane; c < V; c += 32) m = fmaxf(m, row[c]);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  float s = 0.f;
+  for (int c = lane; c < V; c += 32) s = __fadd_rn(s, expf(__fsub_rn(row[c], m)));
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+  const float lse = __fadd_rn(m, logf(s));
+  const int tgt = targets[r];
+  if (lane == 0) rowloss[r] = __fsub_rn(lse, row[tgt]);
+  const float rs = __frcp_rn(s);
+  for (int c = lane; c < V; c += 32) {
+    float p = __fmul_rn(expf(__fsub_rn(row[c], m)), rs);
+    if (c == tgt) p = __fsub_rn(p, 1.f);
+    const float d = __fmul_rn(p, inv_n);
+    dlog[r * ldd + c] = from_f<T>(d);
+    dlog32[r * V + c] = d;
+  }
+  for (int c = V + lane; c < ldd; c += 32) dlog[r * ldd + c] = from_f<T>(0.f);
+}
+
+void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
+                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st) {
+  const int rows_per = 8;
+  dim3 grid(cdiv(n, rows_per));
+  if (ot == OT::BF16)
+    ce_kernel<__nv_bfloat16><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, rowloss,
+                                                             (__nv_bfloat16*)dlog, ldd, dlog32);
+  else
+    ce_kernel<float><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, rowloss, (float*)dlog, ldd,
+                                                     dlog32);
+  LAUNCH_CHECK();
+}
+
+__global__ void sum_scalar_kernel(const float* __restrict__ v, long n, float scale, float* __restrict__ out) {
+  __shared__ float sh[1024];
+  float s = 0.f;
+  for (long i = threadIdx.x; i < n; i += blockDim.x) s = __fadd_rn(s, v[i]);
+  sh[threadIdx.x] = s;
+  __syncthreads();
+  for (int w = blockDim.x / 2; w > 0; w >>= 1) {
+    if (threadIdx.x < w) sh[threadIdx.x] = __fadd_rn(sh[threadIdx.x], sh[threadIdx.x + w]);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *out = __fmul_rn(sh[0], scale);
+}
+
+void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st) {
+  sum_scalar_kernel<<<1, 1024, 0, st>>>(v, n, scale, out);
+  LAUNCH_CHECK();
+}
+
+constexpr int COLSUM_RB = 256;
+size_t colsum_scratch_floats(long rows, int cols) { return (size_t)cdiv(rows, COLSUM_RB) * cols; }
+
+__global__ void colsum_partial_kernel(const float* __restrict__ in, long rows, int cols, long ld,
+                                      float* __restrict__ part) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  const long r0 = (long)blockIdx.y * COLSUM_RB;
+  if (c >= cols) return;
+  const long r1 = min(rows, r0 + COLSUM_RB);
+  float s = 0.f;
+  for (long r = r0; r < r1; ++r) s = __fadd_rn(s, in[r * ld + c]);
+  part[(long)blockIdx.y * cols + c] = s;
+}
+__global__ void colsum_final_kernel(const float* __restrict__ part, int nchunk, int cols, float* __restrict__ out) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= cols) return;
+  float s = 0.f;
+  for (int k = 0; k < nchunk; ++k) s = __fadd_rn(s, part[(long)k * cols + c]);
+  out[c] = s;
+}
+
+void colsum(const float* in, long rows, int cols, long ld, float* scratch, float* out, cudaStream_t st) {
+  const int nchunk = cdiv(rows, COLSUM_RB);
+  colsum_partial_kernel<<<dim3(cdiv(cols, 128), nchunk), 128, 0, st>>>(in, rows, cols, ld, scratch);
+  LAUNCH_CHECK();
+  colsum_final_kernel<<<cdiv(cols, 128), 128, 0, st>>>(scratch, nchunk, cols, out);
+  LAUNCH_CHECK();
+}
+
+// ---- embedding backward: stable radix sort of (token, row) then ordered segment sums
+__global__ void iota_kernel(int32_t* v, long n) {
+  const long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) v[i] = (int32_t)i;
+}
+
+static int key_bits(int V) {
+  int b = 1;
+  while ((1L << b) < V) ++b;
+  return b;
+}
+
+size_t embed_bwd_scratch_bytes(long n, int V) {
+  size_t temp = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
+                                  (int32_t*)nullptr, (int)n, 0, key_bits(V));
+  return round_up(temp, 256) + 3 * round_up(n * 4, 256);
+}
+
+// dE rows: block (v, column chunk); rows of token v are the sorted range [lo, hi).
+__global__ void embed_bwd_kernel(const int32_t* __restrict__ skeys, const int32_t* __restrict__ srows, long n,
+                                 const float* __restrict__ dX, long ldx, int I, float* __restrict__ dE) {
+  const int v = blockIdx.y;
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  __shared__ long lo_hi[2];
+  if (threadIdx.x < 2) {
+    const int key = v + threadIdx.x;  // lower_bound(key)
+    long lo = 0, hi = n;
+    while (lo < hi) {
+      const long mid = (lo + hi) / 2;
+      if (skeys[mid] < key) lo = mid + 1; else hi = mid;
+    }
+    lo_hi[threadIdx.x] = lo;
+  }
+  __syncthreads();
+  if (c >= I) return;
+  float s = 0.f;
+  for (long k = lo_hi[0]; k < lo_hi[1]; ++k) s = __fadd_rn(s, dX[(long)srows[k] * ldx + c]);
+  dE[(long)v * I + c] = s;
+}
+
+void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int I, float* dE, void* scratch,
+               size_t scratch_bytes, cudaStream_t st) {
+  size_t temp = 0;
+  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
+                                  (int32_t*)nullptr, (int)n, 0, key_bits(V));
+  temp = round_up(temp, 256);
+  char* base = (char*)scratch;
+  const size_t nb = round_up(n * 4, 256);
+  ASTRA_CHECK_ARG(scratch_bytes >= temp + 3 * nb, "embed_bwd: scratch too small");
+  int32_t* rows_in = (int32_t*)(base + temp);
+  int32_t* skeys = (int32_t*)(base + temp + nb);
+  int32_t* srows = (int32_t*)(base + temp + 2 * nb);
+  iota_kernel<<<cdiv(n, 256), 256, 0, st>>>(rows_in, n);
+  LAUNCH_CHECK();
+  CUDA_TRY(cub::DeviceRadixSort::SortPairs(base, temp, tok, skeys, rows_in, srows, (int)n, 0, key_bits(V), st));
+  count_launch(4);
+  embed_bwd_kernel<<<dim3(cdiv(I, 256), V), 256, 0, st>>>(skeys, srows, n, dX, ldx, I, dE);
+  LAUNCH_CHECK();
+}
+
+// ============================================================================ SGD
+__global__ void sgd_kernel(float* __restrict__ p, const float* __restrict__ g, size_t n, float lr) {
+  const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const size_t n4 = n / 4;
+  if (i < n4) {
+    float4 a = reinterpret_cast<float4*>(p)[i];
+    const float4 b = reinterpret_cast<const float4*>(g)[i];
+    a.x = __fsub_rn(a.x, __fmul_rn(lr, b.x));
+    a.y = __fsub_rn(a.y, __fmul_rn(lr, b.y));
+    a.z = __fsub_rn(a.z, __fmul_rn(lr, b.z));
+    a.w = __fsub_rn(a.w, __fmul_rn(lr, b.w));
+    reinterpret_cast<float4*>(p)[i] = a;
+  }
+  if (i < n - n4 * 4) {
+    const size_t k = n4 * 4 + i;
+    p[k] = __fsub_rn(p[k], __fmul_rn(lr, g[k]));
+  }
+}
+
+void sgd(float* p, const float* g, size_t n, float lr, cudaStream_t st) {
+  if (!n) return;
+  const size_t n4 = n / 4 > 0 ? n / 4 : 1;
+  sgd_kernel<<<(unsigned)cdiv((long)n4, 256), 256, 0, st>>>(p, g, n, lr);
+  LAUNCH_CHECK();
+}
+
+__global__ void scale_kernel(float* p, size_t n, float s) {
+  const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = __fmul_rn(p[i], s);
+}
+void scale_inplace(float* p, size_t n, float s, cudaStream_t st) {
+  if (!n) return;
+  scale_kernel<<<(unsigned)cdiv((long)n, 256), 256, 0, st>>>(p, n, s);
+  LAUNCH_CHECK();
+}
+
+}  // namespace astra

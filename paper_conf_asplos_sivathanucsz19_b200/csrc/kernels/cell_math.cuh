@@ -1,0 +1,80 @@
+// Per-element cell arithmetic shared by every kernel variant of a precision path:
+// the unfused pointwise kernels and the fused GEMM epilogues call exactly these functions, written
+// with explicit round-to-nearest intrinsics so no variant can be contracted differently.
+#pragma once
+#include <cuda_bf16.h>
+
+namespace astra {
+
+// Internal gate-interleaved column order (the `alloc` layout, unit block u = 64):
+// internal column of (gate g, unit j) = (j / 64)·256 + g·64 + (j % 64).
+constexpr int GATE_U = 64;
+__host__ __device__ __forceinline__ int gcol(int g, int j) { return (j / GATE_U) * (4 * GATE_U) + g * GATE_U + (j % GATE_U); }
+
+__device__ __forceinline__ float sigm(float x) { return __frcp_rn(__fadd_rn(1.f, expf(-x))); }
+__device__ __forceinline__ float tanh_(float x) { return tanhf(x); }
+
+template <typename T> __device__ __forceinline__ float to_f(T v);
+template <> __device__ __forceinline__ float to_f<float>(float v) { return v; }
+template <> __device__ __forceinline__ float to_f<__nv_bfloat16>(__nv_bfloat16 v) { return __bfloat162float(v); }
+template <typename T> __device__ __forceinline__ T from_f(float v);
+template <> __device__ __forceinline__ float from_f<float>(float v) { return v; }
+template <> __device__ __forceinline__ __nv_bfloat16 from_f<__nv_bfloat16>(float v) { return __float2bfloat16_rn(v); }
+
+enum CellKind { K_LSTM = 0, K_MILSTM = 1, K_SUBLSTM = 5 };
+
+// Pre-activation of one gate.  LSTM/subLSTM: a = wx + uh + b.
+// MI-LSTM [36]: a = α·wx·uh + β1·uh + β2·wx + b  (reading R3/R4), evaluated left to right.
+template <int KIND>
+__device__ __forceinline__ float preact(float wx, float uh, float b, float al, float b1, float b2) {
+  if (KIND == K_MILSTM) {
+    float a = __fmul_rn(__fmul_rn(al, wx), uh);
+    a = __fadd_rn(a, __fmul_rn(b1, uh));
+    a = __fadd_rn(a, __fmul_rn(b2, wx));
+    return __fadd_rn(a, b);
+  } else {
+    return __fadd_rn(__fadd_rn(wx, uh), b);
+  }
+}
+
+// Forward cell update from the four pre-activations.  Returns (c_new, h_new).
+template <int KIND>
+__device__ __forceinline__ void cell_fwd(const float (&a)[4], float c_prev, float& c_new, float& h_new) {
+  if (KIND == K_SUBLSTM) {
+    const float i = sigm(a[0]), f = sigm(a[1]), z = sigm(a[2]), o = sigm(a[3]);
+    c_new = __fsub_rn(__fadd_rn(__fmul_rn(f, c_prev), z), i);
+    h_new = __fsub_rn(sigm(c_new), o);
+  } else {
+    const float i = sigm(a[0]), f = sigm(a[1]), g = tanh_(a[2]), o = sigm(a[3]);
+    c_new = __fadd_rn(__fmul_rn(f, c_prev), __fmul_rn(i, g));
+    h_new = __fmul_rn(o, tanh_(c_new));
+  }
+}
+
+// Backward of one cell update.  dh = dL/dh_t, dc = dL/dc_t from step t+1 (in/out: becomes
+// dL/dc_{t-1}).  da[4] = dL/da for the four gates.
+template <int KIND>
+__device__ __forceinline__ void cell_bwd(const float (&a)[4], float c_prev, float c_new, float dh, float& dc,
+                                         float (&da)[4]) {
+  if (KIND == K_SUBLSTM) {
+    const float i = sigm(a[0]), f = sigm(a[1]), z = sigm(a[2]), o = sigm(a[3]);
+    const float sc = sigm(c_new);
+    const float dcc = __fadd_rn(dc, __fmul_rn(dh, __fmul_rn(sc, __fsub_rn(1.f, sc))));
+    da[0] = __fmul_rn(-dcc, __fmul_rn(i, __fsub_rn(1.f, i)));
+    da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), __fmul_rn(f, __fsub_rn(1.f, f)));
+    da[2] = __fmul_rn(dcc, __fmul_rn(z, __fsub_rn(1.f, z)));
+    da[3] = __fmul_rn(-dh, __fmul_rn(o, __fsub_rn(1.f, o)));
+    dc = __fmul_rn(dcc, f);
+  } else {
+    const float i = sigm(a[0]), f = sigm(a[1]), g = tanh_(a[2]), o = sigm(a[3]);
+    const float tau = tanh_(c_new);
+    const float dcc = __fadd_rn(dc, __fmul_rn(__fmul_rn(dh, o), __fsub_rn(1.f, __fmul_rn(tau, tau))));
+    da[0] = __fmul_rn(__fmul_rn(dcc, g), __fmul_rn(i, __fsub_rn(1.f, i)));
+    da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), __fmul_rn(f, __fsub_rn(1.f, f)));
+    da[2] = __fmul_rn(__fmul_rn(dcc, i), __fsub_rn(1.f, __fmul_rn(g, g)));
+    da[3] = __fmul_rn(__fmul_rn(dh, tau), __fmul_rn(o, __fsub_rn(1.f, o)));
+    dc = __fmul_rn(dcc, f);
+  }
+}
+
+}  // namespace astra

@@ -1,0 +1,187 @@
+// Host side of K1 (tcgen05 GEMM) and K10 (SIMT fp32 GEMM).
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <mutex>
+
+#include "../common.h"
+#include "gemm.h"
+
+namespace astra {
+
+int num_sms() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev));
+  }
+  return n;
+}
+
+static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  if (!fn) throw Error(ASTRA_E_CUDA, "cuTensorMapEncodeTiled unavailable (driver too old?)");
+  return fn;
+}
+
+static void make_map(CUtensorMap* m, const Mat2& t, int box_inner, int box_outer) {
+  ASTRA_CHECK_ARG(t.ptr != nullptr, "tensor map: null pointer");
+  ASTRA_CHECK_ARG(((uintptr_t)t.ptr & 15) == 0, "tensor map: base must be 16-byte aligned");
+  ASTRA_CHECK_ARG((t.ld * 2) % 16 == 0, "tensor map: row stride must be a multiple of 16 bytes");
+  ASTRA_CHECK_ARG(t.z == 1 || (t.zstride * 2) % 16 == 0, "tensor map: z stride must be a multiple of 16 bytes");
+  cuuint64_t dims[3] = {(cuuint64_t)t.inner, (cuuint64_t)t.outer, (cuuint64_t)t.z};
+  cuuint64_t strides[2] = {(cuuint64_t)(t.ld * 2), (cuuint64_t)((t.z > 1 ? t.zstride : t.ld * t.outer) * 2)};
+  cuuint32_t box[3] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = encode_fn()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(t.ptr), dims, strides, box,
+                           estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(ASTRA_E_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
+}
+
+static uint32_t make_idesc(int BN, bool a_mn, bool b_mn) {
+  uint32_t d = 0;
+  d |= 1u << 4;                      // D format: F32
+  d |= 1u << 7;                      // A format: BF16
+  d |= 1u << 10;                     // B format: BF16
+  d |= (a_mn ? 1u : 0u) << 15;       // A major
+  d |= (b_mn ? 1u : 0u) << 16;       // B major
+  d |= (uint32_t)(BN >> 3) << 17;    // N >> 3
+  d |= (uint32_t)(TC_BM >> 4) << 24; // M >> 4
+  return d;
+}
+
+template <int BN>
+static int smem_for(int& stages) {
+  int dev = 0, maxs = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  stages = TcSmem<BN>::stages_for(maxs);
+  if (stages > 4) stages = 4;
+  return TcSmem<BN>::bytes(stages);
+}
+
+void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN) {
+  ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256, "tc_gemm: BN must be 64, 128 or 256");
+  ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
+  if (a_mn) make_map(&g.mapA, A, 64, 64); else make_map(&g.mapA, A, 64, TC_BM);
+  if (b_mn) make_map(&g.mapB, B, 64, 64); else make_map(&g.mapB, B, 64, BN);
+  g.BN = BN;
+  g.args.M = M; g.args.N = N; g.args.K = K;
+  g.args.num_m = cdiv(M, TC_BM);
+  g.args.num_n = cdiv(N, BN);
+  g.args.az = g.args.bz = 0;
+  g.args.a_mn = a_mn; g.args.b_mn = b_mn;
+  g.args.idesc = make_idesc(BN, a_mn, b_mn);
+  int stages = 0;
+  switch (BN) {
+    case 64: g.smem = smem_for<64>(stages); break;
+    case 128: g.smem = smem_for<128>(stages); break;
+    default: g.smem = smem_for<256>(stages); break;
+  }
+  g.args.stages = stages;
+  g.ready = true;
+}
+
+template <int BN>
+static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
+  static int attr_bytes = 0;
+  if (g.smem > attr_bytes) {
+    CUDA_TRY(cudaFuncSetAttribute(tc_gemm_kernel<BN, EpiStore>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  g.smem));
+    attr_bytes = g.smem;
+  }
+  TcArgs a = g.args;
+  a.az = az;
+  a.bz = bz;
+  const int tiles = a.num_m * a.num_n;
+  int grid = num_sms();
+  if (max_ctas > 0 && max_ctas < grid) grid = max_ctas;
+  if (tiles < grid) grid = tiles;
+  tc_gemm_kernel<BN, EpiStore><<<grid, TC_THREADS, g.smem, st>>>(g.mapA, g.mapB, a, epi);
+  LAUNCH_CHECK();
+}
+
+void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
+  ASTRA_CHECK_STATE(g.ready, "tc_gemm: not prepared");
+  switch (g.BN) {
+    case 64: launch_bn<64>(g, epi, az, bz, st, max_ctas); break;
+    case 128: launch_bn<128>(g, epi, az, bz, st, max_ctas); break;
+    default: launch_bn<256>(g, epi, az, bz, st, max_ctas); break;
+  }
+}
+
+// ------------------------------------------------------------------------------ K10 SIMT
+// 64x64 output tile per 256-thread CTA, 4x4 per thread, k chunks of 16 staged in shared memory.
+// Each output element is one fp32 FMA chain over k = 0..K-1 in ascending order (R1/R2).
+__global__ void __launch_bounds__(256) simt_gemm_kernel(const float* __restrict__ A, long sam, long sak,
+                                                        const float* __restrict__ B, long sbk, long sbn, int M,
+                                                        int N, int K, EpiStore epi) {
+  __shared__ float As[16][64 + 1];
+  __shared__ float Bs[16][64 + 1];
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  const int m0 = blockIdx.y * 64, n0 = blockIdx.x * 64;
+  float acc[4][4] = {};
+  for (int k0 = 0; k0 < K; k0 += 16) {
+    for (int i = threadIdx.x; i < 16 * 64; i += 256) {
+      const int kk = i / 64, r = i % 64;
+      const int m = m0 + r, n = n0 + r, k = k0 + kk;
+      As[kk][r] = (m < M && k < K) ? A[(long)m * sam + (long)k * sak] : 0.f;
+      Bs[kk][r] = (n < N && k < K) ? B[(long)k * sbk + (long)n * sbn] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < 16; ++kk) {
+      float a[4], b[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) a[i] = As[kk][ty * 4 + i];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) b[j] = Bs[kk][tx * 4 + j];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = __fmaf_rn(a[i], b[j], acc[i][j]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int m = m0 + ty * 4 + i;
+    if (m >= M) continue;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int n = n0 + tx * 4 + j;
+      if (n >= N) continue;
+      int e = n;
+      bool ok = n < epi.Nv;
+      if (epi.perm_u) {
+        const int q = 4 * epi.perm_u;
+        const int tile = n / q, g = (n % q) / epi.perm_u, jj = n % epi.perm_u;
+        const int unit = tile * epi.perm_u + jj;
+        ok = unit < epi.perm_H;
+        e = g * epi.perm_H + unit;
+      }
+      if (!ok || m >= epi.Mv) continue;
+      const float v = __fadd_rn(acc[i][j], epi.bias ? epi.bias[n] : 0.f);
+      reinterpret_cast<float*>(epi.C)[(long)m * epi.ldc + e] = v;
+    }
+  }
+}
+
+void simt_gemm(const float* A, long sam, long sak, const float* B, long sbk, long sbn, int M, int N, int K,
+               const EpiStore& epi, cudaStream_t st) {
+  ASTRA_CHECK_ARG(!epi.out_bf16, "simt_gemm writes fp32");
+  dim3 grid(cdiv(N, 64), cdiv(M, 64));
+  simt_gemm_kernel<<<grid, 256, 0, st>>>(A, sam, sak, B, sbk, sbn, M, N, K, epi);
+  LAUNCH_CHECK();
+}
+
+}  // namespace astra

@@ -1,0 +1,61 @@
+// Host launch wrappers of the non-GEMM kernels (K2/K4 unfused pointwise halves, K5 reductions,
+// K6 embedding, K7 cross-entropy, K9 SGD + operand mirrors).  Every wrapper launches on `st`.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../common.h"
+
+namespace astra {
+
+struct GateParams {          // external-layout fp32 vectors of length 4H (may be null for LSTM)
+  const float* b = nullptr;
+  const float* alpha = nullptr;
+  const float* beta1 = nullptr;
+  const float* beta2 = nullptr;
+};
+
+// ---- mirrors (K9): fp32 params → operand-type copies in the internal layout
+// dst[gcol(g, j)][k] = src[k][g*H + j] for the gate-blocked [K][4H] matrix `src`
+// (dst rows = 4*Hp, row stride ldd ≥ K; padding rows/cols zero).
+void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st);
+// dst[n][k] = src[k][n] (plain transpose), dst [Np][ldd], padding zero.
+void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, long ldd, cudaStream_t st);
+// Operand copy of an external [rows][cols] (OT or fp32 `src_ot`) into [rows][ldd] of type `ot`.
+void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, void* dst, long ldd, cudaStream_t st);
+// dst fp32 [rows][ldd] ← src fp32 [rows][lds] (cols), zero padding; src null → zeros.
+void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, long ldd, int dcols, cudaStream_t st);
+
+// ---- LSTM-family pointwise halves (cell kind: 0 LSTM, 1 MI-LSTM, 5 subLSTM)
+void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
+                        const float* c_prev, float* c_new, void* h_op, void* y, long ldy, OT y_ot, float* hT,
+                        float* cT, cudaStream_t st);
+// dy: row stride ldy of type dy_ot (or fp32); dh_rec: [B][ld_dh] fp32 or null (zeros).
+void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
+                        const float* dh_rec, long ld_dh, float* dc, const float* WX, const float* UH,
+                        const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
+                        float* partials, int nq, bool first, cudaStream_t st);
+int lstm_bwd_row_chunks(int B);
+// grads_q[e] = Σ_chunk partials[chunk][q][gcol(e)] for q < nq (external e < 4H).
+void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,
+                          cudaStream_t st);
+
+// ---- LM pieces
+void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);
+// rowloss[r] = lse - logit[target]; dlog (ot) and dlog32 = (softmax - onehot) * inv_n.
+void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
+                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st);
+void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st);
+// out[c] = Σ_r in[r][c] over rows in fixed order (two-level); scratch ≥ colsum_scratch(rows, cols)
+size_t colsum_scratch_floats(long rows, int cols);
+void colsum(const float* in, long rows, int cols, long ld, float* scratch, float* out, cudaStream_t st);
+// Deterministic embedding backward: dE[v] = Σ_{rows with tok=v} dX[row] in ascending row order.
+size_t embed_bwd_scratch_bytes(long n, int V);
+void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int I, float* dE, void* scratch,
+               size_t scratch_bytes, cudaStream_t st);
+
+// ---- SGD (K9): p -= lr * g over n elements
+void sgd(float* p, const float* g, size_t n, float lr, cudaStream_t st);
+void scale_inplace(float* p, size_t n, float s, cudaStream_t st);
+
+}  // namespace astra

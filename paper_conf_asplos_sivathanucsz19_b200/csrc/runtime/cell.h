@@ -1,0 +1,146 @@
+// L1 runtime: per-cell step plan, workspace carving, the executor of one training step for each
+// variant, and the LM wrapper.  The tuner (L2) chooses the Variant; every variant computes the
+// same bits (R1-R7).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <map>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../common.h"
+#include "../kernels/gemm.h"
+#include "../kernels/kernels.h"
+#include "../tuner/tuner.h"
+
+namespace astra {
+
+struct ParamInfo {
+  std::string name;
+  size_t offset;
+  int rows, cols;
+};
+
+// One binding of every adaptive variable (the enumerator's output for this cell, §8(a.9)).
+struct Variant {
+  int bn_a1 = 256;      // hoisted input projection tile width (K1)
+  int bn_rec = 256;     // per-step recurrent GEMM tile width (K2)
+  int bn_bptt = 128;    // per-step BPTT dgrad GEMM tile width (K4)
+  int bn_wg = 256;      // weight-gradient GEMMs (a6)
+  int bn_dx = 256;      // input dgrad GEMM (a6)
+  int bn_head = 256;    // LM head GEMMs (a4)
+  int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
+  std::string str() const;
+};
+
+// GEMM problem in storage terms; drives both engines (tcgen05 for bf16, SIMT for fp32).
+struct GemmSpec {
+  Mat2 A, B;
+  bool a_mn = false, b_mn = false;
+  int M = 0, N = 0, K = 0;
+};
+
+enum Region { R_A1 = 0, R_FWD, R_HEAD, R_BPTT, R_DU, R_DW, R_DX, R_SE4, R_STEP, R_COUNT };
+
+class Cell {
+ public:
+  explicit Cell(const astra_cell_desc& d);
+  ~Cell();
+
+  astra_cell_desc d;
+  int kind;
+  OT ot;
+  int H, I, B, T, Hp, Ip, NG, Hout;
+  std::vector<ParamInfo> params;
+  size_t n_params = 0;
+
+  // workspace layout (byte offsets)
+  size_t off_X, off_WX, off_UH, off_C, off_H, off_Wm, off_Um, saved_bytes;
+  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part, off_dXf, scratch_bytes;
+  int nchunk;
+
+  // binding
+  float* P = nullptr;
+  float* G = nullptr;
+  char* saved = nullptr;
+  char* scratch = nullptr;
+  bool bound = false, fwd_done = false;
+
+  // streams / events
+  cudaStream_t main_st = nullptr;
+  std::vector<cudaStream_t> side;
+  cudaStream_t comm_st = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+
+  // variant + tuner
+  Variant var;
+  int tune_mode = ASTRA_TUNE_OFF;
+  std::unique_ptr<tuner::Tree> tree;
+  std::unique_ptr<tuner::Wirer> wirer;
+  std::vector<Variant> configs_seen;
+  int tune_reps = 3, rep_i = 0;
+  tuner::Metrics rep_min;
+  bool step_pending = false;
+  cudaEvent_t ev[R_COUNT][2];
+  bool region_used[R_COUNT];
+  bool profiling = true;
+
+  // NCCL
+  void* nccl_comm = nullptr;
+  int rank = 0, world = 1;
+
+  // LM mode hooks (set by LM)
+  bool lm_mode = false;
+  const float* lm_dy = nullptr;  // fp32 [T*B][Hp] internal dY for backward
+
+  size_t find_param(const std::string& n) const;
+  float* p(const std::string& n) { return P + find_param(n); }
+  float* g(const std::string& n) { return G + find_param(n); }
+
+  void bind(float* params, float* grads, void* saved_p, void* scratch_p);
+  void forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT);
+  void backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0);
+  void sgd_step(float lr);
+  void allreduce_grads(float* grads, size_t n, cudaStream_t after);
+
+  // internal buffers
+  template <typename T> T* sv(size_t off) { return reinterpret_cast<T*>(saved + off); }
+  template <typename T> T* sc(size_t off) { return reinterpret_cast<T*>(scratch + off); }
+  size_t esz() const { return ot_size(ot); }
+  void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
+
+  // GEMM execution
+  void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, int BN, cudaStream_t st);
+  std::map<std::pair<int, int>, TcGemm> tc_cache;
+
+  // profiling regions (cudaEvent pairs)
+  void mark(Region r, int which, cudaStream_t st);
+  // tuner
+  void tuner_setup();
+  void apply_config(const tuner::Config& c);
+  int tune_next();
+  std::string report();
+};
+
+class LM {
+ public:
+  LM(Cell* c, int vocab);
+  Cell* cell;
+  int V, Vp;
+  size_t n_cell, n_params;
+  std::vector<ParamInfo> params;
+  size_t off_logits, off_dlog, off_dlog32, off_rowloss, off_dY, off_Wo, off_colsum, off_sort, off_h, off_c,
+      off_cellsaved, off_cellscratch, off_loss, ws_bytes;
+  size_t sort_bytes;
+  float* P = nullptr;
+  float* G = nullptr;
+  char* ws = nullptr;
+  bool bound = false;
+  size_t find(const std::string& n) const;
+  void bind(float* params, float* grads, void* workspace);
+  void set_state(const float* h, const float* c);
+  void step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd);
+};
+
+}  // namespace astra

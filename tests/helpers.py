@@ -1,0 +1,85 @@
+"""Shared test helpers: case construction from synth/, running the CUDA path through the binding,
+and the parity metric (reading R18: per-tensor relative L2 error ‖gpu − oracle‖₂ / ‖oracle‖₂)."""
+from __future__ import annotations
+
+import numpy as np
+
+import synth
+
+TOL_BF16 = 2e-2   # BASELINE.json north_star: bf16 GEMM operands, fp32 accumulate
+TOL_FP32 = 1e-4   # BASELINE.json north_star: fp32 path
+
+
+def rel_err(gpu, ref):
+    gpu = np.asarray(gpu, dtype=np.float64)
+    ref = np.asarray(ref, dtype=np.float64)
+    n = np.linalg.norm(ref.ravel())
+    return float(np.linalg.norm((gpu - ref).ravel()) / (n if n > 0 else 1.0))
+
+
+def bf16_round(a):
+    """Round an fp64 array to the nearest bf16 value (exact in fp64) — the bf16 path's operand."""
+    import torch
+    return torch.as_tensor(np.asarray(a, dtype=np.float32)).to(torch.bfloat16).to(torch.float64).numpy()
+
+
+def cell_shapes(cell, I, H, S=None, L=None):
+    from oracle import cells as C
+    if cell == "milstm":
+        return C.milstm_param_shapes(I, H)
+    if cell in ("lstm", "sublstm"):
+        return C.lstm_param_shapes(I, H)
+    if cell == "scrn":
+        return C.scrn_param_shapes(I, H, S or H)
+    if cell == "rhn":
+        return C.rhn_param_shapes(I, H, L)
+    raise ValueError(cell)
+
+
+def make_cell_case(cell, T, B, I, H, seed, bf16=False, ab_range=(0.5, 1.5)):
+    """Seeded parameters and inputs; for the bf16 path weights and inputs are
+    pre-rounded to bf16 so both sides see identical operands."""
+    p = synth.weights(seed, cell_shapes(cell, I, H), H,
+                      {"alpha": ab_range, "beta1": ab_range, "beta2": ab_range})
+    x = synth.uniform(seed, "x", (T, B, I), -1, 1)
+    if bf16:
+        x = bf16_round(x)
+        for k in ("W", "U"):
+            p[k] = bf16_round(p[k])
+    inp = {"x": x, "h0": synth.uniform(seed, "h0", (B, H), -0.5, 0.5),
+           "c0": synth.uniform(seed, "c0", (B, H), -0.5, 0.5)}
+    dY = synth.normal(seed, "dY", (T, B, H))
+    if bf16:
+        dY = bf16_round(dY)
+    dhT = synth.normal(seed, "dhT", (B, H))
+    dcT = synth.normal(seed, "dcT", (B, H))
+    return p, inp, dY, dhT, dcT
+
+
+def run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, variant=None):
+    """Run fwd + bwd through the C ABI; returns (outputs, grads) as numpy fp64 dicts."""
+    import torch
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I = inp["x"].shape
+    H = inp["h0"].shape[1]
+    c = A.Cell(cell, H, I, B, T, dtype=dtype)
+    if variant is not None:
+        c.tune_mode(A.TUNE_FROZEN, variant)
+    c.load(p)
+    dev = c.device
+    tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
+    f32 = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    x = f32(inp["x"]).to(tdt).contiguous()
+    y = torch.empty(T, B, H, dtype=tdt, device=dev)
+    hT = torch.empty(B, H, device=dev)
+    cT = torch.empty(B, H, device=dev)
+    c.forward(x, f32(inp["h0"]), f32(inp["c0"]), y, hT, cT)
+    dx = torch.empty(T, B, I, dtype=tdt, device=dev)
+    dh0 = torch.empty(B, H, device=dev)
+    dc0 = torch.empty(B, H, device=dev)
+    c.backward(f32(dY).to(tdt).contiguous(), f32(dhT), f32(dcT), dx, dh0, dc0)
+    torch.cuda.synchronize()
+    out = {"y": y.float().cpu().numpy(), "hT": hT.cpu().numpy(), "cT": cT.cpu().numpy()}
+    g = {k: c.view(k, c.grads).cpu().numpy().reshape(np.shape(p[k])) for k in p}
+    g.update(dx=dx.float().cpu().numpy(), dh0=dh0.cpu().numpy(), dc0=dc0.cpu().numpy())
+    return out, g, c

@@ -1,0 +1,73 @@
+"""Cell-level parity of the CUDA path (through the C ABI) against the fp64 oracle on identical seeded
+inputs: every output and every gradient, fp32 path ≤ 1e-4 and bf16 path ≤ 2e-2 relative L2
+(BASELINE.json north_star; reading R18), plus bitwise equality across tuner variants."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import cells as C
+
+from helpers import TOL_BF16, TOL_FP32, make_cell_case, rel_err, run_gpu_cell
+
+pytestmark = pytest.mark.gpu
+
+
+def _check(cell, T, B, I, H, dtype, seed, tol, variant=None):
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, seed, bf16=(dtype == "bf16"))
+    out_o, g_o = C.cell_fwd_bwd(cell, p, inp, dY, dhT, dcT)
+    out_g, g_g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, variant)
+    errs = {}
+    for k in out_o:
+        errs[k] = rel_err(out_g[k], out_o[k])
+    for k in g_o:
+        errs["d" + k if not k.startswith("d") else k] = rel_err(g_g[k], g_o[k])
+    bad = {k: v for k, v in errs.items() if not v <= tol}
+    assert not bad, (cell, dtype, (T, B, I, H), bad, errs)
+    return errs
+
+
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+def test_fp32_cfg1(cell):
+    """BASELINE.json configs[0]: MI-LSTM H64 I32 B4 T8 fp32 (≤ 1e-4)."""
+    _check(cell, 8, 4, 32, 64, "fp32", synth.config_seed(1), TOL_FP32)
+
+
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+def test_fp32_ragged(cell):
+    """Hidden/input sizes that are not multiples of the 64-unit gate block; tiny batch."""
+    _check(cell, 5, 3, 20, 70, "fp32", synth.config_seed(1) + 11, TOL_FP32)
+
+
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+def test_bf16_small(cell):
+    _check(cell, 8, 4, 32, 64, "bf16", synth.config_seed(1) + 1, TOL_BF16)
+
+
+@pytest.mark.parametrize("cell", ["milstm", "lstm"])
+def test_bf16_multi_tile_ragged(cell):
+    """Several M/N tiles and ragged tails: B=200 (2 row tiles), H=200 (Hp=256), I=72."""
+    _check(cell, 6, 200, 72, 200, "bf16", synth.config_seed(5) + 2, TOL_BF16)
+
+
+def test_bf16_cfg5_reduced():
+    """cfg5 reduced rung: full H=I=2048 and per-GPU batch 64, T=8."""
+    _check("milstm", 8, 64, 2048, 2048, "bf16", synth.config_seed(5), TOL_BF16)
+
+
+def test_variants_bitwise():
+    """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
+    T, B, I, H = 6, 160, 128, 192
+    p, inp, dY, dhT, dcT = make_cell_case("milstm", T, B, I, H, 77, bf16=True)
+    variants = ["bn_a1=256,bn_rec=256,bn_bptt=128,bn_wg=256,bn_dx=256,wg_side=0",
+                "bn_a1=128,bn_rec=128,bn_bptt=64,bn_wg=128,bn_dx=128,wg_side=1",
+                "bn_a1=64,bn_rec=64,bn_bptt=256,bn_wg=64,bn_dx=64,wg_side=0"]
+    ref = None
+    for v in variants:
+        out, g, _ = run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", v)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)

@@ -1,0 +1,53 @@
+"""K1 (tcgen05/TMA/TMEM GEMM) on B200 against an fp64 product of the same bf16 operands, for every
+operand layout the step uses, ragged tails, and the bitwise tile-shape invariance (R1, R7)."""
+import numpy as np
+import pytest
+import torch
+
+import paper_conf_asplos_sivathanucsz19_b200 as A
+
+pytestmark = pytest.mark.gpu
+
+
+def _operands(M, N, K, a_mn, b_mn, seed=0):
+    g = torch.Generator().manual_seed(seed)
+    a = torch.randn(M, K, generator=g).to(torch.bfloat16)
+    b = torch.randn(K, N, generator=g).to(torch.bfloat16)
+    ref = a.double() @ b.double()
+    A_store = (a.t() if a_mn else a).contiguous().cuda()      # MN-major A is stored [K][M]
+    B_store = (b if b_mn else b.t()).contiguous().cuda()      # K-major B is stored [N][K]
+    return A_store, B_store, ref
+
+
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 0), (1, 1)])
+@pytest.mark.parametrize("M,N,K", [(128, 256, 64), (256, 512, 1024), (300, 200, 136), (64, 64, 32)])
+def test_gemm_layouts(a_mn, b_mn, M, N, K):
+    if (a_mn and M % 8) or (b_mn and N % 8) or (not a_mn and K % 8) or (not b_mn and K % 8):
+        pytest.skip("TMA needs 16-byte row strides")
+    A_s, B_s, ref = _operands(M, N, K, a_mn, b_mn)
+    for bn in (64, 128, 256):
+        out = A.gemm_bf16(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn)
+        torch.cuda.synchronize()
+        err = (out.double().cpu() - ref).abs().max().item()
+        scale = ref.abs().max().item()
+        assert err <= 1e-5 * scale * max(1, K / 64) + 1e-6, (bn, err, scale)
+
+
+def test_tile_shapes_bitwise():
+    """R1/R7: the accumulation order of every output element does not depend on the tile width."""
+    M, N, K = 512, 768, 2048
+    for a_mn, b_mn in [(0, 0), (1, 1), (0, 1)]:
+        A_s, B_s, _ = _operands(M, N, K, a_mn, b_mn, seed=3)
+        outs = [A.gemm_bf16(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn) for bn in (64, 128, 256)]
+        torch.cuda.synchronize()
+        assert torch.equal(outs[0], outs[1]) and torch.equal(outs[1], outs[2])
+
+
+def test_paper_table1_shapes():
+    """The paper's Table 1 GEMMs: 64x1024x4096 (LSTM fwd fused) and 64x4096x1024 (bwd)."""
+    for M, K, N in [(64, 1024, 4096), (64, 4096, 1024)]:
+        A_s, B_s, ref = _operands(M, N, K, 0, 0, seed=5)
+        out = A.gemm_bf16(A_s, B_s, M, N, K)
+        torch.cuda.synchronize()
+        # fp32 accumulation of exact bf16 products: error ~ sqrt(K)·2^-24·|terms|
+        assert (out.double().cpu() - ref).abs().max().item() <= 2e-6 * K ** 0.5 * ref.abs().max().item()

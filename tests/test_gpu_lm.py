@@ -1,0 +1,86 @@
+"""LM training-step parity (embedding → cell → head → mean CE → backward → SGD) against the fp64
+oracle, through the C ABI; tuner exploration is value-preserving (same loss/params tuner on/off)."""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import lm as OLM
+
+from helpers import TOL_BF16, TOL_FP32, bf16_round, cell_shapes, rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+def _lm_case(cell, T, B, I, H, V, seed, bf16, n_symbols=None):
+    shapes = cell_shapes(cell, I, H)
+    shapes.update({"E": (V, I), "W_o": (H, V), "b_o": (V,)})
+    p = synth.weights(seed, shapes, H, {"alpha": (0.5, 1.5), "beta1": (0.5, 1.5), "beta2": (0.5, 1.5)})
+    if bf16:
+        for k in ("W", "U", "E", "W_o"):
+            p[k] = bf16_round(p[k])
+    tok = synth.zipf_tokens(seed, "tok", (T + 1, B), V, n_symbols)
+    h0 = synth.uniform(seed, "h0", (B, H), -0.5, 0.5)
+    c0 = synth.uniform(seed, "c0", (B, H), -0.5, 0.5)
+    return p, tok, h0, c0
+
+
+def _run(cell, T, B, I, H, V, dtype, seed, n_symbols=None, lr=0.0):
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    p, tok, h0, c0 = _lm_case(cell, T, B, I, H, V, seed, dtype == "bf16", n_symbols)
+    c = A.Cell(cell, H, I, B, T, dtype=dtype)
+    m = A.LM(c, V)
+    m.load(p)
+    dev = c.device
+    f32 = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    m.set_state(f32(h0), f32(c0))
+    tokens = torch.as_tensor(tok, dtype=torch.int32, device=dev)
+    loss = m.fwd_bwd(tokens)
+    torch.cuda.synchronize()
+    g = {k: m.view(k, m.grads).cpu().numpy().reshape(np.shape(p[k])) for k in p}
+    return p, tok, h0, c0, float(loss.item()), g, m
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+@pytest.mark.parametrize("cell", ["milstm", "lstm"])
+def test_lm_grads(cell, dtype, tol):
+    T, B, I, H, V = 6, 8, 64, 64, 50
+    p, tok, h0, c0, loss, g, _ = _run(cell, T, B, I, H, V, dtype, synth.config_seed(5) + 3, n_symbols=40)
+    lo, go, _ = OLM.lm_forward_backward(cell, p, tok, h0, c0)
+    assert abs(loss - lo) / abs(lo) <= tol
+    errs = {k: rel_err(g[k], go[k]) for k in go}
+    bad = {k: v for k, v in errs.items() if not v <= tol}
+    assert not bad, (bad, errs)
+
+
+def test_lm_cfg5_shape_reduced_bf16():
+    """cfg5 shapes (H=I=2048, V=256 over 205 Zipf symbols), per-GPU batch 64, T=4."""
+    T, B, I, H, V = 4, 64, 2048, 2048, 256
+    p, tok, h0, c0, loss, g, _ = _run("milstm", T, B, I, H, V, "bf16", synth.config_seed(5), n_symbols=205)
+    lo, go, _ = OLM.lm_forward_backward("milstm", p, tok, h0, c0)
+    assert abs(loss - lo) / abs(lo) <= TOL_BF16
+    errs = {k: rel_err(g[k], go[k]) for k in go}
+    assert all(v <= TOL_BF16 for v in errs.values()), errs
+
+
+def test_lm_sgd_and_tuner_value_preserving():
+    """20 SGD steps with the tuner exploring vs frozen at the default: bitwise-identical params."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 6, 128, 128, 128, 64
+    seed = synth.config_seed(5) + 9
+    results = []
+    for mode in (A.TUNE_OFF, A.TUNE_ON):
+        p, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, seed, True)
+        c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+        m = A.LM(c, V)
+        m.load(p)
+        c.tune_mode(mode)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(20):
+            m.train_step(tokens, 0.1)
+            c.tune_next()
+        torch.cuda.synchronize()
+        results.append((m.params.clone(), float(m.loss.item()), c.tune_report()))
+    assert torch.equal(results[0][0], results[1][0])
+    assert results[0][1] == results[1][1]
+    assert results[1][2]["configs_explored"] >= 2
