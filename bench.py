@@ -138,6 +138,7 @@ def main():
     ap.add_argument("--impl", default="astra", choices=["astra", "reference"])
     ap.add_argument("--no-tune", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile", action="store_true", help="1 warm-up + --steps steps, nothing else (for ncu)")
     ap.add_argument("--batch", type=int, default=None, help="override global batch (debug)")
     ap.add_argument("--seq", type=int, default=None, help="override seq (debug)")
     args = ap.parse_args()
@@ -197,6 +198,16 @@ def main():
             dist.barrier()
             torch.cuda.synchronize()
 
+    if args.profile:
+        if os.environ.get("ASTRA_VARIANT"):
+            cell.tune_mode(A.TUNE_FROZEN, os.environ["ASTRA_VARIANT"])
+        lm.train_step(tokens, lr)
+        torch.cuda.synchronize()
+        for _ in range(args.steps):
+            lm.train_step(tokens, lr)
+        torch.cuda.synchronize()
+        print(json.dumps({"profile_steps": args.steps, "regions_ms": region_times(cell)}))
+        return
     # ---- online exploration (work-conserving: every explored step is a real training step)
     tune_steps, tune_t0 = 0, time.perf_counter()
     tune_info = {"mode": "off"}
