@@ -167,9 +167,11 @@ astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev
  * tcgen05 path.  A (device bf16): a_mn = 0 → stored [M][lda] (K contiguous); a_mn = 1 → stored
  * [K][lda] (M contiguous).  B (device bf16): b_mn = 0 → stored [N][ldb]; b_mn = 1 → stored
  * [K][ldb].  lda/ldb in elements, multiples of 8; pointers 16-byte aligned.  bn ∈ {64, 128,
- * 256} is the CTA tile width (a tuner variable); the result does not depend on it.          */
+ * 256} is the CTA tile width and cm, cn ∈ {1, 2, 4} (cm·cn ≤ 8) the thread-block-cluster shape
+ * for TMA multicast of B (along M) and A (along N) — tuner variables; the result does not
+ * depend on them (bitwise).                                                                 */
 astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long lda, const void* B, int b_mn,
-                             long ldb, float* C, long ldc, int bn, astra_stream stream);
+                             long ldb, float* C, long ldc, int bn, int cm, int cn, astra_stream stream);
 
 /* ---- diagnostics ----------------------------------------------------------------------- */
 const char* astra_status_string(astra_status s);

@@ -68,7 +68,7 @@ _SIGS = {
     "astra_lm_set_state": [_P, _P, _P],
     "astra_lm_train_step": [_P, _P, _F, _P],
     "astra_lm_fwd_bwd": [_P, _P, _P],
-    "astra_gemm_bf16": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _P],
+    "astra_gemm_bf16": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I, _P],
     "astra_status_string": [_I],
     "astra_last_error": [],
     "astra_kernel_launch_count": [],
@@ -115,13 +115,13 @@ def _stream():
     return ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
 
 
-def gemm_bf16(A, B, M, N, K, a_mn=False, b_mn=False, bn=256, out=None):
+def gemm_bf16(A, B, M, N, K, a_mn=False, b_mn=False, bn=256, cm=1, cn=1, out=None):
     """K1 as a library GEMM: out[M, N] fp32 = A·B (see astra_gemm_bf16)."""
     import torch
     if out is None:
         out = torch.empty(M, N, dtype=torch.float32, device=A.device)
     _check(lib().astra_gemm_bf16(M, N, K, _ptr(A), int(a_mn), A.stride(0), _ptr(B), int(b_mn), B.stride(0),
-                                 _ptr(out), out.stride(0), bn, _stream()))
+                                 _ptr(out), out.stride(0), bn, cm, cn, _stream()))
     return out
 
 

@@ -154,30 +154,7 @@ astra_status astra_tune_mode(astra_cell c, int mode, const char* forced) {
       cc.wirer.reset();
       cc.var = Variant();
     } else if (forced) {
-      Variant v;
-      std::string s(forced);
-      size_t p = 0;
-      while (p < s.size()) {
-        size_t q = s.find(',', p);
-        if (q == std::string::npos) q = s.size();
-        std::string kv = s.substr(p, q - p);
-        size_t eq = kv.find('=');
-        ASTRA_CHECK_ARG(eq != std::string::npos, "tune_mode: variant must be k=v,...");
-        std::string k = kv.substr(0, eq);
-        int val = std::stoi(kv.substr(eq + 1));
-        if (k == "bn_a1") v.bn_a1 = val;
-        else if (k == "bn_rec") v.bn_rec = val;
-        else if (k == "bn_bptt") v.bn_bptt = val;
-        else if (k == "bn_wg") v.bn_wg = val;
-        else if (k == "bn_dx") v.bn_dx = val;
-        else if (k == "bn_head") v.bn_head = val;
-        else if (k == "wg_side") v.wg_side = val;
-        else throw Error(ASTRA_E_ARG, "tune_mode: unknown variable " + k);
-        p = q + 1;
-      }
-      for (int bn : {v.bn_a1, v.bn_rec, v.bn_bptt, v.bn_wg, v.bn_dx, v.bn_head})
-        ASTRA_CHECK_ARG(bn == 64 || bn == 128 || bn == 256, "tune_mode: tile widths must be 64/128/256");
-      cc.var = v;
+      cc.var = Variant::parse(forced);
     }
     cc.tune_mode = mode;
   });
@@ -275,7 +252,7 @@ astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev
 }
 
 astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long lda, const void* Bp, int b_mn,
-                             long ldb, float* C, long ldc, int bn, astra_stream stream) {
+                             long ldb, float* C, long ldc, int bn, int cm, int cn, astra_stream stream) {
   return guard([&] {
     NEED(A); NEED(Bp); NEED(C);
     ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "gemm: sizes must be positive");
@@ -287,7 +264,7 @@ astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long 
     if (b_mn) { b.inner = N; b.outer = K; } else { b.inner = K; b.outer = N; }
     ASTRA_CHECK_ARG(lda >= a.inner && ldb >= b.inner, "gemm: leading dimension too small");
     TcGemm g;
-    tc_gemm_prepare(g, a, a_mn != 0, b, b_mn != 0, M, N, K, bn);
+    tc_gemm_prepare(g, a, a_mn != 0, b, b_mn != 0, M, N, K, bn, cm, cn);
     EpiStore e;
     e.C = C; e.ldc = ldc; e.Mv = M; e.Nv = N; e.out_bf16 = 0; e.bias = nullptr; e.perm_u = 0; e.perm_H = 0;
     tc_gemm_launch(g, e, 0, 0, (cudaStream_t)stream);

@@ -69,11 +69,16 @@ static int smem_for(int& stages) {
   return TcSmem<BN>::bytes(stages);
 }
 
-void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN) {
+void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
+                     int cm, int cn) {
+  ASTRA_CHECK_ARG((cm == 1 || cm == 2 || cm == 4) && (cn == 1 || cn == 2 || cn == 4) && cm * cn <= 8,
+                  "tc_gemm: cluster shape must be cm, cn in {1,2,4}, cm*cn <= 8");
   ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256, "tc_gemm: BN must be 64, 128 or 256");
   ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
-  if (a_mn) make_map(&g.mapA, A, 64, 64); else make_map(&g.mapA, A, 64, TC_BM);
-  if (b_mn) make_map(&g.mapB, B, 64, 64); else make_map(&g.mapB, B, 64, BN);
+  if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
+  if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm);
+  g.args.cm = cm;
+  g.args.cn = cn;
   g.BN = BN;
   g.args.M = M; g.args.N = N; g.args.K = K;
   g.args.num_m = cdiv(M, TC_BM);
@@ -102,11 +107,29 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   TcArgs a = g.args;
   a.az = az;
   a.bz = bz;
-  const int tiles = a.num_m * a.num_n;
-  int grid = num_sms();
-  if (max_ctas > 0 && max_ctas < grid) grid = max_ctas;
-  if (tiles < grid) grid = tiles;
-  tc_gemm_kernel<BN, EpiStore><<<grid, TC_THREADS, g.smem, st>>>(g.mapA, g.mapB, a, epi);
+  const int cs = a.cm * a.cn;
+  const int ctiles = cdiv(a.num_m, a.cm) * cdiv(a.num_n, a.cn);   // cluster tiles
+  int clusters = num_sms() / cs;
+  if (max_ctas > 0 && max_ctas / cs < clusters) clusters = max_ctas / cs > 0 ? max_ctas / cs : 1;
+  if (ctiles < clusters) clusters = ctiles;
+  const int grid = clusters * cs;
+  if (cs == 1) {
+    tc_gemm_kernel<BN, EpiStore><<<grid, TC_THREADS, g.smem, st>>>(g.mapA, g.mapB, a, epi);
+  } else {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(TC_THREADS);
+    cfg.dynamicSmemBytes = g.smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = cs;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, tc_gemm_kernel<BN, EpiStore>, g.mapA, g.mapB, a, epi));
+  }
   LAUNCH_CHECK();
 }
 

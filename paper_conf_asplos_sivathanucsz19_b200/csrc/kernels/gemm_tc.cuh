@@ -34,6 +34,7 @@ struct TcArgs {
   int az, bz;       // third tensor-map coordinate (time slice) of A and B
   int a_mn, b_mn;   // 1 = MN-major operand
   int stages;
+  int cm, cn;       // cluster shape (CTAs sharing B along M, sharing A along N)
   uint32_t idesc;
 };
 
@@ -144,6 +145,12 @@ struct EpiStore {
   }
 };
 
+// Cluster multicast (cm x cn CTAs per cluster, cluster rank r: rm = r % cm, rn = r / cm): the cn
+// CTAs that share an A tile (same rm) each load 1/cn of it and multicast it to the others; the cm
+// CTAs that share a B tile (same rn) do the same for B.  Every CTA's stage is therefore written by
+// cm + cn − 1 CTAs, so its `empty` barrier expects that many MMA-commit arrivals (each MMA issuer
+// commits to the `empty` barriers of all its neighbours).  Cuts L2→SMEM operand traffic by
+// cm (B) and cn (A) without changing any accumulation order.
 template <int BN, class Epi>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
@@ -160,13 +167,22 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
   const int warp = threadIdx.x / 32;
   const int lane = threadIdx.x % 32;
-  const int num_tiles = args.num_m * args.num_n;
+  const int cm = args.cm, cn = args.cn, cs = cm * cn;
+  const int crank = cs > 1 ? (int)sm100::cluster_ctarank() : 0;
+  const int rm = crank % cm, rn = crank / cm;
+  const int ncm = (args.num_m + cm - 1) / cm, ncn = (args.num_n + cn - 1) / cn;
+  const int num_ct = ncm * ncn;                  // cluster tiles
+  const int cluster_id = blockIdx.x / cs, num_clusters = gridDim.x / cs;
   const int nk = (args.K + TC_BK - 1) / TC_BK;
+  uint16_t mask_a = 0, mask_b = 0;
+  for (int j = 0; j < cn; ++j) mask_a |= (uint16_t)(1u << (rm + cm * j));
+  for (int i = 0; i < cm; ++i) mask_b |= (uint16_t)(1u << (i + cm * rn));
+  const uint16_t mask_nb = mask_a | mask_b;
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < stages; ++s) {
       sm100::mbar_init(&full[s], 1);
-      sm100::mbar_init(&empty[s], 1);
+      sm100::mbar_init(&empty[s], cm + cn - 1);
     }
     for (int a = 0; a < 2; ++a) {
       sm100::mbar_init(&tfull[a], 1);
@@ -181,6 +197,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (warp == 1) sm100::tmem_alloc(tmem_slot, S::TMEM_COLS);
   sm100::tc_fence_before();
   __syncthreads();
+  if (cs > 1) sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
@@ -189,26 +206,47 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0;
-      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        const int m0 = (tile % args.num_m) * TC_BM;
-        const int n0 = (tile / args.num_m) * BN;
+      // slices this CTA loads (and multicasts) of the shared A / B tiles
+      const int a_rows = TC_BM / cn, b_rows = BN / cm;       // K-major: rows of the box
+      const int a_krows = TC_BK / cn, b_krows = TC_BK / cm;  // MN-major: K rows of each 64-wide box
+      for (int ct = cluster_id; ct < num_ct; ct += num_clusters) {
+        const int m0 = ((ct % ncm) * cm + rm) * TC_BM;
+        const int n0 = ((ct / ncm) * cn + rn) * BN;
         for (int kb = 0; kb < nk; ++kb) {
           sm100::mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * S::STAGE_BYTES;
           uint8_t* sb = sa + S::A_BYTES;
           sm100::mbar_arrive_expect_tx(&full[s], S::STAGE_BYTES);
           const int k0 = kb * TC_BK;
-          if (args.a_mn) {
-            sm100::tma_load_3d(sa, &mapA, &full[s], m0, k0, args.az);
-            sm100::tma_load_3d(sa + 8192, &mapA, &full[s], m0 + 64, k0, args.az);
-          } else {
-            sm100::tma_load_3d(sa, &mapA, &full[s], k0, m0, args.az);
-          }
-          if (args.b_mn) {
+          if (cs == 1) {
+            if (args.a_mn) {
+              sm100::tma_load_3d(sa, &mapA, &full[s], m0, k0, args.az);
+              sm100::tma_load_3d(sa + 8192, &mapA, &full[s], m0 + 64, k0, args.az);
+            } else {
+              sm100::tma_load_3d(sa, &mapA, &full[s], k0, m0, args.az);
+            }
+            if (args.b_mn) {
 #pragma unroll
-            for (int j = 0; j < BN / 64; ++j) sm100::tma_load_3d(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+              for (int j = 0; j < BN / 64; ++j)
+                sm100::tma_load_3d(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+            } else {
+              sm100::tma_load_3d(sb, &mapB, &full[s], k0, n0, args.bz);
+            }
           } else {
-            sm100::tma_load_3d(sb, &mapB, &full[s], k0, n0, args.bz);
+            if (args.a_mn) {
+              for (int j = 0; j < 2; ++j)
+                sm100::tma_load_3d_mc(sa + j * 8192 + rn * a_krows * 128, &mapA, &full[s], m0 + 64 * j,
+                                      k0 + rn * a_krows, args.az, mask_a);
+            } else {
+              sm100::tma_load_3d_mc(sa + rn * a_rows * 128, &mapA, &full[s], k0, m0 + rn * a_rows, args.az, mask_a);
+            }
+            if (args.b_mn) {
+              for (int j = 0; j < BN / 64; ++j)
+                sm100::tma_load_3d_mc(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
+                                      k0 + rm * b_krows, args.bz, mask_b);
+            } else {
+              sm100::tma_load_3d_mc(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz, mask_b);
+            }
           }
           if (++s == stages) { s = 0; ph ^= 1; }
         }
@@ -220,7 +258,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       int s = 0;
       uint32_t ph = 0;
       int local = 0;
-      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++local) {
+      for (int ct = cluster_id; ct < num_ct; ct += num_clusters, ++local) {
         const int acc = local & 1;
         const uint32_t use = (uint32_t)(local >> 1);
         sm100::mbar_wait(&tempty[acc], (use & 1) ^ 1);
@@ -239,7 +277,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                                           : sm100::smem_desc_sw128(sb + kk * 32, 16, 1024);
             sm100::umma_bf16(d_tmem, ad, bd, args.idesc, (kb | kk) != 0);
           }
-          sm100::umma_commit(&empty[s]);
+          if (cs == 1) sm100::umma_commit(&empty[s]);
+          else sm100::umma_commit_mc(&empty[s], mask_nb);
           if (++s == stages) { s = 0; ph ^= 1; }
         }
         sm100::umma_commit(&tfull[acc]);
@@ -250,20 +289,21 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     const int quarter = warp & 3;           // TMEM lane quarter this warp may access
     const int row = quarter * 32 + lane;    // tile row (= TMEM lane)
     int local = 0;
-    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++local) {
+    for (int ct = cluster_id; ct < num_ct; ct += num_clusters, ++local) {
       const int acc = local & 1;
       const uint32_t use = (uint32_t)(local >> 1);
-      const int m0 = (tile % args.num_m) * TC_BM;
-      const int n0 = (tile / args.num_m) * BN;
+      const int m0 = ((ct % ncm) * cm + rm) * TC_BM;
+      const int n0 = ((ct / ncm) * cn + rn) * BN;
       sm100::mbar_wait(&tfull[acc], use & 1);
       sm100::tc_fence_after();
       const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * BN;
-      epi.template run<BN>(taddr, m0, n0, row);
+      if (m0 < args.M && n0 < args.N) epi.template run<BN>(taddr, m0, n0, row);
       sm100::tc_fence_before();
       sm100::mbar_arrive(&tempty[acc]);
     }
   }
   __syncthreads();
+  if (cs > 1) sm100::cluster_sync();
   if (warp == 1) {
     sm100::tc_fence_after();
     sm100::tmem_dealloc(tmem_base, S::TMEM_COLS);

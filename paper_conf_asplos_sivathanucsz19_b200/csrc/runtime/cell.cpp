@@ -18,11 +18,47 @@
 
 namespace astra {
 
+const char* const ROLE_NAMES[G_ROLES] = {"a1", "rec", "bptt", "du", "dw", "dx", "head"};
+
 std::string Variant::str() const {
   std::ostringstream o;
-  o << "bn_a1=" << bn_a1 << ",bn_rec=" << bn_rec << ",bn_bptt=" << bn_bptt << ",bn_wg=" << bn_wg
-    << ",bn_dx=" << bn_dx << ",bn_head=" << bn_head << ",wg_side=" << wg_side;
+  for (int r = 0; r < G_ROLES; ++r) o << ROLE_NAMES[r] << "=" << g[r].bn << "." << g[r].cm << "." << g[r].cn << ",";
+  o << "wg_side=" << wg_side;
   return o.str();
+}
+
+Variant Variant::parse(const std::string& s) {
+  Variant v;
+  size_t p = 0;
+  while (p < s.size()) {
+    size_t q = s.find(',', p);
+    if (q == std::string::npos) q = s.size();
+    const std::string kv = s.substr(p, q - p);
+    p = q + 1;
+    if (kv.empty()) continue;
+    const size_t eq = kv.find('=');
+    ASTRA_CHECK_ARG(eq != std::string::npos, "variant: expected key=value, got '" + kv + "'");
+    const std::string k = kv.substr(0, eq), val = kv.substr(eq + 1);
+    if (k == "wg_side") {
+      v.wg_side = std::stoi(val);
+      ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    int r = -1;
+    for (int i = 0; i < G_ROLES; ++i)
+      if (k == ROLE_NAMES[i]) r = i;
+    ASTRA_CHECK_ARG(r >= 0, "variant: unknown variable '" + k + "'");
+    KCfg c;
+    int n = std::sscanf(val.c_str(), "%d.%d.%d", &c.bn, &c.cm, &c.cn);
+    ASTRA_CHECK_ARG(n >= 1, "variant: bad kernel choice '" + val + "'");
+    if (n < 3) c.cn = 1;
+    if (n < 2) c.cm = 1;
+    ASTRA_CHECK_ARG((c.bn == 64 || c.bn == 128 || c.bn == 256) && (c.cm == 1 || c.cm == 2 || c.cm == 4) &&
+                        (c.cn == 1 || c.cn == 2 || c.cn == 4) && c.cm * c.cn <= 8,
+                    "variant: tile width must be 64/128/256 and cluster cm, cn in {1,2,4} with cm*cn <= 8");
+    v.g[r] = c;
+  }
+  return v;
 }
 
 static size_t align_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
@@ -123,13 +159,13 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
   if (which) region_used[r] = true;
 }
 
-void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, int BN, cudaStream_t st) {
+void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st) {
   if (ot == OT::BF16) {
-    auto key = std::make_pair(id, BN);
+    auto key = std::make_tuple(id, k.bn, k.cm, k.cn);
     auto it = tc_cache.find(key);
     if (it == tc_cache.end()) {
       TcGemm g;
-      tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, BN);
+      tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, k.cm, k.cn);
       it = tc_cache.emplace(key, g).first;
     }
     tc_gemm_launch(it->second, e, az, bz, st);
@@ -187,7 +223,7 @@ void Cell::forward(const void* x, const float* h0, const float* c0, void* y, flo
   a1.A = mat(X, I, TB, Ip);
   a1.B = mat(Wm, I, NG, Ip);
   a1.M = (int)TB; a1.N = NG; a1.K = I;
-  run_gemm(0, a1, epi(WX, NG, (int)TB, NG), 0, 0, var.bn_a1, st);
+  run_gemm(0, a1, epi(WX, NG, (int)TB, NG), 0, 0, var.g[G_A1], st);
   mark(R_A1, 1, st);
 
   // a3: recurrent chain
@@ -198,7 +234,7 @@ void Cell::forward(const void* x, const float* h0, const float* c0, void* y, flo
   rec.M = B; rec.N = NG; rec.K = Hp;
   for (int t = 0; t < T; ++t) {
     float* UHt = UH + (long)t * B * NG;
-    run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.bn_rec, st);
+    run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st);
     const bool last = t == T - 1;
     void* yt = y ? (char*)y + (size_t)t * B * H * e : nullptr;
     lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
@@ -248,7 +284,7 @@ void Cell::backward(const void* dy, const float* dhT, const float* dcT, void* dx
       dh_rec = dhT;
       ld_dh = H;
     } else {
-      run_gemm(2, bp, epi(dH, Hp, B, Hp), t + 1, 0, var.bn_bptt, st);
+      run_gemm(2, bp, epi(dH, Hp, B, Hp), t + 1, 0, var.g[G_BPTT], st);
       dh_rec = dH;
       ld_dh = Hp;
     }
@@ -261,7 +297,7 @@ void Cell::backward(const void* dy, const float* dhT, const float* dcT, void* dx
                        UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
                        Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
   }
-  if (dh0) run_gemm(2, bp, epi(dh0, H, B, H), 0, 0, var.bn_bptt, st);
+  if (dh0) run_gemm(2, bp, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
   if (dc0) copy_pad(OT::F32, dC, OT::F32, B, H, Hp, dc0, H, st);
   mark(R_BPTT, 1, st);
 
@@ -280,7 +316,7 @@ void Cell::backward(const void* dy, const float* dhT, const float* dcT, void* dx
   gu.b_mn = true;
   gu.M = Hp; gu.N = NG; gu.K = (int)TB;
   if (st_u == st) mark(R_DU, 0, st);
-  run_gemm(4, gu, epi(g("U"), 4L * H, H, NG, 0, nullptr, GATE_U, H), 0, 0, var.bn_wg, st_u);
+  run_gemm(4, gu, epi(g("U"), 4L * H, H, NG, 0, nullptr, GATE_U, H), 0, 0, var.g[G_DU], st_u);
   if (st_u == st) mark(R_DU, 1, st);
 
   GemmSpec gw;
@@ -290,7 +326,7 @@ void Cell::backward(const void* dy, const float* dhT, const float* dcT, void* dx
   gw.b_mn = true;
   gw.M = I; gw.N = NG; gw.K = (int)TB;
   mark(R_DW, 0, st);
-  run_gemm(5, gw, epi(g("W"), 4L * H, I, NG, 0, nullptr, GATE_U, H), 0, 0, var.bn_wg, st);
+  run_gemm(5, gw, epi(g("W"), 4L * H, I, NG, 0, nullptr, GATE_U, H), 0, 0, var.g[G_DW], st);
   mark(R_DW, 1, st);
 
   if (dx) {
@@ -301,9 +337,9 @@ void Cell::backward(const void* dy, const float* dhT, const float* dcT, void* dx
     gx.M = (int)TB; gx.N = I; gx.K = NG;
     mark(R_DX, 0, st);
     if (lm_mode)
-      run_gemm(6, gx, epi(dx, Ip, (int)TB, I), 0, 0, var.bn_dx, st);
+      run_gemm(6, gx, epi(dx, Ip, (int)TB, I), 0, 0, var.g[G_DX], st);
     else
-      run_gemm(6, gx, epi(dx, I, (int)TB, I, ot == OT::BF16), 0, 0, var.bn_dx, st);
+      run_gemm(6, gx, epi(dx, I, (int)TB, I, ot == OT::BF16), 0, 0, var.g[G_DX], st);
     mark(R_DX, 1, st);
   }
   float* gq[4] = {g("b"), nullptr, nullptr, nullptr};
@@ -341,17 +377,47 @@ void Cell::sgd_step(float lr) {
 }
 
 // ------------------------------------------------------------------------ tuner glue
-static const int BN2[2] = {256, 128};
-static const int BN3[3] = {128, 64, 256};
+// The enumerator's static pruning (A19): per GEMM role, the kernel choices whose tile
+// and cluster shape fit the problem; the default (Variant()) first.
+void Cell::role_shape(int role, int& M, int& N) const {
+  const int TB = T * B;
+  switch (role) {
+    case G_A1: M = TB; N = NG; break;
+    case G_REC: M = B; N = NG; break;
+    case G_BPTT: M = B; N = Hp; break;
+    case G_DU: M = Hp; N = NG; break;
+    case G_DW: M = I; N = NG; break;
+    case G_DX: M = TB; N = I; break;
+    default: M = TB; N = lm_V > 0 ? lm_V : Hp; break;
+  }
+}
+
+static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 2, 1}, {256, 4, 1}, {256, 2, 2},
+                                  {256, 1, 2}, {128, 2, 1}, {128, 4, 1}, {128, 2, 2}, {128, 1, 2}, {64, 2, 1},
+                                  {64, 4, 1}, {64, 2, 2}};
 
 void Cell::tuner_setup() {
-  std::string t;
+  const Variant def;
+  std::string par;
+  const char* metric[G_ROLES] = {"t_a1", "t_fwd", "t_bptt", "t_du", "t_dw", "t_dx", "t_head"};
   if (ot == OT::BF16) {
-    t = "(par (leaf bn_a1 2 t_a1) (leaf bn_rec 2 t_fwd) (leaf bn_bptt 3 t_bptt) (leaf bn_wgu 2 t_du)"
-        " (leaf bn_dx 2 t_dx)";
-    if (lm_mode) t += " (leaf bn_head 2 t_head)";
-    t += ")";
+    for (int r = 0; r < G_ROLES; ++r) {
+      if (r == G_HEAD && !lm_mode) continue;
+      int M, N;
+      role_shape(r, M, N);
+      allowed[r].clear();
+      allowed[r].push_back(def.g[r]);
+      for (const KCfg& k : CANDIDATES) {
+        if (k == def.g[r]) continue;
+        const int num_m = cdiv(M, TC_BM), num_n = cdiv(N, k.bn);
+        if (k.bn > 64 && N <= k.bn / 2) continue;                                     // tile wider than N
+        if (k.cm > num_m || k.cn > num_n) continue;                                    // idle cluster ranks
+        allowed[r].push_back(k);
+      }
+      par += std::string(" (leaf g_") + ROLE_NAMES[r] + " " + std::to_string(allowed[r].size()) + " " + metric[r] + ")";
+    }
   }
+  std::string t = par.empty() ? "" : "(par" + par + ")";
   if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
   if (t.empty()) t = "(leaf none 1 t_step)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
@@ -368,13 +434,9 @@ void Cell::apply_config(const tuner::Config& c) {
   for (size_t i = 0; i < tree->avs.size(); ++i) {
     const std::string& n = tree->avs[i];
     const int o = c[i];
-    if (n == "bn_a1") v.bn_a1 = BN2[o];
-    else if (n == "bn_rec") v.bn_rec = BN2[o];
-    else if (n == "bn_bptt") v.bn_bptt = BN3[o];
-    else if (n == "bn_wgu") v.bn_wg = BN2[o];
-    else if (n == "bn_dx") v.bn_dx = BN2[o];
-    else if (n == "bn_head") v.bn_head = BN2[o];
-    else if (n == "wg_side") v.wg_side = o;
+    if (n == "wg_side") { v.wg_side = o; continue; }
+    for (int r = 0; r < G_ROLES; ++r)
+      if (n == std::string("g_") + ROLE_NAMES[r]) v.g[r] = allowed[r].at(o);
   }
   var = v;
   configs_seen.push_back(v);
@@ -409,7 +471,8 @@ int Cell::tune_next() {
     if (n == "t_a1") v = elapsed(ev[R_A1][0], ev[R_A1][1]);
     else if (n == "t_fwd") v = elapsed(ev[R_FWD][0], ev[R_FWD][1]);
     else if (n == "t_bptt") v = elapsed(ev[R_BPTT][0], ev[R_BPTT][1]);
-    else if (n == "t_du") v = region_used[R_DU] ? elapsed(ev[R_DU][0], ev[R_DU][1]) + elapsed(ev[R_DW][0], ev[R_DW][1]) : 0;
+    else if (n == "t_du") v = region_used[R_DU] ? elapsed(ev[R_DU][0], ev[R_DU][1]) : 0;
+    else if (n == "t_dw") v = region_used[R_DW] ? elapsed(ev[R_DW][0], ev[R_DW][1]) : 0;
     else if (n == "t_dx") v = region_used[R_DX] ? elapsed(ev[R_DX][0], ev[R_DX][1]) : 0;
     else if (n == "t_head") v = region_used[R_HEAD] ? elapsed(ev[R_HEAD][0], ev[R_HEAD][1]) : 0;
     else if (n == "t_se4") v = elapsed(ev[R_SE4][0], ev[R_SE4][1]);
@@ -456,6 +519,7 @@ std::string Cell::report() {
 LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
   ASTRA_CHECK_ARG(vocab > 1, "lm: vocab must be > 1");
   Vp = (int)round_up(V, 8);
+  c->lm_V = V;
   params = c->params;
   n_cell = c->n_params;
   n_params = n_cell;
@@ -546,7 +610,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   hd.A = mat(c.Hrow(1), Hp, TB, Hp);
   hd.B = mat(Wom, Hp, V, Hp);
   hd.M = (int)TB; hd.N = V; hd.K = Hp;
-  c.run_gemm(7, hd, epi(logits, V, (int)TB, V, 0, P + find("b_o")), 0, 0, c.var.bn_head, st);
+  c.run_gemm(7, hd, epi(logits, V, (int)TB, V, 0, P + find("b_o")), 0, 0, c.var.g[G_HEAD], st);
   ce_fwd_bwd(c.ot, logits, V, V, tokens + c.B, TB, 1.0f / (float)TB, rowloss, dlog, Vp, dlog32, st);
   sum_rows_to_scalar(rowloss, TB, 1.0f / (float)TB, lossp, st);
   GemmSpec dy;
@@ -554,14 +618,14 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   dy.B = mat(Wom, Hp, V, Hp);
   dy.b_mn = true;
   dy.M = (int)TB; dy.N = Hp; dy.K = V;
-  c.run_gemm(8, dy, epi(dY, Hp, (int)TB, Hp), 0, 0, c.var.bn_head, st);
+  c.run_gemm(8, dy, epi(dY, Hp, (int)TB, Hp), 0, 0, c.var.g[G_HEAD], st);
   GemmSpec dwo;
   dwo.A = mat(c.Hrow(1), Hp, TB, Hp);
   dwo.a_mn = true;
   dwo.B = mat(dlog, V, TB, Vp);
   dwo.b_mn = true;
   dwo.M = Hp; dwo.N = V; dwo.K = (int)TB;
-  c.run_gemm(9, dwo, epi(G + find("W_o"), V, c.H, V), 0, 0, c.var.bn_head, st);
+  c.run_gemm(9, dwo, epi(G + find("W_o"), V, c.H, V), 0, 0, c.var.g[G_HEAD], st);
   colsum(dlog32, TB, V, V, (float*)(ws + off_colsum), G + find("b_o"), st);
   c.mark(R_HEAD, 1, st);
 

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <map>
+#include <tuple>
 #include <memory>
 #include <string>
 #include <vector>
@@ -23,15 +24,21 @@ struct ParamInfo {
 };
 
 // One binding of every adaptive variable (the enumerator's output for this cell, §8(a.9)).
+// K1 kernel choice for one GEMM role (B1, "GEMM kernel selection", as a choice among our
+// own sm_100a kernels): CTA tile width and cluster multicast shape.
+struct KCfg {
+  int bn = 256, cm = 1, cn = 1;
+  bool operator==(const KCfg& o) const { return bn == o.bn && cm == o.cm && cn == o.cn; }
+};
+enum GemmRole { G_A1 = 0, G_REC, G_BPTT, G_DU, G_DW, G_DX, G_HEAD, G_ROLES };
+extern const char* const ROLE_NAMES[G_ROLES];
+
 struct Variant {
-  int bn_a1 = 256;      // hoisted input projection tile width (K1)
-  int bn_rec = 256;     // per-step recurrent GEMM tile width (K2)
-  int bn_bptt = 128;    // per-step BPTT dgrad GEMM tile width (K4)
-  int bn_wg = 256;      // weight-gradient GEMMs (a6)
-  int bn_dx = 256;      // input dgrad GEMM (a6)
-  int bn_head = 256;    // LM head GEMMs (a4)
+  KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
-  std::string str() const;
+  Variant() { g[G_BPTT].bn = 128; }
+  std::string str() const;                    // "a1=256.1.1,rec=...,wg_side=0"
+  static Variant parse(const std::string& s); // inverse of str(); throws ASTRA_E_ARG
 };
 
 // GEMM problem in storage terms; drives both engines (tcgen05 for bf16, SIMT for fp32).
@@ -93,6 +100,7 @@ class Cell {
   // LM mode hooks (set by LM)
   bool lm_mode = false;
   const float* lm_dy = nullptr;  // fp32 [T*B][Hp] internal dY for backward
+  int lm_V = 0;                  // vocabulary of the owning LM (head GEMM shapes)
 
   size_t find_param(const std::string& n) const;
   float* p(const std::string& n) { return P + find_param(n); }
@@ -111,8 +119,10 @@ class Cell {
   void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
 
   // GEMM execution
-  void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, int BN, cudaStream_t st);
-  std::map<std::pair<int, int>, TcGemm> tc_cache;
+  void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st);
+  std::map<std::tuple<int, int, int, int>, TcGemm> tc_cache;
+  std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
+  void role_shape(int role, int& M, int& N) const;
 
   // profiling regions (cudaEvent pairs)
   void mark(Region r, int which, cudaStream_t st);

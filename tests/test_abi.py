@@ -76,12 +76,14 @@ def test_bad_arguments_are_rejected():
         A.Cell("milstm", 64, 32, 4, 8, dtype="fp32", allocate=False).forward(None)   # E_STATE: not bound
     c = A.Cell("milstm", 64, 32, 4, 8, dtype="fp32", allocate=False)
     assert L.astra_tune_mode(c.h, 7, None) == 1
-    assert L.astra_tune_mode(c.h, 2, b"bn_a1=100") == 1
+    assert L.astra_tune_mode(c.h, 2, b"a1=100") == 1
+    assert L.astra_tune_mode(c.h, 2, b"a1=256.8.2") == 1
+    assert L.astra_tune_mode(c.h, 2, b"nonsense=1") == 1
     assert L.astra_status_string(4) == b"ASTRA_E_CUDA"
 
 
 def test_tune_report_is_json():
     c = A.Cell("milstm", 64, 32, 4, 8, dtype="bf16", allocate=False)
-    c.tune_mode(A.TUNE_FROZEN, "bn_a1=128,bn_rec=128,wg_side=1")
+    c.tune_mode(A.TUNE_FROZEN, "a1=128.2.2,rec=256.4.1,wg_side=1")
     r = c.tune_report()
-    assert "bn_a1=128" in r["variant"] and "wg_side=1" in r["variant"]
+    assert "a1=128.2.2" in r["variant"] and "rec=256.4.1" in r["variant"] and "wg_side=1" in r["variant"]

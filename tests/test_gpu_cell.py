@@ -59,9 +59,10 @@ def test_variants_bitwise():
     """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
     T, B, I, H = 6, 160, 128, 192
     p, inp, dY, dhT, dcT = make_cell_case("milstm", T, B, I, H, 77, bf16=True)
-    variants = ["bn_a1=256,bn_rec=256,bn_bptt=128,bn_wg=256,bn_dx=256,wg_side=0",
-                "bn_a1=128,bn_rec=128,bn_bptt=64,bn_wg=128,bn_dx=128,wg_side=1",
-                "bn_a1=64,bn_rec=64,bn_bptt=256,bn_wg=64,bn_dx=64,wg_side=0"]
+    variants = ["a1=256,rec=256,bptt=128,du=256,dw=256,dx=256,wg_side=0",
+                "a1=128.2.2,rec=128.2.1,bptt=64.2.1,du=128.1.2,dw=128,dx=128.4.1,wg_side=1",
+                "a1=64.4.1,rec=64,bptt=256.1.1,du=64.2.2,dw=64.2.1,dx=64.2.2,wg_side=0",
+                "a1=256.2.2,rec=256.2.1,bptt=128.2.1,du=256.2.2,dw=256.1.2,dx=256.4.1,wg_side=1"]
     ref = None
     for v in variants:
         out, g, _ = run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", v)

@@ -33,14 +33,35 @@ def test_gemm_layouts(a_mn, b_mn, M, N, K):
         assert err <= 1e-5 * scale * max(1, K / 64) + 1e-6, (bn, err, scale)
 
 
+CLUSTERS = [(1, 1), (2, 1), (4, 1), (1, 2), (2, 2), (1, 4), (4, 2), (2, 4)]
+
+
 def test_tile_shapes_bitwise():
-    """R1/R7: the accumulation order of every output element does not depend on the tile width."""
+    """R1/R7: the accumulation order of every output element depends on neither the tile width nor
+    the cluster/multicast shape."""
     M, N, K = 512, 768, 2048
-    for a_mn, b_mn in [(0, 0), (1, 1), (0, 1)]:
+    for a_mn, b_mn in [(0, 0), (1, 1), (0, 1), (1, 0)]:
         A_s, B_s, _ = _operands(M, N, K, a_mn, b_mn, seed=3)
-        outs = [A.gemm_bf16(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn) for bn in (64, 128, 256)]
+        outs = [A.gemm_bf16(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn, cm=cm, cn=cn)
+                for bn in (64, 128, 256) for cm, cn in CLUSTERS]
         torch.cuda.synchronize()
-        assert torch.equal(outs[0], outs[1]) and torch.equal(outs[1], outs[2])
+        for o in outs[1:]:
+            assert torch.equal(outs[0], o)
+
+
+@pytest.mark.parametrize("cm,cn", CLUSTERS)
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (1, 1), (0, 1), (1, 0)])
+def test_cluster_multicast_ragged(cm, cn, a_mn, b_mn):
+    """Cluster multicast with tile counts that are not multiples of the cluster shape."""
+    M, N, K = 392, 200, 264
+    if a_mn and M % 8:
+        pytest.skip()
+    A_s, B_s, ref = _operands(M, N, K, a_mn, b_mn, seed=11)
+    for bn in (64, 128, 256):
+        out = A.gemm_bf16(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn, cm=cm, cn=cn)
+        torch.cuda.synchronize()
+        err = (out.double().cpu() - ref).abs().max().item()
+        assert err <= 2e-6 * K ** 0.5 * ref.abs().max().item(), (bn, cm, cn, err)
 
 
 def test_paper_table1_shapes():
