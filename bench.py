@@ -58,7 +58,7 @@ class Clocks:
                 ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
                  "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
                  "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
-                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+                 "--format=csv,noheader,nounits", "-lms", "50"], stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
         return self
@@ -224,16 +224,14 @@ def main():
         cell.tune_mode(A.TUNE_FROZEN, rep["variant"])
         tune_info = {"mode": "explored then frozen", "steps": tune_steps, "configs_explored": rep.get("configs_explored"),
                      "wall_s": round(time.perf_counter() - tune_t0, 3), "variant": rep["variant"]}
-    # ---- warm-up
-    for _ in range(max(3, args.warmup)):
-        lm.train_step(tokens, lr)
-    barrier()
-
-    # ---- timed region (device time, CUDA events on the launching stream; max over ranks)
+    # ---- warm-up, then the timed region (device time, CUDA events on the launching stream; max
+    # over ranks).  nvidia-smi samples clocks from the last warm-up steps through the timed region.
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    a1_ms = []
-    l0 = A.launch_count()
     with Clocks(local) as clk:
+        for _ in range(max(3, args.warmup)):
+            lm.train_step(tokens, lr)
+        barrier()
+        l0 = A.launch_count()
         barrier()
         e0.record(st)
         for _ in range(args.steps):

@@ -56,7 +56,7 @@ astra_status astra_cell_create_ex(astra_cell* out, const astra_cell_desc* d) {
     if (dd.src_seq <= 0) dd.src_seq = dd.seq;
     if (dd.attn_dim <= 0) dd.attn_dim = dd.hidden;
     auto h = std::make_unique<astra_cell_s>();
-    h->c.reset(new Cell(dd));
+    h->c = make_cell(dd);
     *out = h.release();
   });
 }
@@ -265,8 +265,7 @@ astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long 
     ASTRA_CHECK_ARG(lda >= a.inner && ldb >= b.inner, "gemm: leading dimension too small");
     TcGemm g;
     tc_gemm_prepare(g, a, a_mn != 0, b, b_mn != 0, M, N, K, bn, cm, cn);
-    EpiStore e;
-    e.C = C; e.ldc = ldc; e.Mv = M; e.Nv = N; e.out_bf16 = 0; e.bias = nullptr; e.perm_u = 0; e.perm_H = 0;
+    EpiStore e = epi(C, ldc, M, N);
     tc_gemm_launch(g, e, 0, 0, (cudaStream_t)stream);
   });
 }

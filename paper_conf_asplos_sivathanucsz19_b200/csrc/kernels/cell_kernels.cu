@@ -1,6 +1,7 @@
 // Pointwise cell kernels (unfused halves of K2/K4), K5 fixed-order reductions, K6 embedding,
 // K7 cross-entropy, K9 SGD and operand mirrors.
 #include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_scan.cuh>
 
 #include "cell_math.cuh"
 #include "kernels.h"
@@ -66,33 +67,35 @@ void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, 
 
 template <typename TD, typename TS>
 __global__ void copy_pad_kernel(const TS* __restrict__ src, long rows, int cols, long lds, TD* __restrict__ dst,
-                                long ldd) {
+                                long ldd, long dcols) {
   const long r = blockIdx.y;
-  for (long c = blockIdx.x * blockDim.x + threadIdx.x; c < ldd; c += (long)gridDim.x * blockDim.x) {
+  for (long c = blockIdx.x * blockDim.x + threadIdx.x; c < dcols; c += (long)gridDim.x * blockDim.x) {
     float v = (c < cols && src) ? to_f<TS>(src[r * lds + c]) : 0.f;
     dst[r * ldd + c] = from_f<TD>(v);
   }
 }
 
-void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, void* dst, long ldd, cudaStream_t st) {
+void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, void* dst, long ldd, cudaStream_t st,
+              long dcols) {
   if (rows == 0) return;
+  if (dcols < 0) dcols = ldd;
   ASTRA_CHECK_ARG(rows < 65536L * 32768L, "copy_pad: too many rows");
   // grid.y is limited to 65535: fold rows into chunks
   const long ychunk = 65535;
   for (long r0 = 0; r0 < rows; r0 += ychunk) {
     const long nr = rows - r0 < ychunk ? rows - r0 : ychunk;
-    dim3 grid(cdiv(ldd, 256) < 8 ? cdiv(ldd, 256) : 8, (unsigned)nr);
+    dim3 grid(cdiv(dcols, 256) < 8 ? cdiv(dcols, 256) : 8, (unsigned)nr);
     const size_t es = ot_size(src_ot), ed = ot_size(ot);
     const char* s = (const char*)src + (src ? r0 * lds * es : 0);
     char* d = (char*)dst + r0 * ldd * ed;
     if (ot == OT::BF16 && src_ot == OT::BF16)
-      copy_pad_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)(src ? s : nullptr), nr, cols, lds, (__nv_bfloat16*)d, ldd);
+      copy_pad_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)(src ? s : nullptr), nr, cols, lds, (__nv_bfloat16*)d, ldd, dcols);
     else if (ot == OT::BF16)
-      copy_pad_kernel<__nv_bfloat16, float><<<grid, 256, 0, st>>>((const float*)(src ? s : nullptr), nr, cols, lds, (__nv_bfloat16*)d, ldd);
+      copy_pad_kernel<__nv_bfloat16, float><<<grid, 256, 0, st>>>((const float*)(src ? s : nullptr), nr, cols, lds, (__nv_bfloat16*)d, ldd, dcols);
     else if (src_ot == OT::BF16)
-      copy_pad_kernel<float, __nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)(src ? s : nullptr), nr, cols, lds, (float*)d, ldd);
+      copy_pad_kernel<float, __nv_bfloat16><<<grid, 256, 0, st>>>((const __nv_bfloat16*)(src ? s : nullptr), nr, cols, lds, (float*)d, ldd, dcols);
     else
-      copy_pad_kernel<float, float><<<grid, 256, 0, st>>>((const float*)(src ? s : nullptr), nr, cols, lds, (float*)d, ldd);
+      copy_pad_kernel<float, float><<<grid, 256, 0, st>>>((const float*)(src ? s : nullptr), nr, cols, lds, (float*)d, ldd, dcols);
     LAUNCH_CHECK();
   }
 }
@@ -167,27 +170,74 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
   throw Error(ASTRA_E_UNSUPPORTED, "lstm_fwd_pointwise: kind");
 }
 
-constexpr int BWD_RB = 16;  // rows per CTA in the backward pointwise kernel
+constexpr int BWD_RB = 32;  // rows per CTA in the backward pointwise kernel
+constexpr int BWD_UX = 64;  // units per CTA (threadIdx.x)
+constexpr int BWD_RY = 8;   // row lanes per CTA (threadIdx.y); thread handles rows b0 + ty + 8i
 int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 
-// Thread = one hidden unit (all four gates), CTA row chunk of BWD_RB batch rows.  Column partial
-// sums (db, dα, dβ1, dβ2) are accumulated in registers over the chunk's rows in ascending order
-// and added to partials[chunk][q][col] — one owner per element, steps ordered on the stream, so
-// the reduction order is fixed (R5: no floating-point atomics).
+// CTA = 64 hidden units (all four gates) x 32 batch rows; thread (ux, ty) handles unit u0 + ux for
+// rows b0 + ty, b0 + ty + 8, ...  Column partial sums (db, dα, dβ1, dβ2) are accumulated per thread
+// in ascending row order, combined across the 8 row lanes in ty order through shared memory, and
+// added to partials[chunk][q][col] — one owner per element, steps ordered on the stream, so the
+// reduction order is fixed (R5: no floating-point atomics).
 template <int KIND, typename T, typename TDY>
-__global__ void lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy,
-                                   const float* __restrict__ dh_rec, long ld_dh, float* __restrict__ dc,
-                                   const float* __restrict__ WX, const float* __restrict__ UH,
-                                   const float* __restrict__ c_new, const float* __restrict__ c_prev, GateParams gp,
-                                   T* __restrict__ D_uh, T* __restrict__ D_wx, float* __restrict__ partials, int nq,
-                                   int first) {
-  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void __launch_bounds__(BWD_UX * BWD_RY, 2)
+    lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
+                       long ld_dh, float* __restrict__ dc, const float* __restrict__ WX, const float* __restrict__ UH,
+                       const float* __restrict__ c_new, const float* __restrict__ c_prev, GateParams gp,
+                       T* __restrict__ D_uh, T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
+  __shared__ float red[BWD_RY][16][BWD_UX];
+  const int ux = threadIdx.x, ty = threadIdx.y;
+  const int j = blockIdx.x * BWD_UX + ux;
   const int chunk = blockIdx.y;
-  if (j >= Hp) return;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
-  if (j >= H) {
-    for (int b = b0; b < b1; ++b) {
+  float s[16];
+#pragma unroll
+  for (int i = 0; i < 16; ++i) s[i] = 0.f;
+  if (j < H) {
+    float al[4], be1[4], be2[4], bb[4];
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      const int e = g * H + j;
+      bb[g] = gp.b[e];
+      al[g] = KIND == K_MILSTM ? gp.alpha[e] : 0.f;
+      be1[g] = KIND == K_MILSTM ? gp.beta1[e] : 0.f;
+      be2[g] = KIND == K_MILSTM ? gp.beta2[e] : 0.f;
+    }
+    for (int b = b0 + ty; b < b1; b += BWD_RY) {
+      const long rg = (long)b * NG;
+      float wx[4], uh[4], a[4];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        wx[g] = WX[rg + gcol(g, j)];
+        uh[g] = UH[rg + gcol(g, j)];
+        a[g] = preact<KIND>(wx[g], uh[g], bb[g], al[g], be1[g], be2[g]);
+      }
+      float dh = to_f<TDY>(dy[(long)b * ldy + j]);
+      if (dh_rec) dh = __fadd_rn(dh, dh_rec[(long)b * ld_dh + j]);
+      float dcv = dc[(long)b * Hp + j];
+      float da[4];
+      cell_bwd<KIND>(a, c_prev[(long)b * Hp + j], c_new[(long)b * Hp + j], dh, dcv, da);
+      dc[(long)b * Hp + j] = dcv;
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        s[g] = __fadd_rn(s[g], da[g]);
+        if (KIND == K_MILSTM) {
+          const float duh = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], wx[g]), be1[g]));
+          const float dwx = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], uh[g]), be2[g]));
+          D_uh[rg + gcol(g, j)] = from_f<T>(duh);
+          D_wx[rg + gcol(g, j)] = from_f<T>(dwx);
+          s[4 + g] = __fadd_rn(s[4 + g], __fmul_rn(__fmul_rn(da[g], wx[g]), uh[g]));
+          s[8 + g] = __fadd_rn(s[8 + g], __fmul_rn(da[g], uh[g]));
+          s[12 + g] = __fadd_rn(s[12 + g], __fmul_rn(da[g], wx[g]));
+        } else {
+          D_uh[rg + gcol(g, j)] = from_f<T>(da[g]);
+        }
+      }
+    }
+  } else if (j < Hp) {  // padding units: keep their gradients exactly zero
+    for (int b = b0 + ty; b < b1; b += BWD_RY) {
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
         D_uh[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
@@ -195,62 +245,20 @@ __global__ void lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__
       }
       dc[(long)b * Hp + j] = 0.f;
     }
-    return;
   }
-  float s_b[4] = {0, 0, 0, 0}, s_al[4] = {0, 0, 0, 0}, s_b1[4] = {0, 0, 0, 0}, s_b2[4] = {0, 0, 0, 0};
-  float al[4], be1[4], be2[4], bb[4];
+  const int nv = KIND == K_MILSTM ? 16 : 4;
+  for (int i = 0; i < nv; ++i) red[ty][i][ux] = s[i];
+  __syncthreads();
+  if (j >= Hp) return;
+  // thread (ux, ty) finalises quantities i = ty, ty + 8 (fixed ty order inside)
+  for (int i = ty; i < nv; i += BWD_RY) {
+    float v = 0.f;
 #pragma unroll
-  for (int g = 0; g < 4; ++g) {
-    const int e = g * H + j;
-    bb[g] = gp.b[e];
-    al[g] = KIND == K_MILSTM ? gp.alpha[e] : 0.f;
-    be1[g] = KIND == K_MILSTM ? gp.beta1[e] : 0.f;
-    be2[g] = KIND == K_MILSTM ? gp.beta2[e] : 0.f;
-  }
-  for (int b = b0; b < b1; ++b) {
-    const long rg = (long)b * NG;
-    float wx[4], uh[4], a[4];
-#pragma unroll
-    for (int g = 0; g < 4; ++g) {
-      wx[g] = WX[rg + gcol(g, j)];
-      uh[g] = UH[rg + gcol(g, j)];
-      a[g] = preact<KIND>(wx[g], uh[g], bb[g], al[g], be1[g], be2[g]);
-    }
-    float dh = to_f<TDY>(dy[(long)b * ldy + j]);
-    if (dh_rec) dh = __fadd_rn(dh, dh_rec[(long)b * ld_dh + j]);
-    float dcv = dc[(long)b * Hp + j];
-    float da[4];
-    cell_bwd<KIND>(a, c_prev[(long)b * Hp + j], c_new[(long)b * Hp + j], dh, dcv, da);
-    dc[(long)b * Hp + j] = dcv;
-#pragma unroll
-    for (int g = 0; g < 4; ++g) {
-      s_b[g] = __fadd_rn(s_b[g], da[g]);
-      if (KIND == K_MILSTM) {
-        const float duh = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], wx[g]), be1[g]));
-        const float dwx = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], uh[g]), be2[g]));
-        D_uh[rg + gcol(g, j)] = from_f<T>(duh);
-        D_wx[rg + gcol(g, j)] = from_f<T>(dwx);
-        s_al[g] = __fadd_rn(s_al[g], __fmul_rn(__fmul_rn(da[g], wx[g]), uh[g]));
-        s_b1[g] = __fadd_rn(s_b1[g], __fmul_rn(da[g], uh[g]));
-        s_b2[g] = __fadd_rn(s_b2[g], __fmul_rn(da[g], wx[g]));
-      } else {
-        D_uh[rg + gcol(g, j)] = from_f<T>(da[g]);
-      }
-    }
-  }
-#pragma unroll
-  for (int g = 0; g < 4; ++g) {
-    const long base = (long)chunk * nq * NG + gcol(g, j);
-    float* p0 = partials + base;
-    *p0 = first ? s_b[g] : __fadd_rn(*p0, s_b[g]);
-    if (KIND == K_MILSTM) {
-      float* p1 = partials + base + NG;
-      float* p2 = partials + base + 2L * NG;
-      float* p3 = partials + base + 3L * NG;
-      *p1 = first ? s_al[g] : __fadd_rn(*p1, s_al[g]);
-      *p2 = first ? s_b1[g] : __fadd_rn(*p2, s_b1[g]);
-      *p3 = first ? s_b2[g] : __fadd_rn(*p3, s_b2[g]);
-    }
+    for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[y][i][ux]);
+    const int q = i / 4, g = i % 4;
+    if (q >= nq) continue;
+    float* p = partials + ((long)chunk * nq + q) * NG + gcol(g, j);
+    *p = first ? v : __fadd_rn(*p, v);
   }
 }
 
@@ -259,13 +267,14 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
                           long ld_dh, float* dc, const float* WX, const float* UH, const float* c_new,
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
                           bool first, cudaStream_t st) {
-  dim3 grid(cdiv(Hp, 128), lstm_bwd_row_chunks(B));
+  dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
+  dim3 block(BWD_UX, BWD_RY);
   if (dy_f32 || dy_ot == OT::F32)
-    lstm_bwd_pw_kernel<KIND, T, float><<<grid, 128, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, dc, WX,
+    lstm_bwd_pw_kernel<KIND, T, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, dc, WX,
                                                              UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials,
                                                              nq, first);
   else
-    lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, 128, 0, st>>>(B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec,
+    lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, block, 0, st>>>(B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec,
                                                                      ld_dh, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh,
                                                                      (T*)D_wx, partials, nq, first);
   LAUNCH_CHECK();
@@ -436,52 +445,115 @@ static int key_bits(int V) {
   return b;
 }
 
+// Segmented, deterministic embedding backward.  After a stable radix sort of (token, row), the
+// rows of token v occupy the sorted range [lo_v, hi_v) in ascending row order.  That range is cut
+// into segments of EMB_SEG rows (so a hot Zipf token does not serialise onto one CTA); segment
+// partial sums are taken in row order and the segments of a token are then added in order.
+constexpr int EMB_SEG = 64;
+
+static size_t scan_temp_bytes(int V) {
+  size_t t = 0;
+  cub::DeviceScan::ExclusiveSum(nullptr, t, (const int32_t*)nullptr, (int32_t*)nullptr, V + 1);
+  return round_up(t, 256);
+}
+
 size_t embed_bwd_scratch_bytes(long n, int V) {
   size_t temp = 0;
   cub::DeviceRadixSort::SortPairs(nullptr, temp, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
                                   (int32_t*)nullptr, (int)n, 0, key_bits(V));
-  return round_up(temp, 256) + 3 * round_up(n * 4, 256);
+  const size_t max_seg = (size_t)(n / EMB_SEG + V + 1);
+  return round_up(temp, 256) + 3 * round_up(n * 4, 256) + scan_temp_bytes(V) + 3 * round_up((V + 1) * 4L, 256) +
+         round_up(max_seg * 4, 256);  // + partials (allocated by the caller separately)
 }
 
-// dE rows: block (v, column chunk); rows of token v are the sorted range [lo, hi).
-__global__ void embed_bwd_kernel(const int32_t* __restrict__ skeys, const int32_t* __restrict__ srows, long n,
-                                 const float* __restrict__ dX, long ldx, int I, float* __restrict__ dE) {
+__device__ __forceinline__ long lower_bound_i32(const int32_t* a, long n, int key) {
+  long lo = 0, hi = n;
+  while (lo < hi) {
+    const long mid = (lo + hi) / 2;
+    if (a[mid] < key) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void emb_seg_count_kernel(const int32_t* __restrict__ skeys, long n, int V, int32_t* __restrict__ lo,
+                                     int32_t* __restrict__ nseg) {
+  const int v = blockIdx.x * blockDim.x + threadIdx.x;
+  if (v > V) return;
+  if (v == V) { nseg[V] = 0; return; }
+  const long l = lower_bound_i32(skeys, n, v), h = lower_bound_i32(skeys, n, v + 1);
+  lo[v] = (int32_t)l;
+  nseg[v] = (int32_t)((h - l + EMB_SEG - 1) / EMB_SEG);
+}
+
+// partial[s][c] = Σ rows of segment s (ascending); the owning token is found from segoff.
+__global__ void emb_seg_partial_kernel(const int32_t* __restrict__ skeys, const int32_t* __restrict__ srows, long n,
+                                       int V, const int32_t* __restrict__ lo, const int32_t* __restrict__ segoff,
+                                       const float* __restrict__ dX, long ldx, int I, float* __restrict__ part) {
+  const int s = blockIdx.y;
+  const int total = segoff[V];
+  if (s >= total) return;
+  // token v: last v with segoff[v] <= s
+  int a = 0, b = V;  // invariant segoff[a] <= s < segoff[b]
+  while (b - a > 1) {
+    const int m = (a + b) / 2;
+    if (segoff[m] <= s) a = m; else b = m;
+  }
+  const int v = a;
+  const long l = lo[v];
+  const long h = lower_bound_i32(skeys, n, v + 1);
+  const long r0 = l + (long)(s - segoff[v]) * EMB_SEG;
+  const long r1 = min(h, r0 + EMB_SEG);
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= I) return;
+  float acc = 0.f;
+  for (long k = r0; k < r1; ++k) acc = __fadd_rn(acc, dX[(long)srows[k] * ldx + c]);
+  part[(long)s * I + c] = acc;
+}
+
+__global__ void emb_seg_final_kernel(int V, const int32_t* __restrict__ segoff, const float* __restrict__ part, int I,
+                                     float* __restrict__ dE) {
   const int v = blockIdx.y;
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  __shared__ long lo_hi[2];
-  if (threadIdx.x < 2) {
-    const int key = v + threadIdx.x;  // lower_bound(key)
-    long lo = 0, hi = n;
-    while (lo < hi) {
-      const long mid = (lo + hi) / 2;
-      if (skeys[mid] < key) lo = mid + 1; else hi = mid;
-    }
-    lo_hi[threadIdx.x] = lo;
-  }
-  __syncthreads();
   if (c >= I) return;
-  float s = 0.f;
-  for (long k = lo_hi[0]; k < lo_hi[1]; ++k) s = __fadd_rn(s, dX[(long)srows[k] * ldx + c]);
-  dE[(long)v * I + c] = s;
+  float acc = 0.f;
+  for (int s = segoff[v]; s < segoff[v + 1]; ++s) acc = __fadd_rn(acc, part[(long)s * I + c]);
+  dE[(long)v * I + c] = acc;
 }
 
+size_t embed_bwd_partial_floats(long n, int V, int I) { return (size_t)(n / EMB_SEG + V + 1) * I; }
+
 void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int I, float* dE, void* scratch,
-               size_t scratch_bytes, cudaStream_t st) {
+               size_t scratch_bytes, float* part, cudaStream_t st) {
   size_t temp = 0;
   cub::DeviceRadixSort::SortPairs(nullptr, temp, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
                                   (int32_t*)nullptr, (int)n, 0, key_bits(V));
   temp = round_up(temp, 256);
   char* base = (char*)scratch;
   const size_t nb = round_up(n * 4, 256);
-  ASTRA_CHECK_ARG(scratch_bytes >= temp + 3 * nb, "embed_bwd: scratch too small");
+  const size_t vb = round_up((V + 1) * 4L, 256);
+  const size_t stb = scan_temp_bytes(V);
+  ASTRA_CHECK_ARG(scratch_bytes >= temp + 3 * nb + stb + 3 * vb, "embed_bwd: scratch too small");
   int32_t* rows_in = (int32_t*)(base + temp);
   int32_t* skeys = (int32_t*)(base + temp + nb);
   int32_t* srows = (int32_t*)(base + temp + 2 * nb);
+  char* scan_tmp = base + temp + 3 * nb;
+  int32_t* lo = (int32_t*)(scan_tmp + stb);
+  int32_t* nseg = (int32_t*)(scan_tmp + stb + vb);
+  int32_t* segoff = (int32_t*)(scan_tmp + stb + 2 * vb);
   iota_kernel<<<cdiv(n, 256), 256, 0, st>>>(rows_in, n);
   LAUNCH_CHECK();
   CUDA_TRY(cub::DeviceRadixSort::SortPairs(base, temp, tok, skeys, rows_in, srows, (int)n, 0, key_bits(V), st));
   count_launch(4);
-  embed_bwd_kernel<<<dim3(cdiv(I, 256), V), 256, 0, st>>>(skeys, srows, n, dX, ldx, I, dE);
+  emb_seg_count_kernel<<<cdiv(V + 1, 256), 256, 0, st>>>(skeys, n, V, lo, nseg);
+  LAUNCH_CHECK();
+  size_t stb2 = stb;
+  CUDA_TRY(cub::DeviceScan::ExclusiveSum(scan_tmp, stb2, nseg, segoff, V + 1, st));
+  count_launch(1);
+  const long max_seg = n / EMB_SEG + V;
+  emb_seg_partial_kernel<<<dim3(cdiv(I, 256), (unsigned)max_seg), 256, 0, st>>>(skeys, srows, n, V, lo, segoff, dX,
+                                                                                 ldx, I, part);
+  LAUNCH_CHECK();
+  emb_seg_final_kernel<<<dim3(cdiv(I, 256), V), 256, 0, st>>>(V, segoff, part, I, dE);
   LAUNCH_CHECK();
 }
 

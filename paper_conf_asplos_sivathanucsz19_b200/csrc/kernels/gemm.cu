@@ -65,7 +65,6 @@ static int smem_for(int& stages) {
   CUDA_TRY(cudaGetDevice(&dev));
   CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   stages = TcSmem<BN>::stages_for(maxs);
-  if (stages > 4) stages = 4;
   return TcSmem<BN>::bytes(stages);
 }
 
@@ -178,23 +177,17 @@ __global__ void __launch_bounds__(256) simt_gemm_kernel(const float* __restrict_
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     const int m = m0 + ty * 4 + i;
-    if (m >= M) continue;
+    if (m >= M || m >= epi.Mv) continue;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
       const int n = n0 + tx * 4 + j;
       if (n >= N) continue;
-      int e = n;
-      bool ok = n < epi.Nv;
-      if (epi.perm_u) {
-        const int q = 4 * epi.perm_u;
-        const int tile = n / q, g = (n % q) / epi.perm_u, jj = n % epi.perm_u;
-        const int unit = tile * epi.perm_u + jj;
-        ok = unit < epi.perm_H;
-        e = g * epi.perm_H + unit;
-      }
-      if (!ok || m >= epi.Mv) continue;
-      const float v = __fadd_rn(acc[i][j], epi.bias ? epi.bias[n] : 0.f);
-      reinterpret_cast<float*>(epi.C)[(long)m * epi.ldc + e] = v;
+      bool ok;
+      const int e = epi.map_col(n, ok);
+      if (!ok) continue;
+      const float v = __fadd_rn(acc[i][j], (epi.bias && n < epi.Nv) ? epi.bias[n] : 0.f);
+      float* p = reinterpret_cast<float*>(epi.C) + (long)m * epi.ldc + e;
+      *p = epi.accumulate ? __fadd_rn(*p, v) : v;
     }
   }
 }

@@ -46,16 +46,17 @@ struct TcSmem {
   static constexpr int TMEM_COLS = (2 * BN <= 32) ? 32 : (2 * BN <= 64) ? 64 : (2 * BN <= 128) ? 128 : (2 * BN <= 256) ? 256 : 512;
   static int stages_for(int max_smem) {
     int s = (max_smem - 1024 - 256) / STAGE_BYTES;
-    return s > 6 ? 6 : s;
+    return s > 10 ? 10 : s;
   }
   static int bytes(int stages) { return 1024 + stages * STAGE_BYTES + 256; }
 };
 
-// Generic epilogue: store the fp32 accumulator (optionally + bias[n]) as fp32 or bf16 into a
-// row-major [M][ldc] output.  Output columns can be remapped from the internal gate-interleaved
-// order (units grouped by `perm_u` per gate inside each 4·u-column tile) to the external
-// (i, f, g, o)-blocked order of a [*, 4·perm_H] tensor; rows ≥ Mv and invalid columns are
-// dropped (zero padding of hidden sizes that are not a multiple of the tile).
+// Generic epilogue: store the fp32 accumulator (optionally + bias[n], optionally added onto the
+// fp32 value already in C: out = C_old + acc) as fp32 or bf16 into a row-major [M][ldc] output.
+// Output columns can be remapped from an internal gate layout to the external one:
+//   perm_u  > 0: gate-interleaved tiles — internal n = tile·4u + g·u + j ↔ external g·perm_H + tile·u + j
+//   perm_blk > 0: gate-blocked, padded  — internal n = g·perm_blk + j  ↔ external g·perm_H + j
+// Rows ≥ Mv and invalid (padding) columns are dropped.
 struct EpiStore {
   void* C;
   long ldc;
@@ -63,21 +64,38 @@ struct EpiStore {
   int out_bf16;
   const float* bias;  // indexed by internal column n, may be null
   int perm_u, perm_H; // 0 = identity mapping
+  int perm_blk;
+  int accumulate;
+
+  __device__ __forceinline__ int map_col(int n, bool& ok) const {
+    if (n >= Nv) {  // columns past the GEMM's N (tile overhang) are never stored
+      ok = false;
+      return 0;
+    }
+    if (perm_u) {
+      const int q = 4 * perm_u;
+      const int tile = n / q, g = (n % q) / perm_u, j = n % perm_u;
+      const int unit = tile * perm_u + j;
+      ok = unit < perm_H;
+      return g * perm_H + unit;
+    }
+    if (perm_blk) {
+      const int g = n / perm_blk, j = n % perm_blk;
+      ok = j < perm_H;
+      return g * perm_H + j;
+    }
+    ok = n < Nv;
+    return n;
+  }
 
   __device__ __forceinline__ void store16(int m, int n0, const float (&v)[16]) const {
     if (m >= Mv) return;
-    int e0 = n0;
-    bool contiguous = true;
-    if (perm_u) {
-      const int q = 4 * perm_u;
-      const int tile = n0 / q, g = (n0 % q) / perm_u, j = n0 % perm_u;
-      const int unit = tile * perm_u + j;
-      e0 = g * perm_H + unit;
-      // 16 consecutive internal columns stay inside one gate block when perm_u % 16 == 0
-      if (unit + 16 > perm_H) contiguous = false;
-    } else if (n0 + 16 > Nv) {
-      contiguous = false;
-    }
+    bool ok0;
+    const int e0 = map_col(n0, ok0);
+    bool contiguous = n0 + 16 <= Nv;
+    if (!contiguous) {
+    } else if (perm_u) contiguous = ((n0 % perm_u) + 16 <= perm_u) && ((n0 / (4 * perm_u)) * perm_u + n0 % perm_u + 16 <= perm_H);
+    else if (perm_blk) contiguous = (n0 % perm_blk) + 16 <= perm_H;
     float w[16];
 #pragma unroll
     for (int i = 0; i < 16; ++i) w[i] = v[i] + ((bias && n0 + i < Nv) ? bias[n0 + i] : 0.f);
@@ -102,36 +120,34 @@ struct EpiStore {
         float* p = reinterpret_cast<float*>(C) + (long)m * ldc + e0;
         if ((((uintptr_t)p) & 15) == 0) {
 #pragma unroll
-          for (int i = 0; i < 4; ++i)
-            reinterpret_cast<float4*>(p)[i] = make_float4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
+          for (int i = 0; i < 4; ++i) {
+            float4 o = make_float4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
+            if (accumulate) {
+              const float4 c = reinterpret_cast<const float4*>(p)[i];
+              o.x = __fadd_rn(c.x, o.x); o.y = __fadd_rn(c.y, o.y); o.z = __fadd_rn(c.z, o.z); o.w = __fadd_rn(c.w, o.w);
+            }
+            reinterpret_cast<float4*>(p)[i] = o;
+          }
         } else {
 #pragma unroll
-          for (int i = 0; i < 16; ++i) p[i] = w[i];
+          for (int i = 0; i < 16; ++i) p[i] = accumulate ? __fadd_rn(p[i], w[i]) : w[i];
         }
       }
       return;
     }
 #pragma unroll
     for (int i = 0; i < 16; ++i) {
-      const int n = n0 + i;
-      int e;
       bool ok;
-      if (perm_u) {
-        const int q = 4 * perm_u;
-        const int tile = n / q, g = (n % q) / perm_u, j = n % perm_u;
-        const int unit = tile * perm_u + j;
-        ok = unit < perm_H;
-        e = g * perm_H + unit;
-      } else {
-        ok = n < Nv;
-        e = n;
-      }
+      const int e = map_col(n0 + i, ok);
       if (!ok) continue;
-      if (out_bf16)
+      if (out_bf16) {
         reinterpret_cast<__nv_bfloat16*>(C)[(long)m * ldc + e] = __float2bfloat16_rn(w[i]);
-      else
-        reinterpret_cast<float*>(C)[(long)m * ldc + e] = w[i];
+      } else {
+        float* p = reinterpret_cast<float*>(C) + (long)m * ldc + e;
+        *p = accumulate ? __fadd_rn(*p, w[i]) : w[i];
+      }
     }
+    (void)ok0;
   }
 
   template <int BN>

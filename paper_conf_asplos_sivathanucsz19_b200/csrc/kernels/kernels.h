@@ -22,7 +22,9 @@ void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, lo
 // dst[n][k] = src[k][n] (plain transpose), dst [Np][ldd], padding zero.
 void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, long ldd, cudaStream_t st);
 // Operand copy of an external [rows][cols] (OT or fp32 `src_ot`) into [rows][ldd] of type `ot`.
-void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, void* dst, long ldd, cudaStream_t st);
+// dcols (default ldd): number of destination columns written (the rest of the row is left as is).
+void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, void* dst, long ldd, cudaStream_t st,
+              long dcols = -1);
 // dst fp32 [rows][ldd] ← src fp32 [rows][lds] (cols), zero padding; src null → zeros.
 void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, long ldd, int dcols, cudaStream_t st);
 
@@ -40,6 +42,24 @@ int lstm_bwd_row_chunks(int B);
 void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,
                           cudaStream_t st);
 
+// ---- SCRN [22] / RHN [39] pointwise and scan halves (scrn_rhn_kernels.cu)
+int pw_row_chunks(int B);
+void scrn_scan_fwd(OT ot, int B, int S, int Sp, int T, float alpha, const float* XB, long ldxb, const float* s0,
+                   float* Sf, void* HSs, long ldhs, void* y, long ldy, float* sT, cudaStream_t st);
+void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const float* Z, const float* bh, float* Hf,
+                 void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st);
+void scrn_bwd_pw(OT ot, int B, int H, int Hp, const void* dy, long ldy, bool dy_f32, const float* dh, long ld_dh,
+                 const float* Hf, void* DZ, long ldz, float* part, bool first, cudaStream_t st);
+void scrn_scan_bwd(OT ot, int B, int S, int Sp, int T, float alpha, const void* dys, long ldy, bool dy_f32,
+                   const float* DSP, long ldsp, const float* dsT, void* DSa, long ldsa, float* ds0, cudaStream_t st);
+void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* WX, const float* bl, const float* s_prev,
+                float* s_next, void* s_next_op, void* y, long ldy, float* sT, cudaStream_t st);
+void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const void* dy, long ldy, bool dy_f32,
+                const float* Apre, const float* s_prev, void* DA, float* ds_out, float* part, bool first,
+                cudaStream_t st);
+void reduce_blocked_partials(const float* part, int nchunk, int nq, int H, int Hp, float* out, cudaStream_t st);
+void mirror_blocked_T(OT ot, const float* src, int K, int G, int H, int Hp, void* dst, long ldd, cudaStream_t st);
+
 // ---- LM pieces
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);
 // rowloss[r] = lse - logit[target]; dlog (ot) and dlog32 = (softmax - onehot) * inv_n.
@@ -51,8 +71,9 @@ size_t colsum_scratch_floats(long rows, int cols);
 void colsum(const float* in, long rows, int cols, long ld, float* scratch, float* out, cudaStream_t st);
 // Deterministic embedding backward: dE[v] = Σ_{rows with tok=v} dX[row] in ascending row order.
 size_t embed_bwd_scratch_bytes(long n, int V);
+size_t embed_bwd_partial_floats(long n, int V, int I);
 void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int I, float* dE, void* scratch,
-               size_t scratch_bytes, cudaStream_t st);
+               size_t scratch_bytes, float* partials, cudaStream_t st);
 
 // ---- SGD (K9): p -= lr * g over n elements
 void sgd(float* p, const float* g, size_t n, float lr, cudaStream_t st);

@@ -1,0 +1,335 @@
+// Pointwise / scan kernels of the SCRN [22] and RHN [39] steps (
+// equations: DESIGN.md readings R5-R9, oracle/cells.py).  The GEMM halves run on K1 (bf16 path) or
+// K10 (fp32 path); these kernels are the elementwise halves.  Column partial sums (bias gradients)
+// follow the fixed-order scheme of the LSTM backward kernel (R5).
+#include "cell_math.cuh"
+#include "kernels.h"
+
+namespace astra {
+
+constexpr int PW_UX = 64;  // units per CTA
+constexpr int PW_RY = 8;   // row lanes per CTA
+constexpr int PW_RB = 32;  // rows per CTA
+int pw_row_chunks(int B) { return cdiv(B, PW_RB); }
+
+template <typename T>
+__device__ __forceinline__ float ldv(const void* p, long i) { return to_f<T>(reinterpret_cast<const T*>(p)[i]); }
+
+// ---------------------------------------------------------------------------------- SCRN
+// s_t = (1−α)·xb_t + α·s_{t−1}: one thread per (b, s), sequential over t (K8).
+template <typename T, typename TY>
+__global__ void scrn_scan_fwd_kernel(int B, int S, int T_, float alpha, const float* __restrict__ XB, long ldxb,
+                                     const float* __restrict__ s0, float* __restrict__ Sf, int Sp,
+                                     T* __restrict__ HSs, long ldhs, TY* __restrict__ y, long ldy,
+                                     float* __restrict__ sT) {
+  const int s = blockIdx.x * blockDim.x + threadIdx.x;
+  const int b = blockIdx.y;
+  if (s >= Sp) return;
+  const bool valid = s < S;
+  const float oma = __fsub_rn(1.f, alpha);
+  float cur = (valid && s0) ? s0[(long)b * S + s] : 0.f;
+  Sf[(long)b * Sp + s] = cur;
+  HSs[(long)b * ldhs + s] = from_f<T>(cur);
+  for (int t = 0; t < T_; ++t) {
+    const long r = (long)t * B + b;
+    if (valid) cur = __fadd_rn(__fmul_rn(oma, XB[r * ldxb + s]), __fmul_rn(alpha, cur));
+    Sf[(r + B) * Sp + s] = cur;
+    HSs[(r + B) * ldhs + s] = from_f<T>(cur);
+    if (y && valid) y[r * ldy + s] = from_f<TY>(cur);
+  }
+  if (sT && valid) sT[(long)b * S + s] = cur;
+}
+
+void scrn_scan_fwd(OT ot, int B, int S, int Sp, int T, float alpha, const float* XB, long ldxb, const float* s0,
+                   float* Sf, void* HSs, long ldhs, void* y, long ldy, float* sT, cudaStream_t st) {
+  dim3 grid(cdiv(Sp, 128), B);
+  if (ot == OT::BF16)
+    scrn_scan_fwd_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 128, 0, st>>>(
+        B, S, T, alpha, XB, ldxb, s0, Sf, Sp, (__nv_bfloat16*)HSs, ldhs, (__nv_bfloat16*)y, ldy, sT);
+  else
+    scrn_scan_fwd_kernel<float, float><<<grid, 128, 0, st>>>(B, S, T, alpha, XB, ldxb, s0, Sf, Sp, (float*)HSs, ldhs,
+                                                             (float*)y, ldy, sT);
+  LAUNCH_CHECK();
+}
+
+// h_t = σ((q_t + z_t) + b_h)   (q_t = x_t·A + s_t·P, the hoisted ladder; z_t = h_{t−1}·R)
+template <typename T, typename TY>
+__global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ Q, long ldq,
+                                   const float* __restrict__ Z, const float* __restrict__ bh, float* __restrict__ Hf,
+                                   T* __restrict__ HSh, long ldhs, TY* __restrict__ y, long ldy,
+                                   float* __restrict__ hT) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  const int b = blockIdx.y;
+  if (j >= Hp) return;
+  float h = 0.f;
+  if (j < H) h = sigm(__fadd_rn(__fadd_rn(Q[(long)b * ldq + j], Z[(long)b * Hp + j]), bh[j]));
+  Hf[(long)b * Hp + j] = h;
+  HSh[(long)b * ldhs + j] = from_f<T>(h);
+  if (j < H) {
+    if (y) y[(long)b * ldy + j] = from_f<TY>(h);
+    if (hT) hT[(long)b * H + j] = h;
+  }
+}
+
+void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const float* Z, const float* bh, float* Hf,
+                 void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st) {
+  dim3 grid(cdiv(Hp, 128), B);
+  if (ot == OT::BF16)
+    scrn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 128, 0, st>>>(
+        B, H, Hp, Q, ldq, Z, bh, Hf, (__nv_bfloat16*)HSh, ldhs, (__nv_bfloat16*)y, ldy, hT);
+  else
+    scrn_fwd_pw_kernel<float, float><<<grid, 128, 0, st>>>(B, H, Hp, Q, ldq, Z, bh, Hf, (float*)HSh, ldhs, (float*)y,
+                                                           ldy, hT);
+  LAUNCH_CHECK();
+}
+
+// dz_t = (dy^h_t + dh_rec)·h_t·(1 − h_t); db_h partials over rows (fixed order)
+template <typename T, typename TDY>
+__global__ void __launch_bounds__(PW_UX * PW_RY)
+    scrn_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh,
+                       long ld_dh, const float* __restrict__ Hf, T* __restrict__ DZ, long ldz,
+                       float* __restrict__ part, int first) {
+  __shared__ float red[PW_RY][PW_UX];
+  const int ux = threadIdx.x, ty = threadIdx.y;
+  const int j = blockIdx.x * PW_UX + ux;
+  const int chunk = blockIdx.y;
+  const int b0 = chunk * PW_RB, b1 = min(B, b0 + PW_RB);
+  float sacc = 0.f;
+  if (j < Hp) {
+    for (int b = b0 + ty; b < b1; b += PW_RY) {
+      float dz = 0.f;
+      if (j < H) {
+        float g = to_f<TDY>(dy[(long)b * ldy + j]);
+        if (dh) g = __fadd_rn(g, dh[(long)b * ld_dh + j]);
+        const float h = Hf[(long)b * Hp + j];
+        dz = __fmul_rn(__fmul_rn(g, h), __fsub_rn(1.f, h));
+      }
+      DZ[(long)b * ldz + j] = from_f<T>(dz);
+      sacc = __fadd_rn(sacc, dz);
+    }
+  }
+  red[ty][ux] = sacc;
+  __syncthreads();
+  if (ty == 0 && j < Hp) {
+    float v = 0.f;
+#pragma unroll
+    for (int y = 0; y < PW_RY; ++y) v = __fadd_rn(v, red[y][ux]);
+    float* p = part + (long)chunk * Hp + j;
+    *p = first ? v : __fadd_rn(*p, v);
+  }
+}
+
+void scrn_bwd_pw(OT ot, int B, int H, int Hp, const void* dy, long ldy, bool dy_f32, const float* dh, long ld_dh,
+                 const float* Hf, void* DZ, long ldz, float* part, bool first, cudaStream_t st) {
+  dim3 grid(cdiv(Hp, PW_UX), pw_row_chunks(B)), block(PW_UX, PW_RY);
+  if (ot == OT::BF16) {
+    if (dy_f32)
+      scrn_bwd_pw_kernel<__nv_bfloat16, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh, ld_dh,
+                                                                       Hf, (__nv_bfloat16*)DZ, ldz, part, first);
+    else
+      scrn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, block, 0, st>>>(
+          B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh, ld_dh, Hf, (__nv_bfloat16*)DZ, ldz, part, first);
+  } else {
+    scrn_bwd_pw_kernel<float, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh, ld_dh, Hf,
+                                                             (float*)DZ, ldz, part, first);
+  }
+  LAUNCH_CHECK();
+}
+
+// Reverse scan (K8): ds_t = dy^s_t + (dz_t·Pᵀ) + [t = T−1 ? ds_T : α·ds_{t+1}]; writes (1−α)·ds_t as
+// the operand of dBm and dx, and ds0 = α·ds_1.
+template <typename T, typename TDY>
+__global__ void scrn_scan_bwd_kernel(int B, int S, int Sp, int T_, float alpha, const TDY* __restrict__ dys,
+                                     long ldy, const float* __restrict__ DSP, long ldsp, const float* __restrict__ dsT,
+                                     T* __restrict__ DSa, long ldsa, float* __restrict__ ds0) {
+  const int s = blockIdx.x * blockDim.x + threadIdx.x;
+  const int b = blockIdx.y;
+  if (s >= Sp) return;
+  const bool valid = s < S;
+  const float oma = __fsub_rn(1.f, alpha);
+  float ds = 0.f;
+  for (int t = T_ - 1; t >= 0; --t) {
+    const long r = (long)t * B + b;
+    float v = 0.f;
+    if (valid) {
+      v = __fadd_rn(to_f<TDY>(dys[r * ldy + s]), DSP[r * ldsp + s]);
+      const float carry = (t == T_ - 1) ? (dsT ? dsT[(long)b * S + s] : 0.f) : __fmul_rn(alpha, ds);
+      v = __fadd_rn(v, carry);
+    }
+    ds = v;
+    DSa[r * ldsa + s] = from_f<T>(__fmul_rn(oma, ds));
+  }
+  if (ds0 && valid) ds0[(long)b * S + s] = __fmul_rn(alpha, ds);
+}
+
+void scrn_scan_bwd(OT ot, int B, int S, int Sp, int T, float alpha, const void* dys, long ldy, bool dy_f32,
+                   const float* DSP, long ldsp, const float* dsT, void* DSa, long ldsa, float* ds0, cudaStream_t st) {
+  dim3 grid(cdiv(Sp, 128), B);
+  if (ot == OT::BF16) {
+    if (dy_f32)
+      scrn_scan_bwd_kernel<__nv_bfloat16, float><<<grid, 128, 0, st>>>(B, S, Sp, T, alpha, (const float*)dys, ldy, DSP,
+                                                                       ldsp, dsT, (__nv_bfloat16*)DSa, ldsa, ds0);
+    else
+      scrn_scan_bwd_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 128, 0, st>>>(
+          B, S, Sp, T, alpha, (const __nv_bfloat16*)dys, ldy, DSP, ldsp, dsT, (__nv_bfloat16*)DSa, ldsa, ds0);
+  } else {
+    scrn_scan_bwd_kernel<float, float><<<grid, 128, 0, st>>>(B, S, Sp, T, alpha, (const float*)dys, ldy, DSP, ldsp,
+                                                             dsT, (float*)DSa, ldsa, ds0);
+  }
+  LAUNCH_CHECK();
+}
+
+// ---------------------------------------------------------------------------------- RHN
+// Micro-step ℓ of time t (coupled carry): a = z + b_ℓ (+ wx_t at ℓ = 0), stored back as the saved
+// pre-activation; h = tanh a_H, τ = σ(a_T); s' = h·τ + s·(1 − τ).  Internal columns: g·Hp + j.
+template <typename T, typename TY>
+__global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, const float* __restrict__ WX,
+                                  const float* __restrict__ bl, const float* __restrict__ s_prev,
+                                  float* __restrict__ s_next, T* __restrict__ s_next_op, TY* __restrict__ y, long ldy,
+                                  float* __restrict__ sT) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  const int b = blockIdx.y;
+  if (j >= Hp) return;
+  const long rz = (long)b * 2 * Hp;
+  float s_new = 0.f;
+  if (j < H) {
+    float aH = __fadd_rn(Z[rz + j], bl[j]);
+    float aT = __fadd_rn(Z[rz + Hp + j], bl[H + j]);
+    if (WX) {
+      aH = __fadd_rn(aH, WX[rz + j]);
+      aT = __fadd_rn(aT, WX[rz + Hp + j]);
+    }
+    Z[rz + j] = aH;
+    Z[rz + Hp + j] = aT;
+    const float h = tanh_(aH), tau = sigm(aT);
+    const float s = s_prev[(long)b * Hp + j];
+    s_new = __fadd_rn(__fmul_rn(h, tau), __fmul_rn(s, __fsub_rn(1.f, tau)));
+    if (y) y[(long)b * ldy + j] = from_f<TY>(s_new);
+    if (sT) sT[(long)b * H + j] = s_new;
+  }
+  s_next[(long)b * Hp + j] = s_new;
+  s_next_op[(long)b * Hp + j] = from_f<T>(s_new);
+}
+
+void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* WX, const float* bl, const float* s_prev,
+                float* s_next, void* s_next_op, void* y, long ldy, float* sT, cudaStream_t st) {
+  dim3 grid(cdiv(Hp, 128), B);
+  if (ot == OT::BF16)
+    rhn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 128, 0, st>>>(
+        B, H, Hp, Z, WX, bl, s_prev, s_next, (__nv_bfloat16*)s_next_op, (__nv_bfloat16*)y, ldy, sT);
+  else
+    rhn_fwd_pw_kernel<float, float><<<grid, 128, 0, st>>>(B, H, Hp, Z, WX, bl, s_prev, s_next, (float*)s_next_op,
+                                                          (float*)y, ldy, sT);
+  LAUNCH_CHECK();
+}
+
+// Backward of micro-step ℓ:  ds = ds_in (+ dy_t at ℓ = L−1); dh = ds·τ; dτ = ds·(h − s_prev);
+// da_H = dh·(1 − h²); da_T = dτ·τ·(1 − τ); ds_out = ds·(1 − τ) (the BPTT GEMM then adds da·R_ℓᵀ).
+template <typename T, typename TDY>
+__global__ void __launch_bounds__(PW_UX * PW_RY)
+    rhn_bwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ ds_in, const TDY* __restrict__ dy, long ldy,
+                      const float* __restrict__ Apre, const float* __restrict__ s_prev, T* __restrict__ DA,
+                      float* __restrict__ ds_out, float* __restrict__ part, int first) {
+  __shared__ float red[PW_RY][2][PW_UX];
+  const int ux = threadIdx.x, ty = threadIdx.y;
+  const int j = blockIdx.x * PW_UX + ux;
+  const int chunk = blockIdx.y;
+  const int b0 = chunk * PW_RB, b1 = min(B, b0 + PW_RB);
+  float sH = 0.f, sT_ = 0.f;
+  if (j < Hp) {
+    for (int b = b0 + ty; b < b1; b += PW_RY) {
+      const long rz = (long)b * 2 * Hp;
+      float daH = 0.f, daT = 0.f, dso = 0.f;
+      if (j < H) {
+        float ds = ds_in[(long)b * Hp + j];
+        if (dy) ds = __fadd_rn(to_f<TDY>(dy[(long)b * ldy + j]), ds);
+        const float h = tanh_(Apre[rz + j]), tau = sigm(Apre[rz + Hp + j]);
+        const float sp = s_prev[(long)b * Hp + j];
+        const float dh = __fmul_rn(ds, tau);
+        const float dtau = __fmul_rn(ds, __fsub_rn(h, sp));
+        daH = __fmul_rn(dh, __fsub_rn(1.f, __fmul_rn(h, h)));
+        daT = __fmul_rn(__fmul_rn(dtau, tau), __fsub_rn(1.f, tau));
+        dso = __fmul_rn(ds, __fsub_rn(1.f, tau));
+      }
+      DA[rz + j] = from_f<T>(daH);
+      DA[rz + Hp + j] = from_f<T>(daT);
+      ds_out[(long)b * Hp + j] = dso;
+      sH = __fadd_rn(sH, daH);
+      sT_ = __fadd_rn(sT_, daT);
+    }
+  }
+  red[ty][0][ux] = sH;
+  red[ty][1][ux] = sT_;
+  __syncthreads();
+  if (ty < 2 && j < Hp) {
+    float v = 0.f;
+#pragma unroll
+    for (int y = 0; y < PW_RY; ++y) v = __fadd_rn(v, red[y][ty][ux]);
+    float* p = part + (long)chunk * 2 * Hp + ty * Hp + j;
+    *p = first ? v : __fadd_rn(*p, v);
+  }
+}
+
+void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const void* dy, long ldy, bool dy_f32,
+                const float* Apre, const float* s_prev, void* DA, float* ds_out, float* part, bool first,
+                cudaStream_t st) {
+  dim3 grid(cdiv(Hp, PW_UX), pw_row_chunks(B)), block(PW_UX, PW_RY);
+  if (ot == OT::BF16) {
+    if (dy_f32 || !dy)
+      rhn_bwd_pw_kernel<__nv_bfloat16, float><<<grid, block, 0, st>>>(B, H, Hp, ds_in, (const float*)dy, ldy, Apre,
+                                                                      s_prev, (__nv_bfloat16*)DA, ds_out, part, first);
+    else
+      rhn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, block, 0, st>>>(
+          B, H, Hp, ds_in, (const __nv_bfloat16*)dy, ldy, Apre, s_prev, (__nv_bfloat16*)DA, ds_out, part, first);
+  } else {
+    rhn_bwd_pw_kernel<float, float><<<grid, block, 0, st>>>(B, H, Hp, ds_in, (const float*)dy, ldy, Apre, s_prev,
+                                                            (float*)DA, ds_out, part, first);
+  }
+  LAUNCH_CHECK();
+}
+
+// out[q·Hq + j] (external, j < H) = Σ_chunk part[chunk][q·Hp_ + j] in chunk order, for q < nq blocks.
+__global__ void reduce_blocked_partials_kernel(const float* __restrict__ part, int nchunk, int nq, int H, int Hp_,
+                                               float* __restrict__ out) {
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= nq * H) return;
+  const int q = e / H, j = e % H;
+  float s = 0.f;
+  for (int c = 0; c < nchunk; ++c) s = __fadd_rn(s, part[(long)c * nq * Hp_ + q * Hp_ + j]);
+  out[e] = s;
+}
+
+void reduce_blocked_partials(const float* part, int nchunk, int nq, int H, int Hp, float* out, cudaStream_t st) {
+  reduce_blocked_partials_kernel<<<cdiv((long)nq * H, 256), 256, 0, st>>>(part, nchunk, nq, H, Hp, out);
+  LAUNCH_CHECK();
+}
+
+// dst[g·Hp + j][k] = src[k][g·H + j] for a gate-blocked [K][G·H] matrix (mirror rows, padding zero).
+template <typename T>
+__global__ void mirror_blocked_T_kernel(const float* __restrict__ src, int K, int G, int H, int Hp,
+                                        T* __restrict__ dst, long ldd) {
+  __shared__ float tile[32][33];
+  const int r0 = blockIdx.x * 32, k0 = blockIdx.y * 32;
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  for (int i = ty; i < 32; i += 8) {
+    const int k = k0 + i, r = r0 + tx;
+    const int g = r / Hp, j = r % Hp;
+    tile[i][tx] = (k < K && g < G && j < H) ? src[(long)k * G * H + g * H + j] : 0.f;
+  }
+  __syncthreads();
+  for (int i = ty; i < 32; i += 8) {
+    const int r = r0 + i, k = k0 + tx;
+    if (r < G * Hp && k < ldd) dst[(long)r * ldd + k] = from_f<T>(tile[tx][i]);
+  }
+}
+
+void mirror_blocked_T(OT ot, const float* src, int K, int G, int H, int Hp, void* dst, long ldd, cudaStream_t st) {
+  dim3 grid(cdiv((long)G * Hp, 32), cdiv(ldd, 32)), block(32, 8);
+  if (ot == OT::BF16)
+    mirror_blocked_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, G, H, Hp, (__nv_bfloat16*)dst, ldd);
+  else
+    mirror_blocked_T_kernel<float><<<grid, block, 0, st>>>(src, K, G, H, Hp, (float*)dst, ldd);
+  LAUNCH_CHECK();
+}
+
+}  // namespace astra

@@ -1,13 +1,18 @@
 // L1 runtime: per-cell step plan, workspace carving, the executor of one training step for each
 // variant, and the LM wrapper.  The tuner (L2) chooses the Variant; every variant computes the
 // same bits (R1-R7).
+//
+// Cell families (each a subclass with its own plan):
+//   LstmCell  — LSTM, MI-LSTM [36], subLSTM [8]      (cell_lstm.cpp)
+//   ScrnCell  — SC-RNN / SCRN [22]                    (cell_scrn.cpp)
+//   RhnCell   — recurrent highway network [39]        (cell_rhn.cpp)
 #pragma once
 #include <cuda_runtime.h>
 
 #include <map>
-#include <tuple>
 #include <memory>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "../common.h"
@@ -23,7 +28,6 @@ struct ParamInfo {
   int rows, cols;
 };
 
-// One binding of every adaptive variable (the enumerator's output for this cell, §8(a.9)).
 // K1 kernel choice for one GEMM role (B1, "GEMM kernel selection", as a choice among our
 // own sm_100a kernels): CTA tile width and cluster multicast shape.
 struct KCfg {
@@ -33,6 +37,7 @@ struct KCfg {
 enum GemmRole { G_A1 = 0, G_REC, G_BPTT, G_DU, G_DW, G_DX, G_HEAD, G_ROLES };
 extern const char* const ROLE_NAMES[G_ROLES];
 
+// One binding of every adaptive variable (the enumerator's output for a cell).
 struct Variant {
   KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
@@ -48,24 +53,27 @@ struct GemmSpec {
   int M = 0, N = 0, K = 0;
 };
 
+Mat2 mat(const void* p, long inner, long outer, long ld, long z = 1, long zstride = 0);
+EpiStore epi(void* C, long ldc, int Mv, int Nv, int out_bf16 = 0, const float* bias = nullptr);
+EpiStore epi_perm(void* C, long ldc, int Mv, int Nv, int perm_u, int perm_blk, int perm_H);
+inline EpiStore accum(EpiStore e) { e.accumulate = 1; return e; }
+
 enum Region { R_A1 = 0, R_FWD, R_HEAD, R_BPTT, R_DU, R_DW, R_DX, R_SE4, R_STEP, R_COUNT };
+
+// A segment of the head weight's K dimension: operand columns [k0, k0+n) ↔ W_o rows [r0, r0+n).
+struct KSeg { int k0, r0, n; };
 
 class Cell {
  public:
   explicit Cell(const astra_cell_desc& d);
-  ~Cell();
+  virtual ~Cell();
 
   astra_cell_desc d;
-  int kind;
   OT ot;
-  int H, I, B, T, Hp, Ip, NG, Hout;
+  int H, I, B, T, Hp, Ip, Hout;
   std::vector<ParamInfo> params;
   size_t n_params = 0;
-
-  // workspace layout (byte offsets)
-  size_t off_X, off_WX, off_UH, off_C, off_H, off_Wm, off_Um, saved_bytes;
-  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part, off_dXf, scratch_bytes;
-  int nchunk;
+  size_t saved_bytes = 0, scratch_bytes = 0;
 
   // binding
   float* P = nullptr;
@@ -88,10 +96,11 @@ class Cell {
   std::vector<Variant> configs_seen;
   int tune_reps = 3, rep_i = 0;
   tuner::Metrics rep_min;
-  bool step_pending = false;
   cudaEvent_t ev[R_COUNT][2];
   bool region_used[R_COUNT];
   bool profiling = true;
+  std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
+  std::map<std::tuple<int, int, int, int>, TcGemm> tc_cache;
 
   // NCCL
   void* nccl_comm = nullptr;
@@ -99,49 +108,59 @@ class Cell {
 
   // LM mode hooks (set by LM)
   bool lm_mode = false;
-  const float* lm_dy = nullptr;  // fp32 [T*B][Hp] internal dY for backward
-  int lm_V = 0;                  // vocabulary of the owning LM (head GEMM shapes)
+  const float* lm_dy = nullptr;  // fp32 [T*B][y_width()] internal dY for the backward
+  int lm_V = 0;
 
+  // ---- per-family interface
+  virtual void forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT) = 0;
+  virtual void backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0) = 0;
+  virtual void* x_operand() = 0;                 // [T*B][Ip] operand buffer (the LM gathers here)
+  virtual Mat2 y_operand() = 0;                  // [T*B][y_width()] operand (A of the head GEMM)
+  virtual int y_width() const = 0;               // padded K of the head
+  virtual std::vector<KSeg> y_segments() const = 0;
+  virtual int c_width() const { return H; }      // width of the second state (c or s); 0 = none
+  virtual void role_shape(int role, int& M, int& N) const = 0;
+
+  // ---- shared machinery
+  void add_param(const char* n, int r, int c);
   size_t find_param(const std::string& n) const;
   float* p(const std::string& n) { return P + find_param(n); }
   float* g(const std::string& n) { return G + find_param(n); }
-
   void bind(float* params, float* grads, void* saved_p, void* scratch_p);
-  void forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT);
-  void backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0);
   void sgd_step(float lr);
   void allreduce_grads(float* grads, size_t n, cudaStream_t after);
-
-  // internal buffers
-  template <typename T> T* sv(size_t off) { return reinterpret_cast<T*>(saved + off); }
-  template <typename T> T* sc(size_t off) { return reinterpret_cast<T*>(scratch + off); }
   size_t esz() const { return ot_size(ot); }
-  void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
-
-  // GEMM execution
+  template <typename T_> T_* sv(size_t off) { return reinterpret_cast<T_*>(saved + off); }
+  template <typename T_> T_* sc(size_t off) { return reinterpret_cast<T_*>(scratch + off); }
   void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st);
-  std::map<std::tuple<int, int, int, int>, TcGemm> tc_cache;
-  std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
-  void role_shape(int role, int& M, int& N) const;
-
-  // profiling regions (cudaEvent pairs)
   void mark(Region r, int which, cudaStream_t st);
-  // tuner
   void tuner_setup();
   void apply_config(const tuner::Config& c);
   int tune_next();
   std::string report();
 };
 
+std::unique_ptr<Cell> make_cell(const astra_cell_desc& d);
+
+// Byte-offset allocator for workspace carving (256-byte aligned regions).
+struct Carve {
+  size_t o = 0;
+  size_t take(size_t bytes) {
+    size_t r = o;
+    o = (o + bytes + 255) / 256 * 256;
+    return r;
+  }
+};
+
 class LM {
  public:
   LM(Cell* c, int vocab);
   Cell* cell;
-  int V, Vp;
+  int V, Vp, Yw;
   size_t n_cell, n_params;
   std::vector<ParamInfo> params;
   size_t off_logits, off_dlog, off_dlog32, off_rowloss, off_dY, off_Wo, off_colsum, off_sort, off_h, off_c,
-      off_cellsaved, off_cellscratch, off_loss, ws_bytes;
+      off_cellsaved, off_cellscratch, off_loss, off_embpart, off_dx, ws_bytes;
   size_t sort_bytes;
   float* P = nullptr;
   float* G = nullptr;

@@ -1,0 +1,317 @@
+// L1 runtime, shared machinery of every cell family: parameters, binding, workspace, the GEMM
+// dispatch (tcgen05 for the bf16 path, SIMT for the fp32 path), cudaEvent-pair profiling regions
+// (P:286-288), the tuner glue (L2) and the DP gradient sum (K11).
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <sstream>
+
+#include "cell.h"
+
+namespace astra {
+
+const char* const ROLE_NAMES[G_ROLES] = {"a1", "rec", "bptt", "du", "dw", "dx", "head"};
+
+std::string Variant::str() const {
+  std::ostringstream o;
+  for (int r = 0; r < G_ROLES; ++r) o << ROLE_NAMES[r] << "=" << g[r].bn << "." << g[r].cm << "." << g[r].cn << ",";
+  o << "wg_side=" << wg_side;
+  return o.str();
+}
+
+Variant Variant::parse(const std::string& s) {
+  Variant v;
+  size_t p = 0;
+  while (p < s.size()) {
+    size_t q = s.find(',', p);
+    if (q == std::string::npos) q = s.size();
+    const std::string kv = s.substr(p, q - p);
+    p = q + 1;
+    if (kv.empty()) continue;
+    const size_t eq = kv.find('=');
+    ASTRA_CHECK_ARG(eq != std::string::npos, "variant: expected key=value, got '" + kv + "'");
+    const std::string k = kv.substr(0, eq), val = kv.substr(eq + 1);
+    if (k == "wg_side") {
+      v.wg_side = std::stoi(val);
+      ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    int r = -1;
+    for (int i = 0; i < G_ROLES; ++i)
+      if (k == ROLE_NAMES[i]) r = i;
+    ASTRA_CHECK_ARG(r >= 0, "variant: unknown variable '" + k + "'");
+    KCfg c;
+    int n = std::sscanf(val.c_str(), "%d.%d.%d", &c.bn, &c.cm, &c.cn);
+    ASTRA_CHECK_ARG(n >= 1, "variant: bad kernel choice '" + val + "'");
+    if (n < 3) c.cn = 1;
+    if (n < 2) c.cm = 1;
+    ASTRA_CHECK_ARG((c.bn == 64 || c.bn == 128 || c.bn == 256) && (c.cm == 1 || c.cm == 2 || c.cm == 4) &&
+                        (c.cn == 1 || c.cn == 2 || c.cn == 4) && c.cm * c.cn <= 8,
+                    "variant: tile width must be 64/128/256 and cluster cm, cn in {1,2,4} with cm*cn <= 8");
+    v.g[r] = c;
+  }
+  return v;
+}
+
+Mat2 mat(const void* p, long inner, long outer, long ld, long z, long zstride) {
+  Mat2 m;
+  m.ptr = p; m.inner = inner; m.outer = outer; m.ld = ld; m.z = z; m.zstride = zstride;
+  return m;
+}
+EpiStore epi(void* C, long ldc, int Mv, int Nv, int out_bf16, const float* bias) {
+  EpiStore e;
+  std::memset(&e, 0, sizeof(e));
+  e.C = C; e.ldc = ldc; e.Mv = Mv; e.Nv = Nv; e.out_bf16 = out_bf16; e.bias = bias;
+  return e;
+}
+EpiStore epi_perm(void* C, long ldc, int Mv, int Nv, int perm_u, int perm_blk, int perm_H) {
+  EpiStore e = epi(C, ldc, Mv, Nv);
+  e.perm_u = perm_u; e.perm_blk = perm_blk; e.perm_H = perm_H;
+  return e;
+}
+
+Cell::Cell(const astra_cell_desc& dd) : d(dd) {
+  ASTRA_CHECK_ARG(d.hidden > 0 && d.input > 0 && d.batch > 0 && d.seq > 0, "cell: sizes must be positive");
+  ASTRA_CHECK_ARG(d.dtype == ASTRA_BF16 || d.dtype == ASTRA_FP32, "cell: dtype must be ASTRA_BF16 or ASTRA_FP32");
+  ot = d.dtype == ASTRA_BF16 ? OT::BF16 : OT::F32;
+  H = d.hidden; I = d.input; B = d.batch; T = d.seq;
+  Hp = (int)round_up(H, 64);
+  Ip = (int)round_up(I, 64);
+  Hout = H;
+  ASTRA_CHECK_ARG((long)T * B < (1L << 31) / 64, "cell: T*B too large");
+  for (int r = 0; r < R_COUNT; ++r) region_used[r] = false;
+  std::memset(ev, 0, sizeof(ev));
+}
+
+void Cell::add_param(const char* n, int r, int c) {
+  params.push_back({n, n_params, r, c});
+  n_params = (n_params + (size_t)r * c + 63) / 64 * 64;   // every tensor 256-byte aligned
+}
+
+Cell::~Cell() {
+  for (int r = 0; r < R_COUNT; ++r)
+    for (int w = 0; w < 2; ++w)
+      if (ev[r][w]) cudaEventDestroy(ev[r][w]);
+  if (ev_fork) cudaEventDestroy(ev_fork);
+  if (ev_join) cudaEventDestroy(ev_join);
+  if (nccl_comm) ncclCommDestroy((ncclComm_t)nccl_comm);
+}
+
+size_t Cell::find_param(const std::string& n) const {
+  for (auto& p : params)
+    if (p.name == n) return p.offset;
+  throw Error(ASTRA_E_ARG, "no parameter " + n);
+}
+
+void Cell::bind(float* pp, float* gg, void* sv_p, void* sc_p) {
+  ASTRA_CHECK_ARG(pp && gg && sv_p && sc_p, "bind: null pointer");
+  ASTRA_CHECK_ARG(((uintptr_t)pp & 255) == 0 && ((uintptr_t)gg & 255) == 0 && ((uintptr_t)sv_p & 255) == 0 &&
+                      ((uintptr_t)sc_p & 255) == 0,
+                  "bind: pointers must be 256-byte aligned");
+  CUDA_TRY(cudaSetDevice(d.device));
+  P = pp; G = gg; saved = (char*)sv_p; scratch = (char*)sc_p;
+  tc_cache.clear();
+  if (!ev_fork) {
+    CUDA_TRY(cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming));
+    CUDA_TRY(cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming));
+    for (int r = 0; r < R_COUNT; ++r)
+      for (int w = 0; w < 2; ++w) CUDA_TRY(cudaEventCreate(&ev[r][w]));
+  }
+  bound = true;
+  fwd_done = false;
+}
+
+void Cell::mark(Region r, int which, cudaStream_t st) {
+  if (!profiling) return;
+  CUDA_TRY(cudaEventRecord(ev[r][which], st));
+  if (which) region_used[r] = true;
+}
+
+void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st) {
+  if (ot == OT::BF16) {
+    auto key = std::make_tuple(id, k.bn, k.cm, k.cn);
+    auto it = tc_cache.find(key);
+    if (it == tc_cache.end()) {
+      TcGemm g;
+      tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, k.cm, k.cn);
+      it = tc_cache.emplace(key, g).first;
+    }
+    tc_gemm_launch(it->second, e, az, bz, st);
+  } else {
+    const float* A = (const float*)s.A.ptr + (long)az * s.A.zstride;
+    const float* Bm = (const float*)s.B.ptr + (long)bz * s.B.zstride;
+    long sam, sak, sbk, sbn;
+    if (!s.a_mn) { sam = s.A.ld; sak = 1; } else { sam = 1; sak = s.A.ld; }
+    if (!s.b_mn) { sbk = 1; sbn = s.B.ld; } else { sbk = s.B.ld; sbn = 1; }
+    simt_gemm(A, sam, sak, Bm, sbk, sbn, s.M, s.N, s.K, e, st);
+  }
+}
+
+void Cell::allreduce_grads(float* grads, size_t n, cudaStream_t after) {
+  ASTRA_CHECK_STATE(nccl_comm, "allreduce: astra_comm_init not called");
+  cudaStream_t cs = comm_st ? comm_st : after;
+  if (cs != after) {
+    CUDA_TRY(cudaEventRecord(ev_fork, after));
+    CUDA_TRY(cudaStreamWaitEvent(cs, ev_fork, 0));
+  }
+  ncclResult_t r = ncclAllReduce(grads, grads, n, ncclFloat, ncclSum, (ncclComm_t)nccl_comm, cs);
+  if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
+  count_launch();
+  scale_inplace(grads, n, 1.0f / (float)world, cs);
+  if (cs != after) {
+    CUDA_TRY(cudaEventRecord(ev_join, cs));
+    CUDA_TRY(cudaStreamWaitEvent(after, ev_join, 0));
+  }
+}
+
+void Cell::sgd_step(float lr) {
+  ASTRA_CHECK_STATE(bound, "sgd: not bound");
+  sgd(P, G, n_params, lr, main_st);
+}
+
+// ------------------------------------------------------------------------ tuner glue
+// The enumerator's static pruning (A19): per GEMM role, the kernel choices whose tile
+// and cluster shape fit the problem; the default (Variant()) first.
+static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 2, 1}, {256, 4, 1}, {256, 2, 2},
+                                  {256, 1, 2}, {128, 2, 1}, {128, 4, 1}, {128, 2, 2}, {128, 1, 2}, {64, 2, 1},
+                                  {64, 4, 1}, {64, 2, 2}};
+
+void Cell::tuner_setup() {
+  const Variant def;
+  std::string par;
+  const char* metric[G_ROLES] = {"t_a1", "t_fwd", "t_bptt", "t_du", "t_dw", "t_dx", "t_head"};
+  if (ot == OT::BF16) {
+    for (int r = 0; r < G_ROLES; ++r) {
+      if (r == G_HEAD && !lm_mode) continue;
+      int M, N;
+      role_shape(r, M, N);
+      if (M <= 0 || N <= 0) continue;
+      allowed[r].clear();
+      allowed[r].push_back(def.g[r]);
+      for (const KCfg& k : CANDIDATES) {
+        if (k == def.g[r]) continue;
+        const int num_m = cdiv(M, TC_BM), num_n = cdiv(N, k.bn);
+        if (k.bn > 64 && N <= k.bn / 2) continue;                                     // tile wider than N
+        if (k.cm > num_m || k.cn > num_n) continue;                                    // idle cluster ranks
+        allowed[r].push_back(k);
+      }
+      par += std::string(" (leaf g_") + ROLE_NAMES[r] + " " + std::to_string(allowed[r].size()) + " " + metric[r] + ")";
+    }
+  }
+  std::string t = par.empty() ? "" : "(par" + par + ")";
+  if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
+  if (t.empty()) t = "(leaf none 1 t_step)";
+  tree.reset(new tuner::Tree(tuner::parse(t)));
+  wirer.reset(new tuner::Wirer(tree.get()));
+  wirer->start();
+  configs_seen.clear();
+  tuner::Config c;
+  if (wirer->propose(c)) apply_config(c);
+  rep_i = 0;
+}
+
+void Cell::apply_config(const tuner::Config& c) {
+  Variant v = var;
+  for (size_t i = 0; i < tree->avs.size(); ++i) {
+    const std::string& n = tree->avs[i];
+    const int o = c[i];
+    if (n == "wg_side") { v.wg_side = o; continue; }
+    for (int r = 0; r < G_ROLES; ++r)
+      if (n == std::string("g_") + ROLE_NAMES[r]) v.g[r] = allowed[r].at(o);
+  }
+  var = v;
+  configs_seen.push_back(v);
+}
+
+static float elapsed(cudaEvent_t a, cudaEvent_t b) {
+  float ms = 0.f;
+  if (cudaEventElapsedTime(&ms, a, b) != cudaSuccess) {
+    cudaGetLastError();
+    return 1e30f;
+  }
+  return ms;
+}
+
+// One call per step (after the step's work is enqueued).  Per configuration: one warm-up step
+// (absorbs lazy tensor-map creation), then tune_reps measured steps whose region times are min-
+// reduced (reading R19: clocks float on B200 so k = 3 reps instead of the paper's pinned clocks,
+// P:457).  Only the measured steps synchronise on their own end event.
+int Cell::tune_next() {
+  if (tune_mode != ASTRA_TUNE_ON) return tune_mode == ASTRA_TUNE_FROZEN ? ASTRA_TUNE_CONVERGED : ASTRA_TUNE_IDLE;
+  if (!wirer) tuner_setup();
+  if (wirer->converged()) return ASTRA_TUNE_CONVERGED;
+  if (rep_i == 0) {  // warm-up step done
+    rep_i = 1;
+    return ASTRA_TUNE_EXPLORING;
+  }
+  CUDA_TRY(cudaEventSynchronize(ev[R_STEP][1]));
+  tuner::Metrics m(tree->metrics.size(), 0.0);
+  for (size_t i = 0; i < tree->metrics.size(); ++i) {
+    const std::string& n = tree->metrics[i];
+    double v = 0;
+    if (n == "t_a1") v = elapsed(ev[R_A1][0], ev[R_A1][1]);
+    else if (n == "t_fwd") v = elapsed(ev[R_FWD][0], ev[R_FWD][1]);
+    else if (n == "t_bptt") v = elapsed(ev[R_BPTT][0], ev[R_BPTT][1]);
+    else if (n == "t_du") v = region_used[R_DU] ? elapsed(ev[R_DU][0], ev[R_DU][1]) : 0;
+    else if (n == "t_dw") v = region_used[R_DW] ? elapsed(ev[R_DW][0], ev[R_DW][1]) : 0;
+    else if (n == "t_dx") v = region_used[R_DX] ? elapsed(ev[R_DX][0], ev[R_DX][1]) : 0;
+    else if (n == "t_head") v = region_used[R_HEAD] ? elapsed(ev[R_HEAD][0], ev[R_HEAD][1]) : 0;
+    else if (n == "t_se4") v = elapsed(ev[R_SE4][0], ev[R_SE4][1]);
+    else v = elapsed(ev[R_STEP][0], ev[R_STEP][1]);
+    m[i] = v;
+  }
+  if (rep_i == 1) rep_min = m;
+  else
+    for (size_t i = 0; i < m.size(); ++i) rep_min[i] = std::min(rep_min[i], m[i]);
+  if (rep_i < tune_reps) {
+    ++rep_i;
+    return ASTRA_TUNE_EXPLORING;
+  }
+  wirer->feed(rep_min);
+  rep_i = 0;
+  tuner::Config c;
+  if (wirer->propose(c)) {
+    apply_config(c);
+    return ASTRA_TUNE_EXPLORING;
+  }
+  apply_config(wirer->final_config());
+  configs_seen.pop_back();
+  return ASTRA_TUNE_CONVERGED;
+}
+
+std::string Cell::report() {
+  std::ostringstream o;
+  o << "{\"variant\": \"" << var.str() << "\", \"mode\": " << tune_mode;
+  if (wirer) {
+    o << ", \"converged\": " << (wirer->converged() ? "true" : "false") << ", \"configs_explored\": "
+      << wirer->trials() << ", \"steps_per_config\": " << (1 + tune_reps) << ", \"index_entries\": "
+      << wirer->index().d.size() << ", \"tree_avs\": [";
+    for (size_t i = 0; i < tree->avs.size(); ++i) o << (i ? ", " : "") << "\"" << tree->avs[i] << "\"";
+    o << "], \"index\": {";
+    size_t k = 0;
+    for (auto& kv : wirer->index().d) o << (k++ ? ", " : "") << "\"" << kv.first << "\": " << kv.second;
+    o << "}";
+  }
+  o << "}";
+  return o.str();
+}
+
+std::unique_ptr<Cell> make_lstm_cell(const astra_cell_desc& d);
+std::unique_ptr<Cell> make_scrn_cell(const astra_cell_desc& d);
+std::unique_ptr<Cell> make_rhn_cell(const astra_cell_desc& d);
+
+std::unique_ptr<Cell> make_cell(const astra_cell_desc& d) {
+  switch (d.cell_type) {
+    case ASTRA_LSTM:
+    case ASTRA_MILSTM:
+    case ASTRA_SUBLSTM: return make_lstm_cell(d);
+    case ASTRA_SCRNN: return make_scrn_cell(d);
+    case ASTRA_RHN: return make_rhn_cell(d);
+    case ASTRA_LSTM_ATTN: throw Error(ASTRA_E_UNSUPPORTED, "cell: the LSTM-attention CUDA path is not built yet");
+    default: throw Error(ASTRA_E_ARG, "cell: unknown cell_type");
+  }
+}
+
+}  // namespace astra

@@ -1,0 +1,239 @@
+// LSTM-family cells: LSTM, MI-LSTM [36] and subLSTM [8]
+// on both precision paths.
+//
+// Step anatomy:
+//   fwd : mirrors(K9) → x copy → state init → a1 hoisted GEMM WX = X·W (K1) →
+//         for t: UH_t = h_{t-1}·U (K1) ; pointwise gate epilogue (K2 half)
+//   bwd : for t desc: dh_rec = D_uh[t+1]·Uᵀ (K1) ; pointwise cell backward (K4 half, K5 partials)
+//         → dh0 → wgrad dU = Hᵀ·D_uh, dW = Xᵀ·D_wx (K1) → dX = D_wx·Wᵀ (K1) → bias/α/β reductions (K5)
+//         → gradient sum over ranks (K11) when world > 1.
+#include "../kernels/cell_math.cuh"
+#include "cell.h"
+
+namespace astra {
+
+class LstmCell : public Cell {
+ public:
+  int kind, NG, nchunk;
+  size_t off_X, off_WX, off_UH, off_C, off_H, off_Wm, off_Um;
+  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part;
+
+  explicit LstmCell(const astra_cell_desc& dd) : Cell(dd) {
+    kind = d.cell_type == ASTRA_MILSTM ? K_MILSTM : d.cell_type == ASTRA_SUBLSTM ? K_SUBLSTM : K_LSTM;
+    Hp = (int)round_up(H, GATE_U);
+    NG = 4 * Hp;
+    add_param("W", I, 4 * H);
+    add_param("U", H, 4 * H);
+    add_param("b", 1, 4 * H);
+    if (kind == K_MILSTM) {
+      add_param("alpha", 1, 4 * H);
+      add_param("beta1", 1, 4 * H);
+      add_param("beta2", 1, 4 * H);
+    }
+    const size_t e = esz();
+    const size_t TB = (size_t)T * B;
+    Carve s;
+    off_X = s.take(TB * Ip * e);
+    off_WX = s.take(TB * NG * 4);
+    off_UH = s.take(TB * NG * 4);
+    off_C = s.take((TB + B) * Hp * 4);
+    off_H = s.take((TB + B) * Hp * e);
+    off_Wm = s.take((size_t)NG * Ip * e);
+    off_Um = s.take((size_t)NG * Hp * e);
+    saved_bytes = s.o;
+    nchunk = lstm_bwd_row_chunks(B);
+    Carve c;
+    off_Duh = c.take(TB * NG * e);
+    off_Dwx = kind == K_MILSTM ? c.take(TB * NG * e) : off_Duh;
+    off_dH = c.take((size_t)B * Hp * 4);
+    off_dC = c.take((size_t)B * Hp * 4);
+    off_part = c.take((size_t)nchunk * 4 * NG * 4);
+    scratch_bytes = c.o;
+  }
+
+  void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
+  void* x_operand() override { return sv<char>(off_X); }
+  Mat2 y_operand() override { return mat(Hrow(1), Hp, (long)T * B, Hp); }
+  int y_width() const override { return Hp; }
+  std::vector<KSeg> y_segments() const override { return {{0, 0, H}}; }
+  void role_shape(int role, int& M, int& N) const override {
+    const int TB = T * B;
+    switch (role) {
+      case G_A1: M = TB; N = NG; break;
+      case G_REC: M = B; N = NG; break;
+      case G_BPTT: M = B; N = Hp; break;
+      case G_DU: M = Hp; N = NG; break;
+      case G_DW: M = I; N = NG; break;
+      case G_DX: M = TB; N = I; break;
+      default: M = lm_mode ? TB : 0; N = lm_V; break;
+    }
+  }
+  void forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT) override;
+  void backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0) override;
+};
+
+void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT) {
+  ASTRA_CHECK_STATE(bound, "step_fwd: call astra_bind first");
+  ASTRA_CHECK_ARG(lm_mode || x, "step_fwd: x is null");
+  cudaStream_t st = main_st;
+  const long TB = (long)T * B;
+  const size_t e = esz();
+  void* X = sv<char>(off_X);
+  void* Wm = sv<char>(off_Wm);
+  void* Um = sv<char>(off_Um);
+  float* WX = sv<float>(off_WX);
+  float* UH = sv<float>(off_UH);
+  float* Cb = sv<float>(off_C);
+
+  mark(R_STEP, 0, st);
+  // K9 second half: operand mirrors in the internal gate-interleaved layout
+  mirror_gates_T(ot, p("W"), I, H, Hp, Wm, Ip, st);
+  mirror_gates_T(ot, p("U"), H, H, Hp, Um, Hp, st);
+  if (!lm_mode) copy_pad(ot, x, ot, TB, I, I, X, Ip, st);
+  copy_pad(ot, h0, OT::F32, B, H, H, Hrow(0), Hp, st);
+  copy_f32_pad(c0, B, H, H, Cb, Hp, H, st);
+
+  GateParams gp;
+  gp.b = p("b");
+  if (kind == K_MILSTM) { gp.alpha = p("alpha"); gp.beta1 = p("beta1"); gp.beta2 = p("beta2"); }
+
+  // a1: hoisted input projection for all timesteps
+  mark(R_A1, 0, st);
+  GemmSpec a1;
+  a1.A = mat(X, I, TB, Ip);
+  a1.B = mat(Wm, I, NG, Ip);
+  a1.M = (int)TB; a1.N = NG; a1.K = I;
+  run_gemm(0, a1, epi(WX, NG, (int)TB, NG), 0, 0, var.g[G_A1], st);
+  mark(R_A1, 1, st);
+
+  // a3: recurrent chain
+  mark(R_FWD, 0, st);
+  GemmSpec rec;
+  rec.A = mat(Hrow(0), Hp, B, Hp, T + 1, (long)B * Hp);
+  rec.B = mat(Um, Hp, NG, Hp);
+  rec.M = B; rec.N = NG; rec.K = Hp;
+  for (int t = 0; t < T; ++t) {
+    float* UHt = UH + (long)t * B * NG;
+    run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st);
+    const bool last = t == T - 1;
+    void* yt = y ? (char*)y + (size_t)t * B * H * e : nullptr;
+    lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
+                       Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), yt, H, ot, last ? hT : nullptr,
+                       last ? cT : nullptr, st);
+  }
+  mark(R_FWD, 1, st);
+  fwd_done = true;
+}
+
+void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0) {
+  ASTRA_CHECK_STATE(bound && fwd_done, "step_bwd: needs a preceding step_fwd");
+  ASTRA_CHECK_ARG(lm_mode || dy, "step_bwd: dy is null");
+  cudaStream_t st = main_st;
+  const long TB = (long)T * B;
+  const size_t e = esz();
+  void* X = sv<char>(off_X);
+  void* Wm = sv<char>(off_Wm);
+  void* Um = sv<char>(off_Um);
+  float* WX = sv<float>(off_WX);
+  float* UH = sv<float>(off_UH);
+  float* Cb = sv<float>(off_C);
+  char* Duh = sc<char>(off_Duh);
+  char* Dwx = sc<char>(off_Dwx);
+  float* dH = sc<float>(off_dH);
+  float* dC = sc<float>(off_dC);
+  float* part = sc<float>(off_part);
+  const int nq = kind == K_MILSTM ? 4 : 1;
+
+  GateParams gp;
+  gp.b = p("b");
+  if (kind == K_MILSTM) { gp.alpha = p("alpha"); gp.beta1 = p("beta1"); gp.beta2 = p("beta2"); }
+
+  copy_f32_pad(dcT, B, H, H, dC, Hp, H, st);
+
+  // a5: BPTT chain
+  mark(R_BPTT, 0, st);
+  GemmSpec bp;
+  bp.A = mat(Duh, NG, B, NG, T, (long)B * NG);
+  bp.B = mat(Um, Hp, NG, Hp);
+  bp.b_mn = true;
+  bp.M = B; bp.N = Hp; bp.K = NG;
+  for (int t = T - 1; t >= 0; --t) {
+    const float* dh_rec;
+    long ld_dh;
+    if (t == T - 1) {
+      dh_rec = dhT;
+      ld_dh = H;
+    } else {
+      run_gemm(2, bp, epi(dH, Hp, B, Hp), t + 1, 0, var.g[G_BPTT], st);
+      dh_rec = dH;
+      ld_dh = Hp;
+    }
+    const void* dyt;
+    long ldy;
+    bool dyf32;
+    if (lm_mode) { dyt = lm_dy + (long)t * B * Hp; ldy = Hp; dyf32 = true; }
+    else { dyt = (const char*)dy + (size_t)t * B * H * e; ldy = H; dyf32 = false; }
+    lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, dC, WX + (long)t * B * NG,
+                       UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
+                       Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
+  }
+  if (dh0) run_gemm(2, bp, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
+  if (dc0) copy_pad(OT::F32, dC, OT::F32, B, H, Hp, dc0, H, st);
+  mark(R_BPTT, 1, st);
+
+  // a6: weight gradients and input dgrad
+  mark(R_SE4, 0, st);
+  cudaStream_t st_u = st;
+  if (var.wg_side && !side.empty()) {
+    CUDA_TRY(cudaEventRecord(ev_fork, st));
+    CUDA_TRY(cudaStreamWaitEvent(side[0], ev_fork, 0));
+    st_u = side[0];
+  }
+  GemmSpec gu;
+  gu.A = mat(Hrow(0), Hp, TB, Hp);
+  gu.a_mn = true;
+  gu.B = mat(Duh, NG, TB, NG);
+  gu.b_mn = true;
+  gu.M = Hp; gu.N = NG; gu.K = (int)TB;
+  if (st_u == st) mark(R_DU, 0, st);
+  run_gemm(4, gu, epi_perm(g("U"), 4L * H, H, NG, GATE_U, 0, H), 0, 0, var.g[G_DU], st_u);
+  if (st_u == st) mark(R_DU, 1, st);
+
+  GemmSpec gw;
+  gw.A = mat(X, I, TB, Ip);
+  gw.a_mn = true;
+  gw.B = mat(Dwx, NG, TB, NG);
+  gw.b_mn = true;
+  gw.M = I; gw.N = NG; gw.K = (int)TB;
+  mark(R_DW, 0, st);
+  run_gemm(5, gw, epi_perm(g("W"), 4L * H, I, NG, GATE_U, 0, H), 0, 0, var.g[G_DW], st);
+  mark(R_DW, 1, st);
+
+  if (dx) {
+    GemmSpec gx;
+    gx.A = mat(Dwx, NG, TB, NG);
+    gx.B = mat(Wm, I, NG, Ip);
+    gx.b_mn = true;
+    gx.M = (int)TB; gx.N = I; gx.K = NG;
+    mark(R_DX, 0, st);
+    if (lm_mode)
+      run_gemm(6, gx, epi(dx, Ip, (int)TB, I), 0, 0, var.g[G_DX], st);
+    else
+      run_gemm(6, gx, epi(dx, I, (int)TB, I, ot == OT::BF16), 0, 0, var.g[G_DX], st);
+    mark(R_DX, 1, st);
+  }
+  float* gq[4] = {g("b"), nullptr, nullptr, nullptr};
+  if (kind == K_MILSTM) { gq[1] = g("alpha"); gq[2] = g("beta1"); gq[3] = g("beta2"); }
+  reduce_gate_partials(part, nchunk, nq, H, Hp, gq, st);
+  if (st_u != st) {
+    CUDA_TRY(cudaEventRecord(ev_join, st_u));
+    CUDA_TRY(cudaStreamWaitEvent(st, ev_join, 0));
+  }
+  mark(R_SE4, 1, st);
+  if (world > 1 && !lm_mode) allreduce_grads(G, n_params, st);
+  if (!lm_mode) mark(R_STEP, 1, st);
+}
+
+std::unique_ptr<Cell> make_lstm_cell(const astra_cell_desc& d) { return std::unique_ptr<Cell>(new LstmCell(d)); }
+
+}  // namespace astra

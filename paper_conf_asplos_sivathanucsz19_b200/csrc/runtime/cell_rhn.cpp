@@ -1,0 +1,190 @@
+// Recurrent highway network [39] with coupled carry (BASELINE configs[2]),
+// both precision paths.  Reading R9: input only at micro-layer ℓ = 1, output s^L.
+//
+//   s^0_t = s^L_{t−1};  for ℓ = 1..L:  a = [ℓ=1]·x_t·W + s^{ℓ−1}·R_ℓ + b_ℓ;  h = tanh a_H, τ = σ(a_T);
+//                                      s^ℓ = h⊙τ + s^{ℓ−1}⊙(1 − τ)
+//
+// Plan: a1 WX = X·W (K1) hoisted; the chain is T·L dependent micro-steps, each = one K1 GEMM
+// (s·R_ℓ, N = 2H) + one pointwise kernel (a3); BPTT mirrors it with ds = ds(1−τ) + da·R_ℓᵀ
+// (pointwise writes ds(1−τ), the GEMM accumulates da·R_ℓᵀ onto it); dR_ℓ = S_ℓᵀ·DA_ℓ per micro-layer.
+// Internal gate layout: gate-blocked and padded, column g·Hp + j.
+#include "cell.h"
+
+namespace astra {
+
+class RhnCell : public Cell {
+ public:
+  int L, G2, nchunk;
+  size_t off_X, off_WX, off_Apre, off_Sf, off_Sop, off_MW, off_MR;
+  size_t off_DA, off_dS, off_part;
+
+  explicit RhnCell(const astra_cell_desc& dd) : Cell(dd) {
+    L = d.depth;
+    ASTRA_CHECK_ARG(L >= 1 && L <= 64, "rhn: depth must be in 1..64");
+    G2 = 2 * Hp;
+    add_param("W", I, 2 * H);
+    add_param("R", L * H, 2 * H);
+    add_param("b", L, 2 * H);
+    const size_t e = esz();
+    const size_t TB = (size_t)T * B;
+    Carve s;
+    off_X = s.take(TB * Ip * e);
+    off_WX = s.take(TB * G2 * 4);
+    off_Apre = s.take((size_t)L * TB * G2 * 4);
+    off_Sf = s.take((size_t)L * (TB + B) * Hp * 4);
+    off_Sop = s.take((size_t)L * (TB + B) * Hp * e);
+    off_MW = s.take((size_t)G2 * Ip * e);
+    off_MR = s.take((size_t)L * G2 * Hp * e);
+    saved_bytes = s.o;
+    nchunk = pw_row_chunks(B);
+    Carve c;
+    off_DA = c.take((size_t)L * TB * G2 * e);
+    off_dS = c.take((size_t)B * Hp * 4);
+    off_part = c.take((size_t)L * nchunk * G2 * 4);
+    scratch_bytes = c.o;
+  }
+
+  // state slot (ℓ, t): input of micro-step ℓ at time t; slot (0, t+1) = output of time t
+  size_t slot(int l, int t) const { return ((size_t)l * (T + 1) + t) * B * Hp; }
+  float* Sf(int l, int t) { return sv<float>(off_Sf) + slot(l, t); }
+  char* Sop(int l, int t) { return saved + off_Sop + slot(l, t) * esz(); }
+  float* Apre(int l, int t) { return sv<float>(off_Apre) + ((size_t)l * T + t) * B * G2; }
+  char* DA(int l, int t) { return scratch + off_DA + ((size_t)l * T + t) * B * G2 * esz(); }
+
+  void* x_operand() override { return sv<char>(off_X); }
+  Mat2 y_operand() override { return mat(Sop(0, 1), Hp, (long)T * B, Hp); }
+  int y_width() const override { return Hp; }
+  std::vector<KSeg> y_segments() const override { return {{0, 0, H}}; }
+  int c_width() const override { return 0; }
+  void role_shape(int role, int& M, int& N) const override {
+    const int TB = T * B;
+    switch (role) {
+      case G_A1: M = TB; N = G2; break;
+      case G_REC: M = B; N = G2; break;
+      case G_BPTT: M = B; N = Hp; break;
+      case G_DU: M = Hp; N = G2; break;
+      case G_DW: M = I; N = G2; break;
+      case G_DX: M = TB; N = I; break;
+      default: M = lm_mode ? TB : 0; N = lm_V; break;
+    }
+  }
+
+  void forward(const void* x, const float* s0, const float*, void* y, float* sT, float*) override {
+    ASTRA_CHECK_STATE(bound, "step_fwd: call astra_bind first");
+    ASTRA_CHECK_ARG(lm_mode || x, "step_fwd: x is null");
+    cudaStream_t st = main_st;
+    const long TB = (long)T * B;
+    const size_t e = esz();
+    void* X = sv<char>(off_X);
+    float* WX = sv<float>(off_WX);
+    char* MW = sv<char>(off_MW);
+    char* MR = sv<char>(off_MR);
+
+    mark(R_STEP, 0, st);
+    mirror_blocked_T(ot, p("W"), I, 2, H, Hp, MW, Ip, st);
+    for (int l = 0; l < L; ++l)
+      mirror_blocked_T(ot, p("R") + (size_t)l * H * 2 * H, H, 2, H, Hp, MR + (size_t)l * G2 * Hp * e, Hp, st);
+    if (!lm_mode) copy_pad(ot, x, ot, TB, I, I, X, Ip, st);
+    copy_pad(OT::F32, s0, OT::F32, B, H, H, Sf(0, 0), Hp, st);
+    copy_pad(ot, s0, OT::F32, B, H, H, Sop(0, 0), Hp, st);
+
+    mark(R_A1, 0, st);
+    GemmSpec a1;
+    a1.A = mat(X, I, TB, Ip);
+    a1.B = mat(MW, I, G2, Ip);
+    a1.M = (int)TB; a1.N = G2; a1.K = I;
+    run_gemm(0, a1, epi(WX, G2, (int)TB, G2), 0, 0, var.g[G_A1], st);
+    mark(R_A1, 1, st);
+
+    mark(R_FWD, 0, st);
+    GemmSpec rec;
+    rec.A = mat(Sop(0, 0), Hp, B, Hp, (long)L * (T + 1), (long)B * Hp);
+    rec.B = mat(MR, Hp, G2, Hp, L, (long)G2 * Hp);
+    rec.M = B; rec.N = G2; rec.K = Hp;
+    for (int t = 0; t < T; ++t) {
+      for (int l = 0; l < L; ++l) {
+        float* Z = Apre(l, t);
+        run_gemm(1, rec, epi(Z, G2, B, G2), l * (T + 1) + t, l, var.g[G_REC], st);
+        const bool last = l == L - 1;
+        float* sn = last ? Sf(0, t + 1) : Sf(l + 1, t);
+        char* sno = last ? Sop(0, t + 1) : Sop(l + 1, t);
+        rhn_fwd_pw(ot, B, H, Hp, Z, l == 0 ? WX + (long)t * B * G2 : nullptr, p("b") + (size_t)l * 2 * H, Sf(l, t),
+                   sn, sno, (last && y) ? (char*)y + (size_t)t * B * H * e : nullptr, H,
+                   (last && t == T - 1) ? sT : nullptr, st);
+      }
+    }
+    mark(R_FWD, 1, st);
+    fwd_done = true;
+  }
+
+  void backward(const void* dy, const float* dsT, const float*, void* dx, float* ds0, float*) override {
+    ASTRA_CHECK_STATE(bound && fwd_done, "step_bwd: needs a preceding step_fwd");
+    ASTRA_CHECK_ARG(lm_mode || dy, "step_bwd: dy is null");
+    cudaStream_t st = main_st;
+    const long TB = (long)T * B;
+    const size_t e = esz();
+    void* X = sv<char>(off_X);
+    char* MW = sv<char>(off_MW);
+    char* MR = sv<char>(off_MR);
+    float* dS = sc<float>(off_dS);
+    float* part = sc<float>(off_part);
+    const long ldy = lm_mode ? Hp : H;
+
+    copy_pad(OT::F32, dsT, OT::F32, B, H, H, dS, Hp, st);
+    mark(R_BPTT, 0, st);
+    GemmSpec bp;
+    bp.A = mat(scratch + off_DA, G2, B, G2, (long)L * T, (long)B * G2);
+    bp.B = mat(MR, Hp, G2, Hp, L, (long)G2 * Hp);
+    bp.b_mn = true;
+    bp.M = B; bp.N = Hp; bp.K = G2;
+    for (int t = T - 1; t >= 0; --t) {
+      for (int l = L - 1; l >= 0; --l) {
+        const void* dyt = nullptr;
+        if (l == L - 1)
+          dyt = lm_mode ? (const void*)(lm_dy + (long)t * B * Hp) : (const char*)dy + (size_t)t * B * H * e;
+        rhn_bwd_pw(ot, B, H, Hp, dS, dyt, ldy, lm_mode, Apre(l, t), Sf(l, t), DA(l, t), dS,
+                   part + (size_t)l * nchunk * G2, t == T - 1, st);
+        run_gemm(2, bp, accum(epi(dS, Hp, B, Hp)), l * T + t, l, var.g[G_BPTT], st);
+      }
+    }
+    if (ds0) copy_pad(OT::F32, dS, OT::F32, B, H, Hp, ds0, H, st);
+    mark(R_BPTT, 1, st);
+
+    mark(R_SE4, 0, st);
+    mark(R_DU, 0, st);
+    for (int l = 0; l < L; ++l) {
+      GemmSpec gr;
+      gr.A = mat(Sop(l, 0), Hp, TB, Hp); gr.a_mn = true;
+      gr.B = mat(DA(l, 0), G2, TB, G2); gr.b_mn = true;
+      gr.M = Hp; gr.N = G2; gr.K = (int)TB;
+      run_gemm(20 + l, gr, epi_perm(g("R") + (size_t)l * H * 2 * H, 2L * H, H, G2, 0, Hp, H), 0, 0, var.g[G_DU], st);
+    }
+    mark(R_DU, 1, st);
+    mark(R_DW, 0, st);
+    GemmSpec gw;
+    gw.A = mat(X, I, TB, Ip); gw.a_mn = true;
+    gw.B = mat(DA(0, 0), G2, TB, G2); gw.b_mn = true;
+    gw.M = I; gw.N = G2; gw.K = (int)TB;
+    run_gemm(3, gw, epi_perm(g("W"), 2L * H, I, G2, 0, Hp, H), 0, 0, var.g[G_DW], st);
+    mark(R_DW, 1, st);
+    for (int l = 0; l < L; ++l)
+      reduce_blocked_partials(part + (size_t)l * nchunk * G2, nchunk, 2, H, Hp, g("b") + (size_t)l * 2 * H, st);
+    if (dx) {
+      GemmSpec gx;
+      gx.A = mat(DA(0, 0), G2, TB, G2);
+      gx.B = mat(MW, I, G2, Ip); gx.b_mn = true;
+      gx.M = (int)TB; gx.N = I; gx.K = G2;
+      mark(R_DX, 0, st);
+      if (lm_mode) run_gemm(4, gx, epi(dx, Ip, (int)TB, I), 0, 0, var.g[G_DX], st);
+      else run_gemm(4, gx, epi(dx, I, (int)TB, I, ot == OT::BF16), 0, 0, var.g[G_DX], st);
+      mark(R_DX, 1, st);
+    }
+    mark(R_SE4, 1, st);
+    if (world > 1 && !lm_mode) allreduce_grads(G, n_params, st);
+    if (!lm_mode) mark(R_STEP, 1, st);
+  }
+};
+
+std::unique_ptr<Cell> make_rhn_cell(const astra_cell_desc& d) { return std::unique_ptr<Cell>(new RhnCell(d)); }
+
+}  // namespace astra

@@ -1,0 +1,140 @@
+// Language-model wrapper (SURVEY §8(a) rows a0, a4, a6 embedding part, a7, a8): embedding gather →
+// cell forward → head GEMM + mean cross-entropy → head backward → cell BPTT → embedding backward →
+// gradient sum over ranks → SGD.  Works for every cell family through the Cell hooks
+// (x_operand / y_operand / y_segments).
+#include "cell.h"
+
+namespace astra {
+
+LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
+  ASTRA_CHECK_ARG(vocab > 1, "lm: vocab must be > 1");
+  Vp = (int)round_up(V, 8);
+  Yw = c->y_width();
+  c->lm_V = V;
+  params = c->params;
+  n_cell = c->n_params;
+  n_params = n_cell;
+  auto add = [&](const char* n, int r, int cc) {
+    params.push_back({n, n_params, r, cc});
+    n_params = (n_params + (size_t)r * cc + 63) / 64 * 64;
+  };
+  add("E", V, c->I);
+  add("W_o", c->Hout, V);
+  add("b_o", 1, V);
+  const long TB = (long)c->T * c->B;
+  const size_t e = c->esz();
+  Carve w;
+  off_cellsaved = w.take(c->saved_bytes);
+  off_cellscratch = w.take(c->scratch_bytes);
+  off_logits = w.take((size_t)TB * V * 4);
+  off_dlog = w.take((size_t)TB * Vp * e);
+  off_dlog32 = w.take((size_t)TB * V * 4);
+  off_rowloss = w.take((size_t)TB * 4);
+  off_dY = w.take((size_t)TB * Yw * 4);
+  off_Wo = w.take((size_t)round_up(V, 256) * Yw * e);
+  off_colsum = w.take(colsum_scratch_floats(TB, V) * 4);
+  sort_bytes = embed_bwd_scratch_bytes(TB, V);
+  off_sort = w.take(sort_bytes);
+  off_embpart = w.take(embed_bwd_partial_floats(TB, V, c->I) * 4);
+  off_h = w.take((size_t)c->B * c->H * 4);
+  off_c = w.take((size_t)c->B * (c->c_width() > 0 ? c->c_width() : 1) * 4);
+  off_loss = w.take(256);
+  off_dx = w.take((size_t)TB * c->Ip * 4);
+  ws_bytes = w.o;
+}
+
+size_t LM::find(const std::string& n) const {
+  for (auto& p : params)
+    if (p.name == n) return p.offset;
+  throw Error(ASTRA_E_ARG, "no parameter " + n);
+}
+
+void LM::bind(float* pp, float* gg, void* wsp) {
+  ASTRA_CHECK_ARG(pp && gg && wsp, "lm_bind: null pointer");
+  P = pp; G = gg; ws = (char*)wsp;
+  cell->lm_mode = true;
+  cell->bind(pp, gg, ws + off_cellsaved, ws + off_cellscratch);
+  set_state(nullptr, nullptr);
+  bound = true;
+}
+
+void LM::set_state(const float* h, const float* c) {
+  cudaStream_t st = cell->main_st;
+  const size_t nh = (size_t)cell->B * cell->H * 4, nc = (size_t)cell->B * cell->c_width() * 4;
+  if (h) CUDA_TRY(cudaMemcpyAsync(ws + off_h, h, nh, cudaMemcpyDeviceToDevice, st));
+  else CUDA_TRY(cudaMemsetAsync(ws + off_h, 0, nh, st));
+  if (nc) {
+    if (c) CUDA_TRY(cudaMemcpyAsync(ws + off_c, c, nc, cudaMemcpyDeviceToDevice, st));
+    else CUDA_TRY(cudaMemsetAsync(ws + off_c, 0, nc, st));
+  }
+}
+
+void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
+  ASTRA_CHECK_STATE(bound, "lm_train_step: not bound");
+  ASTRA_CHECK_ARG(tokens, "lm_train_step: tokens is null");
+  Cell& c = *cell;
+  cudaStream_t st = c.main_st;
+  const long TB = (long)c.T * c.B;
+  const size_t e = c.esz();
+  float* hs = (float*)(ws + off_h);
+  float* cs = c.c_width() > 0 ? (float*)(ws + off_c) : nullptr;
+  float* logits = (float*)(ws + off_logits);
+  void* dlog = ws + off_dlog;
+  float* dlog32 = (float*)(ws + off_dlog32);
+  float* rowloss = (float*)(ws + off_rowloss);
+  float* dY = (float*)(ws + off_dY);
+  char* Wom = ws + off_Wo;
+  float* dX = (float*)(ws + off_dx);
+  float* lossp = loss_dev ? loss_dev : (float*)(ws + off_loss);
+  const int Vr = (int)round_up(V, 256);
+  const std::vector<KSeg> segs = c.y_segments();
+
+  // a0: embedding gather into the cell's operand buffer
+  embed_gather(c.ot, tokens, TB, P + find("E"), c.I, c.x_operand(), c.Ip, st);
+  // cell forward (SE1); final state carried for the next step (truncated BPTT)
+  c.forward(nullptr, hs, cs, nullptr, hs, cs);
+
+  // a4: head forward + CE + head backward (SE2).  The head reads the cell's output operand
+  // (SCRN: [h | s], a K-concatenated "ladder" [h|s]·[U;V]).
+  c.mark(R_HEAD, 0, st);
+  CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, st));
+  for (const KSeg& s : segs)
+    mirror_T(c.ot, P + find("W_o") + (size_t)s.r0 * V, s.n, V, Vr, s.n, Wom + (size_t)s.k0 * e, Yw, st);
+  const Mat2 Y = c.y_operand();
+  GemmSpec hd;
+  hd.A = Y;
+  hd.B = mat(Wom, Yw, V, Yw);
+  hd.M = (int)TB; hd.N = V; hd.K = Yw;
+  c.run_gemm(100, hd, epi(logits, V, (int)TB, V, 0, P + find("b_o")), 0, 0, c.var.g[G_HEAD], st);
+  ce_fwd_bwd(c.ot, logits, V, V, tokens + c.B, TB, 1.0f / (float)TB, rowloss, dlog, Vp, dlog32, st);
+  sum_rows_to_scalar(rowloss, TB, 1.0f / (float)TB, lossp, st);
+  GemmSpec dy;
+  dy.A = mat(dlog, V, TB, Vp);
+  dy.B = mat(Wom, Yw, V, Yw);
+  dy.b_mn = true;
+  dy.M = (int)TB; dy.N = Yw; dy.K = V;
+  c.run_gemm(101, dy, epi(dY, Yw, (int)TB, Yw), 0, 0, c.var.g[G_HEAD], st);
+  int id = 102;
+  for (const KSeg& s : segs) {
+    GemmSpec dwo;
+    dwo.A = mat((const char*)Y.ptr + (size_t)s.k0 * e, s.n, TB, Y.ld);
+    dwo.a_mn = true;
+    dwo.B = mat(dlog, V, TB, Vp);
+    dwo.b_mn = true;
+    dwo.M = s.n; dwo.N = V; dwo.K = (int)TB;
+    c.run_gemm(id++, dwo, epi(G + find("W_o") + (size_t)s.r0 * V, V, s.n, V), 0, 0, c.var.g[G_HEAD], st);
+  }
+  colsum(dlog32, TB, V, V, (float*)(ws + off_colsum), G + find("b_o"), st);
+  c.mark(R_HEAD, 1, st);
+
+  // cell backward (SE3 + SE4) and the embedding backward
+  c.lm_dy = dY;
+  c.backward(nullptr, nullptr, nullptr, dX, nullptr, nullptr);
+  embed_bwd(tokens, TB, V, dX, c.Ip, c.I, G + find("E"), ws + off_sort, sort_bytes, (float*)(ws + off_embpart), st);
+  // a7: data-parallel gradient sum (mean over ranks), then a8: SGD
+  if (c.world > 1) c.allreduce_grads(G, n_params, st);
+  if (do_sgd) sgd(P, G, n_params, lr, st);
+  c.mark(R_STEP, 1, st);
+}
+
+}  // namespace astra

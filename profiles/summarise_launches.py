@@ -17,7 +17,7 @@ def summarise(path):
             v = float(r[vi].replace(",", ""))
         except ValueError:
             continue
-        name = r[ki].split("(")[0].replace("void ", "")[:70]
+        name = (r[ki].split("(")[0].replace("void ", "").replace("astra::", "")[:52] + " g" + r[gi].replace(" ", ""))[:70]
         agg[name][0] += 1
         agg[name][1] += v
         agg[name][2] = r[gi]

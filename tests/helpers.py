@@ -36,50 +36,64 @@ def cell_shapes(cell, I, H, S=None, L=None):
     raise ValueError(cell)
 
 
-def make_cell_case(cell, T, B, I, H, seed, bf16=False, ab_range=(0.5, 1.5)):
-    """Seeded parameters and inputs; for the bf16 path weights and inputs are
-    pre-rounded to bf16 so both sides see identical operands."""
-    p = synth.weights(seed, cell_shapes(cell, I, H), H,
+GEMM_WEIGHTS = ("W", "U", "A", "Bm", "P", "R")
+
+
+def make_cell_case(cell, T, B, I, H, seed, bf16=False, ab_range=(0.5, 1.5), S=None, L=None):
+    """Seeded parameters and inputs; for the bf16 path the GEMM weights and the
+    inputs are pre-rounded to bf16 so both sides see identical operands."""
+    S = S or H
+    p = synth.weights(seed, cell_shapes(cell, I, H, S, L), H,
                       {"alpha": ab_range, "beta1": ab_range, "beta2": ab_range})
     x = synth.uniform(seed, "x", (T, B, I), -1, 1)
     if bf16:
         x = bf16_round(x)
-        for k in ("W", "U"):
-            p[k] = bf16_round(p[k])
-    inp = {"x": x, "h0": synth.uniform(seed, "h0", (B, H), -0.5, 0.5),
-           "c0": synth.uniform(seed, "c0", (B, H), -0.5, 0.5)}
-    dY = synth.normal(seed, "dY", (T, B, H))
+        for k in GEMM_WEIGHTS:
+            if k in p:
+                p[k] = bf16_round(p[k])
+    inp = {"x": x, "h0": synth.uniform(seed, "h0", (B, H), -0.5, 0.5)}
+    C = S if cell == "scrn" else H
+    Hout = H + S if cell == "scrn" else H
+    if cell != "rhn":
+        inp["c0"] = synth.uniform(seed, "c0", (B, C), -0.5, 0.5)
+    dY = synth.normal(seed, "dY", (T, B, Hout))
     if bf16:
         dY = bf16_round(dY)
     dhT = synth.normal(seed, "dhT", (B, H))
-    dcT = synth.normal(seed, "dcT", (B, H))
+    dcT = synth.normal(seed, "dcT", (B, C)) if cell != "rhn" else None
     return p, inp, dY, dhT, dcT
 
 
-def run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, variant=None):
+def run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, variant=None, **kw):
     """Run fwd + bwd through the C ABI; returns (outputs, grads) as numpy fp64 dicts."""
     import torch
     import paper_conf_asplos_sivathanucsz19_b200 as A
     T, B, I = inp["x"].shape
     H = inp["h0"].shape[1]
-    c = A.Cell(cell, H, I, B, T, dtype=dtype)
+    Hout = dY.shape[2]
+    c = A.Cell(cell, H, I, B, T, dtype=dtype, **kw)
     if variant is not None:
         c.tune_mode(A.TUNE_FROZEN, variant)
     c.load(p)
     dev = c.device
     tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
-    f32 = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    f32 = lambda a: None if a is None else torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
     x = f32(inp["x"]).to(tdt).contiguous()
-    y = torch.empty(T, B, H, dtype=tdt, device=dev)
+    y = torch.empty(T, B, Hout, dtype=tdt, device=dev)
     hT = torch.empty(B, H, device=dev)
-    cT = torch.empty(B, H, device=dev)
-    c.forward(x, f32(inp["h0"]), f32(inp["c0"]), y, hT, cT)
+    has_c = "c0" in inp
+    C = inp["c0"].shape[1] if has_c else 1
+    cT = torch.empty(B, C, device=dev) if has_c else None
+    c.forward(x, f32(inp["h0"]), f32(inp.get("c0")), y, hT, cT)
     dx = torch.empty(T, B, I, dtype=tdt, device=dev)
     dh0 = torch.empty(B, H, device=dev)
-    dc0 = torch.empty(B, H, device=dev)
+    dc0 = torch.empty(B, C, device=dev) if has_c else None
     c.backward(f32(dY).to(tdt).contiguous(), f32(dhT), f32(dcT), dx, dh0, dc0)
     torch.cuda.synchronize()
-    out = {"y": y.float().cpu().numpy(), "hT": hT.cpu().numpy(), "cT": cT.cpu().numpy()}
+    out = {"y": y.float().cpu().numpy(), "hT": hT.cpu().numpy()}
     g = {k: c.view(k, c.grads).cpu().numpy().reshape(np.shape(p[k])) for k in p}
-    g.update(dx=dx.float().cpu().numpy(), dh0=dh0.cpu().numpy(), dc0=dc0.cpu().numpy())
+    g.update(dx=dx.float().cpu().numpy(), dh0=dh0.cpu().numpy())
+    if has_c:
+        out["cT"] = cT.cpu().numpy()
+        g["dc0"] = dc0.cpu().numpy()
     return out, g, c

@@ -41,19 +41,25 @@ def test_library_is_sm100a():
     assert "UTCHMMA" in out and "UTMALDG" in out and "LDTM" in out
 
 
-@pytest.mark.parametrize("cell,shapes", [
-    ("milstm", C.milstm_param_shapes(32, 64)),
-    ("lstm", C.lstm_param_shapes(32, 64)),
-    ("sublstm", C.lstm_param_shapes(32, 64)),
+@pytest.mark.parametrize("cell,shapes,kw", [
+    ("milstm", C.milstm_param_shapes(32, 64), {}),
+    ("lstm", C.lstm_param_shapes(32, 64), {}),
+    ("sublstm", C.lstm_param_shapes(32, 64), {}),
+    ("scrn", C.scrn_param_shapes(32, 64, 40), {"context": 40}),
+    ("rhn", C.rhn_param_shapes(32, 64, 3), {"depth": 3}),
 ])
-def test_param_layout_matches_oracle(cell, shapes):
-    c = A.Cell(cell, 64, 32, 4, 8, dtype="fp32", allocate=False)
+def test_param_layout_matches_oracle(cell, shapes, kw):
+    import numpy as np
+    c = A.Cell(cell, 64, 32, 4, 8, dtype="fp32", allocate=False, **kw)
     assert set(c.param_info) == set(shapes)
     prev_end = 0
     for name, (off, r, cc) in sorted(c.param_info.items(), key=lambda kv: kv[1][0]):
         shp = shapes[name]
-        assert r * cc == int(__import__("numpy").prod(shp))
-        assert (r, cc) == ((shp[0], shp[1]) if len(shp) == 2 else (1, shp[0]))
+        assert r * cc == int(np.prod(shp))
+        if len(shp) == 3:   # RHN R[ℓ] stacked: [L·H][2H]
+            assert (r, cc) == (shp[0] * shp[1], shp[2])
+        else:
+            assert (r, cc) == ((shp[0], shp[1]) if len(shp) == 2 else (1, shp[0]))
         assert off % 64 == 0 and off >= prev_end
         prev_end = off + r * cc
     assert c.n_params >= prev_end

@@ -13,10 +13,19 @@ from helpers import TOL_BF16, TOL_FP32, make_cell_case, rel_err, run_gpu_cell
 pytestmark = pytest.mark.gpu
 
 
-def _check(cell, T, B, I, H, dtype, seed, tol, variant=None):
-    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, seed, bf16=(dtype == "bf16"))
-    out_o, g_o = C.cell_fwd_bwd(cell, p, inp, dY, dhT, dcT)
-    out_g, g_g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, variant)
+ALPHA = 0.95
+
+
+def _check(cell, T, B, I, H, dtype, seed, tol, variant=None, S=None, L=None):
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, seed, bf16=(dtype == "bf16"), S=S, L=L)
+    kw, okw = {}, {}
+    if cell == "scrn":
+        kw = {"context": S or H, "scrn_alpha": ALPHA}
+        okw = {"alpha": np.float32(ALPHA).item()}
+    if cell == "rhn":
+        kw = {"depth": L}
+    out_o, g_o = C.cell_fwd_bwd(cell, p, inp, dY, dhT, dcT, **okw)
+    out_g, g_g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, variant, **kw)
     errs = {}
     for k in out_o:
         errs[k] = rel_err(out_g[k], out_o[k])
@@ -72,3 +81,35 @@ def test_variants_bitwise():
             continue
         for k in ref:
             assert np.array_equal(ref[k], cur[k]), (v, k)
+
+
+# ------------------------------------------------------------------ SCRN [22] and RHN [39]
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_scrn_small(dtype, tol):
+    _check("scrn", 6, 4, 32, 64, dtype, synth.config_seed(2) + 1, tol, S=40)
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_scrn_ragged_multi_tile(dtype, tol):
+    _check("scrn", 5, 130, 72, 100, dtype, synth.config_seed(2) + 2, tol, S=70)
+
+
+def test_scrn_cfg2_reduced():
+    """cfg2 reduced rung: H = S = I = 1024, B = 64, T = 8 (bf16)."""
+    _check("scrn", 8, 64, 1024, 1024, "bf16", synth.config_seed(2), TOL_BF16, S=1024)
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_rhn_small(dtype, tol):
+    _check("rhn", 4, 4, 32, 64, dtype, synth.config_seed(3) + 1, tol, L=3)
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_rhn_ragged(dtype, tol):
+    """H = 830 is the cfg3 hidden size (not a multiple of 64: padded internally)."""
+    _check("rhn", 3, 20, 72, 830, dtype, synth.config_seed(3) + 2, tol, L=2)
+
+
+def test_rhn_cfg3_reduced():
+    """cfg3 reduced rung: L = 10, H = I = 830, B = 64, T = 8 (bf16)."""
+    _check("rhn", 8, 64, 830, 830, "bf16", synth.config_seed(3), TOL_BF16, L=10)

@@ -12,27 +12,41 @@ from helpers import TOL_BF16, TOL_FP32, bf16_round, cell_shapes, rel_err
 pytestmark = pytest.mark.gpu
 
 
+ALPHA = 0.95
+S_CTX, L_DEPTH = 24, 2
+
+
 def _lm_case(cell, T, B, I, H, V, seed, bf16, n_symbols=None):
-    shapes = cell_shapes(cell, I, H)
-    shapes.update({"E": (V, I), "W_o": (H, V), "b_o": (V,)})
+    shapes = cell_shapes(cell, I, H, S_CTX, L_DEPTH)
+    Hout = H + S_CTX if cell == "scrn" else H
+    shapes.update({"E": (V, I), "W_o": (Hout, V), "b_o": (V,)})
     p = synth.weights(seed, shapes, H, {"alpha": (0.5, 1.5), "beta1": (0.5, 1.5), "beta2": (0.5, 1.5)})
     if bf16:
-        for k in ("W", "U", "E", "W_o"):
-            p[k] = bf16_round(p[k])
+        for k in ("W", "U", "A", "Bm", "P", "R", "E", "W_o"):
+            if k in p:
+                p[k] = bf16_round(p[k])
     tok = synth.zipf_tokens(seed, "tok", (T + 1, B), V, n_symbols)
     h0 = synth.uniform(seed, "h0", (B, H), -0.5, 0.5)
-    c0 = synth.uniform(seed, "c0", (B, H), -0.5, 0.5)
+    c0 = None if cell == "rhn" else synth.uniform(seed, "c0", (B, S_CTX if cell == "scrn" else H), -0.5, 0.5)
     return p, tok, h0, c0
+
+
+def _cell_kw(cell):
+    if cell == "scrn":
+        return {"context": S_CTX, "scrn_alpha": ALPHA}, {"alpha": np.float32(ALPHA).item()}
+    if cell == "rhn":
+        return {"depth": L_DEPTH}, {}
+    return {}, {}
 
 
 def _run(cell, T, B, I, H, V, dtype, seed, n_symbols=None, lr=0.0):
     import paper_conf_asplos_sivathanucsz19_b200 as A
     p, tok, h0, c0 = _lm_case(cell, T, B, I, H, V, seed, dtype == "bf16", n_symbols)
-    c = A.Cell(cell, H, I, B, T, dtype=dtype)
+    c = A.Cell(cell, H, I, B, T, dtype=dtype, **_cell_kw(cell)[0])
     m = A.LM(c, V)
     m.load(p)
     dev = c.device
-    f32 = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    f32 = lambda a: None if a is None else torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
     m.set_state(f32(h0), f32(c0))
     tokens = torch.as_tensor(tok, dtype=torch.int32, device=dev)
     loss = m.fwd_bwd(tokens)
@@ -42,11 +56,11 @@ def _run(cell, T, B, I, H, V, dtype, seed, n_symbols=None, lr=0.0):
 
 
 @pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
-@pytest.mark.parametrize("cell", ["milstm", "lstm"])
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm", "scrn", "rhn"])
 def test_lm_grads(cell, dtype, tol):
     T, B, I, H, V = 6, 8, 64, 64, 50
     p, tok, h0, c0, loss, g, _ = _run(cell, T, B, I, H, V, dtype, synth.config_seed(5) + 3, n_symbols=40)
-    lo, go, _ = OLM.lm_forward_backward(cell, p, tok, h0, c0)
+    lo, go, _ = OLM.lm_forward_backward(cell, p, tok, h0, c0, **_cell_kw(cell)[1])
     assert abs(loss - lo) / abs(lo) <= tol
     errs = {k: rel_err(g[k], go[k]) for k in go}
     bad = {k: v for k, v in errs.items() if not v <= tol}
@@ -58,6 +72,22 @@ def test_lm_cfg5_shape_reduced_bf16():
     T, B, I, H, V = 4, 64, 2048, 2048, 256
     p, tok, h0, c0, loss, g, _ = _run("milstm", T, B, I, H, V, "bf16", synth.config_seed(5), n_symbols=205)
     lo, go, _ = OLM.lm_forward_backward("milstm", p, tok, h0, c0)
+    assert abs(loss - lo) / abs(lo) <= TOL_BF16
+    errs = {k: rel_err(g[k], go[k]) for k in go}
+    assert all(v <= TOL_BF16 for v in errs.values()), errs
+
+
+@pytest.mark.parametrize("cell,T,B,I,H,V", [("scrn", 4, 64, 1024, 1024, 10000), ("rhn", 3, 64, 830, 830, 10000)])
+def test_lm_cfg2_cfg3_shapes_reduced_bf16(cell, T, B, I, H, V):
+    """cfg2 (SCRN, H=S=1024, V=10k) and cfg3 (RHN L=10 → 2 here, H=830, V=10k) shapes, short T."""
+    global S_CTX
+    old = S_CTX
+    S_CTX = H if cell == "scrn" else S_CTX
+    try:
+        p, tok, h0, c0, loss, g, _ = _run(cell, T, B, I, H, V, "bf16", synth.config_seed(2), n_symbols=None)
+        lo, go, _ = OLM.lm_forward_backward(cell, p, tok, h0, c0, **_cell_kw(cell)[1])
+    finally:
+        S_CTX = old
     assert abs(loss - lo) / abs(lo) <= TOL_BF16
     errs = {k: rel_err(g[k], go[k]) for k in go}
     assert all(v <= TOL_BF16 for v in errs.values()), errs
