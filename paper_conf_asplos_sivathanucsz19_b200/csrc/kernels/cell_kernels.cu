@@ -11,7 +11,7 @@ namespace astra {
 // ============================================================================ mirrors
 template <typename T>
 __global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int H, int Hp, T* __restrict__ dst,
-                                      long ldd) {
+                                      long ldd, long kcols) {
   // tile 32 (k) x 32 (internal rows r); dst[r][k] = src[k][ext(r)]
   __shared__ float tile[32][33];
   const int r0 = blockIdx.x * 32, k0 = blockIdx.y * 32;
@@ -26,16 +26,17 @@ __global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int 
   __syncthreads();
   for (int i = ty; i < 32; i += 8) {
     const int r = r0 + i, k = k0 + tx;
-    if (r < 4 * Hp && k < ldd) dst[(long)r * ldd + k] = from_f<T>(tile[tx][i]);
+    if (r < 4 * Hp && k < kcols) dst[(long)r * ldd + k] = from_f<T>(tile[tx][i]);
   }
 }
 
-void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st) {
-  dim3 grid(cdiv(4L * Hp, 32), cdiv(ldd, 32)), block(32, 8);
+void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st, long kcols) {
+  if (kcols < 0) kcols = ldd;
+  dim3 grid(cdiv(4L * Hp, 32), cdiv(kcols, 32)), block(32, 8);
   if (ot == OT::BF16)
-    mirror_gates_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd);
+    mirror_gates_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
   else
-    mirror_gates_T_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd);
+    mirror_gates_T_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols);
   LAUNCH_CHECK();
 }
 
@@ -110,15 +111,16 @@ void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, l
 template <int KIND, typename T, typename TY>
 __global__ void lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ WX, const float* __restrict__ UH,
                                    GateParams gp, const float* __restrict__ c_prev, float* __restrict__ c_new,
-                                   T* __restrict__ h_op, TY* __restrict__ y, long ldy, float* __restrict__ hT,
-                                   float* __restrict__ cT) {
+                                   T* __restrict__ h_op, long ldh, TY* __restrict__ y, long ldy,
+                                   float* __restrict__ hT, float* __restrict__ cT) {
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int b = blockIdx.y;
   if (j >= Hp) return;
   const long rowg = (long)b * 4 * Hp, rowh = (long)b * Hp;
   if (j >= H) {  // keep padding units exactly zero
     c_new[rowh + j] = 0.f;
-    h_op[rowh + j] = from_f<T>(0.f);
+    h_op[(long)b * ldh + j] = from_f<T>(0.f);
+    if (y && ldy >= Hp) y[(long)b * ldy + j] = from_f<TY>(0.f);
     return;
   }
   float a[4];
@@ -132,7 +134,7 @@ __global__ void lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
   float c, h;
   cell_fwd<KIND>(a, c_prev[rowh + j], c, h);
   c_new[rowh + j] = c;
-  h_op[rowh + j] = from_f<T>(h);
+  h_op[(long)b * ldh + j] = from_f<T>(h);
   if (y) y[(long)b * ldy + j] = from_f<TY>(h);
   if (hT) hT[(long)b * H + j] = h;
   if (cT) cT[(long)b * H + j] = c;
@@ -140,27 +142,27 @@ __global__ void lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
 
 template <int KIND, typename T>
 static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
-                          const float* c_prev, float* c_new, void* h_op, void* y, long ldy, float* hT, float* cT,
-                          cudaStream_t st) {
+                          const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, float* hT,
+                          float* cT, cudaStream_t st) {
   dim3 grid(cdiv(Hp, 128), B);
   if (y_ot == OT::BF16)
     lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
-                                                                     (__nv_bfloat16*)y, ldy, hT, cT);
+                                                                     ldh, (__nv_bfloat16*)y, ldy, hT, cT);
   else
     lstm_fwd_pw_kernel<KIND, T, float><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
-                                                             (float*)y, ldy, hT, cT);
+                                                             ldh, (float*)y, ldy, hT, cT);
   LAUNCH_CHECK();
 }
 
 void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
-                        const float* c_prev, float* c_new, void* h_op, void* y, long ldy, OT y_ot, float* hT,
-                        float* cT, cudaStream_t st) {
+                        const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, OT y_ot,
+                        float* hT, float* cT, cudaStream_t st) {
 #define FWD_CASE(K)                                                                                          \
   if (kind == K) {                                                                                           \
     if (ot == OT::BF16)                                                                                      \
-      fwd_pw_launch<K, __nv_bfloat16>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, y, ldy, hT, cT, st);  \
+      fwd_pw_launch<K, __nv_bfloat16>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, ldh, y, ldy, hT, cT, st);  \
     else                                                                                                     \
-      fwd_pw_launch<K, float>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, y, ldy, hT, cT, st);          \
+      fwd_pw_launch<K, float>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, ldh, y, ldy, hT, cT, st);          \
     return;                                                                                                  \
   }
   FWD_CASE(K_LSTM)

@@ -18,7 +18,8 @@ struct GateParams {          // external-layout fp32 vectors of length 4H (may b
 // ---- mirrors (K9): fp32 params → operand-type copies in the internal layout
 // dst[gcol(g, j)][k] = src[k][g*H + j] for the gate-blocked [K][4H] matrix `src`
 // (dst rows = 4*Hp, row stride ldd ≥ K; padding rows/cols zero).
-void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st);
+void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st,
+                    long kcols = -1);
 // dst[n][k] = src[k][n] (plain transpose), dst [Np][ldd], padding zero.
 void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, long ldd, cudaStream_t st);
 // Operand copy of an external [rows][cols] (OT or fp32 `src_ot`) into [rows][ldd] of type `ot`.
@@ -29,9 +30,10 @@ void copy_pad(OT ot, const void* src, OT src_ot, long rows, int cols, long lds, 
 void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, long ldd, int dcols, cudaStream_t st);
 
 // ---- LSTM-family pointwise halves (cell kind: 0 LSTM, 1 MI-LSTM, 5 subLSTM)
+// h_op: operand copy of h_t, row stride ldh (≥ Hp); y (type y_ot, row stride ldy) optional.
 void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
-                        const float* c_prev, float* c_new, void* h_op, void* y, long ldy, OT y_ot, float* hT,
-                        float* cT, cudaStream_t st);
+                        const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, OT y_ot,
+                        float* hT, float* cT, cudaStream_t st);
 // dy: row stride ldy of type dy_ot (or fp32); dh_rec: [B][ld_dh] fp32 or null (zeros).
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
                         const float* dh_rec, long ld_dh, float* dc, const float* WX, const float* UH,
@@ -59,6 +61,13 @@ void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const void* dy,
                 cudaStream_t st);
 void reduce_blocked_partials(const float* part, int nchunk, int nq, int H, int Hp, float* out, cudaStream_t st);
 void mirror_blocked_T(OT ot, const float* src, int K, int G, int H, int Hp, void* dst, long ldd, cudaStream_t st);
+
+// ---- K3 attention step (attn_kernels.cu): q [B][Ap], keys/enc [Ts][B][Ap|Hp] fp32, pr [B][Ts]
+void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q, const float* keys, const float* v,
+              const float* enc, float* pr, void* ctx_op, long ldc, void* y_ctx, long ldy, cudaStream_t st);
+void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
+              const float* dctx_rec, long ldr, const float* pr, const float* q, const float* keys, const float* v,
+              const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first, cudaStream_t st);
 
 // ---- LM pieces
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);

@@ -6,6 +6,7 @@
 //   LstmCell  — LSTM, MI-LSTM [36], subLSTM [8]      (cell_lstm.cpp)
 //   ScrnCell  — SC-RNN / SCRN [22]                    (cell_scrn.cpp)
 //   RhnCell   — recurrent highway network [39]        (cell_rhn.cpp)
+//   AttnCell  — LSTM encoder + attentive decoder [35] (cell_attn.cpp)
 #pragma once
 #include <cuda_runtime.h>
 
@@ -108,7 +109,8 @@ class Cell {
 
   // LM mode hooks (set by LM)
   bool lm_mode = false;
-  const float* lm_dy = nullptr;  // fp32 [T*B][y_width()] internal dY for the backward
+  const float* lm_dy = nullptr;  // fp32 [T*B][y_width()] internal dY for the backward (null: external dy)
+  float* y_f32 = nullptr;        // optional internal fp32 output [T*B][y_width()] (LSTM family)
   int lm_V = 0;
 
   // ---- per-family interface
@@ -119,6 +121,7 @@ class Cell {
   virtual int y_width() const = 0;               // padded K of the head
   virtual std::vector<KSeg> y_segments() const = 0;
   virtual int c_width() const { return H; }      // width of the second state (c or s); 0 = none
+  virtual bool lm_capable() const { return true; }
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
   // ---- shared machinery

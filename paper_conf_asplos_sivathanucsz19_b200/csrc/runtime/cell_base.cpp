@@ -301,6 +301,7 @@ std::string Cell::report() {
 std::unique_ptr<Cell> make_lstm_cell(const astra_cell_desc& d);
 std::unique_ptr<Cell> make_scrn_cell(const astra_cell_desc& d);
 std::unique_ptr<Cell> make_rhn_cell(const astra_cell_desc& d);
+std::unique_ptr<Cell> make_attn_cell(const astra_cell_desc& d);
 
 std::unique_ptr<Cell> make_cell(const astra_cell_desc& d) {
   switch (d.cell_type) {
@@ -309,7 +310,7 @@ std::unique_ptr<Cell> make_cell(const astra_cell_desc& d) {
     case ASTRA_SUBLSTM: return make_lstm_cell(d);
     case ASTRA_SCRNN: return make_scrn_cell(d);
     case ASTRA_RHN: return make_rhn_cell(d);
-    case ASTRA_LSTM_ATTN: throw Error(ASTRA_E_UNSUPPORTED, "cell: the LSTM-attention CUDA path is not built yet");
+    case ASTRA_LSTM_ATTN: return make_attn_cell(d);
     default: throw Error(ASTRA_E_ARG, "cell: unknown cell_type");
   }
 }

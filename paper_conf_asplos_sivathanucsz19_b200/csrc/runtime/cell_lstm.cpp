@@ -116,10 +116,14 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     float* UHt = UH + (long)t * B * NG;
     run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st);
     const bool last = t == T - 1;
-    void* yt = y ? (char*)y + (size_t)t * B * H * e : nullptr;
-    lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
-                       Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), yt, H, ot, last ? hT : nullptr,
-                       last ? cT : nullptr, st);
+    if (y_f32)   // internal fp32 output (e.g. the encoder of LSTM-attention), row stride Hp
+      lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
+                         Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y_f32 + (size_t)t * B * Hp, Hp, OT::F32,
+                         last ? hT : nullptr, last ? cT : nullptr, st);
+    else
+      lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
+                         Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y ? (char*)y + (size_t)t * B * H * e : nullptr,
+                         H, ot, last ? hT : nullptr, last ? cT : nullptr, st);
   }
   mark(R_FWD, 1, st);
   fwd_done = true;
@@ -127,7 +131,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
 
 void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0) {
   ASTRA_CHECK_STATE(bound && fwd_done, "step_bwd: needs a preceding step_fwd");
-  ASTRA_CHECK_ARG(lm_mode || dy, "step_bwd: dy is null");
+  ASTRA_CHECK_ARG(lm_dy || dy, "step_bwd: dy is null");
   cudaStream_t st = main_st;
   const long TB = (long)T * B;
   const size_t e = esz();
@@ -171,7 +175,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     const void* dyt;
     long ldy;
     bool dyf32;
-    if (lm_mode) { dyt = lm_dy + (long)t * B * Hp; ldy = Hp; dyf32 = true; }
+    if (lm_dy) { dyt = lm_dy + (long)t * B * Hp; ldy = Hp; dyf32 = true; }
     else { dyt = (const char*)dy + (size_t)t * B * H * e; ldy = H; dyf32 = false; }
     lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, dC, WX + (long)t * B * NG,
                        UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,

@@ -8,6 +8,7 @@ namespace astra {
 
 LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
   ASTRA_CHECK_ARG(vocab > 1, "lm: vocab must be > 1");
+  if (!c->lm_capable()) throw Error(ASTRA_E_UNSUPPORTED, "lm: this cell type has no LM wrapper (reading R10)");
   Vp = (int)round_up(V, 8);
   Yw = c->y_width();
   c->lm_V = V;

@@ -113,3 +113,63 @@ def test_rhn_ragged(dtype, tol):
 def test_rhn_cfg3_reduced():
     """cfg3 reduced rung: L = 10, H = I = 830, B = 64, T = 8 (bf16)."""
     _check("rhn", 8, 64, 830, 830, "bf16", synth.config_seed(3), TOL_BF16, L=10)
+
+
+# ------------------------------------------------------------------ LSTM + attention [35]
+def _attn_case(Ts, Tt, B, I, H, A, seed, bf16):
+    from helpers import bf16_round
+    shapes = C.attn_param_shapes(I, H, A)
+    p = synth.weights(seed, shapes, H)
+    inp = {"xe": synth.uniform(seed, "xe", (Ts, B, I), -1, 1), "xd": synth.uniform(seed, "xd", (Tt, B, I), -1, 1),
+           "h0": synth.uniform(seed, "h0", (B, H), -0.5, 0.5), "c0": synth.uniform(seed, "c0", (B, H), -0.5, 0.5)}
+    dY = synth.normal(seed, "dY", (Tt, B, 2 * H))
+    if bf16:
+        for k in ("W_e", "U_e", "W_k", "W_d", "U_d", "C_d", "W_q"):
+            p[k] = bf16_round(p[k])
+        inp["xe"], inp["xd"], dY = bf16_round(inp["xe"]), bf16_round(inp["xd"]), bf16_round(dY)
+    return p, inp, dY, synth.normal(seed, "dhT", (B, H)), synth.normal(seed, "dcT", (B, H))
+
+
+def _attn_check(Ts, Tt, B, I, H, A, dtype, seed, tol):
+    import paper_conf_asplos_sivathanucsz19_b200 as AS
+    p, inp, dY, dhT, dcT = _attn_case(Ts, Tt, B, I, H, A, seed, dtype == "bf16")
+    out_o, g_o = C.cell_fwd_bwd("attn", p, inp, dY, dhT, dcT)
+    c = AS.Cell("attn", H, I, B, Tt, dtype=dtype, src_seq=Ts, attn_dim=A)
+    c.load(p)
+    dev = c.device
+    tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
+    f32 = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    x = torch.cat([f32(inp["xe"]).reshape(-1), f32(inp["xd"]).reshape(-1)]).to(tdt).contiguous()
+    y = torch.empty(Tt, B, 2 * H, dtype=tdt, device=dev)
+    hT, cT = torch.empty(B, H, device=dev), torch.empty(B, H, device=dev)
+    c.forward(x, f32(inp["h0"]), f32(inp["c0"]), y, hT, cT)
+    dx = torch.empty((Ts + Tt) * B * I, dtype=tdt, device=dev)
+    dh0, dc0 = torch.empty(B, H, device=dev), torch.empty(B, H, device=dev)
+    c.backward(f32(dY).to(tdt).contiguous(), f32(dhT), f32(dcT), dx, dh0, dc0)
+    torch.cuda.synchronize()
+    dxn = dx.float().cpu().numpy()
+    got = {"y": y.float().cpu().numpy(), "hT": hT.cpu().numpy(), "cT": cT.cpu().numpy(),
+           "dxe": dxn[:Ts * B * I].reshape(Ts, B, I), "dxd": dxn[Ts * B * I:].reshape(Tt, B, I),
+           "dh0": dh0.cpu().numpy(), "dc0": dc0.cpu().numpy()}
+    for k in p:
+        got[k] = c.view(k, c.grads).cpu().numpy().reshape(np.shape(p[k]))
+    ref = dict(out_o)
+    ref.update(g_o)
+    errs = {k: rel_err(got[k], ref[k]) for k in ref}
+    bad = {k: v for k, v in errs.items() if not v <= tol}
+    assert not bad, (dtype, bad, errs)
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_attn_small(dtype, tol):
+    _attn_check(5, 4, 4, 32, 64, 48, dtype, synth.config_seed(4) + 1, tol)
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_attn_ragged(dtype, tol):
+    _attn_check(7, 3, 20, 40, 100, 72, dtype, synth.config_seed(4) + 2, tol)
+
+
+def test_attn_cfg4_reduced():
+    """cfg4 reduced rung: H = A = I = 1024, B = 128, Ts = Tt = 8 (bf16)."""
+    _attn_check(8, 8, 128, 1024, 1024, 1024, "bf16", synth.config_seed(4), TOL_BF16)
