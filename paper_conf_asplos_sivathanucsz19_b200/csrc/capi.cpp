@@ -199,6 +199,13 @@ astra_status astra_comm_init(astra_cell c, const void* uid, int rank, int world)
     cc.nccl_comm = comm;
     cc.rank = rank;
     cc.world = world;
+    if (!cc.comm_st) {   // no caller comm stream: own a high-priority one so buckets overlap compute
+      int lo = 0, hi = 0;
+      CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+      CUDA_TRY(cudaStreamCreateWithPriority(&cc.own_comm_st, cudaStreamNonBlocking, hi));
+      cc.comm_st = cc.own_comm_st;
+    }
+    if (!cc.tune_dev) CUDA_TRY(cudaMalloc(&cc.tune_dev, 64 * sizeof(double)));
   });
 }
 

@@ -131,7 +131,13 @@ class Cell {
   float* g(const std::string& n) { return G + find_param(n); }
   void bind(float* params, float* grads, void* saved_p, void* scratch_p);
   void sgd_step(float lr);
-  void allreduce_grads(float* grads, size_t n, cudaStream_t after);
+  void grad_bucket(float* p, size_t n, cudaStream_t producer);   // K11: launch one DP bucket
+  void grad_join(cudaStream_t main);                               // main waits for all buckets
+  cudaEvent_t ev_bucket[4] = {nullptr, nullptr, nullptr, nullptr};
+  int bucket_i = 0;
+  bool sync_pending = false;
+  cudaStream_t own_comm_st = nullptr;
+  double* tune_dev = nullptr;          // 64 doubles: cross-rank max of the tuner's metric vector
   size_t esz() const { return ot_size(ot); }
   template <typename T_> T_* sv(size_t off) { return reinterpret_cast<T_*>(saved + off); }
   template <typename T_> T_* sc(size_t off) { return reinterpret_cast<T_*>(scratch + off); }

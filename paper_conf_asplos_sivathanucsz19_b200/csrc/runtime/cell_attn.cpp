@@ -310,7 +310,8 @@ class AttnCell : public Cell {
     enc->lm_dy = denc;
     enc->backward(nullptr, dh0e, dc0e, dx, dh0, dc0);
     enc->lm_dy = nullptr;
-    if (world > 1) allreduce_grads(G, n_params, st);
+    grad_bucket(G, n_params, st);
+    grad_join(st);
     mark(R_STEP, 1, st);
   }
 };

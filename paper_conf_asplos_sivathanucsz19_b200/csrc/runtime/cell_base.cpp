@@ -96,6 +96,10 @@ Cell::~Cell() {
       if (ev[r][w]) cudaEventDestroy(ev[r][w]);
   if (ev_fork) cudaEventDestroy(ev_fork);
   if (ev_join) cudaEventDestroy(ev_join);
+  for (int k = 0; k < 4; ++k)
+    if (ev_bucket[k]) cudaEventDestroy(ev_bucket[k]);
+  if (own_comm_st) cudaStreamDestroy(own_comm_st);
+  if (tune_dev) cudaFree(tune_dev);
   if (nccl_comm) ncclCommDestroy((ncclComm_t)nccl_comm);
 }
 
@@ -116,6 +120,7 @@ void Cell::bind(float* pp, float* gg, void* sv_p, void* sc_p) {
   if (!ev_fork) {
     CUDA_TRY(cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming));
     CUDA_TRY(cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming));
+    for (int k = 0; k < 4; ++k) CUDA_TRY(cudaEventCreateWithFlags(&ev_bucket[k], cudaEventDisableTiming));
     for (int r = 0; r < R_COUNT; ++r)
       for (int w = 0; w < 2; ++w) CUDA_TRY(cudaEventCreate(&ev[r][w]));
   }
@@ -149,21 +154,33 @@ void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz
   }
 }
 
-void Cell::allreduce_grads(float* grads, size_t n, cudaStream_t after) {
-  ASTRA_CHECK_STATE(nccl_comm, "allreduce: astra_comm_init not called");
-  cudaStream_t cs = comm_st ? comm_st : after;
-  if (cs != after) {
-    CUDA_TRY(cudaEventRecord(ev_fork, after));
-    CUDA_TRY(cudaStreamWaitEvent(cs, ev_fork, 0));
+// K11: bucketed data-parallel gradient sum.  Each bucket is launched on the comm
+// stream as soon as the kernel producing it has been enqueued on `producer` (event edge), so the
+// NCCL all-reduce of the head / dU / dW buckets overlaps the remaining BPTT and weight-gradient
+// work; grad_join() makes `main` wait for every bucket before SGD.  Sum then ×1/world: the mean
+// of the shard-mean gradients = the full-batch mean gradient (oracle/dp.py).
+void Cell::grad_bucket(float* p, size_t n, cudaStream_t producer) {
+  if (world <= 1 || !nccl_comm || n == 0) return;
+  cudaStream_t cs = comm_st ? comm_st : producer;
+  cudaEvent_t evb = ev_bucket[bucket_i++ % 4];
+  if (cs != producer) {
+    CUDA_TRY(cudaEventRecord(evb, producer));
+    CUDA_TRY(cudaStreamWaitEvent(cs, evb, 0));
   }
-  ncclResult_t r = ncclAllReduce(grads, grads, n, ncclFloat, ncclSum, (ncclComm_t)nccl_comm, cs);
+  ncclResult_t r = ncclAllReduce(p, p, n, ncclFloat, ncclSum, (ncclComm_t)nccl_comm, cs);
   if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
   count_launch();
-  scale_inplace(grads, n, 1.0f / (float)world, cs);
-  if (cs != after) {
-    CUDA_TRY(cudaEventRecord(ev_join, cs));
-    CUDA_TRY(cudaStreamWaitEvent(after, ev_join, 0));
+  scale_inplace(p, n, 1.0f / (float)world, cs);
+  sync_pending = true;
+}
+
+void Cell::grad_join(cudaStream_t main) {
+  if (!sync_pending) return;
+  if (comm_st && comm_st != main) {
+    CUDA_TRY(cudaEventRecord(ev_join, comm_st));
+    CUDA_TRY(cudaStreamWaitEvent(main, ev_join, 0));
   }
+  sync_pending = false;
 }
 
 void Cell::sgd_step(float lr) {
@@ -268,6 +285,16 @@ int Cell::tune_next() {
   if (rep_i < tune_reps) {
     ++rep_i;
     return ASTRA_TUNE_EXPLORING;
+  }
+  if (world > 1 && nccl_comm) {
+    // reading R29: every rank must take the same decision — max-reduce the metric vector
+    const size_t n = rep_min.size();
+    ASTRA_CHECK_STATE(n <= 64, "tuner: too many metrics");
+    CUDA_TRY(cudaMemcpyAsync(tune_dev, rep_min.data(), n * sizeof(double), cudaMemcpyHostToDevice, main_st));
+    ncclResult_t r = ncclAllReduce(tune_dev, tune_dev, n, ncclDouble, ncclMax, (ncclComm_t)nccl_comm, main_st);
+    if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclAllReduce(max): ") + ncclGetErrorString(r));
+    CUDA_TRY(cudaMemcpyAsync(rep_min.data(), tune_dev, n * sizeof(double), cudaMemcpyDeviceToHost, main_st));
+    CUDA_TRY(cudaStreamSynchronize(main_st));
   }
   wirer->feed(rep_min);
   rep_i = 0;

@@ -202,6 +202,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   if (st_u == st) mark(R_DU, 0, st);
   run_gemm(4, gu, epi_perm(g("U"), 4L * H, H, NG, GATE_U, 0, H), 0, 0, var.g[G_DU], st_u);
   if (st_u == st) mark(R_DU, 1, st);
+  grad_bucket(g("U"), (size_t)H * 4 * H, st_u);
 
   GemmSpec gw;
   gw.A = mat(X, I, TB, Ip);
@@ -212,6 +213,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   mark(R_DW, 0, st);
   run_gemm(5, gw, epi_perm(g("W"), 4L * H, I, NG, GATE_U, 0, H), 0, 0, var.g[G_DW], st);
   mark(R_DW, 1, st);
+  grad_bucket(g("W"), (size_t)I * 4 * H, st);
 
   if (dx) {
     GemmSpec gx;
@@ -229,12 +231,13 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   float* gq[4] = {g("b"), nullptr, nullptr, nullptr};
   if (kind == K_MILSTM) { gq[1] = g("alpha"); gq[2] = g("beta1"); gq[3] = g("beta2"); }
   reduce_gate_partials(part, nchunk, nq, H, Hp, gq, st);
+  grad_bucket(g("b"), (size_t)(G + n_params - g("b")), st);   // b (and α, β1, β2): the tail of the cell block
   if (st_u != st) {
     CUDA_TRY(cudaEventRecord(ev_join, st_u));
     CUDA_TRY(cudaStreamWaitEvent(st, ev_join, 0));
   }
   mark(R_SE4, 1, st);
-  if (world > 1 && !lm_mode) allreduce_grads(G, n_params, st);
+  if (!lm_mode) grad_join(st);
   if (!lm_mode) mark(R_STEP, 1, st);
 }
 

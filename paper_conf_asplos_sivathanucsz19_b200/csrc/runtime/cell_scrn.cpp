@@ -223,7 +223,8 @@ class ScrnCell : public Cell {
       mark(R_DX, 1, st);
     }
     mark(R_SE4, 1, st);
-    if (world > 1 && !lm_mode) allreduce_grads(G, n_params, st);
+    grad_bucket(G, n_params, st);   // one bucket for the cell's parameters
+    if (!lm_mode) grad_join(st);
     if (!lm_mode) mark(R_STEP, 1, st);
   }
 };

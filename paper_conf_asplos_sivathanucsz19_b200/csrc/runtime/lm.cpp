@@ -127,13 +127,16 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   }
   colsum(dlog32, TB, V, V, (float*)(ws + off_colsum), G + find("b_o"), st);
   c.mark(R_HEAD, 1, st);
+  // a7 bucket 1: the head gradients are final before BPTT — their sum overlaps the chain
+  c.grad_bucket(G + find("W_o"), n_params - find("W_o"), st);
 
   // cell backward (SE3 + SE4) and the embedding backward
   c.lm_dy = dY;
   c.backward(nullptr, nullptr, nullptr, dX, nullptr, nullptr);
   embed_bwd(tokens, TB, V, dX, c.Ip, c.I, G + find("E"), ws + off_sort, sort_bytes, (float*)(ws + off_embpart), st);
-  // a7: data-parallel gradient sum (mean over ranks), then a8: SGD
-  if (c.world > 1) c.allreduce_grads(G, n_params, st);
+  // a7: last bucket (embedding), join, then a8: SGD
+  c.grad_bucket(G + find("E"), (size_t)V * c.I, st);
+  c.grad_join(st);
   if (do_sgd) sgd(P, G, n_params, lr, st);
   c.mark(R_STEP, 1, st);
 }
