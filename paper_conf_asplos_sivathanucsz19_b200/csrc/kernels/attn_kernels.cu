@@ -45,7 +45,7 @@ __global__ void __launch_bounds__(ATT_THREADS)
   for (int j = 0; j < Ts; ++j) {
     const float* kj = keys + ((long)j * B + b) * Ap;
     float s = 0.f;
-    for (int a = threadIdx.x; a < A; a += ATT_THREADS) s = __fadd_rn(s, __fmul_rn(v[a], tanh_(__fadd_rn(qb[a], kj[a]))));
+    for (int a = threadIdx.x; a < A; a += ATT_THREADS) s = __fadd_rn(s, __fmul_rn(v[a], tanh_<FastMath<T>::value>(__fadd_rn(qb[a], kj[a]))));
     const float tot = block_sum(s, red);
     if (threadIdx.x == 0) e[j] = tot;
   }
@@ -139,7 +139,7 @@ __global__ void __launch_bounds__(ATT_THREADS)
       float* dkj = dk + ((long)j * B + b) * Ap + a;
       float du = 0.f;
       if (valid) {
-        const float u = tanh_(__fadd_rn(qb[a], keys[((long)j * B + b) * Ap + a]));
+        const float u = tanh_<FastMath<T>::value>(__fadd_rn(qb[a], keys[((long)j * B + b) * Ap + a]));
         du = __fmul_rn(__fmul_rn(de[j], v[a]), __fsub_rn(1.f, __fmul_rn(u, u)));
         dq = __fadd_rn(dq, du);
         dva = __fadd_rn(dva, __fmul_rn(de[j], u));

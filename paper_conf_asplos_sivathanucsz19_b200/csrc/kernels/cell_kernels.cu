@@ -127,12 +127,12 @@ __global__ void lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
 #pragma unroll
   for (int g = 0; g < 4; ++g) {
     const int col = gcol(g, j), e = g * H + j;
-    const float wx = WX[rowg + col], uh = UH[rowg + col];
+    const float wx = __ldcs(WX + rowg + col), uh = __ldcs(UH + rowg + col);
     a[g] = preact<KIND>(wx, uh, gp.b[e], KIND == K_MILSTM ? gp.alpha[e] : 0.f, KIND == K_MILSTM ? gp.beta1[e] : 0.f,
                         KIND == K_MILSTM ? gp.beta2[e] : 0.f);
   }
   float c, h;
-  cell_fwd<KIND>(a, c_prev[rowh + j], c, h);
+  cell_fwd<KIND, FastMath<T>::value>(a, c_prev[rowh + j], c, h);
   c_new[rowh + j] = c;
   h_op[(long)b * ldh + j] = from_f<T>(h);
   if (y) y[(long)b * ldy + j] = from_f<TY>(h);
@@ -185,7 +185,7 @@ int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 template <int KIND, typename T, typename TDY>
 __global__ void __launch_bounds__(BWD_UX * BWD_RY, 2)
     lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
-                       long ld_dh, float* __restrict__ dc, const float* __restrict__ WX, const float* __restrict__ UH,
+                       long ld_dh, int nsplit, long split_stride, float* __restrict__ dc, const float* __restrict__ WX, const float* __restrict__ UH,
                        const float* __restrict__ c_new, const float* __restrict__ c_prev, GateParams gp,
                        T* __restrict__ D_uh, T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
   __shared__ float red[BWD_RY][16][BWD_UX];
@@ -212,15 +212,19 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 2)
       float wx[4], uh[4], a[4];
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
-        wx[g] = WX[rg + gcol(g, j)];
-        uh[g] = UH[rg + gcol(g, j)];
+        wx[g] = __ldcs(WX + rg + gcol(g, j));
+        uh[g] = __ldcs(UH + rg + gcol(g, j));
         a[g] = preact<KIND>(wx[g], uh[g], bb[g], al[g], be1[g], be2[g]);
       }
       float dh = to_f<TDY>(dy[(long)b * ldy + j]);
-      if (dh_rec) dh = __fadd_rn(dh, dh_rec[(long)b * ld_dh + j]);
+      if (dh_rec) {   // split-K partials of dh_rec summed in chunk order, then added to dy
+        float r = dh_rec[(long)b * ld_dh + j];
+        for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, dh_rec[k * split_stride + (long)b * ld_dh + j]);
+        dh = __fadd_rn(dh, r);
+      }
       float dcv = dc[(long)b * Hp + j];
       float da[4];
-      cell_bwd<KIND>(a, c_prev[(long)b * Hp + j], c_new[(long)b * Hp + j], dh, dcv, da);
+      cell_bwd<KIND, FastMath<T>::value>(a, c_prev[(long)b * Hp + j], c_new[(long)b * Hp + j], dh, dcv, da);
       dc[(long)b * Hp + j] = dcv;
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
@@ -229,7 +233,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 2)
           const float duh = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], wx[g]), be1[g]));
           const float dwx = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], uh[g]), be2[g]));
           D_uh[rg + gcol(g, j)] = from_f<T>(duh);
-          D_wx[rg + gcol(g, j)] = from_f<T>(dwx);
+          __stcs(D_wx + rg + gcol(g, j), from_f<T>(dwx));
           s[4 + g] = __fadd_rn(s[4 + g], __fmul_rn(__fmul_rn(da[g], wx[g]), uh[g]));
           s[8 + g] = __fadd_rn(s[8 + g], __fmul_rn(da[g], uh[g]));
           s[12 + g] = __fadd_rn(s[12 + g], __fmul_rn(da[g], wx[g]));
@@ -266,33 +270,33 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 2)
 
 template <int KIND, typename T>
 static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32, const float* dh_rec,
-                          long ld_dh, float* dc, const float* WX, const float* UH, const float* c_new,
+                          long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH, const float* c_new,
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
                           bool first, cudaStream_t st) {
   dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
   dim3 block(BWD_UX, BWD_RY);
   if (dy_f32 || dy_ot == OT::F32)
-    lstm_bwd_pw_kernel<KIND, T, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, dc, WX,
+    lstm_bwd_pw_kernel<KIND, T, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX,
                                                              UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials,
                                                              nq, first);
   else
     lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, block, 0, st>>>(B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec,
-                                                                     ld_dh, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh,
+                                                                     ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh,
                                                                      (T*)D_wx, partials, nq, first);
   LAUNCH_CHECK();
 }
 
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
-                        const float* dh_rec, long ld_dh, float* dc, const float* WX, const float* UH,
+                        const float* dh_rec, long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH,
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
                         float* partials, int nq, bool first, cudaStream_t st) {
 #define BWD_CASE(K)                                                                                            \
   if (kind == K) {                                                                                             \
     if (ot == OT::BF16)                                                                                        \
-      bwd_pw_launch<K, __nv_bfloat16>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, dc, WX, UH, c_new, c_prev, \
+      bwd_pw_launch<K, __nv_bfloat16>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, \
                                       gp, D_uh, D_wx, partials, nq, first, st);                                \
     else                                                                                                       \
-      bwd_pw_launch<K, float>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, dc, WX, UH, c_new, c_prev, gp,  \
+      bwd_pw_launch<K, float>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp,  \
                               D_uh, D_wx, partials, nq, first, st);                                            \
     return;                                                                                                    \
   }

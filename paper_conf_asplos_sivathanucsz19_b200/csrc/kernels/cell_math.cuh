@@ -11,8 +11,26 @@ namespace astra {
 constexpr int GATE_U = 64;
 __host__ __device__ __forceinline__ int gcol(int g, int j) { return (j / GATE_U) * (4 * GATE_U) + g * GATE_U + (j % GATE_U); }
 
-__device__ __forceinline__ float sigm(float x) { return __frcp_rn(__fadd_rn(1.f, expf(-x))); }
-__device__ __forceinline__ float tanh_(float x) { return tanhf(x); }
+// Transcendentals.  fp32 path (F = false): IEEE-accurate expf / tanhf (the 1e-4 parity bar).  bf16
+// path (F = true, reading R3): the MUFU tanh.approx.f32 (rel. error ≈ 2^-11), σ(x) = ½·tanh(x/2) + ½ —
+// far below the 2e-2 bar and shared by every bf16 kernel variant, so variants stay bitwise equal.
+__device__ __forceinline__ float tanh_approx(float x) {
+  float y;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+template <bool F = false>
+__device__ __forceinline__ float sigm(float x) {
+  if (F) return __fmaf_rn(0.5f, tanh_approx(__fmul_rn(0.5f, x)), 0.5f);
+  return __frcp_rn(__fadd_rn(1.f, expf(-x)));
+}
+template <bool F = false>
+__device__ __forceinline__ float tanh_(float x) {
+  if (F) return tanh_approx(x);
+  return tanhf(x);
+}
+template <typename T> struct FastMath { static constexpr bool value = false; };
+template <> struct FastMath<__nv_bfloat16> { static constexpr bool value = true; };
 
 template <typename T> __device__ __forceinline__ float to_f(T v);
 template <> __device__ __forceinline__ float to_f<float>(float v) { return v; }
@@ -38,27 +56,27 @@ __device__ __forceinline__ float preact(float wx, float uh, float b, float al, f
 }
 
 // Forward cell update from the four pre-activations.  Returns (c_new, h_new).
-template <int KIND>
+template <int KIND, bool F = false>
 __device__ __forceinline__ void cell_fwd(const float (&a)[4], float c_prev, float& c_new, float& h_new) {
   if (KIND == K_SUBLSTM) {
-    const float i = sigm(a[0]), f = sigm(a[1]), z = sigm(a[2]), o = sigm(a[3]);
+    const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), z = sigm<F>(a[2]), o = sigm<F>(a[3]);
     c_new = __fsub_rn(__fadd_rn(__fmul_rn(f, c_prev), z), i);
-    h_new = __fsub_rn(sigm(c_new), o);
+    h_new = __fsub_rn(sigm<F>(c_new), o);
   } else {
-    const float i = sigm(a[0]), f = sigm(a[1]), g = tanh_(a[2]), o = sigm(a[3]);
+    const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), g = tanh_<F>(a[2]), o = sigm<F>(a[3]);
     c_new = __fadd_rn(__fmul_rn(f, c_prev), __fmul_rn(i, g));
-    h_new = __fmul_rn(o, tanh_(c_new));
+    h_new = __fmul_rn(o, tanh_<F>(c_new));
   }
 }
 
 // Backward of one cell update.  dh = dL/dh_t, dc = dL/dc_t from step t+1 (in/out: becomes
 // dL/dc_{t-1}).  da[4] = dL/da for the four gates.
-template <int KIND>
+template <int KIND, bool F = false>
 __device__ __forceinline__ void cell_bwd(const float (&a)[4], float c_prev, float c_new, float dh, float& dc,
                                          float (&da)[4]) {
   if (KIND == K_SUBLSTM) {
-    const float i = sigm(a[0]), f = sigm(a[1]), z = sigm(a[2]), o = sigm(a[3]);
-    const float sc = sigm(c_new);
+    const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), z = sigm<F>(a[2]), o = sigm<F>(a[3]);
+    const float sc = sigm<F>(c_new);
     const float dcc = __fadd_rn(dc, __fmul_rn(dh, __fmul_rn(sc, __fsub_rn(1.f, sc))));
     da[0] = __fmul_rn(-dcc, __fmul_rn(i, __fsub_rn(1.f, i)));
     da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), __fmul_rn(f, __fsub_rn(1.f, f)));
@@ -66,8 +84,8 @@ __device__ __forceinline__ void cell_bwd(const float (&a)[4], float c_prev, floa
     da[3] = __fmul_rn(-dh, __fmul_rn(o, __fsub_rn(1.f, o)));
     dc = __fmul_rn(dcc, f);
   } else {
-    const float i = sigm(a[0]), f = sigm(a[1]), g = tanh_(a[2]), o = sigm(a[3]);
-    const float tau = tanh_(c_new);
+    const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), g = tanh_<F>(a[2]), o = sigm<F>(a[3]);
+    const float tau = tanh_<F>(c_new);
     const float dcc = __fadd_rn(dc, __fmul_rn(__fmul_rn(dh, o), __fsub_rn(1.f, __fmul_rn(tau, tau))));
     da[0] = __fmul_rn(__fmul_rn(dcc, g), __fmul_rn(i, __fsub_rn(1.f, i)));
     da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), __fmul_rn(f, __fsub_rn(1.f, f)));

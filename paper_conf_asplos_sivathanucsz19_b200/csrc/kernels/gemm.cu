@@ -69,7 +69,7 @@ static int smem_for(int& stages) {
 }
 
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
-                     int cm, int cn) {
+                     int cm, int cn, bool b_keep, int ksplit) {
   ASTRA_CHECK_ARG((cm == 1 || cm == 2 || cm == 4) && (cn == 1 || cn == 2 || cn == 4) && cm * cn <= 8,
                   "tc_gemm: cluster shape must be cm, cn in {1,2,4}, cm*cn <= 8");
   ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256, "tc_gemm: BN must be 64, 128 or 256");
@@ -78,6 +78,9 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm);
   g.args.cm = cm;
   g.args.cn = cn;
+  g.args.b_keep = b_keep ? 1 : 0;
+  ASTRA_CHECK_ARG(ksplit >= 1 && (ksplit == 1 || cm * cn == 1), "tc_gemm: split-K needs a 1x1 cluster");
+  g.args.ksplit = ksplit;
   g.BN = BN;
   g.args.M = M; g.args.N = N; g.args.K = K;
   g.args.num_m = cdiv(M, TC_BM);
@@ -107,7 +110,7 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   a.az = az;
   a.bz = bz;
   const int cs = a.cm * a.cn;
-  const int ctiles = cdiv(a.num_m, a.cm) * cdiv(a.num_n, a.cn);   // cluster tiles
+  const int ctiles = cdiv(a.num_m, a.cm) * cdiv(a.num_n, a.cn) * a.ksplit;   // cluster tiles × K chunks
   int clusters = num_sms() / cs;
   if (max_ctas > 0 && max_ctas / cs < clusters) clusters = max_ctas / cs > 0 ? max_ctas / cs : 1;
   if (ctiles < clusters) clusters = ctiles;

@@ -35,6 +35,8 @@ struct TcArgs {
   int a_mn, b_mn;   // 1 = MN-major operand
   int stages;
   int cm, cn;       // cluster shape (CTAs sharing B along M, sharing A along N)
+  int b_keep;       // 1: load B with an L2 evict_last policy (weights re-read every step)
+  int ksplit;       // fixed split of K into ksplit chunks; chunk ks writes its fp32 partial to C + ks·split_stride
   uint32_t idesc;
 };
 
@@ -66,6 +68,7 @@ struct EpiStore {
   int perm_u, perm_H; // 0 = identity mapping
   int perm_blk;
   int accumulate;
+  long split_stride;  // elements between the partial outputs of a split-K GEMM
 
   __device__ __forceinline__ int map_col(int n, bool& ok) const {
     if (n >= Nv) {  // columns past the GEMM's N (tile overhang) are never stored
@@ -151,12 +154,14 @@ struct EpiStore {
   }
 
   template <int BN>
-  __device__ __forceinline__ void run(uint32_t taddr, int m0, int n0, int row) const {
+  __device__ __forceinline__ void run(uint32_t taddr, int m0, int n0, int row, int ks) const {
+    EpiStore e = *this;
+    if (ks) e.C = reinterpret_cast<char*>(C) + (size_t)ks * split_stride * (out_bf16 ? 2 : 4);
 #pragma unroll 1
     for (int c = 0; c < BN; c += 16) {
       float v[16];
       sm100::tmem_ld16(taddr + c, v);
-      store16(m0 + row, n0 + c, v);
+      e.store16(m0 + row, n0 + c, v);
     }
   }
 };
@@ -187,9 +192,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   const int crank = cs > 1 ? (int)sm100::cluster_ctarank() : 0;
   const int rm = crank % cm, rn = crank / cm;
   const int ncm = (args.num_m + cm - 1) / cm, ncn = (args.num_n + cn - 1) / cn;
-  const int num_ct = ncm * ncn;                  // cluster tiles
+  const int num_ct1 = ncm * ncn;                 // cluster tiles of one K chunk
+  const int num_ct = num_ct1 * args.ksplit;      // × fixed K chunks (split-K)
   const int cluster_id = blockIdx.x / cs, num_clusters = gridDim.x / cs;
-  const int nk = (args.K + TC_BK - 1) / TC_BK;
+  const int nk_all = (args.K + TC_BK - 1) / TC_BK;
+  const int kper = (nk_all + args.ksplit - 1) / args.ksplit;
   uint16_t mask_a = 0, mask_b = 0;
   for (int j = 0; j < cn; ++j) mask_a |= (uint16_t)(1u << (rm + cm * j));
   for (int i = 0; i < cm; ++i) mask_b |= (uint16_t)(1u << (i + cm * rn));
@@ -222,13 +229,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0;
+      const uint64_t pol = sm100::l2_policy_evict_last();
       // slices this CTA loads (and multicasts) of the shared A / B tiles
       const int a_rows = TC_BM / cn, b_rows = BN / cm;       // K-major: rows of the box
       const int a_krows = TC_BK / cn, b_krows = TC_BK / cm;  // MN-major: K rows of each 64-wide box
       for (int ct = cluster_id; ct < num_ct; ct += num_clusters) {
-        const int m0 = ((ct % ncm) * cm + rm) * TC_BM;
-        const int n0 = ((ct / ncm) * cn + rn) * BN;
-        for (int kb = 0; kb < nk; ++kb) {
+        const int ks = ct / num_ct1, c1 = ct % num_ct1;
+        const int m0 = ((c1 % ncm) * cm + rm) * TC_BM;
+        const int n0 = ((c1 / ncm) * cn + rn) * BN;
+        const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
+        for (int kb = kb0; kb < kb1; ++kb) {
           sm100::mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * S::STAGE_BYTES;
           uint8_t* sb = sa + S::A_BYTES;
@@ -243,10 +253,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             }
             if (args.b_mn) {
 #pragma unroll
-              for (int j = 0; j < BN / 64; ++j)
-                sm100::tma_load_3d(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+              for (int j = 0; j < BN / 64; ++j) {
+                if (args.b_keep) sm100::tma_load_3d_hint(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz, pol);
+                else sm100::tma_load_3d(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+              }
             } else {
-              sm100::tma_load_3d(sb, &mapB, &full[s], k0, n0, args.bz);
+              if (args.b_keep) sm100::tma_load_3d_hint(sb, &mapB, &full[s], k0, n0, args.bz, pol);
+              else sm100::tma_load_3d(sb, &mapB, &full[s], k0, n0, args.bz);
             }
           } else {
             if (args.a_mn) {
@@ -257,11 +270,20 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
               sm100::tma_load_3d_mc(sa + rn * a_rows * 128, &mapA, &full[s], k0, m0 + rn * a_rows, args.az, mask_a);
             }
             if (args.b_mn) {
-              for (int j = 0; j < BN / 64; ++j)
-                sm100::tma_load_3d_mc(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
-                                      k0 + rm * b_krows, args.bz, mask_b);
+              for (int j = 0; j < BN / 64; ++j) {
+                if (args.b_keep)
+                  sm100::tma_load_3d_mc_hint(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
+                                             k0 + rm * b_krows, args.bz, mask_b, pol);
+                else
+                  sm100::tma_load_3d_mc(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
+                                        k0 + rm * b_krows, args.bz, mask_b);
+              }
             } else {
-              sm100::tma_load_3d_mc(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz, mask_b);
+              if (args.b_keep)
+                sm100::tma_load_3d_mc_hint(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz,
+                                           mask_b, pol);
+              else
+                sm100::tma_load_3d_mc(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz, mask_b);
             }
           }
           if (++s == stages) { s = 0; ph ^= 1; }
@@ -280,7 +302,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         sm100::mbar_wait(&tempty[acc], (use & 1) ^ 1);
         sm100::tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
-        for (int kb = 0; kb < nk; ++kb) {
+        const int kb0 = (ct / num_ct1) * kper, kb1 = min(nk_all, kb0 + kper);
+        for (int kb = kb0; kb < kb1; ++kb) {
           sm100::mbar_wait(&full[s], ph);
           sm100::tc_fence_after();
           const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
@@ -291,7 +314,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                                           : sm100::smem_desc_sw128(sa + kk * 32, 16, 1024);
             const uint64_t bd = args.b_mn ? sm100::smem_desc_sw128(sb + kk * 2048, 8192, 1024)
                                           : sm100::smem_desc_sw128(sb + kk * 32, 16, 1024);
-            sm100::umma_bf16(d_tmem, ad, bd, args.idesc, (kb | kk) != 0);
+            sm100::umma_bf16(d_tmem, ad, bd, args.idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
           }
           if (cs == 1) sm100::umma_commit(&empty[s]);
           else sm100::umma_commit_mc(&empty[s], mask_nb);
@@ -308,12 +331,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     for (int ct = cluster_id; ct < num_ct; ct += num_clusters, ++local) {
       const int acc = local & 1;
       const uint32_t use = (uint32_t)(local >> 1);
-      const int m0 = ((ct % ncm) * cm + rm) * TC_BM;
-      const int n0 = ((ct / ncm) * cn + rn) * BN;
+      const int ks = ct / num_ct1, c1 = ct % num_ct1;
+      const int m0 = ((c1 % ncm) * cm + rm) * TC_BM;
+      const int n0 = ((c1 / ncm) * cn + rn) * BN;
       sm100::mbar_wait(&tfull[acc], use & 1);
       sm100::tc_fence_after();
       const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * BN;
-      if (m0 < args.M && n0 < args.N) epi.template run<BN>(taddr, m0, n0, row);
+      if (m0 < args.M && n0 < args.N && ks * kper < nk_all) epi.template run<BN>(taddr, m0, n0, row, ks);
       sm100::tc_fence_before();
       sm100::mbar_arrive(&tempty[acc]);
     }

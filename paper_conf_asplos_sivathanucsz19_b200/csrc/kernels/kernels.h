@@ -35,8 +35,9 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
                         const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, OT y_ot,
                         float* hT, float* cT, cudaStream_t st);
 // dy: row stride ldy of type dy_ot (or fp32); dh_rec: [B][ld_dh] fp32 or null (zeros).
+// dh_rec: nsplit fp32 partials (split-K) at stride split_stride elements, summed in order.
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
-                        const float* dh_rec, long ld_dh, float* dc, const float* WX, const float* UH,
+                        const float* dh_rec, long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH,
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
                         float* partials, int nq, bool first, cudaStream_t st);
 int lstm_bwd_row_chunks(int B);

@@ -62,7 +62,7 @@ __global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
   const int b = blockIdx.y;
   if (j >= Hp) return;
   float h = 0.f;
-  if (j < H) h = sigm(__fadd_rn(__fadd_rn(Q[(long)b * ldq + j], Z[(long)b * Hp + j]), bh[j]));
+  if (j < H) h = sigm<FastMath<T>::value>(__fadd_rn(__fadd_rn(Q[(long)b * ldq + j], Z[(long)b * Hp + j]), bh[j]));
   Hf[(long)b * Hp + j] = h;
   HSh[(long)b * ldhs + j] = from_f<T>(h);
   if (j < H) {
@@ -201,7 +201,7 @@ __global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, c
     }
     Z[rz + j] = aH;
     Z[rz + Hp + j] = aT;
-    const float h = tanh_(aH), tau = sigm(aT);
+    const float h = tanh_<FastMath<T>::value>(aH), tau = sigm<FastMath<T>::value>(aT);
     const float s = s_prev[(long)b * Hp + j];
     s_new = __fadd_rn(__fmul_rn(h, tau), __fmul_rn(s, __fsub_rn(1.f, tau)));
     if (y) y[(long)b * ldy + j] = from_f<TY>(s_new);
@@ -243,7 +243,7 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
       if (j < H) {
         float ds = ds_in[(long)b * Hp + j];
         if (dy) ds = __fadd_rn(to_f<TDY>(dy[(long)b * ldy + j]), ds);
-        const float h = tanh_(Apre[rz + j]), tau = sigm(Apre[rz + Hp + j]);
+        const float h = tanh_<FastMath<T>::value>(Apre[rz + j]), tau = sigm<FastMath<T>::value>(Apre[rz + Hp + j]);
         const float sp = s_prev[(long)b * Hp + j];
         const float dh = __fmul_rn(ds, tau);
         const float dtau = __fmul_rn(ds, __fsub_rn(h, sp));

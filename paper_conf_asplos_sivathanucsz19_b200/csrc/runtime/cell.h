@@ -42,6 +42,8 @@ extern const char* const ROLE_NAMES[G_ROLES];
 struct Variant {
   KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
+  int fwd_mode = 0;     // K2 (LSTM family, bf16): 0 GEMM + pointwise kernel, 1 fused per step, 2 fused persistent
+  int bwd_mode = 0;     // K4: same encoding
   Variant() { g[G_BPTT].bn = 128; }
   std::string str() const;                    // "a1=256.1.1,rec=...,wg_side=0"
   static Variant parse(const std::string& s); // inverse of str(); throws ASTRA_E_ARG
@@ -51,6 +53,8 @@ struct Variant {
 struct GemmSpec {
   Mat2 A, B;
   bool a_mn = false, b_mn = false;
+  bool b_keep = false;   // B is a weight re-read every step: keep it in L2 (evict_last)
+  int ksplit = 1;        // fixed split-K (part of the canonical numerics: every variant uses it)
   int M = 0, N = 0, K = 0;
 };
 
@@ -122,6 +126,7 @@ class Cell {
   virtual std::vector<KSeg> y_segments() const = 0;
   virtual int c_width() const { return H; }      // width of the second state (c or s); 0 = none
   virtual bool lm_capable() const { return true; }
+  virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
   // ---- shared machinery
@@ -142,6 +147,7 @@ class Cell {
   template <typename T_> T_* sv(size_t off) { return reinterpret_cast<T_*>(saved + off); }
   template <typename T_> T_* sc(size_t off) { return reinterpret_cast<T_*>(scratch + off); }
   void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st);
+  TcGemm& tc_get(int id, const GemmSpec& s, const KCfg& k);   // prepared tensor maps (bf16 path)
   void mark(Region r, int which, cudaStream_t st);
   void tuner_setup();
   void apply_config(const tuner::Config& c);

@@ -174,6 +174,7 @@ class AttnCell : public Cell {
     rec.A = mat(HC(0), 2L * Hp, B, 2L * Hp, T + 1, (long)B * 2 * Hp);
     rec.B = mat(MUC, 2L * Hp, NG, 2L * Hp);
     rec.M = B; rec.N = NG; rec.K = 2 * Hp;
+    rec.b_keep = true;
     GemmSpec qg;
     qg.A = mat(HC(0), Hp, B, 2L * Hp, T + 1, (long)B * 2 * Hp);
     qg.B = mat(MWq, Hp, Ap, Hp);
@@ -238,6 +239,7 @@ class AttnCell : public Cell {
     bp.B = mat(MUC, ld2, NG, ld2);
     bp.b_mn = true;
     bp.M = B; bp.N = (int)ld2; bp.K = NG;
+    bp.b_keep = true;
     GemmSpec dqw;                      // dh += dq·W_qᵀ
     dqw.A = mat(DQ, Ap, B, Ap, T, (long)B * Ap);
     dqw.B = mat(MWq, Hp, Ap, Hp);
@@ -249,7 +251,7 @@ class AttnCell : public Cell {
                Pr + (long)i * B * Ts, Q + (long)i * B * Ap, Keys, p("v"), Encf, DQ + (size_t)i * B * Ap * e, denc,
                DKf, dvb, i == T - 1, st);
       run_gemm(5, dqw, accum(epi(dHC, ld2, B, Hp)), i, 0, var.g[G_BPTT], st);
-      lstm_bwd_pointwise(K_LSTM, ot, B, H, Hp, (const char*)dy + (size_t)i * B * ldy * e, ldy, ot, false, dHC, ld2,
+      lstm_bwd_pointwise(K_LSTM, ot, B, H, Hp, (const char*)dy + (size_t)i * B * ldy * e, ldy, ot, false, dHC, ld2, 1, 0,
                          dC, WXd + (long)i * B * NG, UHd + (long)i * B * NG, Cd + (long)(i + 1) * B * Hp,
                          Cd + (long)i * B * Hp, gp, DA + (size_t)i * B * NG * e, DA + (size_t)i * B * NG * e, part, 1,
                          i == T - 1, st);

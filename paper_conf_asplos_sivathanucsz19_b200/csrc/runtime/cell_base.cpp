@@ -17,7 +17,7 @@ const char* const ROLE_NAMES[G_ROLES] = {"a1", "rec", "bptt", "du", "dw", "dx", 
 std::string Variant::str() const {
   std::ostringstream o;
   for (int r = 0; r < G_ROLES; ++r) o << ROLE_NAMES[r] << "=" << g[r].bn << "." << g[r].cm << "." << g[r].cn << ",";
-  o << "wg_side=" << wg_side;
+  o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode;
   return o.str();
 }
 
@@ -36,6 +36,13 @@ Variant Variant::parse(const std::string& s) {
     if (k == "wg_side") {
       v.wg_side = std::stoi(val);
       ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    if (k == "fwd" || k == "bwd") {
+      const int mode = std::stoi(val);
+      ASTRA_CHECK_ARG(mode >= 0 && mode <= 2, "variant: fwd/bwd mode must be 0 (unfused), 1 (fused per step) or 2 "
+                                               "(fused persistent)");
+      (k == "fwd" ? v.fwd_mode : v.bwd_mode) = mode;
       continue;
     }
     int r = -1;
@@ -134,23 +141,39 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
   if (which) region_used[r] = true;
 }
 
+TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
+  // split-K only runs without clusters; the cluster choice then falls back to 1x1 (same numerics)
+  const int cm = s.ksplit > 1 ? 1 : k.cm, cn = s.ksplit > 1 ? 1 : k.cn;
+  auto key = std::make_tuple(id, k.bn, cm, cn);
+  auto it = tc_cache.find(key);
+  if (it == tc_cache.end()) {
+    TcGemm g;
+    tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit);
+    it = tc_cache.emplace(key, g).first;
+  }
+  return it->second;
+}
+
 void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st) {
   if (ot == OT::BF16) {
-    auto key = std::make_tuple(id, k.bn, k.cm, k.cn);
-    auto it = tc_cache.find(key);
-    if (it == tc_cache.end()) {
-      TcGemm g;
-      tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, k.cm, k.cn);
-      it = tc_cache.emplace(key, g).first;
-    }
-    tc_gemm_launch(it->second, e, az, bz, st);
+    tc_gemm_launch(tc_get(id, s, k), e, az, bz, st);
   } else {
     const float* A = (const float*)s.A.ptr + (long)az * s.A.zstride;
     const float* Bm = (const float*)s.B.ptr + (long)bz * s.B.zstride;
     long sam, sak, sbk, sbn;
     if (!s.a_mn) { sam = s.A.ld; sak = 1; } else { sam = 1; sak = s.A.ld; }
     if (!s.b_mn) { sbk = 1; sbn = s.B.ld; } else { sbk = s.B.ld; sbn = 1; }
-    simt_gemm(A, sam, sak, Bm, sbk, sbn, s.M, s.N, s.K, e, st);
+    if (s.ksplit <= 1) {
+      simt_gemm(A, sam, sak, Bm, sbk, sbn, s.M, s.N, s.K, e, st);
+    } else {
+      const int kper = cdiv(cdiv(s.K, TC_BK), s.ksplit) * TC_BK;
+      for (int ks = 0; ks < s.ksplit; ++ks) {
+        const int k0 = ks * kper, kn = std::min(s.K - k0, kper);
+        EpiStore ek = e;
+        ek.C = (char*)e.C + (size_t)ks * e.split_stride * 4;
+        if (kn > 0) simt_gemm(A + (long)k0 * sak, sam, sak, Bm + (long)k0 * sbk, sbk, sbn, s.M, s.N, kn, ek, st);
+      }
+    }
   }
 }
 
@@ -218,6 +241,10 @@ void Cell::tuner_setup() {
     }
   }
   std::string t = par.empty() ? "" : "(par" + par + ")";
+  // reading R26: the forward fusion choice (GEMM + pointwise kernel vs the fused recurrent kernel,
+  // P:120-126 "fusion" AV) is tuned after the kernel choices, against the forward-chain time
+  if (ot == OT::BF16 && fwd_fusions() > 1)
+    t = "(pre " + t + " (leaf fuse_fwd " + std::to_string(fwd_fusions()) + " t_fwd))";
   if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
   if (t.empty()) t = "(leaf none 1 t_step)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
@@ -235,6 +262,7 @@ void Cell::apply_config(const tuner::Config& c) {
     const std::string& n = tree->avs[i];
     const int o = c[i];
     if (n == "wg_side") { v.wg_side = o; continue; }
+    if (n == "fuse_fwd") { v.fwd_mode = o; continue; }
     for (int r = 0; r < G_ROLES; ++r)
       if (n == std::string("g_") + ROLE_NAMES[r]) v.g[r] = allowed[r].at(o);
   }

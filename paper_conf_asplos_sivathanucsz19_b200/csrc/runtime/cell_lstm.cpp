@@ -8,6 +8,7 @@
 //         → dh0 → wgrad dU = Hᵀ·D_uh, dW = Xᵀ·D_wx (K1) → dX = D_wx·Wᵀ (K1) → bias/α/β reductions (K5)
 //         → gradient sum over ranks (K11) when world > 1.
 #include "../kernels/cell_math.cuh"
+#include "../kernels/rec_fused.h"
 #include "cell.h"
 
 namespace astra {
@@ -16,7 +17,7 @@ class LstmCell : public Cell {
  public:
   int kind, NG, nchunk;
   size_t off_X, off_WX, off_UH, off_C, off_H, off_Wm, off_Um;
-  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part;
+  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part, off_flags;
 
   explicit LstmCell(const astra_cell_desc& dd) : Cell(dd) {
     kind = d.cell_type == ASTRA_MILSTM ? K_MILSTM : d.cell_type == ASTRA_SUBLSTM ? K_SUBLSTM : K_LSTM;
@@ -45,11 +46,19 @@ class LstmCell : public Cell {
     Carve c;
     off_Duh = c.take(TB * NG * e);
     off_Dwx = kind == K_MILSTM ? c.take(TB * NG * e) : off_Duh;
-    off_dH = c.take((size_t)B * Hp * 4);
+    off_dH = c.take((size_t)bptt_ksplit() * B * Hp * 4);
     off_dC = c.take((size_t)B * Hp * 4);
     off_part = c.take((size_t)nchunk * 4 * NG * 4);
+    off_flags = c.take(4096);
     scratch_bytes = c.o;
   }
+
+  // Fixed split-K of the per-step BPTT GEMM (K = 4·Hp): with B rows the GEMM has few output tiles,
+  // so each SM would stream a whole K-panel of Uᵀ; four K-chunks cut the bytes per SM 4× while the
+  // chunk partials are summed in a fixed order by the pointwise kernel (identical for every variant).
+  int bptt_ksplit() const { return (ot == OT::BF16 && NG >= 8192) ? 4 : (ot == OT::BF16 && NG >= 4096) ? 2 : 1; }
+
+  int fwd_fusions() const override { return 3; }
 
   void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
   void* x_operand() override { return sv<char>(off_X); }
@@ -112,18 +121,46 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   rec.A = mat(Hrow(0), Hp, B, Hp, T + 1, (long)B * Hp);
   rec.B = mat(Um, Hp, NG, Hp);
   rec.M = B; rec.N = NG; rec.K = Hp;
-  for (int t = 0; t < T; ++t) {
-    float* UHt = UH + (long)t * B * NG;
-    run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st);
-    const bool last = t == T - 1;
-    if (y_f32)   // internal fp32 output (e.g. the encoder of LSTM-attention), row stride Hp
-      lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
-                         Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y_f32 + (size_t)t * B * Hp, Hp, OT::F32,
-                         last ? hT : nullptr, last ? cT : nullptr, st);
-    else
-      lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
-                         Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y ? (char*)y + (size_t)t * B * H * e : nullptr,
-                         H, ot, last ? hT : nullptr, last ? cT : nullptr, st);
+  rec.b_keep = true;
+  if (ot == OT::BF16 && var.fwd_mode > 0) {
+    // K2 fused: GEMM + gate epilogue in one kernel (per step, or persistent over all steps)
+    const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1});
+    RecFwdArgs ra;
+    ra.B = B; ra.H = H; ra.Hp = Hp; ra.NG = NG; ra.T = T;
+    ra.num_m = cdiv(B, TC_BM); ra.num_n = NG / 256;
+    ra.idesc = tg.args.idesc;
+    ra.WX = WX; ra.UH = UH; ra.C = Cb; ra.Hb = (__nv_bfloat16*)Hrow(0);
+    if (y_f32) { ra.y = y_f32; ra.ldy = Hp; ra.y_kind = 2; }
+    else if (y) { ra.y = y; ra.ldy = H; ra.y_kind = 1; }
+    else { ra.y = nullptr; ra.ldy = 0; ra.y_kind = 0; }
+    ra.hT = hT; ra.cT = cT; ra.gp = gp;
+    ra.flags = sc<unsigned>(off_flags);
+    const bool persistent = var.fwd_mode == 2 && ra.num_m * ra.num_n <= num_sms() && ra.num_m <= 1024;
+    if (persistent) {
+      CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
+      ra.persistent = 1; ra.t0 = 0; ra.t1 = T;
+      lstm_rec_fwd_launch(kind, tg.mapA, tg.mapB, ra, st);
+    } else {
+      ra.persistent = 0;
+      for (int t = 0; t < T; ++t) {
+        ra.t0 = t; ra.t1 = t + 1;
+        lstm_rec_fwd_launch(kind, tg.mapA, tg.mapB, ra, st);
+      }
+    }
+  } else {
+    for (int t = 0; t < T; ++t) {
+      float* UHt = UH + (long)t * B * NG;
+      run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st);
+      const bool last = t == T - 1;
+      if (y_f32)   // internal fp32 output (e.g. the encoder of LSTM-attention), row stride Hp
+        lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
+                           Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y_f32 + (size_t)t * B * Hp, Hp, OT::F32,
+                           last ? hT : nullptr, last ? cT : nullptr, st);
+      else
+        lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
+                           Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y ? (char*)y + (size_t)t * B * H * e : nullptr,
+                           H, ot, last ? hT : nullptr, last ? cT : nullptr, st);
+    }
   }
   mark(R_FWD, 1, st);
   fwd_done = true;
@@ -161,27 +198,34 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   bp.B = mat(Um, Hp, NG, Hp);
   bp.b_mn = true;
   bp.M = B; bp.N = Hp; bp.K = NG;
+  bp.b_keep = true;
+  GemmSpec bp0 = bp;   // dh0 (once, no split)
+  bp.ksplit = bptt_ksplit();
   for (int t = T - 1; t >= 0; --t) {
     const float* dh_rec;
     long ld_dh;
+    int nsplit = 1;
     if (t == T - 1) {
       dh_rec = dhT;
       ld_dh = H;
     } else {
-      run_gemm(2, bp, epi(dH, Hp, B, Hp), t + 1, 0, var.g[G_BPTT], st);
+      EpiStore e = epi(dH, Hp, B, Hp);
+      e.split_stride = (long)B * Hp;
+      run_gemm(2, bp, e, t + 1, 0, var.g[G_BPTT], st);
       dh_rec = dH;
       ld_dh = Hp;
+      nsplit = bp.ksplit;
     }
     const void* dyt;
     long ldy;
     bool dyf32;
     if (lm_dy) { dyt = lm_dy + (long)t * B * Hp; ldy = Hp; dyf32 = true; }
     else { dyt = (const char*)dy + (size_t)t * B * H * e; ldy = H; dyf32 = false; }
-    lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, dC, WX + (long)t * B * NG,
+    lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC, WX + (long)t * B * NG,
                        UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
                        Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
   }
-  if (dh0) run_gemm(2, bp, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
+  if (dh0) run_gemm(3, bp0, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
   if (dc0) copy_pad(OT::F32, dC, OT::F32, B, H, Hp, dc0, H, st);
   mark(R_BPTT, 1, st);
 

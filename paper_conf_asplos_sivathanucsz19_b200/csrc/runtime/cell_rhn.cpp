@@ -101,6 +101,7 @@ class RhnCell : public Cell {
     rec.A = mat(Sop(0, 0), Hp, B, Hp, (long)L * (T + 1), (long)B * Hp);
     rec.B = mat(MR, Hp, G2, Hp, L, (long)G2 * Hp);
     rec.M = B; rec.N = G2; rec.K = Hp;
+    rec.b_keep = true;
     for (int t = 0; t < T; ++t) {
       for (int l = 0; l < L; ++l) {
         float* Z = Apre(l, t);
@@ -137,6 +138,7 @@ class RhnCell : public Cell {
     bp.B = mat(MR, Hp, G2, Hp, L, (long)G2 * Hp);
     bp.b_mn = true;
     bp.M = B; bp.N = Hp; bp.K = G2;
+    bp.b_keep = true;
     for (int t = T - 1; t >= 0; --t) {
       for (int l = L - 1; l >= 0; --l) {
         const void* dyt = nullptr;

@@ -127,6 +127,7 @@ class ScrnCell : public Cell {
     rec.A = mat(HSrow(0), Hp, B, Yw, T + 1, (long)B * Yw);
     rec.B = mat(MR, Hp, Hp, Hp);
     rec.M = B; rec.N = Hp; rec.K = Hp;
+    rec.b_keep = true;
     for (int t = 0; t < T; ++t) {
       run_gemm(2, rec, epi(Z, Hp, B, Hp), t, 0, var.g[G_REC], st);
       scrn_fwd_pw(ot, B, H, Hp, XAB + (long)t * B * Yw, Yw, Z, p("b_h"), Hf + (long)(t + 1) * B * Hp, HSrow(t + 1),
@@ -160,6 +161,7 @@ class ScrnCell : public Cell {
     bp.B = mat(MR, Hp, Hp, Hp);
     bp.b_mn = true;
     bp.M = B; bp.N = Hp; bp.K = Hp;
+    bp.b_keep = true;
     for (int t = T - 1; t >= 0; --t) {
       const float* dh = dhT;
       long ld_dh = H;

@@ -16,7 +16,7 @@ pytestmark = pytest.mark.gpu
 ALPHA = 0.95
 
 
-def _check(cell, T, B, I, H, dtype, seed, tol, variant=None, S=None, L=None):
+def _check(cell, T, B, I, H, dtype, seed, tol, variant=None, S=None, L=None):  # noqa: C901
     p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, seed, bf16=(dtype == "bf16"), S=S, L=L)
     kw, okw = {}, {}
     if cell == "scrn":
@@ -64,14 +64,21 @@ def test_bf16_cfg5_reduced():
     _check("milstm", 8, 64, 2048, 2048, "bf16", synth.config_seed(5), TOL_BF16)
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+@pytest.mark.parametrize("fwd", [0, 1, 2])
+def test_fused_forward_modes(cell, fwd):
+    """K2 unfused / fused-per-step / fused-persistent against the oracle, several row blocks."""
+    _check(cell, 6, 260, 64, 192, "bf16", synth.config_seed(5) + 40, TOL_BF16, variant=f"fwd={fwd}")
+
+
 def test_variants_bitwise():
     """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
     T, B, I, H = 6, 160, 128, 192
     p, inp, dY, dhT, dcT = make_cell_case("milstm", T, B, I, H, 77, bf16=True)
-    variants = ["a1=256,rec=256,bptt=128,du=256,dw=256,dx=256,wg_side=0",
-                "a1=128.2.2,rec=128.2.1,bptt=64.2.1,du=128.1.2,dw=128,dx=128.4.1,wg_side=1",
-                "a1=64.4.1,rec=64,bptt=256.1.1,du=64.2.2,dw=64.2.1,dx=64.2.2,wg_side=0",
-                "a1=256.2.2,rec=256.2.1,bptt=128.2.1,du=256.2.2,dw=256.1.2,dx=256.4.1,wg_side=1"]
+    variants = ["a1=256,rec=256,bptt=128,du=256,dw=256,dx=256,wg_side=0,fwd=0",
+                "a1=128.2.2,rec=128.2.1,bptt=64.2.1,du=128.1.2,dw=128,dx=128.4.1,wg_side=1,fwd=0",
+                "a1=64.4.1,rec=64,bptt=256.1.1,du=64.2.2,dw=64.2.1,dx=64.2.2,wg_side=0,fwd=1",
+                "a1=256.2.2,rec=256.2.1,bptt=128.2.1,du=256.2.2,dw=256.1.2,dx=256.4.1,wg_side=1,fwd=2"]
     ref = None
     for v in variants:
         out, g, _ = run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", v)

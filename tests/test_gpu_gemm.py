@@ -72,3 +72,35 @@ def test_paper_table1_shapes():
         torch.cuda.synchronize()
         # fp32 accumulation of exact bf16 products: error ~ sqrt(K)·2^-24·|terms|
         assert (out.double().cpu() - ref).abs().max().item() <= 2e-6 * K ** 0.5 * ref.abs().max().item()
+
+
+@pytest.mark.parametrize("ksplit", [2, 3, 4])
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 1), (0, 0)])
+def test_split_k_partials(ksplit, a_mn, b_mn):
+    """Fixed split-K (the BPTT GEMM's numerics, R25): partial s equals the fp64 product over its own
+    K chunk (chunk = ceil(ceil(K/64)/ksplit)·64 elements, ragged last chunk), every tile width gives
+    the same bits, and the partials summed in chunk order match the full product."""
+    M, N, K = 200, 320, 64 * 9 + 40
+    A_s, B_s, _ = _operands(M, N, K, a_mn, b_mn, seed=ksplit)
+    g = torch.Generator().manual_seed(ksplit)
+    a = torch.randn(M, K, generator=g).to(torch.bfloat16).double()
+    b = torch.randn(K, N, generator=g).to(torch.bfloat16).double()
+    kper = -(-(-(-K // 64)) // ksplit) * 64
+    outs = []
+    for bn in (64, 128, 256):
+        out = A.gemm_bf16_splitk(A_s, B_s, M, N, K, ksplit, a_mn=a_mn, b_mn=b_mn, bn=bn)
+        torch.cuda.synchronize()
+        outs.append(out.cpu())
+    for o in outs[1:]:
+        assert torch.equal(o, outs[0])
+    o = outs[0].double()
+    for s in range(ksplit):
+        k0, k1 = s * kper, min(K, (s + 1) * kper)
+        ref = a[:, k0:k1] @ b[k0:k1] if k1 > k0 else torch.zeros(M, N, dtype=torch.float64)
+        err = (o[s] - ref).abs().max().item()
+        assert err <= 1e-5 * max(1.0, ref.abs().max().item()) * max(1, (k1 - k0) / 64) + 1e-6, (s, err)
+    full = a @ b
+    tot = o[0].clone()
+    for s in range(1, ksplit):
+        tot = tot + o[s]
+    assert (tot - full).abs().max().item() <= 1e-5 * full.abs().max().item() * K / 64
