@@ -172,13 +172,17 @@ astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev
  * depend on them (bitwise).                                                                 */
 astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long lda, const void* B, int b_mn,
                              long ldb, float* C, long ldc, int bn, int cm, int cn, astra_stream stream);
-/* Fixed split-K form (the BPTT GEMM's canonical numerics): K is cut into ksplit chunks of
- * ceil(ceil(K/64)/ksplit)·64 elements; chunk s writes its fp32 partial Σ_{k in chunk s} A·B to
- * C + s·M·ldc (C holds ksplit·M rows of ldc floats; a chunk past K writes nothing).  The caller
- * sums the partials in chunk order.  ksplit ∈ [1, 16]; ksplit > 1 requires cm = cn = 1.       */
-astra_status astra_gemm_bf16_splitk(int M, int N, int K, const void* A, int a_mn, long lda, const void* B, int b_mn,
-                                    long ldb, float* C, long ldc, int bn, int cm, int cn, int ksplit,
-                                    astra_stream stream);
+/* Extended form.  cta_group = 2 runs the CTA-pair kernel: two CTAs of a cluster share one
+ * 256 x bn tile (each holds half of A's rows and half of B's columns in shared memory; requires
+ * bn ∈ {128, 256} and cm = cn = 1); the result is bitwise identical to cta_group = 1.
+ * ksplit > 1 is the fixed split-K form (the BPTT GEMM's canonical numerics): K is cut into
+ * ksplit chunks of ceil(ceil(K/64)/ksplit)·64 elements; chunk s writes its fp32 partial
+ * Σ_{k in chunk s} A·B to C + s·M·ldc (C holds ksplit·M rows of ldc floats; a chunk past K writes
+ * nothing) and the caller sums the partials in chunk order.  ksplit ∈ [1, 16]; ksplit > 1
+ * requires cm = cn = 1.                                                                      */
+astra_status astra_gemm_bf16_ex(int M, int N, int K, const void* A, int a_mn, long lda, const void* B, int b_mn,
+                                long ldb, float* C, long ldc, int bn, int cm, int cn, int cta_group, int ksplit,
+                                astra_stream stream);
 
 /* ---- diagnostics ----------------------------------------------------------------------- */
 const char* astra_status_string(astra_status s);

@@ -69,8 +69,8 @@ _SIGS = {
     "astra_lm_train_step": [_P, _P, _F, _P],
     "astra_lm_fwd_bwd": [_P, _P, _P],
     "astra_gemm_bf16": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I, _P],
-    "astra_gemm_bf16_splitk": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I,
-                               _I, _P],
+    "astra_gemm_bf16_ex": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I,
+                           _I, _I, _P],
     "astra_status_string": [_I],
     "astra_last_error": [],
     "astra_kernel_launch_count": [],
@@ -127,13 +127,14 @@ def gemm_bf16(A, B, M, N, K, a_mn=False, b_mn=False, bn=256, cm=1, cn=1, out=Non
     return out
 
 
-def gemm_bf16_splitk(A, B, M, N, K, ksplit, a_mn=False, b_mn=False, bn=256, out=None):
-    """Split-K K1: out[ksplit, M, N] fp32 partials (see astra_gemm_bf16_splitk)."""
+def gemm_bf16_ex(A, B, M, N, K, a_mn=False, b_mn=False, bn=256, cm=1, cn=1, cta_group=1, ksplit=1, out=None):
+    """Extended K1 (see astra_gemm_bf16_ex): CTA pairs and fixed split-K.  Returns out[ksplit, M, N]
+    fp32 partials (out[0] is the product when ksplit = 1)."""
     import torch
     if out is None:
         out = torch.zeros(ksplit, M, N, dtype=torch.float32, device=A.device)
-    _check(lib().astra_gemm_bf16_splitk(M, N, K, _ptr(A), int(a_mn), A.stride(0), _ptr(B), int(b_mn), B.stride(0),
-                                        _ptr(out), out.stride(1), bn, 1, 1, ksplit, _stream()))
+    _check(lib().astra_gemm_bf16_ex(M, N, K, _ptr(A), int(a_mn), A.stride(0), _ptr(B), int(b_mn), B.stride(0),
+                                    _ptr(out), out.stride(1), bn, cm, cn, cta_group, ksplit, _stream()))
     return out
 
 

@@ -258,14 +258,15 @@ astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev
   return guard([&] { NEED(m); m->m->step(tokens, 0.f, loss_dev, false); });
 }
 
-astra_status astra_gemm_bf16_splitk(int M, int N, int K, const void* A, int a_mn, long lda, const void* Bp, int b_mn,
-                                    long ldb, float* C, long ldc, int bn, int cm, int cn, int ksplit,
-                                    astra_stream stream) {
+astra_status astra_gemm_bf16_ex(int M, int N, int K, const void* A, int a_mn, long lda, const void* Bp, int b_mn,
+                                long ldb, float* C, long ldc, int bn, int cm, int cn, int cta_group, int ksplit,
+                                astra_stream stream) {
   return guard([&] {
     NEED(A); NEED(Bp); NEED(C);
     ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "gemm: sizes must be positive");
     ASTRA_CHECK_ARG(ldc >= N, "gemm: ldc < N");
     ASTRA_CHECK_ARG(ksplit >= 1 && ksplit <= 16, "gemm: ksplit must be in [1, 16]");
+    ASTRA_CHECK_ARG(cta_group == 1 || cta_group == 2, "gemm: cta_group must be 1 or 2");
     Mat2 a, b;
     a.ptr = A; a.ld = lda;
     if (a_mn) { a.inner = M; a.outer = K; } else { a.inner = K; a.outer = M; }
@@ -273,7 +274,7 @@ astra_status astra_gemm_bf16_splitk(int M, int N, int K, const void* A, int a_mn
     if (b_mn) { b.inner = N; b.outer = K; } else { b.inner = K; b.outer = N; }
     ASTRA_CHECK_ARG(lda >= a.inner && ldb >= b.inner, "gemm: leading dimension too small");
     TcGemm g;
-    tc_gemm_prepare(g, a, a_mn != 0, b, b_mn != 0, M, N, K, bn, cm, cn, false, ksplit);
+    tc_gemm_prepare(g, a, a_mn != 0, b, b_mn != 0, M, N, K, bn, cm, cn, false, ksplit, cta_group);
     EpiStore e = epi(C, ldc, M, N);
     e.split_stride = (long)M * ldc;
     tc_gemm_launch(g, e, 0, 0, (cudaStream_t)stream);
@@ -282,7 +283,7 @@ astra_status astra_gemm_bf16_splitk(int M, int N, int K, const void* A, int a_mn
 
 astra_status astra_gemm_bf16(int M, int N, int K, const void* A, int a_mn, long lda, const void* Bp, int b_mn,
                              long ldb, float* C, long ldc, int bn, int cm, int cn, astra_stream stream) {
-  return astra_gemm_bf16_splitk(M, N, K, A, a_mn, lda, Bp, b_mn, ldb, C, ldc, bn, cm, cn, 1, stream);
+  return astra_gemm_bf16_ex(M, N, K, A, a_mn, lda, Bp, b_mn, ldb, C, ldc, bn, cm, cn, 1, 1, stream);
 }
 
 const char* astra_status_string(astra_status s) {

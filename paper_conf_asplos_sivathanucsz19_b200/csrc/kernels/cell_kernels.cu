@@ -108,43 +108,87 @@ void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, l
 }
 
 // ============================================================================ LSTM-family pointwise
+// K2 forward half.  Thread = 4 consecutive hidden units of one batch row: they share one 64-unit
+// gate group of the interleaved layout, so each gate's WX/UH pre-activations are one 16-byte load.
+constexpr int FWD_U = 4;
+template <typename T>
+__device__ __forceinline__ void store4(T* p, const float (&v)[4]);
+template <>
+__device__ __forceinline__ void store4<float>(float* p, const float (&v)[4]) {
+  *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+}
+template <>
+__device__ __forceinline__ void store4<__nv_bfloat16>(__nv_bfloat16* p, const float (&v)[4]) {
+  __nv_bfloat162 lo = __floats2bfloat162_rn(v[0], v[1]), hi = __floats2bfloat162_rn(v[2], v[3]);
+  uint2 u;
+  u.x = *reinterpret_cast<uint32_t*>(&lo);
+  u.y = *reinterpret_cast<uint32_t*>(&hi);
+  *reinterpret_cast<uint2*>(p) = u;
+}
+
 template <int KIND, typename T, typename TY>
-__global__ void lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ WX, const float* __restrict__ UH,
-                                   GateParams gp, const float* __restrict__ c_prev, float* __restrict__ c_new,
-                                   T* __restrict__ h_op, long ldh, TY* __restrict__ y, long ldy,
-                                   float* __restrict__ hT, float* __restrict__ cT) {
-  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+__global__ void __launch_bounds__(128)
+    lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ WX, const float* __restrict__ UH,
+                       GateParams gp, const float* __restrict__ c_prev, float* __restrict__ c_new,
+                       T* __restrict__ h_op, long ldh, TY* __restrict__ y, long ldy, float* __restrict__ hT,
+                       float* __restrict__ cT) {
+  const int j0 = (blockIdx.x * blockDim.x + threadIdx.x) * FWD_U;
   const int b = blockIdx.y;
-  if (j >= Hp) return;
+  if (j0 >= Hp) return;
   const long rowg = (long)b * 4 * Hp, rowh = (long)b * Hp;
-  if (j >= H) {  // keep padding units exactly zero
-    c_new[rowh + j] = 0.f;
-    h_op[(long)b * ldh + j] = from_f<T>(0.f);
-    if (y && ldy >= Hp) y[(long)b * ldy + j] = from_f<TY>(0.f);
-    return;
-  }
-  float a[4];
+  float4 wx[4], uh[4];
 #pragma unroll
   for (int g = 0; g < 4; ++g) {
-    const int col = gcol(g, j), e = g * H + j;
-    const float wx = __ldcs(WX + rowg + col), uh = __ldcs(UH + rowg + col);
-    a[g] = preact<KIND>(wx, uh, gp.b[e], KIND == K_MILSTM ? gp.alpha[e] : 0.f, KIND == K_MILSTM ? gp.beta1[e] : 0.f,
-                        KIND == K_MILSTM ? gp.beta2[e] : 0.f);
+    wx[g] = __ldcs(reinterpret_cast<const float4*>(WX + rowg + gcol(g, j0)));
+    uh[g] = __ldcs(reinterpret_cast<const float4*>(UH + rowg + gcol(g, j0)));
   }
-  float c, h;
-  cell_fwd<KIND, FastMath<T>::value>(a, c_prev[rowh + j], c, h);
-  c_new[rowh + j] = c;
-  h_op[(long)b * ldh + j] = from_f<T>(h);
-  if (y) y[(long)b * ldy + j] = from_f<TY>(h);
-  if (hT) hT[(long)b * H + j] = h;
-  if (cT) cT[(long)b * H + j] = c;
+  const float4 cp4 = *reinterpret_cast<const float4*>(c_prev + rowh + j0);
+  const float cp[4] = {cp4.x, cp4.y, cp4.z, cp4.w};
+  float cv[4], hv[4];
+#pragma unroll
+  for (int u = 0; u < FWD_U; ++u) {
+    const int j = j0 + u;
+    if (j < H) {   // padding units (H ≤ j < Hp) stay exactly zero
+      float a[4];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        const float w = u == 0 ? wx[g].x : u == 1 ? wx[g].y : u == 2 ? wx[g].z : wx[g].w;
+        const float h = u == 0 ? uh[g].x : u == 1 ? uh[g].y : u == 2 ? uh[g].z : uh[g].w;
+        const int e = g * H + j;
+        a[g] = preact<KIND>(w, h, gp.b[e], KIND == K_MILSTM ? gp.alpha[e] : 0.f,
+                            KIND == K_MILSTM ? gp.beta1[e] : 0.f, KIND == K_MILSTM ? gp.beta2[e] : 0.f);
+      }
+      cell_fwd<KIND, FastMath<T>::value>(a, cp[u], cv[u], hv[u]);
+    } else {
+      cv[u] = 0.f;
+      hv[u] = 0.f;
+    }
+  }
+  store4<float>(c_new + rowh + j0, cv);
+  if ((ldh & 3) == 0) store4<T>(h_op + (long)b * ldh + j0, hv);
+  else
+#pragma unroll
+    for (int u = 0; u < FWD_U; ++u) h_op[(long)b * ldh + j0 + u] = from_f<T>(hv[u]);
+  if (y) {
+    if ((ldy & 3) == 0 && (j0 + FWD_U <= H || ldy >= Hp)) store4<TY>(y + (long)b * ldy + j0, hv);
+    else
+#pragma unroll
+      for (int u = 0; u < FWD_U; ++u)
+        if (j0 + u < H || ldy >= Hp) y[(long)b * ldy + j0 + u] = from_f<TY>(hv[u]);
+  }
+#pragma unroll
+  for (int u = 0; u < FWD_U; ++u) {
+    if (j0 + u >= H) break;
+    if (hT) hT[(long)b * H + j0 + u] = hv[u];
+    if (cT) cT[(long)b * H + j0 + u] = cv[u];
+  }
 }
 
 template <int KIND, typename T>
 static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
                           const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, float* hT,
                           float* cT, cudaStream_t st) {
-  dim3 grid(cdiv(Hp, 128), B);
+  dim3 grid(cdiv(Hp, 128 * FWD_U), B);
   if (y_ot == OT::BF16)
     lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
                                                                      ldh, (__nv_bfloat16*)y, ldy, hT, cT);
@@ -172,97 +216,172 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
   throw Error(ASTRA_E_UNSUPPORTED, "lstm_fwd_pointwise: kind");
 }
 
-constexpr int BWD_RB = 32;  // rows per CTA in the backward pointwise kernel
-constexpr int BWD_UX = 64;  // units per CTA (threadIdx.x)
+constexpr int BWD_RB = 32;  // rows per CTA in the backward pointwise kernel (= one partial chunk)
+constexpr int BWD_UX = 64;  // units per CTA (one gate group)
+constexpr int BWD_TX = 32;  // threads along units: thread tx owns units 2tx, 2tx+1 of the group
 constexpr int BWD_RY = 8;   // row lanes per CTA (threadIdx.y); thread handles rows b0 + ty + 8i
 int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 
-// CTA = 64 hidden units (all four gates) x 32 batch rows; thread (ux, ty) handles unit u0 + ux for
-// rows b0 + ty, b0 + ty + 8, ...  Column partial sums (db, dα, dβ1, dβ2) are accumulated per thread
-// in ascending row order, combined across the 8 row lanes in ty order through shared memory, and
-// added to partials[chunk][q][col] — one owner per element, steps ordered on the stream, so the
-// reduction order is fixed (R5: no floating-point atomics).
+template <typename T>
+__device__ __forceinline__ void store2cs(T* p, float a, float b);
+template <>
+__device__ __forceinline__ void store2cs<float>(float* p, float a, float b) {
+  __stcs(reinterpret_cast<float2*>(p), make_float2(a, b));
+}
+template <>
+__device__ __forceinline__ void store2cs<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
+  __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
+  __stcs(reinterpret_cast<unsigned int*>(p), *reinterpret_cast<unsigned int*>(&v));
+}
+template <typename T>
+__device__ __forceinline__ void store2(T* p, float a, float b);
+template <>
+__device__ __forceinline__ void store2<float>(float* p, float a, float b) {
+  *reinterpret_cast<float2*>(p) = make_float2(a, b);
+}
+template <>
+__device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
+  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);
+}
+
+// K4 backward half + K5 column partials.  CTA = 64 hidden units (all four gates) x 32 batch rows;
+// thread (tx, ty) handles units 2tx, 2tx+1 (8-byte loads of every gate's pre-activations) for rows
+// b0 + ty, b0 + ty + 8, ...  Column partial sums (db, dα, dβ1, dβ2) are accumulated per (thread,
+// unit) in thread-private shared-memory slots in ascending row order, combined across the 8 row
+// lanes in ty order, and added to partials[chunk][q][col] — one owner per element, steps ordered on
+// the stream, so the reduction order is fixed (R5: no floating-point atomics).  256-thread CTAs
+// with shared-memory accumulators keep the register count low enough that the whole grid of a
+// 512-row batch is resident in one wave.
 template <int KIND, typename T, typename TDY>
-__global__ void __launch_bounds__(BWD_UX * BWD_RY, 2)
+__global__ void __launch_bounds__(BWD_TX * BWD_RY, 4)
     lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
-                       long ld_dh, int nsplit, long split_stride, float* __restrict__ dc, const float* __restrict__ WX, const float* __restrict__ UH,
-                       const float* __restrict__ c_new, const float* __restrict__ c_prev, GateParams gp,
-                       T* __restrict__ D_uh, T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
-  __shared__ float red[BWD_RY][16][BWD_UX];
-  const int ux = threadIdx.x, ty = threadIdx.y;
-  const int j = blockIdx.x * BWD_UX + ux;
+                       long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
+                       const float* __restrict__ WX, const float* __restrict__ UH, const float* __restrict__ c_new,
+                       const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
+                       T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
+  constexpr int NV = KIND == K_MILSTM ? 16 : 4;   // accumulated quantities per unit: q*4 + gate
+  __shared__ float red[BWD_RY][NV][2][BWD_TX];     // [row lane][quantity][unit parity][tx]
+  __shared__ float prm[KIND == K_MILSTM ? 4 : 1][4][BWD_UX];
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * BWD_TX + tx;
+  const int u0 = blockIdx.x * BWD_UX;
+  const int j0 = u0 + 2 * tx;
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
-  float s[16];
-#pragma unroll
-  for (int i = 0; i < 16; ++i) s[i] = 0.f;
-  if (j < H) {
-    float al[4], be1[4], be2[4], bb[4];
-#pragma unroll
-    for (int g = 0; g < 4; ++g) {
-      const int e = g * H + j;
-      bb[g] = gp.b[e];
-      al[g] = KIND == K_MILSTM ? gp.alpha[e] : 0.f;
-      be1[g] = KIND == K_MILSTM ? gp.beta1[e] : 0.f;
-      be2[g] = KIND == K_MILSTM ? gp.beta2[e] : 0.f;
-    }
-    for (int b = b0 + ty; b < b1; b += BWD_RY) {
-      const long rg = (long)b * NG;
-      float wx[4], uh[4], a[4];
-#pragma unroll
-      for (int g = 0; g < 4; ++g) {
-        wx[g] = __ldcs(WX + rg + gcol(g, j));
-        uh[g] = __ldcs(UH + rg + gcol(g, j));
-        a[g] = preact<KIND>(wx[g], uh[g], bb[g], al[g], be1[g], be2[g]);
-      }
-      float dh = to_f<TDY>(dy[(long)b * ldy + j]);
-      if (dh_rec) {   // split-K partials of dh_rec summed in chunk order, then added to dy
-        float r = dh_rec[(long)b * ld_dh + j];
-        for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, dh_rec[k * split_stride + (long)b * ld_dh + j]);
-        dh = __fadd_rn(dh, r);
-      }
-      float dcv = dc[(long)b * Hp + j];
-      float da[4];
-      cell_bwd<KIND, FastMath<T>::value>(a, c_prev[(long)b * Hp + j], c_new[(long)b * Hp + j], dh, dcv, da);
-      dc[(long)b * Hp + j] = dcv;
-#pragma unroll
-      for (int g = 0; g < 4; ++g) {
-        s[g] = __fadd_rn(s[g], da[g]);
-        if (KIND == K_MILSTM) {
-          const float duh = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], wx[g]), be1[g]));
-          const float dwx = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], uh[g]), be2[g]));
-          D_uh[rg + gcol(g, j)] = from_f<T>(duh);
-          __stcs(D_wx + rg + gcol(g, j), from_f<T>(dwx));
-          s[4 + g] = __fadd_rn(s[4 + g], __fmul_rn(__fmul_rn(da[g], wx[g]), uh[g]));
-          s[8 + g] = __fadd_rn(s[8 + g], __fmul_rn(da[g], uh[g]));
-          s[12 + g] = __fadd_rn(s[12 + g], __fmul_rn(da[g], wx[g]));
-        } else {
-          D_uh[rg + gcol(g, j)] = from_f<T>(da[g]);
-        }
-      }
-    }
-  } else if (j < Hp) {  // padding units: keep their gradients exactly zero
-    for (int b = b0 + ty; b < b1; b += BWD_RY) {
-#pragma unroll
-      for (int g = 0; g < 4; ++g) {
-        D_uh[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
-        if (KIND == K_MILSTM) D_wx[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
-      }
-      dc[(long)b * Hp + j] = 0.f;
+  for (int i = tid; i < 4 * BWD_UX; i += BWD_TX * BWD_RY) {
+    const int g = i / BWD_UX, ul = i % BWD_UX, j = u0 + ul, e = g * H + j;
+    const bool v = j < H;
+    prm[0][g][ul] = v ? gp.b[e] : 0.f;
+    if (KIND == K_MILSTM) {
+      prm[KIND == K_MILSTM ? 1 : 0][g][ul] = v ? gp.alpha[e] : 0.f;
+      prm[KIND == K_MILSTM ? 2 : 0][g][ul] = v ? gp.beta1[e] : 0.f;
+      prm[KIND == K_MILSTM ? 3 : 0][g][ul] = v ? gp.beta2[e] : 0.f;
     }
   }
-  const int nv = KIND == K_MILSTM ? 16 : 4;
-  for (int i = 0; i < nv; ++i) red[ty][i][ux] = s[i];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    red[ty][i][0][tx] = 0.f;
+    red[ty][i][1][tx] = 0.f;
+  }
   __syncthreads();
-  if (j >= Hp) return;
-  // thread (ux, ty) finalises quantities i = ty, ty + 8 (fixed ty order inside)
-  for (int i = ty; i < nv; i += BWD_RY) {
+  if (j0 < Hp) {
+    const bool v0 = j0 < H, v1 = j0 + 1 < H;
+    const bool vec_dh = ((ld_dh | split_stride) & 1) == 0;
+    for (int b = b0 + ty; b < b1; b += BWD_RY) {
+      const long rg = (long)b * NG;
+      float2 wx[4], uh[4];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        wx[g] = __ldcs(reinterpret_cast<const float2*>(WX + rg + gcol(g, j0)));
+        uh[g] = __ldcs(reinterpret_cast<const float2*>(UH + rg + gcol(g, j0)));
+      }
+      float dh[2] = {v0 ? to_f<TDY>(dy[(long)b * ldy + j0]) : 0.f, v1 ? to_f<TDY>(dy[(long)b * ldy + j0 + 1]) : 0.f};
+      if (dh_rec && v0) {   // split-K partials of dh_rec summed in chunk order, then added to dy
+        const float* r0 = dh_rec + (long)b * ld_dh + j0;
+        float r[2];
+        if (vec_dh) {
+          float2 q = *reinterpret_cast<const float2*>(r0);
+          r[0] = q.x; r[1] = q.y;
+          for (int k = 1; k < nsplit; ++k) {
+            q = *reinterpret_cast<const float2*>(r0 + k * split_stride);
+            r[0] = __fadd_rn(r[0], q.x);
+            r[1] = __fadd_rn(r[1], q.y);
+          }
+        } else {
+          r[0] = r0[0];
+          r[1] = v1 ? r0[1] : 0.f;
+          for (int k = 1; k < nsplit; ++k) {
+            r[0] = __fadd_rn(r[0], r0[k * split_stride]);
+            if (v1) r[1] = __fadd_rn(r[1], r0[k * split_stride + 1]);
+          }
+        }
+        dh[0] = __fadd_rn(dh[0], r[0]);
+        dh[1] = __fadd_rn(dh[1], r[1]);
+      }
+      const long ro = (long)b * Hp + j0;
+      const float2 dc2 = *reinterpret_cast<const float2*>(dc + ro);
+      const float2 cp2 = *reinterpret_cast<const float2*>(c_prev + ro);
+      const float2 cn2 = *reinterpret_cast<const float2*>(c_new + ro);
+      float dco[2], duh[2][4], dwx[2][4];
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int ul = 2 * tx + u;
+        if (!(u == 0 ? v0 : v1)) {   // padding unit: its gradients stay exactly zero
+          dco[u] = 0.f;
+#pragma unroll
+          for (int g = 0; g < 4; ++g) duh[u][g] = dwx[u][g] = 0.f;
+          continue;
+        }
+        float a[4], w[4], h[4];
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          w[g] = u == 0 ? wx[g].x : wx[g].y;
+          h[g] = u == 0 ? uh[g].x : uh[g].y;
+          a[g] = preact<KIND>(w[g], h[g], prm[0][g][ul], KIND == K_MILSTM ? prm[KIND == K_MILSTM ? 1 : 0][g][ul] : 0.f,
+                              KIND == K_MILSTM ? prm[KIND == K_MILSTM ? 2 : 0][g][ul] : 0.f,
+                              KIND == K_MILSTM ? prm[KIND == K_MILSTM ? 3 : 0][g][ul] : 0.f);
+        }
+        float dcv = u == 0 ? dc2.x : dc2.y;
+        float da[4];
+        cell_bwd<KIND, FastMath<T>::value>(a, u == 0 ? cp2.x : cp2.y, u == 0 ? cn2.x : cn2.y, dh[u], dcv, da);
+        dco[u] = dcv;
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          red[ty][g][u][tx] = __fadd_rn(red[ty][g][u][tx], da[g]);
+          if (KIND == K_MILSTM) {
+            const float al = prm[KIND == K_MILSTM ? 1 : 0][g][ul], be1 = prm[KIND == K_MILSTM ? 2 : 0][g][ul],
+                        be2 = prm[KIND == K_MILSTM ? 3 : 0][g][ul];
+            duh[u][g] = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al, w[g]), be1));
+            dwx[u][g] = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al, h[g]), be2));
+            red[ty][(KIND == K_MILSTM ? 4 : 0) + g][u][tx] =
+                __fadd_rn(red[ty][(KIND == K_MILSTM ? 4 : 0) + g][u][tx], __fmul_rn(__fmul_rn(da[g], w[g]), h[g]));
+            red[ty][(KIND == K_MILSTM ? 8 : 0) + g][u][tx] =
+                __fadd_rn(red[ty][(KIND == K_MILSTM ? 8 : 0) + g][u][tx], __fmul_rn(da[g], h[g]));
+            red[ty][(KIND == K_MILSTM ? 12 : 0) + g][u][tx] =
+                __fadd_rn(red[ty][(KIND == K_MILSTM ? 12 : 0) + g][u][tx], __fmul_rn(da[g], w[g]));
+          } else {
+            duh[u][g] = da[g];
+            dwx[u][g] = 0.f;
+          }
+        }
+      }
+      *reinterpret_cast<float2*>(dc + ro) = make_float2(dco[0], dco[1]);
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        store2<T>(D_uh + rg + gcol(g, j0), duh[0][g], duh[1][g]);
+        if (KIND == K_MILSTM) store2cs<T>(D_wx + rg + gcol(g, j0), dwx[0][g], dwx[1][g]);
+      }
+    }
+  }
+  __syncthreads();
+  // finalise: (quantity, unit) items; each sums the 8 row lanes in ty order
+  for (int i = tid; i < NV * BWD_UX; i += BWD_TX * BWD_RY) {
+    const int qi = i / BWD_UX, ul = i % BWD_UX, j = u0 + ul;
+    const int q = qi / 4, g = qi % 4;
+    if (j >= Hp || q >= nq) continue;
     float v = 0.f;
 #pragma unroll
-    for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[y][i][ux]);
-    const int q = i / 4, g = i % 4;
-    if (q >= nq) continue;
+    for (int yy = 0; yy < BWD_RY; ++yy) v = __fadd_rn(v, red[yy][qi][ul & 1][ul >> 1]);
     float* p = partials + ((long)chunk * nq + q) * NG + gcol(g, j);
     *p = first ? v : __fadd_rn(*p, v);
   }
@@ -274,7 +393,7 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
                           bool first, cudaStream_t st) {
   dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
-  dim3 block(BWD_UX, BWD_RY);
+  dim3 block(BWD_TX, BWD_RY);
   if (dy_f32 || dy_ot == OT::F32)
     lstm_bwd_pw_kernel<KIND, T, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX,
                                                              UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials,

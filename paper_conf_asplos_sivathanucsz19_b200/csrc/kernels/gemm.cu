@@ -1,7 +1,10 @@
 // Host side of K1 (tcgen05 GEMM) and K10 (SIMT fp32 GEMM).
 #include <cuda.h>
 #include <cudaTypedefs.h>
+#include <cstring>
 #include <mutex>
+#include <tuple>
+#include <map>
 
 #include "../common.h"
 #include "gemm.h"
@@ -47,7 +50,40 @@ static void make_map(CUtensorMap* m, const Mat2& t, int box_inner, int box_outer
   if (r != CUDA_SUCCESS) throw Error(ASTRA_E_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r));
 }
 
-static uint32_t make_idesc(int BN, bool a_mn, bool b_mn) {
+// Output tensor map of a plain (identity-mapped, non-accumulating) epilogue: [ksplit][Mv][Nv] of
+// fp32 / bf16 at row stride ldc, box 32 x 32 (one epilogue warp's chunk), swizzled like the
+// epilogue's shared-memory tile.  Cached by (pointer, shape): the step's output buffers repeat.
+static bool epi_tma_map(const EpiStore& e, int ksplit, CUtensorMap* out) {
+  const long esz = e.out_bf16 ? 2 : 4;
+  if (e.perm_u || e.perm_blk || e.accumulate) return false;
+  if (((uintptr_t)e.C & 15) || ((e.ldc * esz) & 15) || e.Mv <= 0 || e.Nv <= 0) return false;
+  const long zs = ksplit > 1 ? e.split_stride : (long)e.Mv * e.ldc;
+  if (ksplit > 1 && ((zs * esz) & 15)) return false;
+  using Key = std::tuple<const void*, int, int, long, int, long, int>;
+  static std::map<Key, CUtensorMap> cache;
+  static std::mutex mu;
+  const Key key{e.C, e.Mv, e.Nv, e.ldc, ksplit, zs, e.out_bf16};
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = cache.find(key);
+  if (it == cache.end()) {
+    CUtensorMap m;
+    cuuint64_t dims[3] = {(cuuint64_t)e.Nv, (cuuint64_t)e.Mv, (cuuint64_t)ksplit};
+    cuuint64_t strides[2] = {(cuuint64_t)(e.ldc * esz), (cuuint64_t)(zs * esz)};
+    cuuint32_t box[3] = {32, 32, 1};
+    cuuint32_t estr[3] = {1, 1, 1};
+    CUresult r = encode_fn()(&m, e.out_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
+                             e.C, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                             e.out_bf16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return false;
+    if (cache.size() > 65536) cache.clear();
+    it = cache.emplace(key, m).first;
+  }
+  *out = it->second;
+  return true;
+}
+
+static uint32_t make_idesc(int BN, bool a_mn, bool b_mn, int BM = TC_BM) {
   uint32_t d = 0;
   d |= 1u << 4;                      // D format: F32
   d |= 1u << 7;                      // A format: BF16
@@ -55,7 +91,7 @@ static uint32_t make_idesc(int BN, bool a_mn, bool b_mn) {
   d |= (a_mn ? 1u : 0u) << 15;       // A major
   d |= (b_mn ? 1u : 0u) << 16;       // B major
   d |= (uint32_t)(BN >> 3) << 17;    // N >> 3
-  d |= (uint32_t)(TC_BM >> 4) << 24; // M >> 4
+  d |= (uint32_t)(BM >> 4) << 24;    // M >> 4
   return d;
 }
 
@@ -69,13 +105,16 @@ static int smem_for(int& stages) {
 }
 
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
-                     int cm, int cn, bool b_keep, int ksplit) {
+                     int cm, int cn, bool b_keep, int ksplit, int cg) {
+  ASTRA_CHECK_ARG(cg == 1 || (cg == 2 && cm == 1 && cn == 1 && BN >= 128),
+                  "tc_gemm: CTA pairs (cg = 2) need BN >= 128 and no extra cluster multicast");
   ASTRA_CHECK_ARG((cm == 1 || cm == 2 || cm == 4) && (cn == 1 || cn == 2 || cn == 4) && cm * cn <= 8,
                   "tc_gemm: cluster shape must be cm, cn in {1,2,4}, cm*cn <= 8");
   ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256, "tc_gemm: BN must be 64, 128 or 256");
   ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
   if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
-  if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm);
+  if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm / cg);
+  g.args.cg = cg;
   g.args.cm = cm;
   g.args.cn = cn;
   g.args.b_keep = b_keep ? 1 : 0;
@@ -87,15 +126,50 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   g.args.num_n = cdiv(N, BN);
   g.args.az = g.args.bz = 0;
   g.args.a_mn = a_mn; g.args.b_mn = b_mn;
-  g.args.idesc = make_idesc(BN, a_mn, b_mn);
+  g.args.idesc = make_idesc(BN, a_mn, b_mn, TC_BM * cg);
   int stages = 0;
-  switch (BN) {
+  switch (BN / cg) {
     case 64: g.smem = smem_for<64>(stages); break;
     case 128: g.smem = smem_for<128>(stages); break;
     default: g.smem = smem_for<256>(stages); break;
   }
   g.args.stages = stages;
   g.ready = true;
+}
+
+template <int BN>
+static void launch_pair(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
+  static int attr_bytes = 0;
+  if (g.smem > attr_bytes) {
+    CUDA_TRY(cudaFuncSetAttribute(tc_gemm2_kernel<BN, EpiStore>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  g.smem));
+    attr_bytes = g.smem;
+  }
+  TcArgs a = g.args;
+  a.az = az;
+  a.bz = bz;
+  CUtensorMap mapC;
+  EpiStore e = epi;
+  e.tma = epi_tma_map(epi, a.ksplit, &mapC) ? 1 : 0;
+  if (!e.tma) memset(&mapC, 0, sizeof(mapC));
+  const int ptiles = cdiv(a.M, 2 * TC_BM) * a.num_n * a.ksplit;
+  int pairs = num_sms() / 2;
+  if (max_ctas > 0 && max_ctas / 2 < pairs) pairs = max_ctas / 2 > 0 ? max_ctas / 2 : 1;
+  if (ptiles < pairs) pairs = ptiles;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(2 * pairs);
+  cfg.blockDim = dim3(TC_THREADS);
+  cfg.dynamicSmemBytes = g.smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  CUDA_TRY(cudaLaunchKernelEx(&cfg, tc_gemm2_kernel<BN, EpiStore>, g.mapA, g.mapB, mapC, a, e));
+  LAUNCH_CHECK();
 }
 
 template <int BN>
@@ -109,6 +183,10 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   TcArgs a = g.args;
   a.az = az;
   a.bz = bz;
+  CUtensorMap mapC;
+  EpiStore e = epi;
+  e.tma = epi_tma_map(epi, a.ksplit, &mapC) ? 1 : 0;
+  if (!e.tma) memset(&mapC, 0, sizeof(mapC));
   const int cs = a.cm * a.cn;
   const int ctiles = cdiv(a.num_m, a.cm) * cdiv(a.num_n, a.cn) * a.ksplit;   // cluster tiles × K chunks
   int clusters = num_sms() / cs;
@@ -116,7 +194,7 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   if (ctiles < clusters) clusters = ctiles;
   const int grid = clusters * cs;
   if (cs == 1) {
-    tc_gemm_kernel<BN, EpiStore><<<grid, TC_THREADS, g.smem, st>>>(g.mapA, g.mapB, a, epi);
+    tc_gemm_kernel<BN, EpiStore><<<grid, TC_THREADS, g.smem, st>>>(g.mapA, g.mapB, mapC, a, e);
   } else {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
@@ -130,13 +208,18 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    CUDA_TRY(cudaLaunchKernelEx(&cfg, tc_gemm_kernel<BN, EpiStore>, g.mapA, g.mapB, a, epi));
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, tc_gemm_kernel<BN, EpiStore>, g.mapA, g.mapB, mapC, a, e));
   }
   LAUNCH_CHECK();
 }
 
 void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
   ASTRA_CHECK_STATE(g.ready, "tc_gemm: not prepared");
+  if (g.args.cg == 2) {
+    if (g.BN == 128) launch_pair<128>(g, epi, az, bz, st, max_ctas);
+    else launch_pair<256>(g, epi, az, bz, st, max_ctas);
+    return;
+  }
   switch (g.BN) {
     case 64: launch_bn<64>(g, epi, az, bz, st, max_ctas); break;
     case 128: launch_bn<128>(g, epi, az, bz, st, max_ctas); break;

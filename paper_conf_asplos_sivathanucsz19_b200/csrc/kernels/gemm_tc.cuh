@@ -24,9 +24,24 @@
 
 namespace astra {
 
+#ifdef ASTRA_GEMM_TRACE   // phase timestamps of CTA 0 (scratch/gemm_trace.cu)
+__device__ unsigned long long g_gemm_trace[16];
+__device__ __forceinline__ void gemm_trace(int i) {
+  if (blockIdx.x == 0) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_gemm_trace[i] = t;
+  }
+}
+#define GEMM_TRACE(i) gemm_trace(i)
+#else
+#define GEMM_TRACE(i) do {} while (0)
+#endif
+
 constexpr int TC_BM = 128;
 constexpr int TC_BK = 64;          // one 128-byte swizzle atom of bf16 along K
-constexpr int TC_THREADS = 192;
+constexpr int TC_EPI_WARPS = 4;                    // epilogue warps (one per TMEM lane quarter)
+constexpr int TC_THREADS = 64 + 32 * TC_EPI_WARPS;
 
 struct TcArgs {
   int M, N, K;
@@ -37,6 +52,7 @@ struct TcArgs {
   int cm, cn;       // cluster shape (CTAs sharing B along M, sharing A along N)
   int b_keep;       // 1: load B with an L2 evict_last policy (weights re-read every step)
   int ksplit;       // fixed split of K into ksplit chunks; chunk ks writes its fp32 partial to C + ks·split_stride
+  int cg;           // 1: one CTA per 128 x BN tile; 2: CTA pair per 256 x BN tile (tc_gemm2_kernel)
   uint32_t idesc;
 };
 
@@ -46,11 +62,15 @@ struct TcSmem {
   static constexpr int B_BYTES = BN * TC_BK * 2;      // BN * 128 B
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
   static constexpr int TMEM_COLS = (2 * BN <= 32) ? 32 : (2 * BN <= 64) ? 64 : (2 * BN <= 128) ? 128 : (2 * BN <= 256) ? 256 : 512;
+  // epilogue transpose tiles: one 32 x 36 fp32 tile per epilogue warp (after the barriers)
+  static constexpr int EPI_TILE = 32 * 32 * 4;                  // one 32-row x 32-col fp32 tile (swizzled)
+  static constexpr int EPI_BYTES = TC_EPI_WARPS * 2 * EPI_TILE;   // double-buffered per warp
+  // layout: [stages][epilogue tiles (1024-aligned)][barriers 256 B]
   static int stages_for(int max_smem) {
-    int s = (max_smem - 1024 - 256) / STAGE_BYTES;
+    int s = (max_smem - 1024 - 256 - EPI_BYTES) / STAGE_BYTES;
     return s > 10 ? 10 : s;
   }
-  static int bytes(int stages) { return 1024 + stages * STAGE_BYTES + 256; }
+  static int bytes(int stages) { return 1024 + stages * STAGE_BYTES + EPI_BYTES + 256; }
 };
 
 // Generic epilogue: store the fp32 accumulator (optionally + bias[n], optionally added onto the
@@ -69,6 +89,7 @@ struct EpiStore {
   int perm_blk;
   int accumulate;
   long split_stride;  // elements between the partial outputs of a split-K GEMM
+  int tma;            // 1: plain stores go through the C tensor map (set by tc_gemm_launch)
 
   __device__ __forceinline__ int map_col(int n, bool& ok) const {
     if (n >= Nv) {  // columns past the GEMM's N (tile overhang) are never stored
@@ -91,77 +112,129 @@ struct EpiStore {
     return n;
   }
 
-  __device__ __forceinline__ void store16(int m, int n0, const float (&v)[16]) const {
-    if (m >= Mv) return;
-    bool ok0;
-    const int e0 = map_col(n0, ok0);
-    bool contiguous = n0 + 16 <= Nv;
-    if (!contiguous) {
-    } else if (perm_u) contiguous = ((n0 % perm_u) + 16 <= perm_u) && ((n0 / (4 * perm_u)) * perm_u + n0 % perm_u + 16 <= perm_H);
-    else if (perm_blk) contiguous = (n0 % perm_blk) + 16 <= perm_H;
-    float w[16];
-#pragma unroll
-    for (int i = 0; i < 16; ++i) w[i] = v[i] + ((bias && n0 + i < Nv) ? bias[n0 + i] : 0.f);
-    if (contiguous) {
-      if (out_bf16) {
-        __nv_bfloat16* p = reinterpret_cast<__nv_bfloat16*>(C) + (long)m * ldc + e0;
-        if ((((uintptr_t)p) & 15) == 0) {
-          uint4 pk[2];
-          uint32_t* u = reinterpret_cast<uint32_t*>(pk);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) {
-            __nv_bfloat162 b2 = __floats2bfloat162_rn(w[2 * i], w[2 * i + 1]);
-            u[i] = *reinterpret_cast<uint32_t*>(&b2);
-          }
-          reinterpret_cast<uint4*>(p)[0] = pk[0];
-          reinterpret_cast<uint4*>(p)[1] = pk[1];
-        } else {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) p[i] = __float2bfloat16_rn(w[i]);
-        }
-      } else {
-        float* p = reinterpret_cast<float*>(C) + (long)m * ldc + e0;
-        if ((((uintptr_t)p) & 15) == 0) {
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            float4 o = make_float4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
-            if (accumulate) {
-              const float4 c = reinterpret_cast<const float4*>(p)[i];
-              o.x = __fadd_rn(c.x, o.x); o.y = __fadd_rn(c.y, o.y); o.z = __fadd_rn(c.z, o.z); o.w = __fadd_rn(c.w, o.w);
-            }
-            reinterpret_cast<float4*>(p)[i] = o;
-          }
-        } else {
-#pragma unroll
-          for (int i = 0; i < 16; ++i) p[i] = accumulate ? __fadd_rn(p[i], w[i]) : w[i];
-        }
-      }
-      return;
+  // Scalar store of one element (mapping, bias, bf16 and accumulate handled per element).
+  __device__ __forceinline__ void store1(char* Cb, int m, int n, float v) const {
+    bool ok;
+    const int e = map_col(n, ok);
+    if (!ok) return;
+    v += bias ? bias[n] : 0.f;
+    const long off = (long)m * ldc + e;
+    if (out_bf16) {
+      reinterpret_cast<__nv_bfloat16*>(Cb)[off] = __float2bfloat16_rn(v);
+    } else {
+      float* p = reinterpret_cast<float*>(Cb) + off;
+      *p = accumulate ? __fadd_rn(*p, v) : v;
     }
-#pragma unroll
-    for (int i = 0; i < 16; ++i) {
-      bool ok;
-      const int e = map_col(n0 + i, ok);
-      if (!ok) continue;
-      if (out_bf16) {
-        reinterpret_cast<__nv_bfloat16*>(C)[(long)m * ldc + e] = __float2bfloat16_rn(w[i]);
-      } else {
-        float* p = reinterpret_cast<float*>(C) + (long)m * ldc + e;
-        *p = accumulate ? __fadd_rn(*p, w[i]) : w[i];
-      }
-    }
-    (void)ok0;
   }
 
+  // Epilogue of one 128 x BN accumulator tile, called by each of the 4 epilogue warps for its 32
+  // TMEM lanes (tile rows quarter·32 ..+31), in 32-column chunks: tcgen05.ld (thread = row) →
+  // the thread's row of a 32 x 32 fp32 shared-memory tile (dense 128-byte rows, 16-byte chunks
+  // XOR-swizzled by row % 8 = the TMA SWIZZLE_128B pattern, so the 16-byte stores of 8 rows hit
+  // distinct banks; two tiles per warp, alternating) → global:
+  //  * tma (plain store, identity column map): one lane issues a TMA tensor store of the tile —
+  //    the copy engine writes it out asynchronously and clips rows ≥ Mv / columns ≥ Nv;
+  //  * otherwise (accumulate, remapped columns, bf16 via the same path): transpose through the
+  //    tile and store with 16-byte vector stores, 4 full row segments per warp instruction,
+  //    element stores where a 4-column group is not contiguous and aligned.
   template <int BN>
-  __device__ __forceinline__ void run(uint32_t taddr, int m0, int n0, int row, int ks) const {
-    EpiStore e = *this;
-    if (ks) e.C = reinterpret_cast<char*>(C) + (size_t)ks * split_stride * (out_bf16 ? 2 : 4);
+  __device__ __forceinline__ void run(uint32_t taddr, int m0, int n0, int quarter, int lane, int ks,
+                                      uint32_t stile, int& nbuf, const CUtensorMap* mapC) const {
+    char* Cb = reinterpret_cast<char*>(C) + (ks ? (size_t)ks * split_stride * (out_bf16 ? 2 : 4) : 0);
+    const int r0 = m0 + quarter * 32;
+    const int rr = lane >> 3, c4 = (lane & 7) * 4;
+    const bool ld_al = ((ldc * (out_bf16 ? 2 : 4)) & 15) == 0 && (((uintptr_t)Cb) & 15) == 0;
 #pragma unroll 1
-    for (int c = 0; c < BN; c += 16) {
-      float v[16];
-      sm100::tmem_ld16(taddr + c, v);
-      e.store16(m0 + row, n0 + c, v);
+    for (int c = 0; c < BN; c += 32) {
+      const uint32_t tile = stile + (uint32_t)(nbuf & 1) * (32 * 32 * 4);
+      const int n = n0 + c;
+      float v[32];
+      sm100::tmem_ld32(taddr + c, v);
+      if (tma) {
+        if (n >= Nv) continue;
+        if (bias) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] += (n + i < Nv) ? bias[n + i] : 0.f;
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] += 0.f;
+        }
+        if (lane == 0) sm100::bulk_wait_read<1>();   // the store that last read this tile is done
+        __syncwarp();
+        if (out_bf16) {   // 64-byte rows, SWIZZLE_64B: 16-byte chunk i of row r at i ^ ((r >> 1) & 3)
+          uint32_t u[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            __nv_bfloat162 b2 = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+            u[i] = *reinterpret_cast<uint32_t*>(&b2);
+          }
+          const uint32_t row = tile + (uint32_t)lane * 64;
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+            sm100::sts_v4(row + (uint32_t)((i ^ ((lane >> 1) & 3)) * 16), __uint_as_float(u[4 * i]),
+                          __uint_as_float(u[4 * i + 1]), __uint_as_float(u[4 * i + 2]), __uint_as_float(u[4 * i + 3]));
+        } else {          // 128-byte rows, SWIZZLE_128B: chunk i of row r at i ^ (r & 7)
+          const uint32_t row = tile + (uint32_t)lane * 128;
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            sm100::sts_v4(row + (uint32_t)((i ^ (lane & 7)) * 16), v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+        }
+        sm100::fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          sm100::tma_store_3d(mapC, tile, n, r0, ks);
+          sm100::bulk_commit();
+        }
+        ++nbuf;
+        continue;
+      }
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        sm100::sts_v4(tile + (uint32_t)lane * 128 + (uint32_t)((i ^ (lane & 7)) * 16), v[4 * i], v[4 * i + 1],
+                      v[4 * i + 2], v[4 * i + 3]);
+      __syncwarp();
+      const int nc = n + c4;
+      bool ok0, ok3;
+      const int e0 = map_col(nc, ok0);
+      const int e3 = map_col(nc + 3, ok3);
+      const bool vec = ld_al && ok0 && ok3 && e3 == e0 + 3 && (e0 & 3) == 0;
+      float b4[4] = {0.f, 0.f, 0.f, 0.f};
+      if (vec && bias) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) b4[i] = bias[nc + i];
+      }
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        const int row = q * 4 + rr;
+        float4 w = sm100::lds_v4(tile + (uint32_t)row * 128 + (uint32_t)((((c4 >> 2) ^ (row & 7))) * 16));
+        const int m = r0 + row;
+        if (m >= Mv) continue;
+        if (vec) {
+          w.x += b4[0]; w.y += b4[1]; w.z += b4[2]; w.w += b4[3];
+          const long off = (long)m * ldc + e0;
+          if (out_bf16) {
+            __nv_bfloat162 lo = __floats2bfloat162_rn(w.x, w.y), hi = __floats2bfloat162_rn(w.z, w.w);
+            uint2 u;
+            u.x = *reinterpret_cast<uint32_t*>(&lo);
+            u.y = *reinterpret_cast<uint32_t*>(&hi);
+            *reinterpret_cast<uint2*>(reinterpret_cast<__nv_bfloat16*>(Cb) + off) = u;
+          } else {
+            float4* p = reinterpret_cast<float4*>(reinterpret_cast<float*>(Cb) + off);
+            if (accumulate) {
+              const float4 o = *p;
+              w.x = __fadd_rn(o.x, w.x); w.y = __fadd_rn(o.y, w.y); w.z = __fadd_rn(o.z, w.z); w.w = __fadd_rn(o.w, w.w);
+            }
+            *p = w;
+          }
+        } else {
+          store1(Cb, m, nc, w.x);
+          store1(Cb, m, nc + 1, w.y);
+          store1(Cb, m, nc + 2, w.z);
+          store1(Cb, m, nc + 3, w.w);
+        }
+      }
+      __syncwarp();
+      ++nbuf;
     }
   }
 };
@@ -175,12 +248,14 @@ struct EpiStore {
 template <int BN, class Epi>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     tc_gemm_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
-                   const TcArgs args, const Epi epi) {
+                   const __grid_constant__ CUtensorMap mapC, const TcArgs args, const Epi epi) {
   using S = TcSmem<BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  if (threadIdx.x == 0) GEMM_TRACE(0);
   const int stages = args.stages;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * S::STAGE_BYTES);
+  const uint32_t epi_tiles = sm100::smem_u32(smem + stages * S::STAGE_BYTES);   // 1024-aligned
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * S::STAGE_BYTES + S::EPI_BYTES);
   uint64_t* empty = full + stages;
   uint64_t* tfull = empty + stages;   // [2]
   uint64_t* tempty = tfull + 2;       // [2]
@@ -209,13 +284,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
     for (int a = 0; a < 2; ++a) {
       sm100::mbar_init(&tfull[a], 1);
-      sm100::mbar_init(&tempty[a], 128);
+      sm100::mbar_init(&tempty[a], 32 * TC_EPI_WARPS);
     }
     sm100::fence_barrier_init();
   }
   if (warp == 0 && lane == 0) {
     sm100::tma_prefetch(&mapA);
     sm100::tma_prefetch(&mapB);
+    if (epi.tma) sm100::tma_prefetch(&mapC);
   }
   if (warp == 1) sm100::tmem_alloc(tmem_slot, S::TMEM_COLS);
   sm100::tc_fence_before();
@@ -223,6 +299,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (cs > 1) sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) GEMM_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
@@ -305,6 +382,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const int kb0 = (ct / num_ct1) * kper, kb1 = min(nk_all, kb0 + kper);
         for (int kb = kb0; kb < kb1; ++kb) {
           sm100::mbar_wait(&full[s], ph);
+          if (kb == kb0 && local == 0) GEMM_TRACE(3);
           sm100::tc_fence_after();
           const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
           const uint32_t sb = sa + S::A_BYTES;
@@ -321,12 +399,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           if (++s == stages) { s = 0; ph ^= 1; }
         }
         sm100::umma_commit(&tfull[acc]);
+        GEMM_TRACE(4);
       }
     }
   } else {
     // ------------------------------------------------------------ epilogue warps 2..5
     const int quarter = warp & 3;           // TMEM lane quarter this warp may access
-    const int row = quarter * 32 + lane;    // tile row (= TMEM lane)
+    int nbuf = 0;                           // epilogue tiles used so far (alternating buffers)
     int local = 0;
     for (int ct = cluster_id; ct < num_ct; ct += num_clusters, ++local) {
       const int acc = local & 1;
@@ -335,18 +414,186 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int m0 = ((c1 % ncm) * cm + rm) * TC_BM;
       const int n0 = ((c1 / ncm) * cn + rn) * BN;
       sm100::mbar_wait(&tfull[acc], use & 1);
+      if (warp == 2 && lane == 0) GEMM_TRACE(5);
       sm100::tc_fence_after();
       const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * BN;
-      if (m0 < args.M && n0 < args.N && ks * kper < nk_all) epi.template run<BN>(taddr, m0, n0, row, ks);
+      if (m0 < args.M && n0 < args.N && ks * kper < nk_all) epi.template run<BN>(taddr, m0, n0, quarter, lane, ks, epi_tiles + (uint32_t)(warp - 2) * 2 * S::EPI_TILE, nbuf,
+                                                                                   &mapC);
       sm100::tc_fence_before();
+      if (warp == 2 && lane == 0) GEMM_TRACE(6);
       sm100::mbar_arrive(&tempty[acc]);
     }
+    sm100::bulk_wait_all();   // this thread's bulk stores have landed before the CTA retires
   }
   __syncthreads();
   if (cs > 1) sm100::cluster_sync();
   if (warp == 1) {
     sm100::tc_fence_after();
     sm100::tmem_dealloc(tmem_base, S::TMEM_COLS);
+  }
+  if (threadIdx.x == 0) GEMM_TRACE(7);
+}
+
+// CTA-pair variant (cta_group::2).  A cluster of 2 CTAs on one TPC owns a 256 x BN output tile:
+// CTA r holds rows 128r..128r+127 of A and columns r·BN/2 .. of B in its shared memory, the pair
+// leader (rank 0) issues one M = 256 MMA per K16 that reads both halves, and each CTA's TMEM
+// receives its own 128 rows x BN accumulator.  Every operand byte therefore crosses L2 → SM once
+// per pair instead of once per CTA for B, cutting the per-SM operand traffic of a 128 x BN tile
+// from (128 + BN)·K to (128 + BN/2)·K elements — the bound of the small-M per-step GEMMs.
+// Barriers: both CTAs' TMA loads signal the leader's `full` barrier (the leader expects the
+// pair's bytes); the leader's MMA commit arrives on `empty` and `tfull` of both CTAs (multicast);
+// each CTA's 4 epilogue warps arrive on the leader's `tempty`.  Accumulation order per output
+// element is unchanged (ascending K, one chain per element, split-K chunks as in tc_gemm_kernel),
+// so results are bitwise identical to the single-CTA kernel.
+template <int BN, class Epi>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+    tc_gemm2_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                    const __grid_constant__ CUtensorMap mapC, const TcArgs args, const Epi epi) {
+  constexpr int BH = BN / 2;          // B columns held by each CTA
+  using S = TcSmem<BH>;
+  constexpr int TMEM_COLS = 2 * BN;   // two accumulator buffers of BN columns
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int stages = args.stages;
+  const uint32_t epi_tiles = sm100::smem_u32(smem + stages * S::STAGE_BYTES);   // 1024-aligned
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * S::STAGE_BYTES + S::EPI_BYTES);
+  uint64_t* empty = full + stages;
+  uint64_t* tfull = empty + stages;   // [2]
+  uint64_t* tempty = tfull + 2;       // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x / 32;
+  const int lane = threadIdx.x % 32;
+  const int rank = (int)sm100::cluster_ctarank();
+  const int num_mp = (args.M + 2 * TC_BM - 1) / (2 * TC_BM);
+  const int num_pt1 = num_mp * args.num_n;
+  const int num_pt = num_pt1 * args.ksplit;
+  const int pair_id = blockIdx.x / 2, num_pairs = gridDim.x / 2;
+  const int nk_all = (args.K + TC_BK - 1) / TC_BK;
+  const int kper = (nk_all + args.ksplit - 1) / args.ksplit;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < stages; ++s) {
+      sm100::mbar_init(&full[s], 1);
+      sm100::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      sm100::mbar_init(&tfull[a], 1);
+      sm100::mbar_init(&tempty[a], 2 * TC_EPI_WARPS);
+    }
+    sm100::fence_barrier_init();
+  }
+  if (warp == 0 && lane == 0) {
+    sm100::tma_prefetch(&mapA);
+    sm100::tma_prefetch(&mapB);
+    if (epi.tma) sm100::tma_prefetch(&mapC);
+  }
+  if (warp == 1) sm100::tmem_alloc_cg2(tmem_slot, TMEM_COLS);
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::cluster_sync();
+  sm100::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ TMA producer (both CTAs)
+    if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0;
+      const uint64_t pol = sm100::l2_policy_evict_last();
+      for (int ct = pair_id; ct < num_pt; ct += num_pairs) {
+        const int ks = ct / num_pt1, c1 = ct % num_pt1;
+        const int m0 = (c1 % num_mp) * 2 * TC_BM + rank * TC_BM;
+        const int n0 = (c1 / num_mp) * BN + rank * BH;
+        const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
+        for (int kb = kb0; kb < kb1; ++kb) {
+          sm100::mbar_wait(&empty[s], ph ^ 1);
+          uint8_t* sa = smem + s * S::STAGE_BYTES;
+          uint8_t* sb = sa + S::A_BYTES;
+          if (rank == 0) sm100::mbar_arrive_expect_tx(&full[s], 2 * S::STAGE_BYTES);
+          const uint32_t bar = sm100::mapa_shared(sm100::smem_u32(&full[s]), 0);
+          const int k0 = kb * TC_BK;
+          if (args.a_mn) {
+            sm100::tma_load_3d_cg2(sa, &mapA, bar, m0, k0, args.az);
+            sm100::tma_load_3d_cg2(sa + 8192, &mapA, bar, m0 + 64, k0, args.az);
+          } else {
+            sm100::tma_load_3d_cg2(sa, &mapA, bar, k0, m0, args.az);
+          }
+          if (args.b_mn) {
+#pragma unroll
+            for (int j = 0; j < BH / 64; ++j) {
+              if (args.b_keep) sm100::tma_load_3d_cg2_hint(sb + j * 8192, &mapB, bar, n0 + 64 * j, k0, args.bz, pol);
+              else sm100::tma_load_3d_cg2(sb + j * 8192, &mapB, bar, n0 + 64 * j, k0, args.bz);
+            }
+          } else {
+            if (args.b_keep) sm100::tma_load_3d_cg2_hint(sb, &mapB, bar, k0, n0, args.bz, pol);
+            else sm100::tma_load_3d_cg2(sb, &mapB, bar, k0, n0, args.bz);
+          }
+          if (++s == stages) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------ MMA issuer (pair leader only)
+    if (lane == 0 && rank == 0) {
+      int s = 0;
+      uint32_t ph = 0;
+      int local = 0;
+      for (int ct = pair_id; ct < num_pt; ct += num_pairs, ++local) {
+        const int acc = local & 1;
+        const uint32_t use = (uint32_t)(local >> 1);
+        sm100::mbar_wait(&tempty[acc], (use & 1) ^ 1);
+        sm100::tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        const int kb0 = (ct / num_pt1) * kper, kb1 = min(nk_all, kb0 + kper);
+        for (int kb = kb0; kb < kb1; ++kb) {
+          sm100::mbar_wait(&full[s], ph);
+          sm100::tc_fence_after();
+          const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
+          const uint32_t sb = sa + S::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < TC_BK / 16; ++kk) {
+            const uint64_t ad = args.a_mn ? sm100::smem_desc_sw128(sa + kk * 2048, 8192, 1024)
+                                          : sm100::smem_desc_sw128(sa + kk * 32, 16, 1024);
+            const uint64_t bd = args.b_mn ? sm100::smem_desc_sw128(sb + kk * 2048, 8192, 1024)
+                                          : sm100::smem_desc_sw128(sb + kk * 32, 16, 1024);
+            sm100::umma_bf16_cg2(d_tmem, ad, bd, args.idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
+          }
+          sm100::umma_commit_cg2_mc(&empty[s], 0x3);
+          if (++s == stages) { s = 0; ph ^= 1; }
+        }
+        sm100::umma_commit_cg2_mc(&tfull[acc], 0x3);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue warps 2..5 (both CTAs)
+    const int quarter = warp & 3;
+    int nbuf = 0;
+    const uint32_t tempty_cl[2] = {sm100::mapa_shared(sm100::smem_u32(&tempty[0]), 0),
+                                   sm100::mapa_shared(sm100::smem_u32(&tempty[1]), 0)};
+    int local = 0;
+    for (int ct = pair_id; ct < num_pt; ct += num_pairs, ++local) {
+      const int acc = local & 1;
+      const uint32_t use = (uint32_t)(local >> 1);
+      const int ks = ct / num_pt1, c1 = ct % num_pt1;
+      const int m0 = (c1 % num_mp) * 2 * TC_BM + rank * TC_BM;
+      const int n0 = (c1 / num_mp) * BN;
+      sm100::mbar_wait(&tfull[acc], use & 1);
+      sm100::tc_fence_after();
+      const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * BN;
+      if (m0 < args.M && n0 < args.N && ks * kper < nk_all) epi.template run<BN>(taddr, m0, n0, quarter, lane, ks, epi_tiles + (uint32_t)(warp - 2) * 2 * S::EPI_TILE, nbuf,
+                                                                                   &mapC);
+      sm100::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) sm100::mbar_arrive_cluster(tempty_cl[acc]);
+    }
+    sm100::bulk_wait_all();
+  }
+  __syncthreads();
+  sm100::cluster_sync();
+  if (warp == 1) {
+    sm100::tc_fence_after();
+    sm100::tmem_dealloc_cg2(tmem_base, TMEM_COLS);
   }
 }
 

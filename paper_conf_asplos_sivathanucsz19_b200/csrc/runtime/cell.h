@@ -33,7 +33,8 @@ struct ParamInfo {
 // own sm_100a kernels): CTA tile width and cluster multicast shape.
 struct KCfg {
   int bn = 256, cm = 1, cn = 1;
-  bool operator==(const KCfg& o) const { return bn == o.bn && cm == o.cm && cn == o.cn; }
+  int cg = 1;   // 2: CTA pair (cta_group::2, 256-row tiles)
+  bool operator==(const KCfg& o) const { return bn == o.bn && cm == o.cm && cn == o.cn && cg == o.cg; }
 };
 enum GemmRole { G_A1 = 0, G_REC, G_BPTT, G_DU, G_DW, G_DX, G_HEAD, G_ROLES };
 extern const char* const ROLE_NAMES[G_ROLES];
@@ -105,7 +106,7 @@ class Cell {
   bool region_used[R_COUNT];
   bool profiling = true;
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
-  std::map<std::tuple<int, int, int, int>, TcGemm> tc_cache;
+  std::map<std::tuple<int, int, int, int, int>, TcGemm> tc_cache;
 
   // NCCL
   void* nccl_comm = nullptr;

@@ -16,7 +16,11 @@ const char* const ROLE_NAMES[G_ROLES] = {"a1", "rec", "bptt", "du", "dw", "dx", 
 
 std::string Variant::str() const {
   std::ostringstream o;
-  for (int r = 0; r < G_ROLES; ++r) o << ROLE_NAMES[r] << "=" << g[r].bn << "." << g[r].cm << "." << g[r].cn << ",";
+  for (int r = 0; r < G_ROLES; ++r) {
+    o << ROLE_NAMES[r] << "=" << g[r].bn << "." << g[r].cm << "." << g[r].cn;
+    if (g[r].cg != 1) o << "." << g[r].cg;
+    o << ",";
+  }
   o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode;
   return o.str();
 }
@@ -50,10 +54,13 @@ Variant Variant::parse(const std::string& s) {
       if (k == ROLE_NAMES[i]) r = i;
     ASTRA_CHECK_ARG(r >= 0, "variant: unknown variable '" + k + "'");
     KCfg c;
-    int n = std::sscanf(val.c_str(), "%d.%d.%d", &c.bn, &c.cm, &c.cn);
+    int n = std::sscanf(val.c_str(), "%d.%d.%d.%d", &c.bn, &c.cm, &c.cn, &c.cg);
     ASTRA_CHECK_ARG(n >= 1, "variant: bad kernel choice '" + val + "'");
+    if (n < 4) c.cg = 1;
     if (n < 3) c.cn = 1;
     if (n < 2) c.cm = 1;
+    ASTRA_CHECK_ARG(c.cg == 1 || (c.cg == 2 && c.cm == 1 && c.cn == 1 && c.bn >= 128),
+                    "variant: CTA pair (4th field 2) needs tile width 128/256 and a 1x1 multicast cluster");
     ASTRA_CHECK_ARG((c.bn == 64 || c.bn == 128 || c.bn == 256) && (c.cm == 1 || c.cm == 2 || c.cm == 4) &&
                         (c.cn == 1 || c.cn == 2 || c.cn == 4) && c.cm * c.cn <= 8,
                     "variant: tile width must be 64/128/256 and cluster cm, cn in {1,2,4} with cm*cn <= 8");
@@ -144,11 +151,11 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
 TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
   // split-K only runs without clusters; the cluster choice then falls back to 1x1 (same numerics)
   const int cm = s.ksplit > 1 ? 1 : k.cm, cn = s.ksplit > 1 ? 1 : k.cn;
-  auto key = std::make_tuple(id, k.bn, cm, cn);
+  auto key = std::make_tuple(id, k.bn, cm, cn, k.cg);
   auto it = tc_cache.find(key);
   if (it == tc_cache.end()) {
     TcGemm g;
-    tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit);
+    tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit, k.cg);
     it = tc_cache.emplace(key, g).first;
   }
   return it->second;
@@ -214,9 +221,9 @@ void Cell::sgd_step(float lr) {
 // ------------------------------------------------------------------------ tuner glue
 // The enumerator's static pruning (A19): per GEMM role, the kernel choices whose tile
 // and cluster shape fit the problem; the default (Variant()) first.
-static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 2, 1}, {256, 4, 1}, {256, 2, 2},
-                                  {256, 1, 2}, {128, 2, 1}, {128, 4, 1}, {128, 2, 2}, {128, 1, 2}, {64, 2, 1},
-                                  {64, 4, 1}, {64, 2, 2}};
+static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 1, 1, 2}, {128, 1, 1, 2},
+                                  {256, 2, 1}, {256, 4, 1}, {256, 2, 2}, {256, 1, 2}, {128, 2, 1}, {128, 4, 1},
+                                  {128, 2, 2}, {128, 1, 2}, {64, 2, 1}, {64, 4, 1}, {64, 2, 2}};
 
 void Cell::tuner_setup() {
   const Variant def;
@@ -235,6 +242,7 @@ void Cell::tuner_setup() {
         const int num_m = cdiv(M, TC_BM), num_n = cdiv(N, k.bn);
         if (k.bn > 64 && N <= k.bn / 2) continue;                                     // tile wider than N
         if (k.cm > num_m || k.cn > num_n) continue;                                    // idle cluster ranks
+        if (k.cg == 2 && num_m < 2) continue;                                          // idle pair half
         allowed[r].push_back(k);
       }
       par += std::string(" (leaf g_") + ROLE_NAMES[r] + " " + std::to_string(allowed[r].size()) + " " + metric[r] + ")";

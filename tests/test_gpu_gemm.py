@@ -88,7 +88,7 @@ def test_split_k_partials(ksplit, a_mn, b_mn):
     kper = -(-(-(-K // 64)) // ksplit) * 64
     outs = []
     for bn in (64, 128, 256):
-        out = A.gemm_bf16_splitk(A_s, B_s, M, N, K, ksplit, a_mn=a_mn, b_mn=b_mn, bn=bn)
+        out = A.gemm_bf16_ex(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn, ksplit=ksplit)
         torch.cuda.synchronize()
         outs.append(out.cpu())
     for o in outs[1:]:
@@ -104,3 +104,25 @@ def test_split_k_partials(ksplit, a_mn, b_mn):
     for s in range(1, ksplit):
         tot = tot + o[s]
     assert (tot - full).abs().max().item() <= 1e-5 * full.abs().max().item() * K / 64
+
+
+@pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 0), (1, 1)])
+@pytest.mark.parametrize("M,N,K", [(512, 1024, 512), (300, 200, 136), (128, 256, 64), (700, 640, 1000)])
+def test_cta_pair_bitwise(a_mn, b_mn, M, N, K):
+    """cta_group::2 (CTA pair, 256 x bn tiles) gives the same bits as the single-CTA kernel, with
+    ragged M (half-empty pairs), ragged N and K, every operand layout, and with split-K."""
+    if (a_mn and M % 8) or (b_mn and N % 8) or K % 8:
+        pytest.skip("TMA needs 16-byte row strides")
+    A_s, B_s, ref = _operands(M, N, K, a_mn, b_mn, seed=7)
+    base = A.gemm_bf16(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=128)
+    torch.cuda.synchronize()
+    err = (base.double().cpu() - ref).abs().max().item()
+    assert err <= 1e-5 * ref.abs().max().item() * max(1, K / 64) + 1e-6
+    for bn in (128, 256):
+        out = A.gemm_bf16_ex(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn, cta_group=2)
+        torch.cuda.synchronize()
+        assert torch.equal(out[0].cpu(), base.cpu()), bn
+    s1 = A.gemm_bf16_ex(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=256, ksplit=3)
+    s2 = A.gemm_bf16_ex(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=128, cta_group=2, ksplit=3)
+    torch.cuda.synchronize()
+    assert torch.equal(s1.cpu(), s2.cpu())
