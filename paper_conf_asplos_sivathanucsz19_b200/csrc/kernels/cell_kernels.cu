@@ -5,6 +5,10 @@
 
 #include "cell_math.cuh"
 #include "kernels.h"
+#include "pdl.cuh"
+#include "gemm.h"
+#include "sm100.cuh"
+#include <algorithm>
 
 namespace astra {
 
@@ -108,79 +112,164 @@ void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, l
 }
 
 // ============================================================================ LSTM-family pointwise
-// K2 forward half.  Thread = 4 consecutive hidden units of one batch row: they share one 64-unit
-// gate group of the interleaved layout, so each gate's WX/UH pre-activations are one 16-byte load.
-constexpr int FWD_U = 4;
+// K2 forward half, streamed through shared memory by the TMA engine.  Work item = one batch row
+// x one block of FB_UB hidden units: its gate pre-activations WX and UH (gate-interleaved, so the
+// block is one contiguous FB_UB·4-float run of each) and c_{t-1} are fetched with three 1-D bulk
+// copies into a FB_STAGES-deep ring, so every SM keeps ~100 KB of loads in flight with a handful
+// of instructions; the 256 threads then read their 2 units per gate from shared memory.  Each CTA
+// keeps one unit block (its gate parameters staged once in shared memory) and walks rows
+// b_first, b_first + rstep, ...  Arithmetic per element is the same as the plain kernel.
 template <typename T>
-__device__ __forceinline__ void store4(T* p, const float (&v)[4]);
+__device__ __forceinline__ void store2cs(T* p, float a, float b);
 template <>
-__device__ __forceinline__ void store4<float>(float* p, const float (&v)[4]) {
-  *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+__device__ __forceinline__ void store2cs<float>(float* p, float a, float b) {
+  __stcs(reinterpret_cast<float2*>(p), make_float2(a, b));
 }
 template <>
-__device__ __forceinline__ void store4<__nv_bfloat16>(__nv_bfloat16* p, const float (&v)[4]) {
-  __nv_bfloat162 lo = __floats2bfloat162_rn(v[0], v[1]), hi = __floats2bfloat162_rn(v[2], v[3]);
-  uint2 u;
-  u.x = *reinterpret_cast<uint32_t*>(&lo);
-  u.y = *reinterpret_cast<uint32_t*>(&hi);
-  *reinterpret_cast<uint2*>(p) = u;
+__device__ __forceinline__ void store2cs<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
+  __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
+  __stcs(reinterpret_cast<unsigned int*>(p), *reinterpret_cast<unsigned int*>(&v));
+}
+template <typename T>
+__device__ __forceinline__ void store2(T* p, float a, float b);
+template <>
+__device__ __forceinline__ void store2<float>(float* p, float a, float b) {
+  *reinterpret_cast<float2*>(p) = make_float2(a, b);
+}
+template <>
+__device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
+  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);
+}
+
+constexpr int FB_UB = 512;
+constexpr int FB_THREADS = 256;
+constexpr int FB_STAGES = 4;
+constexpr int FB_SW = FB_UB * 4 * 4;           // bytes of one row block of WX (or UH)
+constexpr int FB_STAGE = 2 * FB_SW + FB_UB * 4;
+
+struct FwdPwArgs {
+  int B, H, Hp, nub, rstep;
+  const float* WX;
+  const float* UH;
+  GateParams gp;
+  const float* c_prev;
+  float* c_new;
+  void* h_op;
+  long ldh;
+  void* y;
+  long ldy;
+  float* hT;
+  float* cT;
+};
+
+template <typename T>
+__device__ __forceinline__ void store_pair(T* p, bool vec, float a, float b, bool ok1) {
+  if (vec) {
+    store2<T>(p, a, b);
+  } else {
+    p[0] = from_f<T>(a);
+    if (ok1) p[1] = from_f<T>(b);
+  }
 }
 
 template <int KIND, typename T, typename TY>
-__global__ void __launch_bounds__(128)
-    lstm_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ WX, const float* __restrict__ UH,
-                       GateParams gp, const float* __restrict__ c_prev, float* __restrict__ c_new,
-                       T* __restrict__ h_op, long ldh, TY* __restrict__ y, long ldy, float* __restrict__ hT,
-                       float* __restrict__ cT) {
-  const int j0 = (blockIdx.x * blockDim.x + threadIdx.x) * FWD_U;
-  const int b = blockIdx.y;
-  if (j0 >= Hp) return;
-  const long rowg = (long)b * 4 * Hp, rowh = (long)b * Hp;
-  float4 wx[4], uh[4];
-#pragma unroll
-  for (int g = 0; g < 4; ++g) {
-    wx[g] = __ldcs(reinterpret_cast<const float4*>(WX + rowg + gcol(g, j0)));
-    uh[g] = __ldcs(reinterpret_cast<const float4*>(UH + rowg + gcol(g, j0)));
+__global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwArgs a) {
+  constexpr int NP = KIND == K_MILSTM ? 4 : 1;
+  extern __shared__ __align__(128) uint8_t sm[];
+  float* prm = reinterpret_cast<float*>(sm + FB_STAGES * FB_STAGE);   // [NP][4][FB_UB]
+  uint64_t* full = reinterpret_cast<uint64_t*>(prm + NP * 4 * FB_UB);
+  const int tid = threadIdx.x;
+  const int ub = blockIdx.x % a.nub, b_first = blockIdx.x / a.nub;
+  const int u0 = ub * FB_UB, nu = min(FB_UB, a.Hp - u0);   // nu: multiple of 64
+  const long NG = 4L * a.Hp;
+  if (tid == 0) {
+    for (int s = 0; s < FB_STAGES; ++s) sm100::mbar_init(&full[s], 1);
+    sm100::fence_barrier_init();
   }
-  const float4 cp4 = *reinterpret_cast<const float4*>(c_prev + rowh + j0);
-  const float cp[4] = {cp4.x, cp4.y, cp4.z, cp4.w};
-  float cv[4], hv[4];
-#pragma unroll
-  for (int u = 0; u < FWD_U; ++u) {
-    const int j = j0 + u;
-    if (j < H) {   // padding units (H ≤ j < Hp) stay exactly zero
-      float a[4];
-#pragma unroll
-      for (int g = 0; g < 4; ++g) {
-        const float w = u == 0 ? wx[g].x : u == 1 ? wx[g].y : u == 2 ? wx[g].z : wx[g].w;
-        const float h = u == 0 ? uh[g].x : u == 1 ? uh[g].y : u == 2 ? uh[g].z : uh[g].w;
-        const int e = g * H + j;
-        a[g] = preact<KIND>(w, h, gp.b[e], KIND == K_MILSTM ? gp.alpha[e] : 0.f,
-                            KIND == K_MILSTM ? gp.beta1[e] : 0.f, KIND == K_MILSTM ? gp.beta2[e] : 0.f);
-      }
-      cell_fwd<KIND, FastMath<T>::value>(a, cp[u], cv[u], hv[u]);
-    } else {
-      cv[u] = 0.f;
-      hv[u] = 0.f;
+  pdl_wait();
+  pdl_trigger();
+  for (int i = tid; i < 4 * nu; i += FB_THREADS) {
+    const int g = i / nu, ul = i % nu, j = u0 + ul, e = g * a.H + j;
+    const bool ok = j < a.H;
+    prm[g * FB_UB + ul] = ok ? a.gp.b[e] : 0.f;
+    if (KIND == K_MILSTM) {
+      prm[(NP > 1 ? 1 : 0) * 4 * FB_UB + g * FB_UB + ul] = ok ? a.gp.alpha[e] : 0.f;
+      prm[(NP > 2 ? 2 : 0) * 4 * FB_UB + g * FB_UB + ul] = ok ? a.gp.beta1[e] : 0.f;
+      prm[(NP > 3 ? 3 : 0) * 4 * FB_UB + g * FB_UB + ul] = ok ? a.gp.beta2[e] : 0.f;
     }
   }
-  store4<float>(c_new + rowh + j0, cv);
-  if ((ldh & 3) == 0) store4<T>(h_op + (long)b * ldh + j0, hv);
-  else
+  __syncthreads();
+  const int nitems = b_first < a.B ? (a.B - b_first + a.rstep - 1) / a.rstep : 0;
+  const uint32_t wbytes = (uint32_t)nu * 16, cbytes = (uint32_t)nu * 4;
+  auto issue = [&](int k) {
+    const int s = k % FB_STAGES;
+    const long b = b_first + (long)k * a.rstep;
+    uint8_t* st = sm + s * FB_STAGE;
+    sm100::mbar_arrive_expect_tx(&full[s], 2 * wbytes + cbytes);
+    sm100::bulk_load(sm100::smem_u32(st), a.WX + b * NG + (long)u0 * 4, wbytes, &full[s]);
+    sm100::bulk_load(sm100::smem_u32(st + FB_SW), a.UH + b * NG + (long)u0 * 4, wbytes, &full[s]);
+    sm100::bulk_load(sm100::smem_u32(st + 2 * FB_SW), a.c_prev + b * a.Hp + u0, cbytes, &full[s]);
+  };
+  if (tid == 0)
+    for (int k = 0; k < FB_STAGES && k < nitems; ++k) issue(k);
+  const int ul = 2 * tid;
+  const bool act = ul < nu;
+  const int base = (ul / 64) * 256 + ul % 64;
+  const bool vh = (a.ldh & 1) == 0, vy = (a.ldy & 1) == 0;
+  for (int k = 0; k < nitems; ++k) {
+    const int s = k % FB_STAGES;
+    sm100::mbar_wait(&full[s], (uint32_t)((k / FB_STAGES) & 1));
+    const long b = b_first + (long)k * a.rstep;
+    if (act) {
+      const float* sw = reinterpret_cast<const float*>(sm + s * FB_STAGE);
+      const float* su = sw + FB_UB * 4;
+      const float* sc = su + FB_UB * 4;
+      float2 wx[4], uh[4];
 #pragma unroll
-    for (int u = 0; u < FWD_U; ++u) h_op[(long)b * ldh + j0 + u] = from_f<T>(hv[u]);
-  if (y) {
-    if ((ldy & 3) == 0 && (j0 + FWD_U <= H || ldy >= Hp)) store4<TY>(y + (long)b * ldy + j0, hv);
-    else
+      for (int g = 0; g < 4; ++g) {
+        wx[g] = *reinterpret_cast<const float2*>(sw + base + g * 64);
+        uh[g] = *reinterpret_cast<const float2*>(su + base + g * 64);
+      }
+      const float2 cp = *reinterpret_cast<const float2*>(sc + ul);
+      float cv[2], hv[2];
 #pragma unroll
-      for (int u = 0; u < FWD_U; ++u)
-        if (j0 + u < H || ldy >= Hp) y[(long)b * ldy + j0 + u] = from_f<TY>(hv[u]);
-  }
+      for (int u = 0; u < 2; ++u) {
+        const int j = u0 + ul + u;
+        if (j < a.H) {
+          float pa[4];
 #pragma unroll
-  for (int u = 0; u < FWD_U; ++u) {
-    if (j0 + u >= H) break;
-    if (hT) hT[(long)b * H + j0 + u] = hv[u];
-    if (cT) cT[(long)b * H + j0 + u] = cv[u];
+          for (int g = 0; g < 4; ++g) {
+            const int pi = g * FB_UB + ul + u;
+            pa[g] = preact<KIND>(u ? wx[g].y : wx[g].x, u ? uh[g].y : uh[g].x, prm[pi],
+                                 KIND == K_MILSTM ? prm[(NP > 1 ? 1 : 0) * 4 * FB_UB + pi] : 0.f,
+                                 KIND == K_MILSTM ? prm[(NP > 2 ? 2 : 0) * 4 * FB_UB + pi] : 0.f,
+                                 KIND == K_MILSTM ? prm[(NP > 3 ? 3 : 0) * 4 * FB_UB + pi] : 0.f);
+          }
+          cell_fwd<KIND, FastMath<T>::value>(pa, u ? cp.y : cp.x, cv[u], hv[u]);
+        } else {   // padding units stay exactly zero
+          cv[u] = 0.f;
+          hv[u] = 0.f;
+        }
+      }
+      const int j = u0 + ul;
+      *reinterpret_cast<float2*>(a.c_new + b * a.Hp + j) = make_float2(cv[0], cv[1]);
+      store_pair<T>(reinterpret_cast<T*>(a.h_op) + b * a.ldh + j, vh, hv[0], hv[1], true);
+      if (a.y) {
+        const bool ok0 = j < a.H || a.ldy >= a.Hp, ok1 = j + 1 < a.H || a.ldy >= a.Hp;
+        if (ok0) store_pair<TY>(reinterpret_cast<TY*>(a.y) + b * a.ldy + j, vy && ok1, hv[0], hv[1], ok1);
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        if (j + u >= a.H) break;
+        if (a.hT) a.hT[b * a.H + j + u] = hv[u];
+        if (a.cT) a.cT[b * a.H + j + u] = cv[u];
+      }
+    }
+    __syncthreads();   // stage s fully consumed
+    if (tid == 0 && k + FB_STAGES < nitems) {
+      sm100::fence_proxy_async_smem();
+      issue(k + FB_STAGES);
+    }
   }
 }
 
@@ -188,13 +277,26 @@ template <int KIND, typename T>
 static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
                           const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, float* hT,
                           float* cT, cudaStream_t st) {
-  dim3 grid(cdiv(Hp, 128 * FWD_U), B);
-  if (y_ot == OT::BF16)
-    lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
-                                                                     ldh, (__nv_bfloat16*)y, ldy, hT, cT);
-  else
-    lstm_fwd_pw_kernel<KIND, T, float><<<grid, 128, 0, st>>>(B, H, Hp, WX, UH, gp, c_prev, c_new, (T*)h_op,
-                                                             ldh, (float*)y, ldy, hT, cT);
+  FwdPwArgs a;
+  a.B = B; a.H = H; a.Hp = Hp;
+  a.nub = cdiv(Hp, FB_UB);
+  a.rstep = std::max(1, std::min(B, 2 * num_sms() / a.nub));
+  a.WX = WX; a.UH = UH; a.gp = gp; a.c_prev = c_prev; a.c_new = c_new;
+  a.h_op = h_op; a.ldh = ldh; a.y = y; a.ldy = ldy; a.hT = hT; a.cT = cT;
+  const int np = KIND == K_MILSTM ? 4 : 1;
+  const size_t smem = (size_t)FB_STAGES * FB_STAGE + (size_t)np * 4 * FB_UB * 4 + FB_STAGES * 8;
+  const dim3 grid(a.nub * a.rstep);
+  if (y_ot == OT::BF16) {
+    auto k = lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16>;
+    static bool attr = false;
+    if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
+    launch_pdl(k, grid, dim3(FB_THREADS), smem, st, 1, a);
+  } else {
+    auto k = lstm_fwd_pw_kernel<KIND, T, float>;
+    static bool attr = false;
+    if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
+    launch_pdl(k, grid, dim3(FB_THREADS), smem, st, 1, a);
+  }
   LAUNCH_CHECK();
 }
 
@@ -222,28 +324,6 @@ constexpr int BWD_TX = 32;  // threads along units: thread tx owns units 2tx, 2t
 constexpr int BWD_RY = 8;   // row lanes per CTA (threadIdx.y); thread handles rows b0 + ty + 8i
 int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 
-template <typename T>
-__device__ __forceinline__ void store2cs(T* p, float a, float b);
-template <>
-__device__ __forceinline__ void store2cs<float>(float* p, float a, float b) {
-  __stcs(reinterpret_cast<float2*>(p), make_float2(a, b));
-}
-template <>
-__device__ __forceinline__ void store2cs<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
-  __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
-  __stcs(reinterpret_cast<unsigned int*>(p), *reinterpret_cast<unsigned int*>(&v));
-}
-template <typename T>
-__device__ __forceinline__ void store2(T* p, float a, float b);
-template <>
-__device__ __forceinline__ void store2<float>(float* p, float a, float b) {
-  *reinterpret_cast<float2*>(p) = make_float2(a, b);
-}
-template <>
-__device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
-  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);
-}
-
 // K4 backward half + K5 column partials.  CTA = 64 hidden units (all four gates) x 32 batch rows;
 // thread (tx, ty) handles units 2tx, 2tx+1 (8-byte loads of every gate's pre-activations) for rows
 // b0 + ty, b0 + ty + 8, ...  Column partial sums (db, dα, dβ1, dβ2) are accumulated per (thread,
@@ -262,6 +342,8 @@ __global__ void __launch_bounds__(BWD_TX * BWD_RY, 4)
   constexpr int NV = KIND == K_MILSTM ? 16 : 4;   // accumulated quantities per unit: q*4 + gate
   __shared__ float red[BWD_RY][NV][2][BWD_TX];     // [row lane][quantity][unit parity][tx]
   __shared__ float prm[KIND == K_MILSTM ? 4 : 1][4][BWD_UX];
+  pdl_wait();
+  pdl_trigger();
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * BWD_TX + tx;
   const int u0 = blockIdx.x * BWD_UX;
   const int j0 = u0 + 2 * tx;
@@ -395,13 +477,13 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
   dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
   dim3 block(BWD_TX, BWD_RY);
   if (dy_f32 || dy_ot == OT::F32)
-    lstm_bwd_pw_kernel<KIND, T, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX,
-                                                             UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials,
-                                                             nq, first);
+    launch_pdl(lstm_bwd_pw_kernel<KIND, T, float>, grid, block, 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec,
+               ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq,
+               (int)first);
   else
-    lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16><<<grid, block, 0, st>>>(B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec,
-                                                                     ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh,
-                                                                     (T*)D_wx, partials, nq, first);
+    launch_pdl(lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16>, grid, block, 0, st, 1, B, H, Hp,
+               (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp,
+               (T*)D_uh, (T*)D_wx, partials, nq, (int)first);
   LAUNCH_CHECK();
 }
 

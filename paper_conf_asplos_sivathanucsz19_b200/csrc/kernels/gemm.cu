@@ -156,19 +156,8 @@ static void launch_pair(const TcGemm& g, const EpiStore& epi, int az, int bz, cu
   int pairs = num_sms() / 2;
   if (max_ctas > 0 && max_ctas / 2 < pairs) pairs = max_ctas / 2 > 0 ? max_ctas / 2 : 1;
   if (ptiles < pairs) pairs = ptiles;
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(2 * pairs);
-  cfg.blockDim = dim3(TC_THREADS);
-  cfg.dynamicSmemBytes = g.smem;
-  cfg.stream = st;
-  cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeClusterDimension;
-  attr[0].val.clusterDim.x = 2;
-  attr[0].val.clusterDim.y = 1;
-  attr[0].val.clusterDim.z = 1;
-  cfg.attrs = attr;
-  cfg.numAttrs = 1;
-  CUDA_TRY(cudaLaunchKernelEx(&cfg, tc_gemm2_kernel<BN, EpiStore>, g.mapA, g.mapB, mapC, a, e));
+  launch_pdl(tc_gemm2_kernel<BN, EpiStore>, dim3(2 * pairs), dim3(TC_THREADS), g.smem, st, 2, g.mapA, g.mapB, mapC, a,
+             e);
   LAUNCH_CHECK();
 }
 
@@ -193,23 +182,7 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   if (max_ctas > 0 && max_ctas / cs < clusters) clusters = max_ctas / cs > 0 ? max_ctas / cs : 1;
   if (ctiles < clusters) clusters = ctiles;
   const int grid = clusters * cs;
-  if (cs == 1) {
-    tc_gemm_kernel<BN, EpiStore><<<grid, TC_THREADS, g.smem, st>>>(g.mapA, g.mapB, mapC, a, e);
-  } else {
-    cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(grid);
-    cfg.blockDim = dim3(TC_THREADS);
-    cfg.dynamicSmemBytes = g.smem;
-    cfg.stream = st;
-    cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = cs;
-    attr[0].val.clusterDim.y = 1;
-    attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    CUDA_TRY(cudaLaunchKernelEx(&cfg, tc_gemm_kernel<BN, EpiStore>, g.mapA, g.mapB, mapC, a, e));
-  }
+  launch_pdl(tc_gemm_kernel<BN, EpiStore>, dim3(grid), dim3(TC_THREADS), g.smem, st, cs, g.mapA, g.mapB, mapC, a, e);
   LAUNCH_CHECK();
 }
 

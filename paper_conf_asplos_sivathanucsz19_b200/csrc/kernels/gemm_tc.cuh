@@ -20,6 +20,7 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 
+#include "pdl.cuh"
 #include "sm100.cuh"
 
 namespace astra {
@@ -299,6 +300,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (cs > 1) sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();      // operands / outputs may belong to the previous kernel in the stream
+  pdl_trigger();
   if (threadIdx.x == 0) GEMM_TRACE(1);
 
   if (warp == 0) {
@@ -494,6 +497,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_wait();
+  pdl_trigger();
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer (both CTAs)
