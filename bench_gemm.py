@@ -3,6 +3,7 @@ and at the paper's Table 1 / fusion-example shapes, 
 width / cluster shape.  Device time from CUDA events over many back-to-back launches.
 
   python bench_gemm.py [--quick]
+Launches are replayed from a CUDA graph (no host overhead in the device time).
 Prints one JSON line per (shape, layout, config) with TFLOP/s and the fraction of the measured
 bf16 peak (MEASURED_PEAKS.json, burst figure: kernels timed alone).
 """
@@ -51,11 +52,17 @@ def run(name, M, N, K, a_mn, b_mn, cfgs, reps):
         try:
             for _ in range(3):
                 A.gemm_bf16_ex(As, Bs, M, N, K, a_mn, b_mn, bn, cm, cn, cg, out=out)
+            torch.cuda.synchronize()
+            # replay the launches from a CUDA graph: device time without host launch overhead
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                for _ in range(reps):
+                    A.gemm_bf16_ex(As, Bs, M, N, K, a_mn, b_mn, bn, cm, cn, cg, out=out)
+            g.replay()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             torch.cuda.synchronize()
             e0.record()
-            for _ in range(reps):
-                A.gemm_bf16_ex(As, Bs, M, N, K, a_mn, b_mn, bn, cm, cn, cg, out=out)
+            g.replay()
             e1.record()
             torch.cuda.synchronize()
             ms = e0.elapsed_time(e1) / reps
@@ -70,10 +77,14 @@ def run(name, M, N, K, a_mn, b_mn, cfgs, reps):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--all", action="store_true")
+    ap.add_argument("--shapes", default="", help="comma-separated substrings of shape names to run")
     args = ap.parse_args()
     for s in SHAPES:
+        if args.shapes and not any(k in s[0] for k in args.shapes.split(",")):
+            continue
         big = s[1] * s[2] * s[3] > 1e11
-        run(*s, CONFIGS[:5] if args.quick else CONFIGS, 5 if big else 50)
+        run(*s, CONFIGS[:5] if args.quick else CONFIGS if args.all else CONFIGS, 5 if big else 50)
 
 
 if __name__ == "__main__":
