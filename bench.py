@@ -42,6 +42,16 @@ def peaks():
         return 1590.0, 1400.0, 6650.0, "fallback (B200_PROFILING.md)"
 
 
+def a1_traffic():
+    """DRAM bytes (read + write) per launch of the a1 GEMM from the committed ncu --set full capture
+    (profiles/r1_roofline_traffic.json, written by profiles/ncu_metrics.py from the .ncu-rep)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r1_roofline_traffic.json")) as f:
+            return json.load(f)["a1_dram_bytes_per_launch"]
+    except Exception:
+        return None
+
+
 class Clocks:
     """nvidia-smi clock/throttle sampling during the timed region (B200_PROFILING.md clocks line)."""
 
@@ -280,9 +290,11 @@ def main():
             "random-init weights)", "config": cfg,
             "tokens_per_s": value * T,
             "roofline": {"bound": "tensor", "kernel": "K1 tcgen05 GEMM, hoisted input projection a1 "
-                         f"[{T*B}x{I}]x[{I}x{4*H}]", "achieved": a1_tf, "peak": sustained, "unit": "TFLOP/s",
-                         "frac": (a1_tf / sustained) if a1_tf else None, "traffic": None,
-                         "peak_source": f"{src} bf16_tflops_sustained (kernel timed inside a long step)",
+                         f"[{T*B}x{I}]x[{I}x{4*H}]", "achieved": a1_tf, "peak": burst, "unit": "TFLOP/s",
+                         "frac": (a1_tf / burst) if a1_tf else None, "traffic": a1_traffic(),
+                         "peak_source": f"{src} bf16_tflops (burst): a1 is the first GEMM of a step launched after "
+                                        "a device synchronize, so it runs at burst clocks (it exceeds the "
+                                        f"sustained figure {sustained})",
                          "step_tflops": step_tf, "step_frac_of_sustained": step_tf / (sustained * args.gpus)},
             "regions_ms": region,
             "e2e": {"value": B_g / (ms_e2e / 1e3), "unit": "samples/s", "h2d_bytes_per_step": int(tok_host.numel() * 4),

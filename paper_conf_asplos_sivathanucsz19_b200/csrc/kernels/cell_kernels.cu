@@ -764,6 +764,33 @@ void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int
   LAUNCH_CHECK();
 }
 
+// ============================================================================ split-K partial sums
+// out[i] = Σ_k part[k][i] in ascending k (the fixed chunk order of R25 / R28).
+__global__ void sum_split_partials_kernel(const float4* __restrict__ part, int ks, long n4, float4* __restrict__ out) {
+  const long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n4) return;
+  float4 v = part[i];
+  for (int k = 1; k < ks; ++k) {
+    const float4 q = part[(long)k * n4 + i];
+    v.x = __fadd_rn(v.x, q.x); v.y = __fadd_rn(v.y, q.y); v.z = __fadd_rn(v.z, q.z); v.w = __fadd_rn(v.w, q.w);
+  }
+  out[i] = v;
+}
+__global__ void sum_split_partials1_kernel(const float* __restrict__ part, int ks, long n, float* __restrict__ out) {
+  const long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  float v = part[i];
+  for (int k = 1; k < ks; ++k) v = __fadd_rn(v, part[(long)k * n + i]);
+  out[i] = v;
+}
+void sum_split_partials(const float* part, int ks, long n, float* out, cudaStream_t st) {
+  if ((n & 3) == 0 && (((uintptr_t)part | (uintptr_t)out) & 15) == 0)
+    sum_split_partials_kernel<<<(unsigned)cdiv(n / 4, 256), 256, 0, st>>>((const float4*)part, ks, n / 4, (float4*)out);
+  else
+    sum_split_partials1_kernel<<<(unsigned)cdiv(n, 256), 256, 0, st>>>(part, ks, n, out);
+  LAUNCH_CHECK();
+}
+
 // ============================================================================ SGD
 __global__ void sgd_kernel(float* __restrict__ p, const float* __restrict__ g, size_t n, float lr) {
   const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;

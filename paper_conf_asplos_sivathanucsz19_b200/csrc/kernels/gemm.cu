@@ -1,7 +1,9 @@
 // Host side of K1 (tcgen05 GEMM) and K10 (SIMT fp32 GEMM).
 #include <cuda.h>
 #include <cudaTypedefs.h>
+#include <cstdlib>
 #include <cstring>
+#include <algorithm>
 #include <mutex>
 #include <tuple>
 #include <map>
@@ -115,6 +117,11 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
   if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm / cg);
   g.args.cg = cg;
+  static const int gm_env = [] {
+    const char* e = std::getenv("ASTRA_GM");   // raster group override (A/B runs)
+    return e ? std::max(1, std::atoi(e)) : 8;
+  }();
+  g.args.gm = gm_env;
   g.args.cm = cm;
   g.args.cn = cn;
   g.args.b_keep = b_keep ? 1 : 0;

@@ -54,8 +54,22 @@ struct TcArgs {
   int b_keep;       // 1: load B with an L2 evict_last policy (weights re-read every step)
   int ksplit;       // fixed split of K into ksplit chunks; chunk ks writes its fp32 partial to C + ks·split_stride
   int cg;           // 1: one CTA per 128 x BN tile; 2: CTA pair per 256 x BN tile (tc_gemm2_kernel)
+  int gm;           // raster group: tiles walk gm M-tiles of one N column before the next column
   uint32_t idesc;
 };
+
+// Grouped raster of the persistent tile loop: tile c1 → (mi, ni) walking `gm` consecutive M-tiles
+// down one N column, then the next column, group after group.  The CTAs resident at any time then
+// share a few A row panels and the B columns stay L2-resident, instead of every N column
+// re-streaming all of A from HBM.  Pure scheduling: no effect on any output bit.
+__device__ __forceinline__ void tile_raster(int c1, int nm, int nn, int gm, int& mi, int& ni) {
+  const int per = gm * nn;
+  const int grp = c1 / per, r = c1 % per;
+  const int mb = grp * gm;
+  const int gs = min(gm, nm - mb);
+  mi = mb + r % gs;
+  ni = r / gs;
+}
 
 template <int BN>
 struct TcSmem {
@@ -315,8 +329,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int a_krows = TC_BK / cn, b_krows = TC_BK / cm;  // MN-major: K rows of each 64-wide box
       for (int ct = cluster_id; ct < num_ct; ct += num_clusters) {
         const int ks = ct / num_ct1, c1 = ct % num_ct1;
-        const int m0 = ((c1 % ncm) * cm + rm) * TC_BM;
-        const int n0 = ((c1 / ncm) * cn + rn) * BN;
+        int mi, ni;
+        tile_raster(c1, ncm, ncn, args.gm, mi, ni);
+        const int m0 = (mi * cm + rm) * TC_BM;
+        const int n0 = (ni * cn + rn) * BN;
         const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
         for (int kb = kb0; kb < kb1; ++kb) {
           sm100::mbar_wait(&empty[s], ph ^ 1);
@@ -414,8 +430,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int acc = local & 1;
       const uint32_t use = (uint32_t)(local >> 1);
       const int ks = ct / num_ct1, c1 = ct % num_ct1;
-      const int m0 = ((c1 % ncm) * cm + rm) * TC_BM;
-      const int n0 = ((c1 / ncm) * cn + rn) * BN;
+      int mi, ni;
+      tile_raster(c1, ncm, ncn, args.gm, mi, ni);
+      const int m0 = (mi * cm + rm) * TC_BM;
+      const int n0 = (ni * cn + rn) * BN;
       sm100::mbar_wait(&tfull[acc], use & 1);
       if (warp == 2 && lane == 0) GEMM_TRACE(5);
       sm100::tc_fence_after();
@@ -508,8 +526,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const uint64_t pol = sm100::l2_policy_evict_last();
       for (int ct = pair_id; ct < num_pt; ct += num_pairs) {
         const int ks = ct / num_pt1, c1 = ct % num_pt1;
-        const int m0 = (c1 % num_mp) * 2 * TC_BM + rank * TC_BM;
-        const int n0 = (c1 / num_mp) * BN + rank * BH;
+        int mi, ni;
+        tile_raster(c1, num_mp, args.num_n, args.gm, mi, ni);
+        const int m0 = mi * 2 * TC_BM + rank * TC_BM;
+        const int n0 = ni * BN + rank * BH;
         const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
         for (int kb = kb0; kb < kb1; ++kb) {
           sm100::mbar_wait(&empty[s], ph ^ 1);
@@ -581,8 +601,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       const int acc = local & 1;
       const uint32_t use = (uint32_t)(local >> 1);
       const int ks = ct / num_pt1, c1 = ct % num_pt1;
-      const int m0 = (c1 % num_mp) * 2 * TC_BM + rank * TC_BM;
-      const int n0 = (c1 / num_mp) * BN;
+      int mi, ni;
+      tile_raster(c1, num_mp, args.num_n, args.gm, mi, ni);
+      const int m0 = mi * 2 * TC_BM + rank * TC_BM;
+      const int n0 = ni * BN;
       sm100::mbar_wait(&tfull[acc], use & 1);
       sm100::tc_fence_after();
       const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * BN;

@@ -176,8 +176,9 @@ class LM {
   size_t n_cell, n_params;
   std::vector<ParamInfo> params;
   size_t off_logits, off_dlog, off_dlog32, off_rowloss, off_dY, off_Wo, off_colsum, off_sort, off_h, off_c,
-      off_cellsaved, off_cellscratch, off_loss, off_embpart, off_dx, ws_bytes;
+      off_cellsaved, off_cellscratch, off_loss, off_embpart, off_dx, off_wopart, ws_bytes;
   size_t sort_bytes;
+  int wo_ksplit = 1;   // fixed split of the head weight-gradient GEMM over K = T·B (reading R28)
   float* P = nullptr;
   float* G = nullptr;
   char* ws = nullptr;
@@ -186,6 +187,25 @@ class LM {
   void bind(float* params, float* grads, void* workspace);
   void set_state(const float* h, const float* c);
   void step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd);
+  void enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd);
+  ~LM();
+
+  // CUDA-graph replay of a frozen step (no exploration): the whole step — every kernel, the side
+  // and comm stream forks/joins, the NCCL buckets, the region events — is captured once per
+  // (tokens, lr, loss, sgd, variant) and replayed with one cudaGraphLaunch, removing the host's
+  // per-kernel launch cost (~10 µs per step-kernel at cfg5) from the critical path.
+  struct GraphEntry {
+    const int32_t* tokens;
+    float lr;
+    float* loss;
+    bool sgd;
+    std::string variant;
+    cudaGraphExec_t exec;
+    uint64_t launches;
+  };
+  std::vector<GraphEntry> graphs;
+  cudaStream_t cap_st = nullptr;
+  void clear_graphs();
 };
 
 }  // namespace astra

@@ -144,7 +144,14 @@ void Cell::bind(float* pp, float* gg, void* sv_p, void* sc_p) {
 
 void Cell::mark(Region r, int which, cudaStream_t st) {
   if (!profiling) return;
-  CUDA_TRY(cudaEventRecord(ev[r][which], st));
+  // External: inside a CUDA-graph capture this becomes a real event-record node (replays keep
+  // timing the regions); outside a capture it is a plain record
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  CUDA_TRY(cudaStreamIsCapturing(st, &cs));
+  if (cs == cudaStreamCaptureStatusActive)
+    CUDA_TRY(cudaEventRecordWithFlags(ev[r][which], st, cudaEventRecordExternal));
+  else
+    CUDA_TRY(cudaEventRecord(ev[r][which], st));
   if (which) region_used[r] = true;
 }
 

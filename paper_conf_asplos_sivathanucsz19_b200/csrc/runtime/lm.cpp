@@ -2,6 +2,9 @@
 // cell forward → head GEMM + mean cross-entropy → head backward → cell BPTT → embedding backward →
 // gradient sum over ranks → SGD.  Works for every cell family through the Cell hooks
 // (x_operand / y_operand / y_segments).
+#include <algorithm>
+#include <cstdlib>
+
 #include "cell.h"
 
 namespace astra {
@@ -41,6 +44,17 @@ LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
   off_c = w.take((size_t)c->B * (c->c_width() > 0 ? c->c_width() : 1) * 4);
   off_loss = w.take(256);
   off_dx = w.take((size_t)TB * c->Ip * 4);
+  // R28: dW_o = Yᵀ·dlogits has few output tiles (Hout x V) and a long K = T·B; a fixed split of K
+  // into wo_ksplit chunks (partials summed in chunk order) lets it use the whole GPU.  The split
+  // depends only on the shapes, so every variant (and the fp32 path) computes the same sums.
+  {
+    int maxn = 0;
+    for (const KSeg& sg : c->y_segments()) maxn = std::max(maxn, sg.n);
+    const long tiles = (long)cdiv(maxn, 256) * cdiv(V, 256);
+    const int kb = cdiv(TB, 64);
+    wo_ksplit = (int)std::max(1L, std::min(std::min(64L / std::max(1L, tiles), 16L), (long)kb / 8));
+    off_wopart = w.take((size_t)wo_ksplit * maxn * V * 4);
+  }
   ws_bytes = w.o;
 }
 
@@ -70,9 +84,78 @@ void LM::set_state(const float* h, const float* c) {
   }
 }
 
+static bool graphs_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("ASTRA_GRAPH");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
+void LM::clear_graphs() {
+  for (auto& g : graphs) cudaGraphExecDestroy(g.exec);
+  graphs.clear();
+}
+
+LM::~LM() {
+  clear_graphs();
+  if (cap_st) cudaStreamDestroy(cap_st);
+}
+
 void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   ASTRA_CHECK_STATE(bound, "lm_train_step: not bound");
   ASTRA_CHECK_ARG(tokens, "lm_train_step: tokens is null");
+  Cell& c = *cell;
+  // exploration steps (and the fp32 parity path) run eagerly; a frozen / untuned bf16 step replays
+  if (!graphs_enabled() || c.tune_mode == ASTRA_TUNE_ON || c.ot != OT::BF16) {
+    enqueue_step(tokens, lr, loss_dev, do_sgd);
+    return;
+  }
+  const std::string vs = c.var.str();
+  for (auto& g : graphs)
+    if (g.tokens == tokens && g.lr == lr && g.loss == loss_dev && g.sgd == do_sgd && g.variant == vs) {
+      CUDA_TRY(cudaGraphLaunch(g.exec, c.main_st));
+      count_launch(g.launches);
+      return;
+    }
+  if (!cap_st) CUDA_TRY(cudaStreamCreateWithFlags(&cap_st, cudaStreamNonBlocking));
+  // the captured work must follow everything already queued on the caller's stream
+  cudaEvent_t e0;
+  CUDA_TRY(cudaEventCreateWithFlags(&e0, cudaEventDisableTiming));
+  CUDA_TRY(cudaEventRecord(e0, c.main_st));
+  CUDA_TRY(cudaStreamWaitEvent(cap_st, e0, 0));
+  CUDA_TRY(cudaEventDestroy(e0));
+  cudaStream_t user = c.main_st;
+  c.main_st = cap_st;
+  const uint64_t l0 = g_launches.load();
+  cudaGraph_t graph = nullptr;
+  CUDA_TRY(cudaStreamBeginCapture(cap_st, cudaStreamCaptureModeThreadLocal));
+  try {
+    enqueue_step(tokens, lr, loss_dev, do_sgd);
+  } catch (...) {
+    cudaStreamEndCapture(cap_st, &graph);
+    if (graph) cudaGraphDestroy(graph);
+    c.main_st = user;
+    throw;
+  }
+  c.main_st = user;
+  CUDA_TRY(cudaStreamEndCapture(cap_st, &graph));
+  GraphEntry ge;
+  ge.tokens = tokens; ge.lr = lr; ge.loss = loss_dev; ge.sgd = do_sgd; ge.variant = vs;
+  ge.launches = g_launches.load() - l0;
+  CUDA_TRY(cudaGraphInstantiate(&ge.exec, graph, 0));
+  CUDA_TRY(cudaGraphDestroy(graph));
+  g_launches.fetch_sub(ge.launches);   // captured, not yet launched
+  if (graphs.size() >= 4) {
+    cudaGraphExecDestroy(graphs.front().exec);
+    graphs.erase(graphs.begin());
+  }
+  graphs.push_back(ge);
+  CUDA_TRY(cudaGraphLaunch(ge.exec, c.main_st));
+  count_launch(ge.launches);
+}
+
+void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   Cell& c = *cell;
   cudaStream_t st = c.main_st;
   const long TB = (long)c.T * c.B;
@@ -123,7 +206,17 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
     dwo.B = mat(dlog, V, TB, Vp);
     dwo.b_mn = true;
     dwo.M = s.n; dwo.N = V; dwo.K = (int)TB;
-    c.run_gemm(id++, dwo, epi(G + find("W_o") + (size_t)s.r0 * V, V, s.n, V), 0, 0, c.var.g[G_HEAD], st);
+    dwo.ksplit = wo_ksplit;
+    float* dWo = G + find("W_o") + (size_t)s.r0 * V;
+    if (wo_ksplit > 1) {
+      float* part = (float*)(ws + off_wopart);
+      EpiStore ep = epi(part, V, s.n, V);
+      ep.split_stride = (long)s.n * V;
+      c.run_gemm(id++, dwo, ep, 0, 0, c.var.g[G_HEAD], st);
+      sum_split_partials(part, wo_ksplit, (long)s.n * V, dWo, st);
+    } else {
+      c.run_gemm(id++, dwo, epi(dWo, V, s.n, V), 0, 0, c.var.g[G_HEAD], st);
+    }
   }
   colsum(dlog32, TB, V, V, (float*)(ws + off_colsum), G + find("b_o"), st);
   c.mark(R_HEAD, 1, st);
