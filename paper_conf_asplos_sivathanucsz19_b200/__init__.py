@@ -84,9 +84,10 @@ def lib():
     """Load lib/libastra.so (raises if it has not been built — no fallback)."""
     global _lib
     if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            raise ImportError(f"{LIB_PATH} not built: run `python -m paper_conf_asplos_sivathanucsz19_b200.build`")
-        L = ctypes.CDLL(LIB_PATH)
+        path = os.environ.get("ASTRA_LIB_OVERRIDE") or LIB_PATH   # A/B runs against another in-tree build
+        if not os.path.exists(path):
+            raise ImportError(f"{path} not built: run `python -m paper_conf_asplos_sivathanucsz19_b200.build`")
+        L = ctypes.CDLL(path)
         for name, args in _SIGS.items():
             f = getattr(L, name)
             f.argtypes = args

@@ -216,6 +216,18 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   const bool act = ul < nu;
   const int base = (ul / 64) * 256 + ul % 64;
   const bool vh = (a.ldh & 1) == 0, vy = (a.ldy & 1) == 0;
+  // this thread's units keep their gate parameters in registers for all its rows
+  float pb[2][4], pal[2][4], pb1[2][4], pb2[2][4];
+#pragma unroll
+  for (int u = 0; u < 2; ++u)
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      const int pi = act ? g * FB_UB + ul + u : 0;
+      pb[u][g] = prm[pi];
+      pal[u][g] = KIND == K_MILSTM ? prm[(NP > 1 ? 1 : 0) * 4 * FB_UB + pi] : 0.f;
+      pb1[u][g] = KIND == K_MILSTM ? prm[(NP > 2 ? 2 : 0) * 4 * FB_UB + pi] : 0.f;
+      pb2[u][g] = KIND == K_MILSTM ? prm[(NP > 3 ? 3 : 0) * 4 * FB_UB + pi] : 0.f;
+    }
   for (int k = 0; k < nitems; ++k) {
     const int s = k % FB_STAGES;
     sm100::mbar_wait(&full[s], (uint32_t)((k / FB_STAGES) & 1));
@@ -238,13 +250,9 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
         if (j < a.H) {
           float pa[4];
 #pragma unroll
-          for (int g = 0; g < 4; ++g) {
-            const int pi = g * FB_UB + ul + u;
-            pa[g] = preact<KIND>(u ? wx[g].y : wx[g].x, u ? uh[g].y : uh[g].x, prm[pi],
-                                 KIND == K_MILSTM ? prm[(NP > 1 ? 1 : 0) * 4 * FB_UB + pi] : 0.f,
-                                 KIND == K_MILSTM ? prm[(NP > 2 ? 2 : 0) * 4 * FB_UB + pi] : 0.f,
-                                 KIND == K_MILSTM ? prm[(NP > 3 ? 3 : 0) * 4 * FB_UB + pi] : 0.f);
-          }
+          for (int g = 0; g < 4; ++g)
+            pa[g] = preact<KIND>(u ? wx[g].y : wx[g].x, u ? uh[g].y : uh[g].x, pb[u][g], pal[u][g], pb1[u][g],
+                                 pb2[u][g]);
           cell_fwd<KIND, FastMath<T>::value>(pa, u ? cp.y : cp.x, cv[u], hv[u]);
         } else {   // padding units stay exactly zero
           cv[u] = 0.f;
