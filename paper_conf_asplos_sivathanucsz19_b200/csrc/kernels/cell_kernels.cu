@@ -327,151 +327,109 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
 }
 
 constexpr int BWD_RB = 32;  // rows per CTA in the backward pointwise kernel (= one partial chunk)
-constexpr int BWD_UX = 64;  // units per CTA (one gate group)
-constexpr int BWD_TX = 32;  // threads along units: thread tx owns units 2tx, 2tx+1 of the group
-constexpr int BWD_RY = 8;   // row lanes per CTA (threadIdx.y); thread handles rows b0 + ty + 8i
+constexpr int BWD_UX = 64;  // units per CTA (one gate group); thread tx owns unit u0 + tx
+constexpr int BWD_RY = 4;   // row lanes per CTA (threadIdx.y); thread handles rows b0 + ty + 4i
 int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 
 // K4 backward half + K5 column partials.  CTA = 64 hidden units (all four gates) x 32 batch rows;
-// thread (tx, ty) handles units 2tx, 2tx+1 (8-byte loads of every gate's pre-activations) for rows
-// b0 + ty, b0 + ty + 8, ...  Column partial sums (db, dα, dβ1, dβ2) are accumulated per (thread,
-// unit) in thread-private shared-memory slots in ascending row order, combined across the 8 row
-// lanes in ty order, and added to partials[chunk][q][col] — one owner per element, steps ordered on
-// the stream, so the reduction order is fixed (R5: no floating-point atomics).  256-thread CTAs
-// with shared-memory accumulators keep the register count low enough that the whole grid of a
-// 512-row batch is resident in one wave.
+// thread (tx, ty) owns unit u0 + tx (its 4 gates' parameters in registers) for rows b0 + ty,
+// b0 + ty + 4, ...; a warp reads 128-byte runs of every gate's pre-activations.  Column partial
+// sums (db, dα, dβ1, dβ2) are accumulated per thread in ascending row order in its own shared-
+// memory slots, combined across the 4 row lanes in ty order, and added to partials[chunk][q][col]
+// — one owner per element, steps ordered on the stream, so the reduction order is fixed (R5: no
+// floating-point atomics).  256-thread CTAs at <= 64 registers: one resident wave at B = 512.
 template <int KIND, typename T, typename TDY>
-__global__ void __launch_bounds__(BWD_TX * BWD_RY, 4)
+__global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
     lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
                        long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
                        const float* __restrict__ WX, const float* __restrict__ UH, const float* __restrict__ c_new,
                        const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
                        T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
   constexpr int NV = KIND == K_MILSTM ? 16 : 4;   // accumulated quantities per unit: q*4 + gate
-  __shared__ float red[BWD_RY][NV][2][BWD_TX];     // [row lane][quantity][unit parity][tx]
-  __shared__ float prm[KIND == K_MILSTM ? 4 : 1][4][BWD_UX];
+  __shared__ float red[BWD_RY][NV][BWD_UX];
   pdl_wait();
   pdl_trigger();
-  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * BWD_TX + tx;
-  const int u0 = blockIdx.x * BWD_UX;
-  const int j0 = u0 + 2 * tx;
+  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int j = blockIdx.x * BWD_UX + tx;
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
-  for (int i = tid; i < 4 * BWD_UX; i += BWD_TX * BWD_RY) {
-    const int g = i / BWD_UX, ul = i % BWD_UX, j = u0 + ul, e = g * H + j;
-    const bool v = j < H;
-    prm[0][g][ul] = v ? gp.b[e] : 0.f;
-    if (KIND == K_MILSTM) {
-      prm[KIND == K_MILSTM ? 1 : 0][g][ul] = v ? gp.alpha[e] : 0.f;
-      prm[KIND == K_MILSTM ? 2 : 0][g][ul] = v ? gp.beta1[e] : 0.f;
-      prm[KIND == K_MILSTM ? 3 : 0][g][ul] = v ? gp.beta2[e] : 0.f;
-    }
-  }
 #pragma unroll
-  for (int i = 0; i < NV; ++i) {
-    red[ty][i][0][tx] = 0.f;
-    red[ty][i][1][tx] = 0.f;
-  }
-  __syncthreads();
-  if (j0 < Hp) {
-    const bool v0 = j0 < H, v1 = j0 + 1 < H;
-    const bool vec_dh = ((ld_dh | split_stride) & 1) == 0;
+  for (int i = 0; i < NV; ++i) red[ty][i][tx] = 0.f;
+  if (j < H) {
+    float bb[4], al[4], be1[4], be2[4];
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      const int e = g * H + j;
+      bb[g] = gp.b[e];
+      al[g] = KIND == K_MILSTM ? gp.alpha[e] : 0.f;
+      be1[g] = KIND == K_MILSTM ? gp.beta1[e] : 0.f;
+      be2[g] = KIND == K_MILSTM ? gp.beta2[e] : 0.f;
+    }
+    const int c0 = gcol(0, j);
+#pragma unroll 1
     for (int b = b0 + ty; b < b1; b += BWD_RY) {
-      const long rg = (long)b * NG;
-      float2 wx[4], uh[4];
+      const float* wxp = WX + (long)b * NG + c0;
+      const float* uhp = UH + (long)b * NG + c0;
+      float w[4], h[4], a[4];
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
-        wx[g] = __ldcs(reinterpret_cast<const float2*>(WX + rg + gcol(g, j0)));
-        uh[g] = __ldcs(reinterpret_cast<const float2*>(UH + rg + gcol(g, j0)));
+        w[g] = __ldcs(wxp + g * GATE_U);
+        h[g] = __ldcs(uhp + g * GATE_U);
       }
-      float dh[2] = {v0 ? to_f<TDY>(dy[(long)b * ldy + j0]) : 0.f, v1 ? to_f<TDY>(dy[(long)b * ldy + j0 + 1]) : 0.f};
-      if (dh_rec && v0) {   // split-K partials of dh_rec summed in chunk order, then added to dy
-        const float* r0 = dh_rec + (long)b * ld_dh + j0;
-        float r[2];
-        if (vec_dh) {
-          float2 q = *reinterpret_cast<const float2*>(r0);
-          r[0] = q.x; r[1] = q.y;
-          for (int k = 1; k < nsplit; ++k) {
-            q = *reinterpret_cast<const float2*>(r0 + k * split_stride);
-            r[0] = __fadd_rn(r[0], q.x);
-            r[1] = __fadd_rn(r[1], q.y);
-          }
+      float dh = to_f<TDY>(dy[(long)b * ldy + j]);
+      if (dh_rec) {   // split-K partials of dh_rec summed in chunk order, then added to dy
+        const float* r0 = dh_rec + (long)b * ld_dh + j;
+        float r = r0[0];
+        for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, r0[k * split_stride]);
+        dh = __fadd_rn(dh, r);
+      }
+      const long ro = (long)b * Hp + j;
+      float dcv = dc[ro];
+      const float cp = c_prev[ro], cn = c_new[ro];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) a[g] = preact<KIND>(w[g], h[g], bb[g], al[g], be1[g], be2[g]);
+      float da[4];
+      cell_bwd<KIND, FastMath<T>::value>(a, cp, cn, dh, dcv, da);
+      dc[ro] = dcv;
+      T* duhp = D_uh + (long)b * NG + c0;
+      T* dwxp = D_wx + (long)b * NG + c0;
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        red[ty][g][tx] = __fadd_rn(red[ty][g][tx], da[g]);
+        if (KIND == K_MILSTM) {
+          duhp[g * GATE_U] = from_f<T>(__fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], w[g]), be1[g])));
+          __stcs(dwxp + g * GATE_U, from_f<T>(__fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], h[g]), be2[g]))));
+          float* r4 = &red[ty][NV > 4 ? 4 : 0][tx];
+          r4[g * BWD_UX] = __fadd_rn(r4[g * BWD_UX], __fmul_rn(__fmul_rn(da[g], w[g]), h[g]));
+          float* r8 = &red[ty][NV > 8 ? 8 : 0][tx];
+          r8[g * BWD_UX] = __fadd_rn(r8[g * BWD_UX], __fmul_rn(da[g], h[g]));
+          float* r12 = &red[ty][NV > 12 ? 12 : 0][tx];
+          r12[g * BWD_UX] = __fadd_rn(r12[g * BWD_UX], __fmul_rn(da[g], w[g]));
         } else {
-          r[0] = r0[0];
-          r[1] = v1 ? r0[1] : 0.f;
-          for (int k = 1; k < nsplit; ++k) {
-            r[0] = __fadd_rn(r[0], r0[k * split_stride]);
-            if (v1) r[1] = __fadd_rn(r[1], r0[k * split_stride + 1]);
-          }
-        }
-        dh[0] = __fadd_rn(dh[0], r[0]);
-        dh[1] = __fadd_rn(dh[1], r[1]);
-      }
-      const long ro = (long)b * Hp + j0;
-      const float2 dc2 = *reinterpret_cast<const float2*>(dc + ro);
-      const float2 cp2 = *reinterpret_cast<const float2*>(c_prev + ro);
-      const float2 cn2 = *reinterpret_cast<const float2*>(c_new + ro);
-      float dco[2], duh[2][4], dwx[2][4];
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int ul = 2 * tx + u;
-        if (!(u == 0 ? v0 : v1)) {   // padding unit: its gradients stay exactly zero
-          dco[u] = 0.f;
-#pragma unroll
-          for (int g = 0; g < 4; ++g) duh[u][g] = dwx[u][g] = 0.f;
-          continue;
-        }
-        float a[4], w[4], h[4];
-#pragma unroll
-        for (int g = 0; g < 4; ++g) {
-          w[g] = u == 0 ? wx[g].x : wx[g].y;
-          h[g] = u == 0 ? uh[g].x : uh[g].y;
-          a[g] = preact<KIND>(w[g], h[g], prm[0][g][ul], KIND == K_MILSTM ? prm[KIND == K_MILSTM ? 1 : 0][g][ul] : 0.f,
-                              KIND == K_MILSTM ? prm[KIND == K_MILSTM ? 2 : 0][g][ul] : 0.f,
-                              KIND == K_MILSTM ? prm[KIND == K_MILSTM ? 3 : 0][g][ul] : 0.f);
-        }
-        float dcv = u == 0 ? dc2.x : dc2.y;
-        float da[4];
-        cell_bwd<KIND, FastMath<T>::value>(a, u == 0 ? cp2.x : cp2.y, u == 0 ? cn2.x : cn2.y, dh[u], dcv, da);
-        dco[u] = dcv;
-#pragma unroll
-        for (int g = 0; g < 4; ++g) {
-          red[ty][g][u][tx] = __fadd_rn(red[ty][g][u][tx], da[g]);
-          if (KIND == K_MILSTM) {
-            const float al = prm[KIND == K_MILSTM ? 1 : 0][g][ul], be1 = prm[KIND == K_MILSTM ? 2 : 0][g][ul],
-                        be2 = prm[KIND == K_MILSTM ? 3 : 0][g][ul];
-            duh[u][g] = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al, w[g]), be1));
-            dwx[u][g] = __fmul_rn(da[g], __fadd_rn(__fmul_rn(al, h[g]), be2));
-            red[ty][(KIND == K_MILSTM ? 4 : 0) + g][u][tx] =
-                __fadd_rn(red[ty][(KIND == K_MILSTM ? 4 : 0) + g][u][tx], __fmul_rn(__fmul_rn(da[g], w[g]), h[g]));
-            red[ty][(KIND == K_MILSTM ? 8 : 0) + g][u][tx] =
-                __fadd_rn(red[ty][(KIND == K_MILSTM ? 8 : 0) + g][u][tx], __fmul_rn(da[g], h[g]));
-            red[ty][(KIND == K_MILSTM ? 12 : 0) + g][u][tx] =
-                __fadd_rn(red[ty][(KIND == K_MILSTM ? 12 : 0) + g][u][tx], __fmul_rn(da[g], w[g]));
-          } else {
-            duh[u][g] = da[g];
-            dwx[u][g] = 0.f;
-          }
+          duhp[g * GATE_U] = from_f<T>(da[g]);
         }
       }
-      *reinterpret_cast<float2*>(dc + ro) = make_float2(dco[0], dco[1]);
+    }
+  } else if (j < Hp) {  // padding units: keep their gradients exactly zero
+    for (int b = b0 + ty; b < b1; b += BWD_RY) {
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
-        store2<T>(D_uh + rg + gcol(g, j0), duh[0][g], duh[1][g]);
-        if (KIND == K_MILSTM) store2cs<T>(D_wx + rg + gcol(g, j0), dwx[0][g], dwx[1][g]);
+        D_uh[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
+        if (KIND == K_MILSTM) D_wx[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
       }
+      dc[(long)b * Hp + j] = 0.f;
     }
   }
   __syncthreads();
-  // finalise: (quantity, unit) items; each sums the 8 row lanes in ty order
-  for (int i = tid; i < NV * BWD_UX; i += BWD_TX * BWD_RY) {
-    const int qi = i / BWD_UX, ul = i % BWD_UX, j = u0 + ul;
-    const int q = qi / 4, g = qi % 4;
-    if (j >= Hp || q >= nq) continue;
+  if (j >= Hp) return;
+  // thread (tx, ty) finalises quantities i = ty, ty + 4, ... (fixed ty order inside)
+  for (int i = ty; i < NV; i += BWD_RY) {
     float v = 0.f;
 #pragma unroll
-    for (int yy = 0; yy < BWD_RY; ++yy) v = __fadd_rn(v, red[yy][qi][ul & 1][ul >> 1]);
+    for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[y][i][tx]);
+    const int q = i / 4, g = i % 4;
+    if (q >= nq) continue;
     float* p = partials + ((long)chunk * nq + q) * NG + gcol(g, j);
     *p = first ? v : __fadd_rn(*p, v);
   }
@@ -483,7 +441,7 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
                           bool first, cudaStream_t st) {
   dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
-  dim3 block(BWD_TX, BWD_RY);
+  dim3 block(BWD_UX, BWD_RY);
   if (dy_f32 || dy_ot == OT::F32)
     launch_pdl(lstm_bwd_pw_kernel<KIND, T, float>, grid, block, 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec,
                ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq,
