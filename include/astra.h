@@ -160,6 +160,9 @@ astra_status astra_lm_set_state(astra_lm m, const float* h, const float* c);
 astra_status astra_lm_train_step(astra_lm m, const int32_t* tokens, float lr, float* loss_dev);
 /* Same step without the SGD update (for parity tests of the gradients).                   */
 astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev);
+/* CUDA-graph replay of frozen / untuned bf16 LM steps (default on; ASTRA_GRAPH=0 turns the default
+ * off).  on = 0: every step is enqueued kernel by kernel; results are bitwise identical either way.  */
+astra_status astra_lm_set_graph(astra_lm m, int on);
 
 /* ---- K1 as a plain library GEMM (tests, microbenchmarks of the paper's Table 1 shapes,
  *      P:107-112, and the fusion example P:122) ------------------------------------------ */

@@ -68,6 +68,7 @@ _SIGS = {
     "astra_lm_set_state": [_P, _P, _P],
     "astra_lm_train_step": [_P, _P, _F, _P],
     "astra_lm_fwd_bwd": [_P, _P, _P],
+    "astra_lm_set_graph": [_P, _I],
     "astra_gemm_bf16": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I, _P],
     "astra_gemm_bf16_ex": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I,
                            _I, _I, _P],
@@ -291,6 +292,10 @@ class LM:
     def train_step(self, tokens, lr, loss=None):
         _check(lib().astra_lm_train_step(self.h, _ptr(tokens), lr, _ptr(self.loss if loss is None else loss)))
         return self.loss if loss is None else loss
+
+    def set_graph(self, on: bool):
+        """CUDA-graph replay of frozen steps (see astra_lm_set_graph)."""
+        _check(lib().astra_lm_set_graph(self.h, int(bool(on))))
 
     def fwd_bwd(self, tokens, loss=None):
         _check(lib().astra_lm_fwd_bwd(self.h, _ptr(tokens), _ptr(self.loss if loss is None else loss)))

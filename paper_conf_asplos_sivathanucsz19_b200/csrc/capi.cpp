@@ -254,6 +254,14 @@ astra_status astra_lm_train_step(astra_lm m, const int32_t* tokens, float lr, fl
   return guard([&] { NEED(m); m->m->step(tokens, lr, loss_dev, true); });
 }
 
+astra_status astra_lm_set_graph(astra_lm m, int on) {
+  return guard([&] {
+    NEED(m);
+    m->m->use_graphs = on != 0;
+    if (!on) m->m->clear_graphs();
+  });
+}
+
 astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev) {
   return guard([&] { NEED(m); m->m->step(tokens, 0.f, loss_dev, false); });
 }

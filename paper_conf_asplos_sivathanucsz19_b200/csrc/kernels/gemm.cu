@@ -85,6 +85,24 @@ static bool epi_tma_map(const EpiStore& e, int ksplit, CUtensorMap* out) {
   return true;
 }
 
+void make_tile_map(CUtensorMap* m, const void* ptr, bool bf16, long inner, long rows, long z, long ld, long zstride,
+                   int box_inner, int box_rows, int swizzle_bytes) {
+  ASTRA_CHECK_ARG(ptr != nullptr && ((uintptr_t)ptr & 15) == 0, "tile map: base must be 16-byte aligned");
+  const long esz = bf16 ? 2 : 4;
+  ASTRA_CHECK_ARG((ld * esz) % 16 == 0 && (z == 1 || (zstride * esz) % 16 == 0), "tile map: strides must be 16-byte multiples");
+  cuuint64_t dims[3] = {(cuuint64_t)inner, (cuuint64_t)rows, (cuuint64_t)z};
+  cuuint64_t strides[2] = {(cuuint64_t)(ld * esz), (cuuint64_t)((z > 1 ? zstride : ld * rows) * esz)};
+  cuuint32_t box[3] = {(cuuint32_t)box_inner, (cuuint32_t)box_rows, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  const CUtensorMapSwizzle sw = swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                : swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                : swizzle_bytes == 32 ? CU_TENSOR_MAP_SWIZZLE_32B : CU_TENSOR_MAP_SWIZZLE_NONE;
+  CUresult r = encode_fn()(m, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3,
+                           const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(ASTRA_E_CUDA, "cuTensorMapEncodeTiled (tile map) failed: " + std::to_string((int)r));
+}
+
 static uint32_t make_idesc(int BN, bool a_mn, bool b_mn, int BM = TC_BM) {
   uint32_t d = 0;
   d |= 1u << 4;                      // D format: F32

@@ -42,4 +42,9 @@ void simt_gemm(const float* A, long sam, long sak, const float* B, long sbk, lon
 
 int num_sms();
 
+// 3-D tiled tensor map ([z][rows][inner], row stride ld, slice stride zstride, in elements) with a
+// {box_inner, box_rows, 1} box and the given swizzle (0 / 32 / 64 / 128 bytes) — epilogue I/O maps.
+void make_tile_map(CUtensorMap* m, const void* ptr, bool bf16, long inner, long rows, long z, long ld, long zstride,
+                   int box_inner, int box_rows, int swizzle_bytes);
+
 }  // namespace astra

@@ -26,6 +26,29 @@ struct RecFwdArgs {
   unsigned* flags;          // [num_m] row-block counters (zeroed before a persistent launch)
 };
 
+// CTA-pair fused forward step (rec_fused2.cu): one launch per step t.
+struct RecFwd2Args {
+  int B, H, Hp, NG, T, t;
+  int num_mp, num_n;        // pair tiles: ceil(B/256) x NG/256
+  int stages, nk;
+  uint32_t idesc;           // M = 256, N = 256 bf16 MMA (cta_group::2)
+  int y_kind;               // 0 none, 1 bf16 [T][B][H] via TMA, 2 the same with element stores (H % 8 != 0)
+  void* y;
+  float* hT;
+  float* cT;
+  GateParams gp;
+};
+struct RecFwd2Maps {
+  CUtensorMap A;    // Hb [(T+1)][B][Hp] bf16, K-major, box {64, 128} (z = t)
+  CUtensorMap B;    // U mirror [NG][Hp] bf16, box {64, 128}
+  CUtensorMap WX;   // [T][B][NG] fp32, box {32, 32}, SWIZZLE_128B
+  CUtensorMap UH;   // [T][B][NG] fp32, box {32, 32}, SWIZZLE_128B
+  CUtensorMap C;    // [(T+1)][B][Hp] fp32, box {32, 32}, SWIZZLE_128B
+  CUtensorMap H;    // [(T+1)][B][Hp] bf16, box {32, 32}, SWIZZLE_64B
+  CUtensorMap Y;    // [T][B][H] bf16, box {32, 32}, SWIZZLE_64B (unused when y_kind = 0)
+};
+void lstm_fwd_pair_launch(int kind, const RecFwd2Maps& m, RecFwd2Args a, cudaStream_t st);
+
 // mapA: Hb as a 3-D K-major map (inner Hp, rows B, z = T+1), box {64, 128};
 // mapB: the U mirror [NG][Hp] K-major, box {64, 256}.
 void lstm_rec_fwd_launch(int kind, const CUtensorMap& mapA, const CUtensorMap& mapB, RecFwdArgs a, cudaStream_t st);

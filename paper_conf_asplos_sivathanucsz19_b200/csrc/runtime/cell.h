@@ -204,6 +204,7 @@ class LM {
     uint64_t launches;
   };
   std::vector<GraphEntry> graphs;
+  bool use_graphs = true;
   cudaStream_t cap_st = nullptr;
   void clear_graphs();
 };

@@ -59,6 +59,9 @@ class LstmCell : public Cell {
   int bptt_ksplit() const { return (ot == OT::BF16 && NG >= 8192) ? 4 : (ot == OT::BF16 && NG >= 4096) ? 2 : 1; }
 
   int fwd_fusions() const override { return 3; }
+  RecFwd2Maps fm;                       // tensor maps of the fused CTA-pair forward (built at first use)
+  const void* fm_key = (const void*)1;  // y pointer the maps were built for
+  const void* fm_wx = nullptr;          // workspace they were built for (rebind ⇒ rebuild)
 
   void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
   void* x_operand() override { return sv<char>(off_X); }
@@ -122,7 +125,36 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   rec.B = mat(Um, Hp, NG, Hp);
   rec.M = B; rec.N = NG; rec.K = Hp;
   rec.b_keep = true;
-  if (ot == OT::BF16 && var.fwd_mode > 0) {
+  if (ot == OT::BF16 && var.fwd_mode == 1 && !y_f32) {
+    // K2 fused, CTA-pair form: GEMM + gate epilogue with TMA-staged epilogue I/O, one launch per step
+    const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1, 2});
+    if (fm_key != (const void*)y || fm_wx != (const void*)WX) {
+      fm.A = tg.mapA;
+      fm.B = tg.mapB;
+      make_tile_map(&fm.WX, WX, false, NG, B, T, NG, (long)B * NG, 32, 32, 128);
+      make_tile_map(&fm.UH, UH, false, NG, B, T, NG, (long)B * NG, 32, 32, 128);
+      make_tile_map(&fm.C, Cb, false, Hp, B, T + 1, Hp, (long)B * Hp, 32, 32, 128);
+      make_tile_map(&fm.H, Hrow(0), true, Hp, B, T + 1, Hp, (long)B * Hp, 32, 32, 64);
+      if (y && H % 8 == 0 && ((uintptr_t)y & 15) == 0) make_tile_map(&fm.Y, y, true, H, B, T, H, (long)B * H, 32, 32, 64);
+      else fm.Y = fm.H;
+      fm_key = (const void*)y;
+      fm_wx = (const void*)WX;
+    }
+    RecFwd2Args ra;
+    ra.B = B; ra.H = H; ra.Hp = Hp; ra.NG = NG; ra.T = T;
+    ra.num_mp = cdiv(B, 2 * TC_BM); ra.num_n = NG / 256;
+    ra.idesc = tg.args.idesc;
+    ra.y_kind = !y ? 0 : (H % 8 == 0 && ((uintptr_t)y & 15) == 0) ? 1 : 2;
+    ra.y = y;
+    ra.gp = gp;
+    for (int t = 0; t < T; ++t) {
+      ra.t = t;
+      const bool last = t == T - 1;
+      ra.hT = last ? hT : nullptr;
+      ra.cT = last ? cT : nullptr;
+      lstm_fwd_pair_launch(kind, fm, ra, st);
+    }
+  } else if (ot == OT::BF16 && var.fwd_mode > 0) {
     // K2 fused: GEMM + gate epilogue in one kernel (per step, or persistent over all steps)
     const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1});
     RecFwdArgs ra;

@@ -107,7 +107,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   ASTRA_CHECK_ARG(tokens, "lm_train_step: tokens is null");
   Cell& c = *cell;
   // exploration steps (and the fp32 parity path) run eagerly; a frozen / untuned bf16 step replays
-  if (!graphs_enabled() || c.tune_mode == ASTRA_TUNE_ON || c.ot != OT::BF16) {
+  if (!use_graphs || !graphs_enabled() || c.tune_mode == ASTRA_TUNE_ON || c.ot != OT::BF16) {
     enqueue_step(tokens, lr, loss_dev, do_sgd);
     return;
   }

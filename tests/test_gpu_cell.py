@@ -71,6 +71,13 @@ def test_fused_forward_modes(cell, fwd):
     _check(cell, 6, 260, 64, 192, "bf16", synth.config_seed(5) + 40, TOL_BF16, variant=f"fwd={fwd}")
 
 
+@pytest.mark.parametrize("cell", ["lstm", "milstm", "sublstm"])
+def test_fused_pair_forward_ragged(cell):
+    """The CTA-pair fused forward (fwd=1): ragged batch (a half-empty CTA pair), hidden size not a
+    multiple of the 32-unit epilogue slice (TMA-clipped tails), and the external y output."""
+    _check(cell, 4, 300, 64, 100, "bf16", synth.config_seed(5) + 41, TOL_BF16, variant="fwd=1")
+
+
 def test_variants_bitwise():
     """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
     T, B, I, H = 6, 160, 128, 192
