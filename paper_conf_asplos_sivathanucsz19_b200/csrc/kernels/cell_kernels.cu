@@ -251,7 +251,7 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
           float pa[4];
 #pragma unroll
           for (int g = 0; g < 4; ++g)
-            pa[g] = preact<KIND>(u ? wx[g].y : wx[g].x, u ? uh[g].y : uh[g].x, pb[u][g], pal[u][g], pb1[u][g],
+            pa[g] = preact<KIND, FastMath<T>::value>(u ? wx[g].y : wx[g].x, u ? uh[g].y : uh[g].x, pb[u][g], pal[u][g], pb1[u][g],
                                  pb2[u][g]);
           cell_fwd<KIND, FastMath<T>::value>(pa, u ? cp.y : cp.x, cv[u], hv[u]);
         } else {   // padding units stay exactly zero
@@ -388,7 +388,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
       float dcv = dc[ro];
       const float cp = c_prev[ro], cn = c_new[ro];
 #pragma unroll
-      for (int g = 0; g < 4; ++g) a[g] = preact<KIND>(w[g], h[g], bb[g], al[g], be1[g], be2[g]);
+      for (int g = 0; g < 4; ++g) a[g] = preact<KIND, FastMath<T>::value>(w[g], h[g], bb[g], al[g], be1[g], be2[g]);
       float da[4];
       cell_bwd<KIND, FastMath<T>::value>(a, cp, cn, dh, dcv, da);
       dc[ro] = dcv;
@@ -398,14 +398,18 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
       for (int g = 0; g < 4; ++g) {
         red[ty][g][tx] = __fadd_rn(red[ty][g][tx], da[g]);
         if (KIND == K_MILSTM) {
-          duhp[g * GATE_U] = from_f<T>(__fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], w[g]), be1[g])));
-          __stcs(dwxp + g * GATE_U, from_f<T>(__fmul_rn(da[g], __fadd_rn(__fmul_rn(al[g], h[g]), be2[g]))));
+          constexpr bool F = FastMath<T>::value;   // bf16 path: fused multiply-adds (reading R27)
+          const float gu = F ? __fmaf_rn(al[g], w[g], be1[g]) : __fadd_rn(__fmul_rn(al[g], w[g]), be1[g]);
+          const float gw = F ? __fmaf_rn(al[g], h[g], be2[g]) : __fadd_rn(__fmul_rn(al[g], h[g]), be2[g]);
+          duhp[g * GATE_U] = from_f<T>(__fmul_rn(da[g], gu));
+          __stcs(dwxp + g * GATE_U, from_f<T>(__fmul_rn(da[g], gw)));
+          const float dw = __fmul_rn(da[g], w[g]);
           float* r4 = &red[ty][NV > 4 ? 4 : 0][tx];
-          r4[g * BWD_UX] = __fadd_rn(r4[g * BWD_UX], __fmul_rn(__fmul_rn(da[g], w[g]), h[g]));
+          r4[g * BWD_UX] = F ? __fmaf_rn(dw, h[g], r4[g * BWD_UX]) : __fadd_rn(r4[g * BWD_UX], __fmul_rn(dw, h[g]));
           float* r8 = &red[ty][NV > 8 ? 8 : 0][tx];
-          r8[g * BWD_UX] = __fadd_rn(r8[g * BWD_UX], __fmul_rn(da[g], h[g]));
+          r8[g * BWD_UX] = F ? __fmaf_rn(da[g], h[g], r8[g * BWD_UX]) : __fadd_rn(r8[g * BWD_UX], __fmul_rn(da[g], h[g]));
           float* r12 = &red[ty][NV > 12 ? 12 : 0][tx];
-          r12[g * BWD_UX] = __fadd_rn(r12[g * BWD_UX], __fmul_rn(da[g], w[g]));
+          r12[g * BWD_UX] = __fadd_rn(r12[g * BWD_UX], dw);
         } else {
           duhp[g * GATE_U] = from_f<T>(da[g]);
         }

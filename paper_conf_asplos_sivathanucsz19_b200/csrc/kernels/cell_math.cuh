@@ -42,10 +42,13 @@ template <> __device__ __forceinline__ __nv_bfloat16 from_f<__nv_bfloat16>(float
 enum CellKind { K_LSTM = 0, K_MILSTM = 1, K_SUBLSTM = 5 };
 
 // Pre-activation of one gate.  LSTM/subLSTM: a = wx + uh + b.
-// MI-LSTM [36]: a = α·wx·uh + β1·uh + β2·wx + b  (reading R3/R4), evaluated left to right.
-template <int KIND>
+// MI-LSTM [36]: a = α·wx·uh + β1·uh + β2·wx + b  (reading R3/R4).  fp32 path: evaluated left to
+// right with separate roundings; bf16 path (F): the same sum as a fixed chain of fused multiply-adds
+// a = fma(α·wx, uh, fma(β1, uh, fma(β2, wx, b))) — fewer instructions, identical in every bf16 kernel.
+template <int KIND, bool F = false>
 __device__ __forceinline__ float preact(float wx, float uh, float b, float al, float b1, float b2) {
   if (KIND == K_MILSTM) {
+    if (F) return __fmaf_rn(__fmul_rn(al, wx), uh, __fmaf_rn(b1, uh, __fmaf_rn(b2, wx, b)));
     float a = __fmul_rn(__fmul_rn(al, wx), uh);
     a = __fadd_rn(a, __fmul_rn(b1, uh));
     a = __fadd_rn(a, __fmul_rn(b2, wx));
@@ -60,37 +63,41 @@ template <int KIND, bool F = false>
 __device__ __forceinline__ void cell_fwd(const float (&a)[4], float c_prev, float& c_new, float& h_new) {
   if (KIND == K_SUBLSTM) {
     const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), z = sigm<F>(a[2]), o = sigm<F>(a[3]);
-    c_new = __fsub_rn(__fadd_rn(__fmul_rn(f, c_prev), z), i);
+    c_new = F ? __fsub_rn(__fmaf_rn(f, c_prev, z), i) : __fsub_rn(__fadd_rn(__fmul_rn(f, c_prev), z), i);
     h_new = __fsub_rn(sigm<F>(c_new), o);
   } else {
     const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), g = tanh_<F>(a[2]), o = sigm<F>(a[3]);
-    c_new = __fadd_rn(__fmul_rn(f, c_prev), __fmul_rn(i, g));
+    c_new = F ? __fmaf_rn(f, c_prev, __fmul_rn(i, g)) : __fadd_rn(__fmul_rn(f, c_prev), __fmul_rn(i, g));
     h_new = __fmul_rn(o, tanh_<F>(c_new));
   }
 }
 
 // Backward of one cell update.  dh = dL/dh_t, dc = dL/dc_t from step t+1 (in/out: becomes
-// dL/dc_{t-1}).  da[4] = dL/da for the four gates.
+// dL/dc_{t-1}).  da[4] = dL/da for the four gates.  x·(1−x) and 1−x² as fused forms in the bf16
+// path (F), separate roundings in the fp32 path.
 template <int KIND, bool F = false>
 __device__ __forceinline__ void cell_bwd(const float (&a)[4], float c_prev, float c_new, float dh, float& dc,
                                          float (&da)[4]) {
+  auto dsig = [](float s) { return F ? __fmaf_rn(-s, s, s) : __fmul_rn(s, __fsub_rn(1.f, s)); };
+  auto dtnh = [](float t) { return F ? __fmaf_rn(-t, t, 1.f) : __fsub_rn(1.f, __fmul_rn(t, t)); };
   if (KIND == K_SUBLSTM) {
     const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), z = sigm<F>(a[2]), o = sigm<F>(a[3]);
     const float sc = sigm<F>(c_new);
-    const float dcc = __fadd_rn(dc, __fmul_rn(dh, __fmul_rn(sc, __fsub_rn(1.f, sc))));
-    da[0] = __fmul_rn(-dcc, __fmul_rn(i, __fsub_rn(1.f, i)));
-    da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), __fmul_rn(f, __fsub_rn(1.f, f)));
-    da[2] = __fmul_rn(dcc, __fmul_rn(z, __fsub_rn(1.f, z)));
-    da[3] = __fmul_rn(-dh, __fmul_rn(o, __fsub_rn(1.f, o)));
+    const float dcc = F ? __fmaf_rn(dh, dsig(sc), dc) : __fadd_rn(dc, __fmul_rn(dh, dsig(sc)));
+    da[0] = __fmul_rn(-dcc, dsig(i));
+    da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), dsig(f));
+    da[2] = __fmul_rn(dcc, dsig(z));
+    da[3] = __fmul_rn(-dh, dsig(o));
     dc = __fmul_rn(dcc, f);
   } else {
     const float i = sigm<F>(a[0]), f = sigm<F>(a[1]), g = tanh_<F>(a[2]), o = sigm<F>(a[3]);
     const float tau = tanh_<F>(c_new);
-    const float dcc = __fadd_rn(dc, __fmul_rn(__fmul_rn(dh, o), __fsub_rn(1.f, __fmul_rn(tau, tau))));
-    da[0] = __fmul_rn(__fmul_rn(dcc, g), __fmul_rn(i, __fsub_rn(1.f, i)));
-    da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), __fmul_rn(f, __fsub_rn(1.f, f)));
-    da[2] = __fmul_rn(__fmul_rn(dcc, i), __fsub_rn(1.f, __fmul_rn(g, g)));
-    da[3] = __fmul_rn(__fmul_rn(dh, tau), __fmul_rn(o, __fsub_rn(1.f, o)));
+    const float dcc = F ? __fmaf_rn(__fmul_rn(dh, o), dtnh(tau), dc)
+                        : __fadd_rn(dc, __fmul_rn(__fmul_rn(dh, o), dtnh(tau)));
+    da[0] = __fmul_rn(__fmul_rn(dcc, g), dsig(i));
+    da[1] = __fmul_rn(__fmul_rn(dcc, c_prev), dsig(f));
+    da[2] = __fmul_rn(__fmul_rn(dcc, i), dtnh(g));
+    da[3] = __fmul_rn(__fmul_rn(dh, tau), dsig(o));
     dc = __fmul_rn(dcc, f);
   }
 }

@@ -202,7 +202,7 @@ __global__ void __launch_bounds__(RF_THREADS, 1)
 #pragma unroll
             for (int g = 0; g < 4; ++g) {
               const int c = g * 64 + ul + i;
-              pa[g] = preact<KIND>(wx[g][i], z[g][i], prm[c], prm[BN + c], prm[2 * BN + c], prm[3 * BN + c]);
+              pa[g] = preact<KIND, true>(wx[g][i], z[g][i], prm[c], prm[BN + c], prm[2 * BN + c], prm[3 * BN + c]);
             }
             float c_, h_;
             cell_fwd<KIND, true>(pa, cp[i], c_, h_);

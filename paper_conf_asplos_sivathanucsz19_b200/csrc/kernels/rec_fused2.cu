@@ -168,7 +168,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
 #pragma unroll
           for (int g = 0; g < 4; ++g) {
             const float4 p = prm[g * 64 + ul];
-            pa[g] = preact<KIND>(wx[g][i], __uint_as_float(zr[g][i]), p.x, p.y, p.z, p.w);
+            pa[g] = preact<KIND, true>(wx[g][i], __uint_as_float(zr[g][i]), p.x, p.y, p.z, p.w);
           }
           cell_fwd<KIND, FastMath<__nv_bfloat16>::value>(pa, cp[i], cv[i], hv[i]);
         } else {
