@@ -444,7 +444,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       if (warp == 2 && lane == 0) GEMM_TRACE(6);
       sm100::mbar_arrive(&tempty[acc]);
     }
-    sm100::bulk_wait_all();   // this thread's bulk stores have landed before the CTA retires
+    sm100::bulk_wait_read<0>();   // the copy engine has read this thread's staged tiles
   }
   __syncthreads();
   if (cs > 1) sm100::cluster_sync();
@@ -515,8 +515,6 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  pdl_wait();
-  pdl_trigger();
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer (both CTAs)
@@ -524,6 +522,39 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       int s = 0;
       uint32_t ph = 0;
       const uint64_t pol = sm100::l2_policy_evict_last();
+      auto load_b = [&](uint8_t* sb, uint32_t bar, int n0, int k0) {
+        if (args.b_mn) {
+#pragma unroll
+          for (int j = 0; j < BH / 64; ++j) {
+            if (args.b_keep) sm100::tma_load_3d_cg2_hint(sb + j * 8192, &mapB, bar, n0 + 64 * j, k0, args.bz, pol);
+            else sm100::tma_load_3d_cg2(sb + j * 8192, &mapB, bar, n0 + 64 * j, k0, args.bz);
+          }
+        } else {
+          if (args.b_keep) sm100::tma_load_3d_cg2_hint(sb, &mapB, bar, k0, n0, args.bz, pol);
+          else sm100::tma_load_3d_cg2(sb, &mapB, bar, k0, n0, args.bz);
+        }
+      };
+      // A weight operand (b_keep: written long before this launch — every kernel of the chain waits
+      // on its predecessor before triggering its successor, so kernels two launches back are
+      // complete) is fetched for the first stages before the grid dependency resolves; the
+      // activations (A) and all outputs wait for it.
+      int pre = 0;
+      if (args.b_keep && pair_id < num_pt) {
+        const int ks = pair_id / num_pt1, c1 = pair_id % num_pt1;
+        int mi, ni;
+        tile_raster(c1, num_mp, args.num_n, args.gm, mi, ni);
+        const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
+        pre = min(stages, max(0, kb1 - kb0));
+        for (int i = 0; i < pre; ++i) {
+          uint8_t* sa = smem + i * S::STAGE_BYTES;
+          if (rank == 0) sm100::mbar_arrive_expect_tx(&full[i], 2 * S::STAGE_BYTES);
+          load_b(sa + S::A_BYTES, sm100::mapa_shared(sm100::smem_u32(&full[i]), 0), ni * BN + rank * BH,
+                 (kb0 + i) * TC_BK);
+        }
+      }
+      pdl_wait();
+      pdl_trigger();
+      int issued = 0;
       for (int ct = pair_id; ct < num_pt; ct += num_pairs) {
         const int ks = ct / num_pt1, c1 = ct % num_pt1;
         int mi, ni;
@@ -531,11 +562,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const int m0 = mi * 2 * TC_BM + rank * TC_BM;
         const int n0 = ni * BN + rank * BH;
         const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
-        for (int kb = kb0; kb < kb1; ++kb) {
-          sm100::mbar_wait(&empty[s], ph ^ 1);
+        for (int kb = kb0; kb < kb1; ++kb, ++issued) {
+          const bool early = issued < pre;          // B of this stage already in flight
+          if (!early) sm100::mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * S::STAGE_BYTES;
           uint8_t* sb = sa + S::A_BYTES;
-          if (rank == 0) sm100::mbar_arrive_expect_tx(&full[s], 2 * S::STAGE_BYTES);
+          if (!early && rank == 0) sm100::mbar_arrive_expect_tx(&full[s], 2 * S::STAGE_BYTES);
           const uint32_t bar = sm100::mapa_shared(sm100::smem_u32(&full[s]), 0);
           const int k0 = kb * TC_BK;
           if (args.a_mn) {
@@ -544,22 +576,16 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           } else {
             sm100::tma_load_3d_cg2(sa, &mapA, bar, k0, m0, args.az);
           }
-          if (args.b_mn) {
-#pragma unroll
-            for (int j = 0; j < BH / 64; ++j) {
-              if (args.b_keep) sm100::tma_load_3d_cg2_hint(sb + j * 8192, &mapB, bar, n0 + 64 * j, k0, args.bz, pol);
-              else sm100::tma_load_3d_cg2(sb + j * 8192, &mapB, bar, n0 + 64 * j, k0, args.bz);
-            }
-          } else {
-            if (args.b_keep) sm100::tma_load_3d_cg2_hint(sb, &mapB, bar, k0, n0, args.bz, pol);
-            else sm100::tma_load_3d_cg2(sb, &mapB, bar, k0, n0, args.bz);
-          }
+          if (!early) load_b(sb, bar, n0, k0);
           if (++s == stages) { s = 0; ph ^= 1; }
         }
       }
+    } else {
+      pdl_wait();
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (pair leader only)
+    pdl_wait();
     if (lane == 0 && rank == 0) {
       int s = 0;
       uint32_t ph = 0;
@@ -592,6 +618,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
   } else {
     // ------------------------------------------------------------ epilogue warps 2..5 (both CTAs)
+    pdl_wait();
     const int quarter = warp & 3;
     int nbuf = 0;
     const uint32_t tempty_cl[2] = {sm100::mapa_shared(sm100::smem_u32(&tempty[0]), 0),
@@ -614,7 +641,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       __syncwarp();
       if (lane == 0) sm100::mbar_arrive_cluster(tempty_cl[acc]);
     }
-    sm100::bulk_wait_all();
+    sm100::bulk_wait_read<0>();
   }
   __syncthreads();
   sm100::cluster_sync();

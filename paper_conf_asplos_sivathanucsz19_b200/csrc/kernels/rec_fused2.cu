@@ -54,6 +54,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
   const int n0 = nt * R2_BN;                   // first gate-interleaved column of the pair tile
   const int u0 = nt * 64;                      // first hidden unit
   const int t = a.t;
+  if (threadIdx.x == 0) GEMM_TRACE(0);
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < stages; ++s) {
@@ -74,6 +75,25 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
   sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) {
+    // WX_t (written by the a1 GEMM long before) → L2 while the main loop runs
+#pragma unroll 1
+    for (int w = 0; w < R2_EPI_WARPS; ++w)
+      for (int g = 0; g < 4; ++g)
+        sm100::tma_prefetch_l2_box(&mapWX, n0 + g * 64 + (w / 4) * 32, m0 + ((w + 2) & 3) * 32, t);
+  }
+  if (warp == 0 && lane == 0) {
+    // the U mirror (weights, written at the start of the step) for the first stages before the grid
+    // dependency resolves; h_{t-1} (A) after it
+    const uint64_t pol = sm100::l2_policy_evict_last();
+    const int pre = a.nk < stages ? a.nk : stages;
+    for (int kb = 0; kb < pre; ++kb) {
+      uint8_t* sa = smem + kb * S::STAGE_BYTES;
+      if (rank == 0) sm100::mbar_arrive_expect_tx(&full[kb], 2 * S::STAGE_BYTES);
+      sm100::tma_load_3d_cg2_hint(sa + S::A_BYTES, &mapB, sm100::mapa_shared(sm100::smem_u32(&full[kb]), 0),
+                                  kb * TC_BK, n0 + rank * (R2_BN / 2), 0, pol);
+    }
+  }
   pdl_wait();
   pdl_trigger();
   for (int i = threadIdx.x; i < 4 * 64; i += R2_THREADS) {   // per-(gate, unit) parameters
@@ -83,20 +103,23 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
                          (ok && KIND == K_MILSTM) ? a.gp.beta1[e] : 0.f, (ok && KIND == K_MILSTM) ? a.gp.beta2[e] : 0.f);
   }
   __syncthreads();
+  if (threadIdx.x == 0) GEMM_TRACE(1);
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer (both CTAs)
     if (lane == 0) {
       const uint64_t pol = sm100::l2_policy_evict_last();
       const uint32_t bar0 = sm100::mapa_shared(sm100::smem_u32(&full[0]), 0);
+      const int pre = a.nk < stages ? a.nk : stages;
       for (int kb = 0; kb < a.nk; ++kb) {
         const int s = kb % stages;
-        sm100::mbar_wait(&empty[s], (uint32_t)((kb / stages) & 1) ^ 1);
+        if (kb >= pre) sm100::mbar_wait(&empty[s], (uint32_t)((kb / stages) & 1) ^ 1);
         uint8_t* sa = smem + s * S::STAGE_BYTES;
-        if (rank == 0) sm100::mbar_arrive_expect_tx(&full[s], 2 * S::STAGE_BYTES);
+        if (kb >= pre && rank == 0) sm100::mbar_arrive_expect_tx(&full[s], 2 * S::STAGE_BYTES);
         const uint32_t bar = bar0 + (uint32_t)s * 8;
         sm100::tma_load_3d_cg2(sa, &mapA, bar, kb * TC_BK, m0, t);
-        sm100::tma_load_3d_cg2_hint(sa + S::A_BYTES, &mapB, bar, kb * TC_BK, n0 + rank * (R2_BN / 2), 0, pol);
+        if (kb >= pre)
+          sm100::tma_load_3d_cg2_hint(sa + S::A_BYTES, &mapB, bar, kb * TC_BK, n0 + rank * (R2_BN / 2), 0, pol);
       }
     }
   } else if (warp == 1) {
@@ -105,6 +128,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
       for (int kb = 0; kb < a.nk; ++kb) {
         const int s = kb % stages;
         sm100::mbar_wait(&full[s], (uint32_t)((kb / stages) & 1));
+        if (kb == 0) GEMM_TRACE(3);
         sm100::tc_fence_after();
         const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
         const uint32_t sb = sa + S::A_BYTES;
@@ -115,6 +139,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
         sm100::umma_commit_cg2_mc(&empty[s], 0x3);
       }
       sm100::umma_commit_cg2_mc(tfull, 0x3);
+      GEMM_TRACE(4);
     }
   } else {
     // ------------------------------------------------------------ fused gate epilogue (8 warps)
@@ -127,6 +152,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
     const uint32_t wx_s = sm100::smem_u32(wbuf), c_s = wx_s + 4 * 4096;
     const uint32_t h_s = sm100::smem_u32(htiles + ew * R2_HTILE);
     sm100::mbar_wait(tfull, 0);              // accumulator complete ⇒ every stage buffer consumed
+    if (ew == 0 && lane == 0) GEMM_TRACE(5);
     sm100::tc_fence_after();
     if (lane == 0) {
       sm100::mbar_arrive_expect_tx(&ebar[ew], R2_WARP_IN);
@@ -135,6 +161,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
       sm100::tma_load_box(c_s, &mapC, &ebar[ew], uc, mq, t);
     }
     sm100::mbar_wait(&ebar[ew], 0);
+    if (ew == 0 && lane == 0) GEMM_TRACE(6);
     const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16);
     const int r = lane;                       // this thread's row within the warp's 32
     const bool last = t == a.T - 1;
@@ -214,6 +241,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
         }
       }
     }
+    if (ew == 0 && lane == 0) GEMM_TRACE(7);
     sm100::tc_fence_before();
     sm100::fence_proxy_async_smem();
     __syncwarp();
@@ -224,10 +252,12 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
       sm100::tma_store_3d(&mapH, h_s, uc, mq, t + 1);
       if (a.y_kind == 1) sm100::tma_store_3d(&mapY, h_s, uc, mq, t);
       sm100::bulk_commit();
-      sm100::bulk_wait_all();
+      sm100::bulk_wait_read<0>();
+      if (ew == 0) GEMM_TRACE(8);
     }
   }
   __syncthreads();
+  if (threadIdx.x == 0) GEMM_TRACE(9);
   sm100::cluster_sync();
   if (warp == 1) {
     sm100::tc_fence_after();

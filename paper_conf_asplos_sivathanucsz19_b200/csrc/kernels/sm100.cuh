@@ -228,6 +228,14 @@ __device__ __forceinline__ void bulk_load(uint32_t sdst, const void* gsrc, uint3
                : "memory");
 }
 
+// Prefetch one tensor box into L2 (no shared-memory destination, no completion tracking).
+__device__ __forceinline__ void tma_prefetch_l2_box(const CUtensorMap* m, int c0, int c1, int c2) {
+  asm volatile("cp.async.bulk.prefetch.tensor.3d.L2.global.tile [%0, {%1, %2, %3}];" ::"l"(
+                   reinterpret_cast<uint64_t>(m)),
+               "r"(c0), "r"(c1), "r"(c2)
+               : "memory");
+}
+
 // TMA tensor store of one box from shared memory (bulk-group completion).
 __device__ __forceinline__ void tma_store_3d(const CUtensorMap* m, uint32_t ssrc, int c0, int c1, int c2) {
   asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
