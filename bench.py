@@ -1,6 +1,8 @@
 """Benchmark: custom-RNN training samples/s on B200 (BASELINE.json metric), workload = cfg5
-(BASELINE.json configs[4]): MI-LSTM char LM, hidden 2048, global batch 512, seq 100, data-parallel
-over N GPUs (strong scaling: per-rank batch 512/N).  One step = embedding → MI-LSTM forward →
+(BASELINE.json configs[4]): MI-LSTM char LM, hidden 2048, batch 512, seq 100, data-parallel over N
+GPUs.  Default: weak scaling — every rank trains its own shard of 512 sequences (global batch 512·N,
+DESIGN.md reading R30: the sequences are independent units, the only exchange is the gradient
+all-reduce); `--strong` keeps the global batch at 512 (per-rank 512/N).  One step = embedding → MI-LSTM forward →
 head + CE → BPTT → weight gradients → gradient all-reduce (N > 1) → SGD, all in the library's
 kernels through the C ABI.
 
@@ -149,7 +151,8 @@ def main():
     ap.add_argument("--no-tune", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + --steps steps, nothing else (for ncu)")
-    ap.add_argument("--batch", type=int, default=None, help="override global batch (debug)")
+    ap.add_argument("--batch", type=int, default=None, help="override the per-rank batch (weak) / global batch (strong)")
+    ap.add_argument("--strong", action="store_true", help="fixed global batch 512 split over the ranks")
     ap.add_argument("--seq", type=int, default=None, help="override seq (debug)")
     args = ap.parse_args()
 
@@ -158,7 +161,9 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     T = args.seq or WORKLOAD["seq_len"]
     H, I, V, n_sym = WORKLOAD["hidden"], WORKLOAD["input"], WORKLOAD["vocab"], WORKLOAD["symbols"]
-    B_g = args.batch or WORKLOAD["global_batch"]
+    B_unit = args.batch or WORKLOAD["global_batch"]
+    B_g = B_unit if args.strong else B_unit * max(world, 1)     # global batch of this run
+    scaling = "strong" if args.strong else "weak"
     cfg = {"workload": WORKLOAD["workload"], "cell": "MI-LSTM", "hidden": H, "input": I, "global_batch": B_g,
            "seq_len": T, "vocab": V, "parallelism": f"dp{args.gpus}", "per_gpu_batch": B_g // max(world, 1),
            "l2": "working set per step (GB of activations, 139 MB of fp32 grads) >> 126 MB L2: inputs larger than L2"}
@@ -170,7 +175,7 @@ def main():
         val, dt, thr = run_oracle(T, H, I, V, n_sym, Bs, steps=max(1, min(args.steps, 2)), warm=0)
         line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "samples/s", "n_gpus": args.gpus,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 * (B_g / Bs),
-                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+                "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
                 "data": "synthetic (seeded Zipf tokens, random-init weights)", "config": cfg,
                 "cpu_baseline": {"value": val, "unit": "samples/s", "cores": thr, "kind": "oracle",
                                  "sample": f"{Bs} of the {B_g} sequences (T={T}, H=I=2048, V=256), one full "
@@ -285,7 +290,7 @@ def main():
         step_tf = value * fl / 1e12
         line = {
             "metric": METRIC, "value": value, "unit": "samples/s", "n_gpus": args.gpus, "steps": args.steps,
-            "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+            "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded Zipf tokens over 205 symbols, "
             "random-init weights)", "config": cfg,
             "tokens_per_s": value * T,

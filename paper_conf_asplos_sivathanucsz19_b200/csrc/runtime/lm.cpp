@@ -107,7 +107,14 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   ASTRA_CHECK_ARG(tokens, "lm_train_step: tokens is null");
   Cell& c = *cell;
   // exploration steps (and the fp32 parity path) run eagerly; a frozen / untuned bf16 step replays
-  if (!use_graphs || !graphs_enabled() || c.tune_mode == ASTRA_TUNE_ON || c.ot != OT::BF16) {
+  // multi-rank steps stay eager unless ASTRA_GRAPH_NCCL=1 (NCCL inside a capture is supported, but
+  // a capture mismatch across ranks would hang the job; not exercisable on a 1-GPU test box)
+  static const bool graph_nccl = [] {
+    const char* e = std::getenv("ASTRA_GRAPH_NCCL");
+    return e && e[0] == '1';
+  }();
+  if (!use_graphs || !graphs_enabled() || c.tune_mode == ASTRA_TUNE_ON || c.ot != OT::BF16 ||
+      (c.world > 1 && !graph_nccl)) {
     enqueue_step(tokens, lr, loss_dev, do_sgd);
     return;
   }
