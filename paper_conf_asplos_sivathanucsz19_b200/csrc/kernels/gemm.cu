@@ -134,6 +134,7 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
   if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
   if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm / cg);
+  g.args.pf = L2Pf{};
   g.args.cg = cg;
   static const int gm_env = [] {
     const char* e = std::getenv("ASTRA_GM");   // raster group override (A/B runs)
@@ -163,7 +164,8 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
 }
 
 template <int BN>
-static void launch_pair(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
+static void launch_pair(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas,
+                        const L2Pf* pf) {
   static int attr_bytes = 0;
   if (g.smem > attr_bytes) {
     CUDA_TRY(cudaFuncSetAttribute(tc_gemm2_kernel<BN, EpiStore>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -173,6 +175,7 @@ static void launch_pair(const TcGemm& g, const EpiStore& epi, int az, int bz, cu
   TcArgs a = g.args;
   a.az = az;
   a.bz = bz;
+  if (pf) a.pf = *pf;
   CUtensorMap mapC;
   EpiStore e = epi;
   e.tma = epi_tma_map(epi, a.ksplit, &mapC) ? 1 : 0;
@@ -187,7 +190,8 @@ static void launch_pair(const TcGemm& g, const EpiStore& epi, int az, int bz, cu
 }
 
 template <int BN>
-static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
+static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas,
+                        const L2Pf* pf) {
   static int attr_bytes = 0;
   if (g.smem > attr_bytes) {
     CUDA_TRY(cudaFuncSetAttribute(tc_gemm_kernel<BN, EpiStore>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -197,6 +201,7 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   TcArgs a = g.args;
   a.az = az;
   a.bz = bz;
+  if (pf) a.pf = *pf;
   CUtensorMap mapC;
   EpiStore e = epi;
   e.tma = epi_tma_map(epi, a.ksplit, &mapC) ? 1 : 0;
@@ -211,17 +216,18 @@ static void launch_bn(const TcGemm& g, const EpiStore& epi, int az, int bz, cuda
   LAUNCH_CHECK();
 }
 
-void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas) {
+void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas,
+                    const L2Pf* pf) {
   ASTRA_CHECK_STATE(g.ready, "tc_gemm: not prepared");
   if (g.args.cg == 2) {
-    if (g.BN == 128) launch_pair<128>(g, epi, az, bz, st, max_ctas);
-    else launch_pair<256>(g, epi, az, bz, st, max_ctas);
+    if (g.BN == 128) launch_pair<128>(g, epi, az, bz, st, max_ctas, pf);
+    else launch_pair<256>(g, epi, az, bz, st, max_ctas, pf);
     return;
   }
   switch (g.BN) {
-    case 64: launch_bn<64>(g, epi, az, bz, st, max_ctas); break;
-    case 128: launch_bn<128>(g, epi, az, bz, st, max_ctas); break;
-    default: launch_bn<256>(g, epi, az, bz, st, max_ctas); break;
+    case 64: launch_bn<64>(g, epi, az, bz, st, max_ctas, pf); break;
+    case 128: launch_bn<128>(g, epi, az, bz, st, max_ctas, pf); break;
+    default: launch_bn<256>(g, epi, az, bz, st, max_ctas, pf); break;
   }
 }
 

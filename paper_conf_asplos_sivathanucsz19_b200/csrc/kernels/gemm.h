@@ -33,7 +33,8 @@ struct TcGemm {
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
                      int cm = 1, int cn = 1, bool b_keep = false, int ksplit = 1, int cg = 1);
 // Launch with the given z-coordinates (time slices) and epilogue; grid ≤ #SMs (persistent).
-void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas = 0);
+void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas = 0,
+                    const L2Pf* pf = nullptr);
 
 // fp32 SIMT GEMM with arbitrary element strides: A(m,k) = A[m*sam + k*sak],
 // B(k,n) = B[k*sbk + n*sbn]; result stored through the same EpiStore rules (out_bf16 = 0).

@@ -44,7 +44,16 @@ constexpr int TC_BK = 64;          // one 128-byte swizzle atom of bf16 along K
 constexpr int TC_EPI_WARPS = 4;                    // epilogue warps (one per TMEM lane quarter)
 constexpr int TC_THREADS = 64 + 32 * TC_EPI_WARPS;
 
+// Up to four global byte ranges the GEMM pulls into L2 while it runs (reading R31): the saved
+// tensors the next pointwise kernel of a recurrent chain will read, so that kernel finds them in
+// L2 instead of waiting on HBM latency.  A prefetch never changes any value.
+struct L2Pf {
+  const void* p[4];
+  unsigned long long n[4];
+};
+
 struct TcArgs {
+  L2Pf pf;          // L2 prefetch ranges (n = 0: none)
   int M, N, K;
   int num_m, num_n;
   int az, bz;       // third tensor-map coordinate (time slice) of A and B
@@ -57,6 +66,24 @@ struct TcArgs {
   int gm;           // raster group: tiles walk gm M-tiles of one N column before the next column
   uint32_t idesc;
 };
+
+// One warp of every CTA issues its slice of the prefetch ranges (cp.async.bulk.prefetch.L2, 16-byte
+// granules): range bytes split evenly over gridDim.x × 32 lanes.
+__device__ __forceinline__ void l2_prefetch_slices(const L2Pf& pf, int lane) {
+  const unsigned long long nthr = (unsigned long long)gridDim.x * 32, id = (unsigned long long)blockIdx.x * 32 + lane;
+#pragma unroll
+  for (int r = 0; r < 4; ++r) {
+    const unsigned long long n = pf.n[r] & ~15ull;
+    if (!n) continue;
+    const unsigned long long piece = ((n + nthr - 1) / nthr + 255) & ~255ull;
+    const unsigned long long lo = id * piece;
+    if (lo >= n) continue;
+    const unsigned long long sz = n - lo < piece ? n - lo : piece;
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(reinterpret_cast<uint64_t>(pf.p[r]) + lo),
+                 "r"((uint32_t)sz)
+                 : "memory");
+  }
+}
 
 // Grouped raster of the persistent tile loop: tile c1 → (mi, ni) walking `gm` consecutive M-tiles
 // down one N column, then the next column, group after group.  The CTAs resident at any time then
@@ -314,6 +341,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   if (cs > 1) sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (warp == 2) l2_prefetch_slices(args.pf, lane);   // old data only: no grid dependency needed
   pdl_wait();      // operands / outputs may belong to the previous kernel in the stream
   pdl_trigger();
   if (threadIdx.x == 0) GEMM_TRACE(1);
@@ -515,6 +543,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   sm100::cluster_sync();
   sm100::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (warp == 2) l2_prefetch_slices(args.pf, lane);   // old data only: no grid dependency needed
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer (both CTAs)

@@ -45,6 +45,7 @@ struct Variant {
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
   int fwd_mode = 0;     // K2 (LSTM family, bf16): 0 GEMM + pointwise kernel, 1 fused per step, 2 fused persistent
   int bwd_mode = 0;     // K4: same encoding
+  int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
   Variant() { g[G_BPTT].bn = 128; }
   std::string str() const;                    // "a1=256.1.1,rec=...,wg_side=0"
   static Variant parse(const std::string& s); // inverse of str(); throws ASTRA_E_ARG
@@ -127,6 +128,7 @@ class Cell {
   virtual std::vector<KSeg> y_segments() const = 0;
   virtual int c_width() const { return H; }      // width of the second state (c or s); 0 = none
   virtual bool lm_capable() const { return true; }
+  virtual bool chain_prefetch() const { return false; }   // supports Variant::l2pf (tuner AVs pf_fwd / pf_bwd)
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
@@ -147,7 +149,8 @@ class Cell {
   size_t esz() const { return ot_size(ot); }
   template <typename T_> T_* sv(size_t off) { return reinterpret_cast<T_*>(saved + off); }
   template <typename T_> T_* sc(size_t off) { return reinterpret_cast<T_*>(scratch + off); }
-  void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st);
+  void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st,
+                const L2Pf* pf = nullptr);
   TcGemm& tc_get(int id, const GemmSpec& s, const KCfg& k);   // prepared tensor maps (bf16 path)
   void mark(Region r, int which, cudaStream_t st);
   void tuner_setup();

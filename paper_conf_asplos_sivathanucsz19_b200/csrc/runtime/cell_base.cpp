@@ -21,7 +21,7 @@ std::string Variant::str() const {
     if (g[r].cg != 1) o << "." << g[r].cg;
     o << ",";
   }
-  o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode;
+  o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf;
   return o.str();
 }
 
@@ -40,6 +40,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "wg_side") {
       v.wg_side = std::stoi(val);
       ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    if (k == "pf") {
+      v.l2pf = std::stoi(val);
+      ASTRA_CHECK_ARG(v.l2pf >= 0 && v.l2pf <= 3, "variant: pf must be 0..3 (bit 0 fwd chain, bit 1 BPTT chain)");
       continue;
     }
     if (k == "fwd" || k == "bwd") {
@@ -168,9 +173,10 @@ TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
   return it->second;
 }
 
-void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st) {
+void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st,
+                    const L2Pf* pf) {
   if (ot == OT::BF16) {
-    tc_gemm_launch(tc_get(id, s, k), e, az, bz, st);
+    tc_gemm_launch(tc_get(id, s, k), e, az, bz, st, 0, pf);
   } else {
     const float* A = (const float*)s.A.ptr + (long)az * s.A.zstride;
     const float* Bm = (const float*)s.B.ptr + (long)bz * s.B.zstride;
@@ -260,6 +266,9 @@ void Cell::tuner_setup() {
   // P:120-126 "fusion" AV) is tuned after the kernel choices, against the forward-chain time
   if (ot == OT::BF16 && fwd_fusions() > 1)
     t = "(pre " + t + " (leaf fuse_fwd " + std::to_string(fwd_fusions()) + " t_fwd))";
+  // reading R31: L2 prefetch by the chain GEMMs, per chain, after the kernel and fusion choices
+  if (ot == OT::BF16 && chain_prefetch())
+    t = "(pre " + t + " (par (leaf pf_fwd 2 t_fwd) (leaf pf_bwd 2 t_bptt)))";
   if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
   if (t.empty()) t = "(leaf none 1 t_step)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
@@ -278,6 +287,8 @@ void Cell::apply_config(const tuner::Config& c) {
     const int o = c[i];
     if (n == "wg_side") { v.wg_side = o; continue; }
     if (n == "fuse_fwd") { v.fwd_mode = o; continue; }
+    if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
+    if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)
       if (n == std::string("g_") + ROLE_NAMES[r]) v.g[r] = allowed[r].at(o);
   }

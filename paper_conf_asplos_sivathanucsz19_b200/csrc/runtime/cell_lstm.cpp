@@ -59,6 +59,7 @@ class LstmCell : public Cell {
   int bptt_ksplit() const { return (ot == OT::BF16 && NG >= 8192) ? 4 : (ot == OT::BF16 && NG >= 4096) ? 2 : 1; }
 
   int fwd_fusions() const override { return 3; }
+  bool chain_prefetch() const override { return true; }
   RecFwd2Maps fm;                       // tensor maps of the fused CTA-pair forward (built at first use)
   const void* fm_key = (const void*)1;  // y pointer the maps were built for
   const void* fm_wx = nullptr;          // workspace they were built for (rebind ⇒ rebuild)
@@ -182,7 +183,9 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   } else {
     for (int t = 0; t < T; ++t) {
       float* UHt = UH + (long)t * B * NG;
-      run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st);
+      L2Pf pf{};   // R31: WX_t, read by this step's pointwise kernel
+      pf.p[0] = WX + (long)t * B * NG; pf.n[0] = (var.l2pf & 1) ? (unsigned long long)B * NG * 4 : 0;
+      run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st, &pf);
       const bool last = t == T - 1;
       if (y_f32)   // internal fp32 output (e.g. the encoder of LSTM-attention), row stride Hp
         lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
@@ -234,6 +237,11 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   GemmSpec bp0 = bp;   // dh0 (once, no split)
   bp.ksplit = bptt_ksplit();
   for (int t = T - 1; t >= 0; --t) {
+    const void* dyt;
+    long ldy;
+    bool dyf32;
+    if (lm_dy) { dyt = lm_dy + (long)t * B * Hp; ldy = Hp; dyf32 = true; }
+    else { dyt = (const char*)dy + (size_t)t * B * H * e; ldy = H; dyf32 = false; }
     const float* dh_rec;
     long ld_dh;
     int nsplit = 1;
@@ -243,16 +251,19 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     } else {
       EpiStore e = epi(dH, Hp, B, Hp);
       e.split_stride = (long)B * Hp;
-      run_gemm(2, bp, e, t + 1, 0, var.g[G_BPTT], st);
+      // R31: the saved tensors step t's pointwise kernel reads (WX_t, UH_t, c_{t-1..t}, dy_t)
+      L2Pf pf{};
+      if (var.l2pf & 2) {
+        pf.p[0] = WX + (long)t * B * NG; pf.n[0] = (unsigned long long)B * NG * 4;
+        pf.p[1] = UH + (long)t * B * NG; pf.n[1] = (unsigned long long)B * NG * 4;
+        pf.p[2] = Cb + (long)t * B * Hp; pf.n[2] = (unsigned long long)2 * B * Hp * 4;
+        pf.p[3] = dyt; pf.n[3] = (unsigned long long)B * ldy * (dyf32 ? 4 : esz());
+      }
+      run_gemm(2, bp, e, t + 1, 0, var.g[G_BPTT], st, &pf);
       dh_rec = dH;
       ld_dh = Hp;
       nsplit = bp.ksplit;
     }
-    const void* dyt;
-    long ldy;
-    bool dyf32;
-    if (lm_dy) { dyt = lm_dy + (long)t * B * Hp; ldy = Hp; dyf32 = true; }
-    else { dyt = (const char*)dy + (size_t)t * B * H * e; ldy = H; dyf32 = false; }
     lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC, WX + (long)t * B * NG,
                        UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
                        Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
