@@ -160,6 +160,19 @@ astra_status astra_lm_set_state(astra_lm m, const float* h, const float* c);
 astra_status astra_lm_train_step(astra_lm m, const int32_t* tokens, float lr, float* loss_dev);
 /* Same step without the SGD update (for parity tests of the gradients).                   */
 astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev);
+/* ---- bucketed profiling for variable-length mini-batches (§5.5; Table 8,
+ *      P:395-404) ------------------------------------------------------------------ */
+/* Bucket sizes (ascending, each in [1, seq]; the paper's PTB calibration is 13, 18, 24, 30, 83).
+ * n = 0 removes the buckets.  Each bucket explores its own update tree and its profile-index keys
+ * carry the bucket ("b=<T_b>"); the workspace stays the one of the largest size (seq).         */
+astra_status astra_lm_set_buckets(astra_lm m, const int* sizes, int n);
+/* One training step on a mini-batch of length len (1 <= len <= seq): tokens device int32
+ * [len+1][B].  The step runs at the smallest bucket T_b >= len (seq if none) on right-padded
+ * tokens; the mean CE is over the first len·B positions only, so loss and gradients equal those
+ * of an unpadded length-len step (padding contributes exact zeros).  Sentence-level semantics:
+ * the initial state is zero and no state is carried to the next step.  E_ARG: len out of range. */
+astra_status astra_lm_train_step_len(astra_lm m, const int32_t* tokens, int len, float lr, float* loss_dev);
+astra_status astra_lm_fwd_bwd_len(astra_lm m, const int32_t* tokens, int len, float* loss_dev);
 /* CUDA-graph replay of frozen / untuned bf16 LM steps (default on; ASTRA_GRAPH=0 turns the default
  * off).  on = 0: every step is enqueued kernel by kernel; results are bitwise identical either way.  */
 astra_status astra_lm_set_graph(astra_lm m, int on);

@@ -69,6 +69,9 @@ _SIGS = {
     "astra_lm_train_step": [_P, _P, _F, _P],
     "astra_lm_fwd_bwd": [_P, _P, _P],
     "astra_lm_set_graph": [_P, _I],
+    "astra_lm_set_buckets": [_P, _P, _I],
+    "astra_lm_train_step_len": [_P, _P, _I, _F, _P],
+    "astra_lm_fwd_bwd_len": [_P, _P, _I, _P],
     "astra_gemm_bf16": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I, _P],
     "astra_gemm_bf16_ex": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I,
                            _I, _I, _P],
@@ -291,6 +294,21 @@ class LM:
 
     def train_step(self, tokens, lr, loss=None):
         _check(lib().astra_lm_train_step(self.h, _ptr(tokens), lr, _ptr(self.loss if loss is None else loss)))
+        return self.loss if loss is None else loss
+
+    def set_buckets(self, sizes):
+        """Bucketed profiling of variable-length mini-batches (astra_lm_set_buckets)."""
+        arr = (ctypes.c_int * max(1, len(sizes)))(*sizes)
+        _check(lib().astra_lm_set_buckets(self.h, ctypes.cast(arr, ctypes.c_void_p), len(sizes)))
+
+    def train_step_len(self, tokens, length, lr, loss=None):
+        """One step on tokens [length+1, B] run at the bucket of `length` (astra_lm_train_step_len)."""
+        _check(lib().astra_lm_train_step_len(self.h, _ptr(tokens), int(length), lr,
+                                             _ptr(self.loss if loss is None else loss)))
+        return self.loss if loss is None else loss
+
+    def fwd_bwd_len(self, tokens, length, loss=None):
+        _check(lib().astra_lm_fwd_bwd_len(self.h, _ptr(tokens), int(length), _ptr(self.loss if loss is None else loss)))
         return self.loss if loss is None else loss
 
     def set_graph(self, on: bool):

@@ -147,6 +147,8 @@ astra_status astra_tune_mode(astra_cell c, int mode, const char* forced) {
     NEED(c);
     Cell& cc = *c->c;
     ASTRA_CHECK_ARG(mode == ASTRA_TUNE_OFF || mode == ASTRA_TUNE_ON || mode == ASTRA_TUNE_FROZEN, "tune_mode: bad mode");
+    // every bucket restarts — except a plain freeze, which keeps each bucket's current variant
+    if (!(mode == ASTRA_TUNE_FROZEN && !forced)) cc.tune_ctx.clear();
     if (mode == ASTRA_TUNE_OFF) {
       cc.var = Variant();
       cc.wirer.reset();
@@ -251,7 +253,32 @@ astra_status astra_lm_set_state(astra_lm m, const float* h, const float* c) {
 }
 
 astra_status astra_lm_train_step(astra_lm m, const int32_t* tokens, float lr, float* loss_dev) {
-  return guard([&] { NEED(m); m->m->step(tokens, lr, loss_dev, true); });
+  return guard([&] {
+    NEED(m);
+    m->m->cell->set_active_T(m->m->cell->Tmax);
+    m->m->step(tokens, lr, loss_dev, true);
+  });
+}
+
+astra_status astra_lm_set_buckets(astra_lm m, const int* sizes, int n) {
+  return guard([&] {
+    NEED(m);
+    ASTRA_CHECK_ARG(n >= 0 && (n == 0 || sizes), "lm_set_buckets: sizes is null");
+    std::vector<int> b(sizes, sizes + n);
+    for (int i = 0; i < n; ++i) {
+      ASTRA_CHECK_ARG(b[i] >= 1 && b[i] <= m->m->cell->Tmax, "lm_set_buckets: bucket sizes must be in [1, seq]");
+      ASTRA_CHECK_ARG(i == 0 || b[i] > b[i - 1], "lm_set_buckets: bucket sizes must be ascending");
+    }
+    m->m->buckets = b;
+  });
+}
+
+astra_status astra_lm_train_step_len(astra_lm m, const int32_t* tokens, int len, float lr, float* loss_dev) {
+  return guard([&] { NEED(m); m->m->step_var(tokens, len, lr, loss_dev, true); });
+}
+
+astra_status astra_lm_fwd_bwd_len(astra_lm m, const int32_t* tokens, int len, float* loss_dev) {
+  return guard([&] { NEED(m); m->m->step_var(tokens, len, 0.f, loss_dev, false); });
 }
 
 astra_status astra_lm_set_graph(astra_lm m, int on) {
@@ -263,7 +290,11 @@ astra_status astra_lm_set_graph(astra_lm m, int on) {
 }
 
 astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev) {
-  return guard([&] { NEED(m); m->m->step(tokens, 0.f, loss_dev, false); });
+  return guard([&] {
+    NEED(m);
+    m->m->cell->set_active_T(m->m->cell->Tmax);
+    m->m->step(tokens, 0.f, loss_dev, false);
+  });
 }
 
 astra_status astra_gemm_bf16_ex(int M, int N, int K, const void* A, int a_mn, long lda, const void* Bp, int b_mn,

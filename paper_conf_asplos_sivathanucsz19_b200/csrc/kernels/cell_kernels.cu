@@ -522,11 +522,21 @@ void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void
 // one warp per row; fixed-order warp-shuffle trees
 template <typename T>
 __global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, const int32_t* __restrict__ targets,
-                          long n, float inv_n, float* __restrict__ rowloss, T* __restrict__ dlog, long ldd,
-                          float* __restrict__ dlog32) {
+                          long n, float inv_n, const int* __restrict__ nvp, float* __restrict__ rowloss,
+                          T* __restrict__ dlog, long ldd, float* __restrict__ dlog32) {
   const long r = (long)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
   const int lane = threadIdx.x % 32;
   if (r >= n) return;
+  if (nvp) {   // rows ≥ *nvp are padding (bucketed steps): no loss, zero gradient; mean over *nvp rows
+    const long nv = *nvp;
+    inv_n = __fdiv_rn(1.f, (float)nv);
+    if (r >= nv) {
+      if (lane == 0) rowloss[r] = 0.f;
+      for (int c = lane; c < ldd; c += 32) dlog[r * ldd + c] = from_f<T>(0.f);
+      for (int c = lane; c < V; c += 32) dlog32[r * V + c] = 0.f;
+      return;
+    }
+  }
   const float* row = logits + r * ldl;
   float m = -INFINITY;
   for (int c = lane; c < V; c += 32) m = fmaxf(m, row[c]);
@@ -551,20 +561,22 @@ __global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, con
 }
 
 void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
-                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st) {
+                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp) {
   const int rows_per = 8;
   dim3 grid(cdiv(n, rows_per));
   if (ot == OT::BF16)
-    ce_kernel<__nv_bfloat16><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, rowloss,
+    ce_kernel<__nv_bfloat16><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, rowloss,
                                                              (__nv_bfloat16*)dlog, ldd, dlog32);
   else
-    ce_kernel<float><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, rowloss, (float*)dlog, ldd,
-                                                     dlog32);
+    ce_kernel<float><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, rowloss, (float*)dlog,
+                                                     ldd, dlog32);
   LAUNCH_CHECK();
 }
 
-__global__ void sum_scalar_kernel(const float* __restrict__ v, long n, float scale, float* __restrict__ out) {
+__global__ void sum_scalar_kernel(const float* __restrict__ v, long n, float scale, const int* __restrict__ nvp,
+                                  float* __restrict__ out) {
   __shared__ float sh[1024];
+  if (nvp) scale = __fdiv_rn(1.f, (float)*nvp);   // mean over the valid rows (the rest are exact zeros)
   float s = 0.f;
   for (long i = threadIdx.x; i < n; i += blockDim.x) s = __fadd_rn(s, v[i]);
   sh[threadIdx.x] = s;
@@ -576,8 +588,14 @@ __global__ void sum_scalar_kernel(const float* __restrict__ v, long n, float sca
   if (threadIdx.x == 0) *out = __fmul_rn(sh[0], scale);
 }
 
-void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st) {
-  sum_scalar_kernel<<<1, 1024, 0, st>>>(v, n, scale, out);
+void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st, const int* nvp) {
+  sum_scalar_kernel<<<1, 1024, 0, st>>>(v, n, scale, nvp, out);
+  LAUNCH_CHECK();
+}
+
+__global__ void set_i32_kernel(int* p, int v) { *p = v; }
+void set_i32(int* p, int v, cudaStream_t st) {
+  set_i32_kernel<<<1, 1, 0, st>>>(p, v);
   LAUNCH_CHECK();
 }
 

@@ -74,10 +74,12 @@ void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);
 // rowloss[r] = lse - logit[target]; dlog (ot) and dlog32 = (softmax - onehot) * inv_n.
 void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
-                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st);
+                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp = nullptr);
 // out[i] = Σ_{k < ks} part[k·n + i] in k order (split-K partials, R25/R28).
 void sum_split_partials(const float* part, int ks, long n, float* out, cudaStream_t st);
-void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st);
+void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st, const int* nvp = nullptr);
+// *p = v (a one-thread kernel: device-side scalars that captured CUDA graphs read)
+void set_i32(int* p, int v, cudaStream_t st);
 // out[c] = Σ_r in[r][c] over rows in fixed order (two-level); scratch ≥ colsum_scratch(rows, cols)
 size_t colsum_scratch_floats(long rows, int cols);
 void colsum(const float* in, long rows, int cols, long ld, float* scratch, float* out, cudaStream_t st);

@@ -78,6 +78,7 @@ class Cell {
   astra_cell_desc d;
   OT ot;
   int H, I, B, T, Hp, Ip, Hout;
+  int Tmax;   // sequence length the workspace is carved for; T = the active length (bucket) ≤ Tmax
   std::vector<ParamInfo> params;
   size_t n_params = 0;
   size_t saved_bytes = 0, scratch_bytes = 0;
@@ -107,7 +108,21 @@ class Cell {
   bool region_used[R_COUNT];
   bool profiling = true;
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
-  std::map<std::tuple<int, int, int, int, int>, TcGemm> tc_cache;
+  std::map<std::tuple<int, int, int, int, int, int>, TcGemm> tc_cache;   // (gemm id, T, bn, cm, cn, cg)
+
+  // Bucketed profiling: one independent exploration per active length T, the
+  // profile index keys prefixed by the bucket; the workspace stays the one of the largest bucket.
+  struct TuneCtx {
+    Variant var;
+    std::unique_ptr<tuner::Tree> tree;
+    std::unique_ptr<tuner::Wirer> wirer;
+    std::vector<Variant> configs_seen;
+    int rep_i = 0;
+    tuner::Metrics rep_min;
+    std::vector<KCfg> allowed[G_ROLES];
+  };
+  std::map<int, TuneCtx> tune_ctx;   // parked contexts of the inactive buckets
+  void set_active_T(int t);
 
   // NCCL
   void* nccl_comm = nullptr;
@@ -191,6 +206,16 @@ class LM {
   void set_state(const float* h, const float* c);
   void step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd);
   void enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd);
+  // Bucketed profiling for variable-length mini-batches: a step of length len runs
+  // at the smallest bucket T_b ≥ len on right-padded tokens, its loss and gradients restricted to
+  // the first len positions (padding contributes exact zeros), from a zero initial state.
+  std::vector<int> buckets;   // ascending, last ≤ cell seq; empty = every step runs at seq
+  int step_len = 0;           // valid length of the step being enqueued (0 = full T)
+  size_t off_tokpad = 0;      // int32 [Tmax+1][B] padded token buffer
+  size_t off_nv = 0;          // int32 device scalar: rows of the step that carry a loss
+  int bucket_for(int len) const;
+  void step_var(const int32_t* tokens, int len, float lr, float* loss_dev, bool do_sgd);
+  int wo_split(long TB) const;   // R28 split for the active T·B
   ~LM();
 
   // CUDA-graph replay of a frozen step (no exploration): the whole step — every kernel, the side
@@ -203,6 +228,7 @@ class LM {
     float* loss;
     bool sgd;
     std::string variant;
+    int T, len;   // active length; len = 1 for a variable-length (bucketed) step
     cudaGraphExec_t exec;
     uint64_t launches;
   };

@@ -95,7 +95,7 @@ Cell::Cell(const astra_cell_desc& dd) : d(dd) {
   ASTRA_CHECK_ARG(d.hidden > 0 && d.input > 0 && d.batch > 0 && d.seq > 0, "cell: sizes must be positive");
   ASTRA_CHECK_ARG(d.dtype == ASTRA_BF16 || d.dtype == ASTRA_FP32, "cell: dtype must be ASTRA_BF16 or ASTRA_FP32");
   ot = d.dtype == ASTRA_BF16 ? OT::BF16 : OT::F32;
-  H = d.hidden; I = d.input; B = d.batch; T = d.seq;
+  H = d.hidden; I = d.input; B = d.batch; T = d.seq; Tmax = T;
   Hp = (int)round_up(H, 64);
   Ip = (int)round_up(I, 64);
   Hout = H;
@@ -163,7 +163,7 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
 TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
   // split-K only runs without clusters; the cluster choice then falls back to 1x1 (same numerics)
   const int cm = s.ksplit > 1 ? 1 : k.cm, cn = s.ksplit > 1 ? 1 : k.cn;
-  auto key = std::make_tuple(id, k.bn, cm, cn, k.cg);
+  auto key = std::make_tuple(id, T, k.bn, cm, cn, k.cg);
   auto it = tc_cache.find(key);
   if (it == tc_cache.end()) {
     TcGemm g;
@@ -238,6 +238,43 @@ static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 1,
                                   {256, 2, 1}, {256, 4, 1}, {256, 2, 2}, {256, 1, 2}, {128, 2, 1}, {128, 4, 1},
                                   {128, 2, 2}, {128, 1, 2}, {64, 2, 1}, {64, 4, 1}, {64, 2, 2}};
 
+// Switch the active sequence length (bucket).  The exploration state of the bucket being left is
+// parked and the target bucket's restored (or started fresh: the default variant under TUNE_ON,
+// the current variant otherwise), so each bucket explores its own update tree.
+void Cell::set_active_T(int t) {
+  ASTRA_CHECK_ARG(t >= 1 && t <= Tmax, "cell: active length must be in [1, seq]");
+  if (t == T) return;
+  TuneCtx& cur = tune_ctx[T];
+  cur.var = var;
+  cur.tree = std::move(tree);
+  cur.wirer = std::move(wirer);
+  cur.configs_seen = std::move(configs_seen);
+  cur.rep_i = rep_i;
+  cur.rep_min = rep_min;
+  for (int r = 0; r < G_ROLES; ++r) cur.allowed[r] = allowed[r];
+  auto it = tune_ctx.find(t);
+  if (it != tune_ctx.end()) {
+    TuneCtx& nx = it->second;
+    var = nx.var;
+    tree = std::move(nx.tree);
+    wirer = std::move(nx.wirer);
+    configs_seen = std::move(nx.configs_seen);
+    rep_i = nx.rep_i;
+    rep_min = nx.rep_min;
+    for (int r = 0; r < G_ROLES; ++r) allowed[r] = nx.allowed[r];
+    tune_ctx.erase(it);
+  } else {
+    if (tune_mode == ASTRA_TUNE_ON) var = Variant();
+    tree.reset();
+    wirer.reset();
+    configs_seen.clear();
+    rep_i = 0;
+    rep_min.clear();
+  }
+  T = t;
+  fwd_done = false;
+}
+
 void Cell::tuner_setup() {
   const Variant def;
   std::string par;
@@ -273,6 +310,7 @@ void Cell::tuner_setup() {
   if (t.empty()) t = "(leaf none 1 t_step)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
   wirer.reset(new tuner::Wirer(tree.get()));
+  wirer->index().bucket = T;
   wirer->start();
   configs_seen.clear();
   tuner::Config c;
@@ -364,7 +402,16 @@ int Cell::tune_next() {
 
 std::string Cell::report() {
   std::ostringstream o;
-  o << "{\"variant\": \"" << var.str() << "\", \"mode\": " << tune_mode;
+  o << "{\"variant\": \"" << var.str() << "\", \"mode\": " << tune_mode << ", \"bucket\": " << T;
+  if (!tune_ctx.empty()) {   // the parked buckets: their current variant and exploration state
+    o << ", \"other_buckets\": {";
+    size_t k = 0;
+    for (auto& kv : tune_ctx)
+      o << (k++ ? ", " : "") << "\"" << kv.first << "\": {\"variant\": \"" << kv.second.var.str()
+        << "\", \"converged\": " << (kv.second.wirer && kv.second.wirer->converged() ? "true" : "false")
+        << ", \"configs_explored\": " << (kv.second.wirer ? kv.second.wirer->trials() : 0) << "}";
+    o << "}";
+  }
   if (wirer) {
     o << ", \"converged\": " << (wirer->converged() ? "true" : "false") << ", \"configs_explored\": "
       << wirer->trials() << ", \"steps_per_config\": " << (1 + tune_reps) << ", \"index_entries\": "

@@ -63,6 +63,7 @@ class LstmCell : public Cell {
   RecFwd2Maps fm;                       // tensor maps of the fused CTA-pair forward (built at first use)
   const void* fm_key = (const void*)1;  // y pointer the maps were built for
   const void* fm_wx = nullptr;          // workspace they were built for (rebind ⇒ rebuild)
+  int fm_T = 0;                         // active length the y map was built for
 
   void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
   void* x_operand() override { return sv<char>(off_X); }
@@ -129,17 +130,18 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   if (ot == OT::BF16 && var.fwd_mode == 1 && !y_f32) {
     // K2 fused, CTA-pair form: GEMM + gate epilogue with TMA-staged epilogue I/O, one launch per step
     const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1, 2});
-    if (fm_key != (const void*)y || fm_wx != (const void*)WX) {
+    if (fm_key != (const void*)y || fm_wx != (const void*)WX || fm_T != T) {
       fm.A = tg.mapA;
       fm.B = tg.mapB;
-      make_tile_map(&fm.WX, WX, false, NG, B, T, NG, (long)B * NG, 32, 32, 128);
-      make_tile_map(&fm.UH, UH, false, NG, B, T, NG, (long)B * NG, 32, 32, 128);
-      make_tile_map(&fm.C, Cb, false, Hp, B, T + 1, Hp, (long)B * Hp, 32, 32, 128);
-      make_tile_map(&fm.H, Hrow(0), true, Hp, B, T + 1, Hp, (long)B * Hp, 32, 32, 64);
+      make_tile_map(&fm.WX, WX, false, NG, B, Tmax, NG, (long)B * NG, 32, 32, 128);
+      make_tile_map(&fm.UH, UH, false, NG, B, Tmax, NG, (long)B * NG, 32, 32, 128);
+      make_tile_map(&fm.C, Cb, false, Hp, B, Tmax + 1, Hp, (long)B * Hp, 32, 32, 128);
+      make_tile_map(&fm.H, Hrow(0), true, Hp, B, Tmax + 1, Hp, (long)B * Hp, 32, 32, 64);
       if (y && H % 8 == 0 && ((uintptr_t)y & 15) == 0) make_tile_map(&fm.Y, y, true, H, B, T, H, (long)B * H, 32, 32, 64);
       else fm.Y = fm.H;
       fm_key = (const void*)y;
       fm_wx = (const void*)WX;
+      fm_T = T;
     }
     RecFwd2Args ra;
     ra.B = B; ra.H = H; ra.Hp = Hp; ra.NG = NG; ra.T = T;

@@ -50,12 +50,51 @@ LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
   {
     int maxn = 0;
     for (const KSeg& sg : c->y_segments()) maxn = std::max(maxn, sg.n);
-    const long tiles = (long)cdiv(maxn, 256) * cdiv(V, 256);
-    const int kb = cdiv(TB, 64);
-    wo_ksplit = (int)std::max(1L, std::min(std::min(64L / std::max(1L, tiles), 16L), (long)kb / 8));
+    wo_ksplit = wo_split(TB);   // non-decreasing in T·B: the largest bucket sizes the partials
     off_wopart = w.take((size_t)wo_ksplit * maxn * V * 4);
   }
+  off_tokpad = w.take((size_t)(c->Tmax + 1) * c->B * 4);
+  off_nv = w.take(4);
   ws_bytes = w.o;
+}
+
+int LM::wo_split(long TB) const {
+  int maxn = 0;
+  for (const KSeg& sg : cell->y_segments()) maxn = std::max(maxn, sg.n);
+  const long tiles = (long)cdiv(maxn, 256) * cdiv(V, 256);
+  const long kb = cdiv(TB, 64);
+  return (int)std::max(1L, std::min(std::min(64L / std::max(1L, tiles), 16L), kb / 8));
+}
+
+int LM::bucket_for(int len) const {
+  for (int b : buckets)
+    if (b >= len) return b;
+  return cell->Tmax;
+}
+
+// One variable-length step: map len to its bucket, right-pad the tokens into the
+// workspace, run the bucket-shaped step with the loss restricted to the first len positions.
+void LM::step_var(const int32_t* tokens, int len, float lr, float* loss_dev, bool do_sgd) {
+  ASTRA_CHECK_STATE(bound, "lm_train_step_len: not bound");
+  ASTRA_CHECK_ARG(tokens, "lm_train_step_len: tokens is null");
+  Cell& c = *cell;
+  ASTRA_CHECK_ARG(len >= 1 && len <= c.Tmax, "lm_train_step_len: len must be in [1, seq]");
+  const int Tb = bucket_for(len);
+  c.set_active_T(Tb);
+  cudaStream_t st = c.main_st;
+  int32_t* tp = (int32_t*)(ws + off_tokpad);
+  CUDA_TRY(cudaMemcpyAsync(tp, tokens, (size_t)(len + 1) * c.B * 4, cudaMemcpyDeviceToDevice, st));
+  if (Tb > len) CUDA_TRY(cudaMemsetAsync(tp + (size_t)(len + 1) * c.B, 0, (size_t)(Tb - len) * c.B * 4, st));
+  set_state(nullptr, nullptr);   // sentence-level mini-batches: zero initial state, no carry
+  set_i32((int*)(ws + off_nv), len * c.B, st);   // read on the device: one graph per bucket
+  step_len = len;
+  try {
+    step(tp, lr, loss_dev, do_sgd);
+  } catch (...) {
+    step_len = 0;
+    throw;
+  }
+  step_len = 0;
 }
 
 size_t LM::find(const std::string& n) const {
@@ -106,21 +145,23 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   ASTRA_CHECK_STATE(bound, "lm_train_step: not bound");
   ASTRA_CHECK_ARG(tokens, "lm_train_step: tokens is null");
   Cell& c = *cell;
-  // exploration steps (and the fp32 parity path) run eagerly; a frozen / untuned bf16 step replays
+  // exploration steps (and the fp32 parity path) run eagerly; a frozen / untuned / converged bf16 step replays
   // multi-rank steps stay eager unless ASTRA_GRAPH_NCCL=1 (NCCL inside a capture is supported, but
   // a capture mismatch across ranks would hang the job; not exercisable on a 1-GPU test box)
   static const bool graph_nccl = [] {
     const char* e = std::getenv("ASTRA_GRAPH_NCCL");
     return e && e[0] == '1';
   }();
-  if (!use_graphs || !graphs_enabled() || c.tune_mode == ASTRA_TUNE_ON || c.ot != OT::BF16 ||
+  const bool exploring = c.tune_mode == ASTRA_TUNE_ON && !(c.wirer && c.wirer->converged());
+  if (!use_graphs || !graphs_enabled() || exploring || c.ot != OT::BF16 ||
       (c.world > 1 && !graph_nccl)) {
     enqueue_step(tokens, lr, loss_dev, do_sgd);
     return;
   }
   const std::string vs = c.var.str();
   for (auto& g : graphs)
-    if (g.tokens == tokens && g.lr == lr && g.loss == loss_dev && g.sgd == do_sgd && g.variant == vs) {
+    if (g.tokens == tokens && g.lr == lr && g.loss == loss_dev && g.sgd == do_sgd && g.variant == vs &&
+        g.T == c.T && g.len == (step_len > 0)) {
       CUDA_TRY(cudaGraphLaunch(g.exec, c.main_st));
       count_launch(g.launches);
       return;
@@ -149,11 +190,12 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   CUDA_TRY(cudaStreamEndCapture(cap_st, &graph));
   GraphEntry ge;
   ge.tokens = tokens; ge.lr = lr; ge.loss = loss_dev; ge.sgd = do_sgd; ge.variant = vs;
+  ge.T = c.T; ge.len = step_len > 0;
   ge.launches = g_launches.load() - l0;
   CUDA_TRY(cudaGraphInstantiate(&ge.exec, graph, 0));
   CUDA_TRY(cudaGraphDestroy(graph));
   g_launches.fetch_sub(ge.launches);   // captured, not yet launched
-  if (graphs.size() >= 4) {
+  if (graphs.size() >= 8) {
     cudaGraphExecDestroy(graphs.front().exec);
     graphs.erase(graphs.begin());
   }
@@ -182,8 +224,13 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
 
   // a0: embedding gather into the cell's operand buffer
   embed_gather(c.ot, tokens, TB, P + find("E"), c.I, c.x_operand(), c.Ip, st);
-  // cell forward (SE1); final state carried for the next step (truncated BPTT)
-  c.forward(nullptr, hs, cs, nullptr, hs, cs);
+  // cell forward (SE1); final state carried for the next step (truncated BPTT) — except for a
+  // variable-length step, whose padded tail would corrupt it (zero state, no carry)
+  if (step_len > 0) c.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
+  else c.forward(nullptr, hs, cs, nullptr, hs, cs);
+  // rows that carry a loss: a device scalar, so a captured step serves every length of its bucket
+  int* nvd = (int*)(ws + off_nv);
+  if (step_len == 0) set_i32(nvd, (int)TB, st);
 
   // a4: head forward + CE + head backward (SE2).  The head reads the cell's output operand
   // (SCRN: [h | s], a K-concatenated "ladder" [h|s]·[U;V]).
@@ -197,8 +244,8 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   hd.B = mat(Wom, Yw, V, Yw);
   hd.M = (int)TB; hd.N = V; hd.K = Yw;
   c.run_gemm(100, hd, epi(logits, V, (int)TB, V, 0, P + find("b_o")), 0, 0, c.var.g[G_HEAD], st);
-  ce_fwd_bwd(c.ot, logits, V, V, tokens + c.B, TB, 1.0f / (float)TB, rowloss, dlog, Vp, dlog32, st);
-  sum_rows_to_scalar(rowloss, TB, 1.0f / (float)TB, lossp, st);
+  ce_fwd_bwd(c.ot, logits, V, V, tokens + c.B, TB, 0.f, rowloss, dlog, Vp, dlog32, st, nvd);
+  sum_rows_to_scalar(rowloss, TB, 0.f, lossp, st, nvd);
   GemmSpec dy;
   dy.A = mat(dlog, V, TB, Vp);
   dy.B = mat(Wom, Yw, V, Yw);
@@ -213,14 +260,15 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
     dwo.B = mat(dlog, V, TB, Vp);
     dwo.b_mn = true;
     dwo.M = s.n; dwo.N = V; dwo.K = (int)TB;
-    dwo.ksplit = wo_ksplit;
+    const int wks = wo_split(TB);
+    dwo.ksplit = wks;
     float* dWo = G + find("W_o") + (size_t)s.r0 * V;
-    if (wo_ksplit > 1) {
+    if (wks > 1) {
       float* part = (float*)(ws + off_wopart);
       EpiStore ep = epi(part, V, s.n, V);
       ep.split_stride = (long)s.n * V;
       c.run_gemm(id++, dwo, ep, 0, 0, c.var.g[G_HEAD], st);
-      sum_split_partials(part, wo_ksplit, (long)s.n * V, dWo, st);
+      sum_split_partials(part, wks, (long)s.n * V, dWo, st);
     } else {
       c.run_gemm(id++, dwo, epi(dWo, V, s.n, V), 0, 0, c.var.g[G_HEAD], st);
     }

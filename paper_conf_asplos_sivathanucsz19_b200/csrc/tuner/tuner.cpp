@@ -56,7 +56,7 @@ struct Leaf : Node {
   }
   void feed(const Metrics& m) override {
     const double v = m.at(metric);
-    idx->record(ProfileIndex::key(ctx < 0 ? 0 : ctx, name, std::to_string(k)), v);
+    idx->record(ProfileIndex::key(ctx < 0 ? 0 : ctx, name, std::to_string(k), idx->bucket), v);
     if (better(v, bm, have)) { best = k; bm = v; have = true; }
     ++k;
   }
@@ -94,7 +94,7 @@ struct Exh : Node {
       nm += (i ? "+" : "") + kids[i]->name;
       ch += (i ? "," : "") + std::to_string(combo[i]);
     }
-    idx->record(ProfileIndex::key(ctx < 0 ? 0 : ctx, nm, ch), v);
+    idx->record(ProfileIndex::key(ctx < 0 ? 0 : ctx, nm, ch, idx->bucket), v);
     if (better(v, bm, have)) { best = combo; bm = v; have = true; }
     // advance: last child varies fastest (itertools.product order)
     int i = (int)kids.size() - 1;
@@ -239,7 +239,7 @@ struct Fork : Node {
     const double v = m.at(metric);
     cur_min = rep == 0 ? v : std::min(cur_min, v);
     if (++rep < reps) return;
-    idx->record(ProfileIndex::key(rc, "race", std::to_string(rc)), cur_min);
+    idx->record(ProfileIndex::key(rc, "race", std::to_string(rc), idx->bucket), cur_min);
     if (better(cur_min, bm, have)) { best = rc; bm = cur_min; have = true; }
     rep = 0;
     ++rc;

@@ -25,6 +25,7 @@ using Metrics = std::vector<double>;  // one value per metric (tree order)
 
 struct ProfileIndex {
   std::map<std::string, double> d;
+  int bucket = 0;   // key prefix "b=": the input-size bucket this index explores
   static std::string key(int ctx, const std::string& node, const std::string& choice, int bucket = 0, int se = 0);
   void record(const std::string& k, double v);
 };

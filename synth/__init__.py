@@ -11,7 +11,10 @@ its own.  The recipe (restated in DESIGN.md "Input recipe"):
 * weights ~ U(-1/sqrt(H), 1/sqrt(H)) (contractive dynamics, SURVEY §8(c.9));
 * MI-LSTM alpha/beta ~ U(0.5, 1.5) for tests;
 * states ~ U(-0.5, 0.5); inputs ~ U(-1, 1); upstream gradients ~ N(0, 1);
-* tokens ~ Zipf(s=1) over a symbol set, i.i.d. (PTB / enwik8-like frequency skew).
+* tokens ~ Zipf(s=1) over a symbol set, i.i.d. (PTB / enwik8-like frequency skew);
+* sentence lengths (bucketed workloads) ~ round(LogNormal(ln 20, 0.5)) clipped to [2, 83]:
+  its quintiles (13, 18, 23, 30) sit near the paper's PTB bucket edges 13/18/24/30 with a tail
+  to the 83 maximum.
 """
 from __future__ import annotations
 
@@ -68,3 +71,9 @@ def weights(seed: int, shapes: dict, hidden: int, overrides: dict | None = None)
         lo, hi = (overrides or {}).get(name, (-bound, bound))
         out[name] = uniform(seed, "param/" + name, shp, lo, hi)
     return out
+
+
+def ptb_like_lengths(seed: int, key: str, n: int, lo: int = 2, hi: int = 83) -> np.ndarray:
+    """n mini-batch lengths ~ round(LogNormal(mu = ln 20, sigma = 0.5)), clipped to [lo, hi]."""
+    x = rng(seed, key).lognormal(np.log(20.0), 0.5, size=n)
+    return np.clip(np.rint(x), lo, hi).astype(np.int64)
