@@ -152,7 +152,7 @@ class Cell:
     """One recurrent cell instance (astra_cell) with its parameters, gradients and workspace."""
 
     def __init__(self, cell, hidden, input, batch, seq, dtype="bf16", device=0, depth=0, context=0,
-                 scrn_alpha=0.0, src_seq=0, attn_dim=0, allocate=True, side_streams=1):
+                 scrn_alpha=0.0, src_seq=0, attn_dim=0, allocate=True, side_streams=2):
         import torch
         L = lib()
         self.cell_type = CELL_TYPES[cell] if isinstance(cell, str) else int(cell)

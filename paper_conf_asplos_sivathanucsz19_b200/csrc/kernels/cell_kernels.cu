@@ -522,7 +522,7 @@ void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void
 // one warp per row; fixed-order warp-shuffle trees
 template <typename T>
 __global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, const int32_t* __restrict__ targets,
-                          long n, float inv_n, const int* __restrict__ nvp, float* __restrict__ rowloss,
+                          long n, float inv_n, const int* __restrict__ nvp, long row0, float* __restrict__ rowloss,
                           T* __restrict__ dlog, long ldd, float* __restrict__ dlog32) {
   const long r = (long)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
   const int lane = threadIdx.x % 32;
@@ -530,7 +530,7 @@ __global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, con
   if (nvp) {   // rows ≥ *nvp are padding (bucketed steps): no loss, zero gradient; mean over *nvp rows
     const long nv = *nvp;
     inv_n = __fdiv_rn(1.f, (float)nv);
-    if (r >= nv) {
+    if (row0 + r >= nv) {
       if (lane == 0) rowloss[r] = 0.f;
       for (int c = lane; c < ldd; c += 32) dlog[r * ldd + c] = from_f<T>(0.f);
       for (int c = lane; c < V; c += 32) dlog32[r * V + c] = 0.f;
@@ -561,14 +561,14 @@ __global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, con
 }
 
 void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
-                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp) {
+                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp, long row0) {
   const int rows_per = 8;
   dim3 grid(cdiv(n, rows_per));
   if (ot == OT::BF16)
-    ce_kernel<__nv_bfloat16><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, rowloss,
+    ce_kernel<__nv_bfloat16><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, row0, rowloss,
                                                              (__nv_bfloat16*)dlog, ldd, dlog32);
   else
-    ce_kernel<float><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, rowloss, (float*)dlog,
+    ce_kernel<float><<<grid, 32 * rows_per, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, row0, rowloss, (float*)dlog,
                                                      ldd, dlog32);
   LAUNCH_CHECK();
 }

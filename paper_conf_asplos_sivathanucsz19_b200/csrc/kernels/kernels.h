@@ -74,7 +74,8 @@ void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);
 // rowloss[r] = lse - logit[target]; dlog (ot) and dlog32 = (softmax - onehot) * inv_n.
 void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
-                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp = nullptr);
+                float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp = nullptr,
+                long row0 = 0);
 // out[i] = Σ_{k < ks} part[k·n + i] in k order (split-K partials, R25/R28).
 void sum_split_partials(const float* part, int ks, long n, float* out, cudaStream_t st);
 void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st, const int* nvp = nullptr);

@@ -8,6 +8,7 @@
 //   RhnCell   — recurrent highway network [39]        (cell_rhn.cpp)
 //   AttnCell  — LSTM encoder + attentive decoder [35] (cell_attn.cpp)
 #pragma once
+#include <functional>
 #include <cuda_runtime.h>
 
 #include <map>
@@ -40,11 +41,13 @@ enum GemmRole { G_A1 = 0, G_REC, G_BPTT, G_DU, G_DW, G_DX, G_HEAD, G_ROLES };
 extern const char* const ROLE_NAMES[G_ROLES];
 
 // One binding of every adaptive variable (the enumerator's output for a cell).
+constexpr int HEAD_CHUNKS[3] = {1, 2, 5};
 struct Variant {
   KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
   int fwd_mode = 0;     // K2 (LSTM family, bf16): 0 GEMM + pointwise kernel, 1 fused per step, 2 fused persistent
   int bwd_mode = 0;     // K4: same encoding
+  int head_ov = 0;      // LM head overlapped with the forward chain in HEAD_CHUNKS[head_ov] time chunks (B3)
   int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
   Variant() { g[G_BPTT].bn = 128; }
   std::string str() const;                    // "a1=256.1.1,rec=...,wg_side=0"
@@ -147,6 +150,14 @@ class Cell {
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
+  // forward-step hook (set by the LM): called after forward step t is enqueued on the main stream,
+  // so the head of a finished time chunk is enqueued on a side stream in host order too (the
+  // overlap then also happens in eager, exploring steps, not only in a replayed graph)
+  std::function<void(int)> fwd_hook;   // called (host side) right after step t is enqueued
+  void fwd_step_done(int t, cudaStream_t) {
+    if (fwd_hook) fwd_hook(t);
+  }
+
   // ---- shared machinery
   void add_param(const char* n, int r, int c);
   size_t find_param(const std::string& n) const;
@@ -213,6 +224,7 @@ class LM {
   int step_len = 0;           // valid length of the step being enqueued (0 = full T)
   size_t off_tokpad = 0;      // int32 [Tmax+1][B] padded token buffer
   size_t off_nv = 0;          // int32 device scalar: rows of the step that carry a loss
+  cudaEvent_t ev_hfork = nullptr, ev_hdy = nullptr, ev_hdone = nullptr, ev_chunk[5] = {};
   int bucket_for(int len) const;
   void step_var(const int32_t* tokens, int len, float lr, float* loss_dev, bool do_sgd);
   int wo_split(long TB) const;   // R28 split for the active T·B

@@ -21,7 +21,7 @@ std::string Variant::str() const {
     if (g[r].cg != 1) o << "." << g[r].cg;
     o << ",";
   }
-  o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf;
+  o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf << ",hov=" << head_ov;
   return o.str();
 }
 
@@ -40,6 +40,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "wg_side") {
       v.wg_side = std::stoi(val);
       ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    if (k == "hov") {
+      v.head_ov = std::stoi(val);
+      ASTRA_CHECK_ARG(v.head_ov >= 0 && v.head_ov <= 2, "variant: hov must be 0..2 (head in 1, 2 or 5 time chunks)");
       continue;
     }
     if (k == "pf") {
@@ -307,6 +312,10 @@ void Cell::tuner_setup() {
   if (ot == OT::BF16 && chain_prefetch())
     t = "(pre " + t + " (par (leaf pf_fwd 2 t_fwd) (leaf pf_bwd 2 t_bptt)))";
   if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
+  // B3 stream assignment for the LM head: time-chunked on a side stream, overlapping the forward
+  // chain (its chunks' logits / CE / dgrad) and the BPTT chain (its weight gradient); step metric
+  if (lm_mode && !side.empty() && T >= 2)
+    t = "(pre " + t + " (leaf head_ov " + std::to_string(T >= 5 ? 3 : 2) + " t_step))";
   if (t.empty()) t = "(leaf none 1 t_step)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
   wirer.reset(new tuner::Wirer(tree.get()));
@@ -325,6 +334,7 @@ void Cell::apply_config(const tuner::Config& c) {
     const int o = c[i];
     if (n == "wg_side") { v.wg_side = o; continue; }
     if (n == "fuse_fwd") { v.fwd_mode = o; continue; }
+    if (n == "head_ov") { v.head_ov = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

@@ -156,6 +156,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
       ra.hT = last ? hT : nullptr;
       ra.cT = last ? cT : nullptr;
       lstm_fwd_pair_launch(kind, fm, ra, st);
+      fwd_step_done(t, st);
     }
   } else if (ot == OT::BF16 && var.fwd_mode > 0) {
     // K2 fused: GEMM + gate epilogue in one kernel (per step, or persistent over all steps)
@@ -175,11 +176,13 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
       CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
       ra.persistent = 1; ra.t0 = 0; ra.t1 = T;
       lstm_rec_fwd_launch(kind, tg.mapA, tg.mapB, ra, st);
+      for (int t = 0; t < T; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
     } else {
       ra.persistent = 0;
       for (int t = 0; t < T; ++t) {
         ra.t0 = t; ra.t1 = t + 1;
         lstm_rec_fwd_launch(kind, tg.mapA, tg.mapB, ra, st);
+        fwd_step_done(t, st);
       }
     }
   } else {
@@ -197,6 +200,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
         lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
                            Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y ? (char*)y + (size_t)t * B * H * e : nullptr,
                            H, ot, last ? hT : nullptr, last ? cT : nullptr, st);
+      fwd_step_done(t, st);
     }
   }
   mark(R_FWD, 1, st);

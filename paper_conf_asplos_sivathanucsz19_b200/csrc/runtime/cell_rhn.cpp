@@ -113,6 +113,7 @@ class RhnCell : public Cell {
                    sn, sno, (last && y) ? (char*)y + (size_t)t * B * H * e : nullptr, H,
                    (last && t == T - 1) ? sT : nullptr, st);
       }
+      fwd_step_done(t, st);
     }
     mark(R_FWD, 1, st);
     fwd_done = true;

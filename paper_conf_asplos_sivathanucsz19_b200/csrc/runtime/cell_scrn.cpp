@@ -132,6 +132,7 @@ class ScrnCell : public Cell {
       run_gemm(2, rec, epi(Z, Hp, B, Hp), t, 0, var.g[G_REC], st);
       scrn_fwd_pw(ot, B, H, Hp, XAB + (long)t * B * Yw, Yw, Z, p("b_h"), Hf + (long)(t + 1) * B * Hp, HSrow(t + 1),
                   Yw, y ? (char*)y + (size_t)t * B * ldy * e : nullptr, ldy, t == T - 1 ? hT : nullptr, st);
+      fwd_step_done(t, st);
     }
     mark(R_FWD, 1, st);
     fwd_done = true;

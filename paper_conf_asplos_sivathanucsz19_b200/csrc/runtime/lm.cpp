@@ -139,6 +139,10 @@ void LM::clear_graphs() {
 LM::~LM() {
   clear_graphs();
   if (cap_st) cudaStreamDestroy(cap_st);
+  for (cudaEvent_t ev : {ev_hfork, ev_hdy, ev_hdone})
+    if (ev) cudaEventDestroy(ev);
+  for (cudaEvent_t ev : ev_chunk)
+    if (ev) cudaEventDestroy(ev);
 }
 
 void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
@@ -222,36 +226,83 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   const int Vr = (int)round_up(V, 256);
   const std::vector<KSeg> segs = c.y_segments();
 
-  // a0: embedding gather into the cell's operand buffer
-  embed_gather(c.ot, tokens, TB, P + find("E"), c.I, c.x_operand(), c.Ip, st);
-  // cell forward (SE1); final state carried for the next step (truncated BPTT) — except for a
-  // variable-length step, whose padded tail would corrupt it (zero state, no carry)
-  if (step_len > 0) c.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
-  else c.forward(nullptr, hs, cs, nullptr, hs, cs);
   // rows that carry a loss: a device scalar, so a captured step serves every length of its bucket
   int* nvd = (int*)(ws + off_nv);
   if (step_len == 0) set_i32(nvd, (int)TB, st);
 
-  // a4: head forward + CE + head backward (SE2).  The head reads the cell's output operand
-  // (SCRN: [h | s], a K-concatenated "ladder" [h|s]·[U;V]).
-  c.mark(R_HEAD, 0, st);
-  CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, st));
+  // B3 stream assignment of the head (AV head_ov): the head of time chunk k (logits, CE, dgrad)
+  // runs on a side stream as soon as forward step t_k is done, overlapping the rest of the forward
+  // chain; its weight gradient overlaps the BPTT chain.  Row chunks of the same GEMMs, same CE and
+  // reductions: bitwise identical to the sequential head.
+  const int nch = HEAD_CHUNKS[std::min(2, std::max(0, c.var.head_ov))];
+  const bool ov = nch > 1 && !c.side.empty() && c.T >= nch;
+  cudaStream_t hst = ov ? c.side.back() : st;
+  if (ov) {
+    if (!ev_hfork) {
+      CUDA_TRY(cudaEventCreateWithFlags(&ev_hfork, cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&ev_hdy, cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&ev_hdone, cudaEventDisableTiming));
+      for (auto& e5 : ev_chunk) CUDA_TRY(cudaEventCreateWithFlags(&e5, cudaEventDisableTiming));
+    }
+    CUDA_TRY(cudaEventRecord(ev_hfork, st));
+    CUDA_TRY(cudaStreamWaitEvent(hst, ev_hfork, 0));
+  }
+  std::vector<int> t_end(nch);   // last forward step of each time chunk
+  for (int k = 0; k < nch; ++k) t_end[k] = (int)((long)(k + 1) * c.T / nch) - 1;
+
+  // a0: embedding gather into the cell's operand buffer
+  embed_gather(c.ot, tokens, TB, P + find("E"), c.I, c.x_operand(), c.Ip, st);
+  // head weight mirror (independent of the forward)
+  c.mark(R_HEAD, 0, hst);
+  CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, hst));
   for (const KSeg& s : segs)
-    mirror_T(c.ot, P + find("W_o") + (size_t)s.r0 * V, s.n, V, Vr, s.n, Wom + (size_t)s.k0 * e, Yw, st);
+    mirror_T(c.ot, P + find("W_o") + (size_t)s.r0 * V, s.n, V, Vr, s.n, Wom + (size_t)s.k0 * e, Yw, hst);
+  // a4 per time chunk: head forward + CE + head dgrad (SE2).  The head reads the cell's output
+  // operand (SCRN: [h | s], a K-concatenated "ladder" [h|s]·[U;V]).
   const Mat2 Y = c.y_operand();
-  GemmSpec hd;
-  hd.A = Y;
-  hd.B = mat(Wom, Yw, V, Yw);
-  hd.M = (int)TB; hd.N = V; hd.K = Yw;
-  c.run_gemm(100, hd, epi(logits, V, (int)TB, V, 0, P + find("b_o")), 0, 0, c.var.g[G_HEAD], st);
-  ce_fwd_bwd(c.ot, logits, V, V, tokens + c.B, TB, 0.f, rowloss, dlog, Vp, dlog32, st, nvd);
-  sum_rows_to_scalar(rowloss, TB, 0.f, lossp, st, nvd);
-  GemmSpec dy;
-  dy.A = mat(dlog, V, TB, Vp);
-  dy.B = mat(Wom, Yw, V, Yw);
-  dy.b_mn = true;
-  dy.M = (int)TB; dy.N = Yw; dy.K = V;
-  c.run_gemm(101, dy, epi(dY, Yw, (int)TB, Yw), 0, 0, c.var.g[G_HEAD], st);
+  auto head_chunk = [&](int k) {
+    const long r0 = k == 0 ? 0 : (long)(t_end[k - 1] + 1) * c.B, r1 = (long)(t_end[k] + 1) * c.B;
+    const int rows = (int)(r1 - r0);
+    if (ov) {
+      CUDA_TRY(cudaEventRecord(ev_chunk[k], st));
+      CUDA_TRY(cudaStreamWaitEvent(hst, ev_chunk[k], 0));
+    }
+    GemmSpec hd;
+    hd.A = mat((const char*)Y.ptr + (size_t)r0 * Y.ld * e, Y.inner, rows, Y.ld);
+    hd.B = mat(Wom, Yw, V, Yw);
+    hd.M = rows; hd.N = V; hd.K = Yw;
+    c.run_gemm(nch > 1 ? 120 + k : 100, hd, epi(logits + r0 * V, V, rows, V, 0, P + find("b_o")), 0, 0,
+               c.var.g[G_HEAD], hst);
+    ce_fwd_bwd(c.ot, logits + r0 * V, V, V, tokens + c.B + r0, rows, 0.f, rowloss + r0, (char*)dlog + (size_t)r0 * Vp * e,
+               Vp, dlog32 + r0 * V, hst, nvd, r0);
+    GemmSpec dy;
+    dy.A = mat((const char*)dlog + (size_t)r0 * Vp * e, V, rows, Vp);
+    dy.B = mat(Wom, Yw, V, Yw);
+    dy.b_mn = true;
+    dy.M = rows; dy.N = Yw; dy.K = V;
+    c.run_gemm(nch > 1 ? 130 + k : 101, dy, epi(dY + r0 * Yw, Yw, rows, Yw), 0, 0, c.var.g[G_HEAD], hst);
+  };
+  // cell forward (SE1); final state carried for the next step (truncated BPTT) — except for a
+  // variable-length step, whose padded tail would corrupt it (zero state, no carry)
+  if (ov)
+    c.fwd_hook = [&](int t) {
+      for (int k = 0; k < nch; ++k)
+        if (t == t_end[k]) head_chunk(k);
+    };
+  try {
+    if (step_len > 0) c.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
+    else c.forward(nullptr, hs, cs, nullptr, hs, cs);
+  } catch (...) {
+    c.fwd_hook = nullptr;
+    throw;
+  }
+  c.fwd_hook = nullptr;
+  if (!ov) head_chunk(0);
+  if (ov) {   // BPTT needs every dY row; the weight gradient of the head stays on the side stream
+    CUDA_TRY(cudaEventRecord(ev_hdy, hst));
+    CUDA_TRY(cudaStreamWaitEvent(st, ev_hdy, 0));
+  }
+  sum_rows_to_scalar(rowloss, TB, 0.f, lossp, hst, nvd);
   int id = 102;
   for (const KSeg& s : segs) {
     GemmSpec dwo;
@@ -267,16 +318,17 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
       float* part = (float*)(ws + off_wopart);
       EpiStore ep = epi(part, V, s.n, V);
       ep.split_stride = (long)s.n * V;
-      c.run_gemm(id++, dwo, ep, 0, 0, c.var.g[G_HEAD], st);
-      sum_split_partials(part, wks, (long)s.n * V, dWo, st);
+      c.run_gemm(id++, dwo, ep, 0, 0, c.var.g[G_HEAD], hst);
+      sum_split_partials(part, wks, (long)s.n * V, dWo, hst);
     } else {
-      c.run_gemm(id++, dwo, epi(dWo, V, s.n, V), 0, 0, c.var.g[G_HEAD], st);
+      c.run_gemm(id++, dwo, epi(dWo, V, s.n, V), 0, 0, c.var.g[G_HEAD], hst);
     }
   }
-  colsum(dlog32, TB, V, V, (float*)(ws + off_colsum), G + find("b_o"), st);
-  c.mark(R_HEAD, 1, st);
+  colsum(dlog32, TB, V, V, (float*)(ws + off_colsum), G + find("b_o"), hst);
+  c.mark(R_HEAD, 1, hst);
   // a7 bucket 1: the head gradients are final before BPTT — their sum overlaps the chain
-  c.grad_bucket(G + find("W_o"), n_params - find("W_o"), st);
+  c.grad_bucket(G + find("W_o"), n_params - find("W_o"), hst);
+  if (ov) CUDA_TRY(cudaEventRecord(ev_hdone, hst));
 
   // cell backward (SE3 + SE4) and the embedding backward
   c.lm_dy = dY;
@@ -284,6 +336,7 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   embed_bwd(tokens, TB, V, dX, c.Ip, c.I, G + find("E"), ws + off_sort, sort_bytes, (float*)(ws + off_embpart), st);
   // a7: last bucket (embedding), join, then a8: SGD
   c.grad_bucket(G + find("E"), (size_t)V * c.I, st);
+  if (ov) CUDA_TRY(cudaStreamWaitEvent(st, ev_hdone, 0));   // head gradients (and their bucket) done
   c.grad_join(st);
   if (do_sgd) sgd(P, G, n_params, lr, st);
   c.mark(R_STEP, 1, st);

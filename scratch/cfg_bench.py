@@ -34,8 +34,13 @@ def lm_run(name, cell, H, I, B, T, V, kw, steps=10):
     for _ in range(steps): m.train_step(tok, 0.01)
     e1.record(); torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / steps
+    import bench
+    m.set_graph(False)
+    m.train_step(tok, 0.01); torch.cuda.synchronize()
+    regions = {k: round(v, 3) for k, v in bench.region_times(c).items()}
+    m.set_graph(True)
     print(json.dumps({"config": name, "samples_per_s": round(B / ms * 1e3, 1), "ms_per_step": round(ms, 3),
-                      "loss": round(float(m.loss.item()), 4), "tuner_steps": n, "configs_explored": rep.get("configs_explored"),
+                      "regions_eager": regions, "loss": round(float(m.loss.item()), 4), "tuner_steps": n, "configs_explored": rep.get("configs_explored"),
                       "tuner_wall_s": round(tw, 2), "variant": rep["variant"]}), flush=True)
 
 

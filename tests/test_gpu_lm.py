@@ -156,3 +156,25 @@ def test_pdl_off_bitwise(tmp_path):
         subprocess.run([sys.executable, "-c", code, f], check=True, env=env, cwd=os.path.dirname(os.path.dirname(__file__)))
         outs.append(np.load(f))
     assert np.array_equal(outs[0], outs[1])
+
+
+@pytest.mark.parametrize("cell", ["milstm", "scrn", "rhn"])
+@pytest.mark.parametrize("hov", [1, 2])
+def test_head_overlap_bitwise(cell, hov):
+    """The LM head in 2 / 5 time chunks on a side stream, overlapping the forward and BPTT chains
+    (AV head_ov), gives the same bits as the sequential head over 4 SGD steps (graph replay)."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 7, 64, 64, 64, 300
+    out = []
+    for v in (0, hov):
+        p, tok, h0, c0 = _lm_case(cell, T, B, I, H, V, synth.config_seed(5) + 40, True)
+        c = A.Cell(cell, H, I, B, T, dtype="bf16", **_cell_kw(cell)[0])
+        m = A.LM(c, V)
+        m.load(p)
+        c.tune_mode(A.TUNE_FROZEN, f"hov={v}")
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(4):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append((m.params.clone(), float(m.loss.item())))
+    assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
