@@ -4,6 +4,7 @@
 #include <cub/device/device_scan.cuh>
 
 #include "cell_math.cuh"
+#include "lstm_bwd_row.cuh"
 #include "kernels.h"
 #include "pdl.cuh"
 #include "gemm.h"
@@ -326,18 +327,13 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
   throw Error(ASTRA_E_UNSUPPORTED, "lstm_fwd_pointwise: kind");
 }
 
-constexpr int BWD_RB = 32;  // rows per CTA in the backward pointwise kernel (= one partial chunk)
-constexpr int BWD_UX = 64;  // units per CTA (one gate group); thread tx owns unit u0 + tx
-constexpr int BWD_RY = 4;   // row lanes per CTA (threadIdx.y); thread handles rows b0 + ty + 4i
 int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 
-// K4 backward half + K5 column partials.  CTA = 64 hidden units (all four gates) x 32 batch rows;
-// thread (tx, ty) owns unit u0 + tx (its 4 gates' parameters in registers) for rows b0 + ty,
-// b0 + ty + 4, ...; a warp reads 128-byte runs of every gate's pre-activations.  Column partial
-// sums (db, dα, dβ1, dβ2) are accumulated per thread in ascending row order in its own shared-
-// memory slots, combined across the 4 row lanes in ty order, and added to partials[chunk][q][col]
-// — one owner per element, steps ordered on the stream, so the reduction order is fixed (R5: no
-// floating-point atomics).  256-thread CTAs at <= 64 registers: one resident wave at B = 512.
+// K4 backward half + K5 column partials (unfused variant).  CTA = 64 hidden units (all four gates)
+// x 32 batch rows; thread (tx, ty) owns unit u0 + tx (its 4 gates' parameters in registers) for
+// rows b0 + ty, b0 + ty + 4, ...; a warp reads 128-byte runs of every gate's pre-activations.  The
+// row arithmetic and the column-sum order are lstm_bwd_row.cuh's, shared with the fused BPTT kernel.
+// 256-thread CTAs at <= 64 registers: one resident wave at B = 512.
 template <int KIND, typename T, typename TDY>
 __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
     lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
@@ -345,7 +341,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
                        const float* __restrict__ WX, const float* __restrict__ UH, const float* __restrict__ c_new,
                        const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
                        T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
-  constexpr int NV = KIND == K_MILSTM ? 16 : 4;   // accumulated quantities per unit: q*4 + gate
+  constexpr int NV = BwdNV<KIND>::value;
   __shared__ float red[BWD_RY][NV][BWD_UX];
   pdl_wait();
   pdl_trigger();
@@ -354,8 +350,9 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
+  float acc[NV];
 #pragma unroll
-  for (int i = 0; i < NV; ++i) red[ty][i][tx] = 0.f;
+  for (int i = 0; i < NV; ++i) acc[i] = 0.f;
   if (j < H) {
     float bb[4], al[4], be1[4], be2[4];
 #pragma unroll
@@ -371,7 +368,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
     for (int b = b0 + ty; b < b1; b += BWD_RY) {
       const float* wxp = WX + (long)b * NG + c0;
       const float* uhp = UH + (long)b * NG + c0;
-      float w[4], h[4], a[4];
+      float w[4], h[4];
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
         w[g] = __ldcs(wxp + g * GATE_U);
@@ -386,34 +383,9 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
       }
       const long ro = (long)b * Hp + j;
       float dcv = dc[ro];
-      const float cp = c_prev[ro], cn = c_new[ro];
-#pragma unroll
-      for (int g = 0; g < 4; ++g) a[g] = preact<KIND, FastMath<T>::value>(w[g], h[g], bb[g], al[g], be1[g], be2[g]);
-      float da[4];
-      cell_bwd<KIND, FastMath<T>::value>(a, cp, cn, dh, dcv, da);
+      lstm_bwd_row<KIND, T>(w, h, dh, dcv, c_prev[ro], c_new[ro], bb, al, be1, be2, acc, D_uh + (long)b * NG + c0,
+                            D_wx + (long)b * NG + c0);
       dc[ro] = dcv;
-      T* duhp = D_uh + (long)b * NG + c0;
-      T* dwxp = D_wx + (long)b * NG + c0;
-#pragma unroll
-      for (int g = 0; g < 4; ++g) {
-        red[ty][g][tx] = __fadd_rn(red[ty][g][tx], da[g]);
-        if (KIND == K_MILSTM) {
-          constexpr bool F = FastMath<T>::value;   // bf16 path: fused multiply-adds (reading R27)
-          const float gu = F ? __fmaf_rn(al[g], w[g], be1[g]) : __fadd_rn(__fmul_rn(al[g], w[g]), be1[g]);
-          const float gw = F ? __fmaf_rn(al[g], h[g], be2[g]) : __fadd_rn(__fmul_rn(al[g], h[g]), be2[g]);
-          duhp[g * GATE_U] = from_f<T>(__fmul_rn(da[g], gu));
-          __stcs(dwxp + g * GATE_U, from_f<T>(__fmul_rn(da[g], gw)));
-          const float dw = __fmul_rn(da[g], w[g]);
-          float* r4 = &red[ty][NV > 4 ? 4 : 0][tx];
-          r4[g * BWD_UX] = F ? __fmaf_rn(dw, h[g], r4[g * BWD_UX]) : __fadd_rn(r4[g * BWD_UX], __fmul_rn(dw, h[g]));
-          float* r8 = &red[ty][NV > 8 ? 8 : 0][tx];
-          r8[g * BWD_UX] = F ? __fmaf_rn(da[g], h[g], r8[g * BWD_UX]) : __fadd_rn(r8[g * BWD_UX], __fmul_rn(da[g], h[g]));
-          float* r12 = &red[ty][NV > 12 ? 12 : 0][tx];
-          r12[g * BWD_UX] = __fadd_rn(r12[g * BWD_UX], dw);
-        } else {
-          duhp[g * GATE_U] = from_f<T>(da[g]);
-        }
-      }
     }
   } else if (j < Hp) {  // padding units: keep their gradients exactly zero
     for (int b = b0 + ty; b < b1; b += BWD_RY) {
@@ -425,18 +397,11 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
       dc[(long)b * Hp + j] = 0.f;
     }
   }
+#pragma unroll
+  for (int i = 0; i < NV; ++i) red[ty][i][tx] = acc[i];
   __syncthreads();
   if (j >= Hp) return;
-  // thread (tx, ty) finalises quantities i = ty, ty + 4, ... (fixed ty order inside)
-  for (int i = ty; i < NV; i += BWD_RY) {
-    float v = 0.f;
-#pragma unroll
-    for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[y][i][tx]);
-    const int q = i / 4, g = i % 4;
-    if (q >= nq) continue;
-    float* p = partials + ((long)chunk * nq + q) * NG + gcol(g, j);
-    *p = first ? v : __fadd_rn(*p, v);
-  }
+  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, gcol(0, j), nq, first);
 }
 
 template <int KIND, typename T>

@@ -53,4 +53,30 @@ void lstm_fwd_pair_launch(int kind, const RecFwd2Maps& m, RecFwd2Args a, cudaStr
 // mapB: the U mirror [NG][Hp] K-major, box {64, 256}.
 void lstm_rec_fwd_launch(int kind, const CUtensorMap& mapA, const CUtensorMap& mapB, RecFwdArgs a, cudaStream_t st);
 
+// Fused BPTT step (bptt_fused.cu): dh_rec = D_uh_{t+1}·Uᵀ (canonical split-K kept as nsplit TMEM
+// accumulators) + the cell backward of step t; one launch per step t < T-1.
+struct BpttFusedArgs {
+  int B, H, Hp, NG, t;
+  int nk, kper, nsplit;     // k-blocks of K = NG, k-blocks per split-K chunk, chunks (reading R25)
+  int stages;
+  uint32_t idesc;           // M = 128, N = 64, A K-major, B MN-major bf16 MMA
+  int nq;                   // column-sum quantities (4 MI-LSTM: b, α, β1, β2; else 1)
+  GateParams gp;
+  void* D_uh;               // bf16 [T·B][NG] (base; the kernel writes step t's slice)
+  void* D_wx;
+  float* dc;                // [B][Hp]
+  float* partials;          // [chunks][nq][NG]
+};
+struct BpttFusedMaps {
+  CUtensorMap A;    // D_uh [T][B][NG] bf16, K-major, box {64, 128} (z = t+1)
+  CUtensorMap B;    // U mirror [NG][Hp] bf16 as MN-major B, box {64, 64}
+  CUtensorMap WX;   // [T][B][NG] fp32, box {256, 16}
+  CUtensorMap UH;   // [T][B][NG] fp32, box {256, 16}
+  CUtensorMap C;    // [T+1][B][Hp] fp32, box {64, 16}
+  CUtensorMap DC;   // [1][B][Hp] fp32, box {64, 16}
+  CUtensorMap DY;   // dy [T][B][ld] fp32 (LM internal, ld = Hp) or bf16 (external, ld = H), box {64, 16}
+};
+bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);
+void lstm_bptt_fused_launch(int kind, bool dy_bf16, const BpttFusedMaps& m, BpttFusedArgs a, cudaStream_t st);
+
 }  // namespace astra

@@ -148,6 +148,7 @@ class Cell {
   virtual bool lm_capable() const { return true; }
   virtual bool chain_prefetch() const { return false; }   // supports Variant::l2pf (tuner AVs pf_fwd / pf_bwd)
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
+  virtual int bwd_fusions() const { return 1; }   // number of K4 fusion choices (tuner AV "fuse_bwd")
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
   // forward-step hook (set by the LM): called after forward step t is enqueued on the main stream,

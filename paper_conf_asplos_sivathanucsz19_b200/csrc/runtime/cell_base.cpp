@@ -308,6 +308,8 @@ void Cell::tuner_setup() {
   // P:120-126 "fusion" AV) is tuned after the kernel choices, against the forward-chain time
   if (ot == OT::BF16 && fwd_fusions() > 1)
     t = "(pre " + t + " (leaf fuse_fwd " + std::to_string(fwd_fusions()) + " t_fwd))";
+  if (ot == OT::BF16 && bwd_fusions() > 1)
+    t = "(pre " + t + " (leaf fuse_bwd " + std::to_string(bwd_fusions()) + " t_bptt))";
   // reading R31: L2 prefetch by the chain GEMMs, per chain, after the kernel and fusion choices
   if (ot == OT::BF16 && chain_prefetch())
     t = "(pre " + t + " (par (leaf pf_fwd 2 t_fwd) (leaf pf_bwd 2 t_bptt)))";
@@ -334,6 +336,7 @@ void Cell::apply_config(const tuner::Config& c) {
     const int o = c[i];
     if (n == "wg_side") { v.wg_side = o; continue; }
     if (n == "fuse_fwd") { v.fwd_mode = o; continue; }
+    if (n == "fuse_bwd") { v.bwd_mode = o; continue; }
     if (n == "head_ov") { v.head_ov = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }

@@ -7,6 +7,8 @@
 //   bwd : for t desc: dh_rec = D_uh[t+1]·Uᵀ (K1) ; pointwise cell backward (K4 half, K5 partials)
 //         → dh0 → wgrad dU = Hᵀ·D_uh, dW = Xᵀ·D_wx (K1) → dX = D_wx·Wᵀ (K1) → bias/α/β reductions (K5)
 //         → gradient sum over ranks (K11) when world > 1.
+#include <cstring>
+
 #include "../kernels/cell_math.cuh"
 #include "../kernels/rec_fused.h"
 #include "cell.h"
@@ -64,6 +66,13 @@ class LstmCell : public Cell {
   const void* fm_key = (const void*)1;  // y pointer the maps were built for
   const void* fm_wx = nullptr;          // workspace they were built for (rebind ⇒ rebuild)
   int fm_T = 0;                         // active length the y map was built for
+  BpttFusedMaps bm;                     // tensor maps of the fused BPTT kernel
+  const void* bm_key[4] = {nullptr, nullptr, nullptr, nullptr};   // (WX, dy, Duh, T) they were built for
+
+  // K4 fusion choices (AV fuse_bwd): GEMM + pointwise kernel, or the fused BPTT kernel
+  int bwd_fusions() const override {
+    return (ot == OT::BF16 && lstm_bptt_fused_supported(B, Hp, bptt_ksplit())) ? 2 : 1;
+  }
 
   void* Hrow(int t) { return saved + off_H + (size_t)t * B * Hp * esz(); }
   void* x_operand() override { return sv<char>(off_X); }
@@ -242,7 +251,39 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   bp.b_keep = true;
   GemmSpec bp0 = bp;   // dh0 (once, no split)
   bp.ksplit = bptt_ksplit();
+  // fused BPTT step (K4 fused): dy must be TMA-mappable (the LM's fp32 dY, or bf16 with H % 8 == 0)
+  const bool fuse = var.bwd_mode == 1 && bwd_fusions() > 1 && T > 1 &&
+                    (lm_dy || (H % 8 == 0 && ((uintptr_t)dy & 15) == 0));
+  BpttFusedArgs fa{};
+  if (fuse) {
+    const TcGemm& tg = tc_get(2, bp, KCfg{64, 1, 1});
+    const void* key[4] = {WX, lm_dy ? (const void*)lm_dy : dy, Duh, (const void*)(uintptr_t)T};
+    if (std::memcmp(key, bm_key, sizeof(key)) != 0) {
+      bm.A = tg.mapA;
+      bm.B = tg.mapB;
+      make_tile_map(&bm.WX, WX, false, NG, B, Tmax, NG, (long)B * NG, 256, 16, 0);
+      make_tile_map(&bm.UH, UH, false, NG, B, Tmax, NG, (long)B * NG, 256, 16, 0);
+      make_tile_map(&bm.C, Cb, false, Hp, B, Tmax + 1, Hp, (long)B * Hp, 64, 16, 0);
+      make_tile_map(&bm.DC, dC, false, Hp, B, 1, Hp, 0, 64, 16, 0);
+      if (lm_dy) make_tile_map(&bm.DY, lm_dy, false, Hp, B, Tmax, Hp, (long)B * Hp, 64, 16, 0);
+      else make_tile_map(&bm.DY, dy, true, H, B, T, H, (long)B * H, 64, 16, 0);
+      std::memcpy(bm_key, key, sizeof(key));
+    }
+    fa.B = B; fa.H = H; fa.Hp = Hp; fa.NG = NG;
+    fa.nk = cdiv(NG, TC_BK);
+    fa.nsplit = bp.ksplit;
+    fa.kper = cdiv(fa.nk, fa.nsplit);
+    fa.idesc = tg.args.idesc;
+    fa.nq = nq;
+    fa.gp = gp;
+    fa.D_uh = Duh; fa.D_wx = Dwx; fa.dc = dC; fa.partials = part;
+  }
   for (int t = T - 1; t >= 0; --t) {
+    if (fuse && t < T - 1) {
+      fa.t = t;
+      lstm_bptt_fused_launch(kind, !lm_dy, bm, fa, st);
+      continue;
+    }
     const void* dyt;
     long ldy;
     bool dyf32;

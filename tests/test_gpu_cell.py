@@ -78,6 +78,25 @@ def test_fused_pair_forward_ragged(cell):
     _check(cell, 4, 300, 64, 100, "bf16", synth.config_seed(5) + 41, TOL_BF16, variant="fwd=1")
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+@pytest.mark.parametrize("T,B,H", [(6, 260, 192), (4, 300, 128), (3, 64, 2048)])
+def test_fused_bwd_bitwise(cell, T, B, H):
+    """K4 fused (GEMM + cell backward in one kernel per step, bwd=1) gives the same bits as the
+    BPTT GEMM + unfused pointwise kernel (bwd=0): ragged row tiles, split-K 1 / 4, and the oracle."""
+    I = 64
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, 91, bf16=True)
+    ref = None
+    for v in ("bwd=0", "bwd=1"):
+        out, g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, "bf16", v)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    _check(cell, T, B, I, H, "bf16", 91, TOL_BF16, variant="bwd=1")
+
+
 def test_variants_bitwise():
     """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
     T, B, I, H = 6, 160, 128, 192

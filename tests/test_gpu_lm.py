@@ -178,3 +178,24 @@ def test_head_overlap_bitwise(cell, hov):
         torch.cuda.synchronize()
         out.append((m.params.clone(), float(m.loss.item())))
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
+
+
+@pytest.mark.parametrize("cell,H", [("milstm", 192), ("milstm", 2048), ("lstm", 256)])
+def test_fused_bptt_lm_bitwise(cell, H):
+    """LM steps with the fused BPTT kernel (bwd=1, the LM's fp32 dY streamed by TMA) give the same
+    bits as GEMM + unfused pointwise (bwd=0) over 3 SGD steps; H = 2048 uses the 4-way split-K."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, V = 4, 96, 128, 64
+    out = []
+    for v in ("bwd=0", "bwd=1"):
+        p, tok, h0, c0 = _lm_case(cell, T, B, I, H, V, synth.config_seed(5) + 50, True)
+        c = A.Cell(cell, H, I, B, T, dtype="bf16")
+        m = A.LM(c, V)
+        m.load(p)
+        c.tune_mode(A.TUNE_FROZEN, v)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(3):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append((m.params.clone(), float(m.loss.item())))
+    assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
