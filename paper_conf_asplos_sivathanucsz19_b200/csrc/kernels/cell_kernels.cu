@@ -183,12 +183,33 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   const int ub = blockIdx.x % a.nub, b_first = blockIdx.x / a.nub;
   const int u0 = ub * FB_UB, nu = min(FB_UB, a.Hp - u0);   // nu: multiple of 64
   const long NG = 4L * a.Hp;
+  const int nitems = b_first < a.B ? (a.B - b_first + a.rstep - 1) / a.rstep : 0;
+  const uint32_t wbytes = (uint32_t)nu * 16, cbytes = (uint32_t)nu * 4;
+  // WX_t (the a1 GEMM's output) and c_{t-1} (the previous pointwise kernel's, complete before the
+  // GEMM of this step released us) are older than the grid dependency: their copies for the first
+  // stages go out before griddepcontrol.wait; UH_t (the GEMM's output) after it.
+  auto issue_old = [&](int k) {
+    const int s = k % FB_STAGES;
+    const long b = b_first + (long)k * a.rstep;
+    uint8_t* st = sm + s * FB_STAGE;
+    sm100::mbar_arrive_expect_tx(&full[s], 2 * wbytes + cbytes);
+    sm100::bulk_load(sm100::smem_u32(st), a.WX + b * NG + (long)u0 * 4, wbytes, &full[s]);
+    sm100::bulk_load(sm100::smem_u32(st + 2 * FB_SW), a.c_prev + b * a.Hp + u0, cbytes, &full[s]);
+  };
+  auto issue_new = [&](int k) {
+    const int s = k % FB_STAGES;
+    const long b = b_first + (long)k * a.rstep;
+    sm100::bulk_load(sm100::smem_u32(sm + s * FB_STAGE + FB_SW), a.UH + b * NG + (long)u0 * 4, wbytes, &full[s]);
+  };
   if (tid == 0) {
     for (int s = 0; s < FB_STAGES; ++s) sm100::mbar_init(&full[s], 1);
     sm100::fence_barrier_init();
+    for (int k = 0; k < FB_STAGES && k < nitems; ++k) issue_old(k);
   }
   pdl_wait();
   pdl_trigger();
+  if (tid == 0)
+    for (int k = 0; k < FB_STAGES && k < nitems; ++k) issue_new(k);
   for (int i = tid; i < 4 * nu; i += FB_THREADS) {
     const int g = i / nu, ul = i % nu, j = u0 + ul, e = g * a.H + j;
     const bool ok = j < a.H;
@@ -200,19 +221,6 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
     }
   }
   __syncthreads();
-  const int nitems = b_first < a.B ? (a.B - b_first + a.rstep - 1) / a.rstep : 0;
-  const uint32_t wbytes = (uint32_t)nu * 16, cbytes = (uint32_t)nu * 4;
-  auto issue = [&](int k) {
-    const int s = k % FB_STAGES;
-    const long b = b_first + (long)k * a.rstep;
-    uint8_t* st = sm + s * FB_STAGE;
-    sm100::mbar_arrive_expect_tx(&full[s], 2 * wbytes + cbytes);
-    sm100::bulk_load(sm100::smem_u32(st), a.WX + b * NG + (long)u0 * 4, wbytes, &full[s]);
-    sm100::bulk_load(sm100::smem_u32(st + FB_SW), a.UH + b * NG + (long)u0 * 4, wbytes, &full[s]);
-    sm100::bulk_load(sm100::smem_u32(st + 2 * FB_SW), a.c_prev + b * a.Hp + u0, cbytes, &full[s]);
-  };
-  if (tid == 0)
-    for (int k = 0; k < FB_STAGES && k < nitems; ++k) issue(k);
   const int ul = 2 * tid;
   const bool act = ul < nu;
   const int base = (ul / 64) * 256 + ul % 64;
@@ -277,7 +285,8 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
     __syncthreads();   // stage s fully consumed
     if (tid == 0 && k + FB_STAGES < nitems) {
       sm100::fence_proxy_async_smem();
-      issue(k + FB_STAGES);
+      issue_old(k + FB_STAGES);
+      issue_new(k + FB_STAGES);
     }
   }
 }
