@@ -78,6 +78,59 @@ def lm_forward_backward(cell, p, tokens, h0, c0, **kw):
     return loss, grads, (hT, cT)
 
 
+def _cell_forward(cell, p, x, h0, c0, **kw):
+    if cell in ("lstm", "milstm", "sublstm"):
+        fwd = {"lstm": C.lstm_forward, "milstm": C.milstm_forward, "sublstm": C.sublstm_forward}[cell]
+        return fwd(p, x, h0, c0)
+    if cell == "scrn":
+        return C.scrn_forward(p, x, h0, c0, kw["alpha"])
+    if cell == "rhn":
+        y, hT, cache = C.rhn_forward(p, x, h0)
+        return y, hT, None, cache
+    raise ValueError(cell)
+
+
+def _cell_backward(cell, p, x, cache, dY, h0, c0, **kw):
+    zeros_h = np.zeros_like(h0)
+    if cell in ("lstm", "milstm", "sublstm"):
+        bwd = {"lstm": C.lstm_backward, "milstm": C.milstm_backward, "sublstm": C.sublstm_backward}[cell]
+        g, dx, _, _ = bwd(p, x, cache, dY, zeros_h, np.zeros_like(c0))
+    elif cell == "scrn":
+        g, dx, _, _ = C.scrn_backward(p, x, cache, dY, zeros_h, np.zeros_like(c0), kw["alpha"])
+    else:
+        g, dx, _ = C.rhn_backward(p, x, cache, dY, zeros_h)
+    return g, dx
+
+
+def stacked_lm_forward_backward(cells, ps, plm, tokens, h0s, c0s, **kw):
+    """Stacked LM (PTB stacked LSTM): x_0 = E[tok], layer l maps
+    x_l to y_l = x_{l+1}, the head reads the top layer; BPTT runs top down, layer l's input
+    gradient being layer l-1's upstream gradient.  ps: per-layer parameter dicts; plm: E, W_o, b_o.
+    Returns (loss, [per-layer grads], head/embedding grads)."""
+    T = tokens.shape[0] - 1
+    B = tokens.shape[1]
+    x = plm["E"][tokens[:T]]
+    xs, caches = [], []
+    for cell, p, h0, c0 in zip(cells, ps, h0s, c0s):
+        xs.append(x)
+        y, _, _, cache = _cell_forward(cell, p, x, h0, c0, **kw)
+        caches.append(cache)
+        x = y
+    Hout = x.shape[2]
+    Y = x.reshape(T * B, Hout)
+    logits = Y @ plm["W_o"] + plm["b_o"]
+    loss, dlogits = cross_entropy(logits, tokens[1:].reshape(-1))
+    glm = {"W_o": Y.T @ dlogits, "b_o": dlogits.sum(0)}
+    dy = (dlogits @ plm["W_o"].T).reshape(T, B, Hout)
+    gl = [None] * len(cells)
+    for l in range(len(cells) - 1, -1, -1):
+        gl[l], dy = _cell_backward(cells[l], ps[l], xs[l], caches[l], dy, h0s[l], c0s[l], **kw)
+    dE = np.zeros_like(plm["E"])
+    np.add.at(dE, tokens[:T].reshape(-1), dy.reshape(T * B, -1))
+    glm["E"] = dE
+    return loss, gl, glm
+
+
 def sgd(p, grads, lr):
     """θ ← θ − lr·g for every parameter that has a gradient (a8)."""
     return {k: (v - lr * grads[k]) if k in grads else v for k, v in p.items()}

@@ -111,3 +111,73 @@ def test_dp_linearity(N):
     assert abs(loss - ldp) < 1e-13
     for k in g:
         np.testing.assert_allclose(gdp[k], g[k], atol=1e-13)
+
+
+def _stack_setup(cells, T=3, B=4, I=5, H=6, V=9, L=2):
+    ps, h0s, c0s = [], [], []
+    n_in = I
+    for l, cell in enumerate(cells):
+        if cell in ("lstm", "milstm"):
+            shapes = C.milstm_param_shapes(n_in, H) if cell == "milstm" else C.lstm_param_shapes(n_in, H)
+        else:
+            shapes = C.rhn_param_shapes(n_in, H, L)
+        ps.append(synth.weights(SEED + l, shapes, H, {"alpha": (0.5, 1.5), "beta1": (0.5, 1.5), "beta2": (0.5, 1.5)}))
+        h0s.append(synth.uniform(SEED + l, "h0", (B, H), -0.5, 0.5))
+        c0s.append(synth.uniform(SEED + l, "c0", (B, H), -0.5, 0.5) if cell != "rhn" else None)
+        n_in = H
+    plm = synth.weights(SEED, {"E": (V, I), **lm.head_param_shapes(H, V)}, H)
+    tok = synth.zipf_tokens(SEED, "tok", (T + 1, B), V, n_symbols=V - 2)
+    return ps, plm, tok, h0s, c0s
+
+
+def test_stacked_lstm_lm_matches_torch():
+    """Two stacked LSTM layers + head + mean CE == torch.nn.LSTM(num_layers=2) + Linear +
+    cross_entropy with autograd (fp64): loss and every gradient (W_ih = Wᵀ, W_hh = Uᵀ, b_hh = 0)."""
+    T, B, I, H, V = 4, 3, 5, 6, 9
+    ps, plm, tok, h0s, c0s = _stack_setup(["lstm", "lstm"], T, B, I, H, V)
+    loss, gl, glm = lm.stacked_lm_forward_backward(["lstm", "lstm"], ps, plm, tok, h0s, c0s)
+    net = torch.nn.LSTM(I, H, num_layers=2).double()
+    with torch.no_grad():
+        for l in range(2):
+            getattr(net, f"weight_ih_l{l}").copy_(torch.tensor(ps[l]["W"].T))
+            getattr(net, f"weight_hh_l{l}").copy_(torch.tensor(ps[l]["U"].T))
+            getattr(net, f"bias_ih_l{l}").copy_(torch.tensor(ps[l]["b"]))
+            getattr(net, f"bias_hh_l{l}").zero_()
+    E = torch.tensor(plm["E"], requires_grad=True)
+    Wo = torch.tensor(plm["W_o"], requires_grad=True)
+    bo = torch.tensor(plm["b_o"], requires_grad=True)
+    x = E[torch.tensor(tok[:T], dtype=torch.long)]
+    h0 = torch.tensor(np.stack(h0s))
+    c0 = torch.tensor(np.stack(c0s))
+    y, _ = net(x, (h0, c0))
+    ref = torch.nn.functional.cross_entropy(y.reshape(T * B, H) @ Wo + bo,
+                                            torch.tensor(tok[1:].reshape(-1), dtype=torch.long))
+    ref.backward()
+    assert abs(loss - ref.item()) < 1e-13
+    np.testing.assert_allclose(glm["E"], E.grad.numpy(), atol=1e-14)
+    np.testing.assert_allclose(glm["W_o"], Wo.grad.numpy(), atol=1e-14)
+    for l in range(2):
+        np.testing.assert_allclose(gl[l]["W"], getattr(net, f"weight_ih_l{l}").grad.numpy().T, atol=1e-14)
+        np.testing.assert_allclose(gl[l]["U"], getattr(net, f"weight_hh_l{l}").grad.numpy().T, atol=1e-14)
+        np.testing.assert_allclose(gl[l]["b"], getattr(net, f"bias_ih_l{l}").grad.numpy(), atol=1e-14)
+
+
+@pytest.mark.parametrize("cells", [["milstm", "milstm"], ["rhn", "rhn", "rhn"]])
+def test_stacked_lm_fd(cells):
+    """Central FD of the stacked LM loss in random directions, every layer's parameters and E."""
+    ps, plm, tok, h0s, c0s = _stack_setup(cells)
+    loss, gl, glm = lm.stacked_lm_forward_backward(cells, ps, plm, tok, h0s, c0s)
+    rng = np.random.default_rng(5)
+    eps = 1e-6
+    targets = [(ps[l], k, gl[l][k]) for l in range(len(cells)) for k in ps[l]] + [(plm, "E", glm["E"])]
+    for p, k, g in targets:
+        d = rng.standard_normal(p[k].shape)
+        orig = p[k].copy()
+        p[k] = orig + eps * d
+        lp = lm.stacked_lm_forward_backward(cells, ps, plm, tok, h0s, c0s)[0]
+        p[k] = orig - eps * d
+        lmn = lm.stacked_lm_forward_backward(cells, ps, plm, tok, h0s, c0s)[0]
+        p[k] = orig
+        fd = (lp - lmn) / (2 * eps)
+        an = float((g * d).sum())
+        assert abs(fd - an) <= 1e-7 * max(1.0, abs(an)) + 1e-10, (k, fd, an)
