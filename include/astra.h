@@ -145,6 +145,15 @@ astra_status astra_comm_unique_id(void* out, size_t len);
 /* ---- language-model wrapper (embedding → cell → linear head → mean CE) ----------------- */
 /* Adds E [V][I], W_o [Hout][V], b_o [V] after the cell's parameters in one flat vector.    */
 astra_status astra_lm_create(astra_lm* out, astra_cell c, int vocab);
+/* Stacked LM (the paper's PTB stacked LSTM, Table 5): cells[0] is
+ * the bottom layer (fed by the embedding), cells[n-1] the top (read by the head); layer l+1's
+ * input size must equal layer l's output size, all layers share batch, seq and dtype, and outputs
+ * must be single-segment (LSTM family, RHN; not SCRN).  Parameters: each layer's block with its
+ * names prefixed "L<l>.", then E, W_o, b_o.  The cells stay owned by the caller and must outlive
+ * the LM; astra_lm_set_state takes the layers' states concatenated in layer order.  Each cell
+ * keeps its own tuner (call astra_tune_next on every layer after a step).  E_ARG on a shape
+ * mismatch, E_UNSUPPORTED for a cell type without an LM form.                                 */
+astra_status astra_lm_create_stacked(astra_lm* out, const astra_cell* cells, int n_layers, int vocab);
 astra_status astra_lm_destroy(astra_lm m);
 astra_status astra_lm_param_count(astra_lm m, size_t* n_params);
 astra_status astra_lm_param_info(astra_lm m, int idx, const char** name, size_t* offset, int* rows, int* cols);

@@ -60,6 +60,7 @@ _SIGS = {
     "astra_comm_unique_id": [_P, _SZ],
     "astra_lm_create": [ctypes.POINTER(_P), _P, _I],
     "astra_lm_destroy": [_P],
+    "astra_lm_create_stacked": [ctypes.POINTER(_P), _P, _I, _I],
     "astra_lm_param_count": [_P, ctypes.POINTER(_SZ)],
     "astra_lm_param_info": [_P, _I, ctypes.POINTER(ctypes.c_char_p), ctypes.POINTER(_SZ), ctypes.POINTER(_I),
                             ctypes.POINTER(_I)],
@@ -256,13 +257,21 @@ def _param_info(fn, h):
 class LM:
     """Embedding → cell → linear head → mean cross-entropy, with SGD (astra_lm)."""
 
-    def __init__(self, cell: Cell, vocab: int):
+    def __init__(self, cell, vocab: int):
+        """cell: one Cell, or a list of Cells stacked bottom first (astra_lm_create_stacked)."""
         import torch
         L = lib()
-        self.cell = cell
+        self.layers = list(cell) if isinstance(cell, (list, tuple)) else [cell]
+        self.cell = self.layers[-1]
+        cell = self.cell
         self.V = vocab
         h = ctypes.c_void_p()
-        _check(L.astra_lm_create(ctypes.byref(h), cell.h, vocab))
+        if len(self.layers) == 1:
+            _check(L.astra_lm_create(ctypes.byref(h), cell.h, vocab))
+        else:
+            arr = (ctypes.c_void_p * len(self.layers))(*[c.h.value for c in self.layers])
+            _check(L.astra_lm_create_stacked(ctypes.byref(h), ctypes.cast(arr, ctypes.c_void_p), len(self.layers),
+                                             vocab))
         self.h = h
         n = ctypes.c_size_t()
         _check(L.astra_lm_param_count(h, ctypes.byref(n)))

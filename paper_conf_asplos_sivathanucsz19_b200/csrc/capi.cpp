@@ -220,6 +220,21 @@ astra_status astra_lm_create(astra_lm* out, astra_cell c, int vocab) {
   });
 }
 
+astra_status astra_lm_create_stacked(astra_lm* out, const astra_cell* cells, int n_layers, int vocab) {
+  return guard([&] {
+    NEED(out); NEED(cells);
+    ASTRA_CHECK_ARG(n_layers >= 1, "lm_create_stacked: n_layers must be >= 1");
+    std::vector<Cell*> v;
+    for (int l = 0; l < n_layers; ++l) {
+      NEED(cells[l]);
+      v.push_back(cells[l]->c.get());
+    }
+    auto h = std::make_unique<astra_lm_s>();
+    h->m.reset(new LM(v, vocab));
+    *out = h.release();
+  });
+}
+
 astra_status astra_lm_destroy(astra_lm m) {
   return guard([&] { delete m; });
 }
@@ -255,7 +270,7 @@ astra_status astra_lm_set_state(astra_lm m, const float* h, const float* c) {
 astra_status astra_lm_train_step(astra_lm m, const int32_t* tokens, float lr, float* loss_dev) {
   return guard([&] {
     NEED(m);
-    m->m->cell->set_active_T(m->m->cell->Tmax);
+    m->m->set_active_T(m->m->cell->Tmax);
     m->m->step(tokens, lr, loss_dev, true);
   });
 }
@@ -292,7 +307,7 @@ astra_status astra_lm_set_graph(astra_lm m, int on) {
 astra_status astra_lm_fwd_bwd(astra_lm m, const int32_t* tokens, float* loss_dev) {
   return guard([&] {
     NEED(m);
-    m->m->cell->set_active_T(m->m->cell->Tmax);
+    m->m->set_active_T(m->m->cell->Tmax);
     m->m->step(tokens, 0.f, loss_dev, false);
   });
 }

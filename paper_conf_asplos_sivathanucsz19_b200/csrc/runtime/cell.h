@@ -201,12 +201,17 @@ struct Carve {
 class LM {
  public:
   LM(Cell* c, int vocab);
-  Cell* cell;
+  LM(std::vector<Cell*> layers, int vocab);   // stacked layers, bottom first
+  std::vector<Cell*> layers;
+  Cell* cell;                                 // the top layer (the head reads its output)
+  std::vector<size_t> layer_poff, off_lsaved, off_lscratch, off_lh, off_lc;
+  size_t off_dxl[2] = {0, 0};
+  void set_active_T(int t);
   int V, Vp, Yw;
   size_t n_cell, n_params;
   std::vector<ParamInfo> params;
-  size_t off_logits, off_dlog, off_dlog32, off_rowloss, off_dY, off_Wo, off_colsum, off_sort, off_h, off_c,
-      off_cellsaved, off_cellscratch, off_loss, off_embpart, off_dx, off_wopart, ws_bytes;
+  size_t off_logits, off_dlog, off_dlog32, off_rowloss, off_dY, off_Wo, off_colsum, off_sort, off_loss, off_embpart,
+      off_dx, off_wopart, ws_bytes;
   size_t sort_bytes;
   int wo_ksplit = 1;   // fixed split of the head weight-gradient GEMM over K = T·B (reading R28)
   float* P = nullptr;

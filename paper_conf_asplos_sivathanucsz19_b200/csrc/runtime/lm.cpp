@@ -9,27 +9,63 @@
 
 namespace astra {
 
-LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
+LM::LM(Cell* c, int vocab) : LM(std::vector<Cell*>{c}, vocab) {}
+
+// A stack of layers (the paper's PTB stacked LSTM, Table 5):
+// layer l+1 reads layer l's output operand as its input, the embedding feeds layer 0 and the
+// head reads the top layer.  Parameters: each layer's block (names prefixed "L<l>." when there is
+// more than one layer), then E, W_o, b_o.
+LM::LM(std::vector<Cell*> cs, int vocab) : layers(cs), cell(cs.empty() ? nullptr : cs.back()), V(vocab) {
   ASTRA_CHECK_ARG(vocab > 1, "lm: vocab must be > 1");
-  if (!c->lm_capable()) throw Error(ASTRA_E_UNSUPPORTED, "lm: this cell type has no LM wrapper (reading R10)");
+  ASTRA_CHECK_ARG(!layers.empty(), "lm: at least one layer");
+  for (size_t l = 0; l < layers.size(); ++l) {
+    Cell* c = layers[l];
+    ASTRA_CHECK_ARG(c != nullptr, "lm: null layer");
+    if (!c->lm_capable()) throw Error(ASTRA_E_UNSUPPORTED, "lm: this cell type has no LM wrapper (reading R10)");
+    for (size_t k = 0; k < l; ++k) ASTRA_CHECK_ARG(layers[k] != c, "lm: a cell can appear only once in a stack");
+    if (l > 0) {
+      const Cell* b = layers[l - 1];
+      ASTRA_CHECK_ARG(c->B == b->B && c->Tmax == b->Tmax && c->ot == b->ot,
+                      "lm: stacked layers need the same batch, seq and dtype");
+      ASTRA_CHECK_ARG(b->y_segments().size() == 1 && c->I == b->y_segments()[0].n && c->Ip == b->y_width(),
+                      "lm: layer l+1's input size must be layer l's output size (single-segment outputs only)");
+    }
+  }
+  Cell* c0 = layers[0];
   Vp = (int)round_up(V, 8);
-  Yw = c->y_width();
-  c->lm_V = V;
-  params = c->params;
-  n_cell = c->n_params;
-  n_params = n_cell;
+  Yw = cell->y_width();
+  cell->lm_V = V;
+  n_params = 0;
+  const bool multi = layers.size() > 1;
+  for (size_t l = 0; l < layers.size(); ++l) {
+    layer_poff.push_back(n_params);
+    for (const ParamInfo& q : layers[l]->params) {
+      ParamInfo r = q;
+      if (multi) r.name = "L" + std::to_string(l) + "." + q.name;
+      r.offset += n_params;
+      params.push_back(r);
+    }
+    n_params += (layers[l]->n_params + 63) / 64 * 64;
+  }
+  n_cell = n_params;
   auto add = [&](const char* n, int r, int cc) {
     params.push_back({n, n_params, r, cc});
     n_params = (n_params + (size_t)r * cc + 63) / 64 * 64;
   };
-  add("E", V, c->I);
-  add("W_o", c->Hout, V);
+  add("E", V, c0->I);
+  add("W_o", cell->Hout, V);
   add("b_o", 1, V);
-  const long TB = (long)c->T * c->B;
-  const size_t e = c->esz();
+  const long TB = (long)cell->T * cell->B;
+  const size_t e = cell->esz();
   Carve w;
-  off_cellsaved = w.take(c->saved_bytes);
-  off_cellscratch = w.take(c->scratch_bytes);
+  int max_ip = 0;
+  for (Cell* c : layers) {
+    off_lsaved.push_back(w.take(c->saved_bytes));
+    off_lscratch.push_back(w.take(c->scratch_bytes));
+    off_lh.push_back(w.take((size_t)c->B * c->H * 4));
+    off_lc.push_back(w.take((size_t)c->B * (c->c_width() > 0 ? c->c_width() : 1) * 4));
+    max_ip = std::max(max_ip, c->Ip);
+  }
   off_logits = w.take((size_t)TB * V * 4);
   off_dlog = w.take((size_t)TB * Vp * e);
   off_dlog32 = w.take((size_t)TB * V * 4);
@@ -39,21 +75,24 @@ LM::LM(Cell* c, int vocab) : cell(c), V(vocab) {
   off_colsum = w.take(colsum_scratch_floats(TB, V) * 4);
   sort_bytes = embed_bwd_scratch_bytes(TB, V);
   off_sort = w.take(sort_bytes);
-  off_embpart = w.take(embed_bwd_partial_floats(TB, V, c->I) * 4);
-  off_h = w.take((size_t)c->B * c->H * 4);
-  off_c = w.take((size_t)c->B * (c->c_width() > 0 ? c->c_width() : 1) * 4);
+  off_embpart = w.take(embed_bwd_partial_floats(TB, V, c0->I) * 4);
   off_loss = w.take(256);
-  off_dx = w.take((size_t)TB * c->Ip * 4);
+  off_dx = w.take((size_t)TB * c0->Ip * 4);
+  // inter-layer input gradients (fp32, ping-pong: layer l's dx is layer l-1's dy)
+  if (multi) {
+    off_dxl[0] = w.take((size_t)TB * max_ip * 4);
+    off_dxl[1] = w.take((size_t)TB * max_ip * 4);
+  }
   // R28: dW_o = Yᵀ·dlogits has few output tiles (Hout x V) and a long K = T·B; a fixed split of K
   // into wo_ksplit chunks (partials summed in chunk order) lets it use the whole GPU.  The split
   // depends only on the shapes, so every variant (and the fp32 path) computes the same sums.
   {
     int maxn = 0;
-    for (const KSeg& sg : c->y_segments()) maxn = std::max(maxn, sg.n);
+    for (const KSeg& sg : cell->y_segments()) maxn = std::max(maxn, sg.n);
     wo_ksplit = wo_split(TB);   // non-decreasing in T·B: the largest bucket sizes the partials
     off_wopart = w.take((size_t)wo_ksplit * maxn * V * 4);
   }
-  off_tokpad = w.take((size_t)(c->Tmax + 1) * c->B * 4);
+  off_tokpad = w.take((size_t)(cell->Tmax + 1) * cell->B * 4);
   off_nv = w.take(4);
   ws_bytes = w.o;
 }
@@ -80,7 +119,7 @@ void LM::step_var(const int32_t* tokens, int len, float lr, float* loss_dev, boo
   Cell& c = *cell;
   ASTRA_CHECK_ARG(len >= 1 && len <= c.Tmax, "lm_train_step_len: len must be in [1, seq]");
   const int Tb = bucket_for(len);
-  c.set_active_T(Tb);
+  set_active_T(Tb);
   cudaStream_t st = c.main_st;
   int32_t* tp = (int32_t*)(ws + off_tokpad);
   CUDA_TRY(cudaMemcpyAsync(tp, tokens, (size_t)(len + 1) * c.B * 4, cudaMemcpyDeviceToDevice, st));
@@ -106,21 +145,39 @@ size_t LM::find(const std::string& n) const {
 void LM::bind(float* pp, float* gg, void* wsp) {
   ASTRA_CHECK_ARG(pp && gg && wsp, "lm_bind: null pointer");
   P = pp; G = gg; ws = (char*)wsp;
-  cell->lm_mode = true;
-  cell->bind(pp, gg, ws + off_cellsaved, ws + off_cellscratch);
+  for (size_t l = 0; l < layers.size(); ++l) {
+    layers[l]->lm_mode = true;
+    layers[l]->bind(pp + layer_poff[l], gg + layer_poff[l], ws + off_lsaved[l], ws + off_lscratch[l]);
+  }
   set_state(nullptr, nullptr);
   bound = true;
 }
 
+// h, c: the layers' states concatenated in layer order ([B][H_l] and [B][c_width_l] each).
 void LM::set_state(const float* h, const float* c) {
-  cudaStream_t st = cell->main_st;
-  const size_t nh = (size_t)cell->B * cell->H * 4, nc = (size_t)cell->B * cell->c_width() * 4;
-  if (h) CUDA_TRY(cudaMemcpyAsync(ws + off_h, h, nh, cudaMemcpyDeviceToDevice, st));
-  else CUDA_TRY(cudaMemsetAsync(ws + off_h, 0, nh, st));
-  if (nc) {
-    if (c) CUDA_TRY(cudaMemcpyAsync(ws + off_c, c, nc, cudaMemcpyDeviceToDevice, st));
-    else CUDA_TRY(cudaMemsetAsync(ws + off_c, 0, nc, st));
+  cudaStream_t st = layers[0]->main_st;
+  for (size_t l = 0; l < layers.size(); ++l) {
+    const Cell* L = layers[l];
+    const size_t nh = (size_t)L->B * L->H * 4, nc = (size_t)L->B * L->c_width() * 4;
+    if (h) {
+      CUDA_TRY(cudaMemcpyAsync(ws + off_lh[l], h, nh, cudaMemcpyDeviceToDevice, st));
+      h += nh / 4;
+    } else {
+      CUDA_TRY(cudaMemsetAsync(ws + off_lh[l], 0, nh, st));
+    }
+    if (nc) {
+      if (c) {
+        CUDA_TRY(cudaMemcpyAsync(ws + off_lc[l], c, nc, cudaMemcpyDeviceToDevice, st));
+        c += nc / 4;
+      } else {
+        CUDA_TRY(cudaMemsetAsync(ws + off_lc[l], 0, nc, st));
+      }
+    }
   }
+}
+
+void LM::set_active_T(int t) {
+  for (Cell* c : layers) c->set_active_T(t);
 }
 
 static bool graphs_enabled() {
@@ -156,13 +213,17 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
     const char* e = std::getenv("ASTRA_GRAPH_NCCL");
     return e && e[0] == '1';
   }();
-  const bool exploring = c.tune_mode == ASTRA_TUNE_ON && !(c.wirer && c.wirer->converged());
+  bool exploring = false;
+  std::string vs;
+  for (Cell* L : layers) {
+    exploring |= L->tune_mode == ASTRA_TUNE_ON && !(L->wirer && L->wirer->converged());
+    vs += L->var.str() + ";";
+  }
   if (!use_graphs || !graphs_enabled() || exploring || c.ot != OT::BF16 ||
       (c.world > 1 && !graph_nccl)) {
     enqueue_step(tokens, lr, loss_dev, do_sgd);
     return;
   }
-  const std::string vs = c.var.str();
   for (auto& g : graphs)
     if (g.tokens == tokens && g.lr == lr && g.loss == loss_dev && g.sgd == do_sgd && g.variant == vs &&
         g.T == c.T && g.len == (step_len > 0)) {
@@ -178,7 +239,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   CUDA_TRY(cudaStreamWaitEvent(cap_st, e0, 0));
   CUDA_TRY(cudaEventDestroy(e0));
   cudaStream_t user = c.main_st;
-  c.main_st = cap_st;
+  for (Cell* L : layers) L->main_st = cap_st;
   const uint64_t l0 = g_launches.load();
   cudaGraph_t graph = nullptr;
   CUDA_TRY(cudaStreamBeginCapture(cap_st, cudaStreamCaptureModeThreadLocal));
@@ -187,10 +248,10 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   } catch (...) {
     cudaStreamEndCapture(cap_st, &graph);
     if (graph) cudaGraphDestroy(graph);
-    c.main_st = user;
+    for (Cell* L : layers) L->main_st = user;
     throw;
   }
-  c.main_st = user;
+  for (Cell* L : layers) L->main_st = user;
   CUDA_TRY(cudaStreamEndCapture(cap_st, &graph));
   GraphEntry ge;
   ge.tokens = tokens; ge.lr = lr; ge.loss = loss_dev; ge.sgd = do_sgd; ge.variant = vs;
@@ -213,8 +274,8 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   cudaStream_t st = c.main_st;
   const long TB = (long)c.T * c.B;
   const size_t e = c.esz();
-  float* hs = (float*)(ws + off_h);
-  float* cs = c.c_width() > 0 ? (float*)(ws + off_c) : nullptr;
+  Cell& c0 = *layers[0];
+  const int nl = (int)layers.size();
   float* logits = (float*)(ws + off_logits);
   void* dlog = ws + off_dlog;
   float* dlog32 = (float*)(ws + off_dlog32);
@@ -250,8 +311,8 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   std::vector<int> t_end(nch);   // last forward step of each time chunk
   for (int k = 0; k < nch; ++k) t_end[k] = (int)((long)(k + 1) * c.T / nch) - 1;
 
-  // a0: embedding gather into the cell's operand buffer
-  embed_gather(c.ot, tokens, TB, P + find("E"), c.I, c.x_operand(), c.Ip, st);
+  // a0: embedding gather into layer 0's operand buffer
+  embed_gather(c.ot, tokens, TB, P + find("E"), c0.I, c0.x_operand(), c0.Ip, st);
   // head weight mirror (independent of the forward)
   c.mark(R_HEAD, 0, hst);
   CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, hst));
@@ -290,8 +351,17 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
         if (t == t_end[k]) head_chunk(k);
     };
   try {
-    if (step_len > 0) c.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
-    else c.forward(nullptr, hs, cs, nullptr, hs, cs);
+    for (int l = 0; l < nl; ++l) {
+      Cell& L = *layers[l];
+      if (l > 0) {   // layer l's input operand = layer l-1's output operand (bf16 / fp32, [T·B][H])
+        const Mat2 yp = layers[l - 1]->y_operand();
+        copy_pad(L.ot, yp.ptr, L.ot, TB, L.I, yp.ld, L.x_operand(), L.Ip, st);
+      }
+      float* hs = (float*)(ws + off_lh[l]);
+      float* cs = L.c_width() > 0 ? (float*)(ws + off_lc[l]) : nullptr;
+      if (step_len > 0) L.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
+      else L.forward(nullptr, hs, cs, nullptr, hs, cs);
+    }
   } catch (...) {
     c.fwd_hook = nullptr;
     throw;
@@ -330,16 +400,21 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   c.grad_bucket(G + find("W_o"), n_params - find("W_o"), hst);
   if (ov) CUDA_TRY(cudaEventRecord(ev_hdone, hst));
 
-  // cell backward (SE3 + SE4) and the embedding backward
-  c.lm_dy = dY;
-  c.backward(nullptr, nullptr, nullptr, dX, nullptr, nullptr);
-  embed_bwd(tokens, TB, V, dX, c.Ip, c.I, G + find("E"), ws + off_sort, sort_bytes, (float*)(ws + off_embpart), st);
+  // layers' backward (SE3 + SE4), top down: layer l's input gradient is layer l-1's dy; then the
+  // embedding backward
+  for (int l = nl - 1; l >= 0; --l) {
+    Cell& L = *layers[l];
+    L.lm_dy = l == nl - 1 ? dY : (float*)(ws + off_dxl[(l + 1) % 2]);
+    float* dx_l = l == 0 ? dX : (float*)(ws + off_dxl[l % 2]);
+    L.backward(nullptr, nullptr, nullptr, dx_l, nullptr, nullptr);
+  }
+  embed_bwd(tokens, TB, V, dX, c0.Ip, c0.I, G + find("E"), ws + off_sort, sort_bytes, (float*)(ws + off_embpart), st);
   // a7: last bucket (embedding), join, then a8: SGD
-  c.grad_bucket(G + find("E"), (size_t)V * c.I, st);
+  c0.grad_bucket(G + find("E"), (size_t)V * c0.I, st);
   if (ov) CUDA_TRY(cudaStreamWaitEvent(st, ev_hdone, 0));   // head gradients (and their bucket) done
-  c.grad_join(st);
+  for (Cell* L : layers) L->grad_join(st);
   if (do_sgd) sgd(P, G, n_params, lr, st);
-  c.mark(R_STEP, 1, st);
+  for (Cell* L : layers) L->mark(R_STEP, 1, st);
 }
 
 }  // namespace astra
