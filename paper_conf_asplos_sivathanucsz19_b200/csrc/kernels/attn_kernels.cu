@@ -8,6 +8,7 @@
 // independent of launch timing (R5).  fp32 throughout (ALU/MUFU-bound).
 #include "cell_math.cuh"
 #include "kernels.h"
+#include "pdl.cuh"
 
 namespace astra {
 
@@ -37,6 +38,8 @@ __global__ void __launch_bounds__(ATT_THREADS)
     attn_fwd_kernel(int B, int Ts, int H, int Hp, int A, int Ap, const float* __restrict__ q,
                     const float* __restrict__ keys, const float* __restrict__ v, const float* __restrict__ enc,
                     float* __restrict__ pr, T* __restrict__ ctx_op, long ldc, TY* __restrict__ y_ctx, long ldy) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   extern __shared__ float sh[];
   float* e = sh;            // [Ts]
   float* red = sh + Ts;     // [33]
@@ -75,10 +78,10 @@ void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q
               const float* enc, float* pr, void* ctx_op, long ldc, void* y_ctx, long ldy, cudaStream_t st) {
   const size_t sm = (Ts + 40) * sizeof(float);
   if (ot == OT::BF16)
-    attn_fwd_kernel<__nv_bfloat16, __nv_bfloat16><<<B, ATT_THREADS, sm, st>>>(
+    launch_pdl(attn_fwd_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(B), dim3(ATT_THREADS), sm, st, 1, 
         B, Ts, H, Hp, A, Ap, q, keys, v, enc, pr, (__nv_bfloat16*)ctx_op, ldc, (__nv_bfloat16*)y_ctx, ldy);
   else
-    attn_fwd_kernel<float, float><<<B, ATT_THREADS, sm, st>>>(B, Ts, H, Hp, A, Ap, q, keys, v, enc, pr,
+    launch_pdl(attn_fwd_kernel<float, float>, dim3(B), dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, A, Ap, q, keys, v, enc, pr,
                                                               (float*)ctx_op, ldc, (float*)y_ctx, ldy);
   LAUNCH_CHECK();
 }
@@ -93,6 +96,8 @@ __global__ void __launch_bounds__(ATT_THREADS)
                     const float* __restrict__ q, const float* __restrict__ keys, const float* __restrict__ v,
                     const float* __restrict__ enc, T* __restrict__ dq_op, float* __restrict__ denc,
                     float* __restrict__ dk, float* __restrict__ dvb, int first) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   extern __shared__ float sh[];
   float* dctx = sh;              // [Hp]
   float* de = sh + Hp;           // [Ts]
@@ -158,15 +163,15 @@ void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy
   const size_t sm = (Hp + Ts + 40) * sizeof(float);
   if (ot == OT::BF16) {
     if (dy_f32 || !dy_ctx)
-      attn_bwd_kernel<__nv_bfloat16, float><<<B, ATT_THREADS, sm, st>>>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy,
+      launch_pdl(attn_bwd_kernel<__nv_bfloat16, float>, dim3(B), dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy,
                                                                         dctx_rec, ldr, pr, q, keys, v, enc,
                                                                         (__nv_bfloat16*)dq_op, denc, dk, dvb, first);
     else
-      attn_bwd_kernel<__nv_bfloat16, __nv_bfloat16><<<B, ATT_THREADS, sm, st>>>(
+      launch_pdl(attn_bwd_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(B), dim3(ATT_THREADS), sm, st, 1, 
           B, Ts, H, Hp, A, Ap, (const __nv_bfloat16*)dy_ctx, ldy, dctx_rec, ldr, pr, q, keys, v, enc,
           (__nv_bfloat16*)dq_op, denc, dk, dvb, first);
   } else {
-    attn_bwd_kernel<float, float><<<B, ATT_THREADS, sm, st>>>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy,
+    launch_pdl(attn_bwd_kernel<float, float>, dim3(B), dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy,
                                                               dctx_rec, ldr, pr, q, keys, v, enc, (float*)dq_op, denc,
                                                               dk, dvb, first);
   }

@@ -4,6 +4,7 @@
 // follow the fixed-order scheme of the LSTM backward kernel (R5).
 #include "cell_math.cuh"
 #include "kernels.h"
+#include "pdl.cuh"
 
 namespace astra {
 
@@ -58,6 +59,8 @@ __global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
                                    const float* __restrict__ Z, const float* __restrict__ bh, float* __restrict__ Hf,
                                    T* __restrict__ HSh, long ldhs, TY* __restrict__ y, long ldy,
                                    float* __restrict__ hT) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int b = blockIdx.y;
   if (j >= Hp) return;
@@ -75,10 +78,10 @@ void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const fl
                  void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st) {
   dim3 grid(cdiv(Hp, 128), B);
   if (ot == OT::BF16)
-    scrn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 128, 0, st>>>(
+    launch_pdl(scrn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(128), 0, st, 1, 
         B, H, Hp, Q, ldq, Z, bh, Hf, (__nv_bfloat16*)HSh, ldhs, (__nv_bfloat16*)y, ldy, hT);
   else
-    scrn_fwd_pw_kernel<float, float><<<grid, 128, 0, st>>>(B, H, Hp, Q, ldq, Z, bh, Hf, (float*)HSh, ldhs, (float*)y,
+    launch_pdl(scrn_fwd_pw_kernel<float, float>, dim3(grid), dim3(128), 0, st, 1, B, H, Hp, Q, ldq, Z, bh, Hf, (float*)HSh, ldhs, (float*)y,
                                                            ldy, hT);
   LAUNCH_CHECK();
 }
@@ -89,6 +92,8 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
     scrn_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh,
                        long ld_dh, const float* __restrict__ Hf, T* __restrict__ DZ, long ldz,
                        float* __restrict__ part, int first) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   __shared__ float red[PW_RY][PW_UX];
   const int ux = threadIdx.x, ty = threadIdx.y;
   const int j = blockIdx.x * PW_UX + ux;
@@ -124,13 +129,13 @@ void scrn_bwd_pw(OT ot, int B, int H, int Hp, const void* dy, long ldy, bool dy_
   dim3 grid(cdiv(Hp, PW_UX), pw_row_chunks(B)), block(PW_UX, PW_RY);
   if (ot == OT::BF16) {
     if (dy_f32)
-      scrn_bwd_pw_kernel<__nv_bfloat16, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh, ld_dh,
+      launch_pdl(scrn_bwd_pw_kernel<__nv_bfloat16, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh, ld_dh,
                                                                        Hf, (__nv_bfloat16*)DZ, ldz, part, first);
     else
-      scrn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, block, 0, st>>>(
+      launch_pdl(scrn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(block), 0, st, 1, 
           B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh, ld_dh, Hf, (__nv_bfloat16*)DZ, ldz, part, first);
   } else {
-    scrn_bwd_pw_kernel<float, float><<<grid, block, 0, st>>>(B, H, Hp, (const float*)dy, ldy, dh, ld_dh, Hf,
+    launch_pdl(scrn_bwd_pw_kernel<float, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh, ld_dh, Hf,
                                                              (float*)DZ, ldz, part, first);
   }
   LAUNCH_CHECK();
@@ -187,6 +192,8 @@ __global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, c
                                   const float* __restrict__ bl, const float* __restrict__ s_prev,
                                   float* __restrict__ s_next, T* __restrict__ s_next_op, TY* __restrict__ y, long ldy,
                                   float* __restrict__ sT) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int b = blockIdx.y;
   if (j >= Hp) return;
@@ -215,10 +222,10 @@ void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* WX, const fl
                 float* s_next, void* s_next_op, void* y, long ldy, float* sT, cudaStream_t st) {
   dim3 grid(cdiv(Hp, 128), B);
   if (ot == OT::BF16)
-    rhn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, 128, 0, st>>>(
+    launch_pdl(rhn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(128), 0, st, 1, 
         B, H, Hp, Z, WX, bl, s_prev, s_next, (__nv_bfloat16*)s_next_op, (__nv_bfloat16*)y, ldy, sT);
   else
-    rhn_fwd_pw_kernel<float, float><<<grid, 128, 0, st>>>(B, H, Hp, Z, WX, bl, s_prev, s_next, (float*)s_next_op,
+    launch_pdl(rhn_fwd_pw_kernel<float, float>, dim3(grid), dim3(128), 0, st, 1, B, H, Hp, Z, WX, bl, s_prev, s_next, (float*)s_next_op,
                                                           (float*)y, ldy, sT);
   LAUNCH_CHECK();
 }
@@ -230,6 +237,8 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
     rhn_bwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ ds_in, const TDY* __restrict__ dy, long ldy,
                       const float* __restrict__ Apre, const float* __restrict__ s_prev, T* __restrict__ DA,
                       float* __restrict__ ds_out, float* __restrict__ part, int first) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   __shared__ float red[PW_RY][2][PW_UX];
   const int ux = threadIdx.x, ty = threadIdx.y;
   const int j = blockIdx.x * PW_UX + ux;
@@ -276,13 +285,13 @@ void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const void* dy,
   dim3 grid(cdiv(Hp, PW_UX), pw_row_chunks(B)), block(PW_UX, PW_RY);
   if (ot == OT::BF16) {
     if (dy_f32 || !dy)
-      rhn_bwd_pw_kernel<__nv_bfloat16, float><<<grid, block, 0, st>>>(B, H, Hp, ds_in, (const float*)dy, ldy, Apre,
+      launch_pdl(rhn_bwd_pw_kernel<__nv_bfloat16, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, ds_in, (const float*)dy, ldy, Apre,
                                                                       s_prev, (__nv_bfloat16*)DA, ds_out, part, first);
     else
-      rhn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16><<<grid, block, 0, st>>>(
+      launch_pdl(rhn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(block), 0, st, 1, 
           B, H, Hp, ds_in, (const __nv_bfloat16*)dy, ldy, Apre, s_prev, (__nv_bfloat16*)DA, ds_out, part, first);
   } else {
-    rhn_bwd_pw_kernel<float, float><<<grid, block, 0, st>>>(B, H, Hp, ds_in, (const float*)dy, ldy, Apre, s_prev,
+    launch_pdl(rhn_bwd_pw_kernel<float, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, ds_in, (const float*)dy, ldy, Apre, s_prev,
                                                             (float*)DA, ds_out, part, first);
   }
   LAUNCH_CHECK();
