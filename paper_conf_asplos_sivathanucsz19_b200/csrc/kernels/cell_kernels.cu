@@ -745,6 +745,18 @@ __global__ void sum_split_partials1_kernel(const float* __restrict__ part, int k
   for (int k = 1; k < ks; ++k) v = __fadd_rn(v, part[(long)k * n + i]);
   out[i] = v;
 }
+__global__ void add_split_partials_kernel(float* __restrict__ out, const float* __restrict__ part, int ks, long n) {
+  const long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  float v = part[i];
+  for (int k = 1; k < ks; ++k) v = __fadd_rn(v, part[(long)k * n + i]);
+  out[i] = __fadd_rn(out[i], v);
+}
+void add_split_partials(float* out, const float* part, int ks, long n, cudaStream_t st) {
+  add_split_partials_kernel<<<(unsigned)cdiv(n, 256), 256, 0, st>>>(out, part, ks, n);
+  LAUNCH_CHECK();
+}
+
 void sum_split_partials(const float* part, int ks, long n, float* out, cudaStream_t st) {
   if ((n & 3) == 0 && (((uintptr_t)part | (uintptr_t)out) & 15) == 0)
     sum_split_partials_kernel<<<(unsigned)cdiv(n / 4, 256), 256, 0, st>>>((const float4*)part, ks, n / 4, (float4*)out);

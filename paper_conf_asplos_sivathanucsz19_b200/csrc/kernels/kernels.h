@@ -55,11 +55,15 @@ void scrn_bwd_pw(OT ot, int B, int H, int Hp, const void* dy, long ldy, bool dy_
                  const float* Hf, void* DZ, long ldz, float* part, bool first, cudaStream_t st);
 void scrn_scan_bwd(OT ot, int B, int S, int Sp, int T, float alpha, const void* dys, long ldy, bool dy_f32,
                    const float* DSP, long ldsp, const float* dsT, void* DSa, long ldsa, float* ds0, cudaStream_t st);
-void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* WX, const float* bl, const float* s_prev,
-                float* s_next, void* s_next_op, void* y, long ldy, float* sT, cudaStream_t st);
-void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const void* dy, long ldy, bool dy_f32,
-                const float* Apre, const float* s_prev, void* DA, float* ds_out, float* part, bool first,
-                cudaStream_t st);
+// a = (Σ_k Zpart[k] in k order, or Z when Zpart is null) + b (+ WX at ℓ = 1), written to Z (saved pre-activations)
+void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* Zpart, int nsplit, long split_stride,
+                const float* WX, const float* bl, const float* s_prev, float* s_next, void* s_next_op, void* y,
+                long ldy, float* sT, cudaStream_t st);
+// ds = ds_in (the carry ds·(1−τ) of the micro-step above) + Σ_k ds_part[k] in k order (the BPTT GEMM's
+// split-K partials, reading R33; null at the first micro-step) (+ dy at the top micro-layer).
+void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const float* ds_part, int nsplit, long split_stride,
+                const void* dy, long ldy, bool dy_f32, const float* Apre, const float* s_prev, void* DA,
+                float* ds_out, float* part, bool first, cudaStream_t st);
 void reduce_blocked_partials(const float* part, int nchunk, int nq, int H, int Hp, float* out, cudaStream_t st);
 void mirror_blocked_T(OT ot, const float* src, int K, int G, int H, int Hp, void* dst, long ldd, cudaStream_t st);
 
@@ -77,6 +81,8 @@ void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targ
                 float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp = nullptr,
                 long row0 = 0);
 // out[i] = Σ_{k < ks} part[k·n + i] in k order (split-K partials, R25/R28).
+// out[i] += Σ_k part[k·n + i] (partials summed in k order first)
+void add_split_partials(float* out, const float* part, int ks, long n, cudaStream_t st);
 void sum_split_partials(const float* part, int ks, long n, float* out, cudaStream_t st);
 void sum_rows_to_scalar(const float* v, long n, float scale, float* out, cudaStream_t st, const int* nvp = nullptr);
 // *p = v (a one-thread kernel: device-side scalars that captured CUDA graphs read)

@@ -188,7 +188,8 @@ void scrn_scan_bwd(OT ot, int B, int S, int Sp, int T, float alpha, const void* 
 // Micro-step ℓ of time t (coupled carry): a = z + b_ℓ (+ wx_t at ℓ = 0), stored back as the saved
 // pre-activation; h = tanh a_H, τ = σ(a_T); s' = h·τ + s·(1 − τ).  Internal columns: g·Hp + j.
 template <typename T, typename TY>
-__global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, const float* __restrict__ WX,
+__global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, const float* __restrict__ Zpart,
+                                  int nsplit, long split_stride, const float* __restrict__ WX,
                                   const float* __restrict__ bl, const float* __restrict__ s_prev,
                                   float* __restrict__ s_next, T* __restrict__ s_next_op, TY* __restrict__ y, long ldy,
                                   float* __restrict__ sT) {
@@ -200,8 +201,20 @@ __global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, c
   const long rz = (long)b * 2 * Hp;
   float s_new = 0.f;
   if (j < H) {
-    float aH = __fadd_rn(Z[rz + j], bl[j]);
-    float aT = __fadd_rn(Z[rz + Hp + j], bl[H + j]);
+    float zH, zT;
+    if (Zpart) {   // reading R33: the recurrent GEMM's split-K partials summed in chunk order
+      zH = Zpart[rz + j];
+      zT = Zpart[rz + Hp + j];
+      for (int k = 1; k < nsplit; ++k) {
+        zH = __fadd_rn(zH, Zpart[k * split_stride + rz + j]);
+        zT = __fadd_rn(zT, Zpart[k * split_stride + rz + Hp + j]);
+      }
+    } else {
+      zH = Z[rz + j];
+      zT = Z[rz + Hp + j];
+    }
+    float aH = __fadd_rn(zH, bl[j]);
+    float aT = __fadd_rn(zT, bl[H + j]);
     if (WX) {
       aH = __fadd_rn(aH, WX[rz + j]);
       aT = __fadd_rn(aT, WX[rz + Hp + j]);
@@ -218,14 +231,15 @@ __global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, c
   s_next_op[(long)b * Hp + j] = from_f<T>(s_new);
 }
 
-void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* WX, const float* bl, const float* s_prev,
-                float* s_next, void* s_next_op, void* y, long ldy, float* sT, cudaStream_t st) {
+void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* Zpart, int nsplit, long split_stride,
+                const float* WX, const float* bl, const float* s_prev, float* s_next, void* s_next_op, void* y,
+                long ldy, float* sT, cudaStream_t st) {
   dim3 grid(cdiv(Hp, 128), B);
   if (ot == OT::BF16)
     launch_pdl(rhn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(128), 0, st, 1, 
-        B, H, Hp, Z, WX, bl, s_prev, s_next, (__nv_bfloat16*)s_next_op, (__nv_bfloat16*)y, ldy, sT);
+        B, H, Hp, Z, Zpart, nsplit, split_stride, WX, bl, s_prev, s_next, (__nv_bfloat16*)s_next_op, (__nv_bfloat16*)y, ldy, sT);
   else
-    launch_pdl(rhn_fwd_pw_kernel<float, float>, dim3(grid), dim3(128), 0, st, 1, B, H, Hp, Z, WX, bl, s_prev, s_next, (float*)s_next_op,
+    launch_pdl(rhn_fwd_pw_kernel<float, float>, dim3(grid), dim3(128), 0, st, 1, B, H, Hp, Z, Zpart, nsplit, split_stride, WX, bl, s_prev, s_next, (float*)s_next_op,
                                                           (float*)y, ldy, sT);
   LAUNCH_CHECK();
 }
@@ -234,7 +248,8 @@ void rhn_fwd_pw(OT ot, int B, int H, int Hp, float* Z, const float* WX, const fl
 // da_H = dh·(1 − h²); da_T = dτ·τ·(1 − τ); ds_out = ds·(1 − τ) (the BPTT GEMM then adds da·R_ℓᵀ).
 template <typename T, typename TDY>
 __global__ void __launch_bounds__(PW_UX * PW_RY)
-    rhn_bwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ ds_in, const TDY* __restrict__ dy, long ldy,
+    rhn_bwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ ds_in, const float* __restrict__ ds_part,
+                      int nsplit, long split_stride, const TDY* __restrict__ dy, long ldy,
                       const float* __restrict__ Apre, const float* __restrict__ s_prev, T* __restrict__ DA,
                       float* __restrict__ ds_out, float* __restrict__ part, int first) {
   pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
@@ -251,6 +266,12 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
       float daH = 0.f, daT = 0.f, dso = 0.f;
       if (j < H) {
         float ds = ds_in[(long)b * Hp + j];
+        if (ds_part) {   // reading R33: carry + the BPTT GEMM's split-K partials summed in chunk order
+          const float* q = ds_part + (long)b * Hp + j;
+          float r = q[0];
+          for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, q[k * split_stride]);
+          ds = __fadd_rn(ds, r);
+        }
         if (dy) ds = __fadd_rn(to_f<TDY>(dy[(long)b * ldy + j]), ds);
         const float h = tanh_<FastMath<T>::value>(Apre[rz + j]), tau = sigm<FastMath<T>::value>(Apre[rz + Hp + j]);
         const float sp = s_prev[(long)b * Hp + j];
@@ -279,19 +300,20 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
   }
 }
 
-void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const void* dy, long ldy, bool dy_f32,
-                const float* Apre, const float* s_prev, void* DA, float* ds_out, float* part, bool first,
-                cudaStream_t st) {
+void rhn_bwd_pw(OT ot, int B, int H, int Hp, const float* ds_in, const float* ds_part, int nsplit, long split_stride,
+                const void* dy, long ldy, bool dy_f32, const float* Apre, const float* s_prev, void* DA,
+                float* ds_out, float* part, bool first, cudaStream_t st) {
   dim3 grid(cdiv(Hp, PW_UX), pw_row_chunks(B)), block(PW_UX, PW_RY);
   if (ot == OT::BF16) {
     if (dy_f32 || !dy)
-      launch_pdl(rhn_bwd_pw_kernel<__nv_bfloat16, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, ds_in, (const float*)dy, ldy, Apre,
+      launch_pdl(rhn_bwd_pw_kernel<__nv_bfloat16, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, ds_in, ds_part, nsplit, split_stride, (const float*)dy, ldy, Apre,
                                                                       s_prev, (__nv_bfloat16*)DA, ds_out, part, first);
     else
       launch_pdl(rhn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(block), 0, st, 1, 
-          B, H, Hp, ds_in, (const __nv_bfloat16*)dy, ldy, Apre, s_prev, (__nv_bfloat16*)DA, ds_out, part, first);
+          B, H, Hp, ds_in, ds_part, nsplit, split_stride, (const __nv_bfloat16*)dy, ldy, Apre, s_prev,
+          (__nv_bfloat16*)DA, ds_out, part, first);
   } else {
-    launch_pdl(rhn_bwd_pw_kernel<float, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, ds_in, (const float*)dy, ldy, Apre, s_prev,
+    launch_pdl(rhn_bwd_pw_kernel<float, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, ds_in, ds_part, nsplit, split_stride, (const float*)dy, ldy, Apre, s_prev,
                                                             (float*)DA, ds_out, part, first);
   }
   LAUNCH_CHECK();

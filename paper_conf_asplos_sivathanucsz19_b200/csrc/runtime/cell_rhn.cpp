@@ -8,6 +8,8 @@
 // (s·R_ℓ, N = 2H) + one pointwise kernel (a3); BPTT mirrors it with ds = ds(1−τ) + da·R_ℓᵀ
 // (pointwise writes ds(1−τ), the GEMM accumulates da·R_ℓᵀ onto it); dR_ℓ = S_ℓᵀ·DA_ℓ per micro-layer.
 // Internal gate layout: gate-blocked and padded, column g·Hp + j.
+#include <algorithm>
+
 #include "cell.h"
 
 namespace astra {
@@ -16,7 +18,23 @@ class RhnCell : public Cell {
  public:
   int L, G2, nchunk;
   size_t off_X, off_WX, off_Apre, off_Sf, off_Sop, off_MW, off_MR;
-  size_t off_DA, off_dS, off_part;
+  size_t off_DA, off_dS, off_dSpart, off_Zpart, off_part;
+
+  // Reading R33: the BPTT GEMM ds·R_ℓᵀ (K = 2·Hp, few output tiles at small batch) is split over K
+  // into s fixed chunks, each accumulated from zero; the next pointwise kernel adds the partials in
+  // chunk order to the carry ds·(1−τ).  Depends only on the shapes (every variant, both paths).
+  int fwd_ksplit() const {   // the same rule for the recurrent GEMM s·R_ℓ (K = Hp, N = 2·Hp)
+    const int tiles = cdiv(B, 128) * cdiv(2 * Hp, 64), nk = cdiv(Hp, 64);
+    int s = std::max(1, std::min(4, 64 / std::max(1, tiles)));
+    while (s > 1 && nk / s < 4) --s;
+    return s;
+  }
+  int bptt_ksplit() const {
+    const int tiles = cdiv(B, 128) * cdiv(Hp, 64), nk = cdiv(2 * Hp, 64);
+    int s = std::max(1, std::min(4, 64 / std::max(1, tiles)));
+    while (s > 1 && nk / s < 4) --s;
+    return s;
+  }
 
   explicit RhnCell(const astra_cell_desc& dd) : Cell(dd) {
     L = d.depth;
@@ -40,6 +58,8 @@ class RhnCell : public Cell {
     Carve c;
     off_DA = c.take((size_t)L * TB * G2 * e);
     off_dS = c.take((size_t)B * Hp * 4);
+    off_dSpart = c.take((size_t)bptt_ksplit() * B * Hp * 4);
+    off_Zpart = c.take((size_t)fwd_ksplit() * B * G2 * 4);
     off_part = c.take((size_t)L * nchunk * G2 * 4);
     scratch_bytes = c.o;
   }
@@ -102,14 +122,20 @@ class RhnCell : public Cell {
     rec.B = mat(MR, Hp, G2, Hp, L, (long)G2 * Hp);
     rec.M = B; rec.N = G2; rec.K = Hp;
     rec.b_keep = true;
+    rec.ksplit = fwd_ksplit();
+    float* Zpart = sc<float>(off_Zpart);
+    EpiStore ez = epi(Zpart, G2, B, G2);
+    ez.split_stride = (long)B * G2;
     for (int t = 0; t < T; ++t) {
       for (int l = 0; l < L; ++l) {
         float* Z = Apre(l, t);
-        run_gemm(1, rec, epi(Z, G2, B, G2), l * (T + 1) + t, l, var.g[G_REC], st);
+        if (rec.ksplit > 1) run_gemm(1, rec, ez, l * (T + 1) + t, l, var.g[G_REC], st);
+        else run_gemm(1, rec, epi(Z, G2, B, G2), l * (T + 1) + t, l, var.g[G_REC], st);
         const bool last = l == L - 1;
         float* sn = last ? Sf(0, t + 1) : Sf(l + 1, t);
         char* sno = last ? Sop(0, t + 1) : Sop(l + 1, t);
-        rhn_fwd_pw(ot, B, H, Hp, Z, l == 0 ? WX + (long)t * B * G2 : nullptr, p("b") + (size_t)l * 2 * H, Sf(l, t),
+        rhn_fwd_pw(ot, B, H, Hp, Z, rec.ksplit > 1 ? Zpart : nullptr, rec.ksplit, (long)B * G2,
+                   l == 0 ? WX + (long)t * B * G2 : nullptr, p("b") + (size_t)l * 2 * H, Sf(l, t),
                    sn, sno, (last && y) ? (char*)y + (size_t)t * B * H * e : nullptr, H,
                    (last && t == T - 1) ? sT : nullptr, st);
       }
@@ -140,16 +166,22 @@ class RhnCell : public Cell {
     bp.b_mn = true;
     bp.M = B; bp.N = Hp; bp.K = G2;
     bp.b_keep = true;
+    bp.ksplit = bptt_ksplit();
+    float* dSpart = sc<float>(off_dSpart);
+    EpiStore ep = epi(dSpart, Hp, B, Hp);
+    ep.split_stride = (long)B * Hp;
     for (int t = T - 1; t >= 0; --t) {
       for (int l = L - 1; l >= 0; --l) {
         const void* dyt = nullptr;
         if (l == L - 1)
           dyt = lm_mode ? (const void*)(lm_dy + (long)t * B * Hp) : (const char*)dy + (size_t)t * B * H * e;
-        rhn_bwd_pw(ot, B, H, Hp, dS, dyt, ldy, lm_mode, Apre(l, t), Sf(l, t), DA(l, t), dS,
-                   part + (size_t)l * nchunk * G2, t == T - 1, st);
-        run_gemm(2, bp, accum(epi(dS, Hp, B, Hp)), l * T + t, l, var.g[G_BPTT], st);
+        const bool top = t == T - 1 && l == L - 1;   // no GEMM before the first micro-step
+        rhn_bwd_pw(ot, B, H, Hp, dS, top ? nullptr : dSpart, bp.ksplit, (long)B * Hp, dyt, ldy, lm_mode, Apre(l, t),
+                   Sf(l, t), DA(l, t), dS, part + (size_t)l * nchunk * G2, t == T - 1, st);
+        run_gemm(2, bp, ep, l * T + t, l, var.g[G_BPTT], st);
       }
     }
+    add_split_partials(dS, dSpart, bp.ksplit, (long)B * Hp, st);   // ds of s^0_0
     if (ds0) copy_pad(OT::F32, dS, OT::F32, B, H, Hp, ds0, H, st);
     mark(R_BPTT, 1, st);
 
