@@ -49,10 +49,12 @@ void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int 
 int pw_row_chunks(int B);
 void scrn_scan_fwd(OT ot, int B, int S, int Sp, int T, float alpha, const float* XB, long ldxb, const float* s0,
                    float* Sf, void* HSs, long ldhs, void* y, long ldy, float* sT, cudaStream_t st);
-void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const float* Z, const float* bh, float* Hf,
-                 void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st);
+// Z / dh: nsplit fp32 partials at split_stride elements (the chain GEMM's split-K, reading R33), summed in order.
+void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const float* Z, int nsplit, long split_stride,
+                 const float* bh, float* Hf, void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st);
 void scrn_bwd_pw(OT ot, int B, int H, int Hp, const void* dy, long ldy, bool dy_f32, const float* dh, long ld_dh,
-                 const float* Hf, void* DZ, long ldz, float* part, bool first, cudaStream_t st);
+                 int nsplit, long split_stride, const float* Hf, void* DZ, long ldz, float* part, bool first,
+                 cudaStream_t st);
 void scrn_scan_bwd(OT ot, int B, int S, int Sp, int T, float alpha, const void* dys, long ldy, bool dy_f32,
                    const float* DSP, long ldsp, const float* dsT, void* DSa, long ldsa, float* ds0, cudaStream_t st);
 // a = (Σ_k Zpart[k] in k order, or Z when Zpart is null) + b (+ WX at ℓ = 1), written to Z (saved pre-activations)

@@ -56,7 +56,8 @@ void scrn_scan_fwd(OT ot, int B, int S, int Sp, int T, float alpha, const float*
 // h_t = σ((q_t + z_t) + b_h)   (q_t = x_t·A + s_t·P, the hoisted ladder; z_t = h_{t−1}·R)
 template <typename T, typename TY>
 __global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict__ Q, long ldq,
-                                   const float* __restrict__ Z, const float* __restrict__ bh, float* __restrict__ Hf,
+                                   const float* __restrict__ Z, int nsplit, long split_stride,
+                                   const float* __restrict__ bh, float* __restrict__ Hf,
                                    T* __restrict__ HSh, long ldhs, TY* __restrict__ y, long ldy,
                                    float* __restrict__ hT) {
   pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
@@ -65,7 +66,11 @@ __global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
   const int b = blockIdx.y;
   if (j >= Hp) return;
   float h = 0.f;
-  if (j < H) h = sigm<FastMath<T>::value>(__fadd_rn(__fadd_rn(Q[(long)b * ldq + j], Z[(long)b * Hp + j]), bh[j]));
+  if (j < H) {
+    float z = Z[(long)b * Hp + j];   // reading R33: split-K partials of h_{t-1}·R summed in chunk order
+    for (int k = 1; k < nsplit; ++k) z = __fadd_rn(z, Z[k * split_stride + (long)b * Hp + j]);
+    h = sigm<FastMath<T>::value>(__fadd_rn(__fadd_rn(Q[(long)b * ldq + j], z), bh[j]));
+  }
   Hf[(long)b * Hp + j] = h;
   HSh[(long)b * ldhs + j] = from_f<T>(h);
   if (j < H) {
@@ -74,14 +79,14 @@ __global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
   }
 }
 
-void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const float* Z, const float* bh, float* Hf,
-                 void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st) {
+void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const float* Z, int nsplit, long split_stride,
+                 const float* bh, float* Hf, void* HSh, long ldhs, void* y, long ldy, float* hT, cudaStream_t st) {
   dim3 grid(cdiv(Hp, 128), B);
   if (ot == OT::BF16)
     launch_pdl(scrn_fwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(128), 0, st, 1, 
-        B, H, Hp, Q, ldq, Z, bh, Hf, (__nv_bfloat16*)HSh, ldhs, (__nv_bfloat16*)y, ldy, hT);
+        B, H, Hp, Q, ldq, Z, nsplit, split_stride, bh, Hf, (__nv_bfloat16*)HSh, ldhs, (__nv_bfloat16*)y, ldy, hT);
   else
-    launch_pdl(scrn_fwd_pw_kernel<float, float>, dim3(grid), dim3(128), 0, st, 1, B, H, Hp, Q, ldq, Z, bh, Hf, (float*)HSh, ldhs, (float*)y,
+    launch_pdl(scrn_fwd_pw_kernel<float, float>, dim3(grid), dim3(128), 0, st, 1, B, H, Hp, Q, ldq, Z, nsplit, split_stride, bh, Hf, (float*)HSh, ldhs, (float*)y,
                                                            ldy, hT);
   LAUNCH_CHECK();
 }
@@ -90,7 +95,8 @@ void scrn_fwd_pw(OT ot, int B, int H, int Hp, const float* Q, long ldq, const fl
 template <typename T, typename TDY>
 __global__ void __launch_bounds__(PW_UX * PW_RY)
     scrn_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh,
-                       long ld_dh, const float* __restrict__ Hf, T* __restrict__ DZ, long ldz,
+                       long ld_dh, int nsplit, long split_stride, const float* __restrict__ Hf, T* __restrict__ DZ,
+                       long ldz,
                        float* __restrict__ part, int first) {
   pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
   pdl_trigger();
@@ -105,7 +111,11 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
       float dz = 0.f;
       if (j < H) {
         float g = to_f<TDY>(dy[(long)b * ldy + j]);
-        if (dh) g = __fadd_rn(g, dh[(long)b * ld_dh + j]);
+        if (dh) {   // reading R33: split-K partials of dz·Rᵀ summed in chunk order, then added to dy
+          float r = dh[(long)b * ld_dh + j];
+          for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, dh[k * split_stride + (long)b * ld_dh + j]);
+          g = __fadd_rn(g, r);
+        }
         const float h = Hf[(long)b * Hp + j];
         dz = __fmul_rn(__fmul_rn(g, h), __fsub_rn(1.f, h));
       }
@@ -125,17 +135,18 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
 }
 
 void scrn_bwd_pw(OT ot, int B, int H, int Hp, const void* dy, long ldy, bool dy_f32, const float* dh, long ld_dh,
-                 const float* Hf, void* DZ, long ldz, float* part, bool first, cudaStream_t st) {
+                 int nsplit, long split_stride, const float* Hf, void* DZ, long ldz, float* part, bool first,
+                 cudaStream_t st) {
   dim3 grid(cdiv(Hp, PW_UX), pw_row_chunks(B)), block(PW_UX, PW_RY);
   if (ot == OT::BF16) {
     if (dy_f32)
-      launch_pdl(scrn_bwd_pw_kernel<__nv_bfloat16, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh, ld_dh,
+      launch_pdl(scrn_bwd_pw_kernel<__nv_bfloat16, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh, ld_dh, nsplit, split_stride,
                                                                        Hf, (__nv_bfloat16*)DZ, ldz, part, first);
     else
       launch_pdl(scrn_bwd_pw_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(grid), dim3(block), 0, st, 1, 
-          B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh, ld_dh, Hf, (__nv_bfloat16*)DZ, ldz, part, first);
+          B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh, ld_dh, nsplit, split_stride, Hf, (__nv_bfloat16*)DZ, ldz, part, first);
   } else {
-    launch_pdl(scrn_bwd_pw_kernel<float, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh, ld_dh, Hf,
+    launch_pdl(scrn_bwd_pw_kernel<float, float>, dim3(grid), dim3(block), 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh, ld_dh, nsplit, split_stride, Hf,
                                                              (float*)DZ, ldz, part, first);
   }
   LAUNCH_CHECK();

@@ -14,6 +14,8 @@
 //
 // Operand layout: HS [(T+1)·B][Hp + Sp] holds h (cols 0..Hp) and s (cols Hp..) side by side, so the
 // LM head reads [h | s] as one K-concatenated operand; DZS [T·B][Hp + Sp] likewise holds dz and (1−α)ds.
+#include <algorithm>
+
 #include "cell.h"
 
 namespace astra {
@@ -24,6 +26,15 @@ class ScrnCell : public Cell {
   float alpha;
   size_t off_X, off_XAB, off_Sf, off_HS, off_Hf, off_MAB, off_MP, off_MR;
   size_t off_Z, off_dH, off_DZS, off_DSP, off_part;
+
+  // Reading R33: both chain GEMMs (h·R and dz·Rᵀ, K = Hp, N = Hp) split over K into s fixed chunks
+  // when the batch gives few output tiles; the pointwise kernels sum the partials in chunk order.
+  int chain_ksplit() const {
+    const int tiles = cdiv(B, 128) * cdiv(Hp, 64), nk = cdiv(Hp, 64);
+    int s = std::max(1, std::min(4, 64 / std::max(1, tiles)));
+    while (s > 1 && nk / s < 4) --s;
+    return s;
+  }
 
   explicit ScrnCell(const astra_cell_desc& dd) : Cell(dd) {
     S = d.context;
@@ -51,8 +62,8 @@ class ScrnCell : public Cell {
     saved_bytes = s.o;
     nchunk = pw_row_chunks(B);
     Carve c;
-    off_Z = c.take((size_t)B * Hp * 4);
-    off_dH = c.take((size_t)B * Hp * 4);
+    off_Z = c.take((size_t)chain_ksplit() * B * Hp * 4);
+    off_dH = c.take((size_t)chain_ksplit() * B * Hp * 4);
     off_DZS = c.take(TB * Yw * e);
     off_DSP = c.take(TB * Sp * 4);
     off_part = c.take((size_t)nchunk * Hp * 4);
@@ -128,9 +139,13 @@ class ScrnCell : public Cell {
     rec.B = mat(MR, Hp, Hp, Hp);
     rec.M = B; rec.N = Hp; rec.K = Hp;
     rec.b_keep = true;
+    rec.ksplit = chain_ksplit();
+    EpiStore ez = epi(Z, Hp, B, Hp);
+    ez.split_stride = (long)B * Hp;
     for (int t = 0; t < T; ++t) {
-      run_gemm(2, rec, epi(Z, Hp, B, Hp), t, 0, var.g[G_REC], st);
-      scrn_fwd_pw(ot, B, H, Hp, XAB + (long)t * B * Yw, Yw, Z, p("b_h"), Hf + (long)(t + 1) * B * Hp, HSrow(t + 1),
+      run_gemm(2, rec, ez, t, 0, var.g[G_REC], st);
+      scrn_fwd_pw(ot, B, H, Hp, XAB + (long)t * B * Yw, Yw, Z, rec.ksplit, (long)B * Hp, p("b_h"),
+                  Hf + (long)(t + 1) * B * Hp, HSrow(t + 1),
                   Yw, y ? (char*)y + (size_t)t * B * ldy * e : nullptr, ldy, t == T - 1 ? hT : nullptr, st);
       fwd_step_done(t, st);
     }
@@ -163,19 +178,25 @@ class ScrnCell : public Cell {
     bp.b_mn = true;
     bp.M = B; bp.N = Hp; bp.K = Hp;
     bp.b_keep = true;
+    GemmSpec bp0 = bp;   // dh0 (once, no split)
+    bp.ksplit = chain_ksplit();
     for (int t = T - 1; t >= 0; --t) {
       const float* dh = dhT;
       long ld_dh = H;
+      int nsplit = 1;
       if (t < T - 1) {
-        run_gemm(3, bp, epi(dH, Hp, B, Hp), t + 1, 0, var.g[G_BPTT], st);
+        EpiStore eh = epi(dH, Hp, B, Hp);
+        eh.split_stride = (long)B * Hp;
+        run_gemm(3, bp, eh, t + 1, 0, var.g[G_BPTT], st);
         dh = dH;
         ld_dh = Hp;
+        nsplit = bp.ksplit;
       }
       const void* dyt = lm_mode ? (const void*)(lm_dy + (long)t * B * Yw) : (const char*)dy + (size_t)t * B * ldy * e;
-      scrn_bwd_pw(ot, B, H, Hp, dyt, ldy, lm_mode, dh, ld_dh, Hf + (long)(t + 1) * B * Hp, DZS + (size_t)t * B * Yw * e,
-                  Yw, part, t == T - 1, st);
+      scrn_bwd_pw(ot, B, H, Hp, dyt, ldy, lm_mode, dh, ld_dh, nsplit, (long)B * Hp, Hf + (long)(t + 1) * B * Hp,
+                  DZS + (size_t)t * B * Yw * e, Yw, part, t == T - 1, st);
     }
-    if (dh0) run_gemm(3, bp, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
+    if (dh0) run_gemm(13, bp0, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
     // s-chain: DSP = DZ·Pᵀ then the reverse scan
     GemmSpec dsp;
     dsp.A = mat(DZS, Hp, TB, Yw);
