@@ -3,9 +3,9 @@
 //
 //   e_j = vᵀ tanh(q + k_j),  p = softmax_j(e),  ctx = Σ_j p_j enc_j          (one decoder step, per b)
 //
-// One CTA per batch row b; every reduction (over the attention width A for e_j, over j for the
-// softmax / context, over the hidden units for dp_j) is a fixed-order block tree, so the result is
-// independent of launch timing (R5).  fp32 throughout (ALU/MUFU-bound).
+// One CTA per batch row b; every reduction (over the attention width A for e_j and the hidden units
+// for dp_j: one warp per source position, lane-strided partials + a fixed xor tree; over j for the
+// softmax: warp 0, the same tree) has a fixed order, so the result is independent of launch timing (R5).  fp32 throughout (ALU/MUFU-bound).
 #include "cell_math.cuh"
 #include "kernels.h"
 #include "pdl.cuh"
@@ -43,25 +43,35 @@ __global__ void __launch_bounds__(ATT_THREADS)
   extern __shared__ float sh[];
   float* e = sh;            // [Ts]
   float* red = sh + Ts;     // [33]
+  (void)red;
   const int b = blockIdx.x;
+  const int w = threadIdx.x / 32, l = threadIdx.x % 32;
   const float* qb = q + (long)b * Ap;
-  for (int j = 0; j < Ts; ++j) {
+  // e_j: one warp per source position j; lane l sums a = l, l + 32, ... in order, then a fixed
+  // xor-butterfly over the lanes (no block-wide barrier per j)
+  for (int j = w; j < Ts; j += ATT_THREADS / 32) {
     const float* kj = keys + ((long)j * B + b) * Ap;
     float s = 0.f;
-    for (int a = threadIdx.x; a < A; a += ATT_THREADS) s = __fadd_rn(s, __fmul_rn(v[a], tanh_<FastMath<T>::value>(__fadd_rn(qb[a], kj[a]))));
-    const float tot = block_sum(s, red);
-    if (threadIdx.x == 0) e[j] = tot;
+    for (int a = l; a < A; a += 32) s = __fadd_rn(s, __fmul_rn(v[a], tanh_<FastMath<T>::value>(__fadd_rn(qb[a], kj[a]))));
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+    if (l == 0) e[j] = s;
   }
   __syncthreads();
-  if (threadIdx.x == 0) {   // softmax over j (Ts is small): sequential, fixed order
+  if (w == 0) {   // softmax over j by warp 0: lane-strided max / sum, fixed xor trees
     float m = -INFINITY;
-    for (int j = 0; j < Ts; ++j) m = fmaxf(m, e[j]);
+    for (int j = l; j < Ts; j += 32) m = fmaxf(m, e[j]);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
     float s = 0.f;
-    for (int j = 0; j < Ts; ++j) {
+    for (int j = l; j < Ts; j += 32) {
       e[j] = expf(__fsub_rn(e[j], m));
       s = __fadd_rn(s, e[j]);
     }
-    for (int j = 0; j < Ts; ++j) e[j] = __fdiv_rn(e[j], s);
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+    __syncwarp();
+    for (int j = l; j < Ts; j += 32) e[j] = __fdiv_rn(e[j], s);
   }
   __syncthreads();
   for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) pr[(long)b * Ts + j] = e[j];
@@ -112,44 +122,72 @@ __global__ void __launch_bounds__(ATT_THREADS)
     dctx[h] = d;
   }
   __syncthreads();
-  for (int j = 0; j < Ts; ++j) {
+  (void)red;
+  const int w = threadIdx.x / 32, l = threadIdx.x % 32;
+  for (int j = w; j < Ts; j += ATT_THREADS / 32) {   // dp_j: one warp per j, lane-strided h, xor tree
     const float* ej = enc + ((long)j * B + b) * Hp;
     float s = 0.f;
-    for (int h = threadIdx.x; h < H; h += ATT_THREADS) s = __fadd_rn(s, __fmul_rn(dctx[h], ej[h]));
-    const float tot = block_sum(s, red);
-    if (threadIdx.x == 0) de[j] = tot;   // dp_j for now
+    for (int h = l; h < H; h += 32) s = __fadd_rn(s, __fmul_rn(dctx[h], ej[h]));
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+    if (l == 0) de[j] = s;   // dp_j for now
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
+  if (w == 0) {   // de_j = p_j (dp_j − Σ p dp), the sum by a fixed xor tree over lane-strided partials
     float s = 0.f;
-    for (int j = 0; j < Ts; ++j) s = __fadd_rn(s, __fmul_rn(pr[(long)b * Ts + j], de[j]));
-    for (int j = 0; j < Ts; ++j) de[j] = __fmul_rn(pr[(long)b * Ts + j], __fsub_rn(de[j], s));
+    for (int j = l; j < Ts; j += 32) s = __fadd_rn(s, __fmul_rn(pr[(long)b * Ts + j], de[j]));
+#pragma unroll
+    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+    __syncwarp();
+    for (int j = l; j < Ts; j += 32) de[j] = __fmul_rn(pr[(long)b * Ts + j], __fsub_rn(de[j], s));
   }
   __syncthreads();
-  // denc_j += p_j dctx
-  for (int j = 0; j < Ts; ++j) {
-    const float pj = pr[(long)b * Ts + j];
-    float* dj = denc + ((long)j * B + b) * Hp;
-    for (int h = threadIdx.x; h < Hp; h += ATT_THREADS) {
-      const float add = __fmul_rn(pj, dctx[h]);
-      dj[h] = first ? add : __fadd_rn(dj[h], add);
+  // denc_j += p_j dctx.  The accumulators (L2-resident) are read-modified-written in groups of
+  // ATT_JG source positions with every load of a group issued before its stores, so a thread keeps
+  // ATT_JG requests in flight instead of one dependent round trip per j.
+  constexpr int ATT_JG = 10;
+  for (int h = threadIdx.x; h < Hp; h += ATT_THREADS) {
+    const float dc = dctx[h];
+    for (int j0 = 0; j0 < Ts; j0 += ATT_JG) {
+      float old[ATT_JG];
+#pragma unroll
+      for (int k = 0; k < ATT_JG; ++k)
+        old[k] = (!first && j0 + k < Ts) ? denc[((long)(j0 + k) * B + b) * Hp + h] : 0.f;
+#pragma unroll
+      for (int k = 0; k < ATT_JG; ++k) {
+        if (j0 + k >= Ts) break;
+        const float add = __fmul_rn(pr[(long)b * Ts + j0 + k], dc);
+        denc[((long)(j0 + k) * B + b) * Hp + h] = first ? add : __fadd_rn(old[k], add);
+      }
     }
   }
-  // attention-width terms
+  // attention-width terms (dq and dv accumulated in ascending j, dk_j read-modify-written in groups)
   const float* qb = q + (long)b * Ap;
   for (int a = threadIdx.x; a < Ap; a += ATT_THREADS) {
     float dq = 0.f, dva = 0.f;
     const bool valid = a < A;
-    for (int j = 0; j < Ts; ++j) {
-      float* dkj = dk + ((long)j * B + b) * Ap + a;
-      float du = 0.f;
-      if (valid) {
-        const float u = tanh_<FastMath<T>::value>(__fadd_rn(qb[a], keys[((long)j * B + b) * Ap + a]));
-        du = __fmul_rn(__fmul_rn(de[j], v[a]), __fsub_rn(1.f, __fmul_rn(u, u)));
-        dq = __fadd_rn(dq, du);
-        dva = __fadd_rn(dva, __fmul_rn(de[j], u));
+    const float qa = valid ? qb[a] : 0.f, va = valid ? v[a] : 0.f;
+    for (int j0 = 0; j0 < Ts; j0 += ATT_JG) {
+      float old[ATT_JG], kk[ATT_JG];
+#pragma unroll
+      for (int k = 0; k < ATT_JG; ++k) {
+        const bool in = j0 + k < Ts;
+        old[k] = (!first && in) ? dk[((long)(j0 + k) * B + b) * Ap + a] : 0.f;
+        kk[k] = (valid && in) ? keys[((long)(j0 + k) * B + b) * Ap + a] : 0.f;
       }
-      *dkj = first ? du : __fadd_rn(*dkj, du);
+#pragma unroll
+      for (int k = 0; k < ATT_JG; ++k) {
+        const int j = j0 + k;
+        if (j >= Ts) break;
+        float du = 0.f;
+        if (valid) {
+          const float u = tanh_<FastMath<T>::value>(__fadd_rn(qa, kk[k]));
+          du = __fmul_rn(__fmul_rn(de[j], va), __fsub_rn(1.f, __fmul_rn(u, u)));
+          dq = __fadd_rn(dq, du);
+          dva = __fadd_rn(dva, __fmul_rn(de[j], u));
+        }
+        dk[((long)j * B + b) * Ap + a] = first ? du : __fadd_rn(old[k], du);
+      }
     }
     dq_op[(long)b * Ap + a] = from_f<T>(dq);
     float* dv = dvb + (long)b * Ap + a;

@@ -79,8 +79,11 @@ def attn_run(name, H, I, A_, B, Ts, Tt, steps=10):
     for _ in range(steps): step()
     e1.record(); torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / steps
+    import bench
+    step(); torch.cuda.synchronize()
+    regions = {k: round(v, 3) for k, v in bench.region_times(c).items()}
     print(json.dumps({"config": name, "samples_per_s": round(B / ms * 1e3, 1), "ms_per_step": round(ms, 3),
-                      "tuner_steps": n, "configs_explored": rep.get("configs_explored"), "variant": rep["variant"]}),
+                      "regions": regions, "tuner_steps": n, "configs_explored": rep.get("configs_explored"), "variant": rep["variant"]}),
           flush=True)
 
 
