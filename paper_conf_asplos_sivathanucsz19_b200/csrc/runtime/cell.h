@@ -42,11 +42,13 @@ extern const char* const ROLE_NAMES[G_ROLES];
 
 // One binding of every adaptive variable (the enumerator's output for a cell).
 constexpr int HEAD_CHUNKS[3] = {1, 2, 5};
+constexpr int WF_CHUNKS[3] = {1, 5, 1 << 20};   // clipped to T: the last option is one chunk per step
 struct Variant {
   KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
   int fwd_mode = 0;     // K2 (LSTM family, bf16): 0 GEMM + pointwise kernel, 1 fused per step, 2 fused persistent
   int bwd_mode = 0;     // K4: same encoding
+  int lwf = 0;          // stacked LM: layer wavefront in WF_CHUNKS[lwf] time chunks (1 = layers one after the other)
   int head_ov = 0;      // LM head overlapped with the forward chain in HEAD_CHUNKS[head_ov] time chunks (B3)
   int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
   Variant() { g[G_BPTT].bn = 128; }
@@ -136,6 +138,15 @@ class Cell {
   const float* lm_dy = nullptr;  // fp32 [T*B][y_width()] internal dY for the backward (null: external dy)
   float* y_f32 = nullptr;        // optional internal fp32 output [T*B][y_width()] (LSTM family)
   int lm_V = 0;
+
+  // time range [rg_t0, rg_t1) of the next forward / backward call (rg_t1 < 0: all of [0, T)): a
+  // stacked LM's layer wavefront runs layers chunk by chunk (cells with supports_ranges() only)
+  int rg_t0 = 0, rg_t1 = -1;
+  virtual bool supports_ranges() const { return false; }
+  int lm_role = 0;      // 0 not in an LM, 1 lower layer of a stack, 2 the layer the head reads
+  int lm_layers = 1;    // layers of the LM this cell belongs to
+  bool lm_wavefront = false;   // (top layer) every layer of the stack supports ranges: AV lwf exists
+  std::function<void()> bwd_hook;   // called after a ranged backward call enqueued its dX rows
 
   // ---- per-family interface
   virtual void forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT) = 0;
@@ -231,6 +242,10 @@ class LM {
   size_t off_tokpad = 0;      // int32 [Tmax+1][B] padded token buffer
   size_t off_nv = 0;          // int32 device scalar: rows of the step that carry a loss
   cudaEvent_t ev_hfork = nullptr, ev_hdy = nullptr, ev_hdone = nullptr, ev_chunk[5] = {};
+  // layer wavefront: one stream per layer above the bottom, events per (layer, chunk)
+  std::vector<cudaStream_t> lstreams;
+  std::vector<cudaEvent_t> wf_ev;
+  cudaEvent_t wf_event(int i);
   int bucket_for(int len) const;
   void step_var(const int32_t* tokens, int len, float lr, float* loss_dev, bool do_sgd);
   int wo_split(long TB) const;   // R28 split for the active T·B

@@ -22,6 +22,7 @@ std::string Variant::str() const {
     o << ",";
   }
   o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf << ",hov=" << head_ov;
+  if (lwf) o << ",lwf=" << lwf;
   return o.str();
 }
 
@@ -40,6 +41,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "wg_side") {
       v.wg_side = std::stoi(val);
       ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    if (k == "lwf") {
+      v.lwf = std::stoi(val);
+      ASTRA_CHECK_ARG(v.lwf >= 0 && v.lwf <= 2, "variant: lwf must be 0..2 (layer wavefront in 1, 5 or T chunks)");
       continue;
     }
     if (k == "hov") {
@@ -316,8 +322,11 @@ void Cell::tuner_setup() {
   if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
   // B3 stream assignment for the LM head: time-chunked on a side stream, overlapping the forward
   // chain (its chunks' logits / CE / dgrad) and the BPTT chain (its weight gradient); step metric
-  if (lm_mode && !side.empty() && T >= 2)
+  if (lm_mode && lm_role == 2 && !side.empty() && T >= 2)
     t = "(pre " + t + " (leaf head_ov " + std::to_string(T >= 5 ? 3 : 2) + " t_step))";
+  // stacked LM (top layer): layer wavefront, against the whole step
+  if (lm_mode && lm_role == 2 && lm_layers > 1 && lm_wavefront && T >= 2)
+    t = "(pre " + t + " (leaf lwf " + std::to_string(T > 5 ? 3 : 2) + " t_step))";
   if (t.empty()) t = "(leaf none 1 t_step)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
   wirer.reset(new tuner::Wirer(tree.get()));
@@ -338,6 +347,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "fuse_fwd") { v.fwd_mode = o; continue; }
     if (n == "fuse_bwd") { v.bwd_mode = o; continue; }
     if (n == "head_ov") { v.head_ov = o; continue; }
+    if (n == "lwf") { v.lwf = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

@@ -62,6 +62,7 @@ class LstmCell : public Cell {
 
   int fwd_fusions() const override { return 3; }
   bool chain_prefetch() const override { return true; }
+  bool supports_ranges() const override { return true; }
   RecFwd2Maps fm;                       // tensor maps of the fused CTA-pair forward (built at first use)
   const void* fm_key = (const void*)1;  // y pointer the maps were built for
   const void* fm_wx = nullptr;          // workspace they were built for (rebind ⇒ rebuild)
@@ -108,29 +109,35 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   float* UH = sv<float>(off_UH);
   float* Cb = sv<float>(off_C);
 
-  mark(R_STEP, 0, st);
-  // K9 second half: operand mirrors in the internal gate-interleaved layout
-  mirror_gates_T(ot, p("W"), I, H, Hp, Wm, Ip, st);
-  mirror_gates_T(ot, p("U"), H, H, Hp, Um, Hp, st);
-  if (!lm_mode) copy_pad(ot, x, ot, TB, I, I, X, Ip, st);
-  copy_pad(ot, h0, OT::F32, B, H, H, Hrow(0), Hp, st);
-  copy_f32_pad(c0, B, H, H, Cb, Hp, H, st);
+  // time range of this call (the layer wavefront of a stacked LM runs the forward in chunks)
+  const int t0 = rg_t1 < 0 ? 0 : rg_t0, t1 = rg_t1 < 0 ? T : rg_t1;
+  const bool whole = t0 == 0 && t1 == T;
+  if (t0 == 0) {
+    if (!lm_mode) mark(R_STEP, 0, st);   // an LM marks its step itself (embedding included)
+    // K9 second half: operand mirrors in the internal gate-interleaved layout
+    mirror_gates_T(ot, p("W"), I, H, Hp, Wm, Ip, st);
+    mirror_gates_T(ot, p("U"), H, H, Hp, Um, Hp, st);
+    if (!lm_mode) copy_pad(ot, x, ot, TB, I, I, X, Ip, st);
+    copy_pad(ot, h0, OT::F32, B, H, H, Hrow(0), Hp, st);
+    copy_f32_pad(c0, B, H, H, Cb, Hp, H, st);
+  }
 
   GateParams gp;
   gp.b = p("b");
   if (kind == K_MILSTM) { gp.alpha = p("alpha"); gp.beta1 = p("beta1"); gp.beta2 = p("beta2"); }
 
-  // a1: hoisted input projection for all timesteps
-  mark(R_A1, 0, st);
+  // a1: hoisted input projection for the range's timesteps (row chunks of one GEMM: same bits)
+  if (t0 == 0) mark(R_A1, 0, st);
   GemmSpec a1;
-  a1.A = mat(X, I, TB, Ip);
+  const long rows = (long)(t1 - t0) * B;
+  a1.A = mat((const char*)X + (size_t)t0 * B * Ip * e, I, rows, Ip);
   a1.B = mat(Wm, I, NG, Ip);
-  a1.M = (int)TB; a1.N = NG; a1.K = I;
-  run_gemm(0, a1, epi(WX, NG, (int)TB, NG), 0, 0, var.g[G_A1], st);
-  mark(R_A1, 1, st);
+  a1.M = (int)rows; a1.N = NG; a1.K = I;
+  run_gemm(whole ? 0 : 100000 + t0 * 1024 + (t1 - t0), a1, epi(WX + (size_t)t0 * B * NG, NG, (int)rows, NG), 0, 0, var.g[G_A1], st);
+  if (t0 == 0) mark(R_A1, 1, st);
 
   // a3: recurrent chain
-  mark(R_FWD, 0, st);
+  if (t0 == 0) mark(R_FWD, 0, st);
   GemmSpec rec;
   rec.A = mat(Hrow(0), Hp, B, Hp, T + 1, (long)B * Hp);
   rec.B = mat(Um, Hp, NG, Hp);
@@ -159,7 +166,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     ra.y_kind = !y ? 0 : (H % 8 == 0 && ((uintptr_t)y & 15) == 0) ? 1 : 2;
     ra.y = y;
     ra.gp = gp;
-    for (int t = 0; t < T; ++t) {
+    for (int t = t0; t < t1; ++t) {
       ra.t = t;
       const bool last = t == T - 1;
       ra.hT = last ? hT : nullptr;
@@ -183,19 +190,19 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     const bool persistent = var.fwd_mode == 2 && ra.num_m * ra.num_n <= num_sms() && ra.num_m <= 1024;
     if (persistent) {
       CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
-      ra.persistent = 1; ra.t0 = 0; ra.t1 = T;
+      ra.persistent = 1; ra.t0 = t0; ra.t1 = t1;
       lstm_rec_fwd_launch(kind, tg.mapA, tg.mapB, ra, st);
-      for (int t = 0; t < T; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
+      for (int t = t0; t < t1; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
     } else {
       ra.persistent = 0;
-      for (int t = 0; t < T; ++t) {
+      for (int t = t0; t < t1; ++t) {
         ra.t0 = t; ra.t1 = t + 1;
         lstm_rec_fwd_launch(kind, tg.mapA, tg.mapB, ra, st);
         fwd_step_done(t, st);
       }
     }
   } else {
-    for (int t = 0; t < T; ++t) {
+    for (int t = t0; t < t1; ++t) {
       float* UHt = UH + (long)t * B * NG;
       L2Pf pf{};   // R31: WX_t, read by this step's pointwise kernel
       pf.p[0] = WX + (long)t * B * NG; pf.n[0] = (var.l2pf & 1) ? (unsigned long long)B * NG * 4 : 0;
@@ -212,8 +219,10 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
       fwd_step_done(t, st);
     }
   }
-  mark(R_FWD, 1, st);
-  fwd_done = true;
+  if (t1 == T) {
+    mark(R_FWD, 1, st);
+    fwd_done = true;
+  }
 }
 
 void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void* dx, float* dh0, float* dc0) {
@@ -239,10 +248,14 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   gp.b = p("b");
   if (kind == K_MILSTM) { gp.alpha = p("alpha"); gp.beta1 = p("beta1"); gp.beta2 = p("beta2"); }
 
-  copy_f32_pad(dcT, B, H, H, dC, Hp, H, st);
-
-  // a5: BPTT chain
-  mark(R_BPTT, 0, st);
+  // time range of this call (descending chunks under the layer wavefront of a stacked LM)
+  const int t0 = rg_t1 < 0 ? 0 : rg_t0, t1 = rg_t1 < 0 ? T : rg_t1;
+  const bool whole = t0 == 0 && t1 == T;
+  if (t1 == T) {
+    copy_f32_pad(dcT, B, H, H, dC, Hp, H, st);
+    // a5: BPTT chain
+    mark(R_BPTT, 0, st);
+  }
   GemmSpec bp;
   bp.A = mat(Duh, NG, B, NG, T, (long)B * NG);
   bp.B = mat(Um, Hp, NG, Hp);
@@ -278,7 +291,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     fa.gp = gp;
     fa.D_uh = Duh; fa.D_wx = Dwx; fa.dc = dC; fa.partials = part;
   }
-  for (int t = T - 1; t >= 0; --t) {
+  for (int t = t1 - 1; t >= t0; --t) {
     if (fuse && t < T - 1) {
       fa.t = t;
       lstm_bptt_fused_launch(kind, !lm_dy, bm, fa, st);
@@ -315,6 +328,22 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
                        UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
                        Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
   }
+  auto dx_rows = [&](int r0, int r1, int id) {   // dX = D_wx·Wᵀ for timesteps [r0, r1) (row chunk: same bits)
+    const long rows = (long)(r1 - r0) * B;
+    GemmSpec gx;
+    gx.A = mat(Dwx + (size_t)r0 * B * NG * e, NG, rows, NG);
+    gx.B = mat(Wm, I, NG, Ip);
+    gx.b_mn = true;
+    gx.M = (int)rows; gx.N = I; gx.K = NG;
+    if (lm_mode)
+      run_gemm(id, gx, epi((float*)dx + (size_t)r0 * B * Ip, Ip, (int)rows, I), 0, 0, var.g[G_DX], st);
+    else
+      run_gemm(id, gx, epi((char*)dx + (size_t)r0 * B * I * ot_size(ot), I, (int)rows, I, ot == OT::BF16), 0, 0,
+               var.g[G_DX], st);
+  };
+  if (!whole && dx) dx_rows(t0, t1, 200000 + t0 * 1024 + (t1 - t0));   // the layer below's dy for this chunk, right away
+  if (bwd_hook) bwd_hook();
+  if (t0 > 0) return;
   if (dh0) run_gemm(3, bp0, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
   if (dc0) copy_pad(OT::F32, dC, OT::F32, B, H, Hp, dc0, H, st);
   mark(R_BPTT, 1, st);
@@ -349,17 +378,9 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   mark(R_DW, 1, st);
   grad_bucket(g("W"), (size_t)I * 4 * H, st);
 
-  if (dx) {
-    GemmSpec gx;
-    gx.A = mat(Dwx, NG, TB, NG);
-    gx.B = mat(Wm, I, NG, Ip);
-    gx.b_mn = true;
-    gx.M = (int)TB; gx.N = I; gx.K = NG;
+  if (dx && whole) {
     mark(R_DX, 0, st);
-    if (lm_mode)
-      run_gemm(6, gx, epi(dx, Ip, (int)TB, I), 0, 0, var.g[G_DX], st);
-    else
-      run_gemm(6, gx, epi(dx, I, (int)TB, I, ot == OT::BF16), 0, 0, var.g[G_DX], st);
+    dx_rows(0, T, 6);
     mark(R_DX, 1, st);
   }
   float* gq[4] = {g("b"), nullptr, nullptr, nullptr};

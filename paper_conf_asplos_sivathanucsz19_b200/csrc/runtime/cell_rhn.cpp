@@ -100,7 +100,7 @@ class RhnCell : public Cell {
     char* MW = sv<char>(off_MW);
     char* MR = sv<char>(off_MR);
 
-    mark(R_STEP, 0, st);
+    if (!lm_mode) mark(R_STEP, 0, st);   // an LM marks its step itself
     mirror_blocked_T(ot, p("W"), I, 2, H, Hp, MW, Ip, st);
     for (int l = 0; l < L; ++l)
       mirror_blocked_T(ot, p("R") + (size_t)l * H * 2 * H, H, 2, H, Hp, MR + (size_t)l * G2 * Hp * e, Hp, st);

@@ -105,7 +105,7 @@ class ScrnCell : public Cell {
     float* Z = sc<float>(off_Z);
     const long ldy = H + S;
 
-    mark(R_STEP, 0, st);
+    if (!lm_mode) mark(R_STEP, 0, st);   // an LM marks its step itself
     // operand mirrors: [A | Bm]ᵀ, Pᵀ (as [H][S]), Rᵀ
     mirror_T(ot, p("A"), I, H, Hp, Ip, MAB, Ip, st);
     mirror_T(ot, p("Bm"), I, S, Sp, Ip, MAB + (size_t)Hp * Ip * e, Ip, st);

@@ -145,8 +145,13 @@ size_t LM::find(const std::string& n) const {
 void LM::bind(float* pp, float* gg, void* wsp) {
   ASTRA_CHECK_ARG(pp && gg && wsp, "lm_bind: null pointer");
   P = pp; G = gg; ws = (char*)wsp;
+  bool ranges = true;
+  for (Cell* L : layers) ranges = ranges && L->supports_ranges();
   for (size_t l = 0; l < layers.size(); ++l) {
     layers[l]->lm_mode = true;
+    layers[l]->lm_role = l + 1 == layers.size() ? 2 : 1;
+    layers[l]->lm_layers = (int)layers.size();
+    layers[l]->lm_wavefront = ranges && layers.size() > 1;
     layers[l]->bind(pp + layer_poff[l], gg + layer_poff[l], ws + off_lsaved[l], ws + off_lscratch[l]);
   }
   set_state(nullptr, nullptr);
@@ -176,6 +181,15 @@ void LM::set_state(const float* h, const float* c) {
   }
 }
 
+cudaEvent_t LM::wf_event(int i) {
+  if ((int)wf_ev.size() <= i) {
+    const size_t n0 = wf_ev.size();
+    wf_ev.resize(i + 1, nullptr);
+    for (size_t j = n0; j < wf_ev.size(); ++j) CUDA_TRY(cudaEventCreateWithFlags(&wf_ev[j], cudaEventDisableTiming));
+  }
+  return wf_ev[i];
+}
+
 void LM::set_active_T(int t) {
   for (Cell* c : layers) c->set_active_T(t);
 }
@@ -200,6 +214,9 @@ LM::~LM() {
     if (ev) cudaEventDestroy(ev);
   for (cudaEvent_t ev : ev_chunk)
     if (ev) cudaEventDestroy(ev);
+  for (cudaEvent_t ev : wf_ev) cudaEventDestroy(ev);
+  for (cudaStream_t s2 : lstreams)
+    if (s2) cudaStreamDestroy(s2);
 }
 
 void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
@@ -311,6 +328,29 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   std::vector<int> t_end(nch);   // last forward step of each time chunk
   for (int k = 0; k < nch; ++k) t_end[k] = (int)((long)(k + 1) * c.T / nch) - 1;
 
+  for (Cell* L : layers) L->mark(R_STEP, 0, st);
+  // layer wavefront (AV lwf of the top layer): layer l runs on its own stream, time chunk by time
+  // chunk; chunk k of layer l starts when layer l-1 finished chunk k (forward) / layer l+1 produced
+  // the dX rows of chunk k (backward).  Row chunks of the same GEMMs, the chains unchanged: the
+  // same bits as layers one after the other.
+  bool wf_ok = nl > 1;
+  for (Cell* L : layers) wf_ok = wf_ok && L->supports_ranges();
+  const int nwc = wf_ok ? std::min({WF_CHUNKS[std::min(2, std::max(0, c.var.lwf))], c.T, 64}) : 1;
+  std::vector<int> tb(nwc + 1);
+  for (int k = 0; k <= nwc; ++k) tb[k] = (int)((long)k * c.T / nwc);
+  auto lst = [&](int l) { return l == 0 || nwc == 1 ? st : lstreams[l]; };
+  if (nwc > 1) {
+    while ((int)lstreams.size() < nl) {
+      cudaStream_t s2 = nullptr;
+      if (!lstreams.empty()) CUDA_TRY(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+      lstreams.push_back(s2);
+    }
+    CUDA_TRY(cudaEventRecord(wf_event(0), st));
+    for (int l = 1; l < nl; ++l) CUDA_TRY(cudaStreamWaitEvent(lstreams[l], wf_event(0), 0));
+  }
+  auto ev_f = [&](int l, int k) { return wf_event(1 + l * 64 + k); };
+  auto ev_b = [&](int l, int k) { return wf_event(1 + 32 * 64 + l * 64 + k); };
+
   // a0: embedding gather into layer 0's operand buffer
   embed_gather(c.ot, tokens, TB, P + find("E"), c0.I, c0.x_operand(), c0.Ip, st);
   // head weight mirror (independent of the forward)
@@ -324,8 +364,8 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   auto head_chunk = [&](int k) {
     const long r0 = k == 0 ? 0 : (long)(t_end[k - 1] + 1) * c.B, r1 = (long)(t_end[k] + 1) * c.B;
     const int rows = (int)(r1 - r0);
-    if (ov) {
-      CUDA_TRY(cudaEventRecord(ev_chunk[k], st));
+    if (ov) {   // recorded on the stream the top layer's forward runs on
+      CUDA_TRY(cudaEventRecord(ev_chunk[k], c.main_st));
       CUDA_TRY(cudaStreamWaitEvent(hst, ev_chunk[k], 0));
     }
     GemmSpec hd;
@@ -350,23 +390,45 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
       for (int k = 0; k < nch; ++k)
         if (t == t_end[k]) head_chunk(k);
     };
+  auto restore = [&] {
+    c.fwd_hook = nullptr;
+    for (Cell* L : layers) {
+      L->main_st = st;
+      L->rg_t0 = 0;
+      L->rg_t1 = -1;
+      L->bwd_hook = nullptr;
+    }
+  };
   try {
-    for (int l = 0; l < nl; ++l) {
-      Cell& L = *layers[l];
-      if (l > 0) {   // layer l's input operand = layer l-1's output operand (bf16 / fp32, [T·B][H])
-        const Mat2 yp = layers[l - 1]->y_operand();
-        copy_pad(L.ot, yp.ptr, L.ot, TB, L.I, yp.ld, L.x_operand(), L.Ip, st);
+    for (int k = 0; k < nwc; ++k) {
+      for (int l = 0; l < nl; ++l) {
+        Cell& L = *layers[l];
+        const cudaStream_t S = lst(l);
+        L.main_st = S;
+        if (nwc > 1) {
+          L.rg_t0 = tb[k];
+          L.rg_t1 = tb[k + 1];
+          if (l > 0) CUDA_TRY(cudaStreamWaitEvent(S, ev_f(l - 1, k), 0));
+        }
+        if (l > 0) {   // layer l's input operand = layer l-1's output operand (bf16 / fp32, [T·B][H])
+          const Mat2 yp = layers[l - 1]->y_operand();
+          const long r0 = (long)tb[k] * c.B, rows = (long)(tb[k + 1] - tb[k]) * c.B;
+          copy_pad(L.ot, (const char*)yp.ptr + (size_t)r0 * yp.ld * e, L.ot, rows, L.I, yp.ld,
+                   (char*)L.x_operand() + (size_t)r0 * L.Ip * e, L.Ip, S);
+        }
+        float* hs = (float*)(ws + off_lh[l]);
+        float* cs = L.c_width() > 0 ? (float*)(ws + off_lc[l]) : nullptr;
+        if (step_len > 0) L.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
+        else L.forward(nullptr, hs, cs, nullptr, hs, cs);
+        if (nwc > 1) CUDA_TRY(cudaEventRecord(ev_f(l, k), S));
       }
-      float* hs = (float*)(ws + off_lh[l]);
-      float* cs = L.c_width() > 0 ? (float*)(ws + off_lc[l]) : nullptr;
-      if (step_len > 0) L.forward(nullptr, hs, cs, nullptr, nullptr, nullptr);
-      else L.forward(nullptr, hs, cs, nullptr, hs, cs);
     }
   } catch (...) {
-    c.fwd_hook = nullptr;
+    restore();
     throw;
   }
-  c.fwd_hook = nullptr;
+  if (nwc > 1) CUDA_TRY(cudaStreamWaitEvent(st, ev_f(nl - 1, nwc - 1), 0));   // top done ⇒ every layer done
+  restore();
   if (!ov) head_chunk(0);
   if (ov) {   // BPTT needs every dY row; the weight gradient of the head stays on the side stream
     CUDA_TRY(cudaEventRecord(ev_hdy, hst));
@@ -402,12 +464,38 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
 
   // layers' backward (SE3 + SE4), top down: layer l's input gradient is layer l-1's dy; then the
   // embedding backward
-  for (int l = nl - 1; l >= 0; --l) {
-    Cell& L = *layers[l];
-    L.lm_dy = l == nl - 1 ? dY : (float*)(ws + off_dxl[(l + 1) % 2]);
-    float* dx_l = l == 0 ? dX : (float*)(ws + off_dxl[l % 2]);
-    L.backward(nullptr, nullptr, nullptr, dx_l, nullptr, nullptr);
+  try {
+    if (nwc > 1) {   // dY is ready on the main stream
+      CUDA_TRY(cudaEventRecord(wf_event(1 + 64 * 64), st));
+      CUDA_TRY(cudaStreamWaitEvent(lst(nl - 1), wf_event(1 + 64 * 64), 0));
+    }
+    for (int k = nwc - 1; k >= 0; --k) {
+      for (int l = nl - 1; l >= 0; --l) {
+        Cell& L = *layers[l];
+        const cudaStream_t S = lst(l);
+        L.main_st = S;
+        L.lm_dy = l == nl - 1 ? dY : (float*)(ws + off_dxl[(l + 1) % 2]);
+        float* dx_l = l == 0 ? dX : (float*)(ws + off_dxl[l % 2]);
+        if (nwc > 1) {
+          L.rg_t0 = tb[k];
+          L.rg_t1 = tb[k + 1];
+          if (l < nl - 1) CUDA_TRY(cudaStreamWaitEvent(S, ev_b(l + 1, k), 0));
+          cudaEvent_t done = ev_b(l, k);
+          L.bwd_hook = [done, S] { CUDA_TRY(cudaEventRecord(done, S)); };
+        }
+        L.backward(nullptr, nullptr, nullptr, dx_l, nullptr, nullptr);
+      }
+    }
+    if (nwc > 1)
+      for (int l = 1; l < nl; ++l) {   // join every layer stream (its weight gradients included)
+        CUDA_TRY(cudaEventRecord(wf_event(2 + 64 * 64 + l), lst(l)));
+        CUDA_TRY(cudaStreamWaitEvent(st, wf_event(2 + 64 * 64 + l), 0));
+      }
+  } catch (...) {
+    restore();
+    throw;
   }
+  restore();
   embed_bwd(tokens, TB, V, dX, c0.Ip, c0.I, G + find("E"), ws + off_sort, sort_bytes, (float*)(ws + off_embpart), st);
   // a7: last bucket (embedding), join, then a8: SGD
   c0.grad_bucket(G + find("E"), (size_t)V * c0.I, st);

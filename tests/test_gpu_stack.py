@@ -105,3 +105,44 @@ def test_stacked_shape_mismatch_rejected():
     u = A.Cell("lstm", 64, 128, 8, 4)
     with pytest.raises(A.AstraError):
         A.LM([s, u], 20)   # SCRN's [h|s] output is two segments
+
+
+@pytest.mark.parametrize("cells", [["milstm", "milstm"], ["lstm", "sublstm", "lstm"]])
+@pytest.mark.parametrize("lwf", [1, 2])
+def test_layer_wavefront_bitwise(cells, lwf):
+    """The layer wavefront (AV lwf: layers on their own streams in 5 / T time chunks, chunked a1 and
+    dX) gives the same bits as layers one after the other, over 4 SGD steps with graph replay."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 7, 64, 128, 128, 64
+    out = []
+    for v in (0, lwf):
+        ps, plm, tok, _, _ = _case(cells, T, B, I, H, V, synth.config_seed(5) + 62, True)
+        layers, m = _build(cells, T, B, I, H, V, "bf16", ps, plm)
+        layers[-1].tune_mode(A.TUNE_FROZEN, f"lwf={v}")
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=layers[0].device)
+        for _ in range(4):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append((m.params.clone(), float(m.loss.item())))
+    assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
+
+
+def test_layer_wavefront_matches_oracle():
+    """lwf = per-step wavefront against the stacked fp64 oracle (fp32 path)."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    cells = ["milstm", "lstm"]
+    T, B, I, H, V = 5, 24, 64, 64, 60
+    ps, plm, tok, h0s, c0s = _case(cells, T, B, I, H, V, synth.config_seed(5) + 63, False)
+    layers, m = _build(cells, T, B, I, H, V, "fp32", ps, plm)
+    layers[-1].tune_mode(A.TUNE_FROZEN, "lwf=2")
+    dev = layers[0].device
+    m.set_state(torch.as_tensor(np.concatenate([x.reshape(-1) for x in h0s]), dtype=torch.float32, device=dev),
+                torch.as_tensor(np.concatenate([x.reshape(-1) for x in c0s]), dtype=torch.float32, device=dev))
+    loss = float(m.fwd_bwd(torch.as_tensor(tok, dtype=torch.int32, device=dev)).item())
+    torch.cuda.synchronize()
+    lo, gl, glm = OLM.stacked_lm_forward_backward(cells, ps, plm, tok, h0s, c0s)
+    assert abs(loss - lo) / abs(lo) <= TOL_FP32
+    for l, g in enumerate(gl):
+        for k in g:
+            e = rel_err(m.view(f"L{l}.{k}", m.grads).cpu().numpy().reshape(np.shape(g[k])), g[k])
+            assert e <= TOL_FP32, (l, k, e)
