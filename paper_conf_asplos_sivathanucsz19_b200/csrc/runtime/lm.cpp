@@ -354,7 +354,6 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   // a0: embedding gather into layer 0's operand buffer
   embed_gather(c.ot, tokens, TB, P + find("E"), c0.I, c0.x_operand(), c0.Ip, st);
   // head weight mirror (independent of the forward)
-  c.mark(R_HEAD, 0, hst);
   CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, hst));
   for (const KSeg& s : segs)
     mirror_T(c.ot, P + find("W_o") + (size_t)s.r0 * V, s.n, V, Vr, s.n, Wom + (size_t)s.k0 * e, Yw, hst);
@@ -368,6 +367,7 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
       CUDA_TRY(cudaEventRecord(ev_chunk[k], c.main_st));
       CUDA_TRY(cudaStreamWaitEvent(hst, ev_chunk[k], 0));
     }
+    if (k == 0) c.mark(R_HEAD, 0, hst);   // region: first head chunk → head weight gradient done
     GemmSpec hd;
     hd.A = mat((const char*)Y.ptr + (size_t)r0 * Y.ld * e, Y.inner, rows, Y.ld);
     hd.B = mat(Wom, Yw, V, Yw);
