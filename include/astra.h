@@ -132,6 +132,10 @@ astra_status astra_tune_next(astra_cell c, int* state);
  * (use `forced_variant`, a string from astra_tune_report's "variant" field, or the best
  * found so far when NULL).                                                                  */
 astra_status astra_tune_mode(astra_cell c, int mode, const char* forced_variant);
+/* Region events (cudaEvent pairs around the step phases) on (default) or off.  The
+ * tuner harvests them, so on = 0 is refused with E_STATE while the mode is ASTRA_TUNE_ON; off is
+ * for measuring the profiling overhead (< 0.5 %).                                   */
+astra_status astra_set_profiling(astra_cell c, int on);
 /* JSON report (current variant, #configs explored, index size, trials).  Writes at most
  * len bytes including the NUL; *needed ← required length.                                  */
 astra_status astra_tune_report(astra_cell c, char* buf, size_t len, size_t* needed);

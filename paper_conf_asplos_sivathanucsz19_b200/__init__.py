@@ -56,6 +56,7 @@ _SIGS = {
     "astra_tune_next": [_P, ctypes.POINTER(_I)],
     "astra_tune_mode": [_P, _I, ctypes.c_char_p],
     "astra_tune_report": [_P, ctypes.c_char_p, _SZ, ctypes.POINTER(_SZ)],
+    "astra_set_profiling": [_P, _I],
     "astra_comm_init": [_P, _P, _I, _I],
     "astra_comm_unique_id": [_P, _SZ],
     "astra_lm_create": [ctypes.POINTER(_P), _P, _I],
@@ -186,6 +187,10 @@ class Cell:
         self._side = [torch.cuda.Stream(device=self.device) for _ in range(n_side)]
         arr = (ctypes.c_void_p * max(1, n_side))(*[s.cuda_stream for s in self._side])
         _check(lib().astra_set_streams(self.h, _stream(), arr, n_side, None))
+
+    def set_profiling(self, on: bool):
+        """Region cudaEvent pairs on/off (astra_set_profiling; off only outside exploration)."""
+        _check(lib().astra_set_profiling(self.h, int(bool(on))))
 
     def view(self, name, t=None):
         """View of parameter `name` inside the flat params (or grads) vector, external layout."""

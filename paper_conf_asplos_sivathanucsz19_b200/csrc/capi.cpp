@@ -149,6 +149,7 @@ astra_status astra_tune_mode(astra_cell c, int mode, const char* forced) {
     ASTRA_CHECK_ARG(mode == ASTRA_TUNE_OFF || mode == ASTRA_TUNE_ON || mode == ASTRA_TUNE_FROZEN, "tune_mode: bad mode");
     // every bucket restarts — except a plain freeze, which keeps each bucket's current variant
     if (!(mode == ASTRA_TUNE_FROZEN && !forced)) cc.tune_ctx.clear();
+    if (mode == ASTRA_TUNE_ON) cc.profiling = true;   // exploration reads the region events
     if (mode == ASTRA_TUNE_OFF) {
       cc.var = Variant();
       cc.wirer.reset();
@@ -159,6 +160,15 @@ astra_status astra_tune_mode(astra_cell c, int mode, const char* forced) {
       cc.var = Variant::parse(forced);
     }
     cc.tune_mode = mode;
+  });
+}
+
+astra_status astra_set_profiling(astra_cell c, int on) {
+  return guard([&] {
+    NEED(c);
+    Cell& cc = *c->c;
+    ASTRA_CHECK_STATE(on || cc.tune_mode != ASTRA_TUNE_ON, "set_profiling: exploration needs the region events");
+    cc.profiling = on != 0;
   });
 }
 

@@ -234,7 +234,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   std::string vs;
   for (Cell* L : layers) {
     exploring |= L->tune_mode == ASTRA_TUNE_ON && !(L->wirer && L->wirer->converged());
-    vs += L->var.str() + ";";
+    vs += L->var.str() + (L->profiling ? ";p" : ";");
   }
   if (!use_graphs || !graphs_enabled() || exploring || c.ot != OT::BF16 ||
       (c.world > 1 && !graph_nccl)) {

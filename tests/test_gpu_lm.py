@@ -199,3 +199,25 @@ def test_fused_bptt_lm_bitwise(cell, H):
         torch.cuda.synchronize()
         out.append((m.params.clone(), float(m.loss.item())))
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
+
+
+def test_profiling_switch():
+    """Region events off changes no value (graph re-captured) and is refused while exploring."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    out = []
+    for prof in (True, False):
+        pa, tok, h0, c0 = _lm_case("milstm", 5, 64, 64, 64, 50, synth.config_seed(5) + 70, True)
+        c = A.Cell("milstm", 64, 64, 64, 5, dtype="bf16")
+        m = A.LM(c, 50)
+        m.load(pa)
+        c.tune_mode(A.TUNE_FROZEN, "fwd=0")
+        c.set_profiling(prof)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(3):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append(m.params.clone())
+        c.tune_mode(A.TUNE_ON)
+        with pytest.raises(A.AstraError):
+            c.set_profiling(False)
+    assert torch.equal(out[0], out[1])
