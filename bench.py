@@ -154,6 +154,9 @@ def main():
     ap.add_argument("--batch", type=int, default=None, help="override the per-rank batch (weak) / global batch (strong)")
     ap.add_argument("--strong", action="store_true", help="fixed global batch 512 split over the ranks")
     ap.add_argument("--seq", type=int, default=None, help="override seq (debug)")
+    ap.add_argument("--dp", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1 gradient sum: NCCL all-reduce (K11) or the deterministic peer-memory "
+                         "reduce-scatter + fused SGD / all-gather over NVLink (K11p)")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -165,7 +168,7 @@ def main():
     B_g = B_unit if args.strong else B_unit * max(world, 1)     # global batch of this run
     scaling = "strong" if args.strong else "weak"
     cfg = {"workload": WORKLOAD["workload"], "cell": "MI-LSTM", "hidden": H, "input": I, "global_batch": B_g,
-           "seq_len": T, "vocab": V, "parallelism": f"dp{args.gpus}", "per_gpu_batch": B_g // max(world, 1),
+           "seq_len": T, "vocab": V, "parallelism": f"dp{args.gpus}", "dp_backend": args.dp, "per_gpu_batch": B_g // max(world, 1),
            "l2": "working set per step (GB of activations, 139 MB of fp32 grads) >> 126 MB L2: inputs larger than L2"}
 
     if args.impl == "reference":
@@ -202,7 +205,9 @@ def main():
     if distributed:   # the process group only broadcasts the NCCL id; the library owns the comm (K11)
         uid = [A.comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
-        cell.comm_init(uid[0], rank, world)
+        cell.comm_init(uid[0], rank, world)   # also carries the tuner's cross-rank decisions (R29)
+        if args.dp == "peer" and world > 1:
+            A.peer_exchange(lm)
     tok_host = torch.as_tensor(make_inputs(B_g, T, V, n_sym, rank, world), dtype=torch.int32).pin_memory()
     tokens = tok_host.to(dev)
     lr = 0.05

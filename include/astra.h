@@ -146,6 +146,34 @@ astra_status astra_comm_init(astra_cell c, const void* nccl_unique_id, int rank,
 /* Write a fresh ncclUniqueId (128 bytes) to host memory `out` (call on rank 0).           */
 astra_status astra_comm_unique_id(void* out, size_t len);
 
+/* Deterministic peer-memory backend (K11p; SURVEY §8(e) "backend 2", the semantics of §8(c.3)
+ * item 8: g = (1/N)·Σ_r g_r over contiguous batch shards).  Replaces the NCCL gradient all-reduce
+ * and the SGD of a world > 1 step by kernels that work directly on every rank's memory over
+ * NVLink / NVSwitch (CUDA IPC mappings):
+ *   - each gradient bucket [off, off+n) is cut into `world` contiguous shards (boundaries rounded
+ *     to 4 floats); rank r sums shard r of all ranks' gradients in rank order 0..N-1, scales by
+ *     1/N and stores it into its OWN gradients.  The sum is bitwise independent of bucketing and
+ *     timing, and identical on every N-rank run;
+ *   - SGD updates the owned shards (θ − lr·g, the rounding of astra_sgd) and stores the new values
+ *     into every rank's parameters (the all-gather), so all ranks hold identical parameters.
+ * After a step_bwd / lm_train_step the gradients hold the global mean only on this rank's owned
+ * shards (other elements: this rank's shard-mean gradient).
+ * Protocol: after bind, each rank calls *_comm_peer_handle (ASTRA_PEER_HANDLE_BYTES of host
+ * memory out), the caller all-gathers the handles over its process group (rank order), then each
+ * rank calls *_comm_peer_init with the world × ASTRA_PEER_HANDLE_BYTES array.  The params/grads
+ * vectors must be cudaMalloc memory (torch's default allocator is) and must not be rebound.  Up
+ * to 8 ranks; ranks may share one device (tests).  Every rank must issue the same sequence of
+ * steps.  Exploration (ASTRA_TUNE_ON) with world > 1 also needs astra_comm_init (the tuner's
+ * cross-rank max, reading R29).  A rank that waits more than ASTRA_PEER_TIMEOUT_S (default 60)
+ * seconds for a peer traps the device (sticky ASTRA_E_CUDA), it never hangs.
+ * The library owns the IPC mappings and a 4 KB signal array per rank.                         */
+#define ASTRA_PEER_HANDLE_BYTES 256
+astra_status astra_comm_peer_handle(astra_cell c, void* out, size_t len);
+astra_status astra_comm_peer_init(astra_cell c, const void* handles, int rank, int world);
+/* The same for an LM: the window is the LM's flat params / grads; every layer uses it.         */
+astra_status astra_lm_comm_peer_handle(astra_lm m, void* out, size_t len);
+astra_status astra_lm_comm_peer_init(astra_lm m, const void* handles, int rank, int world);
+
 /* ---- language-model wrapper (embedding → cell → linear head → mean CE) ----------------- */
 /* Adds E [V][I], W_o [Hout][V], b_o [V] after the cell's parameters in one flat vector.    */
 astra_status astra_lm_create(astra_lm* out, astra_cell c, int vocab);

@@ -59,6 +59,10 @@ _SIGS = {
     "astra_set_profiling": [_P, _I],
     "astra_comm_init": [_P, _P, _I, _I],
     "astra_comm_unique_id": [_P, _SZ],
+    "astra_comm_peer_handle": [_P, _P, _SZ],
+    "astra_comm_peer_init": [_P, _P, _I, _I],
+    "astra_lm_comm_peer_handle": [_P, _P, _SZ],
+    "astra_lm_comm_peer_init": [_P, _P, _I, _I],
     "astra_lm_create": [ctypes.POINTER(_P), _P, _I],
     "astra_lm_destroy": [_P],
     "astra_lm_create_stacked": [ctypes.POINTER(_P), _P, _I, _I],
@@ -232,12 +236,48 @@ class Cell:
         b = ctypes.create_string_buffer(uid, len(uid))
         _check(lib().astra_comm_init(self.h, b, rank, world))
 
+    def comm_peer_handle(self) -> bytes:
+        """This rank's peer-memory window handle (astra_comm_peer_handle, K11p)."""
+        return _peer_handle(lib().astra_comm_peer_handle, self.h)
+
+    def comm_peer_init(self, handles: bytes, rank, world):
+        """Map every rank's window (astra_comm_peer_init); handles = the rank-ordered concatenation."""
+        _peer_init(lib().astra_comm_peer_init, self.h, handles, rank, world)
+
     def __del__(self):
         try:
             if getattr(self, "h", None) and not getattr(self, "_owned", False):
                 lib().astra_cell_destroy(self.h)
         except Exception:
             pass
+
+
+PEER_HANDLE_BYTES = 256   # ASTRA_PEER_HANDLE_BYTES
+
+
+def _peer_handle(fn, h):
+    b = ctypes.create_string_buffer(PEER_HANDLE_BYTES)
+    _check(fn(h, b, PEER_HANDLE_BYTES))
+    return b.raw
+
+
+def _peer_init(fn, h, handles, rank, world):
+    assert len(handles) == world * PEER_HANDLE_BYTES, "handles: world x PEER_HANDLE_BYTES bytes in rank order"
+    b = ctypes.create_string_buffer(bytes(handles), len(handles))
+    _check(fn(h, b, rank, world))
+
+
+def peer_exchange(obj, group=None):
+    """Set up the deterministic peer-memory DP backend (K11p) of `obj` (a Cell or an LM) over a
+    torch.distributed process group: all-gather the ranks' window handles in rank order, then map
+    them.  Host plumbing only — the gradient sum and SGD run in the library's kernels."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    mine = obj.comm_peer_handle()
+    allh = [None] * world
+    dist.all_gather_object(allh, mine, group=group)
+    obj.comm_peer_init(b"".join(allh), rank, world)
+    return rank, world
 
 
 def comm_unique_id() -> bytes:
@@ -332,6 +372,13 @@ class LM:
     def fwd_bwd(self, tokens, loss=None):
         _check(lib().astra_lm_fwd_bwd(self.h, _ptr(tokens), _ptr(self.loss if loss is None else loss)))
         return self.loss if loss is None else loss
+
+    def comm_peer_handle(self) -> bytes:
+        """This rank's peer-memory window handle for the LM's params / grads (K11p)."""
+        return _peer_handle(lib().astra_lm_comm_peer_handle, self.h)
+
+    def comm_peer_init(self, handles: bytes, rank, world):
+        _peer_init(lib().astra_lm_comm_peer_init, self.h, handles, rank, world)
 
     def __del__(self):
         try:

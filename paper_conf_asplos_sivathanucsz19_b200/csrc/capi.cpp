@@ -126,6 +126,7 @@ astra_status astra_step_bwd(astra_cell c, const void* dy, const float* dhT, cons
   return guard([&] {
     NEED(c);
     ASTRA_CHECK_STATE(!c->c->lm_mode, "step_bwd: cell is owned by an LM");
+    if (c->c->peer) c->c->peer->begin_step();
     c->c->backward(dy, dhT, dcT, dx, dh0, dc0);
   });
 }
@@ -211,13 +212,67 @@ astra_status astra_comm_init(astra_cell c, const void* uid, int rank, int world)
     cc.nccl_comm = comm;
     cc.rank = rank;
     cc.world = world;
-    if (!cc.comm_st) {   // no caller comm stream: own a high-priority one so buckets overlap compute
-      int lo = 0, hi = 0;
-      CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-      CUDA_TRY(cudaStreamCreateWithPriority(&cc.own_comm_st, cudaStreamNonBlocking, hi));
-      cc.comm_st = cc.own_comm_st;
-    }
+    ASTRA_CHECK_ARG(!cc.peer || !cc.peer->ready || cc.peer->world == world, "comm_init: world differs from the peer backend's");
+    cc.ensure_comm_stream();
     if (!cc.tune_dev) CUDA_TRY(cudaMalloc(&cc.tune_dev, 64 * sizeof(double)));
+  });
+}
+
+// K11p (SURVEY §8(e) backend 2): the peer-memory window is the flat params / grads vector that
+// SGD updates — the cell's, or the LM's when the cell belongs to one.
+static void peer_export(std::vector<Cell*> cells, float* P, float* G, size_t n, void* out, size_t len) {
+  Cell& c0 = *cells[0];
+  if (!c0.peer) {
+    auto pc = std::make_shared<PeerComm>(c0.d.device, P, G, n);
+    for (Cell* c : cells) c->peer = pc;
+  }
+  ASTRA_CHECK_STATE(c0.peer->P == P && c0.peer->G == G, "comm_peer_handle: rebound since the peer window was made");
+  c0.peer->export_handle(out, len);
+}
+
+static void peer_init(std::vector<Cell*> cells, const void* handles, int rank, int world) {
+  Cell& c0 = *cells[0];
+  ASTRA_CHECK_STATE(c0.peer, "comm_peer_init: call comm_peer_handle first (and exchange the handles)");
+  for (Cell* c : cells)
+    ASTRA_CHECK_ARG(!c->nccl_comm || c->world == world, "comm_peer_init: world differs from the NCCL communicator's");
+  c0.peer->import_handles(handles, rank, world);
+  for (Cell* c : cells) {
+    c->rank = rank;
+    c->world = world;
+    c->ensure_comm_stream();
+  }
+}
+
+astra_status astra_comm_peer_handle(astra_cell c, void* out, size_t len) {
+  return guard([&] {
+    NEED(c); NEED(out);
+    Cell& cc = *c->c;
+    ASTRA_CHECK_STATE(cc.bound && !cc.lm_mode, "comm_peer_handle: cell not bound, or owned by an LM (use the lm_ form)");
+    peer_export({&cc}, cc.P, cc.G, cc.n_params, out, len);
+  });
+}
+
+astra_status astra_comm_peer_init(astra_cell c, const void* handles, int rank, int world) {
+  return guard([&] {
+    NEED(c);
+    ASTRA_CHECK_STATE(!c->c->lm_mode, "comm_peer_init: cell owned by an LM (use the lm_ form)");
+    peer_init({c->c.get()}, handles, rank, world);
+  });
+}
+
+astra_status astra_lm_comm_peer_handle(astra_lm m, void* out, size_t len) {
+  return guard([&] {
+    NEED(m); NEED(out);
+    LM& lm = *m->m;
+    ASTRA_CHECK_STATE(lm.bound, "lm_comm_peer_handle: not bound");
+    peer_export(lm.layers, lm.P, lm.G, lm.n_params, out, len);
+  });
+}
+
+astra_status astra_lm_comm_peer_init(astra_lm m, const void* handles, int rank, int world) {
+  return guard([&] {
+    NEED(m);
+    peer_init(m->m->layers, handles, rank, world);
   });
 }
 

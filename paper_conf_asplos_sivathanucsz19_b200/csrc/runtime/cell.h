@@ -21,6 +21,7 @@
 #include "../kernels/gemm.h"
 #include "../kernels/kernels.h"
 #include "../tuner/tuner.h"
+#include "peer.h"
 
 namespace astra {
 
@@ -132,6 +133,11 @@ class Cell {
   // NCCL
   void* nccl_comm = nullptr;
   int rank = 0, world = 1;
+  // K11p: deterministic peer-memory gradient sum + fused SGD / all-gather (SURVEY §8(e) backend
+  // 2).  When set (world > 1), grad_bucket() launches the rank-ordered reduce instead of NCCL and
+  // SGD is the owned-shard update written to every rank.  Shared by the layers of one LM.
+  std::shared_ptr<PeerComm> peer;
+  void ensure_comm_stream();
 
   // LM mode hooks (set by LM)
   bool lm_mode = false;

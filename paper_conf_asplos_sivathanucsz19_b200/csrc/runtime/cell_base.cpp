@@ -214,12 +214,18 @@ void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz
 // work; grad_join() makes `main` wait for every bucket before SGD.  Sum then ×1/world: the mean
 // of the shard-mean gradients = the full-batch mean gradient (oracle/dp.py).
 void Cell::grad_bucket(float* p, size_t n, cudaStream_t producer) {
-  if (world <= 1 || !nccl_comm || n == 0) return;
+  if (world <= 1 || (!nccl_comm && !peer) || n == 0) return;
   cudaStream_t cs = comm_st ? comm_st : producer;
   cudaEvent_t evb = ev_bucket[bucket_i++ % 4];
   if (cs != producer) {
     CUDA_TRY(cudaEventRecord(evb, producer));
     CUDA_TRY(cudaStreamWaitEvent(cs, evb, 0));
+  }
+  if (peer) {   // K11p: rank-ordered mean of our shard of the bucket, read over NVLink
+    ASTRA_CHECK_STATE(p >= peer->G && p + n <= peer->G + peer->n, "grad_bucket: bucket outside the peer window");
+    peer->reduce((size_t)(p - peer->G), n, cs);
+    sync_pending = true;
+    return;
   }
   ncclResult_t r = ncclAllReduce(p, p, n, ncclFloat, ncclSum, (ncclComm_t)nccl_comm, cs);
   if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclAllReduce: ") + ncclGetErrorString(r));
@@ -239,7 +245,21 @@ void Cell::grad_join(cudaStream_t main) {
 
 void Cell::sgd_step(float lr) {
   ASTRA_CHECK_STATE(bound, "sgd: not bound");
+  if (peer && world > 1) {   // owned shards updated, written into every rank's parameters
+    std::vector<std::pair<size_t, size_t>> cover;
+    for (const ParamInfo& q : params) cover.push_back({q.offset, (size_t)q.rows * q.cols});
+    peer->sgd(lr, main_st, cover);
+    return;
+  }
   sgd(P, G, n_params, lr, main_st);
+}
+
+void Cell::ensure_comm_stream() {
+  if (comm_st) return;   // no caller comm stream: own a high-priority one so buckets overlap compute
+  int lo = 0, hi = 0;
+  CUDA_TRY(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+  CUDA_TRY(cudaStreamCreateWithPriority(&own_comm_st, cudaStreamNonBlocking, hi));
+  comm_st = own_comm_st;
 }
 
 // ------------------------------------------------------------------------ tuner glue
@@ -372,6 +392,8 @@ static float elapsed(cudaEvent_t a, cudaEvent_t b) {
 // P:457).  Only the measured steps synchronise on their own end event.
 int Cell::tune_next() {
   if (tune_mode != ASTRA_TUNE_ON) return tune_mode == ASTRA_TUNE_FROZEN ? ASTRA_TUNE_CONVERGED : ASTRA_TUNE_IDLE;
+  ASTRA_CHECK_STATE(world <= 1 || nccl_comm,
+                    "tune_next: exploring with world > 1 needs astra_comm_init (cross-rank decisions, reading R29)");
   if (!wirer) tuner_setup();
   if (wirer->converged()) return ASTRA_TUNE_CONVERGED;
   if (rep_i == 0) {  // warm-up step done

@@ -329,6 +329,7 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   for (int k = 0; k < nch; ++k) t_end[k] = (int)((long)(k + 1) * c.T / nch) - 1;
 
   for (Cell* L : layers) L->mark(R_STEP, 0, st);
+  if (c.peer) c.peer->begin_step();
   // layer wavefront (AV lwf of the top layer): layer l runs on its own stream, time chunk by time
   // chunk; chunk k of layer l starts when layer l-1 finished chunk k (forward) / layer l+1 produced
   // the dX rows of chunk k (backward).  Row chunks of the same GEMMs, the chains unchanged: the
@@ -501,7 +502,15 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   c0.grad_bucket(G + find("E"), (size_t)V * c0.I, st);
   if (ov) CUDA_TRY(cudaStreamWaitEvent(st, ev_hdone, 0));   // head gradients (and their bucket) done
   for (Cell* L : layers) L->grad_join(st);
-  if (do_sgd) sgd(P, G, n_params, lr, st);
+  if (do_sgd) {
+    if (c.peer && c.world > 1) {   // K11p: owned shards updated and all-gathered into every rank
+      std::vector<std::pair<size_t, size_t>> cover;
+      for (const ParamInfo& q : params) cover.push_back({q.offset, (size_t)q.rows * q.cols});
+      c.peer->sgd(lr, st, cover);
+    } else {
+      sgd(P, G, n_params, lr, st);
+    }
+  }
   for (Cell* L : layers) L->mark(R_STEP, 1, st);
 }
 

@@ -86,6 +86,12 @@ def test_bad_arguments_are_rejected():
     assert L.astra_tune_mode(c.h, 2, b"a1=256.8.2") == 1
     assert L.astra_tune_mode(c.h, 2, b"nonsense=1") == 1
     assert L.astra_status_string(4) == b"ASTRA_E_CUDA"
+    # peer-memory backend (K11p): handle before bind, init before handle, short buffer, null handles
+    buf = ctypes.create_string_buffer(256)
+    assert L.astra_comm_peer_handle(c.h, buf, 256) == 3                        # E_STATE: not bound
+    assert L.astra_comm_peer_init(c.h, buf, 0, 2) == 3                          # E_STATE: no handle yet
+    assert L.astra_comm_peer_handle(c.h, buf, 16) in (1, 3)
+    assert L.astra_comm_peer_handle(c.h, None, 256) == 1                        # E_ARG: null buffer
 
 
 def test_tune_report_is_json():

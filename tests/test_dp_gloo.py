@@ -48,3 +48,46 @@ def test_gloo_world2_dp_mean_equals_full_batch():
         pr.join(120)
         assert pr.exitcode == 0
     assert q.get(timeout=5) < 1e-12
+
+
+class _FakeWindow:
+    """Stands in for a Cell / LM: the handle exchange of the peer-memory backend is host logic."""
+
+    def __init__(self, rank):
+        self.rank = rank
+        self.got = None
+
+    def comm_peer_handle(self):
+        return bytes([self.rank + 1]) * 256
+
+    def comm_peer_init(self, handles, rank, world):
+        self.got = (handles, rank, world)
+
+
+def _peer_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    w = _FakeWindow(rank)
+    A.peer_exchange(w)
+    handles, r, n = w.got
+    q.put((rank, r, n, handles == b"".join(bytes([k + 1]) * 256 for k in range(world))))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gloo_world2_peer_handle_exchange_is_rank_ordered():
+    """K11p host plumbing (SURVEY §8(e) backend 2): every rank receives all window handles in rank
+    order and maps them with its own rank and the world size."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29500 + (os.getpid() + 7) % 1000
+    procs = [ctx.Process(target=_peer_worker, args=(r, 2, port, q)) for r in range(2)]
+    for pr in procs:
+        pr.start()
+    for pr in procs:
+        pr.join(120)
+        assert pr.exitcode == 0
+    got = sorted(q.get(timeout=5) for _ in range(2))
+    assert got == [(0, 0, 2, True), (1, 1, 2, True)]
