@@ -52,6 +52,8 @@ struct Variant {
   int lwf = 0;          // stacked LM: layer wavefront in WF_CHUNKS[lwf] time chunks (1 = layers one after the other)
   int head_ov = 0;      // LM head overlapped with the forward chain in HEAD_CHUNKS[head_ov] time chunks (B3)
   int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
+  int recomp = 0;       // alloc fork: 1 = the recurrent projection UH_t is not
+                        // kept for BPTT but recomputed there from the saved h_{t-1} operands (same bits)
   Variant() { g[G_BPTT].bn = 128; }
   std::string str() const;                    // "a1=256.1.1,rec=...,wg_side=0"
   static Variant parse(const std::string& s); // inverse of str(); throws ASTRA_E_ARG
@@ -164,6 +166,7 @@ class Cell {
   virtual int c_width() const { return H; }      // width of the second state (c or s); 0 = none
   virtual bool lm_capable() const { return true; }
   virtual bool chain_prefetch() const { return false; }   // supports Variant::l2pf (tuner AVs pf_fwd / pf_bwd)
+  virtual bool supports_recompute() const { return false; }   // Variant::recomp (tuner root fork "recomp")
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
   virtual int bwd_fusions() const { return 1; }   // number of K4 fusion choices (tuner AV "fuse_bwd")
   virtual void role_shape(int role, int& M, int& N) const = 0;

@@ -23,6 +23,7 @@ std::string Variant::str() const {
   }
   o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf << ",hov=" << head_ov;
   if (lwf) o << ",lwf=" << lwf;
+  if (recomp) o << ",rc=" << recomp;
   return o.str();
 }
 
@@ -41,6 +42,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "wg_side") {
       v.wg_side = std::stoi(val);
       ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    if (k == "rc") {
+      v.recomp = std::stoi(val);
+      ASTRA_CHECK_ARG(v.recomp == 0 || v.recomp == 1, "variant: rc must be 0 (store UH) or 1 (recompute UH in BPTT)");
       continue;
     }
     if (k == "lwf") {
@@ -348,6 +354,10 @@ void Cell::tuner_setup() {
   if (lm_mode && lm_role == 2 && lm_layers > 1 && lm_wavefront && T >= 2)
     t = "(pre " + t + " (leaf lwf " + std::to_string(T > 5 ? 3 : 2) + " t_step))";
   if (t.empty()) t = "(leaf none 1 t_step)";
+  // SURVEY §8(f) rank 4 / §8(a.9) `alloc`: store-vs-recompute of the recurrent projection is a
+  // memory-allocation context: the whole tree is explored under each context, then
+  // each context's best configuration is raced end to end, 3 steps each
+  if (ot == OT::BF16 && supports_recompute()) t = "(fork (leaf recomp 2 t_step) t_step " + t + " 3)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
   wirer.reset(new tuner::Wirer(tree.get()));
   wirer->index().bucket = T;
@@ -368,6 +378,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "fuse_bwd") { v.bwd_mode = o; continue; }
     if (n == "head_ov") { v.head_ov = o; continue; }
     if (n == "lwf") { v.lwf = o; continue; }
+    if (n == "recomp") { v.recomp = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

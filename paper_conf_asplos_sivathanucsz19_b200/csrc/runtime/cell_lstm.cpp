@@ -7,6 +7,8 @@
 //   bwd : for t desc: dh_rec = D_uh[t+1]·Uᵀ (K1) ; pointwise cell backward (K4 half, K5 partials)
 //         → dh0 → wgrad dU = Hᵀ·D_uh, dW = Xᵀ·D_wx (K1) → dX = D_wx·Wᵀ (K1) → bias/α/β reductions (K5)
 //         → gradient sum over ranks (K11) when world > 1.
+#include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "../kernels/cell_math.cuh"
@@ -19,7 +21,9 @@ class LstmCell : public Cell {
  public:
   int kind, NG, nchunk;
   size_t off_X, off_WX, off_UH, off_C, off_H, off_Wm, off_Um;
-  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part, off_flags;
+  size_t off_Duh, off_Dwx, off_dH, off_dC, off_part, off_flags, off_UHr;
+  int rc_steps = 1;   // recompute variant: timesteps per recomputed UH chunk (ring of 2 chunks)
+  cudaEvent_t ev_rc_done[2] = {nullptr, nullptr}, ev_rc_free[2] = {nullptr, nullptr};
 
   explicit LstmCell(const astra_cell_desc& dd) : Cell(dd) {
     kind = d.cell_type == ASTRA_MILSTM ? K_MILSTM : d.cell_type == ASTRA_SUBLSTM ? K_SUBLSTM : K_LSTM;
@@ -52,8 +56,20 @@ class LstmCell : public Cell {
     off_dC = c.take((size_t)B * Hp * 4);
     off_part = c.take((size_t)nchunk * 4 * NG * 4);
     off_flags = c.take(4096);
+    // recompute variant (Variant::recomp): a ring of two UH chunks of rc_steps timesteps each, sized
+    // so the ring stays L2-resident next to U (the forward writes UH_t into slot 0 of the ring)
+    rc_steps = (int)std::max<long>(1, std::min<long>(T, (32L << 20) / ((long)B * NG * 4)));
+    if (const char* ev = std::getenv("ASTRA_RC_STEPS")) rc_steps = std::max(1, std::min(T, std::atoi(ev)));   // tests
+    off_UHr = c.take((size_t)2 * rc_steps * B * NG * 4);
     scratch_bytes = c.o;
   }
+  ~LstmCell() override {
+    for (int i = 0; i < 2; ++i) {
+      if (ev_rc_done[i]) cudaEventDestroy(ev_rc_done[i]);
+      if (ev_rc_free[i]) cudaEventDestroy(ev_rc_free[i]);
+    }
+  }
+  bool supports_recompute() const override { return true; }
 
   // Fixed split-K of the per-step BPTT GEMM (K = 4·Hp): with B rows the GEMM has few output tiles,
   // so each SM would stream a whole K-panel of Uᵀ; four K-chunks cut the bytes per SM 4× while the
@@ -203,7 +219,8 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     }
   } else {
     for (int t = t0; t < t1; ++t) {
-      float* UHt = UH + (long)t * B * NG;
+      // recompute variant: UH_t is consumed by this step's pointwise kernel only (one L2-resident slot)
+      float* UHt = var.recomp ? sc<float>(off_UHr) : UH + (long)t * B * NG;
       L2Pf pf{};   // R31: WX_t, read by this step's pointwise kernel
       pf.p[0] = WX + (long)t * B * NG; pf.n[0] = (var.l2pf & 1) ? (unsigned long long)B * NG * 4 : 0;
       run_gemm(1, rec, epi(UHt, NG, B, NG), t, 0, var.g[G_REC], st, &pf);
@@ -291,7 +308,59 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     fa.gp = gp;
     fa.D_uh = Duh; fa.D_wx = Dwx; fa.dc = dC; fa.partials = part;
   }
+  // Recompute variant: UH_t = h_{t-1}·U is rebuilt here from the saved bf16
+  // h operands — the forward's GEMM on the same operands in the same K order, so the same bits
+  // (R1, R7).  Chunks of rc_steps timesteps into a two-slot ring, computed on a side stream one
+  // chunk ahead of the BPTT chain (the fused BPTT kernel reads UH through its tensor map: there
+  // the whole range is recomputed into the UH array up front).
+  const bool rc = var.recomp != 0;
+  const int RC = rc_steps;
+  float* UHr = sc<float>(off_UHr);
+  cudaStream_t rs = st;
+  if (rc && !fuse && !side.empty()) rs = side[0];
+  if (rc && !ev_rc_done[0])
+    for (int i = 0; i < 2; ++i) {
+      CUDA_TRY(cudaEventCreateWithFlags(&ev_rc_done[i], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&ev_rc_free[i], cudaEventDisableTiming));
+    }
+  auto recompute = [&](int ta, int tb, float* dst, cudaStream_t s2, int id) {   // UH rows of steps [ta, tb)
+    GemmSpec r = GemmSpec();
+    r.A = mat(Hrow(ta), Hp, (long)(tb - ta) * B, Hp);
+    r.B = mat(Um, Hp, NG, Hp);
+    r.M = (tb - ta) * B; r.N = NG; r.K = Hp;
+    run_gemm(id, r, epi(dst, NG, r.M, NG), 0, 0, var.g[G_REC], s2);
+  };
+  const int kb = t0 / RC;
+  bool released[2] = {false, false};   // slot freed by the chain in this call (else free since the fork)
+  auto chunk_lo = [&](int k) { return std::max(t0, k * RC); };
+  auto chunk_hi = [&](int k) { return std::min(t1, (k + 1) * RC); };
+  auto issue = [&](int k) {   // chunk k into ring slot k & 1, after the chain released that slot
+    if (k < kb) return;
+    const int sl = k & 1;
+    if (rs != st && released[sl]) CUDA_TRY(cudaStreamWaitEvent(rs, ev_rc_free[sl], 0));
+    const int lo = chunk_lo(k), hi = chunk_hi(k);
+    // GEMM id unique per row range: the prepared tensor maps are cached per id (and carry pointers)
+    recompute(lo, hi, UHr + ((size_t)sl * RC + (lo - k * RC)) * B * NG, rs, 7000000 + lo * 1024 + (hi - lo));
+    if (rs != st) CUDA_TRY(cudaEventRecord(ev_rc_done[sl], rs));
+  };
+  auto uh_of = [&](int t) -> float* {
+    if (!rc || fuse) return UH + (long)t * B * NG;
+    const int k = t / RC;
+    return UHr + ((size_t)(k & 1) * RC + (t - k * RC)) * B * NG;
+  };
+  if (rc && fuse) {
+    recompute(t0, t1, UH + (long)t0 * B * NG, st, 8000000 + t0 * 1024 + (t1 - t0));
+  } else if (rc) {
+    if (rs != st) {   // the side stream starts after everything enqueued so far (h operands, Um mirror)
+      CUDA_TRY(cudaEventRecord(ev_fork, st));
+      CUDA_TRY(cudaStreamWaitEvent(rs, ev_fork, 0));
+    }
+    issue((t1 - 1) / RC);
+    issue((t1 - 1) / RC - 1);
+  }
   for (int t = t1 - 1; t >= t0; --t) {
+    const int kc = t / RC;
+    if (rc && !fuse && rs != st && t == chunk_hi(kc) - 1) CUDA_TRY(cudaStreamWaitEvent(st, ev_rc_done[kc & 1], 0));
     if (fuse && t < T - 1) {
       fa.t = t;
       lstm_bptt_fused_launch(kind, !lm_dy, bm, fa, st);
@@ -315,7 +384,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
       L2Pf pf{};
       if (var.l2pf & 2) {
         pf.p[0] = WX + (long)t * B * NG; pf.n[0] = (unsigned long long)B * NG * 4;
-        pf.p[1] = UH + (long)t * B * NG; pf.n[1] = (unsigned long long)B * NG * 4;
+        pf.p[1] = uh_of(t); pf.n[1] = (unsigned long long)B * NG * 4;
         pf.p[2] = Cb + (long)t * B * Hp; pf.n[2] = (unsigned long long)2 * B * Hp * 4;
         pf.p[3] = dyt; pf.n[3] = (unsigned long long)B * ldy * (dyf32 ? 4 : esz());
       }
@@ -325,8 +394,13 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
       nsplit = bp.ksplit;
     }
     lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC, WX + (long)t * B * NG,
-                       UH + (long)t * B * NG, Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
+                       uh_of(t), Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
                        Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
+    if (rc && !fuse && t == chunk_lo(kc)) {   // chunk kc consumed: its slot takes chunk kc - 2
+      if (rs != st) CUDA_TRY(cudaEventRecord(ev_rc_free[kc & 1], st));
+      released[kc & 1] = true;
+      issue(kc - 2);
+    }
   }
   auto dx_rows = [&](int r0, int r1, int id) {   // dX = D_wx·Wᵀ for timesteps [r0, r1) (row chunk: same bits)
     const long rows = (long)(r1 - r0) * B;

@@ -97,6 +97,26 @@ def test_fused_bwd_bitwise(cell, T, B, H):
     _check(cell, T, B, I, H, "bf16", 91, TOL_BF16, variant="bwd=1")
 
 
+@pytest.mark.parametrize("cell", ["lstm", "milstm", "sublstm"])
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_recompute_bitwise_and_parity(cell, dtype, tol, monkeypatch):
+    """Recompute-vs-store fork: UH recomputed in BPTT from the saved h operands
+    in 2-step chunks (the ring wraps at T = 6) — the same bits as the stored UH, and oracle parity."""
+    monkeypatch.setenv("ASTRA_RC_STEPS", "2")
+    T, B, I, H = 6, 72, 64, 96
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, 78, bf16=dtype == "bf16")
+    ref = None
+    for v in ("rc=0", "rc=1", "rc=1,wg_side=1"):
+        out, g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, v)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    _check(cell, T, B, I, H, dtype, 78, tol, variant="rc=1")
+
+
 def test_variants_bitwise():
     """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
     T, B, I, H = 6, 160, 128, 192

@@ -221,3 +221,45 @@ def test_profiling_switch():
         with pytest.raises(A.AstraError):
             c.set_profiling(False)
     assert torch.equal(out[0], out[1])
+
+
+@pytest.mark.parametrize("variant", ["rc=1", "rc=1,fwd=1", "rc=1,fwd=2", "rc=1,bwd=1", "rc=1,wg_side=1,hov=1"])
+def test_recompute_lm_bitwise(variant, monkeypatch):
+    """SURVEY §8(f) rank 4, the alloc fork: recomputing UH_t = h_{t-1}·U in BPTT (ring of 2-step
+    chunks on a side stream, 3 chunks at T = 5 so the ring wraps) gives the same bits as storing it,
+    over 8 SGD steps, with every forward / backward fusion choice and under graph replay."""
+    monkeypatch.setenv("ASTRA_RC_STEPS", "2")
+    pa, la = _steps_params("fwd=0", graph=True)
+    pb, lb = _steps_params(variant, graph=True)
+    assert torch.equal(pa, pb) and la == lb
+    if variant == "rc=1":
+        pc, lc = _steps_params(variant, graph=False)
+        assert torch.equal(pa, pc) and la == lc
+
+
+def test_tuner_fork_explores_both_allocation_contexts():
+    """The live update tree's root is the hierarchical alloc fork: both contexts are
+    explored and raced end to end; the run stays bitwise equal to the default."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 4, 64, 64, 64, 40
+    res = []
+    n_steps = 600
+    for mode in (A.TUNE_ON, A.TUNE_OFF):
+        p, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, synth.config_seed(5) + 60, True)
+        c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+        m = A.LM(c, V)
+        m.load(p)
+        c.tune_mode(mode)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        seen = set()
+        for i in range(n_steps):
+            m.train_step(tokens, 0.05)
+            seen.add("rc=1" in c.tune_report()["variant"])
+            if c.tune_next() == A.TUNE_CONVERGED:
+                n_steps = i + 1
+                break
+        torch.cuda.synchronize()
+        res.append((m.params.clone(), seen))
+    assert n_steps < 600, "the tuner did not converge"
+    assert torch.equal(res[0][0], res[1][0])
+    assert res[0][1] == {False, True}, "the recompute context was never explored"
