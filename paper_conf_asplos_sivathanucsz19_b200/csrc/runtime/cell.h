@@ -52,6 +52,7 @@ struct Variant {
   int lwf = 0;          // stacked LM: layer wavefront in WF_CHUNKS[lwf] time chunks (1 = layers one after the other)
   int head_ov = 0;      // LM head overlapped with the forward chain in HEAD_CHUNKS[head_ov] time chunks (B3)
   int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
+  int dpb = 0;          // K11p bucket cap (§8(a.9) dp_bucket): 0 whole tensors, 1/2/3 = 128/32/8 MB pieces
   int recomp = 0;       // alloc fork: 1 = the recurrent projection UH_t is not
                         // kept for BPTT but recomputed there from the saved h_{t-1} operands (same bits)
   Variant() { g[G_BPTT].bn = 128; }

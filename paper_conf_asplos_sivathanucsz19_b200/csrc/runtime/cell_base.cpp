@@ -1,6 +1,7 @@
 // L1 runtime, shared machinery of every cell family: parameters, binding, workspace, the GEMM
 // dispatch (tcgen05 for the bf16 path, SIMT for the fp32 path), cudaEvent-pair profiling regions
 // (P:286-288), the tuner glue (L2) and the DP gradient sum (K11).
+#include <cstdlib>
 #include <nccl.h>
 
 #include <algorithm>
@@ -24,6 +25,7 @@ std::string Variant::str() const {
   o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf << ",hov=" << head_ov;
   if (lwf) o << ",lwf=" << lwf;
   if (recomp) o << ",rc=" << recomp;
+  if (dpb) o << ",dpb=" << dpb;
   return o.str();
 }
 
@@ -42,6 +44,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "wg_side") {
       v.wg_side = std::stoi(val);
       ASTRA_CHECK_ARG(v.wg_side == 0 || v.wg_side == 1, "variant: wg_side must be 0 or 1");
+      continue;
+    }
+    if (k == "dpb") {
+      v.dpb = std::stoi(val);
+      ASTRA_CHECK_ARG(v.dpb >= 0 && v.dpb <= 3, "variant: dpb must be 0..3 (whole tensors, 128, 32 or 8 MB buckets)");
       continue;
     }
     if (k == "rc") {
@@ -229,7 +236,17 @@ void Cell::grad_bucket(float* p, size_t n, cudaStream_t producer) {
   }
   if (peer) {   // K11p: rank-ordered mean of our shard of the bucket, read over NVLink
     ASTRA_CHECK_STATE(p >= peer->G && p + n <= peer->G + peer->n, "grad_bucket: bucket outside the peer window");
-    peer->reduce((size_t)(p - peer->G), n, cs);
+    // AV dp_bucket: pieces of at most 128 / 32 / 8 MB (value-neutral: the sum is per element);
+    // ASTRA_DPB_DIV shrinks the caps for tests of the splitting on small models
+    static const size_t div = [] {
+      const char* e = std::getenv("ASTRA_DPB_DIV");
+      return e ? std::max<size_t>(1, std::strtoull(e, nullptr, 10)) : 1;
+    }();
+    const size_t capb[4] = {0, 128u << 20, 32u << 20, 8u << 20};
+    // the dp_bucket AV lives on the top layer of an LM (its tree); every layer follows it
+    const int dpb = peer->dpb >= 0 ? peer->dpb : var.dpb;
+    const size_t cap = dpb > 0 ? std::max<size_t>(64, capb[dpb] / div / 4) : n;
+    for (size_t o = 0; o < n; o += cap) peer->reduce((size_t)(p - peer->G) + o, std::min(cap, n - o), cs);
     sync_pending = true;
     return;
   }
@@ -353,6 +370,10 @@ void Cell::tuner_setup() {
   // stacked LM (top layer): layer wavefront, against the whole step
   if (lm_mode && lm_role == 2 && lm_layers > 1 && lm_wavefront && T >= 2)
     t = "(pre " + t + " (leaf lwf " + std::to_string(T > 5 ? 3 : 2) + " t_step))";
+  // §8(a.9) dp_bucket: the gradient bucket size is a free variable only under the rank-ordered
+  // peer-memory sum (K11p: the bits do not depend on it); last in the prefix order, step metric
+  if (world > 1 && peer && peer->ready && (!lm_mode || lm_role == 2))
+    t = t.empty() ? "(leaf dp_bucket 4 t_step)" : "(pre " + t + " (leaf dp_bucket 4 t_step))";
   if (t.empty()) t = "(leaf none 1 t_step)";
   // SURVEY §8(f) rank 4 / §8(a.9) `alloc`: store-vs-recompute of the recurrent projection is a
   // memory-allocation context: the whole tree is explored under each context, then
@@ -379,6 +400,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "head_ov") { v.head_ov = o; continue; }
     if (n == "lwf") { v.lwf = o; continue; }
     if (n == "recomp") { v.recomp = o; continue; }
+    if (n == "dp_bucket") { v.dpb = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

@@ -329,7 +329,10 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   for (int k = 0; k < nch; ++k) t_end[k] = (int)((long)(k + 1) * c.T / nch) - 1;
 
   for (Cell* L : layers) L->mark(R_STEP, 0, st);
-  if (c.peer) c.peer->begin_step();
+  if (c.peer) {
+    c.peer->begin_step();
+    c.peer->dpb = c.var.dpb;   // the top layer's AV sizes every layer's buckets
+  }
   // layer wavefront (AV lwf of the top layer): layer l runs on its own stream, time chunk by time
   // chunk; chunk k of layer l starts when layer l-1 finished chunk k (forward) / layer l+1 produced
   // the dX rows of chunk k (backward).  Row chunks of the same GEMMs, the chains unchanged: the

@@ -25,6 +25,7 @@ class PeerComm {
   size_t n;   // window length in floats
   int rank = 0, world = 1;
   bool ready = false;
+  int dpb = -1;   // bucket cap choice of the LM's top layer (set per step by the LM); -1: the cell's own
 
   // ASTRA_PEER_HANDLE_BYTES of IPC handles + offsets of this rank's window and signal array
   void export_handle(void* out, size_t len) const;

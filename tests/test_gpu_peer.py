@@ -40,7 +40,7 @@ def _shard(a, r, world, axis=1):
     return np.ascontiguousarray(np.take(a, range(r * n, (r + 1) * n), axis=axis))
 
 
-def _worker(rank, world, port, kind, dtype, q):
+def _worker(rank, world, port, kind, dtype, q, variant=None):
     try:
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
@@ -54,6 +54,8 @@ def _worker(rank, world, port, kind, dtype, q):
             c = A.Cell("milstm", H, I, B // world, T, dtype=dtype)
             m = A.LM(c, V)
             m.load(p)
+            if variant:
+                c.tune_mode(A.TUNE_FROZEN, variant)
             A.peer_exchange(m)
             tokens = torch.as_tensor(_shard(tok, rank, world), dtype=torch.int32, device="cuda")
             losses = []
@@ -87,11 +89,11 @@ def _worker(rank, world, port, kind, dtype, q):
         raise
 
 
-def _run_world(kind, dtype, world=2):
+def _run_world(kind, dtype, world=2, variant=None):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = 29650 + os.getpid() % 300
-    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, dtype, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, dtype, q, variant)) for r in range(world)]
     for pr in procs:
         pr.start()
     res = {}
@@ -130,9 +132,12 @@ def _reference_lm(dtype, world=2):
     return newp.cpu().numpy(), g.cpu().numpy(), [m.grads.cpu().numpy() for m in ms], p, tok
 
 
-@pytest.mark.parametrize("dtype", ["fp32", "bf16"])
-def test_peer_lm_bitwise_equals_rank_ordered_mean(dtype):
-    res = _run_world("lm", dtype)
+@pytest.mark.parametrize("dtype,variant", [("fp32", None), ("bf16", None), ("fp32", "dpb=2"), ("bf16", "dpb=3")])
+def test_peer_lm_bitwise_equals_rank_ordered_mean(dtype, variant, monkeypatch):
+    """dpb = 2 / 3 (AV dp_bucket) cut the buckets into 32 / 8 KB pieces here (ASTRA_DPB_DIV = 1024):
+    the bits do not move (the per-element rank-ordered sum does not see bucket boundaries)."""
+    monkeypatch.setenv("ASTRA_DPB_DIV", "1024")
+    res = _run_world("lm", dtype, variant=variant)
     p_ref, g_ref, g_shards, p0, tok = _reference_lm(dtype)
     for r, (pp, gg, losses) in res.items():
         assert np.array_equal(pp, p_ref), f"rank {r}: parameters differ from the rank-ordered mean SGD"
