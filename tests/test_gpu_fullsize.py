@@ -1,0 +1,113 @@
+"""Parity at BASELINE.json's FULL sizes (SURVEY §8(c.8) parity protocol, last rung; §8(c.9)).
+
+cfg2 (SCRN word LM), cfg3 (RHN L=10 LM) and cfg4 (LSTM + attention) are small enough for the fp64
+oracle to run whole: every loss / output / gradient is compared.  cfg5 (MI-LSTM, T=100, B=512,
+H=I=2048) is not (the fp64 step over 512 sequences takes ~10 min), so it runs at full size in the
+bench's launch configuration (its converged variant) with SAMPLED outputs the oracle can compute:
+sequences are independent, so the outputs y / hT / cT and the input gradients dx / dh0 / dc0 of a
+few sampled sequences are those of the oracle run on just those sequences; and with the upstream
+gradients of every other sequence set to zero, their contributions to the weight gradients are
+exactly zero, so the full-batch weight gradients equal the oracle's over the sampled sequences.
+Tolerance: BASELINE north_star, 2e-2 relative (bf16 operands, fp32 accumulate; reading R18).
+"""
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import cells as C
+from oracle import lm as OLM
+
+from helpers import TOL_BF16, bf16_round, cell_shapes, make_cell_case, rel_err
+
+pytestmark = pytest.mark.gpu
+
+# the variant bench.py's tuner converges to at cfg5 (bench line "tuner.variant", profiles/)
+BENCH_VARIANT = ("a1=256.1.1.2,rec=256.1.1.2,bptt=256.1.1.2,du=256.1.1.2,dw=256.1.1.2,dx=256.1.1.2,"
+                 "head=256.1.1,wg_side=1,fwd=0,bwd=0")
+
+
+def test_cfg5_full_size_sampled_sequences():
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H = 100, 512, 2048, 2048
+    S = [0, 257, 511]                      # first, ragged-middle and last sequence of the batch
+    seed = synth.config_seed(5) + 100
+    p, inp, dY, dhT, dcT = make_cell_case("milstm", T, B, I, H, seed, bf16=True)
+    mask = np.zeros(B, bool)
+    mask[S] = True
+    dY[:, ~mask, :] = 0.0
+    dhT[~mask] = 0.0
+    dcT[~mask] = 0.0
+    c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+    c.tune_mode(A.TUNE_FROZEN, BENCH_VARIANT)
+    c.load(p)
+    dev = c.device
+    bf = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev).to(torch.bfloat16).contiguous()
+    f32 = lambda a: torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    y = torch.empty(T, B, H, dtype=torch.bfloat16, device=dev)
+    hT, cT = torch.empty(B, H, device=dev), torch.empty(B, H, device=dev)
+    dx = torch.empty(T, B, I, dtype=torch.bfloat16, device=dev)
+    dh0, dc0 = torch.empty(B, H, device=dev), torch.empty(B, H, device=dev)
+    c.forward(bf(inp["x"]), f32(inp["h0"]), f32(inp["c0"]), y, hT, cT)
+    c.backward(bf(dY), f32(dhT), f32(dcT), dx, dh0, dc0)
+    torch.cuda.synchronize()
+    got = {"y": y.float().cpu().numpy()[:, S], "hT": hT.cpu().numpy()[S], "cT": cT.cpu().numpy()[S],
+           "dx": dx.float().cpu().numpy()[:, S], "dh0": dh0.cpu().numpy()[S], "dc0": dc0.cpu().numpy()[S]}
+    for k in p:
+        got[k] = c.view(k, c.grads).cpu().numpy().reshape(np.shape(p[k]))
+    sub = {"x": inp["x"][:, S], "h0": inp["h0"][S], "c0": inp["c0"][S]}
+    out_o, g_o = C.cell_fwd_bwd("milstm", p, sub, dY[:, S], dhT[S], dcT[S])
+    ref = {**out_o, **g_o}
+    errs = {k: rel_err(got[k], ref[k]) for k in ref if k in got}
+    assert set(errs) >= {"y", "hT", "cT", "dx", "dh0", "dc0", "W", "U", "b", "alpha", "beta1", "beta2"}, errs.keys()
+    bad = {k: v for k, v in errs.items() if not v <= TOL_BF16}
+    assert not bad, (bad, errs)
+
+
+def _lm_full(cell, T, B, I, H, V, seed, cell_kw, oracle_kw, S=None, L=None):
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    shapes = cell_shapes(cell, I, H, S, L)
+    Hout = H + S if cell == "scrn" else H
+    shapes.update({"E": (V, I), "W_o": (Hout, V), "b_o": (V,)})
+    p = synth.weights(seed, shapes, H)
+    if cell == "rhn":   # the benchmark's T-gate bias b_T = -2: b_ℓ = [b_H | b_T]
+        p["b"] = p["b"].copy()
+        p["b"][:, H:] = -2.0
+    for k in ("A", "Bm", "P", "R", "W", "E", "W_o"):
+        if k in p:
+            p[k] = bf16_round(p[k])
+    tok = synth.zipf_tokens(seed, "tok", (T + 1, B), V, None)
+    h0 = synth.uniform(seed, "h0", (B, H), -0.5, 0.5)
+    c0 = None if cell == "rhn" else synth.uniform(seed, "c0", (B, S if cell == "scrn" else H), -0.5, 0.5)
+    c = A.Cell(cell, H, I, B, T, dtype="bf16", **cell_kw)
+    m = A.LM(c, V)
+    m.load(p)
+    dev = c.device
+    f32 = lambda a: None if a is None else torch.as_tensor(np.asarray(a, dtype=np.float32), device=dev)
+    m.set_state(f32(h0), f32(c0))
+    loss = float(m.fwd_bwd(torch.as_tensor(tok, dtype=torch.int32, device=dev)).item())
+    torch.cuda.synchronize()
+    g = {k: m.view(k, m.grads).cpu().numpy().reshape(np.shape(p[k])) for k in p}
+    lo, go, _ = OLM.lm_forward_backward(cell, p, tok, h0, c0, **oracle_kw)
+    assert abs(loss - lo) / abs(lo) <= TOL_BF16, (loss, lo)
+    errs = {k: rel_err(g[k], go[k]) for k in go}
+    bad = {k: v for k, v in errs.items() if not v <= TOL_BF16}
+    assert not bad, (bad, errs)
+
+
+def test_cfg2_scrn_lm_full_size():
+    """cfg2: SC-RNN word LM, H = S = I = 1024, B = 64, T = 35, V = 10k (whole step vs the oracle)."""
+    alpha = np.float32(0.95).item()
+    _lm_full("scrn", 35, 64, 1024, 1024, 10000, synth.config_seed(2) + 100,
+             {"context": 1024, "scrn_alpha": 0.95}, {"alpha": alpha}, S=1024)
+
+
+def test_cfg3_rhn_lm_full_size():
+    """cfg3: RHN word LM, recurrence depth L = 10, H = I = 830, B = 64, T = 35, V = 10k."""
+    _lm_full("rhn", 35, 64, 830, 830, 10000, synth.config_seed(3) + 100, {"depth": 10}, {}, L=10)
+
+
+def test_cfg4_attention_full_size():
+    """cfg4: LSTM with attention, H = A = I = 1024, B = 128, Ts = Tt = 50 (cell API, whole step)."""
+    from test_gpu_cell import _attn_check
+    _attn_check(50, 50, 128, 1024, 1024, 1024, "bf16", synth.config_seed(4) + 100, TOL_BF16)
