@@ -252,6 +252,20 @@ astra_status astra_region_times(astra_cell c, double* out, int cap, int* n);
 /* Number of kernels this library has launched since load (all handles).                    */
 uint64_t astra_kernel_launch_count(void);
 
+/* ---- day-1 microbenchmarks: floors of the latency-bound chains.  Each call
+ *      enqueues its kernels on `stream` and returns; the caller times them with events. -------- */
+/* Read `bytes` (multiple of 16) of device memory `buf` `passes` times with 16-byte L2-cached
+ * loads from 4 CTAs per SM; sink: device float, written only for a sentinel sum (never in
+ * practice).  Bandwidth by size separates L2-resident from HBM streaming (the per-step
+ * weight-stream time of U / R_l).                                                            */
+astra_status astra_micro_stream_read(const void* buf, size_t bytes, int passes, float* sink, astra_stream stream);
+/* One CTA per SM runs `iters` grid-wide flag barriers (release add / acquire spin on *counter,
+ * a device unsigned the call zeroes first): the per-step floor of a persistent fused chain.   */
+astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream stream);
+/* n dependent empty kernels of `blocks` CTAs, launched with programmatic dependent launch
+ * (pdl = 1, as the chain kernels are) or plainly: the per-step floor of a launched chain.     */
+astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream stream);
+
 /* ---- host-only test hooks (no GPU) ------------------------------------------------------ */
 /* Drive the tuner's update tree on a fake clock.  `tree` is an s-expression, e.g.
  *   (par (exh g0 (leaf f0 3 g0) (leaf k0 2 g0)) (pre (leaf e0 2 ep0) (leaf e1 3 ep1)))

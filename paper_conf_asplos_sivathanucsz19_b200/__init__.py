@@ -81,6 +81,9 @@ _SIGS = {
     "astra_gemm_bf16": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I, _P],
     "astra_gemm_bf16_ex": [_I, _I, _I, _P, _I, ctypes.c_long, _P, _I, ctypes.c_long, _P, ctypes.c_long, _I, _I, _I,
                            _I, _I, _P],
+    "astra_micro_stream_read": [_P, _SZ, _I, _P, _P],
+    "astra_micro_grid_barrier": [_P, _I, _P],
+    "astra_micro_launch_chain": [_I, _I, _I, _P],
     "astra_status_string": [_I],
     "astra_last_error": [],
     "astra_kernel_launch_count": [],

@@ -18,6 +18,12 @@ void set_error(const std::string& s) { t_err = s; }
 
 using namespace astra;
 
+namespace astra {   // kernels/micro.cu
+void micro_stream_read(const void* buf, size_t bytes, int passes, float* sink, cudaStream_t st);
+void micro_grid_barrier(unsigned* counter, int iters, cudaStream_t st);
+void micro_launch_chain(int n, int pdl, int blocks, cudaStream_t st);
+}  // namespace astra
+
 struct astra_cell_s {
   std::unique_ptr<Cell> c;
 };
@@ -421,6 +427,18 @@ const char* astra_status_string(astra_status s) {
 const char* astra_last_error(void) { return t_err.c_str(); }
 
 uint64_t astra_kernel_launch_count(void) { return g_launches.load(); }
+
+astra_status astra_micro_stream_read(const void* buf, size_t bytes, int passes, float* sink, astra_stream stream) {
+  return guard([&] { micro_stream_read(buf, bytes, passes, sink, (cudaStream_t)stream); });
+}
+
+astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream stream) {
+  return guard([&] { micro_grid_barrier(counter, iters, (cudaStream_t)stream); });
+}
+
+astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream stream) {
+  return guard([&] { micro_launch_chain(n, pdl, blocks, (cudaStream_t)stream); });
+}
 
 astra_status astra_region_times(astra_cell c, double* out, int cap, int* n) {
   return guard([&] {

@@ -1,0 +1,85 @@
+// Day-1 microbenchmarks of SURVEY §8(d.4b): the floors of the latency-bound recurrent chains that
+// neither MEASURED_PEAKS.json nor the paper gives (§8(d.3) "chain latency ... against a measured
+// floor (an empty grid-barrier step plus the weight-stream time)").
+//   - streaming read of a buffer over `passes` passes: L2-resident vs HBM bandwidth by size (the
+//     per-step weight-stream time of U / R_ℓ);
+//   - a persistent one-CTA-per-SM kernel doing `iters` grid-wide flag barriers (the step floor of a
+//     persistent fused chain);
+//   - a chain of `n` dependent empty kernels launched as the library launches its chain kernels
+//     (with programmatic dependent launch, or without) — the step floor of a launched chain.
+#include "../common.h"
+#include "gemm.h"
+#include "pdl.cuh"
+
+namespace astra {
+
+namespace {
+
+__global__ void __launch_bounds__(512) stream_read_kernel(const float4* __restrict__ p, size_t n4, int passes,
+                                                          float* sink) {
+  float acc = 0.f;
+  const size_t tid = (size_t)blockIdx.x * blockDim.x + threadIdx.x, nth = (size_t)gridDim.x * blockDim.x;
+  for (int r = 0; r < passes; ++r)
+    for (size_t i = tid; i < n4; i += nth) {
+      const float4 v = __ldcg(p + i);
+      acc += v.x + v.y + v.z + v.w;
+    }
+  if (acc == 1.2345e-30f) *sink = acc;   // keeps the loads; never true for the benchmark's data
+}
+
+__device__ __forceinline__ void red_release_gpu(unsigned* p, unsigned v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// counter[0] is zeroed by the host; barrier k completes when it reaches (k + 1) · gridDim.x
+__global__ void grid_barrier_kernel(unsigned* counter, int iters) {
+  for (int k = 0; k < iters; ++k) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      red_release_gpu(counter, 1u);
+      const unsigned target = (unsigned)(k + 1) * gridDim.x;
+      while (ld_acquire_gpu(counter) < target) {
+      }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void empty_pdl_kernel(int) {
+  pdl_wait();
+  pdl_trigger();
+}
+
+__global__ void empty_kernel(int) {}
+
+}  // namespace
+
+void micro_stream_read(const void* buf, size_t bytes, int passes, float* sink, cudaStream_t st) {
+  const size_t n4 = bytes / 16;
+  ASTRA_CHECK_ARG(buf && n4 > 0 && passes > 0 && sink, "micro_stream_read: bad arguments");
+  stream_read_kernel<<<num_sms() * 4, 512, 0, st>>>(reinterpret_cast<const float4*>(buf), n4, passes, sink);
+  LAUNCH_CHECK();
+}
+
+void micro_grid_barrier(unsigned* counter, int iters, cudaStream_t st) {
+  ASTRA_CHECK_ARG(counter && iters > 0, "micro_grid_barrier: bad arguments");
+  CUDA_TRY(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
+  grid_barrier_kernel<<<num_sms(), 128, 0, st>>>(counter, iters);   // one CTA per SM: all co-resident
+  LAUNCH_CHECK();
+}
+
+void micro_launch_chain(int n, int pdl, int blocks, cudaStream_t st) {
+  ASTRA_CHECK_ARG(n > 0 && blocks > 0, "micro_launch_chain: bad arguments");
+  for (int i = 0; i < n; ++i) {
+    if (pdl) launch_pdl(empty_pdl_kernel, dim3(blocks), dim3(128), 0, st, 1, i);
+    else empty_kernel<<<blocks, 128, 0, st>>>(i);
+    LAUNCH_CHECK();
+  }
+}
+
+}  // namespace astra
