@@ -1,0 +1,304 @@
+// K2 persistent fused forward of the RHN chain (SURVEY §8(a) row a3 for cfg3; §8(a.9) `fwd_kernel`
+// "persistent" and `fwd_epilogue` "RHN micro-layers per launch {1, L}"; the cfg3 chain sat
+// 7.5× above its launch-latency floor with one GEMM + one pointwise launch per micro-step).
+//
+// One cooperative launch runs all T·L micro-steps.  CTA (m_blk, n_blk) owns batch rows
+// [128·m_blk, +128) and hidden units [64·n_blk, +64): its B tile is the 64 H-columns and the
+// matching 64 T-columns of R_ℓ's gate-blocked mirror (two 64-row TMA boxes stacked into one
+// 128-wide operand), so the highway epilogue has both pre-activations of its units in TMEM.
+// Per micro-step: TMA (A = s^{ℓ−1} bf16 operand, B = R_ℓ slice) → tcgen05 MMA into the canonical
+// split-K chunk accumulators (reading R33: chunk c accumulated from zero in its own TMEM columns,
+// exactly the chunks of the unfused GEMM) → epilogue warps sum the chunks in chunk order, add b_ℓ
+// (and x_t·W at ℓ = 1), store the pre-activations (for BPTT), apply the highway update and write
+// s^ℓ (fp32 + bf16 operand) → release/acquire counter per row block → the next micro-step's TMA
+// reads the other CTAs' s^ℓ.  R_{ℓ+1} tiles are prefetched while the counter is awaited.  The
+// arithmetic is rhn_fwd_pw_kernel's, operation for operation, so the result is bitwise identical
+// to the unfused chain (tests/test_gpu_cell.py::test_rhn_fused_forward_bitwise).
+#include "cell_math.cuh"
+#include "gemm.h"
+#include "gemm_tc.cuh"
+#include "kernels.h"
+#include "rec_fused.h"
+
+namespace astra {
+
+namespace {
+
+constexpr int RH_EPI_WARPS = 4;
+constexpr int RH_THREADS = 64 + 32 * RH_EPI_WARPS;   // warp 0 TMA, warp 1 MMA, 4 epilogue warps
+constexpr int RH_BN = 128;                            // 64 H-columns + 64 T-columns
+
+__device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
+__device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void wait_flag(const unsigned* p, unsigned target) {
+  while (ld_acquire(p) < target) __nanosleep(32);
+}
+__device__ __forceinline__ void red_release_gpu(unsigned* p, unsigned v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, %0;" ::"n"(32 * RH_EPI_WARPS) : "memory"); }
+
+__global__ void __launch_bounds__(RH_THREADS, 1)
+    rhn_rec_fwd_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                       const RhnFwdArgs a) {
+  using S = TcSmem<RH_BN>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int stages = a.stages;
+  // s^{ℓ−1} of this CTA's rows and units stays on chip between micro-steps (the tile's own epilogue
+  // produced it); the biases of every micro-layer for the tile's units are staged once
+  float* sprev = reinterpret_cast<float*>(smem + stages * S::STAGE_BYTES);   // [128 rows][64 units]
+  float* bls = sprev + TC_BM * 64;                                            // [L][128]: b_H | b_T
+  uint64_t* full = reinterpret_cast<uint64_t*>(bls + a.L * RH_BN);
+  uint64_t* empty = full + stages;
+  uint64_t* tfull = empty + stages;
+  uint64_t* tempty = tfull + 1;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 1);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int m_blk = blockIdx.x % a.num_m, n_blk = blockIdx.x / a.num_m;
+  const int m0 = m_blk * TC_BM, u0 = n_blk * 64;
+  const int nk = a.nk, kper = a.kper;
+  const int L = a.L;
+  const int nsteps = (a.t1 - a.t0) * L;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < stages; ++s) {
+      sm100::mbar_init(&full[s], 1);
+      sm100::mbar_init(&empty[s], 1);
+    }
+    sm100::mbar_init(tfull, 1);
+    sm100::mbar_init(tempty, 32 * RH_EPI_WARPS);
+    sm100::fence_barrier_init();
+  }
+  if (warp == 0 && lane == 0) {
+    sm100::tma_prefetch(&mapA);
+    sm100::tma_prefetch(&mapB);
+  }
+  if (warp == 1) sm100::tmem_alloc(tmem_slot, a.tmem_cols);
+  for (int i = threadIdx.x; i < a.L * RH_BN; i += blockDim.x) {
+    const int l = i / RH_BN, c = i % RH_BN, j = u0 + c % 64;
+    bls[i] = j < a.H ? a.b[(size_t)l * 2 * a.H + (c < 64 ? 0 : a.H) + j] : 0.f;
+  }
+  for (int i = threadIdx.x; i < TC_BM * 64; i += blockDim.x) {   // initial state s^0 at t0
+    const int r = i / 64, m = m0 + r;
+    sprev[i] = m < a.B ? a.Sf[((size_t)a.t0 * a.B + m) * a.Hp + u0 + i % 64] : 0.f;
+  }
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ TMA producer
+    if (lane == 0) {
+      long it = 0;
+      const uint64_t pol = sm100::l2_policy_evict_last();
+      const int pre = nk < stages ? nk : stages;
+      for (int q = 0; q < nsteps; ++q) {
+        const int t = a.t0 + q / L, l = q % L;
+        const int az = l * (a.T + 1) + t;   // the slot of s^{ℓ−1} at time t (RhnCell::slot)
+        auto load_b = [&](int s, int kb) {
+          uint8_t* sb = smem + s * S::STAGE_BYTES + S::A_BYTES;
+          sm100::tma_load_3d_hint(sb, &mapB, &full[s], kb * TC_BK, u0, l, pol);                 // H columns
+          sm100::tma_load_3d_hint(sb + 64 * 128, &mapB, &full[s], kb * TC_BK, a.Hp + u0, l, pol);  // T columns
+        };
+        for (int kb = 0; kb < pre; ++kb) {   // R_ℓ tiles do not depend on the recurrence
+          const long i = it + kb;
+          const int s = (int)(i % stages);
+          sm100::mbar_wait(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
+          sm100::mbar_arrive_expect_tx(&full[s], S::STAGE_BYTES);
+          load_b(s, kb);
+        }
+        if (q > 0) {   // every CTA of the row block has stored s^{ℓ−1}
+          wait_flag(a.flags + m_blk, (unsigned)(a.num_n * q));
+          fence_proxy_async_global();
+        }
+        for (int kb = 0; kb < pre; ++kb) {
+          const int s = (int)((it + kb) % stages);
+          sm100::tma_load_3d(smem + s * S::STAGE_BYTES, &mapA, &full[s], kb * TC_BK, m0, az);
+        }
+        for (int kb = pre; kb < nk; ++kb) {
+          const long i = it + kb;
+          const int s = (int)(i % stages);
+          sm100::mbar_wait(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
+          sm100::mbar_arrive_expect_tx(&full[s], S::STAGE_BYTES);
+          sm100::tma_load_3d(smem + s * S::STAGE_BYTES, &mapA, &full[s], kb * TC_BK, m0, az);
+          load_b(s, kb);
+        }
+        it += nk;
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      long it = 0;
+      for (int q = 0; q < nsteps; ++q) {
+        sm100::mbar_wait(tempty, (uint32_t)(q & 1) ^ 1);
+        sm100::tc_fence_after();
+        for (int kb = 0; kb < nk; ++kb, ++it) {
+          const int s = (int)(it % stages);
+          const int c = kb / kper;                         // canonical split-K chunk (R33)
+          const uint32_t d_tmem = tmem_base + c * RH_BN;
+          sm100::mbar_wait(&full[s], (uint32_t)((it / stages) & 1));
+          sm100::tc_fence_after();
+          const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
+          const uint32_t sb = sa + S::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < TC_BK / 16; ++kk)
+            sm100::umma_bf16(d_tmem, sm100::smem_desc_sw128(sa + kk * 32, 16, 1024),
+                             sm100::smem_desc_sw128(sb + kk * 32, 16, 1024), a.idesc,
+                             (kb != c * kper || kk != 0) ? 1u : 0u);
+          sm100::umma_commit(&empty[s]);
+        }
+        sm100::umma_commit(tfull);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ highway epilogue (4 warps)
+    const int quarter = warp & 3;            // TMEM lane quarter of this warp
+    const int row = quarter * 32 + lane;
+    const int m = m0 + row;
+    const bool valid = m < a.B;
+    const long G2 = 2L * a.Hp;
+    for (int q = 0; q < nsteps; ++q) {
+      const int t = a.t0 + q / L, l = q % L;
+      const bool last = l == L - 1;
+      sm100::mbar_wait(tfull, (uint32_t)(q & 1));
+      sm100::tc_fence_after();
+      const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16);
+      const float* bl = bls + l * RH_BN;
+      const size_t slot_out = last ? (size_t)(t + 1) * a.B * a.Hp : ((size_t)(l + 1) * (a.T + 1) + t) * a.B * a.Hp;
+      float* Z = a.Apre + ((size_t)l * a.T + t) * a.B * G2 + (size_t)m * G2;   // row m
+      const float* wx = a.WX + ((size_t)t * a.B + m) * G2;
+      float* spr = sprev + row * 64;
+#pragma unroll 1
+      for (int uc = 0; uc < 4; ++uc) {
+        const int ul = uc * 16;
+        float xh[16], xt[16];
+        if (l == 0 && valid) {   // x_t·W (ℓ = 1 only): independent of the MMA, issued first
+#pragma unroll
+          for (int q4 = 0; q4 < 4; ++q4) {
+            const float4 h4 = reinterpret_cast<const float4*>(wx + u0 + ul)[q4];
+            const float4 t4 = reinterpret_cast<const float4*>(wx + a.Hp + u0 + ul)[q4];
+            xh[4 * q4] = h4.x; xh[4 * q4 + 1] = h4.y; xh[4 * q4 + 2] = h4.z; xh[4 * q4 + 3] = h4.w;
+            xt[4 * q4] = t4.x; xt[4 * q4 + 1] = t4.y; xt[4 * q4 + 2] = t4.z; xt[4 * q4 + 3] = t4.w;
+          }
+        }
+        float zh[16], zt[16];
+        sm100::tmem_ld16(taddr + ul, zh);
+        sm100::tmem_ld16(taddr + 64 + ul, zt);
+        for (int c = 1; c < a.nsplit; ++c) {   // chunk partials summed in chunk order (rhn_fwd_pw)
+          float ph[16], pt[16];
+          sm100::tmem_ld16(taddr + c * RH_BN + ul, ph);
+          sm100::tmem_ld16(taddr + c * RH_BN + 64 + ul, pt);
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            zh[i] = __fadd_rn(zh[i], ph[i]);
+            zt[i] = __fadd_rn(zt[i], pt[i]);
+          }
+        }
+        if (!valid) continue;
+        float* sn = a.Sf + slot_out + (size_t)m * a.Hp + u0 + ul;
+        __nv_bfloat16* so = a.Sop + slot_out + (size_t)m * a.Hp + u0 + ul;
+        float sv[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) sv[i] = spr[ul + i];
+        float snew[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const int j = u0 + ul + i;
+          float s_new = 0.f, aH = 0.f, aT = 0.f;
+          if (j < a.H) {
+            aH = __fadd_rn(zh[i], bl[ul + i]);
+            aT = __fadd_rn(zt[i], bl[64 + ul + i]);
+            if (l == 0) {
+              aH = __fadd_rn(aH, xh[i]);
+              aT = __fadd_rn(aT, xt[i]);
+            }
+            const float h = tanh_<true>(aH), tau = sigm<true>(aT);
+            s_new = __fadd_rn(__fmul_rn(h, tau), __fmul_rn(sv[i], __fsub_rn(1.f, tau)));
+            if (last && a.y) a.y[((size_t)t * a.B + m) * a.ldy + j] = __float2bfloat16_rn(s_new);
+            if (last && t == a.T - 1 && a.sT) a.sT[(size_t)m * a.H + j] = s_new;
+          }
+          zh[i] = aH;   // the pre-activations saved for BPTT (padding units: 0)
+          zt[i] = aT;
+          snew[i] = s_new;
+          spr[ul + i] = s_new;   // s^ℓ: the next micro-step's s^{ℓ−1} of this row and unit
+        }
+#pragma unroll
+        for (int q4 = 0; q4 < 4; ++q4) {
+          reinterpret_cast<float4*>(Z + u0 + ul)[q4] = make_float4(zh[4 * q4], zh[4 * q4 + 1], zh[4 * q4 + 2], zh[4 * q4 + 3]);
+          reinterpret_cast<float4*>(Z + a.Hp + u0 + ul)[q4] =
+              make_float4(zt[4 * q4], zt[4 * q4 + 1], zt[4 * q4 + 2], zt[4 * q4 + 3]);
+          reinterpret_cast<float4*>(sn)[q4] = make_float4(snew[4 * q4], snew[4 * q4 + 1], snew[4 * q4 + 2], snew[4 * q4 + 3]);
+        }
+        uint4 pk[2];
+        uint32_t* pu = reinterpret_cast<uint32_t*>(pk);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(snew[2 * i], snew[2 * i + 1]);
+          pu[i] = *reinterpret_cast<uint32_t*>(&b2);
+        }
+        reinterpret_cast<uint4*>(so)[0] = pk[0];
+        reinterpret_cast<uint4*>(so)[1] = pk[1];
+      }
+      sm100::tc_fence_before();
+      sm100::mbar_arrive(tempty);
+      if (q + 1 < nsteps) {   // publish s^ℓ of this tile to the row block: every writer orders its
+        fence_proxy_async_global();   // stores before the readers' TMA (async proxy); the CTA barrier
+        epi_bar();                    // and one release add (cumulative) publish them at gpu scope
+        if (warp == 2 && lane == 0) red_release_gpu(a.flags + m_blk, 1u);
+      }
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    sm100::tc_fence_after();
+    sm100::tmem_dealloc(tmem_base, a.tmem_cols);
+  }
+}
+
+}  // namespace
+
+bool rhn_rec_fwd_supported(int B, int Hp, int nsplit) {
+  return nsplit >= 1 && nsplit <= 4 && Hp % 64 == 0 && cdiv(B, TC_BM) * (Hp / 64) <= num_sms();
+}
+
+void rhn_rec_fwd_launch(const CUtensorMap& mapA, const CUtensorMap& mapB, RhnFwdArgs a, cudaStream_t st) {
+  using S = TcSmem<RH_BN>;
+  int dev = 0, maxs = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  ASTRA_CHECK_ARG(rhn_rec_fwd_supported(a.B, a.Hp, a.nsplit), "rhn fused forward: unsupported shape");
+  const int extra = TC_BM * 64 * 4 + a.L * RH_BN * 4;   // sprev + biases
+  int stages = (maxs - 1024 - 256 - extra) / S::STAGE_BYTES;
+  if (stages > 6) stages = 6;
+  ASTRA_CHECK_ARG(stages >= 2, "rhn fused forward: depth too large for shared memory");
+  a.stages = stages;
+  a.nk = cdiv(a.Hp, TC_BK);
+  a.kper = cdiv(a.nk, a.nsplit);
+  a.num_m = cdiv(a.B, TC_BM);
+  a.num_n = a.Hp / 64;
+  a.tmem_cols = a.nsplit <= 1 ? 128 : a.nsplit <= 2 ? 256 : 512;
+  const int smem = 1024 + stages * S::STAGE_BYTES + extra + 256;
+  CUDA_TRY(cudaFuncSetAttribute(rhn_rec_fwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(a.num_m * a.num_n);
+  cfg.blockDim = dim3(RH_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  CUDA_TRY(cudaLaunchKernelEx(&cfg, rhn_rec_fwd_kernel, mapA, mapB, a));
+  LAUNCH_CHECK();
+}
+
+}  // namespace astra

@@ -10,6 +10,7 @@
 // Internal gate layout: gate-blocked and padded, column g·Hp + j.
 #include <algorithm>
 
+#include "../kernels/rec_fused.h"
 #include "cell.h"
 
 namespace astra {
@@ -18,7 +19,7 @@ class RhnCell : public Cell {
  public:
   int L, G2, nchunk;
   size_t off_X, off_WX, off_Apre, off_Sf, off_Sop, off_MW, off_MR;
-  size_t off_DA, off_dS, off_dSpart, off_Zpart, off_part;
+  size_t off_DA, off_dS, off_dSpart, off_Zpart, off_part, off_flags;
 
   // Reading R33: the BPTT GEMM ds·R_ℓᵀ (K = 2·Hp, few output tiles at small batch) is split over K
   // into s fixed chunks, each accumulated from zero; the next pointwise kernel adds the partials in
@@ -61,6 +62,7 @@ class RhnCell : public Cell {
     off_dSpart = c.take((size_t)bptt_ksplit() * B * Hp * 4);
     off_Zpart = c.take((size_t)fwd_ksplit() * B * G2 * 4);
     off_part = c.take((size_t)L * nchunk * G2 * 4);
+    off_flags = c.take(4096);
     scratch_bytes = c.o;
   }
 
@@ -70,6 +72,10 @@ class RhnCell : public Cell {
   char* Sop(int l, int t) { return saved + off_Sop + slot(l, t) * esz(); }
   float* Apre(int l, int t) { return sv<float>(off_Apre) + ((size_t)l * T + t) * B * G2; }
   char* DA(int l, int t) { return scratch + off_DA + ((size_t)l * T + t) * B * G2 * esz(); }
+
+  // K2 choices (AV fuse_fwd): GEMM + pointwise launch per micro-step, or the persistent fused chain
+  bool fused_fwd_ok() const { return ot == OT::BF16 && rhn_rec_fwd_supported(B, Hp, fwd_ksplit()); }
+  int fwd_fusions() const override { return fused_fwd_ok() ? 2 : 1; }
 
   void* x_operand() override { return sv<char>(off_X); }
   Mat2 y_operand() override { return mat(Sop(0, 1), Hp, (long)T * B, Hp); }
@@ -126,6 +132,23 @@ class RhnCell : public Cell {
     float* Zpart = sc<float>(off_Zpart);
     EpiStore ez = epi(Zpart, G2, B, G2);
     ez.split_stride = (long)B * G2;
+    if (var.fwd_mode >= 1 && fused_fwd_ok()) {   // persistent fused chain: one launch for all T·L micro-steps
+      const TcGemm& g64 = tc_get(1, rec, KCfg{64, 1, 1});
+      const TcGemm& g128 = tc_get(9, rec, KCfg{128, 1, 1});   // only for the N = 128 instruction descriptor
+      RhnFwdArgs ra{};
+      ra.B = B; ra.H = H; ra.Hp = Hp; ra.T = T; ra.L = L; ra.t0 = 0; ra.t1 = T;
+      ra.nsplit = rec.ksplit;
+      ra.idesc = g128.args.idesc;
+      ra.WX = WX; ra.b = p("b"); ra.Apre = Apre(0, 0); ra.Sf = Sf(0, 0); ra.Sop = (__nv_bfloat16*)Sop(0, 0);
+      ra.y = (__nv_bfloat16*)y; ra.ldy = H; ra.sT = sT;
+      ra.flags = sc<unsigned>(off_flags);
+      CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
+      rhn_rec_fwd_launch(g64.mapA, g64.mapB, ra, st);
+      for (int t = 0; t < T; ++t) fwd_step_done(t, st);
+      mark(R_FWD, 1, st);
+      fwd_done = true;
+      return;
+    }
     for (int t = 0; t < T; ++t) {
       for (int l = 0; l < L; ++l) {
         float* Z = Apre(l, t);

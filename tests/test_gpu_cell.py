@@ -163,6 +163,26 @@ def test_rhn_ragged(dtype, tol):
     _check("rhn", 3, 20, 72, 830, dtype, synth.config_seed(3) + 2, tol, L=2)
 
 
+@pytest.mark.parametrize("T,B,I,H,L", [(3, 4, 32, 64, 3), (3, 20, 72, 830, 2), (2, 200, 64, 128, 2),
+                                       (4, 64, 830, 830, 10)])
+def test_rhn_fused_forward_bitwise(T, B, I, H, L):
+    """The persistent fused RHN forward chain (fwd=1: one cooperative launch for all T·L micro-steps,
+    split-K chunks as TMEM accumulators, highway epilogue from TMEM) gives the same bits as the
+    GEMM + pointwise launch per micro-step (fwd=0) — outputs and every gradient (the backward reads
+    the pre-activations and states it saved) — and matches the oracle."""
+    p, inp, dY, dhT, dcT = make_cell_case("rhn", T, B, I, H, synth.config_seed(3) + 7, bf16=True, L=L)
+    ref = None
+    for v in ("fwd=0", "fwd=1"):
+        out, g, _ = run_gpu_cell("rhn", p, inp, dY, dhT, dcT, "bf16", v, depth=L)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    _check("rhn", T, B, I, H, "bf16", synth.config_seed(3) + 7, TOL_BF16, variant="fwd=1", L=L)
+
+
 def test_rhn_cfg3_reduced():
     """cfg3 reduced rung: L = 10, H = I = 830, B = 64, T = 8 (bf16)."""
     _check("rhn", 8, 64, 830, 830, "bf16", synth.config_seed(3), TOL_BF16, L=10)

@@ -263,3 +263,25 @@ def test_tuner_fork_explores_both_allocation_contexts():
     assert n_steps < 600, "the tuner did not converge"
     assert torch.equal(res[0][0], res[1][0])
     assert res[0][1] == {False, True}, "the recompute context was never explored"
+
+
+@pytest.mark.parametrize("hov", [0, 1])
+def test_rhn_fused_forward_lm_bitwise(hov):
+    """RHN LM steps with the persistent fused forward chain (fwd=1) give the same bits as the
+    per-micro-step launches (fwd=0), with and without the head overlapping the chain, over 4 SGD
+    steps (state carried between steps, graph replay)."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 5, 64, 128, 192, 300
+    out = []
+    for v in ("fwd=0", "fwd=1"):
+        p, tok, h0, c0 = _lm_case("rhn", T, B, I, H, V, synth.config_seed(3) + 30, True)
+        c = A.Cell("rhn", H, I, B, T, dtype="bf16", depth=L_DEPTH)
+        m = A.LM(c, V)
+        m.load(p)
+        c.tune_mode(A.TUNE_FROZEN, f"{v},hov={hov}")
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(4):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append((m.params.clone(), float(m.loss.item())))
+    assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
