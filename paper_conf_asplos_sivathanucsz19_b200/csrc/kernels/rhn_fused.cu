@@ -34,8 +34,19 @@ __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint64_t global_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// a row block that never completes (a co-residency or protocol fault) traps after 20 s instead of
+// hanging the device: sticky CUDA error, ASTRA_E_CUDA on the next call
 __device__ __forceinline__ void wait_flag(const unsigned* p, unsigned target) {
-  while (ld_acquire(p) < target) __nanosleep(32);
+  const uint64_t t0 = global_ns();
+  while (ld_acquire(p) < target) {
+    __nanosleep(32);
+    if (global_ns() - t0 > 20ull * 1000 * 1000 * 1000) __trap();
+  }
 }
 __device__ __forceinline__ void red_release_gpu(unsigned* p, unsigned v) {
   asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
