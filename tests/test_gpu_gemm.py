@@ -126,3 +126,24 @@ def test_cta_pair_bitwise(a_mn, b_mn, M, N, K):
     s2 = A.gemm_bf16_ex(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=128, cta_group=2, ksplit=3)
     torch.cuda.synchronize()
     assert torch.equal(s1.cpu(), s2.cpu())
+
+
+def test_day1_microbenchmarks_run():
+    """The astra_micro_* kernels (bench_micro.py) run and do what they claim: the
+    grid barrier counter ends at iters × #SMs, the streaming read and the launch chain complete."""
+    import ctypes
+    import torch
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    L = A.lib()
+    sp = ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    buf = torch.rand(4 << 20, device="cuda")
+    sink = torch.zeros(1, device="cuda")
+    A._check(L.astra_micro_stream_read(A._ptr(buf), buf.numel() * 4, 3, A._ptr(sink), sp))
+    ctr = torch.zeros(4, dtype=torch.int32, device="cuda")
+    A._check(L.astra_micro_grid_barrier(A._ptr(ctr), 100, sp))
+    A._check(L.astra_micro_launch_chain(50, 1, 148, sp))
+    A._check(L.astra_micro_launch_chain(50, 0, 148, sp))
+    torch.cuda.synchronize()
+    assert int(ctr[0].item()) == 100 * torch.cuda.get_device_properties(0).multi_processor_count
+    assert float(sink.item()) == 0.0
+    assert L.astra_micro_grid_barrier(None, 10, sp) == 1
