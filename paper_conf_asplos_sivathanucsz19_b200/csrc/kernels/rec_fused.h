@@ -77,12 +77,13 @@ struct BpttFusedMaps {
   CUtensorMap DY;   // dy [T][B][ld] fp32 (LM internal, ld = Hp) or bf16 (external, ld = H), box {64, 16}
 };
 // Persistent fused RHN forward chain (rhn_fused.cu): all T·L micro-steps of [t0, t1) in one
-// cooperative launch; tiles of 128 rows × 64 units (their H and T columns), split-K chunks of the
-// canonical R33 split kept as TMEM accumulators.
+// cooperative launch; tiles of 128 rows × 32 units (their H and T columns), split-K chunks of the
+// canonical R33 split kept as TMEM accumulators, the whole K of a micro-step resident when it fits.
 struct RhnFwdArgs {
   int B, H, Hp, T, L, t0, t1;
   int nsplit;               // canonical split-K chunks of K = Hp (RhnCell::fwd_ksplit)
   int num_m, num_n, stages, nk, kper, tmem_cols;   // set by the launcher
+  int a_rows;               // rows of the A box: 64 when B <= 64 (the MMA's rows 64..127 are never read), else 128
   uint32_t idesc;           // M = 128, N = 128 bf16 MMA, both operands K-major
   const float* WX;          // [T·B][2Hp] hoisted x·W (added at ℓ = 1)
   const float* b;           // [L][2H] external biases
@@ -93,10 +94,11 @@ struct RhnFwdArgs {
   long ldy;
   float* sT;                // optional [B][H]
   unsigned* flags;          // [num_m] row-block counters, zeroed before the launch
+  unsigned long long* trace;   // optional (ASTRA_RHN_TRACE): [grid][T·L][5] globaltimer stamps
 };
 bool rhn_rec_fwd_supported(int B, int Hp, int nsplit);
-// mapA: the bf16 state operands as a 3-D K-major map (inner Hp, rows B, z = L·(T+1)), box {64, 128};
-// mapB: the R mirrors [L][2Hp][Hp] K-major, box {64, 64}.
+// mapA: the bf16 state operands as a 3-D K-major map (inner Hp, rows B, z = L·(T+1)), box {64, a_rows};
+// mapB: the R mirrors [L][2Hp][Hp] K-major, box {64, 32}; both SWIZZLE_128B.
 void rhn_rec_fwd_launch(const CUtensorMap& mapA, const CUtensorMap& mapB, RhnFwdArgs a, cudaStream_t st);
 
 bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);

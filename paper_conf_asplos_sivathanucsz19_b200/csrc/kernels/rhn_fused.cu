@@ -3,9 +3,11 @@
 // 7.5× above its launch-latency floor with one GEMM + one pointwise launch per micro-step).
 //
 // One cooperative launch runs all T·L micro-steps.  CTA (m_blk, n_blk) owns batch rows
-// [128·m_blk, +128) and hidden units [64·n_blk, +64): its B tile is the 64 H-columns and the
-// matching 64 T-columns of R_ℓ's gate-blocked mirror (two 64-row TMA boxes stacked into one
-// 128-wide operand), so the highway epilogue has both pre-activations of its units in TMEM.
+// [128·m_blk, +128) and hidden units [32·n_blk, +32): its B tile is the 32 H-columns and the
+// matching 32 T-columns of R_ℓ's gate-blocked mirror (two 32-row TMA boxes stacked into one
+// 64-wide operand), so the highway epilogue has both pre-activations of its units in TMEM.  When
+// it fits (cfg3: 13 k-blocks of 16 KB) the whole K of a micro-step is resident: R_{ℓ+1} is loaded
+// while micro-step ℓ finishes, and after the row block's counter only A crosses L2, in one round.
 // Per micro-step: TMA (A = s^{ℓ−1} bf16 operand, B = R_ℓ slice) → tcgen05 MMA into the canonical
 // split-K chunk accumulators (reading R33: chunk c accumulated from zero in its own TMEM columns,
 // exactly the chunks of the unfused GEMM) → epilogue warps sum the chunks in chunk order, add b_ℓ
@@ -14,6 +16,8 @@
 // reads the other CTAs' s^ℓ.  R_{ℓ+1} tiles are prefetched while the counter is awaited.  The
 // arithmetic is rhn_fwd_pw_kernel's, operation for operation, so the result is bitwise identical
 // to the unfused chain (tests/test_gpu_cell.py::test_rhn_fused_forward_bitwise).
+#include <algorithm>
+
 #include "cell_math.cuh"
 #include "gemm.h"
 #include "gemm_tc.cuh"
@@ -26,7 +30,10 @@ namespace {
 
 constexpr int RH_EPI_WARPS = 4;
 constexpr int RH_THREADS = 64 + 32 * RH_EPI_WARPS;   // warp 0 TMA, warp 1 MMA, 4 epilogue warps
-constexpr int RH_BN = 128;                            // 64 H-columns + 64 T-columns
+constexpr int RH_UB = 32;                             // hidden units per tile
+constexpr int RH_BN = 2 * RH_UB;                      // MMA N: the units' H-columns then their T-columns
+constexpr int RH_SP = RH_UB + 1;                      // row strides of the per-thread (row) shared buffers,
+constexpr int RH_ZP = RH_BN + 1;                      // padded: a warp's 32 rows hit 32 different banks
 
 __device__ __forceinline__ void fence_proxy_async_global() { asm volatile("fence.proxy.async.global;" ::: "memory"); }
 __device__ __forceinline__ unsigned ld_acquire(const unsigned* p) {
@@ -44,27 +51,44 @@ __device__ __forceinline__ uint64_t global_ns() {
 __device__ __forceinline__ void wait_flag(const unsigned* p, unsigned target) {
   const uint64_t t0 = global_ns();
   while (ld_acquire(p) < target) {
-    __nanosleep(32);
+    __nanosleep(64);
     if (global_ns() - t0 > 20ull * 1000 * 1000 * 1000) __trap();
   }
 }
 __device__ __forceinline__ void red_release_gpu(unsigned* p, unsigned v) {
   asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
+// mbarrier wait with back-off: the producer and MMA warps wait microseconds per micro-step for the
+// epilogue; a hot try_wait loop would take issue slots from the epilogue warps sharing their scheduler
+__device__ __forceinline__ bool mbar_try(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n\t.reg .pred P1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, P1;\n\t}"
+      : "=r"(ok)
+      : "r"(sm100::smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait_idle(uint64_t* bar, uint32_t parity) {
+  while (!mbar_try(bar, parity)) __nanosleep(64);
+}
 __device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, %0;" ::"n"(32 * RH_EPI_WARPS) : "memory"); }
 
 __global__ void __launch_bounds__(RH_THREADS, 1)
     rhn_rec_fwd_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                        const RhnFwdArgs a) {
-  using S = TcSmem<RH_BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int stages = a.stages;
+  const int a_bytes = a.a_rows * TC_BK * 2, stage_bytes = a_bytes + RH_BN * TC_BK * 2;
   // s^{ℓ−1} of this CTA's rows and units stays on chip between micro-steps (the tile's own epilogue
   // produced it); the biases of every micro-layer for the tile's units are staged once
-  float* sprev = reinterpret_cast<float*>(smem + stages * S::STAGE_BYTES);   // [128 rows][64 units]
-  float* bls = sprev + TC_BM * 64;                                            // [L][128]: b_H | b_T
-  uint64_t* full = reinterpret_cast<uint64_t*>(bls + a.L * RH_BN);
+  float* sprev = reinterpret_cast<float*>(smem + stages * stage_bytes);   // [a_rows][RH_SP]
+  float* bls = sprev + a.a_rows * RH_SP;                                  // [L][RH_BN]: b_H | b_T
+  float* zst = bls + a.L * RH_BN;   // [a_rows][RH_ZP] pre-activations staged until after the publish
+  uint64_t* full = reinterpret_cast<uint64_t*>(zst + ((a.a_rows * RH_ZP + 1) & ~1));
   uint64_t* empty = full + stages;
   uint64_t* tfull = empty + stages;
   uint64_t* tempty = tfull + 1;
@@ -72,7 +96,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int m_blk = blockIdx.x % a.num_m, n_blk = blockIdx.x / a.num_m;
-  const int m0 = m_blk * TC_BM, u0 = n_blk * 64;
+  const int m0 = m_blk * TC_BM, u0 = n_blk * RH_UB;
   const int nk = a.nk, kper = a.kper;
   const int L = a.L;
   const int nsteps = (a.t1 - a.t0) * L;
@@ -92,12 +116,12 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
   }
   if (warp == 1) sm100::tmem_alloc(tmem_slot, a.tmem_cols);
   for (int i = threadIdx.x; i < a.L * RH_BN; i += blockDim.x) {
-    const int l = i / RH_BN, c = i % RH_BN, j = u0 + c % 64;
-    bls[i] = j < a.H ? a.b[(size_t)l * 2 * a.H + (c < 64 ? 0 : a.H) + j] : 0.f;
+    const int l = i / RH_BN, c = i % RH_BN, j = u0 + c % RH_UB;
+    bls[i] = j < a.H ? a.b[(size_t)l * 2 * a.H + (c < RH_UB ? 0 : a.H) + j] : 0.f;
   }
-  for (int i = threadIdx.x; i < TC_BM * 64; i += blockDim.x) {   // initial state s^0 at t0
-    const int r = i / 64, m = m0 + r;
-    sprev[i] = m < a.B ? a.Sf[((size_t)a.t0 * a.B + m) * a.Hp + u0 + i % 64] : 0.f;
+  for (int i = threadIdx.x; i < a.a_rows * RH_UB; i += blockDim.x) {   // initial state s^0 at t0
+    const int r = i / RH_UB, m = m0 + r;
+    sprev[r * RH_SP + i % RH_UB] = m < a.B ? a.Sf[((size_t)a.t0 * a.B + m) * a.Hp + u0 + i % RH_UB] : 0.f;
   }
   sm100::tc_fence_before();
   __syncthreads();
@@ -114,31 +138,32 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         const int t = a.t0 + q / L, l = q % L;
         const int az = l * (a.T + 1) + t;   // the slot of s^{ℓ−1} at time t (RhnCell::slot)
         auto load_b = [&](int s, int kb) {
-          uint8_t* sb = smem + s * S::STAGE_BYTES + S::A_BYTES;
-          sm100::tma_load_3d_hint(sb, &mapB, &full[s], kb * TC_BK, u0, l, pol);                 // H columns
-          sm100::tma_load_3d_hint(sb + 64 * 128, &mapB, &full[s], kb * TC_BK, a.Hp + u0, l, pol);  // T columns
+          uint8_t* sb = smem + s * stage_bytes + a_bytes;
+          sm100::tma_load_3d_hint(sb, &mapB, &full[s], kb * TC_BK, u0, l, pol);                        // H columns
+          sm100::tma_load_3d_hint(sb + RH_UB * 128, &mapB, &full[s], kb * TC_BK, a.Hp + u0, l, pol);  // T columns
         };
         for (int kb = 0; kb < pre; ++kb) {   // R_ℓ tiles do not depend on the recurrence
           const long i = it + kb;
           const int s = (int)(i % stages);
-          sm100::mbar_wait(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
-          sm100::mbar_arrive_expect_tx(&full[s], S::STAGE_BYTES);
+          mbar_wait_idle(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
+          sm100::mbar_arrive_expect_tx(&full[s], (uint32_t)stage_bytes);
           load_b(s, kb);
         }
         if (q > 0) {   // every CTA of the row block has stored s^{ℓ−1}
           wait_flag(a.flags + m_blk, (unsigned)(a.num_n * q));
           fence_proxy_async_global();
         }
+        if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 0] = global_ns();
         for (int kb = 0; kb < pre; ++kb) {
           const int s = (int)((it + kb) % stages);
-          sm100::tma_load_3d(smem + s * S::STAGE_BYTES, &mapA, &full[s], kb * TC_BK, m0, az);
+          sm100::tma_load_3d(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
         }
         for (int kb = pre; kb < nk; ++kb) {
           const long i = it + kb;
           const int s = (int)(i % stages);
-          sm100::mbar_wait(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
-          sm100::mbar_arrive_expect_tx(&full[s], S::STAGE_BYTES);
-          sm100::tma_load_3d(smem + s * S::STAGE_BYTES, &mapA, &full[s], kb * TC_BK, m0, az);
+          mbar_wait_idle(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
+          sm100::mbar_arrive_expect_tx(&full[s], (uint32_t)stage_bytes);
+          sm100::tma_load_3d(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
           load_b(s, kb);
         }
         it += nk;
@@ -149,7 +174,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
     if (lane == 0) {
       long it = 0;
       for (int q = 0; q < nsteps; ++q) {
-        sm100::mbar_wait(tempty, (uint32_t)(q & 1) ^ 1);
+        mbar_wait_idle(tempty, (uint32_t)(q & 1) ^ 1);
         sm100::tc_fence_after();
         for (int kb = 0; kb < nk; ++kb, ++it) {
           const int s = (int)(it % stages);
@@ -157,8 +182,12 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           const uint32_t d_tmem = tmem_base + c * RH_BN;
           sm100::mbar_wait(&full[s], (uint32_t)((it / stages) & 1));
           sm100::tc_fence_after();
-          const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
-          const uint32_t sb = sa + S::A_BYTES;
+          if (a.trace && kb == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 1] = global_ns();
+          if (a.trace && kb == nk - 1) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 2] = global_ns();
+          // a_rows = 64: the M = 128 MMA's rows 64..127 read the B tile's bytes — garbage rows of
+          // TMEM that the epilogue never reads (rows ≥ B)
+          const uint32_t sa = sm100::smem_u32(smem + s * stage_bytes);
+          const uint32_t sb = sa + a_bytes;
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
             sm100::umma_bf16(d_tmem, sm100::smem_desc_sw128(sa + kk * 32, 16, 1024),
@@ -181,14 +210,16 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       const bool last = l == L - 1;
       sm100::mbar_wait(tfull, (uint32_t)(q & 1));
       sm100::tc_fence_after();
+      if (a.trace && warp == 2 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 3] = global_ns();
       const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16);
       const float* bl = bls + l * RH_BN;
       const size_t slot_out = last ? (size_t)(t + 1) * a.B * a.Hp : ((size_t)(l + 1) * (a.T + 1) + t) * a.B * a.Hp;
       float* Z = a.Apre + ((size_t)l * a.T + t) * a.B * G2 + (size_t)m * G2;   // row m
       const float* wx = a.WX + ((size_t)t * a.B + m) * G2;
-      float* spr = sprev + row * 64;
+      float* spr = sprev + row * RH_SP;   // valid rows only (m < B ≤ a_rows when a_rows = 64)
+      float* zr = zst + row * RH_ZP;
 #pragma unroll 1
-      for (int uc = 0; uc < 4; ++uc) {
+      for (int uc = 0; uc < RH_UB / 16; ++uc) {
         const int ul = uc * 16;
         float xh[16], xt[16];
         if (l == 0 && valid) {   // x_t·W (ℓ = 1 only): independent of the MMA, issued first
@@ -202,19 +233,19 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         }
         float zh[16], zt[16];
         sm100::tmem_ld16(taddr + ul, zh);
-        sm100::tmem_ld16(taddr + 64 + ul, zt);
+        sm100::tmem_ld16(taddr + RH_UB + ul, zt);
         for (int c = 1; c < a.nsplit; ++c) {   // chunk partials summed in chunk order (rhn_fwd_pw)
           float ph[16], pt[16];
           sm100::tmem_ld16(taddr + c * RH_BN + ul, ph);
-          sm100::tmem_ld16(taddr + c * RH_BN + 64 + ul, pt);
+          sm100::tmem_ld16(taddr + c * RH_BN + RH_UB + ul, pt);
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
             zh[i] = __fadd_rn(zh[i], ph[i]);
             zt[i] = __fadd_rn(zt[i], pt[i]);
           }
         }
+        if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 5] = global_ns();
         if (!valid) continue;
-        float* sn = a.Sf + slot_out + (size_t)m * a.Hp + u0 + ul;
         __nv_bfloat16* so = a.Sop + slot_out + (size_t)m * a.Hp + u0 + ul;
         float sv[16];
 #pragma unroll
@@ -226,7 +257,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           float s_new = 0.f, aH = 0.f, aT = 0.f;
           if (j < a.H) {
             aH = __fadd_rn(zh[i], bl[ul + i]);
-            aT = __fadd_rn(zt[i], bl[64 + ul + i]);
+            aT = __fadd_rn(zt[i], bl[RH_UB + ul + i]);
             if (l == 0) {
               aH = __fadd_rn(aH, xh[i]);
               aT = __fadd_rn(aT, xt[i]);
@@ -236,17 +267,10 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
             if (last && a.y) a.y[((size_t)t * a.B + m) * a.ldy + j] = __float2bfloat16_rn(s_new);
             if (last && t == a.T - 1 && a.sT) a.sT[(size_t)m * a.H + j] = s_new;
           }
-          zh[i] = aH;   // the pre-activations saved for BPTT (padding units: 0)
-          zt[i] = aT;
+          zr[ul + i] = aH;            // pre-activations for BPTT (padding units: 0),
+          zr[RH_UB + ul + i] = aT;    // stored after the publish
           snew[i] = s_new;
           spr[ul + i] = s_new;   // s^ℓ: the next micro-step's s^{ℓ−1} of this row and unit
-        }
-#pragma unroll
-        for (int q4 = 0; q4 < 4; ++q4) {
-          reinterpret_cast<float4*>(Z + u0 + ul)[q4] = make_float4(zh[4 * q4], zh[4 * q4 + 1], zh[4 * q4 + 2], zh[4 * q4 + 3]);
-          reinterpret_cast<float4*>(Z + a.Hp + u0 + ul)[q4] =
-              make_float4(zt[4 * q4], zt[4 * q4 + 1], zt[4 * q4 + 2], zt[4 * q4 + 3]);
-          reinterpret_cast<float4*>(sn)[q4] = make_float4(snew[4 * q4], snew[4 * q4 + 1], snew[4 * q4 + 2], snew[4 * q4 + 3]);
         }
         uint4 pk[2];
         uint32_t* pu = reinterpret_cast<uint32_t*>(pk);
@@ -260,10 +284,28 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       }
       sm100::tc_fence_before();
       sm100::mbar_arrive(tempty);
+      if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 6] = global_ns();
       if (q + 1 < nsteps) {   // publish s^ℓ of this tile to the row block: every writer orders its
         fence_proxy_async_global();   // stores before the readers' TMA (async proxy); the CTA barrier
+        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 7] = global_ns();
         epi_bar();                    // and one release add (cumulative) publish them at gpu scope
-        if (warp == 2 && lane == 0) red_release_gpu(a.flags + m_blk, 1u);
+        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 8] = global_ns();
+        if (warp == 2 && lane == 0) {
+          red_release_gpu(a.flags + m_blk, 1u);
+          if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 4] = global_ns();
+        }
+      }
+      // off the critical path: the fp32 state and the pre-activations, read only by the backward
+      if (valid) {
+        float* sn = a.Sf + slot_out + (size_t)m * a.Hp + u0;
+#pragma unroll
+        for (int q4 = 0; q4 < RH_UB / 4; ++q4) {
+          const int o = 4 * q4;
+          reinterpret_cast<float4*>(sn)[q4] = make_float4(spr[o], spr[o + 1], spr[o + 2], spr[o + 3]);
+          reinterpret_cast<float4*>(Z + u0)[q4] = make_float4(zr[o], zr[o + 1], zr[o + 2], zr[o + 3]);
+          reinterpret_cast<float4*>(Z + a.Hp + u0)[q4] =
+              make_float4(zr[RH_UB + o], zr[RH_UB + o + 1], zr[RH_UB + o + 2], zr[RH_UB + o + 3]);
+        }
       }
     }
   }
@@ -277,26 +319,27 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
 }  // namespace
 
 bool rhn_rec_fwd_supported(int B, int Hp, int nsplit) {
-  return nsplit >= 1 && nsplit <= 4 && Hp % 64 == 0 && cdiv(B, TC_BM) * (Hp / 64) <= num_sms();
+  return nsplit >= 1 && nsplit <= 4 && Hp % RH_UB == 0 && cdiv(B, TC_BM) * (Hp / RH_UB) <= num_sms();
 }
 
 void rhn_rec_fwd_launch(const CUtensorMap& mapA, const CUtensorMap& mapB, RhnFwdArgs a, cudaStream_t st) {
-  using S = TcSmem<RH_BN>;
   int dev = 0, maxs = 0;
   CUDA_TRY(cudaGetDevice(&dev));
   CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
   ASTRA_CHECK_ARG(rhn_rec_fwd_supported(a.B, a.Hp, a.nsplit), "rhn fused forward: unsupported shape");
-  const int extra = TC_BM * 64 * 4 + a.L * RH_BN * 4;   // sprev + biases
-  int stages = (maxs - 1024 - 256 - extra) / S::STAGE_BYTES;
-  if (stages > 6) stages = 6;
-  ASTRA_CHECK_ARG(stages >= 2, "rhn fused forward: depth too large for shared memory");
-  a.stages = stages;
+  ASTRA_CHECK_ARG(a.a_rows == TC_BM || (a.a_rows == 64 && a.B <= 64), "rhn fused forward: bad A box");
   a.nk = cdiv(a.Hp, TC_BK);
   a.kper = cdiv(a.nk, a.nsplit);
   a.num_m = cdiv(a.B, TC_BM);
-  a.num_n = a.Hp / 64;
-  a.tmem_cols = a.nsplit <= 1 ? 128 : a.nsplit <= 2 ? 256 : 512;
-  const int smem = 1024 + stages * S::STAGE_BYTES + extra + 256;
+  a.num_n = a.Hp / RH_UB;
+  a.tmem_cols = a.nsplit <= 1 ? 64 : a.nsplit <= 2 ? 128 : 256;
+  const int stage_bytes = a.a_rows * TC_BK * 2 + RH_BN * TC_BK * 2;
+  const int extra = a.a_rows * RH_SP * 4 + a.L * RH_BN * 4 + ((a.a_rows * RH_ZP + 1) & ~1) * 4;   // state, biases, staging
+  int stages = (maxs - 1024 - 256 - extra) / stage_bytes;
+  if (stages > a.nk) stages = a.nk;   // the whole K of a micro-step resident when it fits
+  ASTRA_CHECK_ARG(stages >= std::min(2, a.nk), "rhn fused forward: depth too large for shared memory");
+  a.stages = stages;
+  const int smem = 1024 + stages * stage_bytes + extra + 256;
   CUDA_TRY(cudaFuncSetAttribute(rhn_rec_fwd_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(a.num_m * a.num_n);

@@ -9,6 +9,7 @@
 // (pointwise writes ds(1−τ), the GEMM accumulates da·R_ℓᵀ onto it); dR_ℓ = S_ℓᵀ·DA_ℓ per micro-layer.
 // Internal gate layout: gate-blocked and padded, column g·Hp + j.
 #include <algorithm>
+#include <cstdlib>
 
 #include "../kernels/rec_fused.h"
 #include "cell.h"
@@ -133,17 +134,22 @@ class RhnCell : public Cell {
     EpiStore ez = epi(Zpart, G2, B, G2);
     ez.split_stride = (long)B * G2;
     if (var.fwd_mode >= 1 && fused_fwd_ok()) {   // persistent fused chain: one launch for all T·L micro-steps
-      const TcGemm& g64 = tc_get(1, rec, KCfg{64, 1, 1});
-      const TcGemm& g128 = tc_get(9, rec, KCfg{128, 1, 1});   // only for the N = 128 instruction descriptor
+      const TcGemm& g64 = tc_get(1, rec, KCfg{64, 1, 1});   // for the M = 128, N = 64 instruction descriptor
       RhnFwdArgs ra{};
       ra.B = B; ra.H = H; ra.Hp = Hp; ra.T = T; ra.L = L; ra.t0 = 0; ra.t1 = T;
       ra.nsplit = rec.ksplit;
-      ra.idesc = g128.args.idesc;
+      ra.idesc = g64.args.idesc;
+      ra.a_rows = B <= 64 ? 64 : TC_BM;
+      CUtensorMap mA, mB;
+      make_tile_map(&mA, Sop(0, 0), true, Hp, B, (long)L * (T + 1), Hp, (long)B * Hp, 64, ra.a_rows, 128);
+      make_tile_map(&mB, MR, true, Hp, G2, L, Hp, (long)G2 * Hp, 64, 32, 128);
       ra.WX = WX; ra.b = p("b"); ra.Apre = Apre(0, 0); ra.Sf = Sf(0, 0); ra.Sop = (__nv_bfloat16*)Sop(0, 0);
       ra.y = (__nv_bfloat16*)y; ra.ldy = H; ra.sT = sT;
       ra.flags = sc<unsigned>(off_flags);
       CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
-      rhn_rec_fwd_launch(g64.mapA, g64.mapB, ra, st);
+      // phase trace of the persistent chain (diagnostics; tests/scratch only): env ASTRA_RHN_TRACE=<device ptr>
+      if (const char* tr = std::getenv("ASTRA_RHN_TRACE")) ra.trace = (unsigned long long*)std::strtoull(tr, nullptr, 0);
+      rhn_rec_fwd_launch(mA, mB, ra, st);
       for (int t = 0; t < T; ++t) fwd_step_done(t, st);
       mark(R_FWD, 1, st);
       fwd_done = true;
