@@ -153,7 +153,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           wait_flag(a.flags + m_blk, (unsigned)(a.num_n * q));
           fence_proxy_async_global();
         }
-        if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 0] = global_ns();
+        if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 0] = global_ns();
         for (int kb = 0; kb < pre; ++kb) {
           const int s = (int)((it + kb) % stages);
           sm100::tma_load_3d(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
@@ -176,14 +176,23 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       for (int q = 0; q < nsteps; ++q) {
         mbar_wait_idle(tempty, (uint32_t)(q & 1) ^ 1);
         sm100::tc_fence_after();
-        for (int kb = 0; kb < nk; ++kb, ++it) {
-          const int s = (int)(it % stages);
+        // Chunk-interleaved issue order (independent accumulators; within a chunk the k order is the
+        // canonical accumulation, R33) is kept as an option for a future A path that lands faster.
+        // (measured: interleaving the chunks slowed the k loop, 5.25 → 6.25 µs at cfg3 — the loop
+        // waits on A arriving, not on accumulator dependencies — so chunks are issued in order)
+        const bool inter = false;
+        const int nr = inter ? a.nsplit * kper : nk;   // (chunk, k) pairs; the last chunk may be shorter
+        for (int r = 0; r < nr; ++r) {
+          const int kb = inter ? (r % a.nsplit) * kper + r / a.nsplit : r;
+          if (kb >= nk) continue;
+          const long i2 = it + kb;
+          const int s = (int)(i2 % stages);
           const int c = kb / kper;                         // canonical split-K chunk (R33)
           const uint32_t d_tmem = tmem_base + c * RH_BN;
-          sm100::mbar_wait(&full[s], (uint32_t)((it / stages) & 1));
+          sm100::mbar_wait(&full[s], (uint32_t)((i2 / stages) & 1));
           sm100::tc_fence_after();
-          if (a.trace && kb == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 1] = global_ns();
-          if (a.trace && kb == nk - 1) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 2] = global_ns();
+          if (a.trace && r == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 1] = global_ns();
+          if (a.trace && r == nr - 1) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 2] = global_ns();
           // a_rows = 64: the M = 128 MMA's rows 64..127 read the B tile's bytes — garbage rows of
           // TMEM that the epilogue never reads (rows ≥ B)
           const uint32_t sa = sm100::smem_u32(smem + s * stage_bytes);
@@ -195,6 +204,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
                              (kb != c * kper || kk != 0) ? 1u : 0u);
           sm100::umma_commit(&empty[s]);
         }
+        it += nk;
         sm100::umma_commit(tfull);
       }
     }
@@ -210,7 +220,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       const bool last = l == L - 1;
       sm100::mbar_wait(tfull, (uint32_t)(q & 1));
       sm100::tc_fence_after();
-      if (a.trace && warp == 2 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 3] = global_ns();
+      if (a.trace && warp == 2 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 3] = global_ns();
       const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16);
       const float* bl = bls + l * RH_BN;
       const size_t slot_out = last ? (size_t)(t + 1) * a.B * a.Hp : ((size_t)(l + 1) * (a.T + 1) + t) * a.B * a.Hp;
@@ -244,34 +254,53 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
             zt[i] = __fadd_rn(zt[i], pt[i]);
           }
         }
-        if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 5] = global_ns();
+        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + (uc == 0 ? 5 : 11)] = global_ns();
         if (!valid) continue;
         __nv_bfloat16* so = a.Sop + slot_out + (size_t)m * a.Hp + u0 + ul;
-        float sv[16];
+        // every shared-memory operand into registers first, results out after: the buffers share
+        // one base, so interleaved loads and stores would serialise the 16 units' dependency chains
+        float sv[16], bh[16], bt[16];
 #pragma unroll
-        for (int i = 0; i < 16; ++i) sv[i] = spr[ul + i];
+        for (int i = 0; i < 16; ++i) {
+          sv[i] = spr[ul + i];
+          bh[i] = bl[ul + i];
+          bt[i] = bl[RH_UB + ul + i];
+        }
         float snew[16];
 #pragma unroll
         for (int i = 0; i < 16; ++i) {
           const int j = u0 + ul + i;
           float s_new = 0.f, aH = 0.f, aT = 0.f;
           if (j < a.H) {
-            aH = __fadd_rn(zh[i], bl[ul + i]);
-            aT = __fadd_rn(zt[i], bl[RH_UB + ul + i]);
+            aH = __fadd_rn(zh[i], bh[i]);
+            aT = __fadd_rn(zt[i], bt[i]);
             if (l == 0) {
               aH = __fadd_rn(aH, xh[i]);
               aT = __fadd_rn(aT, xt[i]);
             }
             const float h = tanh_<true>(aH), tau = sigm<true>(aT);
             s_new = __fadd_rn(__fmul_rn(h, tau), __fmul_rn(sv[i], __fsub_rn(1.f, tau)));
-            if (last && a.y) a.y[((size_t)t * a.B + m) * a.ldy + j] = __float2bfloat16_rn(s_new);
-            if (last && t == a.T - 1 && a.sT) a.sT[(size_t)m * a.H + j] = s_new;
           }
-          zr[ul + i] = aH;            // pre-activations for BPTT (padding units: 0),
-          zr[RH_UB + ul + i] = aT;    // stored after the publish
+          zh[i] = aH;   // pre-activations for BPTT (padding units: 0), stored after the publish
+          zt[i] = aT;
           snew[i] = s_new;
-          spr[ul + i] = s_new;   // s^ℓ: the next micro-step's s^{ℓ−1} of this row and unit
         }
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          spr[ul + i] = snew[i];   // s^ℓ: the next micro-step's s^{ℓ−1} of this row and unit
+          zr[ul + i] = zh[i];
+          zr[RH_UB + ul + i] = zt[i];
+        }
+        if (last) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            const int j = u0 + ul + i;
+            if (j >= a.H) break;
+            if (a.y) a.y[((size_t)t * a.B + m) * a.ldy + j] = __float2bfloat16_rn(snew[i]);
+            if (t == a.T - 1 && a.sT) a.sT[(size_t)m * a.H + j] = snew[i];
+          }
+        }
+        if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 9] = global_ns();
         uint4 pk[2];
         uint32_t* pu = reinterpret_cast<uint32_t*>(pk);
 #pragma unroll
@@ -281,18 +310,19 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         }
         reinterpret_cast<uint4*>(so)[0] = pk[0];
         reinterpret_cast<uint4*>(so)[1] = pk[1];
+        if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 10] = global_ns();
       }
       sm100::tc_fence_before();
       sm100::mbar_arrive(tempty);
-      if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 6] = global_ns();
+      if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 6] = global_ns();
       if (q + 1 < nsteps) {   // publish s^ℓ of this tile to the row block: every writer orders its
         fence_proxy_async_global();   // stores before the readers' TMA (async proxy); the CTA barrier
-        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 7] = global_ns();
+        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 7] = global_ns();
         epi_bar();                    // and one release add (cumulative) publish them at gpu scope
-        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 8] = global_ns();
+        if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 8] = global_ns();
         if (warp == 2 && lane == 0) {
           red_release_gpu(a.flags + m_blk, 1u);
-          if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 9 + 4] = global_ns();
+          if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 4] = global_ns();
         }
       }
       // off the critical path: the fp32 state and the pre-activations, read only by the backward

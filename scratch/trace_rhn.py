@@ -11,13 +11,13 @@ c.tune_mode(A.TUNE_FROZEN, "fwd=1")
 x = (torch.rand(T, B, I, device="cuda") * 2 - 1).to(torch.bfloat16)
 y = torch.empty(T, B, H, dtype=torch.bfloat16, device="cuda")
 Hp = 832; G = Hp // 32; N = T * L
-tr = torch.zeros(G * N * 9, dtype=torch.int64, device="cuda")
+tr = torch.zeros(G * N * 12, dtype=torch.int64, device="cuda")
 for _ in range(2): c.forward(x, None, None, y)
 torch.cuda.synchronize()
 os.environ["ASTRA_RHN_TRACE"] = str(tr.data_ptr())
 c.forward(x, None, None, y)
 torch.cuda.synchronize()
-t = tr.cpu().numpy().reshape(G, N, 9).astype(np.float64) / 1e3   # us
+t = tr.cpu().numpy().reshape(G, N, 12).astype(np.float64) / 1e3   # us
 q = np.arange(1, N)
 flag = t[:, 1:, 0] - t[:, :-1, 4]            # own release -> flag observed for the next step
 a_lat = t[:, :, 1] - t[:, :, 0]              # flag observed -> first A+B stage landed
@@ -29,6 +29,8 @@ prop = t[:, 1:, 0] - lastrel[None, :]        # last CTA's release -> this CTA se
 step = np.diff(t[0, :, 0])
 tm = t[:, :-1, :]
 extra = [("epi: tfull->tmem chunk0", tm[:, :, 5] - tm[:, :, 3]), ("epi: chunk0 tmem -> loop end", tm[:, :, 6] - tm[:, :, 5]),
+         ("epi: chunk0 compute", tm[:, :, 9] - tm[:, :, 5]), ("epi: chunk0 so stores", tm[:, :, 10] - tm[:, :, 9]),
+         ("epi: chunk1 tmem", tm[:, :, 11] - tm[:, :, 10]), ("epi: chunk1 rest", tm[:, :, 6] - tm[:, :, 11]),
          ("epi: fence.proxy.async", tm[:, :, 7] - tm[:, :, 6]), ("epi: bar.sync", tm[:, :, 8] - tm[:, :, 7]),
          ("epi: red.release", tm[:, :, 4] - tm[:, :, 8])]
 for name, v in extra:
