@@ -82,6 +82,40 @@ def main():
             ms = timed(lambda: g.replay())
             chain[f"graph_pdl{pdl}_b{blocks}"] = round(ms * 1e3 / n, 3)
     out["launch_chain_us_per_kernel"] = chain
+    # K11p: the rank-ordered reduce kernel with N simulated ranks on this device (local HBM, not
+    # NVLink): one round reads every rank's cfg5-sized gradient buffer once and writes it once
+    n = 34_640_000   # cfg5 flat gradient (139 MB)
+    k11p = {}
+    seq = 1
+    for world in (2, 4, 8):
+        bufs = [torch.rand(n, device="cuda") for _ in range(world)]
+        sigs = [torch.zeros(1024, dtype=torch.int32, device="cuda") for _ in range(world)]
+        streams = [torch.cuda.Stream() for _ in range(world)]
+        bp = (ctypes.c_void_p * world)(*[b.data_ptr() for b in bufs])
+        sgp = (ctypes.c_void_p * world)(*[g.data_ptr() for g in sigs])
+        stp = (ctypes.c_void_p * world)(*[x.cuda_stream for x in streams])
+        reps = 5
+
+        def run(r=reps):
+            nonlocal seq
+            e0 = torch.cuda.Event()
+            e0.record(st)
+            for x in streams:
+                x.wait_event(e0)
+            A._check(L.astra_micro_peer_reduce(ctypes.cast(bp, ctypes.c_void_p), ctypes.cast(sgp, ctypes.c_void_p),
+                                               world, n, r, seq, ctypes.cast(stp, ctypes.c_void_p)))
+            seq += r
+            for x in streams:
+                e = torch.cuda.Event()
+                e.record(x)
+                st.wait_event(e)
+
+        run(1)
+        ms = timed(run) / reps
+        gbs = 4.0 * n * (world + 1) / (ms / 1e3) / 1e9
+        k11p[str(world)] = {"ms_per_round": round(ms, 4), "gbs": round(gbs, 1), "frac_of_hbm": round(gbs / bw[1024], 3)}
+        del bufs
+    out["k11p_reduce_local"] = k11p
     # per-config floors of one dependent chain step (bf16 weight bytes streamed per launched GEMM)
     launch = chain["graph_pdl1_b148"]
 

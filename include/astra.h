@@ -265,6 +265,14 @@ astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream
 /* n dependent empty kernels of `blocks` CTAs, launched with programmatic dependent launch
  * (pdl = 1, as the chain kernels are) or plainly: the per-step floor of a launched chain.     */
 astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream stream);
+/* K11p's rank-ordered reduce kernel for `world` simulated ranks on one device: bufs[r] (device
+ * fp32 [n]) is rank r's gradient buffer, sigs[r] a zeroed device array of 4096 bytes (the signal
+ * slots), streams[r] its stream.  Each of `reps` rounds launches rank r's kernel on streams[r] with
+ * sequence number seq0 + round (must exceed every value used before on these sigs): rank r writes
+ * (Σ_q bufs[q][i]) / world, q in rank order, into bufs[r][i] for its shard.  The production kernel
+ * and barrier protocol, reading local HBM instead of NVLink (a measure of the kernel itself).     */
+astra_status astra_micro_peer_reduce(float* const* bufs, unsigned* const* sigs, int world, size_t n, int reps,
+                                     unsigned seq0, const astra_stream* streams);
 
 /* ---- host-only test hooks (no GPU) ------------------------------------------------------ */
 /* Drive the tuner's update tree on a fake clock.  `tree` is an s-expression, e.g.

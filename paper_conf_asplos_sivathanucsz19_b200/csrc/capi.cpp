@@ -22,6 +22,8 @@ namespace astra {   // kernels/micro.cu
 void micro_stream_read(const void* buf, size_t bytes, int passes, float* sink, cudaStream_t st);
 void micro_grid_barrier(unsigned* counter, int iters, cudaStream_t st);
 void micro_launch_chain(int n, int pdl, int blocks, cudaStream_t st);
+void micro_peer_reduce(float* const* bufs, uint32_t* const* sigs, int world, size_t n, int reps, uint32_t seq0,
+                       const cudaStream_t* streams);
 }  // namespace astra
 
 struct astra_cell_s {
@@ -438,6 +440,13 @@ astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream
 
 astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream stream) {
   return guard([&] { micro_launch_chain(n, pdl, blocks, (cudaStream_t)stream); });
+}
+
+astra_status astra_micro_peer_reduce(float* const* bufs, unsigned* const* sigs, int world, size_t n, int reps,
+                                     unsigned seq0, const astra_stream* streams) {
+  return guard([&] {
+    micro_peer_reduce(bufs, (uint32_t* const*)sigs, world, n, reps, seq0, (const cudaStream_t*)streams);
+  });
 }
 
 astra_status astra_region_times(astra_cell c, double* out, int cap, int* n) {

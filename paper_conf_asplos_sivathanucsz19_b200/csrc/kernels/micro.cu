@@ -10,6 +10,7 @@
 #include "../common.h"
 #include "gemm.h"
 #include "pdl.cuh"
+#include "peer.h"
 
 namespace astra {
 
@@ -80,6 +81,33 @@ void micro_launch_chain(int n, int pdl, int blocks, cudaStream_t st) {
     else empty_kernel<<<blocks, 128, 0, st>>>(i);
     LAUNCH_CHECK();
   }
+}
+
+}  // namespace astra
+
+// K11p's reduce kernel with `world` ranks simulated on one device: rank r's launch on streams[r]
+// reads shard r of every rank's buffer (all local HBM here) and writes the rank-ordered mean into
+// buffer r — the production kernel and barrier protocol, without NVLink.  Measures the kernel's
+// own efficiency against the HBM roofline (the NVLink-bound case needs a multi-GPU box).
+namespace astra {
+void micro_peer_reduce(float* const* bufs, uint32_t* const* sigs, int world, size_t n, int reps, uint32_t seq0,
+                       const cudaStream_t* streams) {
+  ASTRA_CHECK_ARG(bufs && sigs && streams && world >= 1 && world <= PEER_MAX_WORLD && n > 0 && reps > 0,
+                  "micro_peer_reduce: bad arguments");
+  PeerPtrs a{};
+  a.world = world;
+  for (int q = 0; q < world; ++q) {
+    a.g[q] = bufs[q];
+    a.p[q] = bufs[q];
+    a.sig[q] = sigs[q];
+  }
+  for (int it = 0; it < reps; ++it)
+    for (int r = 0; r < world; ++r) {
+      a.rank = r;
+      size_t lo, hi;
+      peer_shard(0, n, r, world, &lo, &hi);
+      peer_reduce(a, lo, hi, seq0 + (uint32_t)it, 1.0f / (float)world, 32, 60LL * 1000 * 1000 * 1000, streams[r]);
+    }
 }
 
 }  // namespace astra
