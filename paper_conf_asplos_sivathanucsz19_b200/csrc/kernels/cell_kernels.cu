@@ -10,6 +10,7 @@
 #include "gemm.h"
 #include "sm100.cuh"
 #include <algorithm>
+#include <cstdlib>
 
 namespace astra {
 
@@ -161,7 +162,14 @@ struct FwdPwArgs {
   long ldy;
   float* hT;
   float* cT;
+  unsigned long long* trace;   // diagnostics (ASTRA_FWDPW_TRACE): [grid][2 + 2·16] globaltimer stamps
 };
+
+__device__ __forceinline__ unsigned long long gtime_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
 
 template <typename T>
 __device__ __forceinline__ void store_pair(T* p, bool vec, float a, float b, bool ok1) {
@@ -201,6 +209,8 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
     const long b = b_first + (long)k * a.rstep;
     sm100::bulk_load(sm100::smem_u32(sm + s * FB_STAGE + FB_SW), a.UH + b * NG + (long)u0 * 4, wbytes, &full[s]);
   };
+  unsigned long long* tr = a.trace ? a.trace + (size_t)blockIdx.x * 34 : nullptr;
+  if (tr && tid == 0) tr[0] = gtime_ns();
   if (tid == 0) {
     for (int s = 0; s < FB_STAGES; ++s) sm100::mbar_init(&full[s], 1);
     sm100::fence_barrier_init();
@@ -208,6 +218,7 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   }
   pdl_wait();
   pdl_trigger();
+  if (tr && tid == 0) tr[1] = gtime_ns();
   if (tid == 0)
     for (int k = 0; k < FB_STAGES && k < nitems; ++k) issue_new(k);
   for (int i = tid; i < 4 * nu; i += FB_THREADS) {
@@ -240,6 +251,7 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   for (int k = 0; k < nitems; ++k) {
     const int s = k % FB_STAGES;
     sm100::mbar_wait(&full[s], (uint32_t)((k / FB_STAGES) & 1));
+    if (tr && tid == 0 && k < 16) tr[2 + 2 * k] = gtime_ns();
     const long b = b_first + (long)k * a.rstep;
     if (act) {
       const float* sw = reinterpret_cast<const float*>(sm + s * FB_STAGE);
@@ -283,6 +295,7 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
       }
     }
     __syncthreads();   // stage s fully consumed
+    if (tr && tid == 0 && k < 16) tr[3 + 2 * k] = gtime_ns();
     if (tid == 0 && k + FB_STAGES < nitems) {
       sm100::fence_proxy_async_smem();
       issue_old(k + FB_STAGES);
@@ -301,6 +314,8 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
   a.rstep = std::max(1, std::min(B, 2 * num_sms() / a.nub));
   a.WX = WX; a.UH = UH; a.gp = gp; a.c_prev = c_prev; a.c_new = c_new;
   a.h_op = h_op; a.ldh = ldh; a.y = y; a.ldy = ldy; a.hT = hT; a.cT = cT;
+  static const char* tr_env = std::getenv("ASTRA_FWDPW_TRACE");   // diagnostics only
+  a.trace = tr_env ? (unsigned long long*)std::strtoull(tr_env, nullptr, 0) : nullptr;
   const int np = KIND == K_MILSTM ? 4 : 1;
   const size_t smem = (size_t)FB_STAGES * FB_STAGE + (size_t)np * 4 * FB_UB * 4 + FB_STAGES * 8;
   const dim3 grid(a.nub * a.rstep);
