@@ -273,6 +273,13 @@ astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream s
  * and barrier protocol, reading local HBM instead of NVLink (a measure of the kernel itself).     */
 astra_status astra_micro_peer_reduce(float* const* bufs, unsigned* const* sigs, int world, size_t n, int reps,
                                      unsigned seq0, const astra_stream* streams);
+/* Diagnostic phase traces (globaltimer stamps, ns) written by instrumented kernels into a caller
+ * device buffer; NULL turns a trace off (the default).  kind 0: the forward pointwise kernel of the
+ * LSTM family, per CTA [2 + 2·16] stamps (entry, grid-dependency wait done, then per row: operands
+ * ready, row done); kind 1: the persistent fused RHN forward, per CTA and micro-step [12] stamps
+ * (scratch/trace_fwdpw.py, scratch/trace_rhn.py read them).  The buffer must be large enough for
+ * the next launch of that kernel; E_ARG for an unknown kind.                                     */
+astra_status astra_debug_set_trace(int kind, void* device_buffer);
 
 /* ---- host-only test hooks (no GPU) ------------------------------------------------------ */
 /* Drive the tuner's update tree on a fake clock.  `tree` is an s-expression, e.g.

@@ -442,6 +442,10 @@ astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream s
   return guard([&] { micro_launch_chain(n, pdl, blocks, (cudaStream_t)stream); });
 }
 
+astra_status astra_debug_set_trace(int kind, void* device_buffer) {
+  return guard([&] { set_trace_buffer(kind, (unsigned long long*)device_buffer); });
+}
+
 astra_status astra_micro_peer_reduce(float* const* bufs, unsigned* const* sigs, int world, size_t n, int reps,
                                      unsigned seq0, const astra_stream* streams) {
   return guard([&] {

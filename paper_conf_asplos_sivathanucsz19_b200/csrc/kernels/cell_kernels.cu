@@ -162,7 +162,7 @@ struct FwdPwArgs {
   long ldy;
   float* hT;
   float* cT;
-  unsigned long long* trace;   // diagnostics (ASTRA_FWDPW_TRACE): [grid][2 + 2·16] globaltimer stamps
+  unsigned long long* trace;   // diagnostics (astra_debug_set_trace): [grid][2 + 2·16] globaltimer stamps
 };
 
 __device__ __forceinline__ unsigned long long gtime_ns() {
@@ -314,8 +314,7 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
   a.rstep = std::max(1, std::min(B, 2 * num_sms() / a.nub));
   a.WX = WX; a.UH = UH; a.gp = gp; a.c_prev = c_prev; a.c_new = c_new;
   a.h_op = h_op; a.ldh = ldh; a.y = y; a.ldy = ldy; a.hT = hT; a.cT = cT;
-  static const char* tr_env = std::getenv("ASTRA_FWDPW_TRACE");   // diagnostics only
-  a.trace = tr_env ? (unsigned long long*)std::strtoull(tr_env, nullptr, 0) : nullptr;
+  a.trace = trace_buffer(TRACE_FWD_PW);   // diagnostics only (null: no stamps)
   const int np = KIND == K_MILSTM ? 4 : 1;
   const size_t smem = (size_t)FB_STAGES * FB_STAGE + (size_t)np * 4 * FB_UB * 4 + FB_STAGES * 8;
   const dim3 grid(a.nub * a.rstep);
@@ -349,6 +348,13 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
   FWD_CASE(K_SUBLSTM)
 #undef FWD_CASE
   throw Error(ASTRA_E_UNSUPPORTED, "lstm_fwd_pointwise: kind");
+}
+
+static unsigned long long* g_trace[TRACE_KINDS] = {nullptr, nullptr};
+unsigned long long* trace_buffer(int kind) { return kind >= 0 && kind < TRACE_KINDS ? g_trace[kind] : nullptr; }
+void set_trace_buffer(int kind, unsigned long long* buf) {
+  ASTRA_CHECK_ARG(kind >= 0 && kind < TRACE_KINDS, "debug_set_trace: unknown kind");
+  g_trace[kind] = buf;
 }
 
 int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }

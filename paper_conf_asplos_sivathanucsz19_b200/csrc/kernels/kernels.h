@@ -8,6 +8,12 @@
 
 namespace astra {
 
+// Diagnostic phase traces (astra_debug_set_trace): device buffers of globaltimer stamps written by
+// instrumented kernels when set; null (the default) disables the stamps.
+enum TraceKind { TRACE_FWD_PW = 0, TRACE_RHN_FWD = 1, TRACE_KINDS };
+unsigned long long* trace_buffer(int kind);
+void set_trace_buffer(int kind, unsigned long long* buf);
+
 struct GateParams {          // external-layout fp32 vectors of length 4H (may be null for LSTM)
   const float* b = nullptr;
   const float* alpha = nullptr;

@@ -94,7 +94,7 @@ struct RhnFwdArgs {
   long ldy;
   float* sT;                // optional [B][H]
   unsigned* flags;          // [num_m] row-block counters, zeroed before the launch
-  unsigned long long* trace;   // optional (ASTRA_RHN_TRACE): [grid][T·L][5] globaltimer stamps
+  unsigned long long* trace;   // optional (astra_debug_set_trace): [grid][T·L][12] globaltimer stamps
 };
 bool rhn_rec_fwd_supported(int B, int Hp, int nsplit);
 // mapA: the bf16 state operands as a 3-D K-major map (inner Hp, rows B, z = L·(T+1)), box {64, a_rows};

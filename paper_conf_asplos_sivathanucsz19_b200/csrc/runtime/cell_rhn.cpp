@@ -147,8 +147,7 @@ class RhnCell : public Cell {
       ra.y = (__nv_bfloat16*)y; ra.ldy = H; ra.sT = sT;
       ra.flags = sc<unsigned>(off_flags);
       CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
-      // phase trace of the persistent chain (diagnostics; tests/scratch only): env ASTRA_RHN_TRACE=<device ptr>
-      if (const char* tr = std::getenv("ASTRA_RHN_TRACE")) ra.trace = (unsigned long long*)std::strtoull(tr, nullptr, 0);
+      ra.trace = trace_buffer(TRACE_RHN_FWD);   // phase trace of the persistent chain (diagnostics)
       rhn_rec_fwd_launch(mA, mB, ra, st);
       for (int t = 0; t < T; ++t) fwd_step_done(t, st);
       mark(R_FWD, 1, st);

@@ -7,7 +7,7 @@ def main():
     import paper_conf_asplos_sivathanucsz19_b200 as A
     T, B, H, I, V = 100, 512, 2048, 2048, 256
     buf = torch.zeros(400 * 34, dtype=torch.int64, device="cuda")
-    os.environ["ASTRA_FWDPW_TRACE"] = str(buf.data_ptr())
+    A._check(A.lib().astra_debug_set_trace(0, A._ptr(buf)))
     cell = A.Cell("milstm", H, I, B, T, dtype="bf16")
     lm = A.LM(cell, V)
     lm.load(bench.make_params(I, H, V))

@@ -14,7 +14,7 @@ Hp = 832; G = Hp // 32; N = T * L
 tr = torch.zeros(G * N * 12, dtype=torch.int64, device="cuda")
 for _ in range(2): c.forward(x, None, None, y)
 torch.cuda.synchronize()
-os.environ["ASTRA_RHN_TRACE"] = str(tr.data_ptr())
+A._check(A.lib().astra_debug_set_trace(1, A._ptr(tr)))
 c.forward(x, None, None, y)
 torch.cuda.synchronize()
 t = tr.cpu().numpy().reshape(G, N, 12).astype(np.float64) / 1e3   # us

@@ -92,6 +92,8 @@ def test_bad_arguments_are_rejected():
     assert L.astra_comm_peer_init(c.h, buf, 0, 2) == 3                          # E_STATE: no handle yet
     assert L.astra_comm_peer_handle(c.h, buf, 16) in (1, 3)
     assert L.astra_comm_peer_handle(c.h, None, 256) == 1                        # E_ARG: null buffer
+    assert L.astra_debug_set_trace(7, None) == 1                                # E_ARG: unknown trace kind
+    assert L.astra_debug_set_trace(0, None) == 0                                # tracing off
 
 
 def test_tune_report_is_json():
