@@ -39,6 +39,22 @@ template <typename T> __device__ __forceinline__ T from_f(float v);
 template <> __device__ __forceinline__ float from_f<float>(float v) { return v; }
 template <> __device__ __forceinline__ __nv_bfloat16 from_f<__nv_bfloat16>(float v) { return __float2bfloat16_rn(v); }
 
+// p[0] + p[s] + ... + p[(n−1)·s] summed in chunk order (the R25 / R33 split-K partials).  The loads
+// of the first SPLIT_MAX partials are issued together (predicated) before the ordered adds, so a row
+// waits one memory latency instead of n dependent ones; the sum and its rounding order are unchanged.
+constexpr int SPLIT_MAX = 4;   // R25 and R33 never split further
+__device__ __forceinline__ float sum_split(const float* __restrict__ p, int n, long s) {
+  float v[SPLIT_MAX];
+#pragma unroll
+  for (int k = 0; k < SPLIT_MAX; ++k) v[k] = k < n ? p[k * s] : 0.f;
+  float r = v[0];
+#pragma unroll
+  for (int k = 1; k < SPLIT_MAX; ++k)
+    if (k < n) r = __fadd_rn(r, v[k]);
+  for (int k = SPLIT_MAX; k < n; ++k) r = __fadd_rn(r, p[k * s]);
+  return r;
+}
+
 enum CellKind { K_LSTM = 0, K_MILSTM = 1, K_SUBLSTM = 5 };
 
 // Pre-activation of one gate.  LSTM/subLSTM: a = wx + uh + b.

@@ -67,8 +67,7 @@ __global__ void scrn_fwd_pw_kernel(int B, int H, int Hp, const float* __restrict
   if (j >= Hp) return;
   float h = 0.f;
   if (j < H) {
-    float z = Z[(long)b * Hp + j];   // reading R33: split-K partials of h_{t-1}·R summed in chunk order
-    for (int k = 1; k < nsplit; ++k) z = __fadd_rn(z, Z[k * split_stride + (long)b * Hp + j]);
+    const float z = sum_split(Z + (long)b * Hp + j, nsplit, split_stride);   // reading R33: chunk order
     h = sigm<FastMath<T>::value>(__fadd_rn(__fadd_rn(Q[(long)b * ldq + j], z), bh[j]));
   }
   Hf[(long)b * Hp + j] = h;
@@ -112,9 +111,7 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
       if (j < H) {
         float g = to_f<TDY>(dy[(long)b * ldy + j]);
         if (dh) {   // reading R33: split-K partials of dz·Rᵀ summed in chunk order, then added to dy
-          float r = dh[(long)b * ld_dh + j];
-          for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, dh[k * split_stride + (long)b * ld_dh + j]);
-          g = __fadd_rn(g, r);
+          g = __fadd_rn(g, sum_split(dh + (long)b * ld_dh + j, nsplit, split_stride));
         }
         const float h = Hf[(long)b * Hp + j];
         dz = __fmul_rn(__fmul_rn(g, h), __fsub_rn(1.f, h));
@@ -214,12 +211,8 @@ __global__ void rhn_fwd_pw_kernel(int B, int H, int Hp, float* __restrict__ Z, c
   if (j < H) {
     float zH, zT;
     if (Zpart) {   // reading R33: the recurrent GEMM's split-K partials summed in chunk order
-      zH = Zpart[rz + j];
-      zT = Zpart[rz + Hp + j];
-      for (int k = 1; k < nsplit; ++k) {
-        zH = __fadd_rn(zH, Zpart[k * split_stride + rz + j]);
-        zT = __fadd_rn(zT, Zpart[k * split_stride + rz + Hp + j]);
-      }
+      zH = sum_split(Zpart + rz + j, nsplit, split_stride);
+      zT = sum_split(Zpart + rz + Hp + j, nsplit, split_stride);
     } else {
       zH = Z[rz + j];
       zT = Z[rz + Hp + j];
@@ -278,10 +271,7 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
       if (j < H) {
         float ds = ds_in[(long)b * Hp + j];
         if (ds_part) {   // reading R33: carry + the BPTT GEMM's split-K partials summed in chunk order
-          const float* q = ds_part + (long)b * Hp + j;
-          float r = q[0];
-          for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, q[k * split_stride]);
-          ds = __fadd_rn(ds, r);
+          ds = __fadd_rn(ds, sum_split(ds_part + (long)b * Hp + j, nsplit, split_stride));
         }
         if (dy) ds = __fadd_rn(to_f<TDY>(dy[(long)b * ldy + j]), ds);
         const float h = tanh_<FastMath<T>::value>(Apre[rz + j]), tau = sigm<FastMath<T>::value>(Apre[rz + Hp + j]);
