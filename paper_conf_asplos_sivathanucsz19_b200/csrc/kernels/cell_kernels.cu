@@ -372,11 +372,19 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
                        const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
                        T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
   constexpr int NV = BwdNV<KIND>::value;
+  constexpr int NP = KIND == K_MILSTM ? 4 : 1;   // gate parameter sets: b (and α, β1, β2)
   __shared__ float red[BWD_RY][NV][BWD_UX];
-  pdl_wait();
-  pdl_trigger();
+  __shared__ float sgp[NP][4][BWD_UX];   // staged once; re-read per row so they hold no registers
   const int tx = threadIdx.x, ty = threadIdx.y;
   const int j = blockIdx.x * BWD_UX + tx;
+  if (ty < NP) {   // parameters are not written by the chain: staged before the grid dependency
+    const float* src = ty == 0 ? gp.b : ty == 1 ? gp.alpha : ty == 2 ? gp.beta1 : gp.beta2;
+#pragma unroll
+    for (int g = 0; g < 4; ++g) sgp[ty][g][tx] = j < H ? src[g * H + j] : 0.f;
+  }
+  pdl_wait();
+  pdl_trigger();
+  __syncthreads();
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
@@ -384,18 +392,10 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
 #pragma unroll
   for (int i = 0; i < NV; ++i) acc[i] = 0.f;
   if (j < H) {
-    float bb[4], al[4], be1[4], be2[4];
-#pragma unroll
-    for (int g = 0; g < 4; ++g) {
-      const int e = g * H + j;
-      bb[g] = gp.b[e];
-      al[g] = KIND == K_MILSTM ? gp.alpha[e] : 0.f;
-      be1[g] = KIND == K_MILSTM ? gp.beta1[e] : 0.f;
-      be2[g] = KIND == K_MILSTM ? gp.beta2[e] : 0.f;
-    }
     const int c0 = gcol(0, j);
 #pragma unroll 1
     for (int b = b0 + ty; b < b1; b += BWD_RY) {
+      // every operand of the row is loaded before any arithmetic: one memory latency per row
       const float* wxp = WX + (long)b * NG + c0;
       const float* uhp = UH + (long)b * NG + c0;
       float w[4], h[4];
@@ -404,16 +404,22 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
         w[g] = __ldcs(wxp + g * GATE_U);
         h[g] = __ldcs(uhp + g * GATE_U);
       }
-      float dh = to_f<TDY>(dy[(long)b * ldy + j]);
-      if (dh_rec) {   // split-K partials of dh_rec summed in chunk order, then added to dy
-        const float* r0 = dh_rec + (long)b * ld_dh + j;
-        float r = r0[0];
-        for (int k = 1; k < nsplit; ++k) r = __fadd_rn(r, r0[k * split_stride]);
-        dh = __fadd_rn(dh, r);
-      }
       const long ro = (long)b * Hp + j;
       float dcv = dc[ro];
-      lstm_bwd_row<KIND, T>(w, h, dh, dcv, c_prev[ro], c_new[ro], bb, al, be1, be2, acc, D_uh + (long)b * NG + c0,
+      const float cp = c_prev[ro], cn = c_new[ro];
+      float dh = to_f<TDY>(dy[(long)b * ldy + j]);
+      if (dh_rec)   // split-K partials of dh_rec summed in chunk order, then added to dy
+        dh = __fadd_rn(dh, sum_split(dh_rec + (long)b * ld_dh + j, nsplit, split_stride));
+      float bb[4], al[4], be1[4], be2[4];
+      const volatile float* sg = &sgp[0][0][tx];   // volatile: re-read each row, not hoisted into registers
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        bb[g] = sg[g * BWD_UX];
+        al[g] = KIND == K_MILSTM ? sg[(NP > 1 ? 4 : 0) * BWD_UX + g * BWD_UX] : 0.f;
+        be1[g] = KIND == K_MILSTM ? sg[(NP > 2 ? 8 : 0) * BWD_UX + g * BWD_UX] : 0.f;
+        be2[g] = KIND == K_MILSTM ? sg[(NP > 3 ? 12 : 0) * BWD_UX + g * BWD_UX] : 0.f;
+      }
+      lstm_bwd_row<KIND, T>(w, h, dh, dcv, cp, cn, bb, al, be1, be2, acc, D_uh + (long)b * NG + c0,
                             D_wx + (long)b * NG + c0);
       dc[ro] = dcv;
     }
