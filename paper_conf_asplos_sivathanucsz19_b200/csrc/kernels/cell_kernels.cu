@@ -382,32 +382,45 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
 #pragma unroll
     for (int g = 0; g < 4; ++g) sgp[ty][g][tx] = j < H ? src[g * H + j] : 0.f;
   }
-  pdl_wait();
-  pdl_trigger();
-  __syncthreads();
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
+  const int c0 = gcol(0, j);
+  // Operands of one row.  Only dh_rec is produced by the predecessor (the BPTT GEMM); WX, UH, the
+  // cell states and dy are older, and dc was written by the pointwise kernel two launches back
+  // (complete: the GEMM waits on it before triggering this launch).  So the first row is loaded
+  // before the grid dependency resolves — by the CTAs already resident beside the GEMM.  Not at the
+  // first step (`first`): its predecessor may be the kernel that initialised dc or produced dy.
+  const bool early = !first;
+  float w[4], h[4], dcv = 0.f, cp = 0.f, cn = 0.f, dyv = 0.f;
+  auto load_row = [&](int b) {
+    const float* wxp = WX + (long)b * NG + c0;
+    const float* uhp = UH + (long)b * NG + c0;
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      w[g] = __ldcs(wxp + g * GATE_U);
+      h[g] = __ldcs(uhp + g * GATE_U);
+    }
+    const long ro = (long)b * Hp + j;
+    dcv = dc[ro];
+    cp = c_prev[ro];
+    cn = c_new[ro];
+    dyv = to_f<TDY>(dy[(long)b * ldy + j]);
+  };
+  if (early && j < H && b0 + ty < b1) load_row(b0 + ty);
+  pdl_wait();
+  pdl_trigger();
+  __syncthreads();
   float acc[NV];
 #pragma unroll
   for (int i = 0; i < NV; ++i) acc[i] = 0.f;
   if (j < H) {
-    const int c0 = gcol(0, j);
 #pragma unroll 1
     for (int b = b0 + ty; b < b1; b += BWD_RY) {
       // every operand of the row is loaded before any arithmetic: one memory latency per row
-      const float* wxp = WX + (long)b * NG + c0;
-      const float* uhp = UH + (long)b * NG + c0;
-      float w[4], h[4];
-#pragma unroll
-      for (int g = 0; g < 4; ++g) {
-        w[g] = __ldcs(wxp + g * GATE_U);
-        h[g] = __ldcs(uhp + g * GATE_U);
-      }
+      if (!early || b != b0 + ty) load_row(b);
       const long ro = (long)b * Hp + j;
-      float dcv = dc[ro];
-      const float cp = c_prev[ro], cn = c_new[ro];
-      float dh = to_f<TDY>(dy[(long)b * ldy + j]);
+      float dh = dyv;
       if (dh_rec)   // split-K partials of dh_rec summed in chunk order, then added to dy
         dh = __fadd_rn(dh, sum_split(dh_rec + (long)b * ld_dh + j, nsplit, split_stride));
       float bb[4], al[4], be1[4], be2[4];

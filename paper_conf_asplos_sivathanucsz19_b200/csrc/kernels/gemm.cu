@@ -116,16 +116,18 @@ static uint32_t make_idesc(int BN, bool a_mn, bool b_mn, int BM = TC_BM) {
 }
 
 template <int BN>
-static int smem_for(int& stages) {
+static int smem_for(int& stages, int cap) {
   int dev = 0, maxs = 0;
   CUDA_TRY(cudaGetDevice(&dev));
   CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  if (cap > 0 && cap < maxs) maxs = cap;   // leave room for co-resident kernels (fewer stages, same bits)
   stages = TcSmem<BN>::stages_for(maxs);
+  ASTRA_CHECK_ARG(stages >= 2, "tc_gemm: shared-memory cap leaves fewer than 2 stages");
   return TcSmem<BN>::bytes(stages);
 }
 
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
-                     int cm, int cn, bool b_keep, int ksplit, int cg) {
+                     int cm, int cn, bool b_keep, int ksplit, int cg, int smem_cap) {
   ASTRA_CHECK_ARG(cg == 1 || (cg == 2 && cm == 1 && cn == 1 && BN >= 128),
                   "tc_gemm: CTA pairs (cg = 2) need BN >= 128 and no extra cluster multicast");
   ASTRA_CHECK_ARG((cm == 1 || cm == 2 || cm == 4) && (cn == 1 || cn == 2 || cn == 4) && cm * cn <= 8,
@@ -155,9 +157,9 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   g.args.idesc = make_idesc(BN, a_mn, b_mn, TC_BM * cg);
   int stages = 0;
   switch (BN / cg) {
-    case 64: g.smem = smem_for<64>(stages); break;
-    case 128: g.smem = smem_for<128>(stages); break;
-    default: g.smem = smem_for<256>(stages); break;
+    case 64: g.smem = smem_for<64>(stages, smem_cap); break;
+    case 128: g.smem = smem_for<128>(stages, smem_cap); break;
+    default: g.smem = smem_for<256>(stages, smem_cap); break;
   }
   g.args.stages = stages;
   g.ready = true;

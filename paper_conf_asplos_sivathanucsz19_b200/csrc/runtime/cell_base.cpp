@@ -191,7 +191,19 @@ TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
   auto it = tc_cache.find(key);
   if (it == tc_cache.end()) {
     TcGemm g;
-    tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit, k.cg);
+    // A/B knob: cap the shared memory of the per-step BPTT GEMM (id 2) so the backward pointwise
+    // kernel's CTAs can be resident beside it and load their first row before the grid dependency.
+    // Same for the per-step recurrent GEMM (id 1) and the forward pointwise kernel.
+    static const int bptt_cap = [] {
+      const char* e = std::getenv("ASTRA_BPTT_SMEM_KB");
+      return e ? std::atoi(e) * 1024 : 0;
+    }();
+    static const int rec_cap = [] {
+      const char* e = std::getenv("ASTRA_REC_SMEM_KB");
+      return e ? std::atoi(e) * 1024 : 0;
+    }();
+    tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit, k.cg,
+                    id == 2 ? bptt_cap : id == 1 ? rec_cap : 0);
     it = tc_cache.emplace(key, g).first;
   }
   return it->second;
