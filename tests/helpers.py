@@ -10,6 +10,14 @@ TOL_BF16 = 2e-2   # BASELINE.json north_star: bf16 GEMM operands, fp32 accumulat
 TOL_FP32 = 1e-4   # BASELINE.json north_star: fp32 path
 
 
+def golden(name):
+    """A fixture from tests/golden/ (values printed in the paper, each with its citation)."""
+    import json
+    import os
+    with open(os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", name)) as f:
+        return json.load(f)
+
+
 def rel_err(gpu, ref):
     gpu = np.asarray(gpu, dtype=np.float64)
     ref = np.asarray(ref, dtype=np.float64)

@@ -4,6 +4,9 @@ import itertools
 import pytest
 
 from oracle import tuner as TU
+from helpers import golden
+
+PAPER = golden("paper_worked_examples.json")
 
 
 def _additive_cost(tables):
@@ -20,31 +23,36 @@ def _additive_cost(tables):
 def test_parallel_exploration_worked_example_p220():
     """5 fusion groups × (3 fusion chunkings × 2 kernels): parallel exploration needs 3·2 = 6
     trials; an end-to-end one-at-a-time search over the same space needs (3·2)^5 = 7776."""
+    P = PAPER["parallel_exploration"]
+    G, NF, NK = P["groups"], P["fusion_choices"], P["kernel_choices"]
     groups = []
     tables = {}
-    for gi in range(5):
-        fus, ker = TU.Leaf(f"fuse{gi}", 3, f"g{gi}"), TU.Leaf(f"kern{gi}", 2, f"g{gi}")
+    for gi in range(G):
+        fus, ker = TU.Leaf(f"fuse{gi}", NF, f"g{gi}"), TU.Leaf(f"kern{gi}", NK, f"g{gi}")
         groups.append(TU.Exh(f"g{gi}", fus, ker))
         tables[f"g{gi}"] = [(f"fuse{gi}", [5.0 + gi, 3.0, 4.0 - 0.1 * gi]), (f"kern{gi}", [1.0, 0.5 + 0.3 * (gi % 2)])]
     tree = TU.Par(*groups)
     cost = _additive_cost(tables)
     trials, final, _ = TU.run(tree, cost)
-    assert len(trials) == 6
-    full = 1
-    for g in groups:
-        full *= 3 * 2
-    assert full == 7776
+    assert len(trials) == P["parallel_trials"]
+    # the one-at-a-time search space, counted by enumerating every joint configuration
+    full = sum(1 for _ in itertools.product(*[range(NF * NK)] * G))
+    assert full == P["mutation_trials"]
     best, _ = TU.brute_force(tree, cost, "step")
     assert final == best
 
 
 def test_equivalence_exploration_p247():
     """10 equivalent kernels on 2 streams: only the split count matters → 5 choices, not 2^10."""
-    assert len(TU.equivalence_options(10)) == 5
-    assert TU.equivalence_options(10) == [1, 2, 3, 4, 5]
-    # brute force: distinct unordered non-empty 2-stream splits of 10 identical kernels
-    splits = {tuple(sorted((k, 10 - k))) for k in range(1, 10)}
-    assert len(splits) == 5 and 2 ** 10 == 1024
+    P = PAPER["equivalence_exploration"]
+    n = P["kernels"]
+    assert len(TU.equivalence_options(n)) == P["choices"]
+    assert TU.equivalence_options(n) == [1, 2, 3, 4, 5]
+    # brute force: distinct unordered non-empty 2-stream splits of n identical kernels, against the
+    # 2^n assignments of distinguishable kernels to the streams
+    assign = list(itertools.product(range(P["streams"]), repeat=n))
+    splits = {tuple(sorted((a.count(0), a.count(1)))) for a in assign if 0 < a.count(0) < n}
+    assert len(splits) == P["choices"] and len(assign) == P["naive_space"]
 
 
 def test_prefix_exploration_is_additive_p243():

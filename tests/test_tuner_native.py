@@ -7,6 +7,7 @@ import pytest
 
 import paper_conf_asplos_sivathanucsz19_b200 as A
 from oracle import tuner as TU
+from helpers import golden
 
 
 def _to_sexpr(node):
@@ -102,16 +103,18 @@ def test_native_wirer_equals_oracle_random_trees(seed):
 
 
 def test_native_parallel_worked_example_p220():
+    P = golden("paper_worked_examples.json")["parallel_exploration"]
     groups, tables = [], {}
-    for gi in range(5):
-        groups.append(TU.Exh(f"g{gi}", TU.Leaf(f"fuse{gi}", 3, f"g{gi}"), TU.Leaf(f"kern{gi}", 2, f"g{gi}")))
+    for gi in range(P["groups"]):
+        groups.append(TU.Exh(f"g{gi}", TU.Leaf(f"fuse{gi}", P["fusion_choices"], f"g{gi}"),
+                             TU.Leaf(f"kern{gi}", P["kernel_choices"], f"g{gi}")))
         tables[gi] = ([5.0 + gi, 3.0, 4.0 - 0.1 * gi], [1.0, 0.5 + 0.3 * (gi % 2)])
 
     def cost(cfg):
-        out = {f"g{gi}": tables[gi][0][cfg[f"fuse{gi}"]] + tables[gi][1][cfg[f"kern{gi}"]] for gi in range(5)}
+        out = {f"g{gi}": tables[gi][0][cfg[f"fuse{gi}"]] + tables[gi][1][cfg[f"kern{gi}"]] for gi in range(P["groups"])}
         return out
     res = _compare(TU.Par(*groups), cost)
-    assert res["n_trials"] == 6
+    assert res["n_trials"] == P["parallel_trials"]
 
 
 def test_native_prefix_additive_p243():
