@@ -525,7 +525,40 @@ __global__ void embed_gather_kernel(const int32_t* __restrict__ tok, long n, con
   for (int c = threadIdx.x; c < ldx; c += blockDim.x) X[r * ldx + c] = from_f<T>(c < I ? E[src + c] : 0.f);
 }
 
+// bf16 output, I and ldx multiples of 8: one thread converts 8 columns (two 16-byte loads, one
+// 16-byte store) — the same per-element rounding as embed_gather_kernel.
+__global__ void embed_gather8_kernel(const int32_t* __restrict__ tok, const float* __restrict__ E, int I,
+                                     __nv_bfloat16* __restrict__ X, long ldx) {
+  const long r = blockIdx.y;
+  const long c = ((long)blockIdx.x * blockDim.x + threadIdx.x) * 8;
+  if (c >= ldx) return;
+  float v[8];
+  if (c < I) {
+    const float4* src = reinterpret_cast<const float4*>(E + (long)tok[r] * I + c);
+    const float4 p = __ldg(src), q = __ldg(src + 1);
+    v[0] = p.x; v[1] = p.y; v[2] = p.z; v[3] = p.w; v[4] = q.x; v[5] = q.y; v[6] = q.z; v[7] = q.w;
+  } else {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = 0.f;
+  }
+  uint4 o;
+  __nv_bfloat162* ob = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) ob[i] = __halves2bfloat162(__float2bfloat16_rn(v[2 * i]), __float2bfloat16_rn(v[2 * i + 1]));
+  __stcs(reinterpret_cast<uint4*>(X + r * ldx + c), o);
+}
+
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st) {
+  if (n == 0) return;
+  if (ot == OT::BF16 && I % 8 == 0 && ldx % 8 == 0) {
+    for (long r0 = 0; r0 < n; r0 += 65535) {   // grid.y ≤ 65535 rows per launch
+      const long nr = n - r0 < 65535 ? n - r0 : 65535;
+      dim3 grid((unsigned)cdiv(ldx / 8, 128), (unsigned)nr);
+      embed_gather8_kernel<<<grid, 128, 0, st>>>(tok + r0, E, I, (__nv_bfloat16*)X + r0 * ldx, ldx);
+      LAUNCH_CHECK();
+    }
+    return;
+  }
   if (ot == OT::BF16)
     embed_gather_kernel<__nv_bfloat16><<<(unsigned)n, 256, 0, st>>>(tok, n, E, I, (__nv_bfloat16*)X, ldx);
   else
