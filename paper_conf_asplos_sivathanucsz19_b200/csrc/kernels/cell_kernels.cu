@@ -14,6 +14,18 @@
 
 namespace astra {
 
+// two adjacent elements in one store (float2 / bf16 pair)
+template <typename T>
+__device__ __forceinline__ void store2(T* p, float a, float b);
+template <>
+__device__ __forceinline__ void store2<float>(float* p, float a, float b) {
+  *reinterpret_cast<float2*>(p) = make_float2(a, b);
+}
+template <>
+__device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
+  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);
+}
+
 // ============================================================================ mirrors
 template <typename T>
 __global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int H, int Hp, T* __restrict__ dst,
@@ -36,8 +48,38 @@ __global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int 
   }
 }
 
+// Same mapping, tile 32 internal rows x 64 k: a thread stores two adjacent k (one 4-byte bf16 pair,
+// a warp one 128-byte run of a dst row) instead of one 2-byte element.  Same per-element rounding.
+template <typename T>
+__global__ void mirror_gates_T2_kernel(const float* __restrict__ src, int K, int H, int Hp, T* __restrict__ dst,
+                                       long ldd, long kcols) {
+  __shared__ float tile[64][33];
+  const int r0 = blockIdx.x * 32, k0 = blockIdx.y * 64;
+  const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
+  const int r = r0 + tx;
+  const int tileu = r / (4 * GATE_U), g = (r % (4 * GATE_U)) / GATE_U, j = tileu * GATE_U + r % GATE_U;
+  for (int i = ty; i < 64; i += 8) {
+    const int k = k0 + i;
+    tile[i][tx] = (k < K && j < H) ? src[(long)k * 4 * H + g * H + j] : 0.f;
+  }
+  __syncthreads();
+  for (int i = ty; i < 32; i += 8) {
+    const int rr = r0 + i, k = k0 + 2 * tx;
+    if (rr < 4 * Hp && k < kcols) store2<T>(dst + (long)rr * ldd + k, tile[2 * tx][i], tile[2 * tx + 1][i]);
+  }
+}
+
 void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st, long kcols) {
   if (kcols < 0) kcols = ldd;
+  if (kcols % 2 == 0 && ldd % 2 == 0) {
+    dim3 grid(cdiv(4L * Hp, 32), cdiv(kcols, 64)), block(32, 8);
+    if (ot == OT::BF16)
+      mirror_gates_T2_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
+    else
+      mirror_gates_T2_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols);
+    LAUNCH_CHECK();
+    return;
+  }
   dim3 grid(cdiv(4L * Hp, 32), cdiv(kcols, 32)), block(32, 8);
   if (ot == OT::BF16)
     mirror_gates_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
@@ -131,16 +173,6 @@ template <>
 __device__ __forceinline__ void store2cs<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
   __nv_bfloat162 v = __floats2bfloat162_rn(a, b);
   __stcs(reinterpret_cast<unsigned int*>(p), *reinterpret_cast<unsigned int*>(&v));
-}
-template <typename T>
-__device__ __forceinline__ void store2(T* p, float a, float b);
-template <>
-__device__ __forceinline__ void store2<float>(float* p, float a, float b) {
-  *reinterpret_cast<float2*>(p) = make_float2(a, b);
-}
-template <>
-__device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a, float b) {
-  *reinterpret_cast<__nv_bfloat162*>(p) = __floats2bfloat162_rn(a, b);
 }
 
 constexpr int FB_UB = 512;
