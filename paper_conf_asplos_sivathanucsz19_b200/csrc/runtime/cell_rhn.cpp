@@ -214,15 +214,24 @@ class RhnCell : public Cell {
     mark(R_BPTT, 1, st);
 
     mark(R_SE4, 0, st);
-    mark(R_DU, 0, st);
+    // wg_side (B3 stream assignment): the L independent dR_ℓ GEMMs alternate between the
+    // main and a side stream, so one GEMM's tail wave overlaps the next one's (outputs disjoint: same bits)
+    cudaStream_t st_s = st;
+    if (var.wg_side && !side.empty()) {
+      CUDA_TRY(cudaEventRecord(ev_fork, st));
+      CUDA_TRY(cudaStreamWaitEvent(side[0], ev_fork, 0));
+      st_s = side[0];
+    }
+    if (st_s == st) mark(R_DU, 0, st);
     for (int l = 0; l < L; ++l) {
       GemmSpec gr;
       gr.A = mat(Sop(l, 0), Hp, TB, Hp); gr.a_mn = true;
       gr.B = mat(DA(l, 0), G2, TB, G2); gr.b_mn = true;
       gr.M = Hp; gr.N = G2; gr.K = (int)TB;
-      run_gemm(20 + l, gr, epi_perm(g("R") + (size_t)l * H * 2 * H, 2L * H, H, G2, 0, Hp, H), 0, 0, var.g[G_DU], st);
+      run_gemm(20 + l, gr, epi_perm(g("R") + (size_t)l * H * 2 * H, 2L * H, H, G2, 0, Hp, H), 0, 0, var.g[G_DU],
+               (l & 1) ? st_s : st);
     }
-    mark(R_DU, 1, st);
+    if (st_s == st) mark(R_DU, 1, st);
     mark(R_DW, 0, st);
     GemmSpec gw;
     gw.A = mat(X, I, TB, Ip); gw.a_mn = true;
@@ -241,6 +250,10 @@ class RhnCell : public Cell {
       if (lm_mode) run_gemm(4, gx, epi(dx, Ip, (int)TB, I), 0, 0, var.g[G_DX], st);
       else run_gemm(4, gx, epi(dx, I, (int)TB, I, ot == OT::BF16), 0, 0, var.g[G_DX], st);
       mark(R_DX, 1, st);
+    }
+    if (st_s != st) {   // the side stream's dR_ℓ GEMMs overlapped dW / dX
+      CUDA_TRY(cudaEventRecord(ev_join, st_s));
+      CUDA_TRY(cudaStreamWaitEvent(st, ev_join, 0));
     }
     mark(R_SE4, 1, st);
     grad_bucket(G, n_params, st);   // one bucket for the cell's parameters

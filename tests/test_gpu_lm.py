@@ -285,3 +285,23 @@ def test_rhn_fused_forward_lm_bitwise(hov):
         torch.cuda.synchronize()
         out.append((m.params.clone(), float(m.loss.item())))
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
+
+
+def test_rhn_wg_side_lm_bitwise():
+    """RHN weight gradients with the L dR_ℓ GEMMs alternating between the main and a side stream
+    (wg_side=1, overlapping dW / dX) give the same bits as all on the main stream, over 4 SGD steps."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 5, 64, 128, 192, 300
+    out = []
+    for v in ("wg_side=0", "wg_side=1"):
+        p, tok, h0, c0 = _lm_case("rhn", T, B, I, H, V, synth.config_seed(3) + 31, True)
+        c = A.Cell("rhn", H, I, B, T, dtype="bf16", depth=L_DEPTH)
+        m = A.LM(c, V)
+        m.load(p)
+        c.tune_mode(A.TUNE_FROZEN, v)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(4):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append((m.params.clone(), float(m.loss.item())))
+    assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
