@@ -655,14 +655,16 @@ void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targ
 // s + p[0] + p[stride] + ... + p[(n−1)·stride], added in ascending order (the fixed order of every
 // reduction below); the loads are issued 8 at a time, so a thread waits one memory latency per 8
 // terms instead of one per term.  Same bits as the one-term-at-a-time loop.
+// (NB terms ahead: 8 for wide grids; 32 for the few-block final reductions, whose threads are few.)
+template <int NB = 8>
 __device__ __forceinline__ float ordered_sum(const float* __restrict__ p, long n, long stride, float s = 0.f) {
   long i = 0;
-  for (; i + 8 <= n; i += 8) {
-    float v[8];
+  for (; i + NB <= n; i += NB) {
+    float v[NB];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) v[k] = p[(i + k) * stride];
+    for (int k = 0; k < NB; ++k) v[k] = p[(i + k) * stride];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) s = __fadd_rn(s, v[k]);
+    for (int k = 0; k < NB; ++k) s = __fadd_rn(s, v[k]);
   }
   for (; i < n; ++i) s = __fadd_rn(s, p[i * stride]);
   return s;
@@ -673,7 +675,7 @@ __global__ void sum_scalar_kernel(const float* __restrict__ v, long n, float sca
   __shared__ float sh[1024];
   if (nvp) scale = __fdiv_rn(1.f, (float)*nvp);   // mean over the valid rows (the rest are exact zeros)
   const long nt = n > (long)threadIdx.x ? (n - threadIdx.x + blockDim.x - 1) / blockDim.x : 0;
-  sh[threadIdx.x] = ordered_sum(v + threadIdx.x, nt, blockDim.x);
+  sh[threadIdx.x] = ordered_sum<32>(v + threadIdx.x, nt, blockDim.x);
   __syncthreads();
   for (int w = blockDim.x / 2; w > 0; w >>= 1) {
     if (threadIdx.x < w) sh[threadIdx.x] = __fadd_rn(sh[threadIdx.x], sh[threadIdx.x + w]);
@@ -707,7 +709,7 @@ __global__ void colsum_partial_kernel(const float* __restrict__ in, long rows, i
 __global__ void colsum_final_kernel(const float* __restrict__ part, int nchunk, int cols, float* __restrict__ out) {
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= cols) return;
-  out[c] = ordered_sum(part + c, nchunk, cols);
+  out[c] = ordered_sum<32>(part + c, nchunk, cols);
 }
 
 void colsum(const float* in, long rows, int cols, long ld, float* scratch, float* out, cudaStream_t st) {
@@ -801,7 +803,7 @@ __global__ void emb_seg_final_kernel(int V, const int32_t* __restrict__ segoff, 
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= I) return;
   const int s0 = segoff[v];
-  dE[(long)v * I + c] = ordered_sum(part + (long)s0 * I + c, segoff[v + 1] - s0, I);
+  dE[(long)v * I + c] = ordered_sum<32>(part + (long)s0 * I + c, segoff[v + 1] - s0, I);
 }
 
 size_t embed_bwd_partial_floats(long n, int V, int I) { return (size_t)(n / EMB_SEG + V + 1) * I; }
