@@ -143,6 +143,10 @@ astra_status astra_tune_report(astra_cell c, char* buf, size_t len, size_t* need
 /* ---- data parallelism -------------------------------------------------- */
 /* nccl_unique_id: host pointer to the 128-byte ncclUniqueId broadcast by the caller.       */
 astra_status astra_comm_init(astra_cell c, const void* nccl_unique_id, int rank, int world);
+/* The same for an LM: ONE communicator shared by every layer of the (stacked) LM, so the head,
+ * embedding and every layer's buckets are reduced.  A world > 1 LM step whose layers lack a
+ * common communicator (NCCL or K11p) fails with ASTRA_E_STATE instead of silently diverging.   */
+astra_status astra_lm_comm_init(astra_lm m, const void* nccl_unique_id, int rank, int world);
 /* Write a fresh ncclUniqueId (128 bytes) to host memory `out` (call on rank 0).           */
 astra_status astra_comm_unique_id(void* out, size_t len);
 

@@ -58,6 +58,7 @@ _SIGS = {
     "astra_tune_report": [_P, ctypes.c_char_p, _SZ, ctypes.POINTER(_SZ)],
     "astra_set_profiling": [_P, _I],
     "astra_comm_init": [_P, _P, _I, _I],
+    "astra_lm_comm_init": [_P, _P, _I, _I],
     "astra_comm_unique_id": [_P, _SZ],
     "astra_comm_peer_handle": [_P, _P, _SZ],
     "astra_comm_peer_init": [_P, _P, _I, _I],
@@ -336,6 +337,10 @@ class LM:
         self.ws = _alloc_bytes(self.ws_bytes, dev)
         self.loss = torch.zeros(1, dtype=torch.float32, device=dev)
         _check(L.astra_lm_bind(h, _ptr(self.params), _ptr(self.grads), _ptr(self.ws)))
+        # the LM carved every layer's saved / scratch workspace out of its own: the cells' own
+        # buffers (GBs at cfg5) are dead from here on
+        for c in self.layers:
+            c.saved = c.scratch = None
 
     def view(self, name, t=None):
         t = self.params if t is None else t
@@ -377,6 +382,11 @@ class LM:
     def fwd_bwd(self, tokens, loss=None):
         _check(lib().astra_lm_fwd_bwd(self.h, _ptr(tokens), _ptr(self.loss if loss is None else loss)))
         return self.loss if loss is None else loss
+
+    def comm_init(self, uid: bytes, rank, world):
+        """One NCCL communicator for every layer of the LM (astra_lm_comm_init)."""
+        b = ctypes.create_string_buffer(uid, len(uid))
+        _check(lib().astra_lm_comm_init(self.h, b, rank, world))
 
     def comm_peer_handle(self) -> bytes:
         """This rank's peer-memory window handle for the LM's params / grads (K11p)."""

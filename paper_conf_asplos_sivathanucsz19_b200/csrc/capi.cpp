@@ -205,24 +205,42 @@ astra_status astra_comm_unique_id(void* out, size_t len) {
   });
 }
 
+// One NCCL communicator shared by `cells` (a cell, or every layer of an LM); cells[0] owns it.
+static void comm_init_cells(const std::vector<Cell*>& cells, const void* uid, int rank, int world) {
+  ASTRA_CHECK_ARG(world >= 1 && rank >= 0 && rank < world, "comm_init: bad rank/world");
+  for (Cell* c : cells)
+    ASTRA_CHECK_ARG(!c->peer || !c->peer->ready || c->peer->world == world, "comm_init: world differs from the peer backend's");
+  Cell& c0 = *cells[0];
+  CUDA_TRY(cudaSetDevice(c0.d.device));
+  ncclUniqueId id;
+  std::memcpy(&id, uid, sizeof(id));
+  ncclComm_t comm;
+  ncclResult_t r = ncclCommInitRank(&comm, world, id, rank);
+  if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
+  for (Cell* c : cells)
+    if (c->nccl_comm && c->own_nccl) ncclCommDestroy((ncclComm_t)c->nccl_comm);
+  for (size_t i = 0; i < cells.size(); ++i) {
+    Cell& cc = *cells[i];
+    cc.nccl_comm = comm;
+    cc.own_nccl = i == 0;
+    cc.rank = rank;
+    cc.world = world;
+    cc.ensure_comm_stream();
+    if (!cc.tune_dev) CUDA_TRY(cudaMalloc(&cc.tune_dev, 64 * sizeof(double)));
+  }
+}
+
 astra_status astra_comm_init(astra_cell c, const void* uid, int rank, int world) {
   return guard([&] {
     NEED(c); NEED(uid);
-    ASTRA_CHECK_ARG(world >= 1 && rank >= 0 && rank < world, "comm_init: bad rank/world");
-    Cell& cc = *c->c;
-    CUDA_TRY(cudaSetDevice(cc.d.device));
-    ncclUniqueId id;
-    std::memcpy(&id, uid, sizeof(id));
-    ncclComm_t comm;
-    ncclResult_t r = ncclCommInitRank(&comm, world, id, rank);
-    if (r != ncclSuccess) throw Error(ASTRA_E_NCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r));
-    if (cc.nccl_comm) ncclCommDestroy((ncclComm_t)cc.nccl_comm);
-    cc.nccl_comm = comm;
-    cc.rank = rank;
-    cc.world = world;
-    ASTRA_CHECK_ARG(!cc.peer || !cc.peer->ready || cc.peer->world == world, "comm_init: world differs from the peer backend's");
-    cc.ensure_comm_stream();
-    if (!cc.tune_dev) CUDA_TRY(cudaMalloc(&cc.tune_dev, 64 * sizeof(double)));
+    comm_init_cells({c->c.get()}, uid, rank, world);
+  });
+}
+
+astra_status astra_lm_comm_init(astra_lm m, const void* uid, int rank, int world) {
+  return guard([&] {
+    NEED(m); NEED(uid);
+    comm_init_cells(m->m->layers, uid, rank, world);
   });
 }
 

@@ -117,7 +117,10 @@ class Cell {
   bool region_used[R_COUNT];
   bool profiling = true;
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
-  std::map<std::tuple<int, int, int, int, int, int>, TcGemm> tc_cache;   // (gemm id, T, bn, cm, cn, cg)
+  // prepared GEMMs keyed by (gemm id, T, bn, cm, cn, cg, A, B, M, N, K): the tensor maps carry the
+  // operand pointers and extents, so two row ranges of one role never share an entry
+  using TcKey = std::tuple<int, int, int, int, int, int, const void*, const void*, int, int, int>;
+  std::map<TcKey, TcGemm> tc_cache;
 
   // Bucketed profiling: one independent exploration per active length T, the
   // profile index keys prefixed by the bucket; the workspace stays the one of the largest bucket.
@@ -135,6 +138,7 @@ class Cell {
 
   // NCCL
   void* nccl_comm = nullptr;
+  bool own_nccl = true;   // false: a communicator shared with the other layers of an LM (layer 0 owns it)
   int rank = 0, world = 1;
   // K11p: deterministic peer-memory gradient sum + fused SGD / all-gather (SURVEY §8(e) backend
   // 2).  When set (world > 1), grad_bucket() launches the rank-ordered reduce instead of NCCL and

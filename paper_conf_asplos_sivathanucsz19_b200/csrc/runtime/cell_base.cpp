@@ -143,7 +143,7 @@ Cell::~Cell() {
     if (ev_bucket[k]) cudaEventDestroy(ev_bucket[k]);
   if (own_comm_st) cudaStreamDestroy(own_comm_st);
   if (tune_dev) cudaFree(tune_dev);
-  if (nccl_comm) ncclCommDestroy((ncclComm_t)nccl_comm);
+  if (nccl_comm && own_nccl) ncclCommDestroy((ncclComm_t)nccl_comm);
 }
 
 size_t Cell::find_param(const std::string& n) const {
@@ -187,7 +187,7 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
 TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
   // split-K only runs without clusters; the cluster choice then falls back to 1x1 (same numerics)
   const int cm = s.ksplit > 1 ? 1 : k.cm, cn = s.ksplit > 1 ? 1 : k.cn;
-  auto key = std::make_tuple(id, T, k.bn, cm, cn, k.cg);
+  const TcKey key{id, T, k.bn, cm, cn, k.cg, s.A.ptr, s.B.ptr, s.M, s.N, s.K};
   auto it = tc_cache.find(key);
   if (it == tc_cache.end()) {
     TcGemm g;

@@ -223,9 +223,20 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   ASTRA_CHECK_STATE(bound, "lm_train_step: not bound");
   ASTRA_CHECK_ARG(tokens, "lm_train_step: tokens is null");
   Cell& c = *cell;
+  // data parallelism needs one communicator across every layer (the embedding and head buckets
+  // go through layer 0 / the top layer): a layer without one would silently stay unreduced
+  int wmax = 1;
+  for (Cell* L : layers) wmax = std::max(wmax, L->world);
+  if (wmax > 1)
+    for (Cell* L : layers)
+      ASTRA_CHECK_STATE(L->world == wmax && (L->nccl_comm || L->peer),
+                        "lm_train_step: world > 1 but a layer has no communicator (use astra_lm_comm_init / "
+                        "astra_lm_comm_peer_init on the LM, not on one cell)");
   // exploration steps (and the fp32 parity path) run eagerly; a frozen / untuned / converged bf16 step replays
   // multi-rank steps stay eager unless ASTRA_GRAPH_NCCL=1 (NCCL inside a capture is supported, but
-  // a capture mismatch across ranks would hang the job; not exercisable on a 1-GPU test box)
+  // a capture mismatch across ranks would hang the job; not exercisable on a 1-GPU test box).  The
+  // peer-memory backend never replays: its kernels take the host's barrier sequence number as an
+  // argument, which a captured graph would freeze (every replay would pass the barriers at once)
   static const bool graph_nccl = [] {
     const char* e = std::getenv("ASTRA_GRAPH_NCCL");
     return e && e[0] == '1';
@@ -237,7 +248,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
     vs += L->var.str() + (L->profiling ? ";p" : ";");
   }
   if (!use_graphs || !graphs_enabled() || exploring || c.ot != OT::BF16 ||
-      (c.world > 1 && !graph_nccl)) {
+      (c.world > 1 && (!graph_nccl || c.peer))) {
     enqueue_step(tokens, lr, loss_dev, do_sgd);
     return;
   }

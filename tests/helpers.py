@@ -2,6 +2,8 @@
 and the parity metric (reading R18: per-tensor relative L2 error ‖gpu − oracle‖₂ / ‖oracle‖₂)."""
 from __future__ import annotations
 
+import os
+
 import numpy as np
 
 import synth
@@ -18,11 +20,56 @@ def golden(name):
         return json.load(f)
 
 
-def rel_err(gpu, ref):
+def rel_l2(gpu, ref):
+    """Reading R18's per-tensor metric ‖gpu − oracle‖₂ / ‖oracle‖₂."""
     gpu = np.asarray(gpu, dtype=np.float64)
     ref = np.asarray(ref, dtype=np.float64)
     n = np.linalg.norm(ref.ravel())
     return float(np.linalg.norm((gpu - ref).ravel()) / (n if n > 0 else 1.0))
+
+
+def _slice_rel(d, r, axis):
+    """Worst relative L2 error over the rows (axis=1 reduced) or columns (axis=0 reduced) of a 2-D
+    view; each slice's norm is floored at the median slice norm so near-zero slices do not blow up."""
+    nd = np.sqrt((d * d).sum(axis))
+    nr = np.sqrt((r * r).sum(axis))
+    floor = max(float(np.median(nr)), 1e-300)
+    return float((nd / np.maximum(nr, floor)).max())
+
+
+def parity_metrics(gpu, ref):
+    """Element-wise parity (round-2 VERDICT 'parity is a norm, not element-wise'): next to the
+    per-tensor relative L2 error, the largest element error relative to the tensor's largest
+    magnitude, and the worst per-row and per-column relative errors of the tensor viewed as
+    [rows, last dim] — a single wrong hidden unit, timestep or sample shows up as a slice error of
+    order 1 even where it barely moves the whole-tensor norm."""
+    gpu = np.asarray(gpu, dtype=np.float64)
+    ref = np.asarray(ref, dtype=np.float64)
+    assert gpu.shape == ref.shape or gpu.size == ref.size, (gpu.shape, ref.shape)
+    gpu = gpu.reshape(ref.shape)
+    d = gpu - ref
+    m = {"l2": rel_l2(gpu, ref)}
+    amax = float(np.abs(ref).max()) if ref.size else 0.0
+    m["max"] = float(np.abs(d).max() / amax) if amax > 0 else float(np.abs(d).max()) if d.size else 0.0
+    if ref.ndim >= 2 and ref.size:
+        d2 = d.reshape(-1, ref.shape[-1])
+        r2 = ref.reshape(-1, ref.shape[-1])
+        m["row"] = _slice_rel(d2, r2, 1)
+        m["col"] = _slice_rel(d2, r2, 0)
+    return m
+
+
+def rel_err(gpu, ref):
+    """The parity number every test asserts ≤ tol: the largest of parity_metrics() — the per-tensor
+    relative L2 error (R18) and its element-wise / per-row / per-column refinements."""
+    m = parity_metrics(gpu, ref)
+    log = os.environ.get("ASTRA_PARITY_LOG")
+    if log:   # distribution of every metric over the suite (profiles/, DESIGN reading R18)
+        import json
+        with open(log, "a") as f:
+            f.write(json.dumps({"test": os.environ.get("PYTEST_CURRENT_TEST", "").split(" ")[0],
+                                "shape": list(np.shape(ref)), **m}) + "\n")
+    return max(m.values())
 
 
 def bf16_round(a):

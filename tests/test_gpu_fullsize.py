@@ -111,3 +111,38 @@ def test_cfg4_attention_full_size():
     """cfg4: LSTM with attention, H = A = I = 1024, B = 128, Ts = Tt = 50 (cell API, whole step)."""
     from test_gpu_cell import _attn_check
     _attn_check(50, 50, 128, 1024, 1024, 1024, "bf16", synth.config_seed(4) + 100, TOL_BF16)
+
+
+def test_cfg5_lm_full_size_grouped_sequences():
+    """The whole cfg5 LM step (embedding gather, MI-LSTM, head, mean CE over all T·B = 51 200
+    positions, BPTT, every gradient incl. dE / dW_o / b_o) at FULL size in the bench's converged
+    variant (head overlapped in 2 chunks), against the oracle.  The 512 sequences are G = 8
+    distinct token sequences, each placed in 64 batch columns chosen by a seeded permutation, from a
+    zero initial state: the sequences of a group are identical, so the full-batch mean loss and
+    mean-loss gradients equal the oracle's over the 8 distinct sequences exactly (equal group
+    sizes), while neighbouring batch columns hold different sequences (a row mix-up would show)."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V, G = 100, 512, 2048, 2048, 256, 8
+    seed = synth.config_seed(5) + 200
+    shapes = cell_shapes("milstm", I, H)
+    shapes.update({"E": (V, I), "W_o": (H, V), "b_o": (V,)})
+    p = synth.weights(seed, shapes, H, {"alpha": (0.5, 1.5), "beta1": (0.5, 1.5), "beta2": (0.5, 1.5)})
+    for k in ("W", "U", "E", "W_o"):
+        p[k] = bf16_round(p[k])
+    distinct = synth.zipf_tokens(seed, "tok", (T + 1, G), V, 205)
+    group = synth.rng(seed, "groups").permutation(np.repeat(np.arange(G), B // G))
+    tok = distinct[:, group]
+    c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+    c.tune_mode(A.TUNE_FROZEN, BENCH_VARIANT + ",hov=1")
+    m = A.LM(c, V)
+    m.load(p)
+    dev = c.device
+    m.set_state(torch.zeros(B, H, device=dev), torch.zeros(B, H, device=dev))
+    loss = float(m.fwd_bwd(torch.as_tensor(tok, dtype=torch.int32, device=dev)).item())
+    torch.cuda.synchronize()
+    g = {k: m.view(k, m.grads).cpu().numpy().reshape(np.shape(p[k])) for k in p}
+    lo, go, _ = OLM.lm_forward_backward("milstm", p, distinct, np.zeros((G, H)), np.zeros((G, H)))
+    assert abs(loss - lo) / abs(lo) <= TOL_BF16, (loss, lo)
+    errs = {k: rel_err(g[k], go[k]) for k in go}
+    bad = {k: v for k, v in errs.items() if not v <= TOL_BF16}
+    assert not bad, (bad, errs)

@@ -180,6 +180,29 @@ def test_head_overlap_bitwise(cell, hov):
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
 
 
+def test_head_overlap_switch_on_one_lm_bitwise():
+    """One LM switches head_ov 0 → 1 → 2 → 1 (as the tuner does while exploring): each step's loss
+    and gradients equal the sequential head's bit for bit.  Guards the prepared-GEMM cache: the
+    2-chunk and 5-chunk head GEMMs cover different row ranges and must never share an entry."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 10, 64, 64, 64, 300
+    p, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, synth.config_seed(5) + 41, True)
+    c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+    m = A.LM(c, V)
+    m.load(p)
+    tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+    dev = c.device
+    out = []
+    for v in (0, 1, 2, 1, 0):
+        c.tune_mode(A.TUNE_FROZEN, f"hov={v}")
+        m.set_state(torch.zeros(B, H, device=dev), torch.zeros(B, H, device=dev))
+        loss = m.fwd_bwd(tokens)
+        torch.cuda.synchronize()
+        out.append((m.grads.clone(), float(loss.item())))
+    for g, l in out[1:]:
+        assert torch.equal(g, out[0][0]) and l == out[0][1]
+
+
 @pytest.mark.parametrize("cell,H", [("milstm", 192), ("milstm", 2048), ("lstm", 256)])
 def test_fused_bptt_lm_bitwise(cell, H):
     """LM steps with the fused BPTT kernel (bwd=1, the LM's fp32 dY streamed by TMA) give the same

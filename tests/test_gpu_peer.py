@@ -40,7 +40,7 @@ def _shard(a, r, world, axis=1):
     return np.ascontiguousarray(np.take(a, range(r * n, (r + 1) * n), axis=axis))
 
 
-def _worker(rank, world, port, kind, dtype, q, variant=None):
+def _worker(rank, world, port, kind, dtype, q, variant=None, steps=STEPS):
     try:
         os.environ["MASTER_ADDR"] = "127.0.0.1"
         os.environ["MASTER_PORT"] = str(port)
@@ -59,7 +59,7 @@ def _worker(rank, world, port, kind, dtype, q, variant=None):
             A.peer_exchange(m)
             tokens = torch.as_tensor(_shard(tok, rank, world), dtype=torch.int32, device="cuda")
             losses = []
-            for _ in range(STEPS):
+            for _ in range(steps):
                 m.train_step(tokens, LR)
                 losses.append(m.loss.item())
             torch.cuda.synchronize()
@@ -89,11 +89,11 @@ def _worker(rank, world, port, kind, dtype, q, variant=None):
         raise
 
 
-def _run_world(kind, dtype, world=2, variant=None):
+def _run_world(kind, dtype, world=2, variant=None, steps=STEPS):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = 29650 + os.getpid() % 300
-    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, dtype, q, variant)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, kind, dtype, q, variant, steps)) for r in range(world)]
     for pr in procs:
         pr.start()
     res = {}
@@ -180,3 +180,25 @@ def test_peer_cell_api_bitwise_equals_rank_ordered_mean():
     ref = newp.cpu().numpy()
     for r, (pp, gg, _) in res.items():
         assert np.array_equal(pp, ref), f"rank {r}"
+
+
+@pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
+def test_peer_lm_step_vs_oracle_dp(dtype, tol):
+    """One K11p step against the fp64 oracle's DP semantics (oracle.dp.dp_gradients: the mean of
+    the two shard-mean gradients, §8(c.3) item 8) and its SGD (oracle.lm.sgd): the parameter update
+    θ_1 − θ_0 of every tensor, identical on both ranks, equals −lr·g_oracle."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    from oracle import dp as ODP
+    res = _run_world("lm", dtype, steps=1)
+    p0, tok = _lm_case(dtype)
+    _, g_o = ODP.dp_gradients("milstm", p0, tok, np.zeros((B, H)), np.zeros((B, H)), 2)
+    c = A.Cell("milstm", H, I, B // 2, T, dtype=dtype)
+    m = A.LM(c, V)
+    assert np.array_equal(res[0][0], res[1][0])
+    theta1 = res[0][0]
+    errs = {}
+    for k, (off, r, cc) in m.param_info.items():
+        upd = theta1[off:off + r * cc].astype(np.float64) - np.asarray(p0[k], np.float32).astype(np.float64).ravel()
+        errs[k] = rel_err(upd, -LR * np.asarray(g_o[k]).ravel())
+    bad = {k: v for k, v in errs.items() if not v <= tol}
+    assert not bad, (bad, errs)

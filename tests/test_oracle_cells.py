@@ -338,3 +338,118 @@ def test_statefulness_split_sequence(cell):
         y2, h2, _ = C.rhn_forward(p, inp["x"][2:], h1)
     assert np.array_equal(y, np.concatenate([y1, y2]))
     assert np.array_equal(hT, h2)
+
+
+# ------------------------------------------------------------------ round-2 pins (VERDICT r1 "What's weak" #1)
+def test_scrn_context_feeds_h_through_P_closed_form():
+    """A = R = 0, b_h = 0 ⇒ h_t = σ(s_t·P) with s_t the closed form
+    s_t = (1−α)Σ_{k≤t} α^{t−k}(x_k·Bm) + α^{t+1} s_0 (0-based t).  Pins that h_t reads the *current*
+    context s_t through P (s_{t−1}·P, a missing (1−α) or a transposed P fail)."""
+    T, B, I, H, S = 6, 3, 4, 5, 7
+    alpha = 0.9
+    p = synth.weights(SEED, C.scrn_param_shapes(I, H, S), H)
+    p["A"][:] = 0.0
+    p["R"][:] = 0.0
+    p["b_h"][:] = 0.0
+    p["P"] = synth.uniform(SEED, "Pbig", (S, H), -2, 2)   # large enough that σ(s·P) is far from ½
+    inp = _inputs(T, B, I, H)
+    s0 = synth.uniform(SEED, "s0", (B, S), -0.5, 0.5)
+    y, _, _, _ = C.scrn_forward(p, inp["x"], inp["h0"], s0, alpha)
+    for t in range(T):
+        s_t = alpha ** (t + 1) * s0
+        for k in range(t + 1):
+            s_t = s_t + (1 - alpha) * alpha ** (t - k) * (inp["x"][k] @ p["Bm"])
+        h_ref = torch.sigmoid(torch.tensor(s_t) @ torch.tensor(p["P"])).numpy()
+        np.testing.assert_allclose(y[t][:, :H], h_ref, atol=1e-15)
+        np.testing.assert_allclose(y[t][:, H:], s_t, atol=1e-15)
+
+
+def test_attention_two_positions_closed_form():
+    """Ts = 2: softmax over two scores is p_1 = σ(e_1 − e_2), so ctx_i = p_1·enc_1 + (1−p_1)·enc_2
+    with e_j = vᵀtanh(q_i + k_j), q_i = h_i·W_q from the decoder's *current* h_i.  The decoder step
+    itself is torch.nn.LSTMCell on the input-fed vector [x^d_i | ctx_{i−1}] (W_ih = [W_d; C_d]ᵀ,
+    W_hh = U_dᵀ), started from the encoder's final state (torch.nn.LSTM).  Pins: q from h_i (not
+    h_{i−1}), tanh inside the sum, the score vector v, the keys k_j = enc_j·W_k, input feeding of
+    ctx_{i−1} (not ctx_i, not none) through C_d, and y_i = [h_i | ctx_i]."""
+    Ts, Tt, B, I, H, A = 2, 3, 2, 3, 4, 5
+    p, inp = _attn_setup(T_s=Ts, T_t=Tt, B=B, I=I, H=H, A=A)
+    p["v"] = synth.uniform(SEED, "vbig", (A,), -3, 3)           # scores well away from a tie
+    p["C_d"] = synth.uniform(SEED, "Cdbig", (H, 4 * H), -1, 1)   # input feeding clearly visible
+    y, hT, cT, _ = C.attn_forward(p, inp["xe"], inp["xd"], inp["h0"], inp["c0"])
+    encp = {"W": p["W_e"], "U": p["U_e"], "b": p["b_e"]}
+    _, _, _, _, enc, he, ce = _torch_lstm(encp, inp["xe"], inp["h0"], inp["c0"])
+    enc = enc.detach().numpy()
+    keys = [enc[j] @ p["W_k"] for j in range(Ts)]
+    cellm = torch.nn.LSTMCell(I + H, H).double()
+    with torch.no_grad():
+        cellm.weight_ih.copy_(torch.tensor(np.concatenate([p["W_d"], p["C_d"]], 0).T))
+        cellm.weight_hh.copy_(torch.tensor(p["U_d"].T))
+        cellm.bias_ih.copy_(torch.tensor(p["b_d"]))
+        cellm.bias_hh.zero_()
+    h, c = he.detach(), ce.detach()
+    ctx = np.zeros((B, H))
+    sig = lambda z: 1.0 / (1.0 + np.exp(-z))
+    for i in range(Tt):
+        with torch.no_grad():
+            h, c = cellm(torch.tensor(np.concatenate([inp["xd"][i], ctx], 1)), (h, c))
+        q = h.numpy() @ p["W_q"]
+        e1 = np.tanh(q + keys[0]) @ p["v"]
+        e2 = np.tanh(q + keys[1]) @ p["v"]
+        p1 = sig(e1 - e2)[:, None]
+        ctx = p1 * enc[0] + (1.0 - p1) * enc[1]
+        np.testing.assert_allclose(y[i][:, :H], h.numpy(), atol=1e-14)
+        np.testing.assert_allclose(y[i][:, H:], ctx, atol=1e-14)
+    np.testing.assert_allclose(hT, h.numpy(), atol=1e-14)
+    np.testing.assert_allclose(cT, c.numpy(), atol=1e-14)
+
+
+def _torch_attn_loss(p, inp, dY, dhT, dcT):
+    """An independent construction of the attentive LSTM from torch library routines (torch's LSTM
+    cell for encoder and decoder, the decoder on [x | ctx_{i−1}], torch.softmax over positions), fp64, whose
+    autograd gradients pin the oracle's hand-derived attention backward."""
+    I = inp["xe"].shape[2]
+    H = inp["h0"].shape[1]
+    t = {k: torch.tensor(v, requires_grad=True) for k, v in p.items()}
+    xi = {k: torch.tensor(inp[k], requires_grad=True) for k in ("xe", "xd", "h0", "c0")}
+    # torch's own LSTM cell kernel; the parameters are the dict tensors so autograd reaches them
+    def lstm_step(x, h, c, W_ih, W_hh, b):
+        return torch._VF.lstm_cell(x, (h, c), W_ih, W_hh, b, torch.zeros_like(b))
+    h, c = xi["h0"], xi["c0"]
+    enc = []
+    for j in range(inp["xe"].shape[0]):
+        h, c = lstm_step(xi["xe"][j], h, c, t["W_e"].T, t["U_e"].T, t["b_e"])
+        enc.append(h)
+    enc = torch.stack(enc)
+    keys = enc @ t["W_k"]
+    ctx = torch.zeros_like(h)
+    ys = []
+    W_ih = torch.cat([t["W_d"], t["C_d"]], 0).T
+    for i in range(inp["xd"].shape[0]):
+        h, c = lstm_step(torch.cat([xi["xd"][i], ctx], 1), h, c, W_ih, t["U_d"].T, t["b_d"])
+        q = h @ t["W_q"]
+        e = torch.tanh(q[None] + keys) @ t["v"]                 # [Ts, B]
+        pr = torch.softmax(e, 0)
+        ctx = (pr[:, :, None] * enc).sum(0)
+        ys.append(torch.cat([h, ctx], 1))
+    y = torch.stack(ys)
+    L = (y * torch.tensor(dY)).sum() + (h * torch.tensor(dhT)).sum() + (c * torch.tensor(dcT)).sum()
+    L.backward()
+    g = {k: v.grad.numpy() for k, v in t.items()}
+    g.update(dxe=xi["xe"].grad.numpy(), dxd=xi["xd"].grad.numpy(), dh0=xi["h0"].grad.numpy(),
+             dc0=xi["c0"].grad.numpy())
+    return y.detach().numpy(), g
+
+
+def test_attention_backward_matches_torch_autograd():
+    """Every attention gradient (v, W_q, W_k, C_d, the decoder and encoder weights, the inputs and
+    the initial state) equals fp64 autograd through the library-built construction above."""
+    p, inp = _attn_setup(T_s=4, T_t=3, B=2, I=3, H=5, A=4)
+    p["v"] = synth.uniform(SEED, "vbig", (4,), -2, 2)
+    Tt, B, H = 3, 2, 5
+    dY = synth.normal(SEED, "dY", (Tt, B, 2 * H))
+    dhT, dcT = synth.normal(SEED, "dh", (B, H)), synth.normal(SEED, "dc", (B, H))
+    out, g = C.cell_fwd_bwd("attn", p, inp, dY, dhT, dcT)
+    y_t, g_t = _torch_attn_loss(p, inp, dY, dhT, dcT)
+    np.testing.assert_allclose(out["y"], y_t, atol=1e-14)
+    for k in g_t:
+        np.testing.assert_allclose(g[k], g_t[k], atol=1e-12, err_msg=k)
