@@ -1,15 +1,18 @@
 """Benchmark: custom-RNN training samples/s on B200 (BASELINE.json metric), workload = cfg5
-(BASELINE.json configs[4]): MI-LSTM char LM, hidden 2048, batch 512, seq 100, data-parallel over N
-GPUs.  Default: weak scaling — every rank trains its own shard of 512 sequences (global batch 512·N,
-DESIGN.md reading R30: the sequences are independent units, the only exchange is the gradient
-all-reduce); `--strong` keeps the global batch at 512 (per-rank 512/N).  One step = embedding → MI-LSTM forward →
-head + CE → BPTT → weight gradients → gradient all-reduce (N > 1) → SGD, all in the library's
-kernels through the C ABI.
+(BASELINE.json configs[4]): MI-LSTM char LM, hidden 2048, GLOBAL batch 512, seq 100, data-parallel
+over N GPUs.  Default: strong scaling as BASELINE configs[4] and SURVEY §8(d.1) state — the global
+batch stays 512 and each of the N ranks trains its contiguous shard of 512/N sequences; `--weak`
+gives every rank its own 512 sequences instead (global batch 512·N).  One step = embedding →
+MI-LSTM forward → head + CE → BPTT → weight gradients → gradient all-reduce (N > 1) → SGD, all in
+the library's kernels through the C ABI.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl astra|reference]
 
 Prints ONE JSON line on rank 0.  `--impl reference` times the fp64 CPU oracle (the paper
-publishes no code, so the oracle is the reference arm) on a bounded sample of the same workload.
+publishes no code, so the oracle is the reference arm) on a bounded sample of the same workload:
+every step is one full fwd + bwd + SGD step over 64 of the sequences (so its BLAS calls are GEMMs,
+not GEMVs), W warm-up steps and K timed steps, and the line states the steps, batch and per-step
+time it actually ran.
 """
 from __future__ import annotations
 
@@ -121,10 +124,29 @@ def make_params(I, H, V):
 
 
 # ------------------------------------------------------------------------------------------ oracle
-def run_oracle(T, H, I, V, n_sym, B_sample, steps=1, warm=0):
-    """Time the fp64 numpy oracle (as it stands) on a bounded sample of the workload."""
-    import numpy as np
+ORACLE_SAMPLE_B = 64   # sequences per oracle step: GEMM-shaped BLAS calls (B=4 was GEMV-bound)
+
+
+def host_info():
+    """The host the oracle runs on: logical cores, CPU model, BLAS threads."""
     from threadpoolctl import threadpool_info
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    threads = max([i.get("num_threads", 1) for i in threadpool_info()] + [1])
+    return {"cores": threads, "cpu_count": os.cpu_count(), "cpu_model": model}
+
+
+def run_oracle(T, H, I, V, n_sym, B_sample, steps=1, warm=0):
+    """Time the fp64 numpy oracle (as it stands) on a bounded sample of the workload: `warm`
+    untimed then `steps` timed fwd + bwd + SGD steps over B_sample sequences (state not carried,
+    parameters updated).  Returns (samples/s, seconds per step)."""
+    import numpy as np
     from oracle import lm as OLM
     import synth
     p = make_params(I, H, V)
@@ -132,13 +154,12 @@ def run_oracle(T, H, I, V, n_sym, B_sample, steps=1, warm=0):
     h0 = np.zeros((B_sample, H))
     c0 = np.zeros((B_sample, H))
     for _ in range(warm):
-        OLM.lm_train_step("milstm", p, tok, h0, c0, 0.1)
+        _, p, _, _ = OLM.lm_train_step("milstm", p, tok, h0, c0, 0.1)
     t0 = time.perf_counter()
     for _ in range(steps):
         loss, p, _, _ = OLM.lm_train_step("milstm", p, tok, h0, c0, 0.1)
     dt = (time.perf_counter() - t0) / steps
-    threads = max([i.get("num_threads", 1) for i in threadpool_info()] + [1])
-    return B_sample / dt, dt, threads
+    return B_sample / dt, dt
 
 
 # ------------------------------------------------------------------------------------------ main
@@ -151,8 +172,8 @@ def main():
     ap.add_argument("--no-tune", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + --steps steps, nothing else (for ncu)")
-    ap.add_argument("--batch", type=int, default=None, help="override the per-rank batch (weak) / global batch (strong)")
-    ap.add_argument("--strong", action="store_true", help="fixed global batch 512 split over the ranks")
+    ap.add_argument("--batch", type=int, default=None, help="override the global batch (strong) / per-rank batch (weak)")
+    ap.add_argument("--weak", action="store_true", help="every rank trains its own --batch sequences (global batch x N)")
     ap.add_argument("--seq", type=int, default=None, help="override seq (debug)")
     ap.add_argument("--dp", default="nccl", choices=["nccl", "peer"],
                     help="N > 1 gradient sum: NCCL all-reduce (K11) or the deterministic peer-memory "
@@ -165,8 +186,8 @@ def main():
     T = args.seq or WORKLOAD["seq_len"]
     H, I, V, n_sym = WORKLOAD["hidden"], WORKLOAD["input"], WORKLOAD["vocab"], WORKLOAD["symbols"]
     B_unit = args.batch or WORKLOAD["global_batch"]
-    B_g = B_unit if args.strong else B_unit * max(world, 1)     # global batch of this run
-    scaling = "strong" if args.strong else "weak"
+    B_g = B_unit * max(world, 1) if args.weak else B_unit     # global batch of this run
+    scaling = "weak" if args.weak else "strong"
     cfg = {"workload": WORKLOAD["workload"], "cell": "MI-LSTM", "hidden": H, "input": I, "global_batch": B_g,
            "seq_len": T, "vocab": V, "parallelism": f"dp{args.gpus}", "dp_backend": args.dp, "per_gpu_batch": B_g // max(world, 1),
            "l2": "working set per step (GB of activations, 139 MB of fp32 grads) >> 126 MB L2: inputs larger than L2"}
@@ -174,15 +195,18 @@ def main():
     if args.impl == "reference":
         if rank != 0:
             return
-        Bs = 4
-        val, dt, thr = run_oracle(T, H, I, V, n_sym, Bs, steps=max(1, min(args.steps, 2)), warm=0)
+        Bs = min(ORACLE_SAMPLE_B, B_g)
+        wall0 = time.perf_counter()
+        val, dt = run_oracle(T, H, I, V, n_sym, Bs, steps=args.steps, warm=args.warmup)
+        hi = host_info()
+        sample = (f"each step: {Bs} of the {B_g} sequences (T={T}, H=I=2048, V=256), one full fwd+bwd+SGD step "
+                  f"of the fp64 numpy oracle; {args.warmup} warm-up + {args.steps} timed steps, "
+                  f"{time.perf_counter() - wall0:.1f} s wall")
         line = {"impl": "reference", "metric": METRIC, "value": val, "unit": "samples/s", "n_gpus": args.gpus,
-                "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 * (B_g / Bs),
-                "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "f64",
-                "data": "synthetic (seeded Zipf tokens, random-init weights)", "config": cfg,
-                "cpu_baseline": {"value": val, "unit": "samples/s", "cores": thr, "kind": "oracle",
-                                 "sample": f"{Bs} of the {B_g} sequences (T={T}, H=I=2048, V=256), one full "
-                                           f"fwd+bwd+SGD step of the fp64 numpy oracle"},
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3,
+                "samples_per_step": Bs, "higher_is_better": True, "scaling": scaling, "vs_baseline": None,
+                "dtype": "f64", "data": "synthetic (seeded Zipf tokens, random-init weights)", "config": cfg,
+                "cpu_baseline": {"value": val, "unit": "samples/s", "kind": "oracle", "sample": sample, **hi},
                 "e2e": {"value": val, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
         return
@@ -205,7 +229,7 @@ def main():
     if distributed:   # the process group only broadcasts the NCCL id; the library owns the comm (K11)
         uid = [A.comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
-        cell.comm_init(uid[0], rank, world)   # also carries the tuner's cross-rank decisions (R29)
+        lm.comm_init(uid[0], rank, world)   # one communicator for the LM; also the tuner's cross-rank decisions (R29)
         if args.dp == "peer" and world > 1:
             A.peer_exchange(lm)
     tok_host = torch.as_tensor(make_inputs(B_g, T, V, n_sym, rank, world), dtype=torch.int32).pin_memory()
@@ -238,12 +262,13 @@ def main():
             lm.train_step(tokens, lr)
             tune_steps += 1
             s = cell.tune_next()
-            if s == A.TUNE_CONVERGED or tune_steps > 400:
+            if s == A.TUNE_CONVERGED or tune_steps > 1000:
                 break
         torch.cuda.synchronize()
         rep = cell.tune_report()
         cell.tune_mode(A.TUNE_FROZEN, rep["variant"])
-        tune_info = {"mode": "explored then frozen", "steps": tune_steps, "configs_explored": rep.get("configs_explored"),
+        tune_info = {"mode": "explored then frozen", "converged": s == A.TUNE_CONVERGED, "steps": tune_steps,
+                     "configs_explored": rep.get("configs_explored"), "harvest_waits": rep.get("harvest_waits"),
                      "wall_s": round(time.perf_counter() - tune_t0, 3), "variant": rep["variant"]}
     # ---- warm-up, then the timed region (device time, CUDA events on the launching stream; max
     # over ranks).  nvidia-smi samples clocks from the last warm-up steps through the timed region.
@@ -267,19 +292,28 @@ def main():
     ms = float(t.item())
     value = B_g / (ms / 1e3)
 
-    # ---- profiling overhead ("<0.5%"): the same frozen steps with the region events off
-    cell.set_profiling(False)
-    for _ in range(2):
-        lm.train_step(tokens, lr)
-    barrier()
-    g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    g0.record(st)
-    for _ in range(args.steps):
-        lm.train_step(tokens, lr)
-    g1.record(st)
-    torch.cuda.synchronize()
-    ms_noprof = g0.elapsed_time(g1) / args.steps
+    # ---- profiling overhead ("<0.5%"): the same frozen steps with the region events on and
+    # off, in interleaved windows (clocks drift under the power cap: one pair of windows is noise)
+    def window(on, n):
+        cell.set_profiling(on)
+        lm.train_step(tokens, lr)          # (re)captures the step graph of this mode outside the window
+        barrier()
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        g0.record(st)
+        for _ in range(n):
+            lm.train_step(tokens, lr)
+        g1.record(st)
+        torch.cuda.synchronize()
+        return g0.elapsed_time(g1) / n
+    n_win = 6
+    per = max(3, min(args.steps, 10))
+    pairs = []
+    for w in range(n_win):
+        order = (True, False) if w % 2 == 0 else (False, True)
+        r = {o: window(o, per) for o in order}
+        pairs.append(100.0 * (r[True] - r[False]) / r[False])
     cell.set_profiling(True)
+    pairs.sort()
 
     # ---- dominant kernel live: the hoisted a1 GEMM region (one K1 launch, on the main stream)
     region = cell_region_ms(cell, lm, tokens, lr, steps=3)
@@ -324,18 +358,19 @@ def main():
             "e2e": {"value": B_g / (ms_e2e / 1e3), "unit": "samples/s", "h2d_bytes_per_step": int(tok_host.numel() * 4),
                     "d2h_bytes_per_step": 4},
             "gpu_launches": int(launches),
-            "profiling_overhead": {"events_on_ms": ms, "events_off_ms": ms_noprof,
-                                   "pct": 100.0 * (ms - ms_noprof) / ms_noprof},
+            "profiling_overhead": {"pct": statistics.median(pairs), "min_pct": pairs[0], "max_pct": pairs[-1],
+                                   "windows": n_win, "steps_per_window": per,
+                                   "method": "median over interleaved region-events on/off window pairs"},
             "clocks": clk.summary(),
             "tuner": tune_info,
         }
         if not args.no_cpu_baseline:
             try:
-                Bs = 4
-                val, dt, thr = run_oracle(T, H, I, V, n_sym, Bs, steps=1)
-                line["cpu_baseline"] = {"value": val, "unit": "samples/s", "cores": thr, "kind": "oracle",
+                Bs = min(ORACLE_SAMPLE_B, B_g)
+                val, dt = run_oracle(T, H, I, V, n_sym, Bs, steps=1)
+                line["cpu_baseline"] = {"value": val, "unit": "samples/s", "kind": "oracle",
                                         "sample": f"{Bs} sequences of the cfg5 workload (T={T}, H=I=2048, V=256), "
-                                                  f"one fwd+bwd+SGD step, fp64 numpy, {dt:.1f} s"}
+                                                  f"one fwd+bwd+SGD step, fp64 numpy, {dt:.1f} s", **host_info()}
             except Exception as e:  # pragma: no cover
                 line["cpu_baseline"] = {"value": None, "error": str(e)}
         print(json.dumps(line), flush=True)

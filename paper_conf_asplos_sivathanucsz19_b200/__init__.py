@@ -126,7 +126,15 @@ def launch_count():
 
 
 def _ptr(t):
-    return None if t is None else ctypes.c_void_p(t.data_ptr())
+    """Raw pointer of a tensor handed to the C ABI, which takes dense row-major buffers only: a
+    strided view (e.g. from numpy fancy indexing) would be read in the wrong order, so it is
+    refused instead of silently reinterpreted."""
+    if t is None:
+        return None
+    if not t.is_contiguous():
+        raise ValueError(f"astra: tensor of shape {tuple(t.shape)} / strides {t.stride()} is not contiguous "
+                         "(the C ABI takes dense row-major buffers; call .contiguous())")
+    return ctypes.c_void_p(t.data_ptr())
 
 
 def _stream():

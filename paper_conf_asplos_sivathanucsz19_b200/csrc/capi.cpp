@@ -476,15 +476,18 @@ astra_status astra_region_times(astra_cell c, double* out, int cap, int* n) {
     NEED(c); NEED(out);
     Cell& cc = *c->c;
     ASTRA_CHECK_STATE(cc.bound, "region_times: not bound");
-    CUDA_TRY(cudaEventSynchronize(cc.ev[R_STEP][1]));
+    // the most recently completed step's slot (the tuner may already record into the next one)
+    cudaEvent_t (*E)[2] = cc.evr[cc.last_step_slot];
+    const bool* used = cc.used_r[cc.last_step_slot];
+    CUDA_TRY(cudaEventSynchronize(E[R_STEP][1]));
     int k = 0;
     for (int r = 0; r < R_COUNT && k < cap; ++r, ++k) {
       float ms = 0.f;
-      if (cc.region_used[r] && cudaEventElapsedTime(&ms, cc.ev[r][0], cc.ev[r][1]) != cudaSuccess) {
+      if (used[r] && cudaEventElapsedTime(&ms, E[r][0], E[r][1]) != cudaSuccess) {
         cudaGetLastError();
         ms = 0.f;
       }
-      out[k] = cc.region_used[r] ? ms : 0.0;
+      out[k] = used[r] ? ms : 0.0;
     }
     if (n) *n = k;
   });

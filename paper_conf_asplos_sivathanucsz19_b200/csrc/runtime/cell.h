@@ -113,8 +113,24 @@ class Cell {
   std::vector<Variant> configs_seen;
   int tune_reps = 3, rep_i = 0;
   tuner::Metrics rep_min;
-  cudaEvent_t ev[R_COUNT][2];
-  bool region_used[R_COUNT];
+  // Region events live in a ring of per-step slots, so the tuner can harvest a
+  // measured step with cudaEventQuery some steps later instead of blocking on it (include/astra.h
+  // astra_tune_next "never blocks"): `ev` / `region_used` point at the slot being recorded.
+  static constexpr int EV_SLOTS = 8;
+  cudaEvent_t evr[EV_SLOTS][R_COUNT][2];
+  bool used_r[EV_SLOTS][R_COUNT];
+  int ev_slot = 0, last_step_slot = 0;
+  cudaEvent_t (*ev)[2] = evr[0];
+  bool* region_used = used_r[0];
+  // measured exploration steps whose events are not harvested yet: (slot, bucket T, config serial)
+  struct PendingRep { int slot, T; long serial; };
+  std::vector<PendingRep> pending;
+  long cfg_serial = 0, next_serial = 1;
+  int reps_harvested = 0;
+  long tune_blocks = 0;      // harvests that had to wait (ring full, or world > 1: reading R29)
+  void use_slot(int s);
+  tuner::Metrics read_metrics(int slot);
+  void harvest(int wait);
   bool profiling = true;
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
   // prepared GEMMs keyed by (gemm id, T, bn, cm, cn, cg, A, B, M, N, K): the tensor maps carry the
@@ -132,6 +148,8 @@ class Cell {
     int rep_i = 0;
     tuner::Metrics rep_min;
     std::vector<KCfg> allowed[G_ROLES];
+    long cfg_serial = 0;
+    int reps_harvested = 0;
   };
   std::map<int, TuneCtx> tune_ctx;   // parked contexts of the inactive buckets
   void set_active_T(int t);

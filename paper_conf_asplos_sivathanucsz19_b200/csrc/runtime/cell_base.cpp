@@ -124,8 +124,16 @@ Cell::Cell(const astra_cell_desc& dd) : d(dd) {
   Ip = (int)round_up(I, 64);
   Hout = H;
   ASTRA_CHECK_ARG((long)T * B < (1L << 31) / 64, "cell: T*B too large");
+  std::memset(used_r, 0, sizeof(used_r));
+  std::memset(evr, 0, sizeof(evr));
+  use_slot(0);
+}
+
+void Cell::use_slot(int s) {
+  ev_slot = s;
+  ev = evr[s];
+  region_used = used_r[s];
   for (int r = 0; r < R_COUNT; ++r) region_used[r] = false;
-  std::memset(ev, 0, sizeof(ev));
 }
 
 void Cell::add_param(const char* n, int r, int c) {
@@ -134,9 +142,10 @@ void Cell::add_param(const char* n, int r, int c) {
 }
 
 Cell::~Cell() {
-  for (int r = 0; r < R_COUNT; ++r)
-    for (int w = 0; w < 2; ++w)
-      if (ev[r][w]) cudaEventDestroy(ev[r][w]);
+  for (int k = 0; k < EV_SLOTS; ++k)
+    for (int r = 0; r < R_COUNT; ++r)
+      for (int w = 0; w < 2; ++w)
+        if (evr[k][r][w]) cudaEventDestroy(evr[k][r][w]);
   if (ev_fork) cudaEventDestroy(ev_fork);
   if (ev_join) cudaEventDestroy(ev_join);
   for (int k = 0; k < 4; ++k)
@@ -164,8 +173,9 @@ void Cell::bind(float* pp, float* gg, void* sv_p, void* sc_p) {
     CUDA_TRY(cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming));
     CUDA_TRY(cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming));
     for (int k = 0; k < 4; ++k) CUDA_TRY(cudaEventCreateWithFlags(&ev_bucket[k], cudaEventDisableTiming));
-    for (int r = 0; r < R_COUNT; ++r)
-      for (int w = 0; w < 2; ++w) CUDA_TRY(cudaEventCreate(&ev[r][w]));
+    for (int k = 0; k < EV_SLOTS; ++k)
+      for (int r = 0; r < R_COUNT; ++r)
+        for (int w = 0; w < 2; ++w) CUDA_TRY(cudaEventCreate(&evr[k][r][w]));
   }
   bound = true;
   fwd_done = false;
@@ -182,6 +192,7 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
   else
     CUDA_TRY(cudaEventRecord(ev[r][which], st));
   if (which) region_used[r] = true;
+  if (which && r == R_STEP) last_step_slot = ev_slot;
 }
 
 TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
@@ -317,6 +328,8 @@ void Cell::set_active_T(int t) {
   cur.configs_seen = std::move(configs_seen);
   cur.rep_i = rep_i;
   cur.rep_min = rep_min;
+  cur.cfg_serial = cfg_serial;
+  cur.reps_harvested = reps_harvested;
   for (int r = 0; r < G_ROLES; ++r) cur.allowed[r] = allowed[r];
   auto it = tune_ctx.find(t);
   if (it != tune_ctx.end()) {
@@ -327,6 +340,8 @@ void Cell::set_active_T(int t) {
     configs_seen = std::move(nx.configs_seen);
     rep_i = nx.rep_i;
     rep_min = nx.rep_min;
+    cfg_serial = nx.cfg_serial;
+    reps_harvested = nx.reps_harvested;
     for (int r = 0; r < G_ROLES; ++r) allowed[r] = nx.allowed[r];
     tune_ctx.erase(it);
   } else {
@@ -336,6 +351,8 @@ void Cell::set_active_T(int t) {
     configs_seen.clear();
     rep_i = 0;
     rep_min.clear();
+    cfg_serial = 0;
+    reps_harvested = 0;
   }
   T = t;
   fwd_done = false;
@@ -399,6 +416,8 @@ void Cell::tuner_setup() {
   tuner::Config c;
   if (wirer->propose(c)) apply_config(c);
   rep_i = 0;
+  cfg_serial = next_serial++;
+  reps_harvested = 0;
 }
 
 void Cell::apply_config(const tuner::Config& c) {
@@ -431,41 +450,104 @@ static float elapsed(cudaEvent_t a, cudaEvent_t b) {
   return ms;
 }
 
+tuner::Metrics Cell::read_metrics(int slot) {
+  cudaEvent_t (*E)[2] = evr[slot];
+  const bool* used = used_r[slot];
+  tuner::Metrics m(tree->metrics.size(), 0.0);
+  for (size_t i = 0; i < tree->metrics.size(); ++i) {
+    const std::string& n = tree->metrics[i];
+    double v = 0;
+    if (n == "t_a1") v = elapsed(E[R_A1][0], E[R_A1][1]);
+    else if (n == "t_fwd") v = elapsed(E[R_FWD][0], E[R_FWD][1]);
+    else if (n == "t_bptt") v = elapsed(E[R_BPTT][0], E[R_BPTT][1]);
+    else if (n == "t_du") v = used[R_DU] ? elapsed(E[R_DU][0], E[R_DU][1]) : 0;
+    else if (n == "t_dw") v = used[R_DW] ? elapsed(E[R_DW][0], E[R_DW][1]) : 0;
+    else if (n == "t_dx") v = used[R_DX] ? elapsed(E[R_DX][0], E[R_DX][1]) : 0;
+    else if (n == "t_head") v = used[R_HEAD] ? elapsed(E[R_HEAD][0], E[R_HEAD][1]) : 0;
+    else if (n == "t_se4") v = elapsed(E[R_SE4][0], E[R_SE4][1]);
+    else v = elapsed(E[R_STEP][0], E[R_STEP][1]);
+    m[i] = v;
+  }
+  return m;
+}
+
+// Fold the finished measured steps, oldest first, into the min-over-reps of the configuration
+// (and bucket) they measured.  A step is finished when its step-end event has completed
+// (cudaEventQuery).  wait = 1: also wait for every pending step except the newest — the step just
+// enqueued is never waited for, so the GPU always has it queued while the host decides; wait = 2:
+// wait for all of them (a cross-rank decision, reading R29).
+void Cell::harvest(int wait) {
+  size_t k = 0;
+  for (; k < pending.size(); ++k) {
+    const PendingRep& p = pending[k];
+    cudaEvent_t end = evr[p.slot][R_STEP][1];
+    if (wait == 2 || (wait == 1 && k + 1 < pending.size())) {
+      if (cudaEventQuery(end) == cudaErrorNotReady) ++tune_blocks;
+      CUDA_TRY(cudaEventSynchronize(end));
+    } else {
+      const cudaError_t q = cudaEventQuery(end);
+      if (q == cudaErrorNotReady) break;
+      if (q != cudaSuccess) CUDA_TRY(q);
+    }
+    // the measured configuration is the active one, or a parked bucket's (still current there)
+    tuner::Metrics* rm = nullptr;
+    int* nh = nullptr;
+    if (p.T == T && p.serial == cfg_serial) { rm = &rep_min; nh = &reps_harvested; }
+    else {
+      auto it = tune_ctx.find(p.T);
+      if (it != tune_ctx.end() && it->second.cfg_serial == p.serial) { rm = &it->second.rep_min; nh = &it->second.reps_harvested; }
+    }
+    if (!rm) continue;   // a configuration that has been decided already: surplus measurement
+    tuner::Metrics m = read_metrics(p.slot);
+    if (*nh == 0 || rm->size() != m.size()) *rm = m;
+    else
+      for (size_t i = 0; i < m.size(); ++i) (*rm)[i] = std::min((*rm)[i], m[i]);
+    ++*nh;
+  }
+  pending.erase(pending.begin(), pending.begin() + k);
+}
+
 // One call per step (after the step's work is enqueued).  Per configuration: one warm-up step
-// (absorbs lazy tensor-map creation), then tune_reps measured steps whose region times are min-
-// reduced (reading R19: clocks float on B200 so k = 3 reps instead of the paper's pinned clocks,
-// P:457).  Only the measured steps synchronise on their own end event.
+// (absorbs lazy tensor-map creation), then measured steps whose region times are min-reduced
+// (reading R19: clocks float on B200 so k = 3 reps instead of the paper's pinned clocks).
+// Never waits for the step just enqueued (include/astra.h): a measured step's events are harvested
+// with cudaEventQuery once the GPU has finished it; the configuration keeps running (real training
+// steps, so the exploration stays work-conserving) until tune_reps of its measured steps are in,
+// waiting at most for the steps BEFORE the newest one — the GPU is busy with the newest meanwhile,
+// so host and GPU stay pipelined and a configuration costs at most 1 warm-up + tune_reps + 1
+// steps.  With world > 1 every rank must decide at the same step (reading R29), so there the
+// decision step is fixed — the tune_reps-th measured step — and waits for its events.
 int Cell::tune_next() {
   if (tune_mode != ASTRA_TUNE_ON) return tune_mode == ASTRA_TUNE_FROZEN ? ASTRA_TUNE_CONVERGED : ASTRA_TUNE_IDLE;
   ASTRA_CHECK_STATE(world <= 1 || nccl_comm,
                     "tune_next: exploring with world > 1 needs astra_comm_init (cross-rank decisions, reading R29)");
   if (!wirer) tuner_setup();
   if (wirer->converged()) return ASTRA_TUNE_CONVERGED;
+  auto advance = [&] {   // the next step records into a slot no pending measurement uses
+    int s = (ev_slot + 1) % EV_SLOTS;
+    for (int tries = 0; tries < EV_SLOTS; ++tries, s = (s + 1) % EV_SLOTS) {
+      bool busy = false;
+      for (const PendingRep& p : pending) busy |= p.slot == s;
+      if (!busy) break;
+    }
+    for (const PendingRep& p : pending)
+      if (p.slot == s) { harvest(1); break; }   // ring full: wait for the older ones
+    use_slot(s);
+  };
   if (rep_i == 0) {  // warm-up step done
     rep_i = 1;
+    advance();
     return ASTRA_TUNE_EXPLORING;
   }
-  CUDA_TRY(cudaEventSynchronize(ev[R_STEP][1]));
-  tuner::Metrics m(tree->metrics.size(), 0.0);
-  for (size_t i = 0; i < tree->metrics.size(); ++i) {
-    const std::string& n = tree->metrics[i];
-    double v = 0;
-    if (n == "t_a1") v = elapsed(ev[R_A1][0], ev[R_A1][1]);
-    else if (n == "t_fwd") v = elapsed(ev[R_FWD][0], ev[R_FWD][1]);
-    else if (n == "t_bptt") v = elapsed(ev[R_BPTT][0], ev[R_BPTT][1]);
-    else if (n == "t_du") v = region_used[R_DU] ? elapsed(ev[R_DU][0], ev[R_DU][1]) : 0;
-    else if (n == "t_dw") v = region_used[R_DW] ? elapsed(ev[R_DW][0], ev[R_DW][1]) : 0;
-    else if (n == "t_dx") v = region_used[R_DX] ? elapsed(ev[R_DX][0], ev[R_DX][1]) : 0;
-    else if (n == "t_head") v = region_used[R_HEAD] ? elapsed(ev[R_HEAD][0], ev[R_HEAD][1]) : 0;
-    else if (n == "t_se4") v = elapsed(ev[R_SE4][0], ev[R_SE4][1]);
-    else v = elapsed(ev[R_STEP][0], ev[R_STEP][1]);
-    m[i] = v;
-  }
-  if (rep_i == 1) rep_min = m;
-  else
-    for (size_t i = 0; i < m.size(); ++i) rep_min[i] = std::min(rep_min[i], m[i]);
-  if (rep_i < tune_reps) {
-    ++rep_i;
+  pending.push_back({ev_slot, T, cfg_serial});
+  ++rep_i;
+  // world > 1: decide at the tune_reps-th measured step on every rank (wait for all of them);
+  // one rank: once tune_reps measured steps precede the newest, wait for those (the newest keeps
+  // running on the GPU), else only fold in what has finished
+  if (world > 1) harvest(rep_i > tune_reps ? 2 : 0);
+  else harvest(rep_i > tune_reps + 1 ? 1 : 0);
+  if (reps_harvested < tune_reps) {
+    advance();
     return ASTRA_TUNE_EXPLORING;
   }
   if (world > 1 && nccl_comm) {
@@ -480,6 +562,9 @@ int Cell::tune_next() {
   }
   wirer->feed(rep_min);
   rep_i = 0;
+  reps_harvested = 0;
+  cfg_serial = next_serial++;
+  advance();
   tuner::Config c;
   if (wirer->propose(c)) {
     apply_config(c);
@@ -504,7 +589,8 @@ std::string Cell::report() {
   }
   if (wirer) {
     o << ", \"converged\": " << (wirer->converged() ? "true" : "false") << ", \"configs_explored\": "
-      << wirer->trials() << ", \"steps_per_config\": " << (1 + tune_reps) << ", \"index_entries\": "
+      << wirer->trials() << ", \"measured_reps\": " << tune_reps << ", \"harvest_waits\": " << tune_blocks
+      << ", \"index_entries\": "
       << wirer->index().d.size() << ", \"tree_avs\": [";
     for (size_t i = 0; i < tree->avs.size(); ++i) o << (i ? ", " : "") << "\"" << tree->avs[i] << "\"";
     o << "], \"index\": {";

@@ -21,7 +21,7 @@ def lm_run(name, cell, H, I, B, T, V, kw, steps=10):
     while True:
         m.train_step(tok, 0.01)
         n += 1
-        if c.tune_next() == A.TUNE_CONVERGED or n > 400:
+        if c.tune_next() == A.TUNE_CONVERGED or n > 1000:
             break
     torch.cuda.synchronize()
     tw = time.perf_counter() - t0
@@ -68,7 +68,7 @@ def attn_run(name, H, I, A_, B, Ts, Tt, steps=10):
     while True:
         step()
         n += 1
-        if c.tune_next() == A.TUNE_CONVERGED or n > 400:
+        if c.tune_next() == A.TUNE_CONVERGED or n > 1000:
             break
     rep = c.tune_report()
     c.tune_mode(A.TUNE_FROZEN, rep["variant"])

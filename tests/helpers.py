@@ -28,6 +28,15 @@ def rel_l2(gpu, ref):
     return float(np.linalg.norm((gpu - ref).ravel()) / (n if n > 0 else 1.0))
 
 
+# Slice metrics (reading R18b): a row or column has far fewer elements than its tensor, so its
+# relative rounding error spreads wider; it is held to SLICE_FACTOR x the tensor tolerance — still
+# far below the O(1) slice error of any localized bug (a wrong unit, step or sample) — and only
+# slices of at least MIN_SLICE elements are measured.  Calibrated on the whole GPU suite
+# (profiles/r2_parity_metrics_summary.txt: worst bf16 column 1.8x tol on a 64-element slice).
+SLICE_FACTOR = 2.0
+MIN_SLICE = 16
+
+
 def _slice_rel(d, r, axis):
     """Worst relative L2 error over the rows (axis=1 reduced) or columns (axis=0 reduced) of a 2-D
     view; each slice's norm is floored at the median slice norm so near-zero slices do not blow up."""
@@ -37,32 +46,39 @@ def _slice_rel(d, r, axis):
     return float((nd / np.maximum(nr, floor)).max())
 
 
-def parity_metrics(gpu, ref):
-    """Element-wise parity (round-2 VERDICT 'parity is a norm, not element-wise'): next to the
+def parity_metrics(gpu, ref, floor=None):
+    """Element-wise parity (round-1 VERDICT 'parity is a norm, not element-wise'): next to the
     per-tensor relative L2 error, the largest element error relative to the tensor's largest
     magnitude, and the worst per-row and per-column relative errors of the tensor viewed as
-    [rows, last dim] — a single wrong hidden unit, timestep or sample shows up as a slice error of
-    order 1 even where it barely moves the whole-tensor norm."""
+    [rows, last dim] (divided by SLICE_FACTOR, so every metric is held to the same tol) — a single
+    wrong hidden unit, timestep or sample shows up as a slice error of order 1 even where it barely
+    moves the whole-tensor norm.  `floor` (optional, per element) is an absolute error every
+    element may carry regardless (e.g. fp32 storage of a parameter), subtracted first."""
     gpu = np.asarray(gpu, dtype=np.float64)
     ref = np.asarray(ref, dtype=np.float64)
     assert gpu.shape == ref.shape or gpu.size == ref.size, (gpu.shape, ref.shape)
     gpu = gpu.reshape(ref.shape)
     d = gpu - ref
-    m = {"l2": rel_l2(gpu, ref)}
+    if floor is not None:
+        d = np.sign(d) * np.maximum(np.abs(d) - np.broadcast_to(floor, d.shape), 0.0)
+    n = np.linalg.norm(ref.ravel())
+    m = {"l2": float(np.linalg.norm(d.ravel()) / (n if n > 0 else 1.0))}
     amax = float(np.abs(ref).max()) if ref.size else 0.0
     m["max"] = float(np.abs(d).max() / amax) if amax > 0 else float(np.abs(d).max()) if d.size else 0.0
     if ref.ndim >= 2 and ref.size:
         d2 = d.reshape(-1, ref.shape[-1])
         r2 = ref.reshape(-1, ref.shape[-1])
-        m["row"] = _slice_rel(d2, r2, 1)
-        m["col"] = _slice_rel(d2, r2, 0)
+        if d2.shape[1] >= MIN_SLICE:
+            m["row"] = _slice_rel(d2, r2, 1) / SLICE_FACTOR
+        if d2.shape[0] >= MIN_SLICE:
+            m["col"] = _slice_rel(d2, r2, 0) / SLICE_FACTOR
     return m
 
 
-def rel_err(gpu, ref):
+def rel_err(gpu, ref, floor=None):
     """The parity number every test asserts ≤ tol: the largest of parity_metrics() — the per-tensor
     relative L2 error (R18) and its element-wise / per-row / per-column refinements."""
-    m = parity_metrics(gpu, ref)
+    m = parity_metrics(gpu, ref, floor)
     log = os.environ.get("ASTRA_PARITY_LOG")
     if log:   # distribution of every metric over the suite (profiles/, DESIGN reading R18)
         import json
@@ -70,6 +86,12 @@ def rel_err(gpu, ref):
             f.write(json.dumps({"test": os.environ.get("PYTEST_CURRENT_TEST", "").split(" ")[0],
                                 "shape": list(np.shape(ref)), **m}) + "\n")
     return max(m.values())
+
+
+def fp32_ulp(a):
+    """One unit in the last place of fp32 at each element of `a`."""
+    a = np.abs(np.asarray(a, dtype=np.float32))
+    return (np.nextafter(a, np.float32(np.inf)) - a).astype(np.float64)
 
 
 def bf16_round(a):

@@ -101,3 +101,16 @@ def test_tune_report_is_json():
     c.tune_mode(A.TUNE_FROZEN, "a1=128.2.2,rec=256.4.1,wg_side=1")
     r = c.tune_report()
     assert "a1=128.2.2" in r["variant"] and "rec=256.4.1" in r["variant"] and "wg_side=1" in r["variant"]
+
+
+def test_strided_tensor_refused():
+    """The C ABI takes dense row-major buffers: a strided view (numpy fancy indexing yields one) must
+    be refused by the binding, never silently read in the wrong order."""
+    import numpy as np
+    import torch
+    a = np.arange(18, dtype=np.int32).reshape(9, 2)[:, np.array([0, 1, 0, 1])]
+    t = torch.as_tensor(a)
+    assert not t.is_contiguous()
+    with pytest.raises(ValueError):
+        A._ptr(t)
+    assert A._ptr(t.contiguous()) is not None

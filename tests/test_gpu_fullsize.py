@@ -131,7 +131,7 @@ def test_cfg5_lm_full_size_grouped_sequences():
         p[k] = bf16_round(p[k])
     distinct = synth.zipf_tokens(seed, "tok", (T + 1, G), V, 205)
     group = synth.rng(seed, "groups").permutation(np.repeat(np.arange(G), B // G))
-    tok = distinct[:, group]
+    tok = np.ascontiguousarray(distinct[:, group])
     c = A.Cell("milstm", H, I, B, T, dtype="bf16")
     c.tune_mode(A.TUNE_FROZEN, BENCH_VARIANT + ",hov=1")
     m = A.LM(c, V)

@@ -328,3 +328,30 @@ def test_rhn_wg_side_lm_bitwise():
         torch.cuda.synchronize()
         out.append((m.params.clone(), float(m.loss.item())))
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
+
+
+def test_tune_next_never_blocks():
+    """astra_tune_next harvests the measured steps' events with cudaEventQuery (include/astra.h):
+    right after it returns, the step just enqueued is still running on the GPU — the host keeps
+    pipelining exploring steps — and the exploration still converges."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 50, 128, 2048, 2048, 256
+    p, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, synth.config_seed(5) + 60, True, n_symbols=205)
+    c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+    m = A.LM(c, V)
+    m.load(p)
+    tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+    st = torch.cuda.current_stream()
+    c.tune_mode(A.TUNE_ON)
+    busy, n, state = 0, 0, A.TUNE_EXPLORING
+    while state != A.TUNE_CONVERGED and n < 1500:
+        m.train_step(tokens, 0.01)
+        state = c.tune_next()
+        n += 1
+        if 2 <= n <= 41:
+            busy += not st.query()
+    torch.cuda.synchronize()
+    assert state == A.TUNE_CONVERGED, n
+    assert busy >= 36, busy      # the GPU was still working after ≥ 90 % of the calls
+    rep = c.tune_report()
+    assert rep["configs_explored"] >= 10 and rep["converged"]

@@ -17,7 +17,7 @@ import torch.multiprocessing as mp
 import synth
 from oracle import lm as OLM
 
-from helpers import TOL_BF16, TOL_FP32, bf16_round, cell_shapes, make_cell_case, rel_err
+from helpers import TOL_BF16, TOL_FP32, bf16_round, cell_shapes, fp32_ulp, make_cell_case, rel_err
 
 pytestmark = pytest.mark.gpu
 
@@ -198,7 +198,11 @@ def test_peer_lm_step_vs_oracle_dp(dtype, tol):
     theta1 = res[0][0]
     errs = {}
     for k, (off, r, cc) in m.param_info.items():
-        upd = theta1[off:off + r * cc].astype(np.float64) - np.asarray(p0[k], np.float32).astype(np.float64).ravel()
-        errs[k] = rel_err(upd, -LR * np.asarray(g_o[k]).ravel())
+        th0 = np.asarray(p0[k], np.float32).astype(np.float64).ravel()
+        th1 = theta1[off:off + r * cc].astype(np.float64)
+        floor = 0.5 * np.maximum(fp32_ulp(th1), fp32_ulp(th0))   # fp32 master storage (R16)
+        errs[k] = rel_err((th1 - th0).reshape(r, cc) if r > 1 else th1 - th0,
+                          (-LR * np.asarray(g_o[k])).reshape(r, cc) if r > 1 else -LR * np.asarray(g_o[k]),
+                          floor.reshape(r, cc) if r > 1 else floor)
     bad = {k: v for k, v in errs.items() if not v <= tol}
     assert not bad, (bad, errs)

@@ -7,7 +7,9 @@ bf16 path: the library keeps fp32 master weights and regenerates the bf16 operan
 on every forward (K9); the oracle keeps fp64 masters and feeds the bf16-rounded GEMM weights to
 each step (reading R18), so both sides see the same operands up to the master precision.
 Compared: every step's loss, and the accumulated update θ_k − θ_0 of every parameter tensor after
-the last step (the update, not θ itself, so an error in lr·g is not hidden under θ_0)."""
+the last step (the update, not θ itself, so an error in lr·g is not hidden under θ_0), element-wise
+with a floor of ½ fp32 ulp of θ per step (the fp32 master storage, R16: an update far below θ's
+resolution — MI-LSTM's α — is otherwise dominated by storage rounding on both sides)."""
 import numpy as np
 import pytest
 import torch
@@ -15,7 +17,7 @@ import torch
 import synth
 from oracle import lm as OLM
 
-from helpers import TOL_BF16, TOL_FP32, bf16_round, cell_shapes, rel_err
+from helpers import TOL_BF16, TOL_FP32, bf16_round, cell_shapes, fp32_ulp, rel_err
 
 pytestmark = pytest.mark.gpu
 
@@ -61,7 +63,10 @@ def test_lm_sgd_trajectory_vs_oracle(cell, dtype, tol):
     torch.cuda.synchronize()
     errs = {}
     for k in p0:
-        got = m.view(k).cpu().numpy().astype(np.float64).reshape(np.shape(p0[k])) - p0[k]
-        errs[k] = rel_err(got, po[k] - p0[k])
+        theta = m.view(k).cpu().numpy().astype(np.float64).reshape(np.shape(p0[k]))
+        # the library stores fp32 masters (R16): each SGD step rounds θ to fp32 (≤ ½ ulp), a floor
+        # every element of the accumulated update may carry regardless of the gradient's accuracy
+        floor = len(toks) * 0.5 * np.maximum(fp32_ulp(theta), fp32_ulp(p0[k]))
+        errs[k] = rel_err(theta - p0[k], po[k] - p0[k], floor)
     bad = {k: v for k, v in errs.items() if not v <= tol}
     assert not bad, (bad, errs)
