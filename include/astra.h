@@ -268,6 +268,10 @@ astra_status astra_micro_stream_read(const void* buf, size_t bytes, int passes, 
 astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream stream);
 /* n dependent empty kernels of `blocks` CTAs, launched with programmatic dependent launch
  * (pdl = 1, as the chain kernels are) or plainly: the per-step floor of a launched chain.     */
+/* TMA read throughput: `ctas` CTAs each stream `nbox` boxes {64, box_rows} of the bf16 [rows][64·kb]
+ * device buffer through a `stages`-deep shared-memory ring; same = 1: all CTAs read the same boxes. */
+astra_status astra_micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, int stages, int nbox,
+                                  int same, astra_stream stream);
 astra_status astra_micro_launch_chain(int n, int pdl, int blocks, astra_stream stream);
 /* K11p's rank-ordered reduce kernel for `world` simulated ranks on one device: bufs[r] (device
  * fp32 [n]) is rank r's gradient buffer, sigs[r] a zeroed device array of 4096 bytes (the signal

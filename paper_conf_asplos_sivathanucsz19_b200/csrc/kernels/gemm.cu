@@ -103,6 +103,30 @@ void make_tile_map(CUtensorMap* m, const void* ptr, bool bf16, long inner, long 
   if (r != CUDA_SUCCESS) throw Error(ASTRA_E_CUDA, "cuTensorMapEncodeTiled (tile map) failed: " + std::to_string((int)r));
 }
 
+void make_map_nd(CUtensorMap* m, const void* ptr, int rank, const long* dims, const long* strides_bytes,
+                 const int* box, int swizzle_bytes) {
+  ASTRA_CHECK_ARG(ptr != nullptr && ((uintptr_t)ptr & 15) == 0, "tensor map: base must be 16-byte aligned");
+  ASTRA_CHECK_ARG(rank >= 2 && rank <= 5, "tensor map: rank must be 2..5");
+  cuuint64_t d[5], st[4];
+  cuuint32_t bx[5], es[5];
+  for (int i = 0; i < rank; ++i) {
+    d[i] = (cuuint64_t)dims[i];
+    bx[i] = (cuuint32_t)box[i];
+    es[i] = 1;
+    if (i + 1 < rank) {
+      ASTRA_CHECK_ARG(strides_bytes[i] % 16 == 0, "tensor map: strides must be 16-byte multiples");
+      st[i] = (cuuint64_t)strides_bytes[i];
+    }
+  }
+  const CUtensorMapSwizzle sw = swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                : swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                : swizzle_bytes == 32 ? CU_TENSOR_MAP_SWIZZLE_32B : CU_TENSOR_MAP_SWIZZLE_NONE;
+  CUresult r = encode_fn()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, rank, const_cast<void*>(ptr), d, st, bx, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(ASTRA_E_CUDA, "cuTensorMapEncodeTiled (nd map) failed: " + std::to_string((int)r));
+}
+
 static uint32_t make_idesc(int BN, bool a_mn, bool b_mn, int BM = TC_BM) {
   uint32_t d = 0;
   d |= 1u << 4;                      // D format: F32

@@ -43,6 +43,12 @@ void simt_gemm(const float* A, long sam, long sak, const float* B, long sbk, lon
 
 int num_sms();
 
+// bf16 tensor map of rank 2..5 with arbitrary byte strides (dims[0] contiguous; strides_bytes[i] is
+// the stride of dims[i+1]; strides may overlap, e.g. a k-block dimension of stride 128 B next to a
+// row dimension) — lets one TMA box carry several k-block tiles of an MMA operand.
+void make_map_nd(CUtensorMap* m, const void* ptr, int rank, const long* dims, const long* strides_bytes,
+                 const int* box, int swizzle_bytes);
+
 // 3-D tiled tensor map ([z][rows][inner], row stride ld, slice stride zstride, in elements) with a
 // {box_inner, box_rows, 1} box and the given swizzle (0 / 32 / 64 / 128 bytes) — epilogue I/O maps.
 void make_tile_map(CUtensorMap* m, const void* ptr, bool bf16, long inner, long rows, long z, long ld, long zstride,

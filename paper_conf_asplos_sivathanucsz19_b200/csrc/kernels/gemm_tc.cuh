@@ -420,6 +420,14 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       int s = 0;
       uint32_t ph = 0;
       int local = 0;
+      // shared-memory descriptors of stage 0, advanced by adding (bytes >> 4) to the address field
+      // (no carry: addresses < 256 KB): the single issuing thread's scalar work per k-block stays
+      // far below one MMA — at the small-N per-step GEMMs it otherwise bounds the k-loop
+      const uint32_t sa0 = sm100::smem_u32(smem), sb0 = sa0 + S::A_BYTES;
+      const uint64_t dA0 = args.a_mn ? sm100::smem_desc_sw128(sa0, 8192, 1024) : sm100::smem_desc_sw128(sa0, 16, 1024);
+      const uint64_t dB0 = args.b_mn ? sm100::smem_desc_sw128(sb0, 8192, 1024) : sm100::smem_desc_sw128(sb0, 16, 1024);
+      const uint32_t a_kk = args.a_mn ? (2048 >> 4) : (32 >> 4), b_kk = args.b_mn ? (2048 >> 4) : (32 >> 4);
+      const uint32_t idesc = args.idesc;
       for (int ct = cluster_id; ct < num_ct; ct += num_clusters, ++local) {
         const int acc = local & 1;
         const uint32_t use = (uint32_t)(local >> 1);
@@ -431,16 +439,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           sm100::mbar_wait(&full[s], ph);
           if (kb == kb0 && local == 0) GEMM_TRACE(3);
           sm100::tc_fence_after();
-          const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
-          const uint32_t sb = sa + S::A_BYTES;
+          const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
 #pragma unroll
-          for (int kk = 0; kk < TC_BK / 16; ++kk) {
-            const uint64_t ad = args.a_mn ? sm100::smem_desc_sw128(sa + kk * 2048, 8192, 1024)
-                                          : sm100::smem_desc_sw128(sa + kk * 32, 16, 1024);
-            const uint64_t bd = args.b_mn ? sm100::smem_desc_sw128(sb + kk * 2048, 8192, 1024)
-                                          : sm100::smem_desc_sw128(sb + kk * 32, 16, 1024);
-            sm100::umma_bf16(d_tmem, ad, bd, args.idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
-          }
+          for (int kk = 0; kk < TC_BK / 16; ++kk)
+            sm100::umma_bf16(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
           if (cs == 1) sm100::umma_commit(&empty[s]);
           else sm100::umma_commit_mc(&empty[s], mask_nb);
           if (++s == stages) { s = 0; ph ^= 1; }
@@ -619,6 +621,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       int s = 0;
       uint32_t ph = 0;
       int local = 0;
+      const uint32_t sa0 = sm100::smem_u32(smem), sb0 = sa0 + S::A_BYTES;   // (see tc_gemm_kernel)
+      const uint64_t dA0 = args.a_mn ? sm100::smem_desc_sw128(sa0, 8192, 1024) : sm100::smem_desc_sw128(sa0, 16, 1024);
+      const uint64_t dB0 = args.b_mn ? sm100::smem_desc_sw128(sb0, 8192, 1024) : sm100::smem_desc_sw128(sb0, 16, 1024);
+      const uint32_t a_kk = args.a_mn ? (2048 >> 4) : (32 >> 4), b_kk = args.b_mn ? (2048 >> 4) : (32 >> 4);
+      const uint32_t idesc = args.idesc;
       for (int ct = pair_id; ct < num_pt; ct += num_pairs, ++local) {
         const int acc = local & 1;
         const uint32_t use = (uint32_t)(local >> 1);
@@ -629,16 +636,10 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         for (int kb = kb0; kb < kb1; ++kb) {
           sm100::mbar_wait(&full[s], ph);
           sm100::tc_fence_after();
-          const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
-          const uint32_t sb = sa + S::A_BYTES;
+          const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
 #pragma unroll
-          for (int kk = 0; kk < TC_BK / 16; ++kk) {
-            const uint64_t ad = args.a_mn ? sm100::smem_desc_sw128(sa + kk * 2048, 8192, 1024)
-                                          : sm100::smem_desc_sw128(sa + kk * 32, 16, 1024);
-            const uint64_t bd = args.b_mn ? sm100::smem_desc_sw128(sb + kk * 2048, 8192, 1024)
-                                          : sm100::smem_desc_sw128(sb + kk * 32, 16, 1024);
-            sm100::umma_bf16_cg2(d_tmem, ad, bd, args.idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
-          }
+          for (int kk = 0; kk < TC_BK / 16; ++kk)
+            sm100::umma_bf16_cg2(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
           sm100::umma_commit_cg2_mc(&empty[s], 0x3);
           if (++s == stages) { s = 0; ph ^= 1; }
         }

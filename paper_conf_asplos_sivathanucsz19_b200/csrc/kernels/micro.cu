@@ -7,8 +7,11 @@
 //     persistent fused chain);
 //   - a chain of `n` dependent empty kernels launched as the library launches its chain kernels
 //     (with programmatic dependent launch, or without) — the step floor of a launched chain.
+#include <cuda.h>
+
 #include "../common.h"
 #include "gemm.h"
+#include "sm100.cuh"
 #include "pdl.cuh"
 #include "peer.h"
 
@@ -51,6 +54,48 @@ __global__ void grid_barrier_kernel(unsigned* counter, int iters) {
   }
 }
 
+// TMA read throughput per SM: one thread streams `nbox` boxes {64 elements, box_rows} of a bf16
+// [rows][64·kb] tensor through a `stages`-deep shared-memory ring (consumed by a second thread that
+// only waits and releases).  same = 1: every CTA reads the same boxes in the same order (the
+// broadcast pattern of a recurrent chain's h operand); 0: each CTA its own rows.
+__global__ void __launch_bounds__(64, 1) tma_read_kernel(const __grid_constant__ CUtensorMap m, int nbox, int box_rows,
+                                                         int stages, int kb, int row_blocks, int same) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int box_bytes = box_rows * 128;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * box_bytes);
+  uint64_t* empty = full + stages;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < stages; ++s) {
+      sm100::mbar_init(&full[s], 1);
+      sm100::mbar_init(&empty[s], 1);
+    }
+    sm100::fence_barrier_init();
+  }
+  __syncthreads();
+  const int rb0 = same ? 0 : (int)blockIdx.x % row_blocks;
+  if (threadIdx.x == 0) {
+    int s = 0;
+    uint32_t ph = 0;
+    for (int i = 0; i < nbox; ++i) {
+      sm100::mbar_wait(&empty[s], ph ^ 1);
+      sm100::mbar_arrive_expect_tx(&full[s], (uint32_t)box_bytes);
+      const int k = i % kb, rb = (rb0 + i / kb) % row_blocks;
+      sm100::tma_load_3d(smem + s * box_bytes, &m, &full[s], k * 64, rb * box_rows, 0);
+      if (++s == stages) { s = 0; ph ^= 1; }
+    }
+  } else if (threadIdx.x == 32) {
+    int s = 0;
+    uint32_t ph = 0;
+    for (int i = 0; i < nbox; ++i) {
+      sm100::mbar_wait(&full[s], ph);
+      sm100::mbar_arrive(&empty[s]);
+      if (++s == stages) { s = 0; ph ^= 1; }
+    }
+  }
+  __syncthreads();
+}
+
 __global__ void empty_pdl_kernel(int) {
   pdl_wait();
   pdl_trigger();
@@ -71,6 +116,18 @@ void micro_grid_barrier(unsigned* counter, int iters, cudaStream_t st) {
   ASTRA_CHECK_ARG(counter && iters > 0, "micro_grid_barrier: bad arguments");
   CUDA_TRY(cudaMemsetAsync(counter, 0, sizeof(unsigned), st));
   grid_barrier_kernel<<<num_sms(), 128, 0, st>>>(counter, iters);   // one CTA per SM: all co-resident
+  LAUNCH_CHECK();
+}
+
+void micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, int stages, int nbox, int same,
+                    cudaStream_t st) {
+  ASTRA_CHECK_ARG(buf && rows >= box_rows && kb > 0 && ctas > 0 && stages >= 1 && nbox > 0 && box_rows >= 8 &&
+                      box_rows <= 256 && box_rows % 8 == 0, "micro_tma_read: bad arguments");
+  CUtensorMap m;
+  make_tile_map(&m, buf, true, (long)kb * 64, rows, 1, (long)kb * 64, 0, 64, box_rows, 128);
+  const int smem = 1024 + stages * box_rows * 128 + stages * 16;
+  CUDA_TRY(cudaFuncSetAttribute(tma_read_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  tma_read_kernel<<<ctas, 64, smem, st>>>(m, nbox, box_rows, stages, kb, (int)(rows / box_rows), same);
   LAUNCH_CHECK();
 }
 

@@ -101,6 +101,30 @@ bool rhn_rec_fwd_supported(int B, int Hp, int nsplit);
 // mapB: the R mirrors [L][2Hp][Hp] K-major, box {64, 32}; both SWIZZLE_128B.
 void rhn_rec_fwd_launch(const CUtensorMap& mapA, const CUtensorMap& mapB, RhnFwdArgs a, cudaStream_t st);
 
+// Small-batch persistent forward chain (rec_persist.cu, fwd_mode 3): all steps [t0, t1) in one
+// cooperative launch of Hp/16 CTAs (16 units each, their U slice resident in shared memory as far as
+// it fits), B ≤ 128, fused gate epilogue, one grid-wide counter per step.
+struct RecPersistArgs {
+  int B, H, Hp, NG, T, t0, t1;
+  int nk, resident, sa, sb, a_rows, a_bytes, ka, kbs;   // set by the launcher (ka / kbs: k-blocks per A / B stage)
+  uint32_t idesc;
+  const float* WX;          // [T·B][NG]
+  float* UH;                // [T·B][NG] saved for BPTT, or null (recompute context)
+  float* C;                 // [(T+1)·B][Hp]
+  __nv_bfloat16* Hb;        // [(T+1)·B][Hp]
+  void* y;
+  long ldy;
+  int y_kind;               // 0 none, 1 bf16 [T·B][ldy], 2 fp32 [T·B][ldy]
+  float* hT;
+  float* cT;
+  GateParams gp;
+  unsigned* flags;          // one counter, zeroed before the launch
+  unsigned long long* trace;   // optional (astra_debug_set_trace kind 2): [grid][t1-t0][6] globaltimer stamps
+};
+bool lstm_fwd_persist_supported(int B, int Hp);
+// Hb: [(Tmax+1)][B][Hp] bf16 h operands; Um: the U mirror [NG][Hp] (tensor maps built per launch).
+void lstm_fwd_persist_launch(int kind, const void* Hb, const void* Um, int Tmax, RecPersistArgs a, cudaStream_t st);
+
 bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);
 void lstm_bptt_fused_launch(int kind, bool dy_bf16, const BpttFusedMaps& m, BpttFusedArgs a, cudaStream_t st);
 

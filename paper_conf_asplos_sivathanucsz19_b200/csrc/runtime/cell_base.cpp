@@ -26,6 +26,7 @@ std::string Variant::str() const {
   if (lwf) o << ",lwf=" << lwf;
   if (recomp) o << ",rc=" << recomp;
   if (dpb) o << ",dpb=" << dpb;
+  if (gchunk) o << ",gc=" << gchunk;
   return o.str();
 }
 
@@ -51,6 +52,11 @@ Variant Variant::parse(const std::string& s) {
       ASTRA_CHECK_ARG(v.dpb >= 0 && v.dpb <= 3, "variant: dpb must be 0..3 (whole tensors, 128, 32 or 8 MB buckets)");
       continue;
     }
+    if (k == "gc") {
+      v.gchunk = std::stoi(val);
+      ASTRA_CHECK_ARG(v.gchunk >= 0 && v.gchunk <= 4, "variant: gc (gate_chunking) must be 0..4");
+      continue;
+    }
     if (k == "rc") {
       v.recomp = std::stoi(val);
       ASTRA_CHECK_ARG(v.recomp == 0 || v.recomp == 1, "variant: rc must be 0 (store UH) or 1 (recompute UH in BPTT)");
@@ -73,8 +79,8 @@ Variant Variant::parse(const std::string& s) {
     }
     if (k == "fwd" || k == "bwd") {
       const int mode = std::stoi(val);
-      ASTRA_CHECK_ARG(mode >= 0 && mode <= 2, "variant: fwd/bwd mode must be 0 (unfused), 1 (fused per step) or 2 "
-                                               "(fused persistent)");
+      ASTRA_CHECK_ARG(mode >= 0 && mode <= 3, "variant: fwd/bwd mode must be 0 (unfused), 1 (fused per step), 2 "
+                                               "(fused persistent) or 3 (small-batch persistent, weight-resident)");
       (k == "fwd" ? v.fwd_mode : v.bwd_mode) = mode;
       continue;
     }
@@ -381,6 +387,10 @@ void Cell::tuner_setup() {
       par += std::string(" (leaf g_") + ROLE_NAMES[r] + " " + std::to_string(allowed[r].size()) + " " + metric[r] + ")";
     }
   }
+  // §8(a.9) gate_chunking: how many GEMMs the fused gate projection a1 is cut into
+  // and on how many streams they run — a parallel sibling of the kernel choices, metric t_a1
+  if (ot == OT::BF16 && gate_chunkings() > 1)
+    par += " (leaf gate_chunking " + std::to_string(gate_chunkings()) + " t_a1)";
   std::string t = par.empty() ? "" : "(par" + par + ")";
   // reading R26: the forward fusion choice (GEMM + pointwise kernel vs the fused recurrent kernel,
   // P:120-126 "fusion" AV) is tuned after the kernel choices, against the forward-chain time
@@ -432,6 +442,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "lwf") { v.lwf = o; continue; }
     if (n == "recomp") { v.recomp = o; continue; }
     if (n == "dp_bucket") { v.dpb = o; continue; }
+    if (n == "gate_chunking") { v.gchunk = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

@@ -76,7 +76,10 @@ class LstmCell : public Cell {
   // chunk partials are summed in a fixed order by the pointwise kernel (identical for every variant).
   int bptt_ksplit() const { return (ot == OT::BF16 && NG >= 8192) ? 4 : (ot == OT::BF16 && NG >= 4096) ? 2 : 1; }
 
-  int fwd_fusions() const override { return 3; }
+  // K2 fusion choices (AV fuse_fwd): 0 GEMM + pointwise, 1 fused per step (CTA pairs), 2 fused
+  // persistent (256-column tiles), 3 small-batch persistent with the U slice resident (B ≤ 128)
+  int gate_chunkings() const override { return ot == OT::BF16 ? (side.empty() ? 3 : 5) : 1; }
+  int fwd_fusions() const override { return (ot == OT::BF16 && lstm_fwd_persist_supported(B, Hp)) ? 4 : 3; }
   bool chain_prefetch() const override { return true; }
   bool supports_ranges() const override { return true; }
   RecFwd2Maps fm;                       // tensor maps of the fused CTA-pair forward (built at first use)
@@ -142,14 +145,33 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   gp.b = p("b");
   if (kind == K_MILSTM) { gp.alpha = p("alpha"); gp.beta1 = p("beta1"); gp.beta2 = p("beta2"); }
 
-  // a1: hoisted input projection for the range's timesteps (row chunks of one GEMM: same bits)
+  // a1: hoisted input projection for the range's timesteps (row chunks of one GEMM: same bits).
+  // gate_chunking (§8(a.9)): the fused gate GEMM cut into nc GEMMs over ranges of whole 256-column
+  // gate blocks (every output element keeps its single from-zero accumulation over K: same bits,
+  // R1), alternating between the main and a side stream when ns = 2
   if (t0 == 0) mark(R_A1, 0, st);
-  GemmSpec a1;
   const long rows = (long)(t1 - t0) * B;
-  a1.A = mat((const char*)X + (size_t)t0 * B * Ip * e, I, rows, Ip);
-  a1.B = mat(Wm, I, NG, Ip);
-  a1.M = (int)rows; a1.N = NG; a1.K = I;
-  run_gemm(whole ? 0 : 100000 + t0 * 1024 + (t1 - t0), a1, epi(WX + (size_t)t0 * B * NG, NG, (int)rows, NG), 0, 0, var.g[G_A1], st);
+  const int nblk = NG / (4 * GATE_U);
+  const int nc = std::min(GCHUNK_N[var.gchunk], nblk);
+  const bool two = GCHUNK_S[var.gchunk] == 2 && nc > 1 && !side.empty();
+  if (two) {
+    CUDA_TRY(cudaEventRecord(ev_fork, st));
+    CUDA_TRY(cudaStreamWaitEvent(side[0], ev_fork, 0));
+  }
+  for (int k = 0; k < nc; ++k) {
+    const int n0 = (int)((long)nblk * k / nc) * 4 * GATE_U, n1 = (int)((long)nblk * (k + 1) / nc) * 4 * GATE_U;
+    GemmSpec a1;
+    a1.A = mat((const char*)X + (size_t)t0 * B * Ip * e, I, rows, Ip);
+    a1.B = mat((const char*)Wm + (size_t)n0 * Ip * e, I, n1 - n0, Ip);
+    a1.M = (int)rows; a1.N = n1 - n0; a1.K = I;
+    const int id = (whole ? 0 : 100000 + t0 * 1024 + (t1 - t0)) + (nc > 1 ? 9000000 + nc * 64 + k : 0);
+    run_gemm(id, a1, epi(WX + (size_t)t0 * B * NG + n0, NG, (int)rows, n1 - n0), 0, 0, var.g[G_A1],
+             two && (k & 1) ? side[0] : st);
+  }
+  if (two) {
+    CUDA_TRY(cudaEventRecord(ev_join, side[0]));
+    CUDA_TRY(cudaStreamWaitEvent(st, ev_join, 0));
+  }
   if (t0 == 0) mark(R_A1, 1, st);
 
   // a3: recurrent chain
@@ -190,7 +212,21 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
       lstm_fwd_pair_launch(kind, fm, ra, st);
       fwd_step_done(t, st);
     }
-  } else if (ot == OT::BF16 && var.fwd_mode > 0) {
+  } else if (ot == OT::BF16 && var.fwd_mode == 3 && lstm_fwd_persist_supported(B, Hp)) {
+    // K2 small-batch persistent: the whole range in one cooperative launch, U slices resident
+    RecPersistArgs pa{};
+    pa.B = B; pa.H = H; pa.Hp = Hp; pa.NG = NG; pa.T = T; pa.t0 = t0; pa.t1 = t1;
+    pa.WX = WX; pa.UH = var.recomp ? nullptr : UH; pa.C = Cb; pa.Hb = (__nv_bfloat16*)Hrow(0);
+    if (y_f32) { pa.y = y_f32; pa.ldy = Hp; pa.y_kind = 2; }
+    else if (y) { pa.y = y; pa.ldy = H; pa.y_kind = 1; }
+    else { pa.y = nullptr; pa.ldy = 0; pa.y_kind = 0; }
+    pa.hT = hT; pa.cT = cT; pa.gp = gp;
+    pa.flags = sc<unsigned>(off_flags);
+    pa.trace = trace_buffer(TRACE_SB_FWD);   // diagnostics only (null: no stamps)
+    CUDA_TRY(cudaMemsetAsync(pa.flags, 0, 4096, st));
+    lstm_fwd_persist_launch(kind, Hrow(0), Um, Tmax, pa, st);
+    for (int t = t0; t < t1; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
+  } else if (ot == OT::BF16 && var.fwd_mode > 0 && var.fwd_mode < 3) {
     // K2 fused: GEMM + gate epilogue in one kernel (per step, or persistent over all steps)
     const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1});
     RecFwdArgs ra;

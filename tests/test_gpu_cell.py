@@ -71,6 +71,50 @@ def test_fused_forward_modes(cell, fwd):
     _check(cell, 6, 260, 64, 192, "bf16", synth.config_seed(5) + 40, TOL_BF16, variant=f"fwd={fwd}")
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+@pytest.mark.parametrize("T,B,H", [(5, 64, 2048), (4, 100, 256), (3, 16, 200), (6, 1, 64)])
+def test_small_batch_persistent_forward_bitwise(cell, T, B, H):
+    """K2 small-batch persistent form (fwd=3: one cooperative launch, U slices resident in shared
+    memory, fused gate epilogue, grid counter per step) gives the same bits as GEMM + pointwise
+    (fwd=0) for every output and gradient — H = 2048 streams part of U (18 of 32 k-blocks resident),
+    B = 100 uses 128-row A boxes, H = 200 has padding units, B = 1 a nearly empty tile — and also
+    with the recompute context (no UH saved by the forward) and against the oracle."""
+    I = 64
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, 93, bf16=True)
+    ref = None
+    for v in ("fwd=0", "fwd=3", "fwd=3,rc=1"):
+        out, g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, "bf16", v)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    _check(cell, T, B, I, H, "bf16", 93, TOL_BF16, variant="fwd=3")
+
+
+@pytest.mark.parametrize("gc", [1, 2, 3, 4])
+def test_gate_chunking_bitwise(gc):
+    """gate_chunking (§8(a.9), P:196 / P:220): the hoisted gate projection as 2 or 4 GEMMs over
+    gate-column blocks, on one stream or alternating over two, gives the same bits as the
+    one fused GEMM — outputs and every gradient — and the AV is in the live update tree."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H = 4, 96, 64, 320
+    p, inp, dY, dhT, dcT = make_cell_case("milstm", T, B, I, H, 95, bf16=True)
+    ref = None
+    for v in ("gc=0", f"gc={gc}"):
+        out, g, c = run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", v)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    c.tune_mode(A.TUNE_ON)
+    c.tune_next()
+    assert "gate_chunking" in c.tune_report()["tree_avs"]
+
+
 @pytest.mark.parametrize("cell", ["lstm", "milstm", "sublstm"])
 def test_fused_pair_forward_ragged(cell):
     """The CTA-pair fused forward (fwd=1): ragged batch (a half-empty CTA pair), hidden size not a
