@@ -44,6 +44,7 @@ extern const char* const ROLE_NAMES[G_ROLES];
 // One binding of every adaptive variable (the enumerator's output for a cell).
 constexpr int HEAD_CHUNKS[3] = {1, 2, 5};
 constexpr int GCHUNK_N[5] = {1, 2, 4, 2, 4};   // gate GEMMs: 1 fused, G/2, G (G = 4 gate blocks)
+constexpr int WGS_CHUNKS[3] = {1, 4, 10};      // wgrad_schedule time chunks (1: dX after BPTT)
 constexpr int GCHUNK_S[5] = {1, 1, 1, 2, 2};   // streams they run on
 constexpr int WF_CHUNKS[3] = {1, 5, 1 << 20};   // clipped to T: the last option is one chunk per step
 struct Variant {
@@ -55,6 +56,8 @@ struct Variant {
   int head_ov = 0;      // LM head overlapped with the forward chain in HEAD_CHUNKS[head_ov] time chunks (B3)
   int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
   int dpb = 0;          // K11p bucket cap (§8(a.9) dp_bucket): 0 whole tensors, 1/2/3 = 128/32/8 MB pieces
+  int wgs = 0;          // wgrad_schedule (§8(a.9)): the input dgrad dX in WGS_CHUNKS[wgs] time chunks,
+                        // each issued on a side stream as soon as BPTT has produced its rows (0: after BPTT)
   int gchunk = 0;       // gate_chunking (§8(a.9), "chunking the fusion group", P:220 chunk sizes): the
                         // fused gate GEMM of the hoisted projection as GCHUNK_N[gchunk] GEMMs over gate-column
                         // ranges, on GCHUNK_S[gchunk] streams (P:122 two streams vs one fused GEMM)
@@ -198,6 +201,7 @@ class Cell {
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
   virtual int bwd_fusions() const { return 1; }   // number of K4 fusion choices (tuner AV "fuse_bwd")
   virtual int gate_chunkings() const { return 1; }   // options of the tuner AV "gate_chunking" (1: none)
+  virtual int wgrad_schedules() const { return 1; }  // options of the tuner AV "wgrad_schedule" (1: none)
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
   // forward-step hook (set by the LM): called after forward step t is enqueued on the main stream,
@@ -226,7 +230,7 @@ class Cell {
   template <typename T_> T_* sv(size_t off) { return reinterpret_cast<T_*>(saved + off); }
   template <typename T_> T_* sc(size_t off) { return reinterpret_cast<T_*>(scratch + off); }
   void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st,
-                const L2Pf* pf = nullptr);
+                const L2Pf* pf = nullptr, int max_ctas = 0);
   TcGemm& tc_get(int id, const GemmSpec& s, const KCfg& k);   // prepared tensor maps (bf16 path)
   void mark(Region r, int which, cudaStream_t st);
   void tuner_setup();

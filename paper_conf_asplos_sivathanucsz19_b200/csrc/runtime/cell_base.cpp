@@ -27,6 +27,7 @@ std::string Variant::str() const {
   if (recomp) o << ",rc=" << recomp;
   if (dpb) o << ",dpb=" << dpb;
   if (gchunk) o << ",gc=" << gchunk;
+  if (wgs) o << ",wgs=" << wgs;
   return o.str();
 }
 
@@ -50,6 +51,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "dpb") {
       v.dpb = std::stoi(val);
       ASTRA_CHECK_ARG(v.dpb >= 0 && v.dpb <= 3, "variant: dpb must be 0..3 (whole tensors, 128, 32 or 8 MB buckets)");
+      continue;
+    }
+    if (k == "wgs") {
+      v.wgs = std::stoi(val);
+      ASTRA_CHECK_ARG(v.wgs >= 0 && v.wgs <= 2, "variant: wgs (wgrad_schedule) must be 0..2");
       continue;
     }
     if (k == "gc") {
@@ -227,9 +233,9 @@ TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
 }
 
 void Cell::run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st,
-                    const L2Pf* pf) {
+                    const L2Pf* pf, int max_ctas) {
   if (ot == OT::BF16) {
-    tc_gemm_launch(tc_get(id, s, k), e, az, bz, st, 0, pf);
+    tc_gemm_launch(tc_get(id, s, k), e, az, bz, st, max_ctas, pf);
   } else {
     const float* A = (const float*)s.A.ptr + (long)az * s.A.zstride;
     const float* Bm = (const float*)s.B.ptr + (long)bz * s.B.zstride;
@@ -402,6 +408,10 @@ void Cell::tuner_setup() {
   if (ot == OT::BF16 && chain_prefetch())
     t = "(pre " + t + " (par (leaf pf_fwd 2 t_fwd) (leaf pf_bwd 2 t_bptt)))";
   if (!side.empty()) t = t.empty() ? "(leaf wg_side 2 t_se4)" : "(pre " + t + " (leaf wg_side 2 t_se4))";
+  // §8(a.9) wgrad_schedule (P:245-247 equivalence over streams): the input dgrad's time chunks run
+  // on a side stream during BPTT instead of after it; BPTT + SE4 together, so the step metric
+  if (ot == OT::BF16 && !side.empty() && wgrad_schedules() > 1)
+    t = "(pre " + t + " (leaf wgrad_schedule " + std::to_string(wgrad_schedules()) + " t_step))";
   // B3 stream assignment for the LM head: time-chunked on a side stream, overlapping the forward
   // chain (its chunks' logits / CE / dgrad) and the BPTT chain (its weight gradient); step metric
   if (lm_mode && lm_role == 2 && !side.empty() && T >= 2)
@@ -443,6 +453,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "recomp") { v.recomp = o; continue; }
     if (n == "dp_bucket") { v.dpb = o; continue; }
     if (n == "gate_chunking") { v.gchunk = o; continue; }
+    if (n == "wgrad_schedule") { v.wgs = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

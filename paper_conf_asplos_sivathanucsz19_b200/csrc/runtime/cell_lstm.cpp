@@ -64,6 +64,8 @@ class LstmCell : public Cell {
     scratch_bytes = c.o;
   }
   ~LstmCell() override {
+    for (cudaEvent_t e : ev_wgs)
+      if (e) cudaEventDestroy(e);
     for (int i = 0; i < 2; ++i) {
       if (ev_rc_done[i]) cudaEventDestroy(ev_rc_done[i]);
       if (ev_rc_free[i]) cudaEventDestroy(ev_rc_free[i]);
@@ -79,6 +81,8 @@ class LstmCell : public Cell {
   // K2 fusion choices (AV fuse_fwd): 0 GEMM + pointwise, 1 fused per step (CTA pairs), 2 fused
   // persistent (256-column tiles), 3 small-batch persistent with the U slice resident (B ≤ 128)
   int gate_chunkings() const override { return ot == OT::BF16 ? (side.empty() ? 3 : 5) : 1; }
+  int wgrad_schedules() const override { return (ot == OT::BF16 && T >= 4) ? 3 : 1; }
+  cudaEvent_t ev_wgs[11] = {};          // wgrad_schedule: chunk k's D_wx rows complete (+ join)
   int fwd_fusions() const override { return (ot == OT::BF16 && lstm_fwd_persist_supported(B, Hp)) ? 4 : 3; }
   bool chain_prefetch() const override { return true; }
   bool supports_ranges() const override { return true; }
@@ -394,6 +398,34 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     issue((t1 - 1) / RC);
     issue((t1 - 1) / RC - 1);
   }
+  auto dx_rows = [&](int r0, int r1, int id, cudaStream_t s_, int max_ctas) {   // dX = D_wx·Wᵀ, timesteps [r0, r1)
+    const long rows = (long)(r1 - r0) * B;   // (row chunks of one GEMM: same bits, R1)
+    GemmSpec gx;
+    gx.A = mat(Dwx + (size_t)r0 * B * NG * e, NG, rows, NG);
+    gx.B = mat(Wm, I, NG, Ip);
+    gx.b_mn = true;
+    gx.M = (int)rows; gx.N = I; gx.K = NG;
+    if (lm_mode)
+      run_gemm(id, gx, epi((float*)dx + (size_t)r0 * B * Ip, Ip, (int)rows, I), 0, 0, var.g[G_DX], s_, nullptr, max_ctas);
+    else
+      run_gemm(id, gx, epi((char*)dx + (size_t)r0 * B * I * ot_size(ot), I, (int)rows, I, ot == OT::BF16), 0, 0,
+               var.g[G_DX], s_, nullptr, max_ctas);
+  };
+  // wgrad_schedule (§8(a.9)): the input dgrad in time chunks on a side stream, each as
+  // soon as the chain has produced its D_wx rows, on the SMs the per-step BPTT GEMM leaves free
+  const int wgs_n = (whole && dx && var.wgs > 0 && !side.empty() && ot == OT::BF16 && !fuse)
+                        ? std::min(WGS_CHUNKS[var.wgs], T) : 1;
+  cudaStream_t wst = side.empty() ? st : side.back();
+  int wgs_k = 0;
+  auto wgs_lo = [&](int k) { return (int)((long)T * (wgs_n - 1 - k) / wgs_n); };   // chunk k: [lo(k), lo(k-1))
+  int wgs_ctas = 0;
+  if (wgs_n > 1) {
+    const KCfg& kb = var.g[G_BPTT];
+    const int chain = cdiv(B, TC_BM * kb.cg) * cdiv(Hp, kb.bn) * bp.ksplit * kb.cg;
+    wgs_ctas = std::max(8, num_sms() - chain);
+    for (int i = 0; i < wgs_n + 1; ++i)
+      if (!ev_wgs[i]) CUDA_TRY(cudaEventCreateWithFlags(&ev_wgs[i], cudaEventDisableTiming));
+  }
   for (int t = t1 - 1; t >= t0; --t) {
     const int kc = t / RC;
     if (rc && !fuse && rs != st && t == chunk_hi(kc) - 1) CUDA_TRY(cudaStreamWaitEvent(st, ev_rc_done[kc & 1], 0));
@@ -437,21 +469,15 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
       released[kc & 1] = true;
       issue(kc - 2);
     }
+    if (wgs_n > 1 && t == wgs_lo(wgs_k)) {   // D_wx of chunk wgs_k complete: its dX rows on the side stream
+      const int hi = wgs_k == 0 ? T : wgs_lo(wgs_k - 1);
+      CUDA_TRY(cudaEventRecord(ev_wgs[wgs_k], st));
+      CUDA_TRY(cudaStreamWaitEvent(wst, ev_wgs[wgs_k], 0));
+      dx_rows(t, hi, 400000 + t * 1024 + (hi - t), wst, wgs_ctas);
+      ++wgs_k;
+    }
   }
-  auto dx_rows = [&](int r0, int r1, int id) {   // dX = D_wx·Wᵀ for timesteps [r0, r1) (row chunk: same bits)
-    const long rows = (long)(r1 - r0) * B;
-    GemmSpec gx;
-    gx.A = mat(Dwx + (size_t)r0 * B * NG * e, NG, rows, NG);
-    gx.B = mat(Wm, I, NG, Ip);
-    gx.b_mn = true;
-    gx.M = (int)rows; gx.N = I; gx.K = NG;
-    if (lm_mode)
-      run_gemm(id, gx, epi((float*)dx + (size_t)r0 * B * Ip, Ip, (int)rows, I), 0, 0, var.g[G_DX], st);
-    else
-      run_gemm(id, gx, epi((char*)dx + (size_t)r0 * B * I * ot_size(ot), I, (int)rows, I, ot == OT::BF16), 0, 0,
-               var.g[G_DX], st);
-  };
-  if (!whole && dx) dx_rows(t0, t1, 200000 + t0 * 1024 + (t1 - t0));   // the layer below's dy for this chunk, right away
+  if (!whole && dx) dx_rows(t0, t1, 200000 + t0 * 1024 + (t1 - t0), st, 0);   // the layer below's dy for this chunk, right away
   if (bwd_hook) bwd_hook();
   if (t0 > 0) return;
   if (dh0) run_gemm(3, bp0, epi(dh0, H, B, H), 0, 0, var.g[G_BPTT], st);
@@ -488,9 +514,9 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   mark(R_DW, 1, st);
   grad_bucket(g("W"), (size_t)I * 4 * H, st);
 
-  if (dx && whole) {
+  if (dx && whole && wgs_n == 1) {
     mark(R_DX, 0, st);
-    dx_rows(0, T, 6);
+    dx_rows(0, T, 6, st, 0);
     mark(R_DX, 1, st);
   }
   float* gq[4] = {g("b"), nullptr, nullptr, nullptr};
@@ -500,6 +526,10 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   if (st_u != st) {
     CUDA_TRY(cudaEventRecord(ev_join, st_u));
     CUDA_TRY(cudaStreamWaitEvent(st, ev_join, 0));
+  }
+  if (wgs_n > 1) {   // the dX chunks (on the side stream since BPTT) are part of the step
+    CUDA_TRY(cudaEventRecord(ev_wgs[wgs_n], wst));
+    CUDA_TRY(cudaStreamWaitEvent(st, ev_wgs[wgs_n], 0));
   }
   mark(R_SE4, 1, st);
   if (!lm_mode) grad_join(st);

@@ -115,6 +115,28 @@ def test_gate_chunking_bitwise(gc):
     assert "gate_chunking" in c.tune_report()["tree_avs"]
 
 
+@pytest.mark.parametrize("v", ["wgs=1", "wgs=2", "wgs=2,wg_side=1,rc=1", "wgs=1,hov=0,fwd=3"])
+def test_wgrad_schedule_bitwise(v):
+    """wgrad_schedule (§8(a.9)): the input dgrad in 4 / 10 time chunks on a side stream
+    while BPTT is still running (with the dU side stream and the recompute context too) gives the
+    same bits as dX after BPTT, and the AV is in the live update tree."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H = 10, 64, 128, 192
+    p, inp, dY, dhT, dcT = make_cell_case("milstm", T, B, I, H, 97, bf16=True)
+    ref = None
+    for var in ("wgs=0", v):
+        out, g, c = run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", var.replace(",hov=0", ""))
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (var, k)
+    c.tune_mode(A.TUNE_ON)
+    c.tune_next()
+    assert "wgrad_schedule" in c.tune_report()["tree_avs"]
+
+
 @pytest.mark.parametrize("cell", ["lstm", "milstm", "sublstm"])
 def test_fused_pair_forward_ragged(cell):
     """The CTA-pair fused forward (fwd=1): ragged batch (a half-empty CTA pair), hidden size not a

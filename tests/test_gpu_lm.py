@@ -133,7 +133,8 @@ def _steps_params(variant, graph, steps=8):
 
 
 @pytest.mark.parametrize("variant", ["fwd=0", "a1=256.1.1.2,rec=256.1.1.2,bptt=128.1.1.2,du=256.1.1.2,dw=128.1.1.2,"
-                                     "dx=256.1.1.2,head=256.1.1.2,wg_side=1,fwd=1"])
+                                     "dx=256.1.1.2,head=256.1.1.2,wg_side=1,fwd=1",
+                                     "fwd=0,hov=1,wgs=2,gc=3,wg_side=1"])
 def test_graph_replay_bitwise(variant):
     """CUDA-graph replay of frozen steps (the bench path) is bitwise identical to kernel-by-kernel
     enqueueing, over 8 SGD steps (state carried between steps)."""
@@ -355,3 +356,13 @@ def test_tune_next_never_blocks():
     assert busy >= 36, busy      # the GPU was still working after ≥ 90 % of the calls
     rep = c.tune_report()
     assert rep["configs_explored"] >= 10 and rep["converged"]
+
+
+@pytest.mark.parametrize("variant", ["hov=1,wgs=2,gc=3,wg_side=1", "wgs=1,gc=4,fwd=3", "gc=2,wgs=2,rc=1"])
+def test_stream_schedules_lm_bitwise(variant):
+    """The stream-assignment variants together — head overlap, wgrad_schedule's dX chunks during
+    BPTT, gate_chunking's projection GEMMs on two streams, the small-batch persistent forward —
+    give the default variant's parameters bit for bit after 8 SGD steps (CUDA-graph replay)."""
+    pa, la = _steps_params("fwd=0", graph=True)
+    pb, lb = _steps_params(variant, graph=True)
+    assert torch.equal(pa, pb) and la == lb
