@@ -485,11 +485,255 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, gcol(0, j), nq, first);
 }
 
+// K4 backward half, wide form (AV bwd_pw = 1; measured faster at small batch — B = 64: BPTT chain
+// 2.37 → 1.96 ms at cfg5 shapes — and slower at B = 512, where the row-lane kernel above fills the
+// GPU in one wave).  Same row
+// arithmetic and the same R5 column-sum order, different work split: CTA = one 32-row partial chunk
+// x 32 units, thread = (row, 4 consecutive units), so every operand of a row is one 16-byte load per
+// gate (float4 WX / UH / dh partials / dc / c) and all 32 rows of the chunk are in flight at once
+// (the row-per-thread-lane kernel walks 8 rows one after another and is memory-latency bound).
+// The per-row contributions (da, and for MI-LSTM wx, uh) go to shared memory; then thread (unit,
+// gate, lane y) runs lane y's fixed-order accumulation over rows y, y+4, ..., y+28 exactly as the
+// other kernel's thread (tx = unit, ty = y) does, and the lanes are combined in y order.
+constexpr int BW2_UB = 32;                   // units per CTA
+constexpr int BW2_THREADS = BWD_RB * BW2_UB / 4;   // 256: 32 rows x 8 unit quads
+
+template <typename TDY>
+__device__ __forceinline__ void load4_dy(const TDY* p, bool vec, float (&v)[4], int nvalid);
+template <>
+__device__ __forceinline__ void load4_dy<float>(const float* p, bool vec, float (&v)[4], int nvalid) {
+  if (vec) {
+    const float4 x = __ldcs(reinterpret_cast<const float4*>(p));
+    v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  } else {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) v[u] = u < nvalid ? p[u] : 0.f;
+  }
+}
+template <>
+__device__ __forceinline__ void load4_dy<__nv_bfloat16>(const __nv_bfloat16* p, bool vec, float (&v)[4], int nvalid) {
+  if (vec) {
+    const uint2 x = *reinterpret_cast<const uint2*>(p);
+    const __nv_bfloat162 a = *reinterpret_cast<const __nv_bfloat162*>(&x.x), b = *reinterpret_cast<const __nv_bfloat162*>(&x.y);
+    v[0] = __low2float(a); v[1] = __high2float(a); v[2] = __low2float(b); v[3] = __high2float(b);
+  } else {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) v[u] = u < nvalid ? __bfloat162float(p[u]) : 0.f;
+  }
+}
+__device__ __forceinline__ float4 ld4(const float* p) { return *reinterpret_cast<const float4*>(p); }
+__device__ __forceinline__ float4 ld4cs(const float* p) { return __ldcs(reinterpret_cast<const float4*>(p)); }
+__device__ __forceinline__ float f4(const float4& v, int u) { return u == 0 ? v.x : u == 1 ? v.y : u == 2 ? v.z : v.w; }
+template <typename T>
+__device__ __forceinline__ void store4(T* p, const float (&v)[4]);
+template <>
+__device__ __forceinline__ void store4<float>(float* p, const float (&v)[4]) {
+  *reinterpret_cast<float4*>(p) = make_float4(v[0], v[1], v[2], v[3]);
+}
+template <>
+__device__ __forceinline__ void store4<__nv_bfloat16>(__nv_bfloat16* p, const float (&v)[4]) {
+  __nv_bfloat162 a = __floats2bfloat162_rn(v[0], v[1]), b = __floats2bfloat162_rn(v[2], v[3]);
+  uint2 x;
+  x.x = *reinterpret_cast<uint32_t*>(&a);
+  x.y = *reinterpret_cast<uint32_t*>(&b);
+  *reinterpret_cast<uint2*>(p) = x;
+}
+
+template <int KIND, typename T, typename TDY>
+__global__ void __launch_bounds__(BW2_THREADS, 2)
+    lstm_bwd_pw2_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
+                        long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
+                        const float* __restrict__ WX, const float* __restrict__ UH, const float* __restrict__ c_new,
+                        const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
+                        T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
+  constexpr int NV = BwdNV<KIND>::value;
+  constexpr int NP = KIND == K_MILSTM ? 4 : 1;
+  constexpr int NC = KIND == K_MILSTM ? 3 : 1;    // per (row, unit, gate): da (, wx, uh)
+  constexpr bool F = FastMath<T>::value;
+  extern __shared__ float smf[];
+  float* con = smf;                                // [NC][4][32 rows][BW2_UB]; later red [4][NV][BW2_UB]
+  float* sgp = smf + NC * 4 * BWD_RB * BW2_UB;     // [NP][4][BW2_UB]
+  const int tid = threadIdx.x;
+  const int qd = tid % (BW2_UB / 4), r = tid / (BW2_UB / 4);
+  const int u0 = blockIdx.x * BW2_UB, ul = 4 * qd, j0 = u0 + ul;
+  const int chunk = blockIdx.y, b0 = chunk * BWD_RB, b = b0 + r;
+  const long NG = 4L * Hp;
+  for (int i = tid; i < NP * 4 * BW2_UB; i += BW2_THREADS) {   // parameters: not written by the chain
+    const int pi = i / (4 * BW2_UB), g = (i / BW2_UB) % 4, u = i % BW2_UB, j = u0 + u;
+    const float* src = pi == 0 ? gp.b : pi == 1 ? gp.alpha : pi == 2 ? gp.beta1 : gp.beta2;
+    sgp[i] = j < H ? src[g * H + j] : 0.f;
+  }
+  const bool rowok = b < B;
+  const int nvalid = min(4, H - j0);            // units of this quad that exist (≤ 0: padding only)
+  const int c0 = gcol(0, j0);
+  const long ro = (long)b * Hp + j0;
+  // everything except the GEMM's dh_rec is older than the grid dependency: loaded before the wait
+  // (not at the first step, whose predecessor may have produced dy or initialised dc)
+  float4 w4[4], h4[4], dc4, cp4, cn4;
+  float dyv[4];
+  auto load_old = [&] {
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      w4[g] = ld4cs(WX + (long)b * NG + c0 + g * GATE_U);
+      h4[g] = ld4cs(UH + (long)b * NG + c0 + g * GATE_U);
+    }
+    dc4 = ld4(dc + ro);
+    cp4 = ld4cs(c_prev + ro);
+    cn4 = ld4cs(c_new + ro);
+    load4_dy<TDY>(dy + (long)b * ldy + j0, (ldy % 4 == 0) && nvalid == 4 && ((uintptr_t)dy % (4 * sizeof(TDY))) == 0,
+                  dyv, nvalid);
+  };
+  const bool early = !first;
+  if (early && rowok && nvalid > 0) load_old();
+  pdl_wait();
+  pdl_trigger();
+  if (!early && rowok && nvalid > 0) load_old();
+  __syncthreads();   // parameters staged
+  if (rowok) {
+    float duh4[4][4], dwx4[4][4], dcn[4];   // [unit][gate]
+    auto put = [&](int u, int g, float da, float w, float h) {   // this row's column-sum contribution
+      con[((0 * 4 + g) * BWD_RB + r) * BW2_UB + ul + u] = da;
+      if (KIND == K_MILSTM) {
+        con[((1 * 4 + g) * BWD_RB + r) * BW2_UB + ul + u] = w;
+        con[((2 * 4 + g) * BWD_RB + r) * BW2_UB + ul + u] = h;
+      }
+    };
+    if (nvalid > 0) {
+      float dh[4];
+      if (dh_rec) {   // split-K partials of dh_rec summed in chunk order, then added to dy
+        const bool vec = nvalid == 4 && (ld_dh % 4) == 0 && (split_stride % 4) == 0 && ((uintptr_t)dh_rec & 15) == 0;
+        if (vec) {
+          float4 pv[SPLIT_MAX];
+#pragma unroll
+          for (int k = 0; k < SPLIT_MAX; ++k) pv[k] = k < nsplit ? ld4(dh_rec + (long)b * ld_dh + j0 + k * split_stride) : make_float4(0, 0, 0, 0);
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            float s = f4(pv[0], u);
+#pragma unroll
+            for (int k = 1; k < SPLIT_MAX; ++k)
+              if (k < nsplit) s = __fadd_rn(s, f4(pv[k], u));
+            for (int k = SPLIT_MAX; k < nsplit; ++k) s = __fadd_rn(s, dh_rec[(long)b * ld_dh + j0 + u + k * split_stride]);
+            dh[u] = __fadd_rn(dyv[u], s);
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            dh[u] = u < nvalid ? __fadd_rn(dyv[u], sum_split(dh_rec + (long)b * ld_dh + j0 + u, nsplit, split_stride)) : 0.f;
+        }
+      } else {
+#pragma unroll
+        for (int u = 0; u < 4; ++u) dh[u] = dyv[u];
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        float w[4], h[4], bb[4], al[4], be1[4], be2[4], da[4], duh[4], dwx[4];
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          w[g] = f4(w4[g], u);
+          h[g] = f4(h4[g], u);
+          bb[g] = sgp[g * BW2_UB + ul + u];
+          al[g] = KIND == K_MILSTM ? sgp[(NP > 1 ? 1 : 0) * 4 * BW2_UB + g * BW2_UB + ul + u] : 0.f;
+          be1[g] = KIND == K_MILSTM ? sgp[(NP > 2 ? 2 : 0) * 4 * BW2_UB + g * BW2_UB + ul + u] : 0.f;
+          be2[g] = KIND == K_MILSTM ? sgp[(NP > 3 ? 3 : 0) * 4 * BW2_UB + g * BW2_UB + ul + u] : 0.f;
+        }
+        float dcv = f4(dc4, u);
+        if (u < nvalid) {
+          lstm_bwd_da<KIND, F>(w, h, dh[u], dcv, f4(cp4, u), f4(cn4, u), bb, al, be1, be2, da, duh, dwx);
+        } else {   // padding units: exact zeros everywhere (gradients, contributions, dc)
+#pragma unroll
+          for (int g = 0; g < 4; ++g) { da[g] = 0.f; duh[g] = 0.f; dwx[g] = 0.f; w[g] = 0.f; h[g] = 0.f; }
+          dcv = 0.f;
+        }
+        dcn[u] = dcv;
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          put(u, g, da[g], w[g], h[g]);
+          duh4[u][g] = duh[g]; dwx4[u][g] = dwx[g];
+        }
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        dcn[u] = 0.f;
+#pragma unroll
+        for (int g = 0; g < 4; ++g) { put(u, g, 0.f, 0.f, 0.f); duh4[u][g] = 0.f; dwx4[u][g] = 0.f; }
+      }
+    }
+    // outputs: D_uh / D_wx per gate (4 units = one 8- or 16-byte store), dc
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      float v[4] = {duh4[0][g], duh4[1][g], duh4[2][g], duh4[3][g]};
+      store4<T>(D_uh + (long)b * NG + c0 + g * GATE_U, v);
+      if (KIND == K_MILSTM) {
+        float x[4] = {dwx4[0][g], dwx4[1][g], dwx4[2][g], dwx4[3][g]};
+        store4<T>(D_wx + (long)b * NG + c0 + g * GATE_U, x);
+      }
+    }
+    *reinterpret_cast<float4*>(dc + ro) = make_float4(dcn[0], dcn[1], dcn[2], dcn[3]);
+  }
+  __syncthreads();
+  // lane sums: thread (u, y) accumulates rows y, y+4, ... of the chunk in ascending order, every gate
+  const int nrows = min(BWD_RB, B - b0);
+  float acc[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) acc[i] = 0.f;
+  const int su = tid % BW2_UB, sy = tid / BW2_UB;   // tid < 4·BW2_UB = 128 do the sums
+  if (tid < BWD_RY * BW2_UB) {
+    for (int rr = sy; rr < nrows; rr += BWD_RY) {
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        const float da = con[((0 * 4 + g) * BWD_RB + rr) * BW2_UB + su];
+        const float w = KIND == K_MILSTM ? con[((1 * 4 + g) * BWD_RB + rr) * BW2_UB + su] : 0.f;
+        const float h = KIND == K_MILSTM ? con[((2 * 4 + g) * BWD_RB + rr) * BW2_UB + su] : 0.f;
+        lstm_bwd_acc<KIND, F>(acc, g, da, w, h);
+      }
+    }
+  }
+  __syncthreads();   // contributions consumed: the same memory holds the lane sums
+  float* red = con;  // [4 lanes][NV][BW2_UB]
+  if (tid < BWD_RY * BW2_UB) {
+#pragma unroll
+    for (int i = 0; i < NV; ++i) red[(sy * NV + i) * BW2_UB + su] = acc[i];
+  }
+  __syncthreads();
+  // lanes combined in y order and folded into the chunk's partials (bwd_chunk_finalize's order)
+  for (int item = tid; item < NV * BW2_UB; item += BW2_THREADS) {
+    const int u = item % BW2_UB, i = item / BW2_UB, j = u0 + u;
+    const int q = i / 4, g = i % 4;
+    if (q >= nq || j >= Hp) continue;
+    float v = 0.f;
+#pragma unroll
+    for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[(y * NV + i) * BW2_UB + u]);
+    float* pp = partials + (long)chunk * nq * NG + (long)q * NG + gcol(g, j);
+    *pp = first ? v : __fadd_rn(*pp, v);
+  }
+}
+
 template <int KIND, typename T>
 static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32, const float* dh_rec,
                           long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH, const float* c_new,
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
-                          bool first, cudaStream_t st) {
+                          bool first, cudaStream_t st, int form) {
+  if (form == 1) {
+    constexpr int NC = KIND == K_MILSTM ? 3 : 1, NP = KIND == K_MILSTM ? 4 : 1;
+    const size_t smem = (size_t)(NC * 4 * BWD_RB * BW2_UB + NP * 4 * BW2_UB) * 4;
+    dim3 grid2(cdiv(Hp, BW2_UB), lstm_bwd_row_chunks(B));
+    if (dy_f32 || dy_ot == OT::F32) {
+      auto k = lstm_bwd_pw2_kernel<KIND, T, float>;
+      static bool attr = false;
+      if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
+      launch_pdl(k, grid2, dim3(BW2_THREADS), smem, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit,
+                 split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first);
+    } else {
+      auto k = lstm_bwd_pw2_kernel<KIND, T, __nv_bfloat16>;
+      static bool attr = false;
+      if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
+      launch_pdl(k, grid2, dim3(BW2_THREADS), smem, st, 1, B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh,
+                 nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first);
+    }
+    LAUNCH_CHECK();
+    return;
+  }
   dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
   dim3 block(BWD_UX, BWD_RY);
   if (dy_f32 || dy_ot == OT::F32)
@@ -506,15 +750,15 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
                         const float* dh_rec, long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH,
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
-                        float* partials, int nq, bool first, cudaStream_t st) {
+                        float* partials, int nq, bool first, cudaStream_t st, int form) {
 #define BWD_CASE(K)                                                                                            \
   if (kind == K) {                                                                                             \
     if (ot == OT::BF16)                                                                                        \
       bwd_pw_launch<K, __nv_bfloat16>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, \
-                                      gp, D_uh, D_wx, partials, nq, first, st);                                \
+                                      gp, D_uh, D_wx, partials, nq, first, st, form);                          \
     else                                                                                                       \
       bwd_pw_launch<K, float>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp,  \
-                              D_uh, D_wx, partials, nq, first, st);                                            \
+                              D_uh, D_wx, partials, nq, first, st, form);                                      \
     return;                                                                                                    \
   }
   BWD_CASE(K_LSTM)

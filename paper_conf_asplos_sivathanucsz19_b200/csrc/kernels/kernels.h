@@ -45,7 +45,9 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
                         const float* dh_rec, long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH,
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
-                        float* partials, int nq, bool first, cudaStream_t st);
+                        float* partials, int nq, bool first, cudaStream_t st, int form = 0);
+// form (AV "bwd_pw", bitwise interchangeable): 0 the row-lane kernel (thread = unit, rows walked 4
+// lanes x 8), 1 the wide kernel (thread = row x 4 units, all rows of a 32-row chunk in flight).
 int lstm_bwd_row_chunks(int B);
 // grads_q[e] = Σ_chunk partials[chunk][q][gcol(e)] for q < nq (external e < 4H).
 void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,

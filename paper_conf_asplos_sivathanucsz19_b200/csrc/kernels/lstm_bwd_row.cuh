@@ -17,38 +17,65 @@ constexpr int BWD_RY = 4;   // row lanes (threadIdx.y)
 template <int KIND>
 struct BwdNV { static constexpr int value = KIND == K_MILSTM ? 16 : 4; };   // quantities per unit: q*4 + gate
 
-// Cell backward of one (row, unit): pre-activations from (w, h) = (WX, UH) and the gate
-// parameters, cell_bwd, then D_uh / D_wx (bf16 or fp32, gate stride GATE_U) and the quantities
-// accumulated for the column sums: q0 da (→ db), q1 da·wx·uh (→ dα), q2 da·uh (→ dβ1), q3 da·wx (→ dβ2).
-template <int KIND, typename T>
-__device__ __forceinline__ void lstm_bwd_row(const float (&w)[4], const float (&h)[4], float dh, float& dcv, float cp,
-                                             float cn, const float (&bb)[4], const float (&al)[4],
-                                             const float (&be1)[4], const float (&be2)[4],
-                                             float (&acc)[BwdNV<KIND>::value], T* duhp, T* dwxp) {
-  constexpr int NV = BwdNV<KIND>::value;
-  constexpr bool F = FastMath<T>::value;   // bf16 path: fused multiply-adds (reading R27)
-  float a[4], da[4];
+// Cell backward of one (row, unit), split in two so a kernel may run the row arithmetic and the
+// column-sum accumulation in different threads (lstm_bwd_pw2_kernel) with the same operations:
+//   lstm_bwd_da:  pre-activations from (w, h) = (WX, UH) and the gate parameters, cell_bwd → da,
+//                 and the gate gradients D_uh / D_wx (bf16 or fp32) returned in duh / dwx;
+//   lstm_bwd_acc: the quantities accumulated for the column sums, in this order:
+//                 q0 da (→ db), q1 da·wx·uh (→ dα), q2 da·uh (→ dβ1), q3 da·wx (→ dβ2).
+template <int KIND, bool F>
+__device__ __forceinline__ void lstm_bwd_da(const float (&w)[4], const float (&h)[4], float dh, float& dcv, float cp,
+                                            float cn, const float (&bb)[4], const float (&al)[4],
+                                            const float (&be1)[4], const float (&be2)[4], float (&da)[4],
+                                            float (&duh)[4], float (&dwx)[4]) {
+  float a[4];
 #pragma unroll
   for (int g = 0; g < 4; ++g) a[g] = preact<KIND, F>(w[g], h[g], bb[g], al[g], be1[g], be2[g]);
   cell_bwd<KIND, F>(a, cp, cn, dh, dcv, da);
 #pragma unroll
   for (int g = 0; g < 4; ++g) {
-    acc[g] = __fadd_rn(acc[g], da[g]);
     if (KIND == K_MILSTM) {
       const float gu = F ? __fmaf_rn(al[g], w[g], be1[g]) : __fadd_rn(__fmul_rn(al[g], w[g]), be1[g]);
       const float gw = F ? __fmaf_rn(al[g], h[g], be2[g]) : __fadd_rn(__fmul_rn(al[g], h[g]), be2[g]);
-      duhp[g * GATE_U] = from_f<T>(__fmul_rn(da[g], gu));
-      __stcs(dwxp + g * GATE_U, from_f<T>(__fmul_rn(da[g], gw)));
-      const float dw = __fmul_rn(da[g], w[g]);
-      float& r4 = acc[(NV > 4 ? 4 : 0) + g];
-      r4 = F ? __fmaf_rn(dw, h[g], r4) : __fadd_rn(r4, __fmul_rn(dw, h[g]));
-      float& r8 = acc[(NV > 8 ? 8 : 0) + g];
-      r8 = F ? __fmaf_rn(da[g], h[g], r8) : __fadd_rn(r8, __fmul_rn(da[g], h[g]));
-      float& r12 = acc[(NV > 12 ? 12 : 0) + g];
-      r12 = __fadd_rn(r12, dw);
+      duh[g] = __fmul_rn(da[g], gu);
+      dwx[g] = __fmul_rn(da[g], gw);
     } else {
-      duhp[g * GATE_U] = from_f<T>(da[g]);
+      duh[g] = da[g];
+      dwx[g] = da[g];
     }
+  }
+}
+
+template <int KIND, bool F>
+__device__ __forceinline__ void lstm_bwd_acc(float (&acc)[BwdNV<KIND>::value], int g, float da, float w, float h) {
+  constexpr int NV = BwdNV<KIND>::value;
+  acc[g] = __fadd_rn(acc[g], da);
+  if (KIND == K_MILSTM) {
+    const float dw = __fmul_rn(da, w);
+    float& r4 = acc[(NV > 4 ? 4 : 0) + g];
+    r4 = F ? __fmaf_rn(dw, h, r4) : __fadd_rn(r4, __fmul_rn(dw, h));
+    float& r8 = acc[(NV > 8 ? 8 : 0) + g];
+    r8 = F ? __fmaf_rn(da, h, r8) : __fadd_rn(r8, __fmul_rn(da, h));
+    float& r12 = acc[(NV > 12 ? 12 : 0) + g];
+    r12 = __fadd_rn(r12, dw);
+  }
+}
+
+// Both halves for one (row, unit) with the accumulation in this thread (the unfused kernel's and the
+// fused BPTT kernel's form): D_uh / D_wx stored at gate stride GATE_U.
+template <int KIND, typename T>
+__device__ __forceinline__ void lstm_bwd_row(const float (&w)[4], const float (&h)[4], float dh, float& dcv, float cp,
+                                             float cn, const float (&bb)[4], const float (&al)[4],
+                                             const float (&be1)[4], const float (&be2)[4],
+                                             float (&acc)[BwdNV<KIND>::value], T* duhp, T* dwxp) {
+  constexpr bool F = FastMath<T>::value;   // bf16 path: fused multiply-adds (reading R27)
+  float da[4], duh[4], dwx[4];
+  lstm_bwd_da<KIND, F>(w, h, dh, dcv, cp, cn, bb, al, be1, be2, da, duh, dwx);
+#pragma unroll
+  for (int g = 0; g < 4; ++g) {
+    lstm_bwd_acc<KIND, F>(acc, g, da[g], w[g], h[g]);
+    duhp[g * GATE_U] = from_f<T>(duh[g]);
+    if (KIND == K_MILSTM) __stcs(dwxp + g * GATE_U, from_f<T>(dwx[g]));
   }
 }
 

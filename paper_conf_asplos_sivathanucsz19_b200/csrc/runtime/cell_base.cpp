@@ -28,6 +28,7 @@ std::string Variant::str() const {
   if (dpb) o << ",dpb=" << dpb;
   if (gchunk) o << ",gc=" << gchunk;
   if (wgs) o << ",wgs=" << wgs;
+  if (bpw) o << ",bpw=" << bpw;
   return o.str();
 }
 
@@ -51,6 +52,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "dpb") {
       v.dpb = std::stoi(val);
       ASTRA_CHECK_ARG(v.dpb >= 0 && v.dpb <= 3, "variant: dpb must be 0..3 (whole tensors, 128, 32 or 8 MB buckets)");
+      continue;
+    }
+    if (k == "bpw") {
+      v.bpw = std::stoi(val);
+      ASTRA_CHECK_ARG(v.bpw == 0 || v.bpw == 1, "variant: bpw (backward pointwise form) must be 0 or 1");
       continue;
     }
     if (k == "wgs") {
@@ -404,6 +410,9 @@ void Cell::tuner_setup() {
     t = "(pre " + t + " (leaf fuse_fwd " + std::to_string(fwd_fusions()) + " t_fwd))";
   if (ot == OT::BF16 && bwd_fusions() > 1)
     t = "(pre " + t + " (leaf fuse_bwd " + std::to_string(bwd_fusions()) + " t_bptt))";
+  // the backward pointwise kernel's form (bwd_kernel AV), against the BPTT-chain time
+  if (ot == OT::BF16 && bwd_pw_forms() > 1)
+    t = "(pre " + t + " (leaf bwd_pw " + std::to_string(bwd_pw_forms()) + " t_bptt))";
   // reading R31: L2 prefetch by the chain GEMMs, per chain, after the kernel and fusion choices
   if (ot == OT::BF16 && chain_prefetch())
     t = "(pre " + t + " (par (leaf pf_fwd 2 t_fwd) (leaf pf_bwd 2 t_bptt)))";
@@ -454,6 +463,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "dp_bucket") { v.dpb = o; continue; }
     if (n == "gate_chunking") { v.gchunk = o; continue; }
     if (n == "wgrad_schedule") { v.wgs = o; continue; }
+    if (n == "bwd_pw") { v.bpw = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

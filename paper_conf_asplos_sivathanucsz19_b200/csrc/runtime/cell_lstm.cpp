@@ -82,6 +82,7 @@ class LstmCell : public Cell {
   // persistent (256-column tiles), 3 small-batch persistent with the U slice resident (B ≤ 128)
   int gate_chunkings() const override { return ot == OT::BF16 ? (side.empty() ? 3 : 5) : 1; }
   int wgrad_schedules() const override { return (ot == OT::BF16 && T >= 4) ? 3 : 1; }
+  int bwd_pw_forms() const override { return ot == OT::BF16 ? 2 : 1; }
   cudaEvent_t ev_wgs[11] = {};          // wgrad_schedule: chunk k's D_wx rows complete (+ join)
   int fwd_fusions() const override { return (ot == OT::BF16 && lstm_fwd_persist_supported(B, Hp)) ? 4 : 3; }
   bool chain_prefetch() const override { return true; }
@@ -463,7 +464,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     }
     lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC, WX + (long)t * B * NG,
                        uh_of(t), Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
-                       Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st);
+                       Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st, var.bpw);
     if (rc && !fuse && t == chunk_lo(kc)) {   // chunk kc consumed: its slot takes chunk kc - 2
       if (rs != st) CUDA_TRY(cudaEventRecord(ev_rc_free[kc & 1], st));
       released[kc & 1] = true;

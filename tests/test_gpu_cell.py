@@ -115,6 +115,27 @@ def test_gate_chunking_bitwise(gc):
     assert "gate_chunking" in c.tune_report()["tree_avs"]
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+@pytest.mark.parametrize("dtype", ["bf16", "fp32"])
+@pytest.mark.parametrize("T,B,H", [(4, 100, 200), (3, 512, 2048), (5, 33, 130)])
+def test_bwd_pointwise_forms_bitwise(cell, dtype, T, B, H):
+    """The backward pointwise kernel's two forms (AV bwd_pw: the wide row x 4-unit kernel and the
+    row-lane kernel) give the same bits — D_uh / D_wx, dc, and the fixed-order bias / α / β column
+    sums (R5) — with ragged row chunks, padding units (H = 130, 200) and the R25 4-way split."""
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, 64, H, 99, bf16=dtype == "bf16")
+    ref = None
+    for v in ("bpw=0", "bpw=1"):
+        out, g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, dtype, v)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    if T * B * H <= 5 * 33 * 130:
+        _check(cell, T, B, 64, H, dtype, 99, TOL_BF16 if dtype == "bf16" else TOL_FP32)
+
+
 @pytest.mark.parametrize("v", ["wgs=1", "wgs=2", "wgs=2,wg_side=1,rc=1", "wgs=1,hov=0,fwd=3"])
 def test_wgrad_schedule_bitwise(v):
     """wgrad_schedule (§8(a.9)): the input dgrad in 4 / 10 time chunks on a side stream
