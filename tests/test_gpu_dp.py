@@ -62,3 +62,73 @@ def test_virtual_dp_mean_of_shards_equals_full_batch():
     # and the full-batch gradient matches the oracle
     lo, go, _ = OLM.lm_forward_backward("milstm", p, tok, np.zeros((B, H)), np.zeros((B, H)))
     assert rel_err(full.view("U", full.grads).cpu().numpy(), go["U"]) <= TOL_FP32
+
+
+def _case_bf16(T, B, I, H, V, seed):
+    from helpers import bf16_round
+    p, tok = _case(T, B, I, H, V, seed)
+    for k in ("W", "U", "E", "W_o"):
+        p[k] = bf16_round(p[k])
+    return p, tok
+
+
+def _nccl_worker(rank, world, port, q, stacked):
+    """One rank per GPU: the library's bucketed NCCL all-reduce (one communicator for the LM,
+    astra_lm_comm_init) on the rank's contiguous batch shard; returns its gradients and loss."""
+    import os
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    try:
+        import torch.distributed as dist
+        import paper_conf_asplos_sivathanucsz19_b200 as A
+        torch.cuda.set_device(rank)
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        T, B, I, H, V = 5, 16, 64, 64, 40
+        p, tok = _case_bf16(T, B, I, H, V, 33)
+        sl = slice(rank * B // world, (rank + 1) * B // world)
+        cells = [A.Cell("milstm", H, I, B // world, T, dtype="bf16", device=rank)]
+        m = A.LM(cells[0], V)
+        m.load(p)
+        uid = [A.comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        m.comm_init(uid[0], rank, world)
+        tokens = torch.as_tensor(np.ascontiguousarray(tok[:, sl]), dtype=torch.int32, device=f"cuda:{rank}")
+        m.fwd_bwd(tokens)
+        torch.cuda.synchronize()
+        q.put((rank, m.grads.cpu().numpy(), float(m.loss.item()), {k: v for k, v in m.param_info.items()}))
+        dist.barrier()
+        dist.destroy_process_group()
+    except Exception as e:   # surface the failure in the parent
+        q.put((rank, None, repr(e), None))
+
+
+@pytest.mark.skipif(torch.cuda.device_count() < 2, reason="NCCL needs one GPU per rank (a 1-GPU box cannot run it)")
+def test_nccl_world2_bucketed_allreduce_vs_oracle_dp():
+    """The NCCL bucketed gradient all-reduce with world = 2 (two GPUs): both ranks hold the same
+    gradients, equal to the fp64 oracle's DP semantics (mean of the two shard-mean gradients,
+    oracle.dp.dp_gradients) within the bf16 tolerance."""
+    import os
+    import torch.multiprocessing as mp
+    from oracle import dp as ODP
+    from helpers import TOL_BF16
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29950 + os.getpid() % 40
+    procs = [ctx.Process(target=_nccl_worker, args=(r, 2, port, q, False)) for r in range(2)]
+    for pr in procs:
+        pr.start()
+    res = {}
+    for _ in range(2):
+        r, g, loss, info = q.get(timeout=300)
+        assert g is not None, loss
+        res[r] = (g, loss, info)
+    for pr in procs:
+        pr.join(60)
+    assert np.array_equal(res[0][0], res[1][0])
+    T, B, I, H, V = 5, 16, 64, 64, 40
+    p, tok = _case_bf16(T, B, I, H, V, 33)
+    _, g_o = ODP.dp_gradients("milstm", p, tok, np.zeros((B, H)), np.zeros((B, H)), 2)
+    info = res[0][2]
+    for k, (off, r_, c_) in info.items():
+        got = res[0][0][off:off + r_ * c_].reshape(np.shape(g_o[k]))
+        assert rel_err(got, g_o[k]) <= TOL_BF16, k
