@@ -125,6 +125,27 @@ bool lstm_fwd_persist_supported(int B, int Hp);
 // Hb: [(Tmax+1)][B][Hp] bf16 h operands; Um: the U mirror [NG][Hp] (tensor maps built per launch).
 void lstm_fwd_persist_launch(int kind, const void* Hb, const void* Um, int Tmax, RecPersistArgs a, cudaStream_t st);
 
+// SC-RNN persistent forward h-chain (scrn_persist.cu, ScrnCell fwd_mode 1): all steps [t0, t1) in one
+// cooperative launch of Hp/16 CTAs, B ≤ 128, the R slice resident, the R33 split kept as TMEM
+// accumulators, h_t = σ(Q_t + Σ partials + b_h) fused.
+struct ScrnPersistArgs {
+  int B, H, Hp, T, t0, t1, nsplit;
+  int nk, kper, ka, a_rows, a_bytes;   // set by the launcher
+  uint32_t idesc;
+  const float* Q;           // [T·B][ldq] hoisted x·A + s·P
+  long ldq;
+  const float* bh;          // [H]
+  float* Hf;                // [(T+1)·B][Hp] fp32 h
+  __nv_bfloat16* HS;        // [(T+1)·B][ldhs] bf16 [h | s] operand rows (h part written)
+  long ldhs;
+  __nv_bfloat16* y;         // optional [T·B][ldy] external y (h part)
+  long ldy;
+  float* hT;
+  unsigned* flags;          // one counter, zeroed before the launch
+};
+bool scrn_fwd_persist_supported(int B, int Hp, int nsplit);
+void scrn_fwd_persist_launch(const void* HS, long ldhs, const void* MR, int Tmax, ScrnPersistArgs a, cudaStream_t st);
+
 bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);
 void lstm_bptt_fused_launch(int kind, bool dy_bf16, const BpttFusedMaps& m, BpttFusedArgs a, cudaStream_t st);
 

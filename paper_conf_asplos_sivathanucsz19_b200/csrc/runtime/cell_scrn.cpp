@@ -16,6 +16,7 @@
 // LM head reads [h | s] as one K-concatenated operand; DZS [T·B][Hp + Sp] likewise holds dz and (1−α)ds.
 #include <algorithm>
 
+#include "../kernels/rec_fused.h"
 #include "cell.h"
 
 namespace astra {
@@ -25,7 +26,7 @@ class ScrnCell : public Cell {
   int S, Sp, Yw, nchunk;
   float alpha;
   size_t off_X, off_XAB, off_Sf, off_HS, off_Hf, off_MAB, off_MP, off_MR;
-  size_t off_Z, off_dH, off_DZS, off_DSP, off_part;
+  size_t off_Z, off_dH, off_DZS, off_DSP, off_part, off_flags;
 
   // Reading R33: both chain GEMMs (h·R and dz·Rᵀ, K = Hp, N = Hp) split over K into s fixed chunks
   // when the batch gives few output tiles; the pointwise kernels sum the partials in chunk order.
@@ -67,10 +68,16 @@ class ScrnCell : public Cell {
     off_DZS = c.take(TB * Yw * e);
     off_DSP = c.take(TB * Sp * 4);
     off_part = c.take((size_t)nchunk * Hp * 4);
+    off_flags = c.take(4096);
     scratch_bytes = c.o;
   }
 
   char* HSrow(int t) { return saved + off_HS + (size_t)t * B * Yw * esz(); }
+  // K2 fusion choices (AV fuse_fwd): 0 chain GEMM + pointwise per step, 1 the persistent fused
+  // h-chain (scrn_persist.cu) when B ≤ 128
+  int fwd_fusions() const override {
+    return (ot == OT::BF16 && scrn_fwd_persist_supported(B, Hp, chain_ksplit())) ? 2 : 1;
+  }
   void* x_operand() override { return sv<char>(off_X); }
   Mat2 y_operand() override { return mat(HSrow(1), Yw, (long)T * B, Yw); }
   int y_width() const override { return Yw; }
@@ -142,6 +149,20 @@ class ScrnCell : public Cell {
     rec.ksplit = chain_ksplit();
     EpiStore ez = epi(Z, Hp, B, Hp);
     ez.split_stride = (long)B * Hp;
+    if (var.fwd_mode == 1 && ot == OT::BF16 && scrn_fwd_persist_supported(B, Hp, rec.ksplit)) {
+      ScrnPersistArgs pa{};
+      pa.B = B; pa.H = H; pa.Hp = Hp; pa.T = T; pa.t0 = 0; pa.t1 = T; pa.nsplit = rec.ksplit;
+      pa.Q = XAB; pa.ldq = Yw; pa.bh = p("b_h"); pa.Hf = Hf;
+      pa.HS = (__nv_bfloat16*)HSrow(0); pa.ldhs = Yw;
+      pa.y = y ? (__nv_bfloat16*)y : nullptr; pa.ldy = ldy; pa.hT = hT;
+      pa.flags = sc<unsigned>(off_flags);
+      CUDA_TRY(cudaMemsetAsync(pa.flags, 0, 4096, st));
+      scrn_fwd_persist_launch(HSrow(0), Yw, MR, Tmax, pa, st);
+      for (int t = 0; t < T; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
+      mark(R_FWD, 1, st);
+      fwd_done = true;
+      return;
+    }
     for (int t = 0; t < T; ++t) {
       run_gemm(2, rec, ez, t, 0, var.g[G_REC], st);
       scrn_fwd_pw(ot, B, H, Hp, XAB + (long)t * B * Yw, Yw, Z, rec.ksplit, (long)B * Hp, p("b_h"),
