@@ -1,8 +1,5 @@
 // Pointwise cell kernels (unfused halves of K2/K4), K5 fixed-order reductions, K6 embedding,
 // K7 cross-entropy, K9 SGD and operand mirrors.
-#include <cub/device/device_radix_sort.cuh>
-#include <cub/device/device_scan.cuh>
-
 #include "cell_math.cuh"
 #include "lstm_bwd_row.cuh"
 #include "kernels.h"
@@ -964,62 +961,121 @@ void colsum(const float* in, long rows, int cols, long ld, float* scratch, float
   LAUNCH_CHECK();
 }
 
-// ---- embedding backward: stable radix sort of (token, row) then ordered segment sums
-__global__ void iota_kernel(int32_t* v, long n) {
-  const long i = (long)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i < n) v[i] = (int32_t)i;
-}
-
-static int key_bits(int V) {
-  int b = 1;
-  while ((1L << b) < V) ++b;
-  return b;
-}
-
-// Segmented, deterministic embedding backward.  After a stable radix sort of (token, row), the
-// rows of token v occupy the sorted range [lo_v, hi_v) in ascending row order.  That range is cut
-// into segments of EMB_SEG rows (so a hot Zipf token does not serialise onto one CTA); segment
-// partial sums are taken in row order and the segments of a token are then added in order.
+// ---- embedding backward: stable counting sort of (token, row) then ordered segment sums
+// Segmented, deterministic embedding backward.  A stable counting sort of (token, row) — hand-written:
+// per-block token histograms, one scan CTA, and a one-warp-per-block stable scatter — puts the rows
+// of token v in the sorted range [lo_v, lo_v + n_v) in ascending row order.  That range is cut into
+// segments of EMB_SEG rows (so a hot Zipf token does not serialise onto one CTA); segment partial
+// sums are taken in row order and the segments of a token are then added in order.
 constexpr int EMB_SEG = 64;
+constexpr int EMB_BLK = 1024;   // rows per counting block
 
-static size_t scan_temp_bytes(int V) {
-  size_t t = 0;
-  cub::DeviceScan::ExclusiveSum(nullptr, t, (const int32_t*)nullptr, (int32_t*)nullptr, V + 1);
-  return round_up(t, 256);
-}
+static long emb_blocks(long n) { return (n + EMB_BLK - 1) / EMB_BLK; }
 
 size_t embed_bwd_scratch_bytes(long n, int V) {
-  size_t temp = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
-                                  (int32_t*)nullptr, (int)n, 0, key_bits(V));
-  const size_t max_seg = (size_t)(n / EMB_SEG + V + 1);
-  return round_up(temp, 256) + 3 * round_up(n * 4, 256) + scan_temp_bytes(V) + 3 * round_up((V + 1) * 4L, 256) +
-         round_up(max_seg * 4, 256);  // + partials (allocated by the caller separately)
+  const size_t nb = round_up(n * 4, 256), vb = round_up((V + 1) * 4L, 256);
+  const size_t cb = round_up((size_t)emb_blocks(n) * V * 4, 256);
+  return cb + 2 * nb + 3 * vb;
 }
 
-__device__ __forceinline__ long lower_bound_i32(const int32_t* a, long n, int key) {
-  long lo = 0, hi = n;
-  while (lo < hi) {
-    const long mid = (lo + hi) / 2;
-    if (a[mid] < key) lo = mid + 1; else hi = mid;
+// cnt[b][v] = rows of block b with token v (integer atomics: the counts do not depend on the order)
+__global__ void emb_count_kernel(const int32_t* __restrict__ tok, long n, int V, int32_t* __restrict__ cnt) {
+  const long b = blockIdx.x;
+  const long r0 = b * EMB_BLK, r1 = min(n, r0 + EMB_BLK);
+  for (long i = r0 + threadIdx.x; i < r1; i += blockDim.x) {
+    const int v = tok[i];
+    if (v >= 0 && v < V) atomicAdd(&cnt[b * V + v], 1);
   }
-  return lo;
 }
 
-__global__ void emb_seg_count_kernel(const int32_t* __restrict__ skeys, long n, int V, int32_t* __restrict__ lo,
-                                     int32_t* __restrict__ nseg) {
-  const int v = blockIdx.x * blockDim.x + threadIdx.x;
-  if (v > V) return;
-  if (v == V) { nseg[V] = 0; return; }
-  const long l = lower_bound_i32(skeys, n, v), h = lower_bound_i32(skeys, n, v + 1);
-  lo[v] = (int32_t)l;
-  nseg[v] = (int32_t)((h - l + EMB_SEG - 1) / EMB_SEG);
+// One CTA: total_v = Σ_b cnt[b][v]; cnt[b][v] ← lo_v + Σ_{b' < b} cnt[b'][v] (the first sorted
+// position of block b's rows of token v); lo = exclusive scan of total; segoff = exclusive scan of
+// the per-token segment counts ⌈total_v / EMB_SEG⌉ (segoff[V] = number of segments).
+__global__ void __launch_bounds__(1024) emb_scan_kernel(int32_t* __restrict__ cnt, long nblk, int V,
+                                                        int32_t* __restrict__ lo, int32_t* __restrict__ segoff) {
+  __shared__ int32_t wsum[2][32];
+  const int tid = threadIdx.x, nt = blockDim.x;
+  const int per = (V + nt - 1) / nt, v0 = tid * per, v1 = min(V, v0 + per);
+  int tsum = 0, ssum = 0;   // this thread's range: rows and segments
+  for (int v = v0; v < v1; ++v) {
+    int tot = 0;
+    for (long b = 0; b < nblk; ++b) tot += cnt[b * V + v];
+    tsum += tot;
+    ssum += (tot + EMB_SEG - 1) / EMB_SEG;
+  }
+  // exclusive scan of (tsum, ssum) over threads in thread order
+  const int lane = tid % 32, w = tid / 32;
+  int it = tsum, is = ssum;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const int a = __shfl_up_sync(0xffffffffu, it, d), c = __shfl_up_sync(0xffffffffu, is, d);
+    if (lane >= d) { it += a; is += c; }
+  }
+  if (lane == 31) { wsum[0][w] = it; wsum[1][w] = is; }
+  __syncthreads();
+  if (w == 0) {
+    int a = lane < nt / 32 ? wsum[0][lane] : 0, c = lane < nt / 32 ? wsum[1][lane] : 0;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int x = __shfl_up_sync(0xffffffffu, a, d), y = __shfl_up_sync(0xffffffffu, c, d);
+      if (lane >= d) { a += x; c += y; }
+    }
+    wsum[0][lane] = a;
+    wsum[1][lane] = c;
+  }
+  __syncthreads();
+  int rbase = (it - tsum) + (w > 0 ? wsum[0][w - 1] : 0);
+  int sbase = (is - ssum) + (w > 0 ? wsum[1][w - 1] : 0);
+  for (int v = v0; v < v1; ++v) {
+    lo[v] = rbase;
+    segoff[v] = sbase;
+    int run = rbase, tot = 0;
+    for (long b = 0; b < nblk; ++b) {
+      const int c = cnt[b * V + v];
+      cnt[b * V + v] = run;
+      run += c;
+      tot += c;
+    }
+    rbase += tot;
+    sbase += (tot + EMB_SEG - 1) / EMB_SEG;
+  }
+  if (tid == nt - 1) { lo[V] = rbase; segoff[V] = sbase; }
+}
+
+// Stable scatter: one warp per block walks its rows 32 at a time in ascending order; lanes with the
+// same token rank themselves by lane (match.any), the lowest of them advances the token's cursor.
+__global__ void __launch_bounds__(32) emb_scatter_kernel(const int32_t* __restrict__ tok, long n, int V,
+                                                         int32_t* __restrict__ cnt, int32_t* __restrict__ skeys,
+                                                         int32_t* __restrict__ srows) {
+  const long b = blockIdx.x;
+  const int lane = threadIdx.x;
+  const long r0 = b * EMB_BLK, r1 = min(n, r0 + EMB_BLK);
+  int32_t* cur = cnt + b * V;   // this block's cursors (first positions, from emb_scan_kernel)
+  for (long base = r0; base < r1; base += 32) {
+    const long i = base + lane;
+    const bool ok = i < r1;
+    const int v = ok ? tok[i] : -1 - lane;   // unique dummy keys for the tail lanes
+    const bool valid = ok && v >= 0 && v < V;
+    const unsigned peers = __match_any_sync(0xffffffffu, v);
+    const int rank = __popc(peers & ((1u << lane) - 1u));
+    const int leader = __ffs(peers) - 1;
+    int pos = 0;
+    if (valid && lane == leader) pos = cur[v];
+    pos = __shfl_sync(0xffffffffu, pos, leader) + rank;
+    __syncwarp();
+    if (valid) {
+      skeys[pos] = v;
+      srows[pos] = (int32_t)i;
+      if (lane == leader) cur[v] = pos - rank + __popc(peers);
+    }
+    __syncwarp();
+  }
 }
 
 // partial[s][c] = Σ rows of segment s (ascending); the owning token is found from segoff.
-__global__ void emb_seg_partial_kernel(const int32_t* __restrict__ skeys, const int32_t* __restrict__ srows, long n,
-                                       int V, const int32_t* __restrict__ lo, const int32_t* __restrict__ segoff,
-                                       const float* __restrict__ dX, long ldx, int I, float* __restrict__ part) {
+__global__ void emb_seg_partial_kernel(const int32_t* __restrict__ srows, int V, const int32_t* __restrict__ lo,
+                                       const int32_t* __restrict__ segoff, const float* __restrict__ dX, long ldx,
+                                       int I, float* __restrict__ part) {
   const int s = blockIdx.y;
   const int total = segoff[V];
   if (s >= total) return;
@@ -1031,7 +1087,7 @@ __global__ void emb_seg_partial_kernel(const int32_t* __restrict__ skeys, const 
   }
   const int v = a;
   const long l = lo[v];
-  const long h = lower_bound_i32(skeys, n, v + 1);
+  const long h = lo[v + 1];
   const long r0 = l + (long)(s - segoff[v]) * EMB_SEG;
   const long r1 = min(h, r0 + EMB_SEG);
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -1054,34 +1110,25 @@ size_t embed_bwd_partial_floats(long n, int V, int I) { return (size_t)(n / EMB_
 
 void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int I, float* dE, void* scratch,
                size_t scratch_bytes, float* part, cudaStream_t st) {
-  size_t temp = 0;
-  cub::DeviceRadixSort::SortPairs(nullptr, temp, (const int32_t*)nullptr, (int32_t*)nullptr, (const int32_t*)nullptr,
-                                  (int32_t*)nullptr, (int)n, 0, key_bits(V));
-  temp = round_up(temp, 256);
+  const long nblk = emb_blocks(n);
+  const size_t nb = round_up(n * 4, 256), vb = round_up((V + 1) * 4L, 256);
+  const size_t cb = round_up((size_t)nblk * V * 4, 256);
+  ASTRA_CHECK_ARG(scratch_bytes >= cb + 2 * nb + 3 * vb, "embed_bwd: scratch too small");
   char* base = (char*)scratch;
-  const size_t nb = round_up(n * 4, 256);
-  const size_t vb = round_up((V + 1) * 4L, 256);
-  const size_t stb = scan_temp_bytes(V);
-  ASTRA_CHECK_ARG(scratch_bytes >= temp + 3 * nb + stb + 3 * vb, "embed_bwd: scratch too small");
-  int32_t* rows_in = (int32_t*)(base + temp);
-  int32_t* skeys = (int32_t*)(base + temp + nb);
-  int32_t* srows = (int32_t*)(base + temp + 2 * nb);
-  char* scan_tmp = base + temp + 3 * nb;
-  int32_t* lo = (int32_t*)(scan_tmp + stb);
-  int32_t* nseg = (int32_t*)(scan_tmp + stb + vb);
-  int32_t* segoff = (int32_t*)(scan_tmp + stb + 2 * vb);
-  iota_kernel<<<cdiv(n, 256), 256, 0, st>>>(rows_in, n);
+  int32_t* cnt = (int32_t*)base;
+  int32_t* skeys = (int32_t*)(base + cb);
+  int32_t* srows = (int32_t*)(base + cb + nb);
+  int32_t* lo = (int32_t*)(base + cb + 2 * nb);
+  int32_t* segoff = (int32_t*)(base + cb + 2 * nb + vb);
+  CUDA_TRY(cudaMemsetAsync(cnt, 0, (size_t)nblk * V * 4, st));
+  emb_count_kernel<<<(unsigned)nblk, 256, 0, st>>>(tok, n, V, cnt);
   LAUNCH_CHECK();
-  CUDA_TRY(cub::DeviceRadixSort::SortPairs(base, temp, tok, skeys, rows_in, srows, (int)n, 0, key_bits(V), st));
-  count_launch(4);
-  emb_seg_count_kernel<<<cdiv(V + 1, 256), 256, 0, st>>>(skeys, n, V, lo, nseg);
+  emb_scan_kernel<<<1, 1024, 0, st>>>(cnt, nblk, V, lo, segoff);
   LAUNCH_CHECK();
-  size_t stb2 = stb;
-  CUDA_TRY(cub::DeviceScan::ExclusiveSum(scan_tmp, stb2, nseg, segoff, V + 1, st));
-  count_launch(1);
+  emb_scatter_kernel<<<(unsigned)nblk, 32, 0, st>>>(tok, n, V, cnt, skeys, srows);
+  LAUNCH_CHECK();
   const long max_seg = n / EMB_SEG + V;
-  emb_seg_partial_kernel<<<dim3(cdiv(I, 256), (unsigned)max_seg), 256, 0, st>>>(skeys, srows, n, V, lo, segoff, dX,
-                                                                                 ldx, I, part);
+  emb_seg_partial_kernel<<<dim3(cdiv(I, 256), (unsigned)max_seg), 256, 0, st>>>(srows, V, lo, segoff, dX, ldx, I, part);
   LAUNCH_CHECK();
   emb_seg_final_kernel<<<dim3(cdiv(I, 256), V), 256, 0, st>>>(V, segoff, part, I, dE);
   LAUNCH_CHECK();

@@ -366,3 +366,29 @@ def test_stream_schedules_lm_bitwise(variant):
     pa, la = _steps_params("fwd=0", graph=True)
     pb, lb = _steps_params(variant, graph=True)
     assert torch.equal(pa, pb) and la == lb
+
+
+@pytest.mark.parametrize("T,B,V,nsym", [(100, 512, 256, 205), (35, 64, 10000, None), (7, 33, 50, 3)])
+def test_embedding_backward_counting_sort(T, B, V, nsym):
+    """The embedding backward's hand-written stable counting sort + ordered segment sums (R5) against
+    the oracle's dE[v] = Σ_{(t,b): tok = v} dx[t,b] on the fp32 path (1e-4, element-wise): the cfg5
+    token statistics (hot Zipf symbols, segments of many 64-row pieces), a 10k vocabulary (mostly
+    empty rows, which must be exactly zero) and a 3-symbol batch."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    I, H = 64, 64
+    tok = synth.zipf_tokens(7, "tok", (T + 1, B), V, nsym)
+    shapes = cell_shapes("lstm", I, H)
+    shapes.update({"E": (V, I), "W_o": (H, V), "b_o": (V,)})
+    p = synth.weights(7, shapes, H)
+    c = A.Cell("lstm", H, I, B, T, dtype="fp32")
+    m = A.LM(c, V)
+    m.load(p)
+    tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+    m.fwd_bwd(tokens)
+    torch.cuda.synchronize()
+    dE = m.view("E", m.grads).cpu().numpy()
+    _, go, _ = OLM.lm_forward_backward("lstm", p, tok, np.zeros((B, H)), np.zeros((B, H)))
+    used = np.zeros(V, bool)
+    used[tok[:T].reshape(-1)] = True
+    assert np.all(dE[~used] == 0.0), "tokens absent from the batch must get exactly zero"
+    assert rel_err(dE[used], go["E"][used]) <= TOL_FP32
