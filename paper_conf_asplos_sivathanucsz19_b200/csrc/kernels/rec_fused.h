@@ -144,6 +144,25 @@ struct ScrnPersistArgs {
   unsigned* flags;          // one counter, zeroed before the launch
 };
 bool scrn_fwd_persist_supported(int B, int Hp, int nsplit);
+// SC-RNN persistent BPTT h-chain (ScrnCell bwd_mode 1): t = T−1 … 0 in one cooperative launch;
+// dh_rec = dz_{t+1}·Rᵀ with the R33 split as TMEM accumulators (R resident as a K-major copy),
+// dz_t = (dy^h + dh_rec)·h(1−h) fused, db_h partials in the row-lane order of scrn_bwd_pw_kernel.
+struct ScrnBpttArgs {
+  int B, H, Hp, T, nsplit;
+  int nk, kper, ka, a_rows, a_bytes;   // set by the launcher
+  uint32_t idesc;
+  const void* dy;           // h part of dy: fp32 [T·B][ldy] (LM) or bf16 [T·B][ldy] (external)
+  long ldy;
+  const float* dhT;         // optional [B][H]
+  const float* Hf;          // [(T+1)·B][Hp] fp32 h
+  __nv_bfloat16* DZ;        // [T·B][lddz] dz operand rows (dz part written)
+  long lddz;
+  float* part;              // [ceil(B/32)][Hp] db_h partials (written at the end)
+  unsigned* flags;          // one counter, zeroed before the launch
+};
+bool scrn_bwd_persist_supported(int B, int Hp, int nsplit, int T);
+void scrn_bwd_persist_launch(const void* DZ, long lddz, const void* Rk, int T, bool dy_f32, ScrnBpttArgs a,
+                             cudaStream_t st);
 void scrn_fwd_persist_launch(const void* HS, long ldhs, const void* MR, int Tmax, ScrnPersistArgs a, cudaStream_t st);
 
 bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);

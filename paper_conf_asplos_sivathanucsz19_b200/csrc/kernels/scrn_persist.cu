@@ -237,6 +237,286 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
   }
 }
 
+// ============================================================================ BPTT (bwd_mode 1)
+// The SC-RNN h-chain backward in one cooperative launch (SURVEY §8(a) row a5 for a non-LSTM cell):
+//   dh_rec_t = dz_{t+1}·Rᵀ (R33 split kept as TMEM accumulators, R resident as a K-major copy);
+//   dz_t = (dy^h_t + Σ partials)·h_t·(1 − h_t) (scrn_bwd_pw_kernel's expression and rounding);
+//   db_h partials: 32-row chunks, 8 row lanes each summing rows y, y+8, … in ascending order, lanes
+//   combined in y order, folded into the running partial step after step (its fixed order, R5).
+// dz_t (bf16) is the next step's A operand: written, fenced, released through one grid counter.
+constexpr int SPB_RB = 32, SPB_RY = 8;   // scrn_bwd_pw_kernel's PW_RB / PW_RY
+
+template <typename TDY>
+__global__ void __launch_bounds__(SP_THREADS, 1)
+    scrn_bwd_persist_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                            const ScrnBpttArgs a) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int nk = a.nk, ka = a.ka, SA = SP_SA;
+  const int stage_bytes = ka * a.a_bytes;
+  const int nch = (a.B + SPB_RB - 1) / SPB_RB;   // db_h row chunks
+  uint8_t* sA = smem;
+  uint8_t* sRes = sA + SA * stage_bytes;
+  float* sdz = reinterpret_cast<float*>(sRes + nk * SP_BT);    // [128 rows][16 units] this step's dz
+  float* slane = sdz + 128 * SP_UC;                            // [4 chunks][8 lanes][16 units]
+  float* spart = slane + 4 * SPB_RY * SP_UC;                   // [4 chunks][16 units] running partials
+  uint64_t* fullA = reinterpret_cast<uint64_t*>(spart + 4 * SP_UC);
+  uint64_t* emptyA = fullA + SA;
+  uint64_t* resbar = emptyA + SA;
+  uint64_t* tfull = resbar + 1;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int u0 = blockIdx.x * SP_UC;
+  const unsigned nct = gridDim.x;
+  const int ns = a.nsplit, kper = a.kper;
+  const int acc_cols = ns * SP_UC;
+  const int T = a.T;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < SA; ++s) {
+      sm100::mbar_init(&fullA[s], 1);
+      sm100::mbar_init(&emptyA[s], 1);
+    }
+    sm100::mbar_init(resbar, 1);
+    for (int q = 0; q < 2; ++q) {
+      sm100::mbar_init(&tfull[q], 1);
+      sm100::mbar_init(&tempty[q], 32 * SP_EPI_WARPS);
+    }
+    sm100::fence_barrier_init();
+  }
+  if (warp == 0 && lane == 0) {
+    sm100::tma_prefetch(&mapA);
+    sm100::tma_prefetch(&mapB);
+  }
+  if (warp == 1) sm100::tmem_alloc(tmem_slot, 128);
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ producer: R once, then dz_{t+1}
+    if (lane == 0) {
+      const uint64_t pol = sm100::l2_policy_evict_last();
+      pdl_wait();
+      sm100::mbar_arrive_expect_tx(resbar, (uint32_t)(nk * SP_BT));
+      for (int kb = 0; kb < nk; ++kb) sm100::tma_load_3d_hint(sRes + kb * SP_BT, &mapB, resbar, 0, u0, kb, pol);
+      int s = 0;
+      uint32_t ph = 0;
+      for (int t = T - 2; t >= 0; --t) {
+        // every CTA has published dz_{t+1} (step t+1 is the (T−2−t)-th release)
+        while (sp_ld_acquire(a.flags) < nct * (unsigned)(T - 1 - t)) __nanosleep(32);
+        sp_fence_proxy_async_global();
+        for (int kb = 0; kb < nk; kb += ka) {
+          sm100::mbar_wait(&emptyA[s], ph ^ 1);
+          sm100::mbar_arrive_expect_tx(&fullA[s], (uint32_t)stage_bytes);
+          sm100::tma_load_4d(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t + 1);
+          if (++s == SA) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      sm100::mbar_wait(resbar, 0);
+      sm100::tc_fence_after();
+      const uint32_t idesc = a.idesc;
+      const uint64_t dA0 = sm100::smem_desc_sw128(sm100::smem_u32(sA), 16, 1024);
+      const uint64_t dR0 = sm100::smem_desc_sw128(sm100::smem_u32(sRes), 16, 1024);
+      const uint32_t a_kb = (uint32_t)a.a_bytes >> 4, a_st = (uint32_t)stage_bytes >> 4, b_kb = SP_BT >> 4;
+      int sa = 0;
+      uint32_t pa = 0;
+      int local = 0;
+      for (int t = T - 2; t >= 0; --t, ++local) {
+        const int acc = local & 1;
+        sm100::mbar_wait(&tempty[acc], (uint32_t)((local >> 1) & 1) ^ 1);
+        sm100::tc_fence_after();
+        int ja = ka, jk = 0, q = 0;
+        uint64_t adesc = 0;
+        for (int kb = 0; kb < nk; ++kb) {
+          if (ja == ka) {
+            sm100::mbar_wait(&fullA[sa], pa);
+            sm100::tc_fence_after();
+            adesc = dA0 + (uint64_t)(sa * a_st);
+            ja = 0;
+          }
+          const uint32_t d_tmem = tmem_base + acc * acc_cols + q * SP_UC;
+          const uint64_t bd = dR0 + (uint64_t)(kb * b_kb);
+#pragma unroll
+          for (int kk = 0; kk < TC_BK / 16; ++kk)
+            sm100::umma_bf16(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
+          adesc += a_kb;
+          if (++ja == ka) {
+            sm100::umma_commit(&emptyA[sa]);
+            if (++sa == SA) { sa = 0; pa ^= 1; }
+          }
+          if (++jk == kper) { jk = 0; ++q; }
+        }
+        sm100::umma_commit(&tfull[acc]);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue (8 warps)
+    const int ew = warp - 2;
+    const int quarter = warp & 3;
+    const int half = ew >> 2;
+    const int row = quarter * 32 + lane;
+    const bool valid = row < a.B;
+    const int ul0 = half * 8, unit0 = u0 + ul0;
+    const int etid = ew * 32 + lane;   // 0..255
+    pdl_wait();
+    int local = 0;
+    for (int t = T - 1; t >= 0; --t) {
+      const long r = (long)t * a.B + row;
+      float gv[8], hv[8];   // dy^h_t and h_t: older than the chain, loaded before the MMAs finish
+      if (valid) {
+        const TDY* dp = reinterpret_cast<const TDY*>(a.dy) + r * a.ldy + unit0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) gv[i] = unit0 + i < a.H ? to_f<TDY>(dp[i]) : 0.f;
+        const float4* hp = reinterpret_cast<const float4*>(a.Hf + (r + a.B) * a.Hp + unit0);
+        const float4 h0 = hp[0], h1 = hp[1];
+        hv[0] = h0.x; hv[1] = h0.y; hv[2] = h0.z; hv[3] = h0.w;
+        hv[4] = h1.x; hv[5] = h1.y; hv[6] = h1.z; hv[7] = h1.w;
+      }
+      if (t < T - 1) {
+        const int acc = local & 1;
+        sm100::mbar_wait(&tfull[acc], (uint32_t)((local >> 1) & 1));
+        sm100::tc_fence_after();
+        const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * acc_cols + ul0;
+        float z[8];
+        uint32_t zr[8];
+        sm100::tmem_ld8_nowait(taddr, zr);
+        sm100::tmem_wait_ld();
+#pragma unroll
+        for (int i = 0; i < 8; ++i) z[i] = __uint_as_float(zr[i]);
+        for (int c = 1; c < ns; ++c) {   // partials summed in chunk order (sum_split)
+          sm100::tmem_ld8_nowait(taddr + c * SP_UC, zr);
+          sm100::tmem_wait_ld();
+#pragma unroll
+          for (int i = 0; i < 8; ++i) z[i] = __fadd_rn(z[i], __uint_as_float(zr[i]));
+        }
+        sm100::tc_fence_before();
+        sm100::mbar_arrive(&tempty[acc]);
+        ++local;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) gv[i] = __fadd_rn(gv[i], z[i]);
+      } else if (a.dhT && valid) {   // t = T − 1: the caller's dhT (one "partial")
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+          if (unit0 + i < a.H) gv[i] = __fadd_rn(gv[i], a.dhT[(long)row * a.H + unit0 + i]);
+      }
+      float dz[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        dz[i] = (valid && unit0 + i < a.H) ? __fmul_rn(__fmul_rn(gv[i], hv[i]), __fsub_rn(1.f, hv[i])) : 0.f;
+      if (valid) {
+        uint4 pk;
+        uint32_t* pw = reinterpret_cast<uint32_t*>(&pk);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          __nv_bfloat162 b2 = __floats2bfloat162_rn(dz[2 * i], dz[2 * i + 1]);
+          pw[i] = *reinterpret_cast<uint32_t*>(&b2);
+        }
+        *reinterpret_cast<uint4*>(a.DZ + r * a.lddz + unit0) = pk;   // the next step's operand
+      }
+      if (t > 0) {   // publish dz_t
+        sp_fence_proxy_async_global();
+        __threadfence();
+        sp_epi_bar();
+        if (ew == 0 && lane == 0) atomicAdd(a.flags, 1u);
+      }
+      // db_h column partials in scrn_bwd_pw_kernel's order
+#pragma unroll
+      for (int i = 0; i < 8; ++i) sdz[row * SP_UC + ul0 + i] = dz[i];
+      sp_epi_bar();
+      for (int it = etid; it < nch * SPB_RY * SP_UC; it += 32 * SP_EPI_WARPS) {
+        const int u = it % SP_UC, y = (it / SP_UC) % SPB_RY, c = it / (SP_UC * SPB_RY);
+        float sacc = 0.f;
+        for (int rr = y; rr < SPB_RB && c * SPB_RB + rr < a.B; rr += SPB_RY)
+          sacc = __fadd_rn(sacc, sdz[(c * SPB_RB + rr) * SP_UC + u]);
+        slane[(c * SPB_RY + y) * SP_UC + u] = sacc;
+      }
+      sp_epi_bar();
+      for (int it = etid; it < nch * SP_UC; it += 32 * SP_EPI_WARPS) {
+        const int u = it % SP_UC, c = it / SP_UC;
+        float v = 0.f;
+#pragma unroll
+        for (int y = 0; y < SPB_RY; ++y) v = __fadd_rn(v, slane[(c * SPB_RY + y) * SP_UC + u]);
+        spart[c * SP_UC + u] = t == T - 1 ? v : __fadd_rn(spart[c * SP_UC + u], v);
+      }
+      sp_epi_bar();
+    }
+    for (int it = etid; it < nch * SP_UC; it += 32 * SP_EPI_WARPS) {
+      const int u = it % SP_UC, c = it / SP_UC;
+      if (u0 + u < a.Hp) a.part[(long)c * a.Hp + u0 + u] = spart[c * SP_UC + u];
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    sm100::tc_fence_after();
+    sm100::tmem_dealloc(tmem_base, 128);
+  }
+}
+
+bool scrn_bwd_persist_supported(int B, int Hp, int nsplit, int T) {
+  return T >= 2 && scrn_fwd_persist_supported(B, Hp, nsplit);
+}
+
+void scrn_bwd_persist_launch(const void* DZ, long lddz, const void* Rk, int T, bool dy_f32, ScrnBpttArgs a,
+                             cudaStream_t st) {
+  ASTRA_CHECK_ARG(scrn_bwd_persist_supported(a.B, a.Hp, a.nsplit, T), "persistent SCRN BPTT: unsupported shape");
+  a.T = T;
+  a.nk = a.Hp / TC_BK;
+  a.kper = (a.nk + a.nsplit - 1) / a.nsplit;
+  a.a_rows = a.B <= 64 ? 64 : 128;
+  a.a_bytes = a.a_rows * TC_BK * 2;
+  a.ka = 1;
+  for (int c = SP_KA; c > 1; --c)
+    if (a.nk % c == 0) { a.ka = c; break; }
+  a.idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(SP_UC >> 3) << 17) | ((uint32_t)(TC_BM >> 4) << 24);
+  CUtensorMap mA, mB;
+  {   // dz part of the [dz | (1−α)ds] rows: {64 k, rows B, k-block (stride 128 B), t}
+    const long dims[4] = {64, a.B, a.nk, T};
+    const long str[3] = {lddz * 2, 128, (long)a.B * lddz * 2};
+    const int box[4] = {64, a.a_rows, a.ka, 1};
+    make_map_nd(&mA, DZ, 4, dims, str, box, 128);
+  }
+  {   // R (not transposed) rows k: {64 j, row k, k-block (stride 128 B)}
+    const long dims[3] = {64, a.Hp, a.nk};
+    const long str[2] = {(long)a.Hp * 2, 128};
+    const int box[3] = {64, SP_UC, 1};
+    make_map_nd(&mB, Rk, 3, dims, str, box, 128);
+  }
+  const int bars = (2 * SP_SA + 1 + 4) * 8 + 16;
+  const int smem = 1024 + SP_SA * a.ka * a.a_bytes + a.nk * SP_BT + (128 * SP_UC + 4 * SPB_RY * SP_UC + 4 * SP_UC) * 4 + bars;
+  int dev = 0, maxs = 0;
+  CUDA_TRY(cudaGetDevice(&dev));
+  CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+  ASTRA_CHECK_ARG(smem <= maxs, "persistent SCRN BPTT: the R slice does not fit in shared memory");
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(a.Hp / SP_UC);
+  cfg.blockDim = dim3(SP_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  if (dy_f32) {
+    auto k = scrn_bwd_persist_kernel<float>;
+    CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, k, mA, mB, a));
+  } else {
+    auto k = scrn_bwd_persist_kernel<__nv_bfloat16>;
+    CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    CUDA_TRY(cudaLaunchKernelEx(&cfg, k, mA, mB, a));
+  }
+  LAUNCH_CHECK();
+}
+
 bool scrn_fwd_persist_supported(int B, int Hp, int nsplit) {
   return B >= 1 && B <= 128 && Hp % SP_UC == 0 && Hp / SP_UC <= num_sms() && nsplit >= 1 && nsplit <= 4 &&
          2 * nsplit * SP_UC <= 128;

@@ -26,7 +26,7 @@ class ScrnCell : public Cell {
   int S, Sp, Yw, nchunk;
   float alpha;
   size_t off_X, off_XAB, off_Sf, off_HS, off_Hf, off_MAB, off_MP, off_MR;
-  size_t off_Z, off_dH, off_DZS, off_DSP, off_part, off_flags;
+  size_t off_Z, off_dH, off_DZS, off_DSP, off_part, off_flags, off_Rk;
 
   // Reading R33: both chain GEMMs (h·R and dz·Rᵀ, K = Hp, N = Hp) split over K into s fixed chunks
   // when the batch gives few output tiles; the pointwise kernels sum the partials in chunk order.
@@ -69,6 +69,7 @@ class ScrnCell : public Cell {
     off_DSP = c.take(TB * Sp * 4);
     off_part = c.take((size_t)nchunk * Hp * 4);
     off_flags = c.take(4096);
+    off_Rk = c.take((size_t)Hp * Hp * e);   // R (not transposed) bf16, K-major B of the persistent BPTT
     scratch_bytes = c.o;
   }
 
@@ -77,6 +78,11 @@ class ScrnCell : public Cell {
   // h-chain (scrn_persist.cu) when B ≤ 128
   int fwd_fusions() const override {
     return (ot == OT::BF16 && scrn_fwd_persist_supported(B, Hp, chain_ksplit())) ? 2 : 1;
+  }
+  // K4 fusion choices (AV fuse_bwd): 0 BPTT GEMM + pointwise per step, 1 the persistent fused h-chain
+  // backward (scrn_persist.cu)
+  int bwd_fusions() const override {
+    return (ot == OT::BF16 && scrn_bwd_persist_supported(B, Hp, chain_ksplit(), T)) ? 2 : 1;
   }
   void* x_operand() override { return sv<char>(off_X); }
   Mat2 y_operand() override { return mat(HSrow(1), Yw, (long)T * B, Yw); }
@@ -201,7 +207,20 @@ class ScrnCell : public Cell {
     bp.b_keep = true;
     GemmSpec bp0 = bp;   // dh0 (once, no split)
     bp.ksplit = chain_ksplit();
-    for (int t = T - 1; t >= 0; --t) {
+    const bool fused = var.bwd_mode == 1 && ot == OT::BF16 && scrn_bwd_persist_supported(B, Hp, bp.ksplit, T);
+    if (fused) {   // K4 fused persistent: every step of the h-chain in one launch
+      char* Rk = sc<char>(off_Rk);
+      CUDA_TRY(cudaMemsetAsync(Rk, 0, (size_t)Hp * Hp * e, st));
+      copy_pad(ot, p("R"), OT::F32, H, H, H, Rk, Hp, st);   // rows k, columns j (padding exactly zero)
+      ScrnBpttArgs ba{};
+      ba.B = B; ba.H = H; ba.Hp = Hp; ba.nsplit = bp.ksplit;
+      ba.dy = lm_mode ? (const void*)lm_dy : dy; ba.ldy = ldy;
+      ba.dhT = dhT; ba.Hf = Hf; ba.DZ = (__nv_bfloat16*)DZS; ba.lddz = Yw; ba.part = part;
+      ba.flags = sc<unsigned>(off_flags);
+      CUDA_TRY(cudaMemsetAsync(ba.flags, 0, 4096, st));
+      scrn_bwd_persist_launch(DZS, Yw, Rk, T, lm_mode, ba, st);
+    }
+    for (int t = T - 1; t >= 0 && !fused; --t) {
       const float* dh = dhT;
       long ld_dh = H;
       int nsplit = 1;

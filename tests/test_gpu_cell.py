@@ -236,14 +236,16 @@ def test_scrn_ragged_multi_tile(dtype, tol):
 
 @pytest.mark.parametrize("T,B,I,H,S", [(6, 64, 1024, 1024, 1024), (5, 33, 72, 200, 70), (3, 100, 64, 128, 40)])
 def test_scrn_persistent_forward_bitwise(T, B, I, H, S):
-    """SC-RNN's fused persistent h-chain (fwd=1: one cooperative launch, R slices resident, the R33
-    split kept as TMEM accumulators, σ(Q + Σ partials + b_h) in the epilogue) gives the same bits as
-    GEMM + pointwise per step (fwd=0) for every output and gradient — cfg2's shapes (H = S = 1024,
-    4-way split), a ragged batch with padding units, a 128-row A box — and matches the oracle."""
+    """SC-RNN's fused persistent h-chains — forward (fwd=1: one cooperative launch, R slices resident,
+    the R33 split kept as TMEM accumulators, σ(Q + Σ partials + b_h) in the epilogue) and BPTT (bwd=1:
+    dz·Rᵀ split likewise, dz = (dy + Σ partials)·h(1−h) and the db_h row-lane partials fused) — give
+    the same bits as GEMM + pointwise per step for every output and gradient — cfg2's shapes
+    (H = S = 1024, 4-way split), a ragged batch with padding units, a 128-row A box — and match the
+    oracle."""
     p, inp, dY, dhT, dcT = make_cell_case("scrn", T, B, I, H, 101, bf16=True, S=S)
     kw = {"context": S, "scrn_alpha": ALPHA}
     ref = None
-    for v in ("fwd=0", "fwd=1"):
+    for v in ("fwd=0", "fwd=1", "bwd=1", "fwd=1,bwd=1"):
         out, g, _ = run_gpu_cell("scrn", p, inp, dY, dhT, dcT, "bf16", v, **kw)
         cur = {**out, **g}
         if ref is None:
@@ -252,7 +254,7 @@ def test_scrn_persistent_forward_bitwise(T, B, I, H, S):
         for k in ref:
             assert np.array_equal(ref[k], cur[k]), (v, k)
     if T * B * H <= 5 * 33 * 200:
-        _check("scrn", T, B, I, H, "bf16", 101, TOL_BF16, variant="fwd=1", S=S)
+        _check("scrn", T, B, I, H, "bf16", 101, TOL_BF16, variant="fwd=1,bwd=1", S=S)
 
 
 def test_scrn_cfg2_reduced():
