@@ -123,20 +123,23 @@ __global__ void __launch_bounds__(BF_THREADS, 1)
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer: one accumulator per split-K chunk
     pdl_wait();
-    if (lane == 0) {
+    if (lane == 0) {   // lean issue loop: counters and descriptors advanced by (bytes >> 4)
+      const uint32_t sa0 = sm100::smem_u32(smem);
+      const uint64_t dA0 = sm100::smem_desc_sw128(sa0, 16, 1024);
+      const uint64_t dB0 = sm100::smem_desc_sw128(sa0 + TC_BM * TC_BK * 2, 8192, 1024);
+      const uint32_t idesc = a.idesc, kper = (uint32_t)a.kper;
+      int s = 0, c = 0;
+      uint32_t ph = 0, jk = 0;
       for (int kb = 0; kb < a.nk; ++kb) {
-        const int s = kb % stages;
-        const int c = kb / a.kper;
-        sm100::mbar_wait(&full[s], (uint32_t)((kb / stages) & 1));
+        sm100::mbar_wait(&full[s], ph);
         sm100::tc_fence_after();
-        const uint32_t sa = sm100::smem_u32(smem + s * BF_STAGE);
-        const uint32_t sb = sa + TC_BM * TC_BK * 2;
+        const uint64_t ad = dA0 + (uint64_t)(s * (BF_STAGE >> 4)), bd = dB0 + (uint64_t)(s * (BF_STAGE >> 4));
 #pragma unroll
         for (int kk = 0; kk < TC_BK / 16; ++kk)
-          sm100::umma_bf16(tmem_base + c * BF_BN, sm100::smem_desc_sw128(sa + kk * 32, 16, 1024),
-                           sm100::smem_desc_sw128(sb + kk * 2048, 8192, 1024), a.idesc,
-                           (kb != c * a.kper || kk != 0) ? 1u : 0u);
+          sm100::umma_bf16(tmem_base + c * BF_BN, ad + 2 * kk, bd + 128 * kk, idesc, (jk | kk) != 0);
         sm100::umma_commit(&empty[s]);
+        if (++s == stages) { s = 0; ph ^= 1; }
+        if (++jk == kper) { jk = 0; ++c; }
       }
       sm100::umma_commit(tfull);
     }

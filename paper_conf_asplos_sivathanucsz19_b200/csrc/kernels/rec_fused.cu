@@ -132,25 +132,28 @@ __global__ void __launch_bounds__(RF_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
-    if (lane == 0) {
-      long it = 0;
+    if (lane == 0) {   // lean issue loop: counters and descriptors advanced by (bytes >> 4)
+      const uint32_t sa0 = sm100::smem_u32(smem);
+      const uint64_t dA0 = sm100::smem_desc_sw128(sa0, 16, 1024);
+      const uint64_t dB0 = sm100::smem_desc_sw128(sa0 + S::A_BYTES, 16, 1024);
+      const uint32_t idesc = a.idesc;
+      int s = 0;
+      uint32_t ph = 0;
       int local = 0;
       for (int t = a.t0; t < a.t1; ++t, ++local) {
         const int acc = local & 1;
         sm100::mbar_wait(&tempty[acc], (uint32_t)((local >> 1) & 1) ^ 1);
         sm100::tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
-        for (int kb = 0; kb < nk; ++kb, ++it) {
-          const int s = (int)(it % stages);
-          sm100::mbar_wait(&full[s], (uint32_t)((it / stages) & 1));
+        for (int kb = 0; kb < nk; ++kb) {
+          sm100::mbar_wait(&full[s], ph);
           sm100::tc_fence_after();
-          const uint32_t sa = sm100::smem_u32(smem + s * S::STAGE_BYTES);
-          const uint32_t sb = sa + S::A_BYTES;
+          const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, sm100::smem_desc_sw128(sa + kk * 32, 16, 1024),
-                             sm100::smem_desc_sw128(sb + kk * 32, 16, 1024), a.idesc, (kb | kk) != 0);
+            sm100::umma_bf16(d_tmem, ad + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
           sm100::umma_commit(&empty[s]);
+          if (++s == stages) { s = 0; ph ^= 1; }
         }
         sm100::umma_commit(&tfull[acc]);
       }

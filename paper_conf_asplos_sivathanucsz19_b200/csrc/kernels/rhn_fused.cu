@@ -28,8 +28,9 @@ namespace astra {
 
 namespace {
 
-constexpr int RH_EPI_WARPS = 4;
-constexpr int RH_THREADS = 64 + 32 * RH_EPI_WARPS;   // warp 0 TMA, warp 1 MMA, 4 epilogue warps
+constexpr int RH_EPI_WARPS = 8;
+constexpr int RH_THREADS = 64 + 32 * RH_EPI_WARPS;   // warp 0 TMA, warp 1 MMA, 8 epilogue warps (two per
+                                                      // TMEM lane quarter, one per 16-unit half of the tile)
 constexpr int RH_UB = 32;                             // hidden units per tile
 constexpr int RH_BN = 2 * RH_UB;                      // MMA N: the units' H-columns then their T-columns
 constexpr int RH_SP = RH_UB + 1;                      // row strides of the per-thread (row) shared buffers,
@@ -171,46 +172,44 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
+    // Lean issue loop (round 2, cf. rec_persist.cu): stage bookkeeping by counters and shared-memory
+    // descriptors advanced by adding (bytes >> 4) — the per-k-block scalar work (long divisions,
+    // descriptor rebuilds) otherwise paced the k loop, not the operands' arrival.
     if (lane == 0) {
-      long it = 0;
+      const uint64_t dA0 = sm100::smem_desc_sw128(sm100::smem_u32(smem), 16, 1024);
+      const uint64_t dB0 = sm100::smem_desc_sw128(sm100::smem_u32(smem) + a_bytes, 16, 1024);
+      const uint32_t st_step = (uint32_t)stage_bytes >> 4;
+      const uint32_t idesc = a.idesc;
+      int s = 0;
+      uint32_t ph = 0;
       for (int q = 0; q < nsteps; ++q) {
         mbar_wait_idle(tempty, (uint32_t)(q & 1) ^ 1);
         sm100::tc_fence_after();
-        // Chunk-interleaved issue order (independent accumulators; within a chunk the k order is the
-        // canonical accumulation, R33) is kept as an option for a future A path that lands faster.
-        // (measured: interleaving the chunks slowed the k loop, 5.25 → 6.25 µs at cfg3 — the loop
-        // waits on A arriving, not on accumulator dependencies — so chunks are issued in order)
-        const bool inter = false;
-        const int nr = inter ? a.nsplit * kper : nk;   // (chunk, k) pairs; the last chunk may be shorter
-        for (int r = 0; r < nr; ++r) {
-          const int kb = inter ? (r % a.nsplit) * kper + r / a.nsplit : r;
-          if (kb >= nk) continue;
-          const long i2 = it + kb;
-          const int s = (int)(i2 % stages);
-          const int c = kb / kper;                         // canonical split-K chunk (R33)
-          const uint32_t d_tmem = tmem_base + c * RH_BN;
-          sm100::mbar_wait(&full[s], (uint32_t)((i2 / stages) & 1));
+        int c = 0, jk = 0;   // canonical split-K chunk (R33) and k-block within it
+        for (int kb = 0; kb < nk; ++kb) {
+          sm100::mbar_wait(&full[s], ph);
           sm100::tc_fence_after();
-          if (a.trace && r == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 1] = global_ns();
-          if (a.trace && r == nr - 1) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 2] = global_ns();
+          if (a.trace && kb == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 1] = global_ns();
+          if (a.trace && kb == nk - 1) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 2] = global_ns();
           // a_rows = 64: the M = 128 MMA's rows 64..127 read the B tile's bytes — garbage rows of
           // TMEM that the epilogue never reads (rows ≥ B)
-          const uint32_t sa = sm100::smem_u32(smem + s * stage_bytes);
-          const uint32_t sb = sa + a_bytes;
+          const uint64_t ad = dA0 + (uint64_t)(s * st_step), bd = dB0 + (uint64_t)(s * st_step);
+          const uint32_t d_tmem = tmem_base + c * RH_BN;
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, sm100::smem_desc_sw128(sa + kk * 32, 16, 1024),
-                             sm100::smem_desc_sw128(sb + kk * 32, 16, 1024), a.idesc,
-                             (kb != c * kper || kk != 0) ? 1u : 0u);
+            sm100::umma_bf16(d_tmem, ad + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
           sm100::umma_commit(&empty[s]);
+          if (++s == stages) { s = 0; ph ^= 1; }
+          if (++jk == kper) { jk = 0; ++c; }
         }
-        it += nk;
         sm100::umma_commit(tfull);
       }
     }
   } else {
-    // ------------------------------------------------------------ highway epilogue (4 warps)
+    // ------------------------------------------------------------ highway epilogue (8 warps)
     const int quarter = warp & 3;            // TMEM lane quarter of this warp
+    const int uc = (warp - 2) / 4;           // the 16-unit half of the tile this warp applies (round 2:
+                                             // the two halves ran one after the other in 4 warps)
     const int row = quarter * 32 + lane;
     const int m = m0 + row;
     const bool valid = m < a.B;
@@ -228,8 +227,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       const float* wx = a.WX + ((size_t)t * a.B + m) * G2;
       float* spr = sprev + row * RH_SP;   // valid rows only (m < B ≤ a_rows when a_rows = 64)
       float* zr = zst + row * RH_ZP;
-#pragma unroll 1
-      for (int uc = 0; uc < RH_UB / 16; ++uc) {
+      {
         const int ul = uc * 16;
         float xh[16], xt[16];
         if (l == 0 && valid) {   // x_t·W (ℓ = 1 only): independent of the MMA, issued first
@@ -255,7 +253,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           }
         }
         if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + (uc == 0 ? 5 : 11)] = global_ns();
-        if (!valid) continue;
+        if (valid) {
         __nv_bfloat16* so = a.Sop + slot_out + (size_t)m * a.Hp + u0 + ul;
         // every shared-memory operand into registers first, results out after: the buffers share
         // one base, so interleaved loads and stores would serialise the 16 units' dependency chains
@@ -311,6 +309,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         reinterpret_cast<uint4*>(so)[0] = pk[0];
         reinterpret_cast<uint4*>(so)[1] = pk[1];
         if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 10] = global_ns();
+        }
       }
       sm100::tc_fence_before();
       sm100::mbar_arrive(tempty);
@@ -329,7 +328,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       if (valid) {
         float* sn = a.Sf + slot_out + (size_t)m * a.Hp + u0;
 #pragma unroll
-        for (int q4 = 0; q4 < RH_UB / 4; ++q4) {
+        for (int q4 = 4 * uc; q4 < 4 * uc + 4; ++q4) {   // this warp's 16 units
           const int o = 4 * q4;
           reinterpret_cast<float4*>(sn)[q4] = make_float4(spr[o], spr[o + 1], spr[o + 2], spr[o + 3]);
           reinterpret_cast<float4*>(Z + u0)[q4] = make_float4(zr[o], zr[o + 1], zr[o + 2], zr[o + 3]);

@@ -1,0 +1,9 @@
+#!/bin/bash
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests/test_gpu_cell.py tests/test_gpu_lm.py -q -x -k "fused or bwd or pair or persistent" > gpurun_out/r2_t10.log 2>&1
+echo "rc=$?" >> gpurun_out/r2_t10.log
+timeout 300 python scratch/trace_rhn.py > gpurun_out/r2_trace_rhn.log 2>&1
+V512="a1=256.1.1.2,rec=256.1.1.2,bptt=256.1.1.2,du=256.1.1.2,dw=256.1.1.2,dx=256.1.1.2,head=256.1.1,wg_side=1,fwd=0,bwd=0,pf=0,hov=0"
+for v in "fwd=0,bwd=0" "fwd=1,bwd=0" "fwd=2,bwd=0" "fwd=0,bwd=1"; do
+  ASTRA_VARIANT="$V512,$v" timeout 300 python bench.py --profile --steps 5 >> gpurun_out/r2_prof10.log 2>&1
+done
