@@ -49,9 +49,9 @@ def peaks():
 
 def a1_traffic():
     """DRAM bytes (read + write) per launch of the a1 GEMM from the committed ncu --set full capture
-    (profiles/r1_roofline_traffic.json, written by profiles/ncu_metrics.py from the .ncu-rep)."""
+    (profiles/r2_roofline_traffic.json: the round-2 ncu --set full capture of the tuned variant's a1)."""
     try:
-        with open(os.path.join(ROOT, "profiles", "r1_roofline_traffic.json")) as f:
+        with open(os.path.join(ROOT, "profiles", "r2_roofline_traffic.json")) as f:
             return json.load(f)["a1_dram_bytes_per_launch"]
     except Exception:
         return None

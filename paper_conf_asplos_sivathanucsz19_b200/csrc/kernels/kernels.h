@@ -49,6 +49,7 @@ void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, l
 // form (AV "bwd_pw", bitwise interchangeable): 0 the row-lane kernel (thread = unit, rows walked 4
 // lanes x 8), 1 the wide kernel (thread = row x 4 units, all rows of a 32-row chunk in flight).
 int lstm_bwd_row_chunks(int B);
+constexpr int BWD_ROW_CHUNK = 32;   // rows per column-partial chunk of the backward pointwise kernels (R5)
 // grads_q[e] = Σ_chunk partials[chunk][q][gcol(e)] for q < nq (external e < 4H).
 void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,
                           cudaStream_t st);

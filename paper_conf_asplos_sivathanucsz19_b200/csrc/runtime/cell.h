@@ -56,6 +56,9 @@ struct Variant {
   int head_ov = 0;      // LM head overlapped with the forward chain in HEAD_CHUNKS[head_ov] time chunks (B3)
   int l2pf = 0;         // chain GEMMs prefetch the next pointwise kernel's saved tensors into L2 (R31): bit 0 fwd, bit 1 BPTT
   int dpb = 0;          // K11p bucket cap (§8(a.9) dp_bucket): 0 whole tensors, 1/2/3 = 128/32/8 MB pieces
+  int rsp = 0;          // row_streams (B3 stream assignment): 1 = the batch's two row halves run as two
+                        // independent chains on two streams (the sequences are independent), so one half's
+                        // pointwise kernel overlaps the other half's recurrent GEMM (LSTM family, B ≥ 256)
   int bpw = 0;          // bwd_pw (§8(a.9) bwd_kernel / bwd_epilogue): backward pointwise form, 0 row-lane (unit per
                         // thread, 8 rows walked), 1 wide (row x 4 units per thread, whole 32-row chunk in flight)
   int wgs = 0;          // wgrad_schedule (§8(a.9)): the input dgrad dX in WGS_CHUNKS[wgs] time chunks,
@@ -205,6 +208,7 @@ class Cell {
   virtual int gate_chunkings() const { return 1; }   // options of the tuner AV "gate_chunking" (1: none)
   virtual int wgrad_schedules() const { return 1; }  // options of the tuner AV "wgrad_schedule" (1: none)
   virtual int bwd_pw_forms() const { return 1; }     // options of the tuner AV "bwd_pw" (1: none)
+  virtual int row_stream_options() const { return 1; }   // options of the tuner AV "row_streams" (1: none)
   virtual void role_shape(int role, int& M, int& N) const = 0;
 
   // forward-step hook (set by the LM): called after forward step t is enqueued on the main stream,

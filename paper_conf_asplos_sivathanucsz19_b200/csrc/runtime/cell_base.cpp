@@ -29,6 +29,7 @@ std::string Variant::str() const {
   if (gchunk) o << ",gc=" << gchunk;
   if (wgs) o << ",wgs=" << wgs;
   if (bpw) o << ",bpw=" << bpw;
+  if (rsp) o << ",rsp=" << rsp;
   return o.str();
 }
 
@@ -52,6 +53,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "dpb") {
       v.dpb = std::stoi(val);
       ASTRA_CHECK_ARG(v.dpb >= 0 && v.dpb <= 3, "variant: dpb must be 0..3 (whole tensors, 128, 32 or 8 MB buckets)");
+      continue;
+    }
+    if (k == "rsp") {
+      v.rsp = std::stoi(val);
+      ASTRA_CHECK_ARG(v.rsp == 0 || v.rsp == 1, "variant: rsp (row_streams) must be 0 or 1");
       continue;
     }
     if (k == "bpw") {
@@ -413,6 +419,10 @@ void Cell::tuner_setup() {
   // the backward pointwise kernel's form (bwd_kernel AV), against the BPTT-chain time
   if (ot == OT::BF16 && bwd_pw_forms() > 1)
     t = "(pre " + t + " (leaf bwd_pw " + std::to_string(bwd_pw_forms()) + " t_bptt))";
+  // B3 stream assignment of the chains themselves: the batch's row halves as two independent chains
+  // on two streams, against the whole step (both chains and everything they overlap with)
+  if (ot == OT::BF16 && !side.empty() && row_stream_options() > 1)
+    t = "(pre " + t + " (leaf row_streams " + std::to_string(row_stream_options()) + " t_step))";
   // reading R31: L2 prefetch by the chain GEMMs, per chain, after the kernel and fusion choices
   if (ot == OT::BF16 && chain_prefetch())
     t = "(pre " + t + " (par (leaf pf_fwd 2 t_fwd) (leaf pf_bwd 2 t_bptt)))";
@@ -464,6 +474,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "gate_chunking") { v.gchunk = o; continue; }
     if (n == "wgrad_schedule") { v.wgs = o; continue; }
     if (n == "bwd_pw") { v.bpw = o; continue; }
+    if (n == "row_streams") { v.rsp = o; continue; }
     if (n == "pf_fwd") { v.l2pf = (v.l2pf & ~1) | o; continue; }
     if (n == "pf_bwd") { v.l2pf = (v.l2pf & ~2) | (o << 1); continue; }
     for (int r = 0; r < G_ROLES; ++r)

@@ -66,6 +66,8 @@ class LstmCell : public Cell {
   ~LstmCell() override {
     for (cudaEvent_t e : ev_wgs)
       if (e) cudaEventDestroy(e);
+    for (cudaEvent_t e : ev_rs)
+      if (e) cudaEventDestroy(e);
     for (int i = 0; i < 2; ++i) {
       if (ev_rc_done[i]) cudaEventDestroy(ev_rc_done[i]);
       if (ev_rc_free[i]) cudaEventDestroy(ev_rc_free[i]);
@@ -83,6 +85,23 @@ class LstmCell : public Cell {
   int gate_chunkings() const override { return ot == OT::BF16 ? (side.empty() ? 3 : 5) : 1; }
   int wgrad_schedules() const override { return (ot == OT::BF16 && T >= 4) ? 3 : 1; }
   int bwd_pw_forms() const override { return ot == OT::BF16 ? 2 : 1; }
+  int row_stream_options() const override { return (ot == OT::BF16 && B >= 256 && B % 64 == 0) ? 2 : 1; }
+  cudaEvent_t ev_rs[2] = {nullptr, nullptr};   // row_streams fork / join
+  // the two row halves of the chains as independent chains on (main, side[0]): value-preserving —
+  // row chunks of the same GEMMs (R1), the same per-row pointwise arithmetic, 32-row partial chunks
+  bool row_split_ok(bool hooks) const {
+    return var.rsp == 1 && ot == OT::BF16 && B >= 256 && B % 64 == 0 && !side.empty() && !var.recomp && !hooks;
+  }
+  void rs_fork(cudaStream_t st) {
+    for (int i = 0; i < 2; ++i)
+      if (!ev_rs[i]) CUDA_TRY(cudaEventCreateWithFlags(&ev_rs[i], cudaEventDisableTiming));
+    CUDA_TRY(cudaEventRecord(ev_rs[0], st));
+    CUDA_TRY(cudaStreamWaitEvent(side[0], ev_rs[0], 0));
+  }
+  void rs_join(cudaStream_t st) {
+    CUDA_TRY(cudaEventRecord(ev_rs[1], side[0]));
+    CUDA_TRY(cudaStreamWaitEvent(st, ev_rs[1], 0));
+  }
   cudaEvent_t ev_wgs[11] = {};          // wgrad_schedule: chunk k's D_wx rows complete (+ join)
   int fwd_fusions() const override { return (ot == OT::BF16 && lstm_fwd_persist_supported(B, Hp)) ? 4 : 3; }
   bool chain_prefetch() const override { return true; }
@@ -258,6 +277,32 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
         fwd_step_done(t, st);
       }
     }
+  } else if (row_split_ok((bool)fwd_hook)) {
+    // row_streams: rows [0, B/2) on the main stream, [B/2, B) on side[0], each an independent chain
+    const int Bh = B / 2;
+    rs_fork(st);
+    for (int t = t0; t < t1; ++t) {
+      const bool last = t == T - 1;
+      for (int hh = 0; hh < 2; ++hh) {
+        const cudaStream_t S = hh ? side[0] : st;
+        const long r0 = (long)hh * Bh;
+        GemmSpec rh = rec;
+        rh.A = mat((const char*)Hrow(0) + (size_t)r0 * Hp * e, Hp, Bh, Hp, T + 1, (long)B * Hp);
+        rh.M = Bh;
+        float* UHt = UH + (long)t * B * NG + r0 * NG;
+        run_gemm(1, rh, epi(UHt, NG, Bh, NG), t, 0, var.g[G_REC], S);
+        const long rr = (long)t * B + r0;
+        if (y_f32)
+          lstm_fwd_pointwise(kind, ot, Bh, H, Hp, WX + rr * NG, UHt, gp, Cb + rr * Hp, Cb + (rr + B) * Hp,
+                             (char*)Hrow(t + 1) + (size_t)r0 * Hp * e, Hp, y_f32 + (size_t)rr * Hp, Hp, OT::F32,
+                             last && hT ? hT + r0 * H : nullptr, last && cT ? cT + r0 * H : nullptr, S);
+        else
+          lstm_fwd_pointwise(kind, ot, Bh, H, Hp, WX + rr * NG, UHt, gp, Cb + rr * Hp, Cb + (rr + B) * Hp,
+                             (char*)Hrow(t + 1) + (size_t)r0 * Hp * e, Hp, y ? (char*)y + (size_t)rr * H * e : nullptr,
+                             H, ot, last && hT ? hT + r0 * H : nullptr, last && cT ? cT + r0 * H : nullptr, S);
+      }
+    }
+    rs_join(st);
   } else {
     for (int t = t0; t < t1; ++t) {
       // recompute variant: UH_t is consumed by this step's pointwise kernel only (one L2-resident slot)
@@ -427,7 +472,46 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     for (int i = 0; i < wgs_n + 1; ++i)
       if (!ev_wgs[i]) CUDA_TRY(cudaEventCreateWithFlags(&ev_wgs[i], cudaEventDisableTiming));
   }
-  for (int t = t1 - 1; t >= t0; --t) {
+  const bool rsplit = row_split_ok(bwd_hook != nullptr) && !fuse && whole && wgs_n == 1;
+  if (rsplit) {   // row_streams: the two row halves' BPTT chains on (main, side[0])
+    const int Bh = B / 2;
+    rs_fork(st);
+    for (int t = T - 1; t >= 0; --t) {
+      for (int hh = 0; hh < 2; ++hh) {
+        const cudaStream_t S = hh ? side[0] : st;
+        const long r0 = (long)hh * Bh;
+        const long rr = (long)t * B + r0;
+        const void* dyt;
+        long ldy;
+        bool dyf32;
+        if (lm_dy) { dyt = lm_dy + rr * Hp; ldy = Hp; dyf32 = true; }
+        else { dyt = (const char*)dy + (size_t)rr * H * e; ldy = H; dyf32 = false; }
+        const float* dh_rec;
+        long ld_dh;
+        int nsplit = 1;
+        if (t == T - 1) {
+          dh_rec = dhT ? dhT + r0 * H : nullptr;
+          ld_dh = H;
+        } else {
+          GemmSpec bh = bp;
+          bh.A = mat(Duh + (size_t)r0 * NG * e, NG, Bh, NG, T, (long)B * NG);
+          bh.M = Bh;
+          EpiStore eh = epi(dH + r0 * Hp, Hp, Bh, Hp);
+          eh.split_stride = (long)B * Hp;
+          run_gemm(2, bh, eh, t + 1, 0, var.g[G_BPTT], S);
+          dh_rec = dH + r0 * Hp;
+          ld_dh = Hp;
+          nsplit = bp.ksplit;
+        }
+        lstm_bwd_pointwise(kind, ot, Bh, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC + r0 * Hp,
+                           WX + rr * NG, UH + rr * NG, Cb + (rr + B) * Hp, Cb + rr * Hp, gp,
+                           Duh + (size_t)rr * NG * e, Dwx + (size_t)rr * NG * e,
+                           part + (size_t)(r0 / BWD_ROW_CHUNK) * nq * NG, nq, t == T - 1, S, var.bpw);
+      }
+    }
+    rs_join(st);
+  }
+  for (int t = rsplit ? t0 - 1 : t1 - 1; t >= t0; --t) {
     const int kc = t / RC;
     if (rc && !fuse && rs != st && t == chunk_hi(kc) - 1) CUDA_TRY(cudaStreamWaitEvent(st, ev_rc_done[kc & 1], 0));
     if (fuse && t < T - 1) {

@@ -136,6 +136,29 @@ def test_bwd_pointwise_forms_bitwise(cell, dtype, T, B, H):
         _check(cell, T, B, 64, H, dtype, 99, TOL_BF16 if dtype == "bf16" else TOL_FP32)
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm"])
+@pytest.mark.parametrize("T,B,H", [(4, 256, 192), (5, 320, 130)])
+@pytest.mark.parametrize("v", ["rsp=1", "rsp=1,bpw=1,wg_side=1"])
+def test_row_streams_bitwise(cell, T, B, H, v):
+    """row_streams (stream assignment): the batch's two row halves as independent chains on two
+    streams (forward and BPTT) give the same bits as the one chain — outputs, every gradient, the
+    fixed-order column sums — and the AV is in the live tree."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, 64, H, 103, bf16=True)
+    ref = None
+    for var in ("rsp=0", v):
+        out, g, c = run_gpu_cell(cell, p, inp, dY, dhT, dcT, "bf16", var)
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (var, k)
+    c.tune_mode(A.TUNE_ON)
+    c.tune_next()
+    assert "row_streams" in c.tune_report()["tree_avs"]
+
+
 @pytest.mark.parametrize("v", ["wgs=1", "wgs=2", "wgs=2,wg_side=1,rc=1", "wgs=1,hov=0,fwd=3"])
 def test_wgrad_schedule_bitwise(v):
     """wgrad_schedule (§8(a.9)): the input dgrad in 4 / 10 time chunks on a side stream

@@ -358,7 +358,8 @@ def test_tune_next_never_blocks():
     assert rep["configs_explored"] >= 10 and rep["converged"]
 
 
-@pytest.mark.parametrize("variant", ["hov=1,wgs=2,gc=3,wg_side=1", "wgs=1,gc=4,fwd=3", "gc=2,wgs=2,rc=1"])
+@pytest.mark.parametrize("variant", ["hov=1,wgs=2,gc=3,wg_side=1", "wgs=1,gc=4,fwd=3", "gc=2,wgs=2,rc=1",
+                                     "rsp=1,bpw=1,gc=3"])
 def test_stream_schedules_lm_bitwise(variant):
     """The stream-assignment variants together — head overlap, wgrad_schedule's dX chunks during
     BPTT, gate_chunking's projection GEMMs on two streams, the small-batch persistent forward —
