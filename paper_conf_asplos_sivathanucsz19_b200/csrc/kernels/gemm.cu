@@ -152,11 +152,15 @@ static int smem_for(int& stages, int cap) {
 
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
                      int cm, int cn, bool b_keep, int ksplit, int cg, int smem_cap) {
+  // BN = 224 (74 CTA pairs fill all 148 SMs on an 8192-column chain GEMM instead of 64 pairs of 256)
+  // exists only for CTA pairs with a K-major B (each CTA holds 112 B rows); elsewhere the same tile
+  // width is run as 256 — same bits (R1: every output element is one accumulation over K)
+  if (BN == 224 && (cg != 2 || b_mn)) BN = 256;
   ASTRA_CHECK_ARG(cg == 1 || (cg == 2 && cm == 1 && cn == 1 && BN >= 128),
                   "tc_gemm: CTA pairs (cg = 2) need BN >= 128 and no extra cluster multicast");
   ASTRA_CHECK_ARG((cm == 1 || cm == 2 || cm == 4) && (cn == 1 || cn == 2 || cn == 4) && cm * cn <= 8,
                   "tc_gemm: cluster shape must be cm, cn in {1,2,4}, cm*cn <= 8");
-  ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256, "tc_gemm: BN must be 64, 128 or 256");
+  ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256 || BN == 224, "tc_gemm: BN must be 64, 128, 224 or 256");
   ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
   if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
   if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm / cg);
@@ -182,6 +186,7 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   int stages = 0;
   switch (BN / cg) {
     case 64: g.smem = smem_for<64>(stages, smem_cap); break;
+    case 112: g.smem = smem_for<112>(stages, smem_cap); break;
     case 128: g.smem = smem_for<128>(stages, smem_cap); break;
     default: g.smem = smem_for<256>(stages, smem_cap); break;
   }
@@ -247,6 +252,7 @@ void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaSt
   ASTRA_CHECK_STATE(g.ready, "tc_gemm: not prepared");
   if (g.args.cg == 2) {
     if (g.BN == 128) launch_pair<128>(g, epi, az, bz, st, max_ctas, pf);
+    else if (g.BN == 224) launch_pair<224>(g, epi, az, bz, st, max_ctas, pf);
     else launch_pair<256>(g, epi, az, bz, st, max_ctas, pf);
     return;
   }

@@ -502,7 +502,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                     const __grid_constant__ CUtensorMap mapC, const TcArgs args, const Epi epi) {
   constexpr int BH = BN / 2;          // B columns held by each CTA
   using S = TcSmem<BH>;
-  constexpr int TMEM_COLS = 2 * BN;   // two accumulator buffers of BN columns
+  constexpr int TMEM_COLS = 2 * BN <= 256 ? 256 : 512;   // two accumulator buffers of BN columns (power of 2)
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   const int stages = args.stages;

@@ -114,9 +114,9 @@ Variant Variant::parse(const std::string& s) {
     if (n < 2) c.cm = 1;
     ASTRA_CHECK_ARG(c.cg == 1 || (c.cg == 2 && c.cm == 1 && c.cn == 1 && c.bn >= 128),
                     "variant: CTA pair (4th field 2) needs tile width 128/256 and a 1x1 multicast cluster");
-    ASTRA_CHECK_ARG((c.bn == 64 || c.bn == 128 || c.bn == 256) && (c.cm == 1 || c.cm == 2 || c.cm == 4) &&
-                        (c.cn == 1 || c.cn == 2 || c.cn == 4) && c.cm * c.cn <= 8,
-                    "variant: tile width must be 64/128/256 and cluster cm, cn in {1,2,4} with cm*cn <= 8");
+    ASTRA_CHECK_ARG((c.bn == 64 || c.bn == 128 || c.bn == 256 || (c.bn == 224 && c.cg == 2)) &&
+                        (c.cm == 1 || c.cm == 2 || c.cm == 4) && (c.cn == 1 || c.cn == 2 || c.cn == 4) && c.cm * c.cn <= 8,
+                    "variant: tile width must be 64/128/256 (224: CTA pairs only) and cluster cm, cn in {1,2,4} with cm*cn <= 8");
     v.g[r] = c;
   }
   return v;
@@ -335,7 +335,7 @@ void Cell::ensure_comm_stream() {
 // ------------------------------------------------------------------------ tuner glue
 // The enumerator's static pruning (A19): per GEMM role, the kernel choices whose tile
 // and cluster shape fit the problem; the default (Variant()) first.
-static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 1, 1, 2}, {128, 1, 1, 2},
+static const KCfg CANDIDATES[] = {{256, 1, 1}, {128, 1, 1}, {64, 1, 1}, {256, 1, 1, 2}, {128, 1, 1, 2}, {224, 1, 1, 2},
                                   {256, 2, 1}, {256, 4, 1}, {256, 2, 2}, {256, 1, 2}, {128, 2, 1}, {128, 4, 1},
                                   {128, 2, 2}, {128, 1, 2}, {64, 2, 1}, {64, 4, 1}, {64, 2, 2}};
 

@@ -118,7 +118,7 @@ def test_cta_pair_bitwise(a_mn, b_mn, M, N, K):
     torch.cuda.synchronize()
     err = (base.double().cpu() - ref).abs().max().item()
     assert err <= 1e-5 * ref.abs().max().item() * max(1, K / 64) + 1e-6
-    for bn in (128, 256):
+    for bn in (128, 224, 256):   # 224: 112 B rows per CTA (K-major B; MN-major B runs it as 256)
         out = A.gemm_bf16_ex(A_s, B_s, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn, cta_group=2)
         torch.cuda.synchronize()
         assert torch.equal(out[0].cpu(), base.cpu()), bn
