@@ -102,7 +102,57 @@ __global__ void mirror_T_kernel(const float* __restrict__ src, int K, int N, int
   }
 }
 
+// 64×64 tiles, float4 loads (N % 4 == 0), 4 consecutive k per thread on the store side
+template <typename T>
+__global__ void __launch_bounds__(256) mirror_T4_kernel(const float* __restrict__ src, int K, int N, int Np, int Kp,
+                                                        T* __restrict__ dst, long ldd) {
+  __shared__ float tile[64][65];
+  const int n0 = blockIdx.x * 64, k0 = blockIdx.y * 64, tid = threadIdx.x;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int kl = tid / 16 + 16 * j, q = tid % 16, k = k0 + kl, n = n0 + 4 * q;
+    float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (k < K && n < N) x = *reinterpret_cast<const float4*>(src + (long)k * N + n);
+    tile[kl][4 * q] = x.x;
+    tile[kl][4 * q + 1] = x.y;
+    tile[kl][4 * q + 2] = x.z;
+    tile[kl][4 * q + 3] = x.w;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const int nl = tid / 16 + 16 * j, q = tid % 16, n = n0 + nl, k = k0 + 4 * q;
+    if (n >= Np || k >= Kp) continue;
+    T* d = dst + (long)n * ldd + k;
+    if (k + 4 <= Kp) {
+      if constexpr (sizeof(T) == 2) {
+        __nv_bfloat162 lo = __floats2bfloat162_rn(tile[4 * q][nl], tile[4 * q + 1][nl]);
+        __nv_bfloat162 hi = __floats2bfloat162_rn(tile[4 * q + 2][nl], tile[4 * q + 3][nl]);
+        uint2 u;
+        u.x = *reinterpret_cast<uint32_t*>(&lo);
+        u.y = *reinterpret_cast<uint32_t*>(&hi);
+        *reinterpret_cast<uint2*>(d) = u;
+      } else {
+        *reinterpret_cast<float4*>(d) =
+            make_float4(tile[4 * q][nl], tile[4 * q + 1][nl], tile[4 * q + 2][nl], tile[4 * q + 3][nl]);
+      }
+    } else {
+      for (int i = 0; k + i < Kp; ++i) d[i] = from_f<T>(tile[4 * q + i][nl]);
+    }
+  }
+}
+
 void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, long ldd, cudaStream_t st) {
+  const size_t e = ot == OT::BF16 ? 2 : 4;
+  if (N % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)src & 15) == 0 && ((uintptr_t)dst & (4 * e - 1)) == 0) {
+    dim3 grid(cdiv(Np, 64), cdiv(Kp, 64));
+    if (ot == OT::BF16)
+      mirror_T4_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(src, K, N, Np, Kp, (__nv_bfloat16*)dst, ldd);
+    else
+      mirror_T4_kernel<float><<<grid, 256, 0, st>>>(src, K, N, Np, Kp, (float*)dst, ldd);
+    LAUNCH_CHECK();
+    return;
+  }
   dim3 grid(cdiv(Np, 32), cdiv(Kp, 32)), block(32, 8);
   if (ot == OT::BF16)
     mirror_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, N, Np, Kp, (__nv_bfloat16*)dst, ldd);
@@ -880,8 +930,111 @@ __global__ void ce_kernel(const float* __restrict__ logits, long ldl, int V, con
   for (int c = V + lane; c < ldd; c += 32) dlog[r * ldd + c] = from_f<T>(0.f);
 }
 
+// One 256-thread CTA per row, float4 loads/stores (V % 4 == 0): thread t takes the quads t, t+256,
+// … in ascending order, then a warp xor tree and the 8 warp sums in warp order — a fixed order for
+// every row, so the row's bits do not depend on how the rows are chunked or launched.
+constexpr int CE_T = 256;
+template <typename T> __device__ __forceinline__ void ce_store4(T* p, float a, float b, float c, float d);
+template <> __device__ __forceinline__ void ce_store4<float>(float* p, float a, float b, float c, float d) {
+  *reinterpret_cast<float4*>(p) = make_float4(a, b, c, d);
+}
+template <> __device__ __forceinline__ void ce_store4<__nv_bfloat16>(__nv_bfloat16* p, float a, float b, float c,
+                                                                      float d) {
+  __nv_bfloat162 lo = __floats2bfloat162_rn(a, b), hi = __floats2bfloat162_rn(c, d);
+  uint2 u;
+  u.x = *reinterpret_cast<uint32_t*>(&lo);
+  u.y = *reinterpret_cast<uint32_t*>(&hi);
+  *reinterpret_cast<uint2*>(p) = u;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(CE_T) ce_row_kernel(const float* __restrict__ logits, long ldl, int V,
+                                                      const int32_t* __restrict__ targets, long n, float inv_n,
+                                                      const int* __restrict__ nvp, long row0,
+                                                      float* __restrict__ rowloss, T* __restrict__ dlog, long ldd,
+                                                      float* __restrict__ dlog32) {
+  __shared__ float red[CE_T / 32];
+  const long r = blockIdx.x;
+  const int tid = threadIdx.x, lane = tid % 32, w = tid / 32;
+  const int V4 = V / 4;
+  T* drow = dlog + r * ldd;
+  float* d32 = dlog32 + r * V;
+  if (nvp) {   // rows ≥ *nvp are padding (bucketed steps): no loss, zero gradient; mean over *nvp rows
+    const long nv = *nvp;
+    inv_n = __fdiv_rn(1.f, (float)nv);
+    if (row0 + r >= nv) {
+      if (tid == 0) rowloss[r] = 0.f;
+      for (int q = tid; q < V4; q += CE_T) {
+        ce_store4<T>(drow + 4 * q, 0.f, 0.f, 0.f, 0.f);
+        ce_store4<float>(d32 + 4 * q, 0.f, 0.f, 0.f, 0.f);
+      }
+      for (int c = V + tid; c < ldd; c += CE_T) drow[c] = from_f<T>(0.f);
+      return;
+    }
+  }
+  const float4* row = reinterpret_cast<const float4*>(logits + r * ldl);
+  float m = -INFINITY;
+  for (int q = tid; q < V4; q += CE_T) {
+    const float4 x = row[q];
+    m = fmaxf(fmaxf(m, fmaxf(x.x, x.y)), fmaxf(x.z, x.w));
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+  if (lane == 0) red[w] = m;
+  __syncthreads();
+  m = red[0];
+#pragma unroll
+  for (int k = 1; k < CE_T / 32; ++k) m = fmaxf(m, red[k]);
+  __syncthreads();
+  float s = 0.f;
+  for (int q = tid; q < V4; q += CE_T) {
+    const float4 x = row[q];
+    s = __fadd_rn(s, expf(__fsub_rn(x.x, m)));
+    s = __fadd_rn(s, expf(__fsub_rn(x.y, m)));
+    s = __fadd_rn(s, expf(__fsub_rn(x.z, m)));
+    s = __fadd_rn(s, expf(__fsub_rn(x.w, m)));
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+  if (lane == 0) red[w] = s;
+  __syncthreads();
+  s = red[0];
+#pragma unroll
+  for (int k = 1; k < CE_T / 32; ++k) s = __fadd_rn(s, red[k]);
+  const float lse = __fadd_rn(m, logf(s));
+  const int tgt = targets[r];
+  if (tid == 0) rowloss[r] = __fsub_rn(lse, logits[r * ldl + tgt]);
+  const float rs = __frcp_rn(s);
+  for (int q = tid; q < V4; q += CE_T) {
+    const float4 x = row[q];
+    float p[4] = {__fmul_rn(expf(__fsub_rn(x.x, m)), rs), __fmul_rn(expf(__fsub_rn(x.y, m)), rs),
+                  __fmul_rn(expf(__fsub_rn(x.z, m)), rs), __fmul_rn(expf(__fsub_rn(x.w, m)), rs)};
+    if ((tgt >> 2) == q) p[tgt & 3] = __fsub_rn(p[tgt & 3], 1.f);
+#pragma unroll
+    for (int k = 0; k < 4; ++k) p[k] = __fmul_rn(p[k], inv_n);
+    ce_store4<T>(drow + 4 * q, p[0], p[1], p[2], p[3]);
+    ce_store4<float>(d32 + 4 * q, p[0], p[1], p[2], p[3]);
+  }
+  for (int c = V + tid; c < ldd; c += CE_T) drow[c] = from_f<T>(0.f);
+}
+
 void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,
                 float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp, long row0) {
+  if (n == 0) return;
+  const size_t e = ot == OT::BF16 ? 2 : 4;
+  const bool vec = V % 4 == 0 && ldl % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)logits & 15) == 0 &&
+                   ((uintptr_t)dlog & (4 * e - 1)) == 0 && ((uintptr_t)dlog32 & 15) == 0;
+  if (vec) {
+    ASTRA_CHECK_ARG(n < (1L << 31), "ce_fwd_bwd: too many rows");
+    if (ot == OT::BF16)
+      ce_row_kernel<__nv_bfloat16><<<(unsigned)n, CE_T, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, row0, rowloss,
+                                                                 (__nv_bfloat16*)dlog, ldd, dlog32);
+    else
+      ce_row_kernel<float><<<(unsigned)n, CE_T, 0, st>>>(logits, ldl, V, targets, n, inv_n, nvp, row0, rowloss,
+                                                         (float*)dlog, ldd, dlog32);
+    LAUNCH_CHECK();
+    return;
+  }
   const int rows_per = 8;
   dim3 grid(cdiv(n, rows_per));
   if (ot == OT::BF16)
@@ -963,14 +1116,20 @@ void colsum(const float* in, long rows, int cols, long ld, float* scratch, float
 
 // ---- embedding backward: stable counting sort of (token, row) then ordered segment sums
 // Segmented, deterministic embedding backward.  A stable counting sort of (token, row) — hand-written:
-// per-block token histograms, one scan CTA, and a one-warp-per-block stable scatter — puts the rows
+// per-block token histograms, a parallel scan, and a one-warp-per-block stable scatter — puts the rows
 // of token v in the sorted range [lo_v, lo_v + n_v) in ascending row order.  That range is cut into
 // segments of EMB_SEG rows (so a hot Zipf token does not serialise onto one CTA); segment partial
-// sums are taken in row order and the segments of a token are then added in order.
+// sums are taken in row order and the segments of a token are then added in order.  (The block
+// size only changes how the sort is computed, never the sorted order: the bits do not depend on it.)
 constexpr int EMB_SEG = 64;
-constexpr int EMB_BLK = 1024;   // rows per counting block
 
-static long emb_blocks(long n) { return (n + EMB_BLK - 1) / EMB_BLK; }
+// rows per counting block: ~2 blocks per SM, at least 128 rows, a multiple of 32
+static long emb_blk(long n) {
+  long b = (n + 295) / 296;
+  b = (b + 31) / 32 * 32;
+  return b < 128 ? 128 : b;
+}
+static long emb_blocks(long n) { return n > 0 ? (n + emb_blk(n) - 1) / emb_blk(n) : 0; }
 
 size_t embed_bwd_scratch_bytes(long n, int V) {
   const size_t nb = round_up(n * 4, 256), vb = round_up((V + 1) * 4L, 256);
@@ -979,78 +1138,118 @@ size_t embed_bwd_scratch_bytes(long n, int V) {
 }
 
 // cnt[b][v] = rows of block b with token v (integer atomics: the counts do not depend on the order)
-__global__ void emb_count_kernel(const int32_t* __restrict__ tok, long n, int V, int32_t* __restrict__ cnt) {
+__global__ void emb_count_kernel(const int32_t* __restrict__ tok, long n, long blk, int V, int32_t* __restrict__ cnt) {
   const long b = blockIdx.x;
-  const long r0 = b * EMB_BLK, r1 = min(n, r0 + EMB_BLK);
+  const long r0 = b * blk, r1 = min(n, r0 + blk);
   for (long i = r0 + threadIdx.x; i < r1; i += blockDim.x) {
     const int v = tok[i];
     if (v >= 0 && v < V) atomicAdd(&cnt[b * V + v], 1);
   }
 }
 
-// One CTA: total_v = Σ_b cnt[b][v]; cnt[b][v] ← lo_v + Σ_{b' < b} cnt[b'][v] (the first sorted
-// position of block b's rows of token v); lo = exclusive scan of total; segoff = exclusive scan of
-// the per-token segment counts ⌈total_v / EMB_SEG⌉ (segoff[V] = number of segments).
-__global__ void __launch_bounds__(1024) emb_scan_kernel(int32_t* __restrict__ cnt, long nblk, int V,
-                                                        int32_t* __restrict__ lo, int32_t* __restrict__ segoff) {
-  __shared__ int32_t wsum[2][32];
-  const int tid = threadIdx.x, nt = blockDim.x;
-  const int per = (V + nt - 1) / nt, v0 = tid * per, v1 = min(V, v0 + per);
-  int tsum = 0, ssum = 0;   // this thread's range: rows and segments
-  for (int v = v0; v < v1; ++v) {
-    int tot = 0;
-    for (long b = 0; b < nblk; ++b) tot += cnt[b * V + v];
-    tsum += tot;
-    ssum += (tot + EMB_SEG - 1) / EMB_SEG;
-  }
-  // exclusive scan of (tsum, ssum) over threads in thread order
-  const int lane = tid % 32, w = tid / 32;
-  int it = tsum, is = ssum;
+// tot[v] = Σ_b cnt[b][v]; nseg[v] = ⌈tot[v] / EMB_SEG⌉ (written to lo / segoff, scanned next)
+__global__ void emb_total_kernel(const int32_t* __restrict__ cnt, long nblk, int V, int32_t* __restrict__ lo,
+                                 int32_t* __restrict__ segoff) {
+  const int v = blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= V) return;
+  int tot = 0;
+  long b = 0;
+  for (; b + 8 <= nblk; b += 8) {
+    int c[8];
 #pragma unroll
-  for (int d = 1; d < 32; d <<= 1) {
-    const int a = __shfl_up_sync(0xffffffffu, it, d), c = __shfl_up_sync(0xffffffffu, is, d);
-    if (lane >= d) { it += a; is += c; }
+    for (int k = 0; k < 8; ++k) c[k] = cnt[(b + k) * V + v];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) tot += c[k];
   }
-  if (lane == 31) { wsum[0][w] = it; wsum[1][w] = is; }
+  for (; b < nblk; ++b) tot += cnt[b * V + v];
+  lo[v] = tot;
+  segoff[v] = (tot + EMB_SEG - 1) / EMB_SEG;
+}
+
+// One CTA: in-place exclusive scans of lo[0..V) and segoff[0..V), totals into lo[V] / segoff[V];
+// tiles of 4·1024 entries, 4 consecutive per thread, carried across tiles.
+__global__ void __launch_bounds__(1024) emb_scan_kernel(int V, int32_t* __restrict__ lo, int32_t* __restrict__ segoff) {
+  __shared__ int32_t wsum[2][32];
+  __shared__ int32_t carry[2];
+  const int tid = threadIdx.x, lane = tid % 32, w = tid / 32;
+  if (tid == 0) { carry[0] = 0; carry[1] = 0; }
   __syncthreads();
-  if (w == 0) {
-    int a = lane < nt / 32 ? wsum[0][lane] : 0, c = lane < nt / 32 ? wsum[1][lane] : 0;
+  for (int t0 = 0; t0 < V; t0 += 4 * 1024) {
+    int a[4], s[4], ta = 0, ts = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int v = t0 + tid * 4 + k;
+      a[k] = v < V ? lo[v] : 0;
+      s[k] = v < V ? segoff[v] : 0;
+      ta += a[k];
+      ts += s[k];
+    }
+    int it = ta, is = ts;
 #pragma unroll
     for (int d = 1; d < 32; d <<= 1) {
-      const int x = __shfl_up_sync(0xffffffffu, a, d), y = __shfl_up_sync(0xffffffffu, c, d);
-      if (lane >= d) { a += x; c += y; }
+      const int x = __shfl_up_sync(0xffffffffu, it, d), y = __shfl_up_sync(0xffffffffu, is, d);
+      if (lane >= d) { it += x; is += y; }
     }
-    wsum[0][lane] = a;
-    wsum[1][lane] = c;
-  }
-  __syncthreads();
-  int rbase = (it - tsum) + (w > 0 ? wsum[0][w - 1] : 0);
-  int sbase = (is - ssum) + (w > 0 ? wsum[1][w - 1] : 0);
-  for (int v = v0; v < v1; ++v) {
-    lo[v] = rbase;
-    segoff[v] = sbase;
-    int run = rbase, tot = 0;
-    for (long b = 0; b < nblk; ++b) {
-      const int c = cnt[b * V + v];
-      cnt[b * V + v] = run;
-      run += c;
-      tot += c;
+    if (lane == 31) { wsum[0][w] = it; wsum[1][w] = is; }
+    __syncthreads();
+    if (w == 0) {
+      int x = wsum[0][lane], y = wsum[1][lane];
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const int p = __shfl_up_sync(0xffffffffu, x, d), q = __shfl_up_sync(0xffffffffu, y, d);
+        if (lane >= d) { x += p; y += q; }
+      }
+      wsum[0][lane] = x;
+      wsum[1][lane] = y;
     }
-    rbase += tot;
-    sbase += (tot + EMB_SEG - 1) / EMB_SEG;
+    __syncthreads();
+    int ra = carry[0] + (it - ta) + (w > 0 ? wsum[0][w - 1] : 0);
+    int rs = carry[1] + (is - ts) + (w > 0 ? wsum[1][w - 1] : 0);
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const int v = t0 + tid * 4 + k;
+      if (v < V) { lo[v] = ra; segoff[v] = rs; }
+      ra += a[k];
+      rs += s[k];
+    }
+    __syncthreads();   // everyone has read carry
+    if (tid == 1023) { carry[0] = ra; carry[1] = rs; }
+    __syncthreads();
   }
-  if (tid == nt - 1) { lo[V] = rbase; segoff[V] = sbase; }
+  if (tid == 0) { lo[V] = carry[0]; segoff[V] = carry[1]; }
+}
+
+// cnt[b][v] ← lo_v + Σ_{b' < b} cnt[b'][v]: the first sorted position of block b's rows of token v
+__global__ void emb_cursor_kernel(int32_t* __restrict__ cnt, long nblk, int V, const int32_t* __restrict__ lo) {
+  const int v = blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= V) return;
+  int run = lo[v];
+  long b = 0;
+  for (; b + 8 <= nblk; b += 8) {
+    int c[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) c[k] = cnt[(b + k) * V + v];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      cnt[(b + k) * V + v] = run;
+      run += c[k];
+    }
+  }
+  for (; b < nblk; ++b) {
+    const int c = cnt[b * V + v];
+    cnt[b * V + v] = run;
+    run += c;
+  }
 }
 
 // Stable scatter: one warp per block walks its rows 32 at a time in ascending order; lanes with the
 // same token rank themselves by lane (match.any), the lowest of them advances the token's cursor.
-__global__ void __launch_bounds__(32) emb_scatter_kernel(const int32_t* __restrict__ tok, long n, int V,
-                                                         int32_t* __restrict__ cnt, int32_t* __restrict__ skeys,
-                                                         int32_t* __restrict__ srows) {
+__global__ void __launch_bounds__(32) emb_scatter_kernel(const int32_t* __restrict__ tok, long n, long blk, int V,
+                                                         int32_t* __restrict__ cnt, int32_t* __restrict__ srows) {
   const long b = blockIdx.x;
   const int lane = threadIdx.x;
-  const long r0 = b * EMB_BLK, r1 = min(n, r0 + EMB_BLK);
-  int32_t* cur = cnt + b * V;   // this block's cursors (first positions, from emb_scan_kernel)
+  const long r0 = b * blk, r1 = min(n, r0 + blk);
+  int32_t* cur = cnt + b * V;   // this block's cursors (first positions, from emb_cursor_kernel)
   for (long base = r0; base < r1; base += 32) {
     const long i = base + lane;
     const bool ok = i < r1;
@@ -1064,7 +1263,6 @@ __global__ void __launch_bounds__(32) emb_scatter_kernel(const int32_t* __restri
     pos = __shfl_sync(0xffffffffu, pos, leader) + rank;
     __syncwarp();
     if (valid) {
-      skeys[pos] = v;
       srows[pos] = (int32_t)i;
       if (lane == leader) cur[v] = pos - rank + __popc(peers);
     }
@@ -1072,65 +1270,115 @@ __global__ void __launch_bounds__(32) emb_scatter_kernel(const int32_t* __restri
   }
 }
 
-// partial[s][c] = Σ rows of segment s (ascending); the owning token is found from segoff.
-__global__ void emb_seg_partial_kernel(const int32_t* __restrict__ srows, int V, const int32_t* __restrict__ lo,
-                                       const int32_t* __restrict__ segoff, const float* __restrict__ dX, long ldx,
-                                       int I, float* __restrict__ part) {
-  const int s = blockIdx.y;
-  const int total = segoff[V];
-  if (s >= total) return;
-  // token v: last v with segoff[v] <= s
-  int a = 0, b = V;  // invariant segoff[a] <= s < segoff[b]
-  while (b - a > 1) {
-    const int m = (a + b) / 2;
-    if (segoff[m] <= s) a = m; else b = m;
-  }
-  const int v = a;
-  const long l = lo[v];
-  const long h = lo[v + 1];
-  const long r0 = l + (long)(s - segoff[v]) * EMB_SEG;
-  const long r1 = min(h, r0 + EMB_SEG);
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= I) return;
-  float acc = 0.f;
-  for (long k = r0; k < r1; ++k) acc = __fadd_rn(acc, dX[(long)srows[k] * ldx + c]);
-  part[(long)s * I + c] = acc;
+// W consecutive columns per thread (4 where I and the row stride allow float4, else 1)
+template <int W> struct emb_vec;
+template <> struct emb_vec<4> { using t = float4; };
+template <> struct emb_vec<1> { using t = float; };
+__device__ __forceinline__ void emb_acc(float4& a, const float4& x) {
+  a.x = __fadd_rn(a.x, x.x); a.y = __fadd_rn(a.y, x.y); a.z = __fadd_rn(a.z, x.z); a.w = __fadd_rn(a.w, x.w);
+}
+__device__ __forceinline__ void emb_acc(float& a, const float& x) { a = __fadd_rn(a, x); }
+template <int W> __device__ __forceinline__ typename emb_vec<W>::t emb_zero() {
+  if constexpr (W == 4) return make_float4(0.f, 0.f, 0.f, 0.f); else return 0.f;
 }
 
+// partial[s][c] = Σ rows of segment s (ascending); the owning token is found from segoff.  A
+// grid-stride loop over the segments actually present (segoff[V]).
+template <int W>
+__global__ void __launch_bounds__(256) emb_seg_partial_kernel(const int32_t* __restrict__ srows, int V,
+                                                              const int32_t* __restrict__ lo,
+                                                              const int32_t* __restrict__ segoff,
+                                                              const float* __restrict__ dX, long ldx, int I,
+                                                              float* __restrict__ part) {
+  using VT = typename emb_vec<W>::t;
+  const int total = segoff[V];
+  const int c = (blockIdx.x * blockDim.x + threadIdx.x) * W;
+  if (c >= I) return;
+  for (int s = blockIdx.y; s < total; s += gridDim.y) {
+    // token v: last v with segoff[v] <= s
+    int a = 0, b = V;  // invariant segoff[a] <= s < segoff[b]
+    while (b - a > 1) {
+      const int m = (a + b) / 2;
+      if (segoff[m] <= s) a = m; else b = m;
+    }
+    const long r0 = lo[a] + (long)(s - segoff[a]) * EMB_SEG;
+    const long r1 = min((long)lo[a + 1], r0 + EMB_SEG);
+    VT acc = emb_zero<W>();
+    long k = r0;
+    for (; k + 8 <= r1; k += 8) {
+      VT x[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) x[j] = *reinterpret_cast<const VT*>(dX + (long)srows[k + j] * ldx + c);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) emb_acc(acc, x[j]);
+    }
+    for (; k < r1; ++k) emb_acc(acc, *reinterpret_cast<const VT*>(dX + (long)srows[k] * ldx + c));
+    *reinterpret_cast<VT*>(part + (long)s * I + c) = acc;
+  }
+}
+
+// dE[v][c] = Σ_s part[s][c] over token v's segments in order (0 for an absent token); W columns
+// per thread, one flat grid over V·I/W.
+template <int W>
 __global__ void emb_seg_final_kernel(int V, const int32_t* __restrict__ segoff, const float* __restrict__ part, int I,
                                      float* __restrict__ dE) {
-  const int v = blockIdx.y;
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= I) return;
-  const int s0 = segoff[v];
-  dE[(long)v * I + c] = ordered_sum<32>(part + (long)s0 * I + c, segoff[v + 1] - s0, I);
+  using VT = typename emb_vec<W>::t;
+  const long q = (long)blockIdx.x * blockDim.x + threadIdx.x;
+  const int iw = I / W;
+  if (q >= (long)V * iw) return;
+  const int v = (int)(q / iw), c = (int)(q % iw) * W;
+  const int s0 = segoff[v], s1 = segoff[v + 1];
+  VT acc = emb_zero<W>();
+  for (int s = s0; s < s1; ++s) emb_acc(acc, *reinterpret_cast<const VT*>(part + (long)s * I + c));
+  *reinterpret_cast<VT*>(dE + (long)v * I + c) = acc;
 }
 
-size_t embed_bwd_partial_floats(long n, int V, int I) { return (size_t)(n / EMB_SEG + V + 1) * I; }
+size_t embed_bwd_partial_floats(long n, int V, int I) {
+  return (size_t)(n / EMB_SEG + (n < V ? n : V) + 1) * I;   // segments ≤ n/EMB_SEG + distinct tokens
+}
 
 void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int I, float* dE, void* scratch,
                size_t scratch_bytes, float* part, cudaStream_t st) {
-  const long nblk = emb_blocks(n);
+  if (n == 0) {
+    CUDA_TRY(cudaMemsetAsync(dE, 0, (size_t)V * I * 4, st));
+    return;
+  }
+  const long blk = emb_blk(n), nblk = emb_blocks(n);
   const size_t nb = round_up(n * 4, 256), vb = round_up((V + 1) * 4L, 256);
   const size_t cb = round_up((size_t)nblk * V * 4, 256);
   ASTRA_CHECK_ARG(scratch_bytes >= cb + 2 * nb + 3 * vb, "embed_bwd: scratch too small");
   char* base = (char*)scratch;
   int32_t* cnt = (int32_t*)base;
-  int32_t* skeys = (int32_t*)(base + cb);
   int32_t* srows = (int32_t*)(base + cb + nb);
   int32_t* lo = (int32_t*)(base + cb + 2 * nb);
   int32_t* segoff = (int32_t*)(base + cb + 2 * nb + vb);
   CUDA_TRY(cudaMemsetAsync(cnt, 0, (size_t)nblk * V * 4, st));
-  emb_count_kernel<<<(unsigned)nblk, 256, 0, st>>>(tok, n, V, cnt);
+  emb_count_kernel<<<(unsigned)nblk, 256, 0, st>>>(tok, n, blk, V, cnt);
   LAUNCH_CHECK();
-  emb_scan_kernel<<<1, 1024, 0, st>>>(cnt, nblk, V, lo, segoff);
+  emb_total_kernel<<<cdiv(V, 256), 256, 0, st>>>(cnt, nblk, V, lo, segoff);
   LAUNCH_CHECK();
-  emb_scatter_kernel<<<(unsigned)nblk, 32, 0, st>>>(tok, n, V, cnt, skeys, srows);
+  emb_scan_kernel<<<1, 1024, 0, st>>>(V, lo, segoff);
   LAUNCH_CHECK();
-  const long max_seg = n / EMB_SEG + V;
-  emb_seg_partial_kernel<<<dim3(cdiv(I, 256), (unsigned)max_seg), 256, 0, st>>>(srows, V, lo, segoff, dX, ldx, I, part);
+  emb_cursor_kernel<<<cdiv(V, 256), 256, 0, st>>>(cnt, nblk, V, lo);
   LAUNCH_CHECK();
-  emb_seg_final_kernel<<<dim3(cdiv(I, 256), V), 256, 0, st>>>(V, segoff, part, I, dE);
+  emb_scatter_kernel<<<(unsigned)nblk, 32, 0, st>>>(tok, n, blk, V, cnt, srows);
+  LAUNCH_CHECK();
+  const long max_seg = n / EMB_SEG + (n < V ? n : V);
+  const bool vec = I % 4 == 0 && ldx % 4 == 0 && ((uintptr_t)dX & 15) == 0 && ((uintptr_t)dE & 15) == 0 &&
+                   ((uintptr_t)part & 15) == 0;
+  const int W = vec ? 4 : 1;
+  const int gx = cdiv(I, 256 * W);
+  const long gy = std::min<long>(max_seg, 148L * 16 / gx + 1);
+  const unsigned gf = (unsigned)cdiv((long)V * (I / W), 256);
+  if (vec) {
+    emb_seg_partial_kernel<4><<<dim3(gx, (unsigned)gy), 256, 0, st>>>(srows, V, lo, segoff, dX, ldx, I, part);
+    LAUNCH_CHECK();
+    emb_seg_final_kernel<4><<<gf, 256, 0, st>>>(V, segoff, part, I, dE);
+  } else {
+    emb_seg_partial_kernel<1><<<dim3(gx, (unsigned)gy), 256, 0, st>>>(srows, V, lo, segoff, dX, ldx, I, part);
+    LAUNCH_CHECK();
+    emb_seg_final_kernel<1><<<gf, 256, 0, st>>>(V, segoff, part, I, dE);
+  }
   LAUNCH_CHECK();
 }
 

@@ -370,9 +370,14 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
   // a0: embedding gather into layer 0's operand buffer
   embed_gather(c.ot, tokens, TB, P + find("E"), c0.I, c0.x_operand(), c0.Ip, st);
   // head weight mirror (independent of the forward)
-  CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, hst));
-  for (const KSeg& s : segs)
-    mirror_T(c.ot, P + find("W_o") + (size_t)s.r0 * V, s.n, V, Vr, s.n, Wom + (size_t)s.k0 * e, Yw, hst);
+  // each segment's mirror writes its whole padded width [k0, next k0) × Vr rows (zeros past the
+  // segment's rows and past V), so the mirror covers [0, Yw) without a separate memset
+  if (segs.empty() || segs[0].k0 != 0) CUDA_TRY(cudaMemsetAsync(Wom, 0, (size_t)Vr * Yw * e, hst));
+  for (size_t i = 0; i < segs.size(); ++i) {
+    const KSeg& s = segs[i];
+    const int kend = i + 1 < segs.size() ? segs[i + 1].k0 : Yw;
+    mirror_T(c.ot, P + find("W_o") + (size_t)s.r0 * V, s.n, V, Vr, kend - s.k0, Wom + (size_t)s.k0 * e, Yw, hst);
+  }
   // a4 per time chunk: head forward + CE + head dgrad (SE2).  The head reads the cell's output
   // operand (SCRN: [h | s], a K-concatenated "ladder" [h|s]·[U;V]).
   const Mat2 Y = c.y_operand();

@@ -369,14 +369,16 @@ def test_stream_schedules_lm_bitwise(variant):
     assert torch.equal(pa, pb) and la == lb
 
 
-@pytest.mark.parametrize("T,B,V,nsym", [(100, 512, 256, 205), (35, 64, 10000, None), (7, 33, 50, 3)])
-def test_embedding_backward_counting_sort(T, B, V, nsym):
+@pytest.mark.parametrize("T,B,V,nsym,I", [(100, 512, 256, 205, 64), (35, 64, 10000, None, 64), (7, 33, 50, 3, 64),
+                                         (9, 40, 50, 5, 30)])
+def test_embedding_backward_counting_sort(T, B, V, nsym, I):
     """The embedding backward's hand-written stable counting sort + ordered segment sums (R5) against
     the oracle's dE[v] = Σ_{(t,b): tok = v} dx[t,b] on the fp32 path (1e-4, element-wise): the cfg5
     token statistics (hot Zipf symbols, segments of many 64-row pieces), a 10k vocabulary (mostly
-    empty rows, which must be exactly zero) and a 3-symbol batch."""
+    empty rows, which must be exactly zero), a 3-symbol batch, and an embedding width that is not a
+    multiple of 4 (the scalar column path) with a vocabulary that is not either (the scalar CE)."""
     import paper_conf_asplos_sivathanucsz19_b200 as A
-    I, H = 64, 64
+    H = 64
     tok = synth.zipf_tokens(7, "tok", (T + 1, B), V, nsym)
     shapes = cell_shapes("lstm", I, H)
     shapes.update({"E": (V, I), "W_o": (H, V), "b_o": (V,)})
