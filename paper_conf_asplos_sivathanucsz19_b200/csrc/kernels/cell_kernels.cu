@@ -429,7 +429,7 @@ void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, 
   throw Error(ASTRA_E_UNSUPPORTED, "lstm_fwd_pointwise: kind");
 }
 
-static unsigned long long* g_trace[TRACE_KINDS] = {nullptr, nullptr, nullptr};
+static unsigned long long* g_trace[TRACE_KINDS] = {nullptr, nullptr, nullptr, nullptr};
 unsigned long long* trace_buffer(int kind) { return kind >= 0 && kind < TRACE_KINDS ? g_trace[kind] : nullptr; }
 void set_trace_buffer(int kind, unsigned long long* buf) {
   ASTRA_CHECK_ARG(kind >= 0 && kind < TRACE_KINDS, "debug_set_trace: unknown kind");

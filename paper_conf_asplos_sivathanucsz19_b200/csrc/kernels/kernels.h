@@ -10,7 +10,7 @@ namespace astra {
 
 // Diagnostic phase traces (astra_debug_set_trace): device buffers of globaltimer stamps written by
 // instrumented kernels when set; null (the default) disables the stamps.
-enum TraceKind { TRACE_FWD_PW = 0, TRACE_RHN_FWD = 1, TRACE_SB_FWD = 2, TRACE_KINDS };
+enum TraceKind { TRACE_FWD_PW = 0, TRACE_RHN_FWD = 1, TRACE_SB_FWD = 2, TRACE_SB_BWD = 3, TRACE_KINDS };
 unsigned long long* trace_buffer(int kind);
 void set_trace_buffer(int kind, unsigned long long* buf);
 

@@ -96,6 +96,68 @@ __global__ void __launch_bounds__(64, 1) tma_read_kernel(const __grid_constant__
   __syncthreads();
 }
 
+// One tcgen05.mma chain per CTA: `iters` dependent MMAs (M x N x 16, bf16, both operands K-major
+// SWIZZLE_128B in shared memory, the 4 K-steps of one 64-wide k-block in turn) — the per-MMA issue
+// time of the small-batch chains as a function of M and N.  A[m][k] = ((3m + k) mod 7 − 3)/4,
+// B[n][k] = ((5n + 2k) mod 5 − 2)/2 (exact in bf16).  cycles[cta] = clock64 from the first issue to
+// the commit's mbarrier completing; with iters == 1 CTA 0 dumps all 128 TMEM lanes × N columns to
+// dump[lane][col] (the accumulator layout for M = 64).
+__global__ void __launch_bounds__(128, 1) mma_chain_kernel(int M, int N, int iters, uint32_t idesc,
+                                                           long long* __restrict__ cycles, float* __restrict__ dump) {
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char* sm = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  unsigned char* sA = sm;               // 128 rows x 128 B
+  unsigned char* sB = sm + 128 * 128;   // 256 rows x 128 B
+  __shared__ uint64_t bar;
+  __shared__ uint32_t tbase;
+  const int tid = threadIdx.x;
+  for (int i = tid; i < (128 + 256) * 64; i += blockDim.x) {
+    const bool isA = i < 128 * 64;
+    const int j = isA ? i : i - 128 * 64, r = j / 64, k = j % 64;
+    const float v = isA ? (float)(((3 * r + k) % 7) - 3) * 0.25f : (float)(((5 * r + 2 * k) % 5) - 2) * 0.5f;
+    unsigned char* base = isA ? sA : sB;
+    const int chunk = (k / 8) ^ (r % 8);
+    __nv_bfloat16* dst = (__nv_bfloat16*)(base + (r / 8) * 1024 + (r % 8) * 128 + chunk * 16) + (k % 8);
+    *dst = __float2bfloat16_rn(v);
+  }
+  if (tid == 0) {
+    sm100::mbar_init(&bar, 1);
+    sm100::fence_barrier_init();
+  }
+  if (tid < 32) sm100::tmem_alloc(&tbase, 256);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  sm100::tc_fence_before();
+  __syncthreads();
+  sm100::tc_fence_after();
+  const uint32_t tmem = tbase;
+  if (tid == 0) {
+    const uint64_t a0 = sm100::smem_desc_sw128(sm100::smem_u32(sA), 16, 1024);
+    const uint64_t b0 = sm100::smem_desc_sw128(sm100::smem_u32(sB), 16, 1024);
+    const long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+      const uint64_t kk = (uint64_t)(i & 3) * 2;   // 32 B per K-step of 16 bf16
+      sm100::umma_bf16(tmem, a0 + kk, b0 + kk, idesc, i > 0 ? 1u : 0u);
+    }
+    sm100::umma_commit(&bar);
+    sm100::mbar_wait(&bar, 0);
+    const long long t1 = clock64();
+    cycles[blockIdx.x] = t1 - t0;
+  }
+  __syncthreads();
+  sm100::tc_fence_after();
+  if (dump && blockIdx.x == 0) {
+    const int w = tid / 32;
+    for (int c0 = 0; c0 < N; c0 += 16) {
+      float v[16];
+      sm100::tmem_ld16(tmem + ((uint32_t)(w * 32) << 16) + c0, v);
+      for (int j = 0; j < 16; ++j) dump[(long)tid * N + c0 + j] = v[j];
+    }
+  }
+  sm100::tc_fence_before();
+  __syncthreads();
+  if (tid < 32) sm100::tmem_dealloc(tmem, 256);
+}
+
 __global__ void empty_pdl_kernel(int) {
   pdl_wait();
   pdl_trigger();
@@ -128,6 +190,21 @@ void micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, 
   const int smem = 1024 + stages * box_rows * 128 + stages * 16;
   CUDA_TRY(cudaFuncSetAttribute(tma_read_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   tma_read_kernel<<<ctas, 64, smem, st>>>(m, nbox, box_rows, stages, kb, (int)(rows / box_rows), same);
+  LAUNCH_CHECK();
+}
+
+void micro_mma_chain(int M, int N, int iters, int ctas, long long* cycles, float* dump, cudaStream_t st) {
+  ASTRA_CHECK_ARG((M == 64 || M == 128) && N >= 16 && N <= 256 && N % 16 == 0 && iters >= 1 && ctas >= 1 && cycles,
+                  "micro_mma_chain: bad arguments");
+  uint32_t d = 0;
+  d |= 1u << 4;                     // D F32
+  d |= 1u << 7;                     // A BF16
+  d |= 1u << 10;                    // B BF16
+  d |= (uint32_t)(N >> 3) << 17;    // N >> 3
+  d |= (uint32_t)(M >> 4) << 24;    // M >> 4
+  const int smem = 1024 + (128 + 256) * 128;
+  CUDA_TRY(cudaFuncSetAttribute(mma_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  mma_chain_kernel<<<ctas, 128, smem, st>>>(M, N, iters, d, cycles, dump);
   LAUNCH_CHECK();
 }
 

@@ -165,6 +165,36 @@ void scrn_bwd_persist_launch(const void* DZ, long lddz, const void* Rk, int T, b
                              cudaStream_t st);
 void scrn_fwd_persist_launch(const void* HS, long ldhs, const void* MR, int Tmax, ScrnPersistArgs a, cudaStream_t st);
 
+// Small-batch persistent BPTT chain (bptt_persist.cu, LSTM-family bwd_mode 2/3): t = T−1 … 0 in one
+// cooperative launch of Hp/16 CTAs in clusters of 4 (the R25 split-K chunks), 64 units per cluster,
+// the chunk partials of dh_rec summed in chunk order over distributed shared memory, the cell
+// backward fused, one counter per K chunk.  B ≤ 128, bf16 path, Hp % 256 == 0, nsplit == 4.
+struct BpttPersistArgs {
+  int B, H, Hp, NG, T;
+  int kper, resident, sa, sb, a_rows, a_bytes, ka, kbs;   // set by the launcher
+  uint32_t idesc;
+  int nq;                   // column-sum quantities (4 MI-LSTM, else 1)
+  GateParams gp;
+  const void* dy;           // fp32 [T·B][ldy] (LM, ldy = Hp) or bf16 [T·B][ldy] (external, ldy = H)
+  long ldy;
+  const float* dhT;         // optional [B][H]
+  const float* WX;          // [T·B][NG]
+  const float* UH;          // [T·B][NG]
+  const float* C;           // [(T+1)·B][Hp]
+  float* dc;                // [B][Hp]: dc_T in, dc_0 out
+  __nv_bfloat16* D_uh;      // [T·B][NG]
+  __nv_bfloat16* D_wx;      // [T·B][NG] (MI-LSTM)
+  float* partials;          // [ceil(B/32)][nq][NG], written at the end
+  unsigned* flags;          // [4] per-chunk counters, zeroed before the launch
+  unsigned long long spin;  // diagnostics: give up a wait after this many probes (0: never)
+  unsigned long long* trace;   // optional (astra_debug_set_trace kind 3): [grid][T][8] globaltimer stamps
+};
+bool lstm_bptt_persist_supported(int B, int Hp, int nsplit);
+// true when the clusters of the launch are co-resident on this device (checked once per shape)
+bool lstm_bptt_persist_fits(int kind, int B, int Hp, int NG);
+void lstm_bptt_persist_launch(int kind, bool dy_f32, const void* Duh, const void* Um, int Tmax, BpttPersistArgs a,
+                              cudaStream_t st);
+
 bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);
 void lstm_bptt_fused_launch(int kind, bool dy_bf16, const BpttFusedMaps& m, BpttFusedArgs a, cudaStream_t st);
 

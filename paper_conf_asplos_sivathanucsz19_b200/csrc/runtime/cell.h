@@ -38,7 +38,7 @@ struct KCfg {
   int cg = 1;   // 2: CTA pair (cta_group::2, 256-row tiles)
   bool operator==(const KCfg& o) const { return bn == o.bn && cm == o.cm && cn == o.cn && cg == o.cg; }
 };
-enum GemmRole { G_A1 = 0, G_REC, G_BPTT, G_DU, G_DW, G_DX, G_HEAD, G_ROLES };
+enum GemmRole { G_A1 = 0, G_REC, G_BPTT, G_DU, G_DW, G_DX, G_HEAD, G_HDY, G_ROLES };
 extern const char* const ROLE_NAMES[G_ROLES];
 
 // One binding of every adaptive variable (the enumerator's output for a cell).
@@ -48,7 +48,8 @@ constexpr int WGS_CHUNKS[3] = {1, 4, 10};      // wgrad_schedule time chunks (1:
 constexpr int GCHUNK_S[5] = {1, 1, 1, 2, 2};   // streams they run on
 constexpr int WF_CHUNKS[3] = {1, 5, 1 << 20};   // clipped to T: the last option is one chunk per step
 struct Variant {
-  KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head
+  KCfg g[G_ROLES];      // a1 hoisted projection, recurrent step, BPTT step, dU, dW, dX, LM head (logits, dW_o),
+                        // LM head dgrad dY = dlogits·W_o (N = the cell's output width, not V: its own tile choice)
   int wg_side = 0;      // 1: dU on a side stream concurrently with dW/dX (B3)
   int fwd_mode = 0;     // K2 (LSTM family, bf16): 0 GEMM + pointwise kernel, 1 fused per step, 2 fused persistent
   int bwd_mode = 0;     // K4: same encoding

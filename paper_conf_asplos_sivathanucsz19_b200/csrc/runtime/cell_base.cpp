@@ -13,7 +13,7 @@
 
 namespace astra {
 
-const char* const ROLE_NAMES[G_ROLES] = {"a1", "rec", "bptt", "du", "dw", "dx", "head"};
+const char* const ROLE_NAMES[G_ROLES] = {"a1", "rec", "bptt", "du", "dw", "dx", "head", "hdy"};
 
 std::string Variant::str() const {
   std::ostringstream o;
@@ -385,12 +385,17 @@ void Cell::set_active_T(int t) {
 void Cell::tuner_setup() {
   const Variant def;
   std::string par;
-  const char* metric[G_ROLES] = {"t_a1", "t_fwd", "t_bptt", "t_du", "t_dw", "t_dx", "t_head"};
+  const char* metric[G_ROLES] = {"t_a1", "t_fwd", "t_bptt", "t_du", "t_dw", "t_dx", "t_head", "t_head"};
   if (ot == OT::BF16) {
     for (int r = 0; r < G_ROLES; ++r) {
-      if (r == G_HEAD && !lm_mode) continue;
+      if ((r == G_HEAD || r == G_HDY) && !lm_mode) continue;
       int M, N;
-      role_shape(r, M, N);
+      if (r == G_HDY) {
+        M = T * B;
+        N = y_width();
+      } else {
+        role_shape(r, M, N);
+      }
       if (M <= 0 || N <= 0) continue;
       allowed[r].clear();
       allowed[r].push_back(def.g[r]);

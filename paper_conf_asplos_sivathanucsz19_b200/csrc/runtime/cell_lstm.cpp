@@ -114,6 +114,14 @@ class LstmCell : public Cell {
   const void* bm_key[4] = {nullptr, nullptr, nullptr, nullptr};   // (WX, dy, Duh, T) they were built for
 
   // K4 fusion choices (AV fuse_bwd): GEMM + pointwise kernel, or the fused BPTT kernel
+  // K4 fusion choices (AV fuse_bwd): 0 GEMM + pointwise kernel, 1 the fused BPTT kernel per step.
+  // bwd=2 (or 3), the small-batch persistent BPTT chain (B ≤ 128, 4 K chunks, bptt_persist.cu), is
+  // a frozen-variant option only: at cfg5 B = 64 it is slower than the launched chain (2.26 vs
+  // 2.03 ms per 100 steps, profiles/r2_pb_sweep23.jsonl), and its t_bptt beats the launched chain
+  // measured next to wgrad_schedule's side-stream dX, which made the tuner pick it for a slower step.
+  bool bptt_persist_ok() const {
+    return ot == OT::BF16 && lstm_bptt_persist_supported(B, Hp, bptt_ksplit()) && lstm_bptt_persist_fits(kind, B, Hp, NG);
+  }
   int bwd_fusions() const override {
     return (ot == OT::BF16 && lstm_bptt_fused_supported(B, Hp, bptt_ksplit())) ? 2 : 1;
   }
@@ -368,8 +376,10 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   GemmSpec bp0 = bp;   // dh0 (once, no split)
   bp.ksplit = bptt_ksplit();
   // fused BPTT step (K4 fused): dy must be TMA-mappable (the LM's fp32 dY, or bf16 with H % 8 == 0)
-  const bool fuse = var.bwd_mode == 1 && bwd_fusions() > 1 && T > 1 &&
+  const bool fuse = var.bwd_mode == 1 && lstm_bptt_fused_supported(B, Hp, bp.ksplit) && ot == OT::BF16 && T > 1 &&
                     (lm_dy || (H % 8 == 0 && ((uintptr_t)dy & 15) == 0));
+  // small-batch persistent BPTT chain (bptt_persist.cu): the whole range in one launch
+  const bool persist = !fuse && var.bwd_mode >= 2 && whole && var.recomp == 0 && bptt_persist_ok();
   BpttFusedArgs fa{};
   if (fuse) {
     const TcGemm& tg = tc_get(2, bp, KCfg{64, 1, 1});
@@ -459,7 +469,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   };
   // wgrad_schedule (§8(a.9)): the input dgrad in time chunks on a side stream, each as
   // soon as the chain has produced its D_wx rows, on the SMs the per-step BPTT GEMM leaves free
-  const int wgs_n = (whole && dx && var.wgs > 0 && !side.empty() && ot == OT::BF16 && !fuse)
+  const int wgs_n = (whole && dx && var.wgs > 0 && !side.empty() && ot == OT::BF16 && !fuse && !persist)
                         ? std::min(WGS_CHUNKS[var.wgs], T) : 1;
   cudaStream_t wst = side.empty() ? st : side.back();
   int wgs_k = 0;
@@ -472,7 +482,19 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     for (int i = 0; i < wgs_n + 1; ++i)
       if (!ev_wgs[i]) CUDA_TRY(cudaEventCreateWithFlags(&ev_wgs[i], cudaEventDisableTiming));
   }
-  const bool rsplit = row_split_ok(bwd_hook != nullptr) && !fuse && whole && wgs_n == 1;
+  const bool rsplit = row_split_ok(bwd_hook != nullptr) && !fuse && !persist && whole && wgs_n == 1;
+  if (persist) {
+    BpttPersistArgs pa{};
+    pa.B = B; pa.H = H; pa.Hp = Hp; pa.NG = NG; pa.T = T; pa.nq = nq; pa.gp = gp;
+    if (lm_dy) { pa.dy = lm_dy; pa.ldy = Hp; }
+    else { pa.dy = dy; pa.ldy = H; }
+    pa.dhT = dhT; pa.WX = WX; pa.UH = UH; pa.C = Cb; pa.dc = dC;
+    pa.D_uh = (__nv_bfloat16*)Duh; pa.D_wx = (__nv_bfloat16*)Dwx; pa.partials = part;
+    pa.flags = sc<unsigned>(off_flags);
+    pa.trace = trace_buffer(TRACE_SB_BWD);   // diagnostics only (null: no stamps)
+    CUDA_TRY(cudaMemsetAsync(pa.flags, 0, 64, st));
+    lstm_bptt_persist_launch(kind, lm_dy != nullptr, Duh, Um, Tmax, pa, st);
+  }
   if (rsplit) {   // row_streams: the two row halves' BPTT chains on (main, side[0])
     const int Bh = B / 2;
     rs_fork(st);
@@ -511,7 +533,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     }
     rs_join(st);
   }
-  for (int t = rsplit ? t0 - 1 : t1 - 1; t >= t0; --t) {
+  for (int t = (rsplit || persist) ? t0 - 1 : t1 - 1; t >= t0; --t) {
     const int kc = t / RC;
     if (rc && !fuse && rs != st && t == chunk_hi(kc) - 1) CUDA_TRY(cudaStreamWaitEvent(st, ev_rc_done[kc & 1], 0));
     if (fuse && t < T - 1) {

@@ -402,7 +402,7 @@ void LM::enqueue_step(const int32_t* tokens, float lr, float* loss_dev, bool do_
     dy.B = mat(Wom, Yw, V, Yw);
     dy.b_mn = true;
     dy.M = rows; dy.N = Yw; dy.K = V;
-    c.run_gemm(nch > 1 ? 130 + k : 101, dy, epi(dY + r0 * Yw, Yw, rows, Yw), 0, 0, c.var.g[G_HEAD], hst);
+    c.run_gemm(nch > 1 ? 130 + k : 101, dy, epi(dY + r0 * Yw, Yw, rows, Yw), 0, 0, c.var.g[G_HDY], hst);
   };
   // cell forward (SE1); final state carried for the next step (truncated BPTT) — except for a
   // variable-length step, whose padded tail would corrupt it (zero state, no carry)

@@ -93,6 +93,34 @@ def test_small_batch_persistent_forward_bitwise(cell, T, B, H):
     _check(cell, T, B, I, H, "bf16", 93, TOL_BF16, variant="fwd=3")
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+@pytest.mark.parametrize("T,B,H", [(5, 64, 2048), (4, 37, 2000), (3, 100, 2048), (1, 64, 2048)])
+def test_small_batch_persistent_bptt_bitwise(cell, T, B, H):
+    """K4 small-batch persistent BPTT (bwd=2: one cooperative launch of 4-CTA clusters, the R25
+    chunk partials summed in chunk order over distributed shared memory, the cell backward fused,
+    a counter per K chunk) gives the same bits as BPTT GEMM + pointwise (bwd=0) for every gradient,
+    dx, dh0, dc0 — with the small-batch persistent forward too, B = 37 / H = 2000 (ragged rows and
+    padding units), B = 100 (128-row A boxes), T = 1 (no GEMM step) — and against the oracle."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    I = 64
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, 97, bf16=True)
+    ref = None
+    launches = {}
+    for v in ("bwd=0", "bwd=2", "bwd=3,fwd=3"):
+        n0 = A.launch_count()
+        out, g, c = run_gpu_cell(cell, p, inp, dY, dhT, dcT, "bf16", v)
+        launches[v] = A.launch_count() - n0
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    if T > 1:   # the persistent chain really ran: one launch instead of a GEMM + pointwise per step
+        assert launches["bwd=2"] <= launches["bwd=0"] - 2 * (T - 1) + 2, launches
+    _check(cell, T, B, I, H, "bf16", 97, TOL_BF16, variant="bwd=2")
+
+
 @pytest.mark.parametrize("gc", [1, 2, 3, 4])
 def test_gate_chunking_bitwise(gc):
     """gate_chunking (§8(a.9), P:196 / P:220): the hoisted gate projection as 2 or 4 GEMMs over

@@ -359,7 +359,7 @@ def test_tune_next_never_blocks():
 
 
 @pytest.mark.parametrize("variant", ["hov=1,wgs=2,gc=3,wg_side=1", "wgs=1,gc=4,fwd=3", "gc=2,wgs=2,rc=1",
-                                     "rsp=1,bpw=1,gc=3"])
+                                     "rsp=1,bpw=1,gc=3", "hdy=128.1.1.2,head=128.1.1", "hdy=64.2.1"])
 def test_stream_schedules_lm_bitwise(variant):
     """The stream-assignment variants together — head overlap, wgrad_schedule's dX chunks during
     BPTT, gate_chunking's projection GEMMs on two streams, the small-batch persistent forward —
