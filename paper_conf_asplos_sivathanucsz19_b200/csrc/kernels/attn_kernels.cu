@@ -3,9 +3,15 @@
 //
 //   e_j = vᵀ tanh(q + k_j),  p = softmax_j(e),  ctx = Σ_j p_j enc_j          (one decoder step, per b)
 //
-// One CTA per batch row b; every reduction (over the attention width A for e_j and the hidden units
-// for dp_j: one warp per source position, lane-strided partials + a fixed xor tree; over j for the
-// softmax: warp 0, the same tree) has a fixed order, so the result is independent of launch timing (R5).  fp32 throughout (ALU/MUFU-bound).
+// Each direction is two kernels over many CTAs (round 1 ran one CTA per batch row: 128 CTAs doing
+// the whole step serially, 60-130 µs per decoder step at cfg4): forward = scores (one warp per
+// (b, j)) then softmax + context (B × ⌈Hp/256⌉ CTAs); backward = dp_j (one warp per (b, j)) then
+// de, denc, dq, dk, dv (B × ⌈max(Hp, Ap)/256⌉ CTAs).  Every reduction has a fixed order (a warp's
+// lanes take float4 quads in ascending order + a fixed xor tree; the softmax and Σ p dp by warp 0
+// over lane-strided j; the context, dq, dv and the denc / dk accumulators in ascending j), so the
+// result is independent of launch timing (R5).  fp32 throughout (ALU/MUFU-bound).
+#include <algorithm>
+
 #include "cell_math.cuh"
 #include "kernels.h"
 #include "pdl.cuh"
@@ -14,51 +20,54 @@ namespace astra {
 
 constexpr int ATT_THREADS = 256;
 
-// Fixed-order block sum of one value per thread (ATT_THREADS threads); result broadcast to all.
-__device__ __forceinline__ float block_sum(float v, float* red) {
-#pragma unroll
-  for (int o = 16; o; o >>= 1) v = __fadd_rn(v, __shfl_xor_sync(0xffffffffu, v, o));
+// Scores, one warp per (b, j) over a grid of B × ⌈Ts/8⌉ CTAs: lane l takes the float4 quads
+// c = l, l + 32, … of the attention width in ascending order (tanh per element, then the products
+// added in element order), then a fixed xor tree over the lanes.  Rows b of the q / keys buffers
+// hold Ap floats (A ≤ Ap, the pad columns are ignored).
+template <typename T>
+__global__ void __launch_bounds__(ATT_THREADS)
+    attn_score_kernel(int B, int Ts, int A, int Ap, const float* __restrict__ q, const float* __restrict__ keys,
+                      const float* __restrict__ v, float* __restrict__ e) {
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   const int w = threadIdx.x / 32, l = threadIdx.x % 32;
-  __syncthreads();
-  if (l == 0) red[w] = v;
-  __syncthreads();
+  const int b = blockIdx.y, j = blockIdx.x * (ATT_THREADS / 32) + w;
+  if (j >= Ts) return;
+  const float4* qb = reinterpret_cast<const float4*>(q + (long)b * Ap);
+  const float4* kj = reinterpret_cast<const float4*>(keys + ((long)j * B + b) * Ap);
+  const float4* v4 = reinterpret_cast<const float4*>(v);
+  constexpr bool F = FastMath<T>::value;
   float s = 0.f;
-  if (threadIdx.x < 32) {
-    s = threadIdx.x < ATT_THREADS / 32 ? red[threadIdx.x] : 0.f;
-#pragma unroll
-    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
-    if (threadIdx.x == 0) red[32] = s;
+  const int nq = (A + 3) / 4;
+  for (int c = l; c < nq; c += 32) {
+    const float4 qa = qb[c], ka = __ldcs(kj + c), va = v4[c];
+    const int a0 = 4 * c;
+    s = __fadd_rn(s, __fmul_rn(va.x, tanh_<F>(__fadd_rn(qa.x, ka.x))));
+    if (a0 + 1 < A) s = __fadd_rn(s, __fmul_rn(va.y, tanh_<F>(__fadd_rn(qa.y, ka.y))));
+    if (a0 + 2 < A) s = __fadd_rn(s, __fmul_rn(va.z, tanh_<F>(__fadd_rn(qa.z, ka.z))));
+    if (a0 + 3 < A) s = __fadd_rn(s, __fmul_rn(va.w, tanh_<F>(__fadd_rn(qa.w, ka.w))));
   }
-  __syncthreads();
-  return red[32];
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+  if (l == 0) e[(long)b * Ts + j] = s;
 }
 
+// Softmax over j (every CTA of row b recomputes it from the scores: warp 0, lane-strided max / sum,
+// fixed xor trees), then ctx_h = Σ_j p_j enc_j,h in ascending j for the CTA's 256 hidden units;
+// the blockIdx.x == 0 CTA of each row stores p (saved for the backward).
 template <typename T, typename TY>
 __global__ void __launch_bounds__(ATT_THREADS)
-    attn_fwd_kernel(int B, int Ts, int H, int Hp, int A, int Ap, const float* __restrict__ q,
-                    const float* __restrict__ keys, const float* __restrict__ v, const float* __restrict__ enc,
+    attn_ctx_kernel(int B, int Ts, int H, int Hp, const float* __restrict__ escore, const float* __restrict__ enc,
                     float* __restrict__ pr, T* __restrict__ ctx_op, long ldc, TY* __restrict__ y_ctx, long ldy) {
-  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_wait();
   pdl_trigger();
   extern __shared__ float sh[];
   float* e = sh;            // [Ts]
-  float* red = sh + Ts;     // [33]
-  (void)red;
-  const int b = blockIdx.x;
+  const int b = blockIdx.y;
   const int w = threadIdx.x / 32, l = threadIdx.x % 32;
-  const float* qb = q + (long)b * Ap;
-  // e_j: one warp per source position j; lane l sums a = l, l + 32, ... in order, then a fixed
-  // xor-butterfly over the lanes (no block-wide barrier per j)
-  for (int j = w; j < Ts; j += ATT_THREADS / 32) {
-    const float* kj = keys + ((long)j * B + b) * Ap;
-    float s = 0.f;
-    for (int a = l; a < A; a += 32) s = __fadd_rn(s, __fmul_rn(v[a], tanh_<FastMath<T>::value>(__fadd_rn(qb[a], kj[a]))));
-#pragma unroll
-    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
-    if (l == 0) e[j] = s;
-  }
+  for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) e[j] = escore[(long)b * Ts + j];
   __syncthreads();
-  if (w == 0) {   // softmax over j by warp 0: lane-strided max / sum, fixed xor trees
+  if (w == 0) {
     float m = -INFINITY;
     for (int j = l; j < Ts; j += 32) m = fmaxf(m, e[j]);
 #pragma unroll
@@ -74,64 +83,105 @@ __global__ void __launch_bounds__(ATT_THREADS)
     for (int j = l; j < Ts; j += 32) e[j] = __fdiv_rn(e[j], s);
   }
   __syncthreads();
-  for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) pr[(long)b * Ts + j] = e[j];
-  for (int h = threadIdx.x; h < Hp; h += ATT_THREADS) {
-    float c = 0.f;
-    if (h < H)
-      for (int j = 0; j < Ts; ++j) c = __fadd_rn(c, __fmul_rn(e[j], enc[((long)j * B + b) * Hp + h]));
-    ctx_op[(long)b * ldc + h] = from_f<T>(c);
-    if (y_ctx && h < H) y_ctx[(long)b * ldy + h] = from_f<TY>(c);
+  if (blockIdx.x == 0)
+    for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) pr[(long)b * Ts + j] = e[j];
+  const int h = blockIdx.x * ATT_THREADS + threadIdx.x;
+  if (h >= Hp) return;
+  float c = 0.f;
+  if (h < H) {
+    constexpr int JG = 10;   // loads of a group issued before its adds (the sum order is unchanged)
+    for (int j0 = 0; j0 < Ts; j0 += JG) {
+      float x[JG];
+#pragma unroll
+      for (int k = 0; k < JG; ++k) x[k] = j0 + k < Ts ? enc[((long)(j0 + k) * B + b) * Hp + h] : 0.f;
+#pragma unroll
+      for (int k = 0; k < JG; ++k)
+        if (j0 + k < Ts) c = __fadd_rn(c, __fmul_rn(e[j0 + k], x[k]));
+    }
   }
+  ctx_op[(long)b * ldc + h] = from_f<T>(c);
+  if (y_ctx && h < H) y_ctx[(long)b * ldy + h] = from_f<TY>(c);
 }
 
 void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q, const float* keys, const float* v,
-              const float* enc, float* pr, void* ctx_op, long ldc, void* y_ctx, long ldy, cudaStream_t st) {
-  const size_t sm = (Ts + 40) * sizeof(float);
-  if (ot == OT::BF16)
-    launch_pdl(attn_fwd_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(B), dim3(ATT_THREADS), sm, st, 1, 
-        B, Ts, H, Hp, A, Ap, q, keys, v, enc, pr, (__nv_bfloat16*)ctx_op, ldc, (__nv_bfloat16*)y_ctx, ldy);
-  else
-    launch_pdl(attn_fwd_kernel<float, float>, dim3(B), dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, A, Ap, q, keys, v, enc, pr,
-                                                              (float*)ctx_op, ldc, (float*)y_ctx, ldy);
+              const float* enc, float* pr, float* escratch, void* ctx_op, long ldc, void* y_ctx, long ldy,
+              cudaStream_t st) {
+  ASTRA_CHECK_ARG(Ap % 4 == 0 && ((uintptr_t)q & 15) == 0 && ((uintptr_t)keys & 15) == 0 && ((uintptr_t)v & 15) == 0,
+                  "attn_fwd: q / keys / v rows must be 16-byte aligned float4 rows");
+  const dim3 gs(cdiv(Ts, ATT_THREADS / 32), B), gc(cdiv(Hp, ATT_THREADS), B);
+  const size_t sm = (Ts + 8) * sizeof(float);
+  if (ot == OT::BF16) {
+    launch_pdl(attn_score_kernel<__nv_bfloat16>, gs, dim3(ATT_THREADS), 0, st, 1, B, Ts, A, Ap, q, keys, v, escratch);
+    LAUNCH_CHECK();
+    launch_pdl(attn_ctx_kernel<__nv_bfloat16, __nv_bfloat16>, gc, dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp,
+               (const float*)escratch, enc, pr, (__nv_bfloat16*)ctx_op, ldc, (__nv_bfloat16*)y_ctx, ldy);
+  } else {
+    launch_pdl(attn_score_kernel<float>, gs, dim3(ATT_THREADS), 0, st, 1, B, Ts, A, Ap, q, keys, v, escratch);
+    LAUNCH_CHECK();
+    launch_pdl(attn_ctx_kernel<float, float>, gc, dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, (const float*)escratch,
+               enc, pr, (float*)ctx_op, ldc, (float*)y_ctx, ldy);
+  }
   LAUNCH_CHECK();
 }
 
 // Backward of one attention step (oracle/cells.py attn_backward):
 //   dctx = dy_ctx + dctx_rec;  dp_j = dctx·enc_j;  de_j = p_j (dp_j − Σ p dp);  denc_j += p_j dctx;
 //   u_j = tanh(q + k_j);  du_j = de_j v (1 − u_j²);  dq = Σ_j du_j;  dk_j += du_j;  dv_b += Σ_j de_j u_j
+// dctx_h of row b = dy_ctx + dctx_rec (0 past H)
+template <typename TDY>
+__device__ __forceinline__ float attn_dctx(const TDY* __restrict__ dy_ctx, long ldy, const float* __restrict__ dctx_rec,
+                                           long ldr, int b, int h, int H) {
+  if (h >= H) return 0.f;
+  float d = dy_ctx ? to_f<TDY>(dy_ctx[(long)b * ldy + h]) : 0.f;
+  if (dctx_rec) d = __fadd_rn(d, dctx_rec[(long)b * ldr + h]);
+  return d;
+}
+
+// dp_j = dctx·enc_j, one warp per (b, j): lane l takes the hidden quads c = l, l + 32, … in
+// ascending order, then a fixed xor tree.
+template <typename TDY>
+__global__ void __launch_bounds__(ATT_THREADS)
+    attn_dp_kernel(int B, int Ts, int H, int Hp, const TDY* __restrict__ dy_ctx, long ldy,
+                   const float* __restrict__ dctx_rec, long ldr, const float* __restrict__ enc, float* __restrict__ dp) {
+  pdl_wait();
+  pdl_trigger();
+  const int w = threadIdx.x / 32, l = threadIdx.x % 32;
+  const int b = blockIdx.y, j = blockIdx.x * (ATT_THREADS / 32) + w;
+  if (j >= Ts) return;
+  const float4* ej = reinterpret_cast<const float4*>(enc + ((long)j * B + b) * Hp);
+  float s = 0.f;
+  for (int c = l; 4 * c < H; c += 32) {
+    const float4 x = ej[c];
+    const int h = 4 * c;
+    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h, H), x.x));
+    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h + 1, H), x.y));
+    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h + 2, H), x.z));
+    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h + 3, H), x.w));
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
+  if (l == 0) dp[(long)b * Ts + j] = s;
+}
+
+// The rest of one attention step's backward, grid ⌈max(Hp, Ap)/256⌉ × B: every CTA of row b forms
+// de_j = p_j (dp_j − Σ p dp) (warp 0, lane-strided j, fixed xor tree), then thread index x does
+//   hidden unit x:  denc_j += p_j dctx  (read-modify-write in groups of ATT_JG source positions);
+//   width x:        u_j = tanh(q + k_j), du_j = de_j v (1 − u_j²), dq = Σ_j du_j, dk_j += du_j,
+//                   dv_b += Σ_j de_j u_j   (ascending j).
 template <typename T, typename TDY>
 __global__ void __launch_bounds__(ATT_THREADS)
     attn_bwd_kernel(int B, int Ts, int H, int Hp, int A, int Ap, const TDY* __restrict__ dy_ctx, long ldy,
                     const float* __restrict__ dctx_rec, long ldr, const float* __restrict__ pr,
-                    const float* __restrict__ q, const float* __restrict__ keys, const float* __restrict__ v,
-                    const float* __restrict__ enc, T* __restrict__ dq_op, float* __restrict__ denc,
+                    const float* __restrict__ dpv, const float* __restrict__ q, const float* __restrict__ keys,
+                    const float* __restrict__ v, T* __restrict__ dq_op, float* __restrict__ denc,
                     float* __restrict__ dk, float* __restrict__ dvb, int first) {
   pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
   pdl_trigger();
   extern __shared__ float sh[];
-  float* dctx = sh;              // [Hp]
-  float* de = sh + Hp;           // [Ts]
-  float* red = de + Ts;          // [33]
-  const int b = blockIdx.x;
-  for (int h = threadIdx.x; h < Hp; h += ATT_THREADS) {
-    float d = 0.f;
-    if (h < H) {
-      d = dy_ctx ? to_f<TDY>(dy_ctx[(long)b * ldy + h]) : 0.f;
-      if (dctx_rec) d = __fadd_rn(d, dctx_rec[(long)b * ldr + h]);
-    }
-    dctx[h] = d;
-  }
-  __syncthreads();
-  (void)red;
+  float* de = sh;                // [Ts]
+  const int b = blockIdx.y;
   const int w = threadIdx.x / 32, l = threadIdx.x % 32;
-  for (int j = w; j < Ts; j += ATT_THREADS / 32) {   // dp_j: one warp per j, lane-strided h, xor tree
-    const float* ej = enc + ((long)j * B + b) * Hp;
-    float s = 0.f;
-    for (int h = l; h < H; h += 32) s = __fadd_rn(s, __fmul_rn(dctx[h], ej[h]));
-#pragma unroll
-    for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
-    if (l == 0) de[j] = s;   // dp_j for now
-  }
+  for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) de[j] = dpv[(long)b * Ts + j];
   __syncthreads();
   if (w == 0) {   // de_j = p_j (dp_j − Σ p dp), the sum by a fixed xor tree over lane-strided partials
     float s = 0.f;
@@ -142,12 +192,11 @@ __global__ void __launch_bounds__(ATT_THREADS)
     for (int j = l; j < Ts; j += 32) de[j] = __fmul_rn(pr[(long)b * Ts + j], __fsub_rn(de[j], s));
   }
   __syncthreads();
-  // denc_j += p_j dctx.  The accumulators (L2-resident) are read-modified-written in groups of
-  // ATT_JG source positions with every load of a group issued before its stores, so a thread keeps
-  // ATT_JG requests in flight instead of one dependent round trip per j.
   constexpr int ATT_JG = 10;
-  for (int h = threadIdx.x; h < Hp; h += ATT_THREADS) {
-    const float dc = dctx[h];
+  const int x = blockIdx.x * ATT_THREADS + threadIdx.x;
+  if (x < Hp) {   // denc_j += p_j dctx
+    const int h = x;
+    const float dc = attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h, H);
     for (int j0 = 0; j0 < Ts; j0 += ATT_JG) {
       float old[ATT_JG];
 #pragma unroll
@@ -161,9 +210,9 @@ __global__ void __launch_bounds__(ATT_THREADS)
       }
     }
   }
-  // attention-width terms (dq and dv accumulated in ascending j, dk_j read-modify-written in groups)
-  const float* qb = q + (long)b * Ap;
-  for (int a = threadIdx.x; a < Ap; a += ATT_THREADS) {
+  if (x < Ap) {   // attention-width terms
+    const int a = x;
+    const float* qb = q + (long)b * Ap;
     float dq = 0.f, dva = 0.f;
     const bool valid = a < A;
     const float qa = valid ? qb[a] : 0.f, va = valid ? v[a] : 0.f;
@@ -195,25 +244,37 @@ __global__ void __launch_bounds__(ATT_THREADS)
   }
 }
 
+template <typename T, typename TDY>
+static void attn_bwd_launch(int B, int Ts, int H, int Hp, int A, int Ap, const TDY* dy_ctx, long ldy,
+                            const float* dctx_rec, long ldr, const float* pr, float* dp, const float* q,
+                            const float* keys, const float* v, const float* enc, T* dq_op, float* denc, float* dk,
+                            float* dvb, bool first, cudaStream_t st) {
+  launch_pdl(attn_dp_kernel<TDY>, dim3(cdiv(Ts, ATT_THREADS / 32), B), dim3(ATT_THREADS), 0, st, 1, B, Ts, H, Hp,
+             dy_ctx, ldy, dctx_rec, ldr, enc, dp);
+  LAUNCH_CHECK();
+  launch_pdl(attn_bwd_kernel<T, TDY>, dim3(cdiv(std::max(Hp, Ap), ATT_THREADS), B), dim3(ATT_THREADS),
+             (Ts + 8) * sizeof(float), st, 1, B, Ts, H, Hp, A, Ap, dy_ctx, ldy, dctx_rec, ldr, pr, (const float*)dp, q,
+             keys, v, dq_op, denc, dk, dvb, (int)first);
+  LAUNCH_CHECK();
+}
+
 void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
-              const float* dctx_rec, long ldr, const float* pr, const float* q, const float* keys, const float* v,
-              const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first, cudaStream_t st) {
-  const size_t sm = (Hp + Ts + 40) * sizeof(float);
+              const float* dctx_rec, long ldr, const float* pr, float* dpscratch, const float* q, const float* keys,
+              const float* v, const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first,
+              cudaStream_t st) {
+  ASTRA_CHECK_ARG(Hp % 4 == 0 && ((uintptr_t)enc & 15) == 0, "attn_bwd: enc rows must be 16-byte aligned");
   if (ot == OT::BF16) {
     if (dy_f32 || !dy_ctx)
-      launch_pdl(attn_bwd_kernel<__nv_bfloat16, float>, dim3(B), dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy,
-                                                                        dctx_rec, ldr, pr, q, keys, v, enc,
-                                                                        (__nv_bfloat16*)dq_op, denc, dk, dvb, first);
+      attn_bwd_launch<__nv_bfloat16, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, pr,
+                                            dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op, denc, dk, dvb, first, st);
     else
-      launch_pdl(attn_bwd_kernel<__nv_bfloat16, __nv_bfloat16>, dim3(B), dim3(ATT_THREADS), sm, st, 1, 
-          B, Ts, H, Hp, A, Ap, (const __nv_bfloat16*)dy_ctx, ldy, dctx_rec, ldr, pr, q, keys, v, enc,
-          (__nv_bfloat16*)dq_op, denc, dk, dvb, first);
+      attn_bwd_launch<__nv_bfloat16, __nv_bfloat16>(B, Ts, H, Hp, A, Ap, (const __nv_bfloat16*)dy_ctx, ldy, dctx_rec,
+                                                    ldr, pr, dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op, denc,
+                                                    dk, dvb, first, st);
   } else {
-    launch_pdl(attn_bwd_kernel<float, float>, dim3(B), dim3(ATT_THREADS), sm, st, 1, B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy,
-                                                              dctx_rec, ldr, pr, q, keys, v, enc, (float*)dq_op, denc,
-                                                              dk, dvb, first);
+    attn_bwd_launch<float, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, pr, dpscratch, q,
+                                  keys, v, enc, (float*)dq_op, denc, dk, dvb, first, st);
   }
-  LAUNCH_CHECK();
 }
 
 }  // namespace astra

@@ -79,11 +79,14 @@ void reduce_blocked_partials(const float* part, int nchunk, int nq, int H, int H
 void mirror_blocked_T(OT ot, const float* src, int K, int G, int H, int Hp, void* dst, long ldd, cudaStream_t st);
 
 // ---- K3 attention step (attn_kernels.cu): q [B][Ap], keys/enc [Ts][B][Ap|Hp] fp32, pr [B][Ts]
+// escratch / dpscratch: [B][Ts] fp32 (the scores / dp_j between the step's two kernels)
 void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q, const float* keys, const float* v,
-              const float* enc, float* pr, void* ctx_op, long ldc, void* y_ctx, long ldy, cudaStream_t st);
+              const float* enc, float* pr, float* escratch, void* ctx_op, long ldc, void* y_ctx, long ldy,
+              cudaStream_t st);
 void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
-              const float* dctx_rec, long ldr, const float* pr, const float* q, const float* keys, const float* v,
-              const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first, cudaStream_t st);
+              const float* dctx_rec, long ldr, const float* pr, float* dpscratch, const float* q, const float* keys,
+              const float* v, const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first,
+              cudaStream_t st);
 
 // ---- LM pieces
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);

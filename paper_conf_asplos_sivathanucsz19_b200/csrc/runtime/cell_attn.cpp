@@ -26,7 +26,7 @@ class AttnCell : public Cell {
   size_t off_Encf, off_Keys, off_Xd, off_WXd, off_UHd, off_Cd, off_HC, off_Q, off_Pr, off_MWd, off_MUC, off_MWq,
       off_MWk, off_he, off_ce;
   size_t off_DA, off_dHC, off_dC, off_DQ, off_denc, off_DKf, off_DK, off_dvb, off_part, off_dh0e, off_dc0e,
-      off_colsum;
+      off_colsum, off_att;
 
   explicit AttnCell(const astra_cell_desc& dd) : Cell(dd) {
     Ts = d.src_seq;
@@ -86,6 +86,7 @@ class AttnCell : public Cell {
     off_dh0e = c.take((size_t)B * H * 4);
     off_dc0e = c.take((size_t)B * H * 4);
     off_colsum = c.take(colsum_scratch_floats(B, A) * 4);
+    off_att = c.take((size_t)B * Ts * 4);   // attention scores / dp_j between a step's two kernels
     scratch_bytes = c.o;
   }
 
@@ -189,7 +190,7 @@ class AttnCell : public Cell {
                          last ? cT : nullptr, st);
       float* Qi = Q + (long)i * B * Ap;
       run_gemm(3, qg, epi(Qi, Ap, B, Ap), i + 1, 0, var.g[G_REC], st);
-      attn_fwd(ot, B, Ts, H, Hp, A, Ap, Qi, Keys, p("v"), Encf, Pr + (long)i * B * Ts, HC(i + 1) + (size_t)Hp * e,
+      attn_fwd(ot, B, Ts, H, Hp, A, Ap, Qi, Keys, p("v"), Encf, Pr + (long)i * B * Ts, sc<float>(off_att), HC(i + 1) + (size_t)Hp * e,
                2L * Hp, y ? (char*)y + ((size_t)i * B * ldy + H) * e : nullptr, ldy, st);
     }
     mark(R_FWD, 1, st);
@@ -248,7 +249,7 @@ class AttnCell : public Cell {
     for (int i = T - 1; i >= 0; --i) {
       if (i < T - 1) run_gemm(4, bp, epi(dHC, ld2, B, (int)ld2), i + 1, 0, var.g[G_BPTT], st);
       attn_bwd(ot, B, Ts, H, Hp, A, Ap, (const char*)dy + ((size_t)i * B * ldy + H) * e, ldy, false, dHC + Hp, ld2,
-               Pr + (long)i * B * Ts, Q + (long)i * B * Ap, Keys, p("v"), Encf, DQ + (size_t)i * B * Ap * e, denc,
+               Pr + (long)i * B * Ts, sc<float>(off_att), Q + (long)i * B * Ap, Keys, p("v"), Encf, DQ + (size_t)i * B * Ap * e, denc,
                DKf, dvb, i == T - 1, st);
       run_gemm(5, dqw, accum(epi(dHC, ld2, B, Hp)), i, 0, var.g[G_BPTT], st);
       lstm_bwd_pointwise(K_LSTM, ot, B, H, Hp, (const char*)dy + (size_t)i * B * ldy * e, ldy, ot, false, dHC, ld2, 1, 0,
