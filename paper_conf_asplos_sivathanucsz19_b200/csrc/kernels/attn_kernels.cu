@@ -165,16 +165,17 @@ __global__ void __launch_bounds__(ATT_THREADS)
 
 // The rest of one attention step's backward, grid ⌈max(Hp, Ap)/256⌉ × B: every CTA of row b forms
 // de_j = p_j (dp_j − Σ p dp) (warp 0, lane-strided j, fixed xor tree), then thread index x does
-//   hidden unit x:  denc_j += p_j dctx  (read-modify-write in groups of ATT_JG source positions);
-//   width x:        u_j = tanh(q + k_j), du_j = de_j v (1 − u_j²), dq = Σ_j du_j, dk_j += du_j,
-//                   dv_b += Σ_j de_j u_j   (ascending j).
+//   hidden unit x:  saves dctx (the step's dctx row) for the deferred denc accumulation;
+//   width x:        u_j = tanh(q + k_j), du_j = de_j v (1 − u_j²), dq = Σ_j du_j, dv_b += Σ_j de_j u_j
+//                   (ascending j);
+// and the row's de is saved for the deferred dk accumulation (attn_acc_kernel).
 template <typename T, typename TDY>
 __global__ void __launch_bounds__(ATT_THREADS)
     attn_bwd_kernel(int B, int Ts, int H, int Hp, int A, int Ap, const TDY* __restrict__ dy_ctx, long ldy,
                     const float* __restrict__ dctx_rec, long ldr, const float* __restrict__ pr,
                     const float* __restrict__ dpv, const float* __restrict__ q, const float* __restrict__ keys,
-                    const float* __restrict__ v, T* __restrict__ dq_op, float* __restrict__ denc,
-                    float* __restrict__ dk, float* __restrict__ dvb, int first) {
+                    const float* __restrict__ v, T* __restrict__ dq_op, float* __restrict__ dctx_save,
+                    float* __restrict__ de_save, float* __restrict__ dvb, int first) {
   pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
   pdl_trigger();
   extern __shared__ float sh[];
@@ -192,50 +193,31 @@ __global__ void __launch_bounds__(ATT_THREADS)
     for (int j = l; j < Ts; j += 32) de[j] = __fmul_rn(pr[(long)b * Ts + j], __fsub_rn(de[j], s));
   }
   __syncthreads();
-  constexpr int ATT_JG = 10;
+  if (blockIdx.x == 0)
+    for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) de_save[(long)b * Ts + j] = de[j];
   const int x = blockIdx.x * ATT_THREADS + threadIdx.x;
-  if (x < Hp) {   // denc_j += p_j dctx
-    const int h = x;
-    const float dc = attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h, H);
-    for (int j0 = 0; j0 < Ts; j0 += ATT_JG) {
-      float old[ATT_JG];
-#pragma unroll
-      for (int k = 0; k < ATT_JG; ++k)
-        old[k] = (!first && j0 + k < Ts) ? denc[((long)(j0 + k) * B + b) * Hp + h] : 0.f;
-#pragma unroll
-      for (int k = 0; k < ATT_JG; ++k) {
-        if (j0 + k >= Ts) break;
-        const float add = __fmul_rn(pr[(long)b * Ts + j0 + k], dc);
-        denc[((long)(j0 + k) * B + b) * Hp + h] = first ? add : __fadd_rn(old[k], add);
-      }
-    }
-  }
+  if (x < Hp) dctx_save[(long)b * Hp + x] = attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, x, H);
   if (x < Ap) {   // attention-width terms
+    constexpr int JG = 10;
     const int a = x;
     const float* qb = q + (long)b * Ap;
     float dq = 0.f, dva = 0.f;
     const bool valid = a < A;
     const float qa = valid ? qb[a] : 0.f, va = valid ? v[a] : 0.f;
-    for (int j0 = 0; j0 < Ts; j0 += ATT_JG) {
-      float old[ATT_JG], kk[ATT_JG];
+    if (valid) {
+      for (int j0 = 0; j0 < Ts; j0 += JG) {
+        float kk[JG];
 #pragma unroll
-      for (int k = 0; k < ATT_JG; ++k) {
-        const bool in = j0 + k < Ts;
-        old[k] = (!first && in) ? dk[((long)(j0 + k) * B + b) * Ap + a] : 0.f;
-        kk[k] = (valid && in) ? keys[((long)(j0 + k) * B + b) * Ap + a] : 0.f;
-      }
+        for (int k = 0; k < JG; ++k) kk[k] = j0 + k < Ts ? keys[((long)(j0 + k) * B + b) * Ap + a] : 0.f;
 #pragma unroll
-      for (int k = 0; k < ATT_JG; ++k) {
-        const int j = j0 + k;
-        if (j >= Ts) break;
-        float du = 0.f;
-        if (valid) {
+        for (int k = 0; k < JG; ++k) {
+          const int j = j0 + k;
+          if (j >= Ts) break;
           const float u = tanh_<FastMath<T>::value>(__fadd_rn(qa, kk[k]));
-          du = __fmul_rn(__fmul_rn(de[j], va), __fsub_rn(1.f, __fmul_rn(u, u)));
+          const float du = __fmul_rn(__fmul_rn(de[j], va), __fsub_rn(1.f, __fmul_rn(u, u)));
           dq = __fadd_rn(dq, du);
           dva = __fadd_rn(dva, __fmul_rn(de[j], u));
         }
-        dk[((long)j * B + b) * Ap + a] = first ? du : __fadd_rn(old[k], du);
       }
     }
     dq_op[(long)b * Ap + a] = from_f<T>(dq);
@@ -244,36 +226,125 @@ __global__ void __launch_bounds__(ATT_THREADS)
   }
 }
 
+// The encoder-side accumulators over the T decoder steps, after the BPTT loop, in the loop's order
+// (step T−1 first, then T−2, …, 0 — the order the round-1 per-step read-modify-write used):
+//   denc_j,h = Σ_i p_i,j · dctx_i,h               (blockIdx.z == 0, thread per hidden unit h)
+//   dk_j,a   = Σ_i de_i,j · v_a · (1 − u_ij,a²),   u_ij,a = tanh(q_i,a + k_j,a)   (blockIdx.z == 1, per a)
+// Grid ⌈max(Hp, Ap)/256⌉ × B × 2; the row's p / de of every step are staged in shared memory.
+template <typename T>
+__global__ void __launch_bounds__(ATT_THREADS)
+    attn_acc_kernel(int T_, int B, int Ts, int Hp, int A, int Ap, const float* __restrict__ pr,
+                    const float* __restrict__ de_save, const float* __restrict__ dctx_save,
+                    const float* __restrict__ q, const float* __restrict__ keys, const float* __restrict__ v,
+                    float* __restrict__ denc, float* __restrict__ dk) {
+  extern __shared__ float sh[];   // [T][Ts] p (z = 0) or de (z = 1) of row b, then [T][256] per-thread columns
+  const int b = blockIdx.y, z = blockIdx.z;
+  const float* src = z == 0 ? pr : de_save;
+  for (int k = threadIdx.x; k < T_ * Ts; k += ATT_THREADS) {
+    const int i = k / Ts, j = k % Ts;
+    sh[k] = src[((long)i * B + b) * Ts + j];
+  }
+  float* col = sh + T_ * Ts;      // col[i·256 + thread]: this thread's dctx_i (z = 0) or q_i (z = 1)
+  const int x = blockIdx.x * ATT_THREADS + threadIdx.x;
+  const int n = z == 0 ? Hp : Ap;
+  if (x < n)
+    for (int i = 0; i < T_; ++i)
+      col[i * ATT_THREADS + threadIdx.x] =
+          z == 0 ? dctx_save[((long)i * B + b) * Hp + x] : q[((long)i * B + b) * Ap + x];
+  __syncthreads();
+  if (x >= n) return;
+  const float* cx = col + threadIdx.x;
+  // terms of 8 steps are formed independently (instruction-level parallelism), then added in order
+  constexpr int IG = 8;
+  if (z == 0) {
+    for (int j = 0; j < Ts; ++j) {
+      float acc = 0.f;
+      for (int i0 = T_ - 1; i0 >= 0; i0 -= IG) {
+        float t[IG];
+#pragma unroll
+        for (int k = 0; k < IG; ++k) t[k] = i0 - k >= 0 ? __fmul_rn(sh[(i0 - k) * Ts + j], cx[(i0 - k) * ATT_THREADS]) : 0.f;
+#pragma unroll
+        for (int k = 0; k < IG; ++k)
+          if (i0 - k >= 0) acc = i0 - k == T_ - 1 ? t[k] : __fadd_rn(acc, t[k]);
+      }
+      denc[((long)j * B + b) * Hp + x] = acc;
+    }
+  } else {
+    const bool valid = x < A;
+    const float va = valid ? v[x] : 0.f;
+    for (int j = 0; j < Ts; ++j) {
+      const float kj = valid ? keys[((long)j * B + b) * Ap + x] : 0.f;
+      float acc = 0.f;
+      for (int i0 = T_ - 1; i0 >= 0; i0 -= IG) {
+        float t[IG];
+#pragma unroll
+        for (int k = 0; k < IG; ++k) {
+          const int i = i0 - k;
+          float du = 0.f;
+          if (valid && i >= 0) {
+            const float u = tanh_<FastMath<T>::value>(__fadd_rn(cx[i * ATT_THREADS], kj));
+            du = __fmul_rn(__fmul_rn(sh[i * Ts + j], va), __fsub_rn(1.f, __fmul_rn(u, u)));
+          }
+          t[k] = du;
+        }
+#pragma unroll
+        for (int k = 0; k < IG; ++k)
+          if (i0 - k >= 0) acc = i0 - k == T_ - 1 ? t[k] : __fadd_rn(acc, t[k]);
+      }
+      dk[((long)j * B + b) * Ap + x] = acc;
+    }
+  }
+}
+
+void attn_acc(OT ot, int T, int B, int Ts, int Hp, int A, int Ap, const float* pr, const float* de_save,
+              const float* dctx_save, const float* q, const float* keys, const float* v, float* denc, float* dk,
+              cudaStream_t st) {
+  const dim3 grid(cdiv(std::max(Hp, Ap), ATT_THREADS), B, 2);
+  const size_t sm = (size_t)T * (Ts + ATT_THREADS) * sizeof(float);
+  ASTRA_CHECK_ARG(sm <= 200 * 1024, "attn_acc: too many decoder steps for the shared-memory staging");
+  if (ot == OT::BF16) {
+    CUDA_TRY(cudaFuncSetAttribute(attn_acc_kernel<__nv_bfloat16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    attn_acc_kernel<__nv_bfloat16><<<grid, ATT_THREADS, sm, st>>>(T, B, Ts, Hp, A, Ap, pr, de_save, dctx_save, q, keys,
+                                                                  v, denc, dk);
+  } else {
+    CUDA_TRY(cudaFuncSetAttribute(attn_acc_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm));
+    attn_acc_kernel<float><<<grid, ATT_THREADS, sm, st>>>(T, B, Ts, Hp, A, Ap, pr, de_save, dctx_save, q, keys, v, denc,
+                                                          dk);
+  }
+  LAUNCH_CHECK();
+}
+
 template <typename T, typename TDY>
 static void attn_bwd_launch(int B, int Ts, int H, int Hp, int A, int Ap, const TDY* dy_ctx, long ldy,
                             const float* dctx_rec, long ldr, const float* pr, float* dp, const float* q,
-                            const float* keys, const float* v, const float* enc, T* dq_op, float* denc, float* dk,
-                            float* dvb, bool first, cudaStream_t st) {
+                            const float* keys, const float* v, const float* enc, T* dq_op, float* dctx_save,
+                            float* de_save, float* dvb, bool first, cudaStream_t st) {
   launch_pdl(attn_dp_kernel<TDY>, dim3(cdiv(Ts, ATT_THREADS / 32), B), dim3(ATT_THREADS), 0, st, 1, B, Ts, H, Hp,
              dy_ctx, ldy, dctx_rec, ldr, enc, dp);
   LAUNCH_CHECK();
   launch_pdl(attn_bwd_kernel<T, TDY>, dim3(cdiv(std::max(Hp, Ap), ATT_THREADS), B), dim3(ATT_THREADS),
              (Ts + 8) * sizeof(float), st, 1, B, Ts, H, Hp, A, Ap, dy_ctx, ldy, dctx_rec, ldr, pr, (const float*)dp, q,
-             keys, v, dq_op, denc, dk, dvb, (int)first);
+             keys, v, dq_op, dctx_save, de_save, dvb, (int)first);
   LAUNCH_CHECK();
 }
 
 void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
               const float* dctx_rec, long ldr, const float* pr, float* dpscratch, const float* q, const float* keys,
-              const float* v, const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first,
+              const float* v, const float* enc, void* dq_op, float* dctx_save, float* de_save, float* dvb, bool first,
               cudaStream_t st) {
   ASTRA_CHECK_ARG(Hp % 4 == 0 && ((uintptr_t)enc & 15) == 0, "attn_bwd: enc rows must be 16-byte aligned");
   if (ot == OT::BF16) {
     if (dy_f32 || !dy_ctx)
       attn_bwd_launch<__nv_bfloat16, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, pr,
-                                            dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op, denc, dk, dvb, first, st);
+                                            dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op, dctx_save, de_save, dvb,
+                                            first, st);
     else
       attn_bwd_launch<__nv_bfloat16, __nv_bfloat16>(B, Ts, H, Hp, A, Ap, (const __nv_bfloat16*)dy_ctx, ldy, dctx_rec,
-                                                    ldr, pr, dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op, denc,
-                                                    dk, dvb, first, st);
+                                                    ldr, pr, dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op,
+                                                    dctx_save, de_save, dvb, first, st);
   } else {
     attn_bwd_launch<float, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, pr, dpscratch, q,
-                                  keys, v, enc, (float*)dq_op, denc, dk, dvb, first, st);
+                                  keys, v, enc, (float*)dq_op, dctx_save, de_save, dvb, first, st);
   }
 }
 

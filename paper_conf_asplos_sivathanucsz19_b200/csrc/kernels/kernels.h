@@ -83,9 +83,14 @@ void mirror_blocked_T(OT ot, const float* src, int K, int G, int H, int Hp, void
 void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q, const float* keys, const float* v,
               const float* enc, float* pr, float* escratch, void* ctx_op, long ldc, void* y_ctx, long ldy,
               cudaStream_t st);
+// dctx_save: [B][Hp], de_save: [B][Ts] — this step's rows for attn_acc
 void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
               const float* dctx_rec, long ldr, const float* pr, float* dpscratch, const float* q, const float* keys,
-              const float* v, const float* enc, void* dq_op, float* denc, float* dk, float* dvb, bool first,
+              const float* v, const float* enc, void* dq_op, float* dctx_save, float* de_save, float* dvb, bool first,
+              cudaStream_t st);
+// denc / dk ([Ts][B][Hp] / [Ts][B][Ap], overwritten) from the T steps' saved p, de, dctx and q
+void attn_acc(OT ot, int T, int B, int Ts, int Hp, int A, int Ap, const float* pr, const float* de_save,
+              const float* dctx_save, const float* q, const float* keys, const float* v, float* denc, float* dk,
               cudaStream_t st);
 
 // ---- LM pieces

@@ -26,7 +26,7 @@ class AttnCell : public Cell {
   size_t off_Encf, off_Keys, off_Xd, off_WXd, off_UHd, off_Cd, off_HC, off_Q, off_Pr, off_MWd, off_MUC, off_MWq,
       off_MWk, off_he, off_ce;
   size_t off_DA, off_dHC, off_dC, off_DQ, off_denc, off_DKf, off_DK, off_dvb, off_part, off_dh0e, off_dc0e,
-      off_colsum, off_att;
+      off_colsum, off_att, off_dctxs, off_des;
 
   explicit AttnCell(const astra_cell_desc& dd) : Cell(dd) {
     Ts = d.src_seq;
@@ -87,6 +87,8 @@ class AttnCell : public Cell {
     off_dc0e = c.take((size_t)B * H * 4);
     off_colsum = c.take(colsum_scratch_floats(B, A) * 4);
     off_att = c.take((size_t)B * Ts * 4);   // attention scores / dp_j between a step's two kernels
+    off_dctxs = c.take(TB * Hp * 4);        // per-step dctx and de rows for the deferred denc / dk
+    off_des = c.take(TB * Ts * 4);
     scratch_bytes = c.o;
   }
 
@@ -249,14 +251,16 @@ class AttnCell : public Cell {
     for (int i = T - 1; i >= 0; --i) {
       if (i < T - 1) run_gemm(4, bp, epi(dHC, ld2, B, (int)ld2), i + 1, 0, var.g[G_BPTT], st);
       attn_bwd(ot, B, Ts, H, Hp, A, Ap, (const char*)dy + ((size_t)i * B * ldy + H) * e, ldy, false, dHC + Hp, ld2,
-               Pr + (long)i * B * Ts, sc<float>(off_att), Q + (long)i * B * Ap, Keys, p("v"), Encf, DQ + (size_t)i * B * Ap * e, denc,
-               DKf, dvb, i == T - 1, st);
+               Pr + (long)i * B * Ts, sc<float>(off_att), Q + (long)i * B * Ap, Keys, p("v"), Encf, DQ + (size_t)i * B * Ap * e,
+               sc<float>(off_dctxs) + (long)i * B * Hp, sc<float>(off_des) + (long)i * B * Ts, dvb, i == T - 1, st);
       run_gemm(5, dqw, accum(epi(dHC, ld2, B, Hp)), i, 0, var.g[G_BPTT], st);
       lstm_bwd_pointwise(K_LSTM, ot, B, H, Hp, (const char*)dy + (size_t)i * B * ldy * e, ldy, ot, false, dHC, ld2, 1, 0,
                          dC, WXd + (long)i * B * NG, UHd + (long)i * B * NG, Cd + (long)(i + 1) * B * Hp,
                          Cd + (long)i * B * Hp, gp, DA + (size_t)i * B * NG * e, DA + (size_t)i * B * NG * e, part, 1,
                          i == T - 1, st);
     }
+    // encoder-side attention accumulators over the T steps (same per-element order as per-step updates)
+    attn_acc(ot, T, B, Ts, Hp, A, Ap, Pr, sc<float>(off_des), sc<float>(off_dctxs), Q, Keys, p("v"), denc, DKf, st);
     // decoder initial-state gradient → encoder final-state gradient
     run_gemm(4, bp, epi(dHC, ld2, B, (int)ld2), 0, 0, var.g[G_BPTT], st);
     copy_pad(OT::F32, dHC, OT::F32, B, H, ld2, dh0e, H, st);
