@@ -66,8 +66,61 @@ __global__ void mirror_gates_T2_kernel(const float* __restrict__ src, int K, int
   }
 }
 
+// Same mapping, tile = one 64-unit gate block (64 internal rows) x 64 k: float4 loads of the 64
+// consecutive source columns g·H + j0 … (H % 4 == 0), 4 consecutive k per thread on the store side.
+template <typename T>
+__global__ void __launch_bounds__(256) mirror_gates_T4_kernel(const float* __restrict__ src, int K, int H, int Hp,
+                                                              T* __restrict__ dst, long ldd, long kcols) {
+  __shared__ float tile[64][65];
+  const int rb = blockIdx.x, k0 = blockIdx.y * 64, tid = threadIdx.x;
+  const int tileu = rb / 4, g = rb % 4, r0 = rb * 64, j0 = tileu * GATE_U;
+#pragma unroll
+  for (int jj = 0; jj < 4; ++jj) {
+    const int kl = tid / 16 + 16 * jj, q = tid % 16, k = k0 + kl, j = j0 + 4 * q;
+    float4 x = make_float4(0.f, 0.f, 0.f, 0.f);
+    if (k < K && j < H) x = *reinterpret_cast<const float4*>(src + (long)k * 4 * H + (long)g * H + j);
+    tile[kl][4 * q] = x.x;
+    tile[kl][4 * q + 1] = x.y;
+    tile[kl][4 * q + 2] = x.z;
+    tile[kl][4 * q + 3] = x.w;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int jj = 0; jj < 4; ++jj) {
+    const int nl = tid / 16 + 16 * jj, q = tid % 16, r = r0 + nl, k = k0 + 4 * q;
+    if (r >= 4 * Hp || k >= kcols) continue;
+    T* d = dst + (long)r * ldd + k;
+    if (k + 4 <= kcols) {
+      if constexpr (sizeof(T) == 2) {
+        __nv_bfloat162 lo = __floats2bfloat162_rn(tile[4 * q][nl], tile[4 * q + 1][nl]);
+        __nv_bfloat162 hi = __floats2bfloat162_rn(tile[4 * q + 2][nl], tile[4 * q + 3][nl]);
+        uint2 u;
+        u.x = *reinterpret_cast<uint32_t*>(&lo);
+        u.y = *reinterpret_cast<uint32_t*>(&hi);
+        *reinterpret_cast<uint2*>(d) = u;
+      } else {
+        *reinterpret_cast<float4*>(d) =
+            make_float4(tile[4 * q][nl], tile[4 * q + 1][nl], tile[4 * q + 2][nl], tile[4 * q + 3][nl]);
+      }
+    } else {
+      for (int i = 0; k + i < kcols; ++i) d[i] = from_f<T>(tile[4 * q + i][nl]);
+    }
+  }
+}
+
 void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st, long kcols) {
   if (kcols < 0) kcols = ldd;
+  const size_t e = ot == OT::BF16 ? 2 : 4;
+  if (H % 4 == 0 && ldd % 4 == 0 && Hp % GATE_U == 0 && ((uintptr_t)src & 15) == 0 &&
+      ((uintptr_t)dst & (4 * e - 1)) == 0) {
+    dim3 grid(4 * Hp / 64, cdiv(kcols, 64));
+    if (ot == OT::BF16)
+      mirror_gates_T4_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
+    else
+      mirror_gates_T4_kernel<float><<<grid, 256, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols);
+    LAUNCH_CHECK();
+    return;
+  }
   if (kcols % 2 == 0 && ldd % 2 == 0) {
     dim3 grid(cdiv(4L * Hp, 32), cdiv(kcols, 64)), block(32, 8);
     if (ot == OT::BF16)
