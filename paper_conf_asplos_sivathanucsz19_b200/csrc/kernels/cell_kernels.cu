@@ -1075,7 +1075,9 @@ void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targ
                 float* rowloss, void* dlog, long ldd, float* dlog32, cudaStream_t st, const int* nvp, long row0) {
   if (n == 0) return;
   const size_t e = ot == OT::BF16 ? 2 : 4;
-  const bool vec = V % 4 == 0 && ldl % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)logits & 15) == 0 &&
+  // one CTA per row pays off for wide rows only (cfg2/cfg3, V = 10k: 75 -> 25 µs per chunk); at V = 256
+  // (cfg5) most of its threads would idle and a warp per row is faster (33 vs 112 µs per step)
+  const bool vec = V >= 2048 && V % 4 == 0 && ldl % 4 == 0 && ldd % 4 == 0 && ((uintptr_t)logits & 15) == 0 &&
                    ((uintptr_t)dlog & (4 * e - 1)) == 0 && ((uintptr_t)dlog32 & 15) == 0;
   if (vec) {
     ASTRA_CHECK_ARG(n < (1L << 31), "ce_fwd_bwd: too many rows");
@@ -1200,23 +1202,20 @@ __global__ void emb_count_kernel(const int32_t* __restrict__ tok, long n, long b
   }
 }
 
-// tot[v] = Σ_b cnt[b][v]; nseg[v] = ⌈tot[v] / EMB_SEG⌉ (written to lo / segoff, scanned next)
+// tot[v] = Σ_b cnt[b][v]; nseg[v] = ⌈tot[v] / EMB_SEG⌉ (written to lo / segoff, scanned next).
+// One warp per token: lanes take 32 consecutive blocks at a time (integer sums: exact in any order).
 __global__ void emb_total_kernel(const int32_t* __restrict__ cnt, long nblk, int V, int32_t* __restrict__ lo,
                                  int32_t* __restrict__ segoff) {
-  const int v = blockIdx.x * blockDim.x + threadIdx.x;
+  const int v = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
   if (v >= V) return;
   int tot = 0;
-  long b = 0;
-  for (; b + 8 <= nblk; b += 8) {
-    int c[8];
+  for (long b = lane; b < nblk; b += 32) tot += cnt[b * V + v];
 #pragma unroll
-    for (int k = 0; k < 8; ++k) c[k] = cnt[(b + k) * V + v];
-#pragma unroll
-    for (int k = 0; k < 8; ++k) tot += c[k];
+  for (int o = 16; o; o >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, o);
+  if (lane == 0) {
+    lo[v] = tot;
+    segoff[v] = (tot + EMB_SEG - 1) / EMB_SEG;
   }
-  for (; b < nblk; ++b) tot += cnt[b * V + v];
-  lo[v] = tot;
-  segoff[v] = (tot + EMB_SEG - 1) / EMB_SEG;
 }
 
 // One CTA: in-place exclusive scans of lo[0..V) and segoff[0..V), totals into lo[V] / segoff[V];
@@ -1272,26 +1271,23 @@ __global__ void __launch_bounds__(1024) emb_scan_kernel(int V, int32_t* __restri
   if (tid == 0) { lo[V] = carry[0]; segoff[V] = carry[1]; }
 }
 
-// cnt[b][v] ← lo_v + Σ_{b' < b} cnt[b'][v]: the first sorted position of block b's rows of token v
+// cnt[b][v] ← lo_v + Σ_{b' < b} cnt[b'][v]: the first sorted position of block b's rows of token v.
+// One warp per token: an exclusive warp scan over 32 consecutive blocks at a time, carried.
 __global__ void emb_cursor_kernel(int32_t* __restrict__ cnt, long nblk, int V, const int32_t* __restrict__ lo) {
-  const int v = blockIdx.x * blockDim.x + threadIdx.x;
+  const int v = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
   if (v >= V) return;
   int run = lo[v];
-  long b = 0;
-  for (; b + 8 <= nblk; b += 8) {
-    int c[8];
+  for (long b0 = 0; b0 < nblk; b0 += 32) {
+    const long b = b0 + lane;
+    const int c = b < nblk ? cnt[b * V + v] : 0;
+    int incl = c;
 #pragma unroll
-    for (int k = 0; k < 8; ++k) c[k] = cnt[(b + k) * V + v];
-#pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      cnt[(b + k) * V + v] = run;
-      run += c[k];
+    for (int d = 1; d < 32; d <<= 1) {
+      const int x = __shfl_up_sync(0xffffffffu, incl, d);
+      if (lane >= d) incl += x;
     }
-  }
-  for (; b < nblk; ++b) {
-    const int c = cnt[b * V + v];
-    cnt[b * V + v] = run;
-    run += c;
+    if (b < nblk) cnt[b * V + v] = run + incl - c;
+    run += __shfl_sync(0xffffffffu, incl, 31);
   }
 }
 
@@ -1382,7 +1378,15 @@ __global__ void emb_seg_final_kernel(int V, const int32_t* __restrict__ segoff, 
   const int v = (int)(q / iw), c = (int)(q % iw) * W;
   const int s0 = segoff[v], s1 = segoff[v + 1];
   VT acc = emb_zero<W>();
-  for (int s = s0; s < s1; ++s) emb_acc(acc, *reinterpret_cast<const VT*>(part + (long)s * I + c));
+  int s = s0;
+  for (; s + 8 <= s1; s += 8) {   // 8 loads in flight, then the ordered adds (same sum)
+    VT x[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) x[k] = *reinterpret_cast<const VT*>(part + (long)(s + k) * I + c);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) emb_acc(acc, x[k]);
+  }
+  for (; s < s1; ++s) emb_acc(acc, *reinterpret_cast<const VT*>(part + (long)s * I + c));
   *reinterpret_cast<VT*>(dE + (long)v * I + c) = acc;
 }
 
@@ -1408,11 +1412,11 @@ void embed_bwd(const int32_t* tok, long n, int V, const float* dX, long ldx, int
   CUDA_TRY(cudaMemsetAsync(cnt, 0, (size_t)nblk * V * 4, st));
   emb_count_kernel<<<(unsigned)nblk, 256, 0, st>>>(tok, n, blk, V, cnt);
   LAUNCH_CHECK();
-  emb_total_kernel<<<cdiv(V, 256), 256, 0, st>>>(cnt, nblk, V, lo, segoff);
+  emb_total_kernel<<<cdiv(V, 8), 256, 0, st>>>(cnt, nblk, V, lo, segoff);
   LAUNCH_CHECK();
   emb_scan_kernel<<<1, 1024, 0, st>>>(V, lo, segoff);
   LAUNCH_CHECK();
-  emb_cursor_kernel<<<cdiv(V, 256), 256, 0, st>>>(cnt, nblk, V, lo);
+  emb_cursor_kernel<<<cdiv(V, 8), 256, 0, st>>>(cnt, nblk, V, lo);
   LAUNCH_CHECK();
   emb_scatter_kernel<<<(unsigned)nblk, 32, 0, st>>>(tok, n, blk, V, cnt, srows);
   LAUNCH_CHECK();
