@@ -256,28 +256,56 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
                       int nsplit, long split_stride, const TDY* __restrict__ dy, long ldy,
                       const float* __restrict__ Apre, const float* __restrict__ s_prev, T* __restrict__ DA,
                       float* __restrict__ ds_out, float* __restrict__ part, int first) {
-  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
-  pdl_trigger();
+  constexpr int NR = PW_RB / PW_RY;   // rows per thread: b0 + ty, b0 + ty + PW_RY, … (in this order)
   __shared__ float red[PW_RY][2][PW_UX];
   const int ux = threadIdx.x, ty = threadIdx.y;
   const int j = blockIdx.x * PW_UX + ux;
   const int chunk = blockIdx.y;
   const int b0 = chunk * PW_RB, b1 = min(B, b0 + PW_RB);
+  const bool unit = j < H;
+  // every operand of the thread's rows is loaded before the arithmetic (one memory latency, not NR);
+  // the saved forward tensors, dy and the carry are older than the grid dependency: loaded before
+  // it, except at the first micro-step (ds_part == null), whose predecessor initialised the carry
+  float aH[NR], aT[NR], sp[NR], dsv[NR], dyv[NR];
+  auto load_old = [&] {
+#pragma unroll
+    for (int k = 0; k < NR; ++k) {
+      const int b = b0 + ty + k * PW_RY;
+      const bool ok = unit && b < b1;
+      const long rz = (long)b * 2 * Hp;
+      aH[k] = ok ? Apre[rz + j] : 0.f;
+      aT[k] = ok ? Apre[rz + Hp + j] : 0.f;
+      sp[k] = ok ? s_prev[(long)b * Hp + j] : 0.f;
+      dsv[k] = ok ? ds_in[(long)b * Hp + j] : 0.f;
+      dyv[k] = (ok && dy) ? to_f<TDY>(dy[(long)b * ldy + j]) : 0.f;
+    }
+  };
+  const bool early = ds_part != nullptr;
+  if (early) load_old();
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
+  if (!early) load_old();
+  float pz[NR];   // the BPTT GEMM's split-K partials (this launch's dependency), summed in chunk order
+#pragma unroll
+  for (int k = 0; k < NR; ++k) {
+    const int b = b0 + ty + k * PW_RY;
+    pz[k] = (ds_part && unit && b < b1) ? sum_split(ds_part + (long)b * Hp + j, nsplit, split_stride) : 0.f;
+  }
   float sH = 0.f, sT_ = 0.f;
   if (j < Hp) {
-    for (int b = b0 + ty; b < b1; b += PW_RY) {
+#pragma unroll
+    for (int k = 0; k < NR; ++k) {
+      const int b = b0 + ty + k * PW_RY;
+      if (b >= b1) break;
       const long rz = (long)b * 2 * Hp;
       float daH = 0.f, daT = 0.f, dso = 0.f;
-      if (j < H) {
-        float ds = ds_in[(long)b * Hp + j];
-        if (ds_part) {   // reading R33: carry + the BPTT GEMM's split-K partials summed in chunk order
-          ds = __fadd_rn(ds, sum_split(ds_part + (long)b * Hp + j, nsplit, split_stride));
-        }
-        if (dy) ds = __fadd_rn(to_f<TDY>(dy[(long)b * ldy + j]), ds);
-        const float h = tanh_<FastMath<T>::value>(Apre[rz + j]), tau = sigm<FastMath<T>::value>(Apre[rz + Hp + j]);
-        const float sp = s_prev[(long)b * Hp + j];
+      if (unit) {
+        float ds = dsv[k];
+        if (ds_part) ds = __fadd_rn(ds, pz[k]);   // reading R33: carry + the partials in chunk order
+        if (dy) ds = __fadd_rn(dyv[k], ds);
+        const float h = tanh_<FastMath<T>::value>(aH[k]), tau = sigm<FastMath<T>::value>(aT[k]);
         const float dh = __fmul_rn(ds, tau);
-        const float dtau = __fmul_rn(ds, __fsub_rn(h, sp));
+        const float dtau = __fmul_rn(ds, __fsub_rn(h, sp[k]));
         daH = __fmul_rn(dh, __fsub_rn(1.f, __fmul_rn(h, h)));
         daT = __fmul_rn(__fmul_rn(dtau, tau), __fsub_rn(1.f, tau));
         dso = __fmul_rn(ds, __fsub_rn(1.f, tau));
