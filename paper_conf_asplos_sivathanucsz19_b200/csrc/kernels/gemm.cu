@@ -151,7 +151,7 @@ static int smem_for(int& stages, int cap) {
 }
 
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
-                     int cm, int cn, bool b_keep, int ksplit, int cg, int smem_cap) {
+                     int cm, int cn, bool b_keep, int ksplit, int cg, int smem_cap, bool plain_maps) {
   // BN = 224 (74 CTA pairs fill all 148 SMs on an 8192-column chain GEMM instead of 64 pairs of 256)
   // exists only for CTA pairs with a K-major B (each CTA holds 112 B rows); elsewhere the same tile
   // width is run as 256 — same bits (R1: every output element is one accumulation over K)
@@ -162,8 +162,59 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
                   "tc_gemm: cluster shape must be cm, cn in {1,2,4}, cm*cn <= 8");
   ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256 || BN == 224, "tc_gemm: BN must be 64, 128, 224 or 256");
   ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
-  if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
-  if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm / cg);
+  // multi-k-block stages (TcArgs::kb; tc_gemm_kernel without a cluster): the largest of 4 / 2 that
+  // divides the per-chunk k-block count and still leaves >= 3 stages; K-major operands need K % 64 == 0
+  // (their 4-D view reads whole 64-element k-blocks)
+  int KB = 1;
+  {
+    static const int kb_env = [] {
+      const char* e = std::getenv("ASTRA_GEMM_KB");   // A/B runs: 1 disables
+      return e ? std::atoi(e) : 0;
+    }();
+    const int nk_all = cdiv(K, TC_BK), kper = cdiv(nk_all, ksplit);
+    const bool kmaj_ok = (a_mn || K % TC_BK == 0) && (b_mn || K % TC_BK == 0);
+    if (cg == 1 && cm * cn == 1 && kmaj_ok && kb_env != 1 && !plain_maps) {
+      int dev = 0, maxs = 0;
+      CUDA_TRY(cudaGetDevice(&dev));
+      CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+      if (smem_cap > 0 && smem_cap < maxs) maxs = smem_cap;
+      for (int kb : {4, 2}) {
+        if (kb_env > 1 && kb != kb_env) continue;
+        const int a_kb = a_mn ? TC_BM * TC_BK * 2 : ((M <= 64 ? 64 : TC_BM) * TC_BK * 2);
+        const int sb = kb * (a_kb + BN * TC_BK * 2);
+        const int epi_bytes = TC_EPI_WARPS * 2 * 32 * 32 * 4;
+        const int st = std::min(10, (maxs - 1024 - 256 - epi_bytes) / sb);
+        if (kper % kb == 0 && st >= 3) {
+          KB = kb;
+          break;
+        }
+      }
+    }
+  }
+  const int a_rows = (KB > 1 && !a_mn && M <= 64) ? 64 : TC_BM;
+  if (KB > 1) {
+    if (a_mn) {
+      make_map(&g.mapA, A, 64, 64 * KB);
+    } else {
+      const long dims[4] = {64, A.outer, A.inner / 64, A.z};
+      const long str[3] = {A.ld * 2, 128, (A.z > 1 ? A.zstride : A.ld * A.outer) * 2};
+      const int box[4] = {64, a_rows, KB, 1};
+      make_map_nd(&g.mapA, A.ptr, 4, dims, str, box, 128);
+    }
+    if (b_mn) {
+      make_map(&g.mapB, B, 64, 64 * KB);
+    } else {
+      const long dims[4] = {64, B.outer, B.inner / 64, B.z};
+      const long str[3] = {B.ld * 2, 128, (B.z > 1 ? B.zstride : B.ld * B.outer) * 2};
+      const int box[4] = {64, BN, KB, 1};
+      make_map_nd(&g.mapB, B.ptr, 4, dims, str, box, 128);
+    }
+  } else {
+    if (a_mn) make_map(&g.mapA, A, 64, 64 / cn); else make_map(&g.mapA, A, 64, TC_BM / cn);
+    if (b_mn) make_map(&g.mapB, B, 64, 64 / cm); else make_map(&g.mapB, B, 64, BN / cm / cg);
+  }
+  g.args.kb = KB;
+  g.args.a_rows = a_rows;
   g.args.pf = L2Pf{};
   g.args.cg = cg;
   static const int gm_env = [] {
@@ -189,6 +240,17 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
     case 112: g.smem = smem_for<112>(stages, smem_cap); break;
     case 128: g.smem = smem_for<128>(stages, smem_cap); break;
     default: g.smem = smem_for<256>(stages, smem_cap); break;
+  }
+  if (KB > 1) {   // stages of KB k-blocks (A tiles of a_rows rows)
+    int dev = 0, maxs = 0;
+    CUDA_TRY(cudaGetDevice(&dev));
+    CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    if (smem_cap > 0 && smem_cap < maxs) maxs = smem_cap;
+    const int a_kb = a_mn ? TC_BM * TC_BK * 2 : a_rows * TC_BK * 2;
+    const int sb = KB * (a_kb + BN * TC_BK * 2);
+    const int epi_bytes = TC_EPI_WARPS * 2 * 32 * 32 * 4;
+    stages = std::min(10, (maxs - 1024 - 256 - epi_bytes) / sb);
+    g.smem = 1024 + stages * sb + epi_bytes + 256;
   }
   g.args.stages = stages;
   g.ready = true;

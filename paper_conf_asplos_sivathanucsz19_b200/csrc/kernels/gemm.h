@@ -30,8 +30,11 @@ struct TcGemm {
 
 // D[M,N] = A·B.  A is [M,K]: K-major ⇒ storage rows = M, inner = K; MN-major ⇒ storage rows =
 // K, inner = M.  B is [K,N]: K-major ⇒ storage rows = N, inner = K; MN-major ⇒ rows = K, inner = N.
+// plain_maps: one-k-block tensor maps (TcArgs::kb = 1) — for callers that hand g.mapA / g.mapB to
+// another kernel (the fused recurrent / BPTT kernels load single k-block boxes through them).
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
-                     int cm = 1, int cn = 1, bool b_keep = false, int ksplit = 1, int cg = 1, int smem_cap = 0);
+                     int cm = 1, int cn = 1, bool b_keep = false, int ksplit = 1, int cg = 1, int smem_cap = 0,
+                     bool plain_maps = false);
 // Launch with the given z-coordinates (time slices) and epilogue; grid ≤ #SMs (persistent).
 void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas = 0,
                     const L2Pf* pf = nullptr);

@@ -65,6 +65,14 @@ struct TcArgs {
   int cg;           // 1: one CTA per 128 x BN tile; 2: CTA pair per 256 x BN tile (tc_gemm2_kernel)
   int gm;           // raster group: tiles walk gm M-tiles of one N column before the next column
   uint32_t idesc;
+  // tc_gemm_kernel without a cluster: kb k-blocks per pipeline stage, loaded by ONE tensor-map box
+  // per operand (K-major: a 4-D map whose k-block dimension has a 128-byte stride; MN-major: a box
+  // 64·kb K-rows tall) — a CTA's TMA unit retires ~1 box per 128 ns however small it is
+  // (profiles/r2_tma_micro.jsonl), which bounds the small-M chain GEMMs; a_rows: rows of the K-major
+  // A box (64 when M ≤ 64: the MMA's rows 64..127 read stale shared memory and are never stored).
+  // The pair kernel (tc_gemm2) ignores both (kb = 1, a_rows = 128).
+  int kb;
+  int a_rows;
 };
 
 // One warp of every CTA issues its slice of the prefetch ranges (cp.async.bulk.prefetch.L2, 16-byte
@@ -296,8 +304,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   if (threadIdx.x == 0) GEMM_TRACE(0);
   const int stages = args.stages;
-  const uint32_t epi_tiles = sm100::smem_u32(smem + stages * S::STAGE_BYTES);   // 1024-aligned
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * S::STAGE_BYTES + S::EPI_BYTES);
+  const int KB = args.kb;
+  // per k-block: A tile (K-major: a_rows x 128 B; MN-major: two 64-wide halves x 64 K-rows), B tile
+  const int a_kb_bytes = args.a_mn ? S::A_BYTES : args.a_rows * TC_BK * 2;
+  const int stage_bytes = KB * (a_kb_bytes + S::B_BYTES);
+  const uint32_t epi_tiles = sm100::smem_u32(smem + stages * stage_bytes);   // 1024-aligned
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + stages * stage_bytes + S::EPI_BYTES);
   uint64_t* empty = full + stages;
   uint64_t* tfull = empty + stages;   // [2]
   uint64_t* tempty = tfull + 2;       // [2]
@@ -362,13 +374,30 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         const int m0 = (mi * cm + rm) * TC_BM;
         const int n0 = (ni * cn + rn) * BN;
         const int kb0 = ks * kper, kb1 = min(nk_all, kb0 + kper);
-        for (int kb = kb0; kb < kb1; ++kb) {
+        for (int kb = kb0; kb < kb1; kb += KB) {
           sm100::mbar_wait(&empty[s], ph ^ 1);
-          uint8_t* sa = smem + s * S::STAGE_BYTES;
-          uint8_t* sb = sa + S::A_BYTES;
-          sm100::mbar_arrive_expect_tx(&full[s], S::STAGE_BYTES);
+          uint8_t* sa = smem + s * stage_bytes;
+          uint8_t* sb = sa + KB * a_kb_bytes;
+          sm100::mbar_arrive_expect_tx(&full[s], stage_bytes);
           const int k0 = kb * TC_BK;
-          if (cs == 1) {
+          if (KB > 1) {   // (cs == 1) one box per operand for the KB k-blocks of the stage
+            if (args.a_mn) {
+              sm100::tma_load_3d(sa, &mapA, &full[s], m0, k0, args.az);
+              sm100::tma_load_3d(sa + KB * 8192, &mapA, &full[s], m0 + 64, k0, args.az);
+            } else {
+              sm100::tma_load_4d(sa, &mapA, &full[s], 0, m0, kb, args.az);
+            }
+            if (args.b_mn) {
+#pragma unroll
+              for (int j = 0; j < BN / 64; ++j) {
+                if (args.b_keep) sm100::tma_load_3d_hint(sb + j * KB * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz, pol);
+                else sm100::tma_load_3d(sb + j * KB * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+              }
+            } else {
+              if (args.b_keep) sm100::tma_load_4d_hint(sb, &mapB, &full[s], 0, n0, kb, args.bz, pol);
+              else sm100::tma_load_4d(sb, &mapB, &full[s], 0, n0, kb, args.bz);
+            }
+          } else if (cs == 1) {
             if (args.a_mn) {
               sm100::tma_load_3d(sa, &mapA, &full[s], m0, k0, args.az);
               sm100::tma_load_3d(sa + 8192, &mapA, &full[s], m0 + 64, k0, args.az);
@@ -423,10 +452,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
       // shared-memory descriptors of stage 0, advanced by adding (bytes >> 4) to the address field
       // (no carry: addresses < 256 KB): the single issuing thread's scalar work per k-block stays
       // far below one MMA — at the small-N per-step GEMMs it otherwise bounds the k-loop
-      const uint32_t sa0 = sm100::smem_u32(smem), sb0 = sa0 + S::A_BYTES;
-      const uint64_t dA0 = args.a_mn ? sm100::smem_desc_sw128(sa0, 8192, 1024) : sm100::smem_desc_sw128(sa0, 16, 1024);
-      const uint64_t dB0 = args.b_mn ? sm100::smem_desc_sw128(sb0, 8192, 1024) : sm100::smem_desc_sw128(sb0, 16, 1024);
+      const uint32_t sa0 = sm100::smem_u32(smem), sb0 = sa0 + KB * a_kb_bytes;
+      // MN-major: the 64-wide halves of a stage's tile are KB·8 KB apart (LBO)
+      const uint64_t dA0 = args.a_mn ? sm100::smem_desc_sw128(sa0, 8192 * KB, 1024) : sm100::smem_desc_sw128(sa0, 16, 1024);
+      const uint64_t dB0 = args.b_mn ? sm100::smem_desc_sw128(sb0, 8192 * KB, 1024) : sm100::smem_desc_sw128(sb0, 16, 1024);
       const uint32_t a_kk = args.a_mn ? (2048 >> 4) : (32 >> 4), b_kk = args.b_mn ? (2048 >> 4) : (32 >> 4);
+      // k-block j of a stage: K-major + j tiles; MN-major + j·64 K-rows (8 KB)
+      const uint32_t a_j = (uint32_t)(args.a_mn ? 8192 : a_kb_bytes) >> 4, b_j = (uint32_t)(args.b_mn ? 8192 : S::B_BYTES) >> 4;
       const uint32_t idesc = args.idesc;
       for (int ct = cluster_id; ct < num_ct; ct += num_clusters, ++local) {
         const int acc = local & 1;
@@ -435,14 +467,17 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
         sm100::tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
         const int kb0 = (ct / num_ct1) * kper, kb1 = min(nk_all, kb0 + kper);
-        for (int kb = kb0; kb < kb1; ++kb) {
+        for (int kb = kb0; kb < kb1; kb += KB) {
           sm100::mbar_wait(&full[s], ph);
           if (kb == kb0 && local == 0) GEMM_TRACE(3);
           sm100::tc_fence_after();
-          const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
+          const uint64_t ad0 = dA0 + (uint64_t)(s * (stage_bytes >> 4)), bd0 = dB0 + (uint64_t)(s * (stage_bytes >> 4));
+          for (int j = 0; j < KB; ++j) {
+            const uint64_t ad = ad0 + j * a_j, bd = bd0 + j * b_j;
 #pragma unroll
-          for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
+            for (int kk = 0; kk < TC_BK / 16; ++kk)
+              sm100::umma_bf16(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb + j != kb0 || kk != 0) ? 1u : 0u);
+          }
           if (cs == 1) sm100::umma_commit(&empty[s]);
           else sm100::umma_commit_mc(&empty[s], mask_nb);
           if (++s == stages) { s = 0; ph ^= 1; }

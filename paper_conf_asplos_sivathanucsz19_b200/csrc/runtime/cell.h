@@ -149,7 +149,7 @@ class Cell {
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
   // prepared GEMMs keyed by (gemm id, T, bn, cm, cn, cg, A, B, M, N, K): the tensor maps carry the
   // operand pointers and extents, so two row ranges of one role never share an entry
-  using TcKey = std::tuple<int, int, int, int, int, int, const void*, const void*, int, int, int>;
+  using TcKey = std::tuple<int, int, int, int, int, int, const void*, const void*, int, int, int, bool>;
   std::map<TcKey, TcGemm> tc_cache;
 
   // Bucketed profiling: one independent exploration per active length T, the
@@ -239,7 +239,8 @@ class Cell {
   template <typename T_> T_* sc(size_t off) { return reinterpret_cast<T_*>(scratch + off); }
   void run_gemm(int id, const GemmSpec& s, const EpiStore& e, int az, int bz, const KCfg& k, cudaStream_t st,
                 const L2Pf* pf = nullptr, int max_ctas = 0);
-  TcGemm& tc_get(int id, const GemmSpec& s, const KCfg& k);   // prepared tensor maps (bf16 path)
+  // prepared tensor maps (bf16 path); plain_maps: single-k-block maps for the fused kernels
+  TcGemm& tc_get(int id, const GemmSpec& s, const KCfg& k, bool plain_maps = false);
   void mark(Region r, int which, cudaStream_t st);
   void tuner_setup();
   void apply_config(const tuner::Config& c);

@@ -219,10 +219,10 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
   if (which && r == R_STEP) last_step_slot = ev_slot;
 }
 
-TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
+TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k, bool plain_maps) {
   // split-K only runs without clusters; the cluster choice then falls back to 1x1 (same numerics)
   const int cm = s.ksplit > 1 ? 1 : k.cm, cn = s.ksplit > 1 ? 1 : k.cn;
-  const TcKey key{id, T, k.bn, cm, cn, k.cg, s.A.ptr, s.B.ptr, s.M, s.N, s.K};
+  const TcKey key{id, T, k.bn, cm, cn, k.cg, s.A.ptr, s.B.ptr, s.M, s.N, s.K, plain_maps};
   auto it = tc_cache.find(key);
   if (it == tc_cache.end()) {
     TcGemm g;
@@ -238,7 +238,7 @@ TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k) {
       return e ? std::atoi(e) * 1024 : 0;
     }();
     tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit, k.cg,
-                    id == 2 ? bptt_cap : id == 1 ? rec_cap : 0);
+                    id == 2 ? bptt_cap : id == 1 ? rec_cap : 0, plain_maps);
     it = tc_cache.emplace(key, g).first;
   }
   return it->second;

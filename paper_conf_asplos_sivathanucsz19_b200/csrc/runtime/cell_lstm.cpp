@@ -215,7 +215,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   rec.b_keep = true;
   if (ot == OT::BF16 && var.fwd_mode == 1 && !y_f32) {
     // K2 fused, CTA-pair form: GEMM + gate epilogue with TMA-staged epilogue I/O, one launch per step
-    const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1, 2});
+    const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1, 2}, true);
     if (fm_key != (const void*)y || fm_wx != (const void*)WX || fm_T != T) {
       fm.A = tg.mapA;
       fm.B = tg.mapB;
@@ -260,7 +260,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     for (int t = t0; t < t1; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
   } else if (ot == OT::BF16 && var.fwd_mode > 0 && var.fwd_mode < 3) {
     // K2 fused: GEMM + gate epilogue in one kernel (per step, or persistent over all steps)
-    const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1});
+    const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1}, true);
     RecFwdArgs ra;
     ra.B = B; ra.H = H; ra.Hp = Hp; ra.NG = NG; ra.T = T;
     ra.num_m = cdiv(B, TC_BM); ra.num_n = NG / 256;
@@ -382,7 +382,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   const bool persist = !fuse && var.bwd_mode >= 2 && whole && var.recomp == 0 && bptt_persist_ok();
   BpttFusedArgs fa{};
   if (fuse) {
-    const TcGemm& tg = tc_get(2, bp, KCfg{64, 1, 1});
+    const TcGemm& tg = tc_get(2, bp, KCfg{64, 1, 1}, true);
     const void* key[4] = {WX, lm_dy ? (const void*)lm_dy : dy, Duh, (const void*)(uintptr_t)T};
     if (std::memcmp(key, bm_key, sizeof(key)) != 0) {
       bm.A = tg.mapA;

@@ -134,7 +134,7 @@ class RhnCell : public Cell {
     EpiStore ez = epi(Zpart, G2, B, G2);
     ez.split_stride = (long)B * G2;
     if (var.fwd_mode >= 1 && fused_fwd_ok()) {   // persistent fused chain: one launch for all T·L micro-steps
-      const TcGemm& g64 = tc_get(1, rec, KCfg{64, 1, 1});   // for the M = 128, N = 64 instruction descriptor
+      const TcGemm& g64 = tc_get(1, rec, KCfg{64, 1, 1}, true);   // for the M = 128, N = 64 instruction descriptor
       RhnFwdArgs ra{};
       ra.B = B; ra.H = H; ra.Hp = Hp; ra.T = T; ra.L = L; ra.t0 = 0; ra.t1 = T;
       ra.nsplit = rec.ksplit;

@@ -12,9 +12,16 @@ def run(M, N, K, a_mn, b_mn, cfgs, tag):
             f = lambda: A.gemm_bf16_ex(a, b, M, N, K, a_mn=a_mn, b_mn=b_mn, bn=bn, cm=cm, cn=cn, cta_group=cg, ksplit=ks, out=out)
             for _ in range(3): f()
             torch.cuda.synchronize()
+            # 20 launches captured in a CUDA graph: device time without the host's per-call map setup
+            g = torch.cuda.CUDAGraph()
+            s = torch.cuda.Stream()
+            with torch.cuda.stream(s):
+                with torch.cuda.graph(g, stream=s):
+                    for _ in range(20): f()
+            g.replay(); torch.cuda.synchronize()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record()
-            for _ in range(20): f()
+            g.replay()
             e1.record(); torch.cuda.synchronize()
             us = e0.elapsed_time(e1) / 20 * 1e3
             print(json.dumps({"tag": tag, "M": M, "N": N, "K": K, "a_mn": a_mn, "b_mn": b_mn, "bn": bn, "cm": cm, "cn": cn,
