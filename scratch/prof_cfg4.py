@@ -11,6 +11,8 @@ y = torch.empty(Tt, B, 2 * H, dtype=torch.bfloat16, device="cuda")
 dY = (torch.randn(Tt, B, 2 * H, device="cuda") * 0.01).to(torch.bfloat16)
 h0, c0 = torch.zeros(B, H, device="cuda"), torch.zeros(B, H, device="cuda")
 dx = torch.empty((Ts + Tt) * B * I, dtype=torch.bfloat16, device="cuda")
+if len(sys.argv) > 1:
+    c.tune_mode(A.TUNE_FROZEN, sys.argv[1])
 for _ in range(2):
     c.forward(x, h0, c0, y, None, None); c.backward(dY, None, None, dx, None, None); c.sgd(0.01)
 torch.cuda.synchronize()
