@@ -273,10 +273,11 @@ astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream
 /* Per-MMA issue time of a tcgen05.mma chain (the serial MMA chain of a small-batch recurrent step,
  * DESIGN §6c): `ctas` CTAs each issue `iters` dependent M x N x 16 bf16 MMAs (M ∈ {64, 128}, N a
  * multiple of 16 ≤ 256) from shared memory into TMEM; cycles (device int64[ctas]) ← clock64 from
- * the first issue to completion.  dump (device fp32[128][N], or null): with iters = 1, CTA 0's
- * 128 TMEM lanes × N columns, for the M = 64 accumulator layout.  Errors: bad arguments →
- * ASTRA_ERR_ARG.                                                                             */
-astra_status astra_micro_mma_chain(int M, int N, int iters, int ctas, long long* cycles, float* dump,
+ * the first issue to completion.  mode (bits, per group of 4 MMAs = one k-block, as a k loop
+ * does): 1 an mbarrier wait on an already completed phase, 2 tcgen05.fence::after_thread_sync,
+ * 4 a tcgen05.commit to an mbarrier.  dump (device fp32[128][N], or null): with iters = 1, CTA
+ * 0's 128 TMEM lanes × N columns.  Errors: bad arguments → ASTRA_ERR_ARG.                      */
+astra_status astra_micro_mma_chain(int M, int N, int iters, int ctas, int mode, long long* cycles, float* dump,
                                    astra_stream stream);
 astra_status astra_micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, int stages, int nbox,
                                   int same, astra_stream stream);

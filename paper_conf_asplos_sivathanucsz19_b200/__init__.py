@@ -86,7 +86,7 @@ _SIGS = {
     "astra_micro_grid_barrier": [_P, _I, _P],
     "astra_micro_launch_chain": [_I, _I, _I, _P],
     "astra_micro_tma_read": [_P, ctypes.c_long, _I, _I, _I, _I, _I, _I, _P],
-    "astra_micro_mma_chain": [_I, _I, _I, _I, _P, _P, _P],
+    "astra_micro_mma_chain": [_I, _I, _I, _I, _I, _P, _P, _P],
     "astra_micro_peer_reduce": [_P, _P, _I, _SZ, _I, ctypes.c_uint, _P],
     "astra_debug_set_trace": [_I, _P],
     "astra_status_string": [_I],

@@ -22,7 +22,7 @@ namespace astra {   // kernels/micro.cu
 void micro_stream_read(const void* buf, size_t bytes, int passes, float* sink, cudaStream_t st);
 void micro_grid_barrier(unsigned* counter, int iters, cudaStream_t st);
 void micro_launch_chain(int n, int pdl, int blocks, cudaStream_t st);
-void micro_mma_chain(int M, int N, int iters, int ctas, long long* cycles, float* dump, cudaStream_t st);
+void micro_mma_chain(int M, int N, int iters, int ctas, int mode, long long* cycles, float* dump, cudaStream_t st);
 void micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, int stages, int nbox, int same,
                     cudaStream_t st);
 void micro_peer_reduce(float* const* bufs, uint32_t* const* sigs, int world, size_t n, int reps, uint32_t seq0,
@@ -459,9 +459,9 @@ astra_status astra_micro_grid_barrier(unsigned* counter, int iters, astra_stream
   return guard([&] { micro_grid_barrier(counter, iters, (cudaStream_t)stream); });
 }
 
-astra_status astra_micro_mma_chain(int M, int N, int iters, int ctas, long long* cycles, float* dump,
-                                  astra_stream stream) {
-  return guard([&] { micro_mma_chain(M, N, iters, ctas, cycles, dump, (cudaStream_t)stream); });
+astra_status astra_micro_mma_chain(int M, int N, int iters, int ctas, int mode, long long* cycles, float* dump,
+                                   astra_stream stream) {
+  return guard([&] { micro_mma_chain(M, N, iters, ctas, mode, cycles, dump, (cudaStream_t)stream); });
 }
 astra_status astra_micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, int stages, int nbox,
                                   int same, astra_stream stream) {

@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(BF_THREADS, 1)
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer: one accumulator per split-K chunk
     pdl_wait();
-    if (lane == 0) {   // lean issue loop: counters and descriptors advanced by (bytes >> 4)
+    {   // whole warp (umma_*_warp elect the issuing lane); lean loop: descriptors advanced by (bytes >> 4)
       const uint32_t sa0 = sm100::smem_u32(smem);
       const uint64_t dA0 = sm100::smem_desc_sw128(sa0, 16, 1024);
       const uint64_t dB0 = sm100::smem_desc_sw128(sa0 + TC_BM * TC_BK * 2, 8192, 1024);
@@ -136,12 +136,12 @@ __global__ void __launch_bounds__(BF_THREADS, 1)
         const uint64_t ad = dA0 + (uint64_t)(s * (BF_STAGE >> 4)), bd = dB0 + (uint64_t)(s * (BF_STAGE >> 4));
 #pragma unroll
         for (int kk = 0; kk < TC_BK / 16; ++kk)
-          sm100::umma_bf16(tmem_base + c * BF_BN, ad + 2 * kk, bd + 128 * kk, idesc, (jk | kk) != 0);
-        sm100::umma_commit(&empty[s]);
+          sm100::umma_bf16_warp(tmem_base + c * BF_BN, ad + 2 * kk, bd + 128 * kk, idesc, (jk | kk) != 0);
+        sm100::umma_commit_warp(&empty[s]);
         if (++s == stages) { s = 0; ph ^= 1; }
         if (++jk == kper) { jk = 0; ++c; }
       }
-      sm100::umma_commit(tfull);
+      sm100::umma_commit_warp(tfull);
     }
   } else {
     // ------------------------------------------------------------ fused cell backward (8 warps)

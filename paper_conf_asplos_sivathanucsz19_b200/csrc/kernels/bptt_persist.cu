@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(PB_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (lean loop, rec_persist.cu)
-    if (lane == 0) {
+    {   // whole warp: umma_*_warp elect the issuing lane
       PB_WAIT(pb_try(resbar, 0), "resbar", 0);
       sm100::tc_fence_after();
       const uint32_t idesc = a.idesc;
@@ -263,21 +263,21 @@ __global__ void __launch_bounds__(PB_THREADS, 1)
           if (waited) sm100::tc_fence_after();
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)   // A K-major: +32 B per K step; B MN-major: +2048 B
-            sm100::umma_bf16(d_tmem, adesc + 2 * kk, bd + 128 * kk, idesc, (kb | kk) != 0);
+            sm100::umma_bf16_warp(d_tmem, adesc + 2 * kk, bd + 128 * kk, idesc, (kb | kk) != 0);
           adesc += a_kb;
           if (++ja == ka) {
-            sm100::umma_commit(&emptyA[sa]);
+            sm100::umma_commit_warp(&emptyA[sa]);
             if (++sa == SA) { sa = 0; pa ^= 1; }
           }
           if (kb >= R) {
             bdesc += b_kb;
             if (++jb == kbs) {
-              sm100::umma_commit(&emptyB[sb]);
+              sm100::umma_commit_warp(&emptyB[sb]);
               if (++sb == SB) { sb = 0; pb ^= 1; }
             }
           }
         }
-        sm100::umma_commit(&tfull[acc]);
+        sm100::umma_commit_warp(&tfull[acc]);
         if (a.trace) a.trace[((size_t)blockIdx.x * T + (T - 2 - i)) * 8 + 2] = pb_gtime();
       }
     }

@@ -445,7 +445,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
-    if (lane == 0) {
+    {   // whole warp: umma_*_warp elect the issuing lane
       int s = 0;
       uint32_t ph = 0;
       int local = 0;
@@ -476,13 +476,13 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
             const uint64_t ad = ad0 + j * a_j, bd = bd0 + j * b_j;
 #pragma unroll
             for (int kk = 0; kk < TC_BK / 16; ++kk)
-              sm100::umma_bf16(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb + j != kb0 || kk != 0) ? 1u : 0u);
+              sm100::umma_bf16_warp(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb + j != kb0 || kk != 0) ? 1u : 0u);
           }
-          if (cs == 1) sm100::umma_commit(&empty[s]);
-          else sm100::umma_commit_mc(&empty[s], mask_nb);
+          if (cs == 1) sm100::umma_commit_warp(&empty[s]);
+          else sm100::umma_commit_mc_warp(&empty[s], mask_nb);
           if (++s == stages) { s = 0; ph ^= 1; }
         }
-        sm100::umma_commit(&tfull[acc]);
+        sm100::umma_commit_warp(&tfull[acc]);
         GEMM_TRACE(4);
       }
     }
@@ -652,7 +652,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (pair leader only)
     pdl_wait();
-    if (lane == 0 && rank == 0) {
+    if (rank == 0) {   // whole warp: umma_*_warp elect the issuing lane
       int s = 0;
       uint32_t ph = 0;
       int local = 0;
@@ -674,11 +674,11 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16_cg2(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
-          sm100::umma_commit_cg2_mc(&empty[s], 0x3);
+            sm100::umma_bf16_cg2_warp(d_tmem, ad + kk * a_kk, bd + kk * b_kk, idesc, (kb != kb0 || kk != 0) ? 1u : 0u);
+          sm100::umma_commit_cg2_mc_warp(&empty[s], 0x3);
           if (++s == stages) { s = 0; ph ^= 1; }
         }
-        sm100::umma_commit_cg2_mc(&tfull[acc], 0x3);
+        sm100::umma_commit_cg2_mc_warp(&tfull[acc], 0x3);
       }
     }
   } else {

@@ -102,13 +102,13 @@ __global__ void __launch_bounds__(64, 1) tma_read_kernel(const __grid_constant__
 // B[n][k] = ((5n + 2k) mod 5 − 2)/2 (exact in bf16).  cycles[cta] = clock64 from the first issue to
 // the commit's mbarrier completing; with iters == 1 CTA 0 dumps all 128 TMEM lanes × N columns to
 // dump[lane][col] (the accumulator layout for M = 64).
-__global__ void __launch_bounds__(128, 1) mma_chain_kernel(int M, int N, int iters, uint32_t idesc,
+__global__ void __launch_bounds__(128, 1) mma_chain_kernel(int M, int N, int iters, int mode, uint32_t idesc,
                                                            long long* __restrict__ cycles, float* __restrict__ dump) {
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* sm = (unsigned char*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   unsigned char* sA = sm;               // 128 rows x 128 B
   unsigned char* sB = sm + 128 * 128;   // 256 rows x 128 B
-  __shared__ uint64_t bar;
+  __shared__ uint64_t bar, done, cbar;
   __shared__ uint32_t tbase;
   const int tid = threadIdx.x;
   for (int i = tid; i < (128 + 256) * 64; i += blockDim.x) {
@@ -122,7 +122,10 @@ __global__ void __launch_bounds__(128, 1) mma_chain_kernel(int M, int N, int ite
   }
   if (tid == 0) {
     sm100::mbar_init(&bar, 1);
+    sm100::mbar_init(&done, 1);
+    sm100::mbar_init(&cbar, (iters + 3) / 4);
     sm100::fence_barrier_init();
+    sm100::mbar_arrive(&done);   // phase 0 complete: a wait on it returns at once (a k loop's landed stage)
   }
   if (tid < 32) sm100::tmem_alloc(&tbase, 256);
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -130,13 +133,37 @@ __global__ void __launch_bounds__(128, 1) mma_chain_kernel(int M, int N, int ite
   __syncthreads();
   sm100::tc_fence_after();
   const uint32_t tmem = tbase;
-  if (tid == 0) {
+  if ((mode & 8) && tid < 32) {   // whole-warp issue (umma_bf16_warp)
     const uint64_t a0 = sm100::smem_desc_sw128(sm100::smem_u32(sA), 16, 1024);
     const uint64_t b0 = sm100::smem_desc_sw128(sm100::smem_u32(sB), 16, 1024);
     const long long t0 = clock64();
     for (int i = 0; i < iters; ++i) {
+      if ((i & 3) == 0) {
+        if (mode & 1) sm100::mbar_wait(&done, 0);
+        if (mode & 2) sm100::tc_fence_after();
+      }
+      const uint64_t kk = (uint64_t)(i & 3) * 2;
+      sm100::umma_bf16_warp(tmem, a0 + kk, b0 + kk, idesc, i > 0 ? 1u : 0u);
+      if ((mode & 4) && (i & 3) == 3) sm100::umma_commit_warp(&cbar);
+    }
+    sm100::umma_commit_warp(&bar);
+    sm100::mbar_wait(&bar, 0);
+    const long long t1 = clock64();
+    if (tid == 0) cycles[blockIdx.x] = t1 - t0;
+  } else if (!(mode & 8) && tid == 0) {
+    const uint64_t a0 = sm100::smem_desc_sw128(sm100::smem_u32(sA), 16, 1024);
+    const uint64_t b0 = sm100::smem_desc_sw128(sm100::smem_u32(sB), 16, 1024);
+    const long long t0 = clock64();
+    for (int i = 0; i < iters; ++i) {
+      // mode bits, per k-block of 4 MMAs, as a k loop does: 1 = mbarrier wait (on a completed phase),
+      // 2 = tcgen05.fence::after_thread_sync, 4 = tcgen05.commit to an mbarrier after the 4 MMAs
+      if ((i & 3) == 0) {
+        if (mode & 1) sm100::mbar_wait(&done, 0);
+        if (mode & 2) sm100::tc_fence_after();
+      }
       const uint64_t kk = (uint64_t)(i & 3) * 2;   // 32 B per K-step of 16 bf16
       sm100::umma_bf16(tmem, a0 + kk, b0 + kk, idesc, i > 0 ? 1u : 0u);
+      if ((mode & 4) && (i & 3) == 3) sm100::umma_commit(&cbar);
     }
     sm100::umma_commit(&bar);
     sm100::mbar_wait(&bar, 0);
@@ -193,7 +220,7 @@ void micro_tma_read(const void* buf, long rows, int kb, int box_rows, int ctas, 
   LAUNCH_CHECK();
 }
 
-void micro_mma_chain(int M, int N, int iters, int ctas, long long* cycles, float* dump, cudaStream_t st) {
+void micro_mma_chain(int M, int N, int iters, int ctas, int mode, long long* cycles, float* dump, cudaStream_t st) {
   ASTRA_CHECK_ARG((M == 64 || M == 128) && N >= 16 && N <= 256 && N % 16 == 0 && iters >= 1 && ctas >= 1 && cycles,
                   "micro_mma_chain: bad arguments");
   uint32_t d = 0;
@@ -204,7 +231,7 @@ void micro_mma_chain(int M, int N, int iters, int ctas, long long* cycles, float
   d |= (uint32_t)(M >> 4) << 24;    // M >> 4
   const int smem = 1024 + (128 + 256) * 128;
   CUDA_TRY(cudaFuncSetAttribute(mma_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  mma_chain_kernel<<<ctas, 128, smem, st>>>(M, N, iters, d, cycles, dump);
+  mma_chain_kernel<<<ctas, 128, smem, st>>>(M, N, iters, mode, d, cycles, dump);
   LAUNCH_CHECK();
 }
 

@@ -132,7 +132,7 @@ __global__ void __launch_bounds__(RF_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
-    if (lane == 0) {   // lean issue loop: counters and descriptors advanced by (bytes >> 4)
+    {   // whole warp (umma_*_warp elect the issuing lane); lean loop: descriptors advanced by (bytes >> 4)
       const uint32_t sa0 = sm100::smem_u32(smem);
       const uint64_t dA0 = sm100::smem_desc_sw128(sa0, 16, 1024);
       const uint64_t dB0 = sm100::smem_desc_sw128(sa0 + S::A_BYTES, 16, 1024);
@@ -151,11 +151,11 @@ __global__ void __launch_bounds__(RF_THREADS, 1)
           const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, ad + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
-          sm100::umma_commit(&empty[s]);
+            sm100::umma_bf16_warp(d_tmem, ad + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
+          sm100::umma_commit_warp(&empty[s]);
           if (++s == stages) { s = 0; ph ^= 1; }
         }
-        sm100::umma_commit(&tfull[acc]);
+        sm100::umma_commit_warp(&tfull[acc]);
       }
     }
   } else {

@@ -124,7 +124,7 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (pair leader)
-    if (lane == 0 && rank == 0) {   // lean issue loop: counters and descriptors advanced by (bytes >> 4)
+    if (rank == 0) {   // whole warp (umma_*_warp elect the issuing lane); lean loop: descriptors advanced by (bytes >> 4)
       const uint32_t sa0 = sm100::smem_u32(smem);
       const uint64_t dA0 = sm100::smem_desc_sw128(sa0, 16, 1024);
       const uint64_t dB0 = sm100::smem_desc_sw128(sa0 + S::A_BYTES, 16, 1024);
@@ -138,11 +138,11 @@ __global__ void __launch_bounds__(R2_THREADS, 1)
         const uint64_t ad = dA0 + (uint64_t)(s * (S::STAGE_BYTES >> 4)), bd = dB0 + (uint64_t)(s * (S::STAGE_BYTES >> 4));
 #pragma unroll
         for (int kk = 0; kk < TC_BK / 16; ++kk)
-          sm100::umma_bf16_cg2(tmem_base, ad + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
-        sm100::umma_commit_cg2_mc(&empty[s], 0x3);
+          sm100::umma_bf16_cg2_warp(tmem_base, ad + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
+        sm100::umma_commit_cg2_mc_warp(&empty[s], 0x3);
         if (++s == stages) { s = 0; ph ^= 1; }
       }
-      sm100::umma_commit_cg2_mc(tfull, 0x3);
+      sm100::umma_commit_cg2_mc_warp(tfull, 0x3);
       GEMM_TRACE(4);
     }
   } else {

@@ -185,7 +185,7 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
     // work (divisions, descriptor rebuilds, constant loads) must stay well below that — shared-
     // memory descriptors are advanced by adding (bytes >> 4) to their address field (addresses
     // < 256 KB never carry out of the 14-bit field), stage bookkeeping is counter-based.
-    if (lane == 0) {
+    {   // the whole warp runs the loop (warp-uniform operands); one elected lane issues (umma_*_warp)
       sm100::mbar_wait(resbar, 0);
       sm100::tc_fence_after();
       const uint32_t idesc = a.idesc;
@@ -228,22 +228,22 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
           if (waited) sm100::tc_fence_after();   // only after a new barrier wait
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
+            sm100::umma_bf16_warp(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (kb | kk) != 0);
           adesc += a_kb;
           if (++ja == ka) {
-            sm100::umma_commit(&emptyA[sa]);
+            sm100::umma_commit_warp(&emptyA[sa]);
             if (++sa == SA) { sa = 0; pa ^= 1; }
           }
           if (kb >= R) {
             bdesc += b_kb;
             if (++jb == kbs) {
-              sm100::umma_commit(&emptyB[sb]);
+              sm100::umma_commit_warp(&emptyB[sb]);
               if (++sb == SB) { sb = 0; pb ^= 1; }
             }
           }
         }
-        sm100::umma_commit(&tfull[acc]);
-        if (a.trace) a.trace[((size_t)blockIdx.x * (a.t1 - a.t0) + (t - a.t0)) * 6 + 2] = sb_gtime();
+        sm100::umma_commit_warp(&tfull[acc]);
+        if (a.trace && lane == 0) a.trace[((size_t)blockIdx.x * (a.t1 - a.t0) + (t - a.t0)) * 6 + 2] = sb_gtime();
       }
     }
   } else {

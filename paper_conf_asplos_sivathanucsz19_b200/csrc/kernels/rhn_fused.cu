@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
     // Lean issue loop (round 2, cf. rec_persist.cu): stage bookkeeping by counters and shared-memory
     // descriptors advanced by adding (bytes >> 4) — the per-k-block scalar work (long divisions,
     // descriptor rebuilds) otherwise paced the k loop, not the operands' arrival.
-    if (lane == 0) {
+    {   // whole warp: umma_*_warp elect the issuing lane
       const uint64_t dA0 = sm100::smem_desc_sw128(sm100::smem_u32(smem), 16, 1024);
       const uint64_t dB0 = sm100::smem_desc_sw128(sm100::smem_u32(smem) + a_bytes, 16, 1024);
       const uint32_t st_step = (uint32_t)stage_bytes >> 4;
@@ -197,12 +197,12 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           const uint32_t d_tmem = tmem_base + c * RH_BN;
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, ad + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
-          sm100::umma_commit(&empty[s]);
+            sm100::umma_bf16_warp(d_tmem, ad + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
+          sm100::umma_commit_warp(&empty[s]);
           if (++s == stages) { s = 0; ph ^= 1; }
           if (++jk == kper) { jk = 0; ++c; }
         }
-        sm100::umma_commit(tfull);
+        sm100::umma_commit_warp(tfull);
       }
     }
   } else {

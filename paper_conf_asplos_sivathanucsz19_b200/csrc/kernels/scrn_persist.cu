@@ -115,7 +115,7 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer (lean loop, see rec_persist.cu)
-    if (lane == 0) {
+    {   // whole warp: umma_*_warp elect the issuing lane
       sm100::mbar_wait(resbar, 0);
       sm100::tc_fence_after();
       const uint32_t idesc = a.idesc;
@@ -142,15 +142,15 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
           const uint64_t bd = dR0 + (uint64_t)(kb * b_kb);
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
+            sm100::umma_bf16_warp(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
           adesc += a_kb;
           if (++ja == ka) {
-            sm100::umma_commit(&emptyA[sa]);
+            sm100::umma_commit_warp(&emptyA[sa]);
             if (++sa == SA) { sa = 0; pa ^= 1; }
           }
           if (++jk == kper) { jk = 0; ++q; }   // next canonical split-K chunk (R33): a fresh accumulator
         }
-        sm100::umma_commit(&tfull[acc]);
+        sm100::umma_commit_warp(&tfull[acc]);
       }
     }
   } else {
@@ -319,7 +319,7 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
     }
   } else if (warp == 1) {
     // ------------------------------------------------------------ MMA issuer
-    if (lane == 0) {
+    {   // whole warp: umma_*_warp elect the issuing lane
       sm100::mbar_wait(resbar, 0);
       sm100::tc_fence_after();
       const uint32_t idesc = a.idesc;
@@ -346,15 +346,15 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
           const uint64_t bd = dR0 + (uint64_t)(kb * b_kb);
 #pragma unroll
           for (int kk = 0; kk < TC_BK / 16; ++kk)
-            sm100::umma_bf16(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
+            sm100::umma_bf16_warp(d_tmem, adesc + 2 * kk, bd + 2 * kk, idesc, (jk | kk) != 0);
           adesc += a_kb;
           if (++ja == ka) {
-            sm100::umma_commit(&emptyA[sa]);
+            sm100::umma_commit_warp(&emptyA[sa]);
             if (++sa == SA) { sa = 0; pa ^= 1; }
           }
           if (++jk == kper) { jk = 0; ++q; }
         }
-        sm100::umma_commit(&tfull[acc]);
+        sm100::umma_commit_warp(&tfull[acc]);
       }
     }
   } else {

@@ -9,7 +9,7 @@ cyc = torch.zeros(148, dtype=torch.int64, device="cuda")
 for M in (64, 128):
     N = 64
     dump = torch.zeros(128, N, device="cuda")
-    A._check(L.astra_micro_mma_chain(M, N, 1, 1, A._ptr(cyc), A._ptr(dump), st))
+    A._check(L.astra_micro_mma_chain(M, N, 1, 1, 0, A._ptr(cyc), A._ptr(dump), st))
     torch.cuda.synchronize()
     a = np.array([[((3 * m + k) % 7 - 3) * 0.25 for k in range(16)] for m in range(128)])
     b = np.array([[((5 * n + 2 * k) % 5 - 2) * 0.5 for k in range(16)] for n in range(N)])
@@ -26,10 +26,19 @@ for ctas in (1, 148):
     for M in (64, 128):
         for N in (32, 64, 128, 256):
             for iters in (64, 512):
-                A._check(L.astra_micro_mma_chain(M, N, iters, ctas, A._ptr(cyc), None, st))
+                A._check(L.astra_micro_mma_chain(M, N, iters, ctas, 0, A._ptr(cyc), None, st))
                 torch.cuda.synchronize()
-                A._check(L.astra_micro_mma_chain(M, N, iters, ctas, A._ptr(cyc), None, st))
+                A._check(L.astra_micro_mma_chain(M, N, iters, ctas, 0, A._ptr(cyc), None, st))
                 torch.cuda.synchronize()
                 c = cyc[:ctas].cpu().numpy()
                 print(json.dumps({"ctas": ctas, "M": M, "N": N, "iters": iters, "cyc_per_mma_med": round(float(np.median(c)) / iters, 1),
                                   "cyc_per_mma_max": round(float(c.max()) / iters, 1)}), flush=True)
+
+for mode in (0, 7, 8, 15):
+    for N in (64, 256):
+        iters = 512
+        for _ in range(2):
+            A._check(L.astra_micro_mma_chain(128, N, iters, 1, mode, A._ptr(cyc), None, st))
+            torch.cuda.synchronize()
+        c = cyc[:1].cpu().numpy()
+        print(json.dumps({"mode": mode, "M": 128, "N": N, "iters": iters, "cyc_per_mma": round(float(c[0]) / iters, 1)}), flush=True)
