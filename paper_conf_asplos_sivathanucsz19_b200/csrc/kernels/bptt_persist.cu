@@ -165,7 +165,7 @@ __global__ void __launch_bounds__(PB_THREADS, 1)
 
   if (warp == 0) {
     // ------------------------------------------------------------ A producer: D_uh,{t+1} chunk rows
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       pdl_wait();
       int s = 0;
       uint32_t ph = 0;
@@ -178,8 +178,8 @@ __global__ void __launch_bounds__(PB_THREADS, 1)
         if (a.trace) a.trace[((size_t)blockIdx.x * T + t) * 8 + 0] = pb_gtime();
         for (int kb = 0; kb < kper; kb += a.ka) {
           PB_WAIT(pb_try(&emptyA[s], ph ^ 1), "emptyA", i);
-          sm100::mbar_arrive_expect_tx(&fullA[s], stage_bytes);
-          sm100::tma_load_4d(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb0 + kb, t + 1);
+          sm100::mbar_arrive_expect_tx_warp(&fullA[s], stage_bytes);
+          sm100::tma_load_4d_warp(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb0 + kb, t + 1);
           if (++s == SA) { s = 0; ph ^= 1; }
         }
       }
@@ -188,22 +188,22 @@ __global__ void __launch_bounds__(PB_THREADS, 1)
     // ------------------------------------------------------------ B producer: the Uᵀ slice of the chunk
     // (the U mirror does not change during the chain: resident part once, streamed part paced by
     // the MMAs only)
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       const uint64_t pol = sm100::l2_policy_evict_last();
       pdl_wait();
       const int n0 = grp * PB_UG;
       if (R > 0) {
-        sm100::mbar_arrive_expect_tx(resbar, (uint32_t)(R * PB_BT));
+        sm100::mbar_arrive_expect_tx_warp(resbar, (uint32_t)(R * PB_BT));
         for (int kb = 0; kb < R; kb += 8) {
           const int n = R - kb < 8 ? R - kb : 8;
           if (n == 8)
-            sm100::tma_load_3d_hint(sRes + kb * PB_BT, &mapBr, resbar, n0, 0, kb0 + kb, pol);
+            sm100::tma_load_3d_hint_warp(sRes + kb * PB_BT, &mapBr, resbar, n0, 0, kb0 + kb, pol);
           else
             for (int j = 0; j < n; ++j)
-              sm100::tma_load_3d_hint(sRes + (kb + j) * PB_BT, &mapB1, resbar, n0, 0, kb0 + kb + j, pol);
+              sm100::tma_load_3d_hint_warp(sRes + (kb + j) * PB_BT, &mapB1, resbar, n0, 0, kb0 + kb + j, pol);
         }
       } else {
-        sm100::mbar_arrive(resbar);
+        sm100::mbar_arrive_warp(resbar);
       }
       if (R < kper && nmm > 0) {
         int s = 0;
@@ -212,8 +212,8 @@ __global__ void __launch_bounds__(PB_THREADS, 1)
         for (int i = 0; i < nmm; ++i)
           for (int kb = R; kb < kper; kb += a.kbs) {
             PB_WAIT(pb_try(&emptyB[s], ph ^ 1), "emptyB", i);
-            sm100::mbar_arrive_expect_tx(&fullB[s], stage_bytes);
-            sm100::tma_load_3d_hint(sB + s * stage_bytes, &mapB, &fullB[s], n0, 0, kb0 + kb, pol);
+            sm100::mbar_arrive_expect_tx_warp(&fullB[s], stage_bytes);
+            sm100::tma_load_3d_hint_warp(sB + s * stage_bytes, &mapB, &fullB[s], n0, 0, kb0 + kb, pol);
             if (++s == SB) { s = 0; ph ^= 1; }
           }
       }

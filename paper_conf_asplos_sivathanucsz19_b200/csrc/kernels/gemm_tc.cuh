@@ -360,7 +360,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA forms elect the issuing lane
       int s = 0;
       uint32_t ph = 0;
       const uint64_t pol = sm100::l2_policy_evict_last();
@@ -378,65 +378,65 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           sm100::mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * stage_bytes;
           uint8_t* sb = sa + KB * a_kb_bytes;
-          sm100::mbar_arrive_expect_tx(&full[s], stage_bytes);
+          sm100::mbar_arrive_expect_tx_warp(&full[s], stage_bytes);
           const int k0 = kb * TC_BK;
           if (KB > 1) {   // (cs == 1) one box per operand for the KB k-blocks of the stage
             if (args.a_mn) {
-              sm100::tma_load_3d(sa, &mapA, &full[s], m0, k0, args.az);
-              sm100::tma_load_3d(sa + KB * 8192, &mapA, &full[s], m0 + 64, k0, args.az);
+              sm100::tma_load_3d_warp(sa, &mapA, &full[s], m0, k0, args.az);
+              sm100::tma_load_3d_warp(sa + KB * 8192, &mapA, &full[s], m0 + 64, k0, args.az);
             } else {
-              sm100::tma_load_4d(sa, &mapA, &full[s], 0, m0, kb, args.az);
+              sm100::tma_load_4d_warp(sa, &mapA, &full[s], 0, m0, kb, args.az);
             }
             if (args.b_mn) {
 #pragma unroll
               for (int j = 0; j < BN / 64; ++j) {
-                if (args.b_keep) sm100::tma_load_3d_hint(sb + j * KB * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz, pol);
-                else sm100::tma_load_3d(sb + j * KB * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+                if (args.b_keep) sm100::tma_load_3d_hint_warp(sb + j * KB * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz, pol);
+                else sm100::tma_load_3d_warp(sb + j * KB * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
               }
             } else {
-              if (args.b_keep) sm100::tma_load_4d_hint(sb, &mapB, &full[s], 0, n0, kb, args.bz, pol);
-              else sm100::tma_load_4d(sb, &mapB, &full[s], 0, n0, kb, args.bz);
+              if (args.b_keep) sm100::tma_load_4d_hint_warp(sb, &mapB, &full[s], 0, n0, kb, args.bz, pol);
+              else sm100::tma_load_4d_warp(sb, &mapB, &full[s], 0, n0, kb, args.bz);
             }
           } else if (cs == 1) {
             if (args.a_mn) {
-              sm100::tma_load_3d(sa, &mapA, &full[s], m0, k0, args.az);
-              sm100::tma_load_3d(sa + 8192, &mapA, &full[s], m0 + 64, k0, args.az);
+              sm100::tma_load_3d_warp(sa, &mapA, &full[s], m0, k0, args.az);
+              sm100::tma_load_3d_warp(sa + 8192, &mapA, &full[s], m0 + 64, k0, args.az);
             } else {
-              sm100::tma_load_3d(sa, &mapA, &full[s], k0, m0, args.az);
+              sm100::tma_load_3d_warp(sa, &mapA, &full[s], k0, m0, args.az);
             }
             if (args.b_mn) {
 #pragma unroll
               for (int j = 0; j < BN / 64; ++j) {
-                if (args.b_keep) sm100::tma_load_3d_hint(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz, pol);
-                else sm100::tma_load_3d(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
+                if (args.b_keep) sm100::tma_load_3d_hint_warp(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz, pol);
+                else sm100::tma_load_3d_warp(sb + j * 8192, &mapB, &full[s], n0 + 64 * j, k0, args.bz);
               }
             } else {
-              if (args.b_keep) sm100::tma_load_3d_hint(sb, &mapB, &full[s], k0, n0, args.bz, pol);
-              else sm100::tma_load_3d(sb, &mapB, &full[s], k0, n0, args.bz);
+              if (args.b_keep) sm100::tma_load_3d_hint_warp(sb, &mapB, &full[s], k0, n0, args.bz, pol);
+              else sm100::tma_load_3d_warp(sb, &mapB, &full[s], k0, n0, args.bz);
             }
           } else {
             if (args.a_mn) {
               for (int j = 0; j < 2; ++j)
-                sm100::tma_load_3d_mc(sa + j * 8192 + rn * a_krows * 128, &mapA, &full[s], m0 + 64 * j,
+                sm100::tma_load_3d_mc_warp(sa + j * 8192 + rn * a_krows * 128, &mapA, &full[s], m0 + 64 * j,
                                       k0 + rn * a_krows, args.az, mask_a);
             } else {
-              sm100::tma_load_3d_mc(sa + rn * a_rows * 128, &mapA, &full[s], k0, m0 + rn * a_rows, args.az, mask_a);
+              sm100::tma_load_3d_mc_warp(sa + rn * a_rows * 128, &mapA, &full[s], k0, m0 + rn * a_rows, args.az, mask_a);
             }
             if (args.b_mn) {
               for (int j = 0; j < BN / 64; ++j) {
                 if (args.b_keep)
-                  sm100::tma_load_3d_mc_hint(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
+                  sm100::tma_load_3d_mc_hint_warp(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
                                              k0 + rm * b_krows, args.bz, mask_b, pol);
                 else
-                  sm100::tma_load_3d_mc(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
+                  sm100::tma_load_3d_mc_warp(sb + j * 8192 + rm * b_krows * 128, &mapB, &full[s], n0 + 64 * j,
                                         k0 + rm * b_krows, args.bz, mask_b);
               }
             } else {
               if (args.b_keep)
-                sm100::tma_load_3d_mc_hint(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz,
+                sm100::tma_load_3d_mc_hint_warp(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz,
                                            mask_b, pol);
               else
-                sm100::tma_load_3d_mc(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz, mask_b);
+                sm100::tma_load_3d_mc_warp(sb + rm * b_rows * 128, &mapB, &full[s], k0, n0 + rm * b_rows, args.bz, mask_b);
             }
           }
           if (++s == stages) { s = 0; ph ^= 1; }

@@ -73,16 +73,26 @@ __global__ void __launch_bounds__(64, 1) tma_read_kernel(const __grid_constant__
     sm100::fence_barrier_init();
   }
   __syncthreads();
-  const int rb0 = same ? 0 : (int)blockIdx.x % row_blocks;
-  if (threadIdx.x == 0) {
-    int s = 0;
+  const int rb0 = (same & 1) ? 0 : (int)blockIdx.x % row_blocks;
+  if ((same & 2) && threadIdx.x < 32) {   // whole-warp issue (tma_load_3d_warp)
+    int s = 0, k = 0, rb = rb0;
+    uint32_t ph = 0;
+    for (int i = 0; i < nbox; ++i) {
+      sm100::mbar_wait(&empty[s], ph ^ 1);
+      sm100::mbar_arrive_expect_tx_warp(&full[s], (uint32_t)box_bytes);
+      sm100::tma_load_3d_warp(smem + s * box_bytes, &m, &full[s], k * 64, rb * box_rows, 0);
+      if (++s == stages) { s = 0; ph ^= 1; }
+      if (++k == kb) { k = 0; if (++rb == row_blocks) rb = 0; }
+    }
+  } else if (!(same & 2) && threadIdx.x == 0) {
+    int s = 0, k = 0, rb = rb0;
     uint32_t ph = 0;
     for (int i = 0; i < nbox; ++i) {
       sm100::mbar_wait(&empty[s], ph ^ 1);
       sm100::mbar_arrive_expect_tx(&full[s], (uint32_t)box_bytes);
-      const int k = i % kb, rb = (rb0 + i / kb) % row_blocks;
       sm100::tma_load_3d(smem + s * box_bytes, &m, &full[s], k * 64, rb * box_rows, 0);
       if (++s == stages) { s = 0; ph ^= 1; }
+      if (++k == kb) { k = 0; if (++rb == row_blocks) rb = 0; }
     }
   } else if (threadIdx.x == 32) {
     int s = 0;

@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
     // ------------------------------------------------------------ A producer: h_{t−1}, KA k-blocks per box
     // One 4-D TMA box {64, a_rows, KA, 1} lands KA consecutive k-block tiles (the k-block dimension
     // has a 128-byte stride in the map): the per-box issue cost, not bandwidth, bounds small boxes.
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA forms elect the issuing lane
       pdl_wait();
       int s = 0;
       uint32_t ph = 0;
@@ -133,8 +133,8 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
         if (a.trace) a.trace[((size_t)blockIdx.x * (a.t1 - a.t0) + (t - a.t0)) * 6 + 0] = sb_gtime();
         for (int kb = 0; kb < nk; kb += a.ka) {
           sm100::mbar_wait(&emptyA[s], ph ^ 1);
-          sm100::mbar_arrive_expect_tx(&fullA[s], stage_bytes);
-          sm100::tma_load_4d(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t);
+          sm100::mbar_arrive_expect_tx_warp(&fullA[s], stage_bytes);
+          sm100::tma_load_4d_warp(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t);
           if (a.trace && blockIdx.x == 0 && t == a.t0 + (a.t1 - a.t0) / 2)
             a.trace[(size_t)gridDim.x * (a.t1 - a.t0) * 6 + kb / a.ka] = clock64();
           if (++s == SA) { s = 0; ph ^= 1; }
@@ -148,21 +148,21 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
     // the streamed part runs ahead of the recurrence (its ring is paced by the MMAs only).  A 4-D box
     // {64, 16 units, 4 gates, k-blocks} lands the B tiles of several k-blocks in MMA order
     // ([k-block][gate strip][16 rows][64]).
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       const uint64_t pol = sm100::l2_policy_evict_last();
       pdl_wait();
       if (R > 0) {
-        sm100::mbar_arrive_expect_tx(resbar, (uint32_t)(R * SB_BT));
+        sm100::mbar_arrive_expect_tx_warp(resbar, (uint32_t)(R * SB_BT));
         for (int kb = 0; kb < R; kb += 8) {
           const int n = R - kb < 8 ? R - kb : 8;   // resmap box: 8 k-blocks (the last may be clipped below)
           if (n == 8)
-            sm100::tma_load_4d_hint(sRes + kb * SB_BT, &mapBr, resbar, 0, col0, 0, kb, pol);
+            sm100::tma_load_4d_hint_warp(sRes + kb * SB_BT, &mapBr, resbar, 0, col0, 0, kb, pol);
           else
             for (int j = 0; j < n; ++j)
-              sm100::tma_load_4d_hint(sRes + (kb + j) * SB_BT, &mapB1, resbar, 0, col0, 0, kb + j, pol);
+              sm100::tma_load_4d_hint_warp(sRes + (kb + j) * SB_BT, &mapB1, resbar, 0, col0, 0, kb + j, pol);
         }
       } else {
-        sm100::mbar_arrive(resbar);
+        sm100::mbar_arrive_warp(resbar);
       }
       if (R < nk) {
         int s = 0;
@@ -171,8 +171,8 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
         for (int t = a.t0; t < a.t1; ++t)
           for (int kb = R; kb < nk; kb += a.kbs) {
             sm100::mbar_wait(&emptyB[s], ph ^ 1);
-            sm100::mbar_arrive_expect_tx(&fullB[s], stage_bytes);
-            sm100::tma_load_4d_hint(sB + s * stage_bytes, &mapB, &fullB[s], 0, col0, 0, kb, pol);
+            sm100::mbar_arrive_expect_tx_warp(&fullB[s], stage_bytes);
+            sm100::tma_load_4d_hint_warp(sB + s * stage_bytes, &mapB, &fullB[s], 0, col0, 0, kb, pol);
             if (a.trace && blockIdx.x == 0 && t == a.t0 + (a.t1 - a.t0) / 2)
               a.trace[(size_t)gridDim.x * (a.t1 - a.t0) * 6 + 32 + (kb - R) / a.kbs] = clock64();
             if (++s == SB) { s = 0; ph ^= 1; }

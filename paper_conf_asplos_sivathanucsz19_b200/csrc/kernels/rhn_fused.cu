@@ -131,7 +131,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
 
   if (warp == 0) {
     // ------------------------------------------------------------ TMA producer
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       long it = 0;
       const uint64_t pol = sm100::l2_policy_evict_last();
       const int pre = nk < stages ? nk : stages;
@@ -140,14 +140,14 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         const int az = l * (a.T + 1) + t;   // the slot of s^{ℓ−1} at time t (RhnCell::slot)
         auto load_b = [&](int s, int kb) {
           uint8_t* sb = smem + s * stage_bytes + a_bytes;
-          sm100::tma_load_3d_hint(sb, &mapB, &full[s], kb * TC_BK, u0, l, pol);                        // H columns
-          sm100::tma_load_3d_hint(sb + RH_UB * 128, &mapB, &full[s], kb * TC_BK, a.Hp + u0, l, pol);  // T columns
+          sm100::tma_load_3d_hint_warp(sb, &mapB, &full[s], kb * TC_BK, u0, l, pol);                        // H columns
+          sm100::tma_load_3d_hint_warp(sb + RH_UB * 128, &mapB, &full[s], kb * TC_BK, a.Hp + u0, l, pol);  // T columns
         };
         for (int kb = 0; kb < pre; ++kb) {   // R_ℓ tiles do not depend on the recurrence
           const long i = it + kb;
           const int s = (int)(i % stages);
           mbar_wait_idle(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
-          sm100::mbar_arrive_expect_tx(&full[s], (uint32_t)stage_bytes);
+          sm100::mbar_arrive_expect_tx_warp(&full[s], (uint32_t)stage_bytes);
           load_b(s, kb);
         }
         if (q > 0) {   // every CTA of the row block has stored s^{ℓ−1}
@@ -157,14 +157,14 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         if (a.trace) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 0] = global_ns();
         for (int kb = 0; kb < pre; ++kb) {
           const int s = (int)((it + kb) % stages);
-          sm100::tma_load_3d(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
+          sm100::tma_load_3d_warp(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
         }
         for (int kb = pre; kb < nk; ++kb) {
           const long i = it + kb;
           const int s = (int)(i % stages);
           mbar_wait_idle(&empty[s], (uint32_t)((i / stages) & 1) ^ 1);
-          sm100::mbar_arrive_expect_tx(&full[s], (uint32_t)stage_bytes);
-          sm100::tma_load_3d(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
+          sm100::mbar_arrive_expect_tx_warp(&full[s], (uint32_t)stage_bytes);
+          sm100::tma_load_3d_warp(smem + s * stage_bytes, &mapA, &full[s], kb * TC_BK, m0, az);
           load_b(s, kb);
         }
         it += nk;

@@ -89,14 +89,14 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
 
   if (warp == 0) {
     // ------------------------------------------------------------ producer: R slice once, then h_{t−1}
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       const uint64_t pol = sm100::l2_policy_evict_last();
       pdl_wait();
-      sm100::mbar_arrive_expect_tx(resbar, (uint32_t)(nk * SP_BT));
+      sm100::mbar_arrive_expect_tx_warp(resbar, (uint32_t)(nk * SP_BT));
       for (int kb = 0; kb < nk; kb += 8) {
         const int n = nk - kb < 8 ? nk - kb : 8;
         for (int j = 0; j < n; ++j)   // 3-D box {64, 16 units, 1 k-block}
-          sm100::tma_load_3d_hint(sRes + (kb + j) * SP_BT, &mapB, resbar, 0, u0, kb + j, pol);
+          sm100::tma_load_3d_hint_warp(sRes + (kb + j) * SP_BT, &mapB, resbar, 0, u0, kb + j, pol);
       }
       int s = 0;
       uint32_t ph = 0;
@@ -107,8 +107,8 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
         }
         for (int kb = 0; kb < nk; kb += ka) {
           sm100::mbar_wait(&emptyA[s], ph ^ 1);
-          sm100::mbar_arrive_expect_tx(&fullA[s], (uint32_t)stage_bytes);
-          sm100::tma_load_4d(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t);
+          sm100::mbar_arrive_expect_tx_warp(&fullA[s], (uint32_t)stage_bytes);
+          sm100::tma_load_4d_warp(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t);
           if (++s == SA) { s = 0; ph ^= 1; }
         }
       }
@@ -298,11 +298,11 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
 
   if (warp == 0) {
     // ------------------------------------------------------------ producer: R once, then dz_{t+1}
-    if (lane == 0) {
+    {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       const uint64_t pol = sm100::l2_policy_evict_last();
       pdl_wait();
-      sm100::mbar_arrive_expect_tx(resbar, (uint32_t)(nk * SP_BT));
-      for (int kb = 0; kb < nk; ++kb) sm100::tma_load_3d_hint(sRes + kb * SP_BT, &mapB, resbar, 0, u0, kb, pol);
+      sm100::mbar_arrive_expect_tx_warp(resbar, (uint32_t)(nk * SP_BT));
+      for (int kb = 0; kb < nk; ++kb) sm100::tma_load_3d_hint_warp(sRes + kb * SP_BT, &mapB, resbar, 0, u0, kb, pol);
       int s = 0;
       uint32_t ph = 0;
       for (int t = T - 2; t >= 0; --t) {
@@ -311,8 +311,8 @@ __global__ void __launch_bounds__(SP_THREADS, 1)
         sp_fence_proxy_async_global();
         for (int kb = 0; kb < nk; kb += ka) {
           sm100::mbar_wait(&emptyA[s], ph ^ 1);
-          sm100::mbar_arrive_expect_tx(&fullA[s], (uint32_t)stage_bytes);
-          sm100::tma_load_4d(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t + 1);
+          sm100::mbar_arrive_expect_tx_warp(&fullA[s], (uint32_t)stage_bytes);
+          sm100::tma_load_4d_warp(sA + s * stage_bytes, &mapA, &fullA[s], 0, 0, kb, t + 1);
           if (++s == SA) { s = 0; ph ^= 1; }
         }
       }
