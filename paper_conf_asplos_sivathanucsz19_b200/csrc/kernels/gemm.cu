@@ -163,7 +163,7 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   ASTRA_CHECK_ARG(BN == 64 || BN == 128 || BN == 256 || BN == 224, "tc_gemm: BN must be 64, 128, 224 or 256");
   ASTRA_CHECK_ARG(M > 0 && N > 0 && K > 0, "tc_gemm: empty problem");
   // multi-k-block stages (TcArgs::kb; tc_gemm_kernel without a cluster): the largest of 4 / 2 that
-  // divides the per-chunk k-block count and still leaves >= 3 stages; K-major operands need K % 64 == 0
+  // fits the per-chunk k-block count and still leaves >= 3 stages; K-major operands need K % 64 == 0
   // (their 4-D view reads whole 64-element k-blocks)
   int KB = 1;
   {
@@ -184,7 +184,10 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
         const int sb = kb * (a_kb + BN * TC_BK * 2);
         const int epi_bytes = TC_EPI_WARPS * 2 * 32 * 32 * 4;
         const int st = std::min(10, (maxs - 1024 - 256 - epi_bytes) / sb);
-        if (kper % kb == 0 && st >= 3) {
+        // a chunk whose k-block count kb does not divide ends in a partial stage (the box still
+        // lands kb tiles; the extra ones are never multiplied): allowed up to 25 % extra bytes
+        const int waste = (kper + kb - 1) / kb * kb - kper;
+        if (kper >= kb && 4 * waste <= kper && st >= 3) {
           KB = kb;
           break;
         }

@@ -472,7 +472,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           if (kb == kb0 && local == 0) GEMM_TRACE(3);
           sm100::tc_fence_after();
           const uint64_t ad0 = dA0 + (uint64_t)(s * (stage_bytes >> 4)), bd0 = dB0 + (uint64_t)(s * (stage_bytes >> 4));
-          for (int j = 0; j < KB; ++j) {
+          const int nj = kb1 - kb < KB ? kb1 - kb : KB;   // a chunk's last stage may be partial
+          for (int j = 0; j < nj; ++j) {
             const uint64_t ad = ad0 + j * a_j, bd = bd0 + j * b_j;
 #pragma unroll
             for (int kk = 0; kk < TC_BK / 16; ++kk)
