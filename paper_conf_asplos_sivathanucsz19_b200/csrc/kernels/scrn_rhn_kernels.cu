@@ -8,7 +8,7 @@
 
 namespace astra {
 
-constexpr int PW_UX = 64;  // units per CTA
+constexpr int PW_UX = 32;  // units per CTA (a warp = 32 consecutive units of one row lane; the sums are per unit, so the CTA width never changes a bit)
 constexpr int PW_RY = 8;   // row lanes per CTA
 constexpr int PW_RB = 32;  // rows per CTA
 int pw_row_chunks(int B) { return cdiv(B, PW_RB); }
