@@ -28,9 +28,10 @@ namespace astra {
 
 namespace {
 
-constexpr int RH_EPI_WARPS = 8;
-constexpr int RH_THREADS = 64 + 32 * RH_EPI_WARPS;   // warp 0 TMA, warp 1 MMA, 8 epilogue warps (two per
-                                                      // TMEM lane quarter, one per 16-unit half of the tile)
+constexpr int RH_EPI_WARPS = 16;
+constexpr int RH_THREADS = 64 + 32 * RH_EPI_WARPS;   // warp 0 TMA, warp 1 MMA, 16 epilogue warps (four per
+                                                      // TMEM lane quarter, one per 8-unit quarter of the tile)
+constexpr int RH_UW = 32 * 4 / (RH_EPI_WARPS);        // units per epilogue thread (8)
 constexpr int RH_UB = 32;                             // hidden units per tile
 constexpr int RH_BN = 2 * RH_UB;                      // MMA N: the units' H-columns then their T-columns
 constexpr int RH_SP = RH_UB + 1;                      // row strides of the per-thread (row) shared buffers,
@@ -206,10 +207,11 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       }
     }
   } else {
-    // ------------------------------------------------------------ highway epilogue (8 warps)
+    // ------------------------------------------------------------ highway epilogue (16 warps)
     const int quarter = warp & 3;            // TMEM lane quarter of this warp
-    const int uc = (warp - 2) / 4;           // the 16-unit half of the tile this warp applies (round 2:
-                                             // the two halves ran one after the other in 4 warps)
+    const int uc = (warp - 2) / 4;           // the RH_UW-unit part of the tile this warp applies: at B ≤ 64
+                                             // only the warps of lane quarters 0 / 1 have rows, so the
+                                             // units are spread over four of them per quarter
     const int row = quarter * 32 + lane;
     const int m = m0 + row;
     const bool valid = m < a.B;
@@ -228,28 +230,38 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       float* spr = sprev + row * RH_SP;   // valid rows only (m < B ≤ a_rows when a_rows = 64)
       float* zr = zst + row * RH_ZP;
       {
-        const int ul = uc * 16;
-        float xh[16], xt[16];
+        const int ul = uc * RH_UW;
+        float xh[RH_UW], xt[RH_UW];
         if (l == 0 && valid) {   // x_t·W (ℓ = 1 only): independent of the MMA, issued first
 #pragma unroll
-          for (int q4 = 0; q4 < 4; ++q4) {
+          for (int q4 = 0; q4 < RH_UW / 4; ++q4) {
             const float4 h4 = reinterpret_cast<const float4*>(wx + u0 + ul)[q4];
             const float4 t4 = reinterpret_cast<const float4*>(wx + a.Hp + u0 + ul)[q4];
             xh[4 * q4] = h4.x; xh[4 * q4 + 1] = h4.y; xh[4 * q4 + 2] = h4.z; xh[4 * q4 + 3] = h4.w;
             xt[4 * q4] = t4.x; xt[4 * q4 + 1] = t4.y; xt[4 * q4 + 2] = t4.z; xt[4 * q4 + 3] = t4.w;
           }
         }
-        float zh[16], zt[16];
-        sm100::tmem_ld16(taddr + ul, zh);
-        sm100::tmem_ld16(taddr + RH_UB + ul, zt);
-        for (int c = 1; c < a.nsplit; ++c) {   // chunk partials summed in chunk order (rhn_fwd_pw)
-          float ph[16], pt[16];
-          sm100::tmem_ld16(taddr + c * RH_BN + ul, ph);
-          sm100::tmem_ld16(taddr + c * RH_BN + RH_UB + ul, pt);
+        float zh[RH_UW], zt[RH_UW];
+        {
+          uint32_t rh[RH_UW], rt[RH_UW];
+          sm100::tmem_ld8_nowait(taddr + ul, rh);
+          sm100::tmem_ld8_nowait(taddr + RH_UB + ul, rt);
+          sm100::tmem_wait_ld();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            zh[i] = __fadd_rn(zh[i], ph[i]);
-            zt[i] = __fadd_rn(zt[i], pt[i]);
+          for (int i = 0; i < RH_UW; ++i) {
+            zh[i] = __uint_as_float(rh[i]);
+            zt[i] = __uint_as_float(rt[i]);
+          }
+        }
+        for (int c = 1; c < a.nsplit; ++c) {   // chunk partials summed in chunk order (rhn_fwd_pw)
+          uint32_t ph[RH_UW], pt[RH_UW];
+          sm100::tmem_ld8_nowait(taddr + c * RH_BN + ul, ph);
+          sm100::tmem_ld8_nowait(taddr + c * RH_BN + RH_UB + ul, pt);
+          sm100::tmem_wait_ld();
+#pragma unroll
+          for (int i = 0; i < RH_UW; ++i) {
+            zh[i] = __fadd_rn(zh[i], __uint_as_float(ph[i]));
+            zt[i] = __fadd_rn(zt[i], __uint_as_float(pt[i]));
           }
         }
         if (a.trace && warp == 4 && lane == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + (uc == 0 ? 5 : 11)] = global_ns();
@@ -257,16 +269,16 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
         __nv_bfloat16* so = a.Sop + slot_out + (size_t)m * a.Hp + u0 + ul;
         // every shared-memory operand into registers first, results out after: the buffers share
         // one base, so interleaved loads and stores would serialise the 16 units' dependency chains
-        float sv[16], bh[16], bt[16];
+        float sv[RH_UW], bh[RH_UW], bt[RH_UW];
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
+        for (int i = 0; i < RH_UW; ++i) {
           sv[i] = spr[ul + i];
           bh[i] = bl[ul + i];
           bt[i] = bl[RH_UB + ul + i];
         }
-        float snew[16];
+        float snew[RH_UW];
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
+        for (int i = 0; i < RH_UW; ++i) {
           const int j = u0 + ul + i;
           float s_new = 0.f, aH = 0.f, aT = 0.f;
           if (j < a.H) {
@@ -284,14 +296,14 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           snew[i] = s_new;
         }
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
+        for (int i = 0; i < RH_UW; ++i) {
           spr[ul + i] = snew[i];   // s^ℓ: the next micro-step's s^{ℓ−1} of this row and unit
           zr[ul + i] = zh[i];
           zr[RH_UB + ul + i] = zt[i];
         }
         if (last) {
 #pragma unroll
-          for (int i = 0; i < 16; ++i) {
+          for (int i = 0; i < RH_UW; ++i) {
             const int j = u0 + ul + i;
             if (j >= a.H) break;
             if (a.y) a.y[((size_t)t * a.B + m) * a.ldy + j] = __float2bfloat16_rn(snew[i]);
@@ -299,15 +311,15 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
           }
         }
         if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 9] = global_ns();
-        uint4 pk[2];
+        uint4 pk[RH_UW / 8];
         uint32_t* pu = reinterpret_cast<uint32_t*>(pk);
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
+        for (int i = 0; i < RH_UW / 2; ++i) {
           __nv_bfloat162 b2 = __floats2bfloat162_rn(snew[2 * i], snew[2 * i + 1]);
           pu[i] = *reinterpret_cast<uint32_t*>(&b2);
         }
-        reinterpret_cast<uint4*>(so)[0] = pk[0];
-        reinterpret_cast<uint4*>(so)[1] = pk[1];
+#pragma unroll
+        for (int i = 0; i < RH_UW / 8; ++i) reinterpret_cast<uint4*>(so)[i] = pk[i];
         if (a.trace && warp == 4 && lane == 0 && uc == 0) a.trace[((size_t)blockIdx.x * nsteps + q) * 12 + 10] = global_ns();
         }
       }
@@ -328,7 +340,7 @@ __global__ void __launch_bounds__(RH_THREADS, 1)
       if (valid) {
         float* sn = a.Sf + slot_out + (size_t)m * a.Hp + u0;
 #pragma unroll
-        for (int q4 = 4 * uc; q4 < 4 * uc + 4; ++q4) {   // this warp's 16 units
+        for (int q4 = (RH_UW / 4) * uc; q4 < (RH_UW / 4) * (uc + 1); ++q4) {   // this warp's units
           const int o = 4 * q4;
           reinterpret_cast<float4*>(sn)[q4] = make_float4(spr[o], spr[o + 1], spr[o + 2], spr[o + 3]);
           reinterpret_cast<float4*>(Z + u0)[q4] = make_float4(zr[o], zr[o + 1], zr[o + 2], zr[o + 3]);
