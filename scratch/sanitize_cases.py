@@ -19,9 +19,18 @@ elif case == "bptt_fused":     # fused BPTT step (bwd=1)
 elif case == "rhn_fused":      # persistent RHN forward (fwd=1)
     p, inp, dY, dhT, dcT = make_cell_case("rhn", 2, 16, 64, 64, 5, bf16=True, L=2)
     run_gpu_cell("rhn", p, inp, dY, dhT, dcT, "bf16", "fwd=1", depth=2)
-elif case == "bptt_persist":   # small-batch persistent BPTT (bwd=3)
-    p, inp, dY, dhT, dcT = make_cell_case("milstm", 3, 16, 64, 128, 5, bf16=True)
-    run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", "bwd=3")
+elif case == "bptt_persist":   # small-batch persistent BPTT (bwd=2: clusters of 4, needs 4 K chunks: H >= 2048)
+    p, inp, dY, dhT, dcT = make_cell_case("milstm", 2, 16, 64, 2048, 5, bf16=True)
+    run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", "bwd=2")
+elif case == "scrn_persist":   # SC-RNN persistent forward + BPTT (fwd=1, bwd=1)
+    p, inp, dY, dhT, dcT = make_cell_case("scrn", 3, 16, 64, 128, 5, bf16=True, S=128)
+    run_gpu_cell("scrn", p, inp, dY, dhT, dcT, "bf16", "fwd=1,bwd=1", context=128, scrn_alpha=0.95)
+elif case == "gemm_kb":        # K1 with multi-k-block stages (K-major and MN-major, partial last stage)
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    for (M, N, K, amn, bmn, ks) in ((64, 256, 512, 0, 0, 1), (64, 256, 448, 0, 1, 1), (128, 128, 1792, 1, 1, 4)):
+        a = (torch.randn(K, M) if amn else torch.randn(M, K)).cuda().to(torch.bfloat16)
+        b = (torch.randn(K, N) if bmn else torch.randn(N, K)).cuda().to(torch.bfloat16)
+        A.gemm_bf16_ex(a, b, M, N, K, a_mn=bool(amn), b_mn=bool(bmn), bn=64, ksplit=ks)
 else:
     raise SystemExit(f"unknown case {case}")
 torch.cuda.synchronize()
