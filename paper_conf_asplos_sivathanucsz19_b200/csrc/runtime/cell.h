@@ -205,6 +205,7 @@ class Cell {
   virtual bool chain_prefetch() const { return false; }   // supports Variant::l2pf (tuner AVs pf_fwd / pf_bwd)
   virtual bool supports_recompute() const { return false; }   // Variant::recomp (tuner root fork "recomp")
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
+  virtual const char* fwd_fusion_metric() const { return "t_fwd"; }   // the region that judges it
   virtual int bwd_fusions() const { return 1; }   // number of K4 fusion choices (tuner AV "fuse_bwd")
   virtual int gate_chunkings() const { return 1; }   // options of the tuner AV "gate_chunking" (1: none)
   virtual int wgrad_schedules() const { return 1; }  // options of the tuner AV "wgrad_schedule" (1: none)

@@ -12,6 +12,7 @@
 //            (K1, accumulated); LSTM cell backward; then the weight gradients, the keys backward
 //            (dW_k, denc += dk·W_kᵀ) and the encoder BPTT driven by denc.                   (a5, a6)
 #include "../kernels/cell_math.cuh"
+#include "../kernels/rec_fused.h"
 #include "cell.h"
 
 namespace astra {
@@ -117,7 +118,13 @@ class AttnCell : public Cell {
     enc->main_st = main_st;
     enc->side = side;
     enc->var = var;
+    // the attention cell's fuse_fwd AV acts on the encoder chain: 1 = the small-batch persistent
+    // forward (fwd_mode 3, B ≤ 128) — the decoder step has no fused form
+    enc->var.fwd_mode = var.fwd_mode == 1 ? 3 : 0;
   }
+  int fwd_fusions() const override { return (ot == OT::BF16 && lstm_fwd_persist_supported(B, Hp)) ? 2 : 1; }
+  // the encoder runs outside the decoder-chain region: the choice is judged on the whole step
+  const char* fwd_fusion_metric() const override { return "t_step"; }
 
   void forward(const void* x, const float* h0, const float* c0, void* y, float* hT, float* cT) override {
     ASTRA_CHECK_STATE(bound, "step_fwd: call astra_bind first");

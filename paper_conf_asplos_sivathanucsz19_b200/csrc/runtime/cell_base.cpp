@@ -418,7 +418,7 @@ void Cell::tuner_setup() {
   // reading R26: the forward fusion choice (GEMM + pointwise kernel vs the fused recurrent kernel,
   // P:120-126 "fusion" AV) is tuned after the kernel choices, against the forward-chain time
   if (ot == OT::BF16 && fwd_fusions() > 1)
-    t = "(pre " + t + " (leaf fuse_fwd " + std::to_string(fwd_fusions()) + " t_fwd))";
+    t = "(pre " + t + " (leaf fuse_fwd " + std::to_string(fwd_fusions()) + " " + fwd_fusion_metric() + "))";
   if (ot == OT::BF16 && bwd_fusions() > 1)
     t = "(pre " + t + " (leaf fuse_bwd " + std::to_string(bwd_fusions()) + " t_bptt))";
   // the backward pointwise kernel's form (bwd_kernel AV), against the BPTT-chain time

@@ -63,15 +63,20 @@ def attn_run(name, H, I, A_, B, Ts, Tt, steps=10):
         c.backward(dY, None, None, dx, None, None)
         c.sgd(0.01)
 
-    c.tune_mode(A.TUNE_ON)
+    import os
     n = 0
-    while True:
-        step()
-        n += 1
-        if c.tune_next() == A.TUNE_CONVERGED or n > 1000:
-            break
-    rep = c.tune_report()
-    c.tune_mode(A.TUNE_FROZEN, rep["variant"])
+    if os.environ.get("CFG_VARIANT"):   # A/B runs: a forced variant, no exploration
+        c.tune_mode(A.TUNE_FROZEN, os.environ["CFG_VARIANT"])
+        rep = {"variant": os.environ["CFG_VARIANT"]}
+    else:
+        c.tune_mode(A.TUNE_ON)
+        while True:
+            step()
+            n += 1
+            if c.tune_next() == A.TUNE_CONVERGED or n > 1000:
+                break
+        rep = c.tune_report()
+        c.tune_mode(A.TUNE_FROZEN, rep["variant"])
     for _ in range(3): step()
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

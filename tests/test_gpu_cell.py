@@ -364,11 +364,13 @@ def _attn_case(Ts, Tt, B, I, H, A, seed, bf16):
     return p, inp, dY, synth.normal(seed, "dhT", (B, H)), synth.normal(seed, "dcT", (B, H))
 
 
-def _attn_check(Ts, Tt, B, I, H, A, dtype, seed, tol):
+def _attn_check(Ts, Tt, B, I, H, A, dtype, seed, tol, variant=None):
     import paper_conf_asplos_sivathanucsz19_b200 as AS
     p, inp, dY, dhT, dcT = _attn_case(Ts, Tt, B, I, H, A, seed, dtype == "bf16")
     out_o, g_o = C.cell_fwd_bwd("attn", p, inp, dY, dhT, dcT)
     c = AS.Cell("attn", H, I, B, Tt, dtype=dtype, src_seq=Ts, attn_dim=A)
+    if variant is not None:
+        c.tune_mode(AS.TUNE_FROZEN, variant)
     c.load(p)
     dev = c.device
     tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
@@ -392,6 +394,18 @@ def _attn_check(Ts, Tt, B, I, H, A, dtype, seed, tol):
     errs = {k: rel_err(got[k], ref[k]) for k in ref}
     bad = {k: v for k, v in errs.items() if not v <= tol}
     assert not bad, (dtype, bad, errs)
+    return got
+
+
+@pytest.mark.parametrize("Ts,Tt,B,H", [(6, 4, 128, 256), (5, 3, 37, 128)])
+def test_attn_encoder_persistent_bitwise(Ts, Tt, B, H):
+    """The attention cell's fuse_fwd AV runs its encoder chain as the small-batch persistent forward
+    (fwd=1 → encoder fwd_mode 3): every output and gradient bitwise equal to the launched encoder
+    chain (fwd=0), both against the oracle."""
+    ga = _attn_check(Ts, Tt, B, 64, H, H, "bf16", synth.config_seed(4) + 7, TOL_BF16, variant="fwd=0")
+    gb = _attn_check(Ts, Tt, B, 64, H, H, "bf16", synth.config_seed(4) + 7, TOL_BF16, variant="fwd=1")
+    for k in ga:
+        assert np.array_equal(ga[k], gb[k]), k
 
 
 @pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
