@@ -254,44 +254,53 @@ __global__ void __launch_bounds__(ATT_THREADS)
   __syncthreads();
   if (x >= n) return;
   const float* cx = col + threadIdx.x;
-  // terms of 8 steps are formed independently (instruction-level parallelism), then added in order
-  constexpr int IG = 8;
+  // four source positions j at a time: four independent accumulators (instruction-level
+  // parallelism, q_i / dctx_i read once for the four), each still summed over i in the loop's order
+  constexpr int JB = 4;
   if (z == 0) {
-    for (int j = 0; j < Ts; ++j) {
-      float acc = 0.f;
-      for (int i0 = T_ - 1; i0 >= 0; i0 -= IG) {
-        float t[IG];
+    for (int j0 = 0; j0 < Ts; j0 += JB) {
+      float acc[JB];
 #pragma unroll
-        for (int k = 0; k < IG; ++k) t[k] = i0 - k >= 0 ? __fmul_rn(sh[(i0 - k) * Ts + j], cx[(i0 - k) * ATT_THREADS]) : 0.f;
+      for (int jj = 0; jj < JB; ++jj) acc[jj] = 0.f;
+      for (int i = T_ - 1; i >= 0; --i) {
+        const float c = cx[i * ATT_THREADS];
 #pragma unroll
-        for (int k = 0; k < IG; ++k)
-          if (i0 - k >= 0) acc = i0 - k == T_ - 1 ? t[k] : __fadd_rn(acc, t[k]);
+        for (int jj = 0; jj < JB; ++jj) {
+          if (j0 + jj >= Ts) break;
+          const float add = __fmul_rn(sh[i * Ts + j0 + jj], c);
+          acc[jj] = i == T_ - 1 ? add : __fadd_rn(acc[jj], add);
+        }
       }
-      denc[((long)j * B + b) * Hp + x] = acc;
+#pragma unroll
+      for (int jj = 0; jj < JB; ++jj)
+        if (j0 + jj < Ts) denc[((long)(j0 + jj) * B + b) * Hp + x] = acc[jj];
     }
   } else {
     const bool valid = x < A;
     const float va = valid ? v[x] : 0.f;
-    for (int j = 0; j < Ts; ++j) {
-      const float kj = valid ? keys[((long)j * B + b) * Ap + x] : 0.f;
-      float acc = 0.f;
-      for (int i0 = T_ - 1; i0 >= 0; i0 -= IG) {
-        float t[IG];
+    for (int j0 = 0; j0 < Ts; j0 += JB) {
+      float kj[JB], acc[JB];
 #pragma unroll
-        for (int k = 0; k < IG; ++k) {
-          const int i = i0 - k;
-          float du = 0.f;
-          if (valid && i >= 0) {
-            const float u = tanh_<FastMath<T>::value>(__fadd_rn(cx[i * ATT_THREADS], kj));
-            du = __fmul_rn(__fmul_rn(sh[i * Ts + j], va), __fsub_rn(1.f, __fmul_rn(u, u)));
-          }
-          t[k] = du;
-        }
-#pragma unroll
-        for (int k = 0; k < IG; ++k)
-          if (i0 - k >= 0) acc = i0 - k == T_ - 1 ? t[k] : __fadd_rn(acc, t[k]);
+      for (int jj = 0; jj < JB; ++jj) {
+        kj[jj] = (valid && j0 + jj < Ts) ? keys[((long)(j0 + jj) * B + b) * Ap + x] : 0.f;
+        acc[jj] = 0.f;
       }
-      dk[((long)j * B + b) * Ap + x] = acc;
+      for (int i = T_ - 1; i >= 0; --i) {
+        const float qi = cx[i * ATT_THREADS];
+#pragma unroll
+        for (int jj = 0; jj < JB; ++jj) {
+          if (j0 + jj >= Ts) break;
+          float du = 0.f;
+          if (valid) {
+            const float u = tanh_<FastMath<T>::value>(__fadd_rn(qi, kj[jj]));
+            du = __fmul_rn(__fmul_rn(sh[i * Ts + j0 + jj], va), __fsub_rn(1.f, __fmul_rn(u, u)));
+          }
+          acc[jj] = i == T_ - 1 ? du : __fadd_rn(acc[jj], du);
+        }
+      }
+#pragma unroll
+      for (int jj = 0; jj < JB; ++jj)
+        if (j0 + jj < Ts) dk[((long)(j0 + jj) * B + b) * Ap + x] = acc[jj];
     }
   }
 }
