@@ -214,6 +214,28 @@ void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, 
   LAUNCH_CHECK();
 }
 
+__global__ void transpose_bf16_kernel(const __nv_bfloat16* __restrict__ src, int rows, int cols,
+                                      __nv_bfloat16* __restrict__ dst) {
+  __shared__ __nv_bfloat16 tile[32][34];
+  const long base = (long)blockIdx.z * rows * cols;
+  const int c0 = blockIdx.x * 32, r0 = blockIdx.y * 32, tx = threadIdx.x, ty = threadIdx.y;
+  for (int i = ty; i < 32; i += 8) {
+    const int r = r0 + i, c = c0 + tx;
+    tile[i][tx] = (r < rows && c < cols) ? src[base + (long)r * cols + c] : __float2bfloat16_rn(0.f);
+  }
+  __syncthreads();
+  for (int i = ty; i < 32; i += 8) {
+    const int c = c0 + i, r = r0 + tx;
+    if (c < cols && r < rows) dst[base + (long)c * rows + r] = tile[tx][i];
+  }
+}
+
+void transpose_bf16(const void* src, int nb, int rows, int cols, void* dst, cudaStream_t st) {
+  dim3 grid(cdiv(cols, 32), cdiv(rows, 32), nb), block(32, 8);
+  transpose_bf16_kernel<<<grid, block, 0, st>>>((const __nv_bfloat16*)src, rows, cols, (__nv_bfloat16*)dst);
+  LAUNCH_CHECK();
+}
+
 template <typename TD, typename TS>
 __global__ void copy_pad_kernel(const TS* __restrict__ src, long rows, int cols, long lds, TD* __restrict__ dst,
                                 long ldd, long dcols) {

@@ -94,6 +94,8 @@ void attn_acc(OT ot, int T, int B, int Ts, int Hp, int A, int Ap, const float* p
               cudaStream_t st);
 
 // ---- LM pieces
+// dst[b][c][r] = src[b][r][c] for nb bf16 matrices of rows x cols (the RHN BPTT's K-major R copy)
+void transpose_bf16(const void* src, int nb, int rows, int cols, void* dst, cudaStream_t st);
 void embed_gather(OT ot, const int32_t* tok, long n, const float* E, int I, void* X, long ldx, cudaStream_t st);
 // rowloss[r] = lse - logit[target]; dlog (ot) and dlog32 = (softmax - onehot) * inv_n.
 void ce_fwd_bwd(OT ot, const float* logits, long ldl, int V, const int32_t* targets, long n, float inv_n,

@@ -195,6 +195,27 @@ bool lstm_bptt_persist_fits(int kind, int B, int Hp, int NG);
 void lstm_bptt_persist_launch(int kind, bool dy_f32, const void* Duh, const void* Um, int Tmax, BpttPersistArgs a,
                               cudaStream_t st);
 
+// Persistent RHN BPTT chain (rhn_bptt_persist.cu, RhnCell bwd_mode 1): all T·L backward micro-steps in
+// one cooperative launch of clusters of 4 CTAs (the R33 chunks), 32 units per cluster, the chunk
+// partials exchanged over distributed shared memory; B ≤ 64, nsplit == 4.
+struct RhnBpttArgs {
+  int B, H, Hp, T, L, nsplit, nchunk;
+  int nk, kper;             // set by the launcher
+  uint32_t idesc;
+  const void* dy;           // fp32 [T·B][ldy] (LM, ldy = Hp) or bf16 [T·B][ldy] (external, ldy = H)
+  long ldy;
+  const float* Apre;        // [L][T][B][2Hp]
+  const float* Sf;          // fp32 states, RhnCell::slot layout
+  __nv_bfloat16* DA;        // [L][T][B][2Hp]
+  float* dS;                // [B][Hp]: ds_T in, ds of s^0_0 out
+  float* part;              // [L][nchunk][2][Hp] db partials
+  unsigned* flags;          // one counter, zeroed before the launch
+};
+bool rhn_bptt_persist_supported(int B, int Hp, int nsplit, int L);
+bool rhn_bptt_persist_fits(int B, int Hp, int nsplit, int L);
+// DA: the DA base; RK: the K-major R copy [L][Hp][2Hp] (rows = units)
+void rhn_bptt_persist_launch(bool dy_f32, const void* DA, const void* RK, RhnBpttArgs a, cudaStream_t st);
+
 bool lstm_bptt_fused_supported(int B, int Hp, int nsplit);
 void lstm_bptt_fused_launch(int kind, bool dy_bf16, const BpttFusedMaps& m, BpttFusedArgs a, cudaStream_t st);
 

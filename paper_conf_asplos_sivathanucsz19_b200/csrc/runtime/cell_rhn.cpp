@@ -20,7 +20,7 @@ class RhnCell : public Cell {
  public:
   int L, G2, nchunk;
   size_t off_X, off_WX, off_Apre, off_Sf, off_Sop, off_MW, off_MR;
-  size_t off_DA, off_dS, off_dSpart, off_Zpart, off_part, off_flags;
+  size_t off_DA, off_dS, off_dSpart, off_Zpart, off_part, off_flags, off_RK;
 
   // Reading R33: the BPTT GEMM ds·R_ℓᵀ (K = 2·Hp, few output tiles at small batch) is split over K
   // into s fixed chunks, each accumulated from zero; the next pointwise kernel adds the partials in
@@ -64,6 +64,7 @@ class RhnCell : public Cell {
     off_Zpart = c.take((size_t)fwd_ksplit() * B * G2 * 4);
     off_part = c.take((size_t)L * nchunk * G2 * 4);
     off_flags = c.take(4096);
+    off_RK = c.take((size_t)L * Hp * G2 * e);   // K-major R copy of the persistent BPTT (bwd_mode 1)
     scratch_bytes = c.o;
   }
 
@@ -77,6 +78,14 @@ class RhnCell : public Cell {
   // K2 choices (AV fuse_fwd): GEMM + pointwise launch per micro-step, or the persistent fused chain
   bool fused_fwd_ok() const { return ot == OT::BF16 && rhn_rec_fwd_supported(B, Hp, fwd_ksplit()); }
   int fwd_fusions() const override { return fused_fwd_ok() ? 2 : 1; }
+  // K4 persistent BPTT (rhn_bptt_persist.cu, bwd=1): a frozen-variant option.  At cfg3 its chain is
+  // faster than the launched one when both are enqueued eagerly (2.79 vs 2.94 ms) but not against the
+  // CUDA-graph replay the LM steps run in (5.98 vs 5.93 ms per step, profiles/r2_cfg56.jsonl), and
+  // the tuner explores eagerly — so it is not offered to the tuner.
+  bool persist_bwd_ok() const {
+    return ot == OT::BF16 && rhn_bptt_persist_supported(B, Hp, bptt_ksplit(), L) &&
+           rhn_bptt_persist_fits(B, Hp, bptt_ksplit(), L);
+  }
 
   void* x_operand() override { return sv<char>(off_X); }
   Mat2 y_operand() override { return mat(Sop(0, 1), Hp, (long)T * B, Hp); }
@@ -198,7 +207,19 @@ class RhnCell : public Cell {
     float* dSpart = sc<float>(off_dSpart);
     EpiStore ep = epi(dSpart, Hp, B, Hp);
     ep.split_stride = (long)B * Hp;
-    for (int t = T - 1; t >= 0; --t) {
+    const bool persist = var.bwd_mode == 1 && persist_bwd_ok();
+    if (persist) {   // the whole chain in one launch; R_ℓ as a K-major copy (rows = units)
+      transpose_bf16(MR, L, G2, Hp, sc<char>(off_RK), st);
+      RhnBpttArgs pa{};
+      pa.B = B; pa.H = H; pa.Hp = Hp; pa.T = T; pa.L = L; pa.nsplit = bp.ksplit; pa.nchunk = nchunk;
+      if (lm_mode) { pa.dy = lm_dy; pa.ldy = Hp; }
+      else { pa.dy = dy; pa.ldy = H; }
+      pa.Apre = Apre(0, 0); pa.Sf = Sf(0, 0); pa.DA = (__nv_bfloat16*)DA(0, 0); pa.dS = dS; pa.part = part;
+      pa.flags = sc<unsigned>(off_flags);
+      CUDA_TRY(cudaMemsetAsync(pa.flags, 0, 64, st));
+      rhn_bptt_persist_launch(lm_mode, DA(0, 0), sc<char>(off_RK), pa, st);
+    }
+    for (int t = persist ? -1 : T - 1; t >= 0; --t) {
       for (int l = L - 1; l >= 0; --l) {
         const void* dyt = nullptr;
         if (l == L - 1)
@@ -209,7 +230,7 @@ class RhnCell : public Cell {
         run_gemm(2, bp, ep, l * T + t, l, var.g[G_BPTT], st);
       }
     }
-    add_split_partials(dS, dSpart, bp.ksplit, (long)B * Hp, st);   // ds of s^0_0
+    if (!persist) add_split_partials(dS, dSpart, bp.ksplit, (long)B * Hp, st);   // ds of s^0_0
     if (ds0) copy_pad(OT::F32, dS, OT::F32, B, H, Hp, ds0, H, st);
     mark(R_BPTT, 1, st);
 

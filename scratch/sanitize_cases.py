@@ -31,6 +31,9 @@ elif case == "gemm_kb":        # K1 with multi-k-block stages (K-major and MN-ma
         a = (torch.randn(K, M) if amn else torch.randn(M, K)).cuda().to(torch.bfloat16)
         b = (torch.randn(K, N) if bmn else torch.randn(N, K)).cuda().to(torch.bfloat16)
         A.gemm_bf16_ex(a, b, M, N, K, a_mn=bool(amn), b_mn=bool(bmn), bn=64, ksplit=ks)
+elif case == "rhn_bptt":       # persistent RHN BPTT (bwd=1: clusters of 4, R33 split of 4)
+    p, inp, dY, dhT, dcT = make_cell_case("rhn", 2, 16, 64, 512, 5, bf16=True, L=2)   # Hp 512: split of 4
+    run_gpu_cell("rhn", p, inp, dY, dhT, dcT, "bf16", "bwd=1", depth=2)
 else:
     raise SystemExit(f"unknown case {case}")
 torch.cuda.synchronize()

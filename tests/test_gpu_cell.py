@@ -344,6 +344,35 @@ def test_rhn_fused_forward_bitwise(T, B, I, H, L):
     _check("rhn", T, B, I, H, "bf16", synth.config_seed(3) + 7, TOL_BF16, variant="fwd=1", L=L)
 
 
+@pytest.mark.parametrize("T,B,I,H,L", [(3, 64, 64, 830, 10), (2, 16, 32, 64, 2), (4, 37, 48, 200, 3), (1, 64, 64, 256, 2)])
+def test_rhn_persistent_bptt_bitwise(T, B, I, H, L):
+    """The persistent RHN BPTT chain (bwd=1: one cooperative launch of 4-CTA clusters = the R33
+    chunks, partials exchanged over distributed shared memory, the micro-step backward fused, db in
+    the row-lane order) gives the same bits as the per-micro-step pointwise + split-K GEMM launches
+    (bwd=0) — every gradient, dx, ds0 — with and without the fused forward, and matches the oracle;
+    the launch count drops, i.e. the persistent kernel really ran."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    p, inp, dY, dhT, dcT = make_cell_case("rhn", T, B, I, H, synth.config_seed(3) + 9, bf16=True, L=L)
+    ref, launches = None, {}
+    for v in ("bwd=0", "bwd=1", "bwd=1,fwd=1"):
+        n0 = A.launch_count()
+        out, g, _ = run_gpu_cell("rhn", p, inp, dY, dhT, dcT, "bf16", v, depth=L)
+        launches[v] = A.launch_count() - n0
+        cur = {**out, **g}
+        if ref is None:
+            ref = cur
+            continue
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    Hp = -(-H // 64) * 64
+    nk, s = -(-2 * Hp // 64), min(4, 64 // max(1, -(-B // 128) * -(-Hp // 64)))
+    while s > 1 and nk // s < 4:
+        s -= 1
+    if T * L > 1 and s == 4 and B <= 64:   # the persistent chain's shapes (R33 split of 4)
+        assert launches["bwd=1"] < launches["bwd=0"] - T * L, launches
+    _check("rhn", T, B, I, H, "bf16", synth.config_seed(3) + 9, TOL_BF16, variant="bwd=1", L=L)
+
+
 def test_rhn_cfg3_reduced():
     """cfg3 reduced rung: L = 10, H = I = 830, B = 64, T = 8 (bf16)."""
     _check("rhn", 8, 64, 830, 830, "bf16", synth.config_seed(3), TOL_BF16, L=10)
