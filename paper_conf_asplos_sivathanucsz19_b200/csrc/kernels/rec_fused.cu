@@ -196,7 +196,7 @@ __global__ void __launch_bounds__(RF_THREADS, 1)
           }
           const float* cp = a.C + r * a.Hp + u0 + ul;
           float* cn = a.C + (r + a.B) * a.Hp + u0 + ul;
-          __nv_bfloat16* hn = a.Hb + (r + a.B) * a.Hp + u0 + ul;
+          __nv_bfloat16* hn = a.Hb + (r + a.B) * (a.ldh ? a.ldh : (long)a.Hp) + u0 + ul;
           float cv[16], hv[16];
 #pragma unroll
           for (int i = 0; i < 16; ++i) {
@@ -269,7 +269,7 @@ void lstm_rec_fwd_launch(int kind, const CUtensorMap& mapA, const CUtensorMap& m
   int stages = (maxs - 1024 - 256 - 4 * 256 * 4) / S::STAGE_BYTES;
   if (stages > 4) stages = 4;
   a.stages = stages;
-  a.nk = cdiv(a.Hp, TC_BK);
+  a.nk = cdiv(a.K ? a.K : a.Hp, TC_BK);
   const int smem = rf_smem_bytes(stages, S::STAGE_BYTES, 4 * 256);
   const int grid = a.num_m * a.num_n;
   ASTRA_CHECK_ARG(!a.persistent || grid <= nsm, "fused recurrent kernel: persistent mode needs one CTA per SM");

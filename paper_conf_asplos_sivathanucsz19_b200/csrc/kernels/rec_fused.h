@@ -24,6 +24,9 @@ struct RecFwdArgs {
   float* cT;
   GateParams gp;
   unsigned* flags;          // [num_m] row-block counters (zeroed before a persistent launch)
+  int K = 0;                // contraction length of the recurrent GEMM (0: Hp; the attentive decoder's
+                            // K-concatenated [h | ctx]·[U_d; C_d] has K = 2Hp)
+  long ldh = 0;             // row stride of Hb (0: Hp; the decoder's [h | ctx] operand rows: 2Hp)
 };
 
 // CTA-pair fused forward step (rec_fused2.cu): one launch per step t.
@@ -120,6 +123,13 @@ struct RecPersistArgs {
   GateParams gp;
   unsigned* flags;          // one counter, zeroed before the launch
   unsigned long long* trace;   // optional (astra_debug_set_trace kind 2): [grid][t1-t0][6] globaltimer stamps
+  int K = 0;                // contraction length (0: Hp); the attentive decoder's [h | ctx]·[U_d; C_d]: 2Hp.
+                            // Hb rows and U-mirror rows then have stride K
+  long ldh = 0;             // row stride of Hb (0: K; set by the launcher)
+  int max_resident = -1;    // cap on the resident U k-blocks (-1: as many as fit); a one-step launch
+                            // streams its whole U slice through the ring (0) so the MMAs start at once
+  int b_old = 0;            // 1: the U mirror was written ≥ 2 launches back (PDL launch): the B producer
+                            // starts before the grid dependency resolves
 };
 bool lstm_fwd_persist_supported(int B, int Hp);
 // Hb: [(Tmax+1)][B][Hp] bf16 h operands; Um: the U mirror [NG][Hp] (tensor maps built per launch).

@@ -150,7 +150,7 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
     // ([k-block][gate strip][16 rows][64]).
     {   // whole warp: the *_warp TMA / arrive forms elect the issuing lane
       const uint64_t pol = sm100::l2_policy_evict_last();
-      pdl_wait();
+      if (!a.b_old) pdl_wait();
       if (R > 0) {
         sm100::mbar_arrive_expect_tx_warp(resbar, (uint32_t)(R * SB_BT));
         for (int kb = 0; kb < R; kb += 8) {
@@ -326,7 +326,7 @@ __global__ void __launch_bounds__(SB_THREADS, 1)
           __nv_bfloat162 b2 = __floats2bfloat162_rn(hv[2 * i], hv[2 * i + 1]);
           hw[i] = *reinterpret_cast<uint32_t*>(&b2);
         }
-        *reinterpret_cast<uint4*>(a.Hb + (r + a.B) * a.Hp + unit0) = hp;
+        *reinterpret_cast<uint4*>(a.Hb + (r + a.B) * a.ldh + unit0) = hp;
         hpk = hp;
 #pragma unroll
         for (int i = 0; i < 8; ++i) hv_keep[i] = hv[i];
@@ -409,7 +409,10 @@ void lstm_fwd_persist_launch(int kind, const void* Hb, const void* Um, int Tmax,
   auto knob = [](const char* n, int d) { const char* e = std::getenv(n); return e ? std::atoi(e) : d; };
   static const int k_ka = knob("ASTRA_SB_KA", 4), k_sa = knob("ASTRA_SB_SA", 3), k_kb = knob("ASTRA_SB_KB", 2),
                    k_sb = knob("ASTRA_SB_SB", 2), k_res = knob("ASTRA_SB_RES", -1);
-  a.nk = a.Hp / TC_BK;
+  const long K = a.K ? a.K : a.Hp;   // U-mirror rows and h rows have stride K
+  ASTRA_CHECK_ARG(K % TC_BK == 0, "persistent small-batch forward: K must be a multiple of 64");
+  a.ldh = K;
+  a.nk = (int)(K / TC_BK);
   a.a_rows = a.B <= 64 ? 64 : 128;
   a.a_bytes = a.a_rows * TC_BK * 2;
   a.ka = 1;
@@ -421,11 +424,17 @@ void lstm_fwd_persist_launch(int kind, const void* Hb, const void* Um, int Tmax,
   a.resident = a.nk;
   // the rest of shared memory holds resident U k-blocks; the streamed ones go through the B ring in
   // stages of kbs k-blocks (the streamed count is a multiple of kbs)
-  while (sb_smem_bytes(a) > maxs || (k_res >= 0 && a.resident > k_res) || (a.nk - a.resident) % a.kbs != 0) {
+  const int res_cap = a.max_resident >= 0 ? (k_res >= 0 ? std::min(k_res, a.max_resident) : a.max_resident) : k_res;
+  while (sb_smem_bytes(a) > maxs || (res_cap >= 0 && a.resident > res_cap) || (a.nk - a.resident) % a.kbs != 0) {
     a.sb = std::max(1, k_sb);
     --a.resident;
     ASTRA_CHECK_ARG(a.resident >= 0, "persistent small-batch forward: shared memory too small");
   }
+  if (a.max_resident == 0)   // streaming the whole slice: as deep a B ring as fits (≤ 8 stages)
+    while (a.sb < 8) {
+      ++a.sb;
+      if (sb_smem_bytes(a) > maxs) { --a.sb; break; }
+    }
   // instruction descriptor: D f32, A/B bf16 K-major, N = 64, M = 128
   a.idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(SB_N >> 3) << 17) | ((uint32_t)(TC_BM >> 4) << 24);
   // maps.  A: h as {64 k, rows B, k-block (stride 128 B), t}; B: U mirror rows as {64 k, unit row,
@@ -433,13 +442,13 @@ void lstm_fwd_persist_launch(int kind, const void* Hb, const void* Um, int Tmax,
   CUtensorMap mA, mB, mBr, mB1;
   {
     const long dims[4] = {64, a.B, a.nk, Tmax + 1};
-    const long str[3] = {(long)a.Hp * 2, 128, (long)a.B * a.Hp * 2};
+    const long str[3] = {K * 2, 128, (long)a.B * K * 2};
     const int box[4] = {64, a.a_rows, a.ka, 1};
     make_map_nd(&mA, Hb, 4, dims, str, box, 128);
   }
   {
     const long dims[4] = {64, a.NG, 4, a.nk};
-    const long str[3] = {(long)a.Hp * 2, (long)GATE_U * a.Hp * 2, 128};
+    const long str[3] = {K * 2, (long)GATE_U * K * 2, 128};
     const int box[4] = {64, SB_UC, 4, a.kbs};
     make_map_nd(&mB, Um, 4, dims, str, box, 128);
     const int boxr[4] = {64, SB_UC, 4, 8};
@@ -461,8 +470,14 @@ void lstm_fwd_persist_launch(int kind, const void* Hb, const void* Um, int Tmax,
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[1];
-  attr[0].id = cudaLaunchAttributeCooperative;   // every CTA resident: the per-step counter is a grid barrier
-  attr[0].val.cooperative = 1;
+  if (a.t1 - a.t0 > 1) {
+    attr[0].id = cudaLaunchAttributeCooperative;   // every CTA resident: the per-step counter is a grid barrier
+    attr[0].val.cooperative = 1;
+  } else {   // one step (no grid barrier): a PDL launch whose prologue overlaps the predecessor —
+             // h_{t−1} and U are read after pdl_wait, c_{t−1} / WX_t are ≥ 2 launches old
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  }
   cfg.attrs = attr;
   cfg.numAttrs = 1;
   CUDA_TRY(cudaLaunchKernelEx(&cfg, fn, mA, mB, mBr, mB1, a));

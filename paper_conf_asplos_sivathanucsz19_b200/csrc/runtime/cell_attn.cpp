@@ -118,11 +118,14 @@ class AttnCell : public Cell {
     enc->main_st = main_st;
     enc->side = side;
     enc->var = var;
-    // the attention cell's fuse_fwd AV acts on the encoder chain: 1 = the small-batch persistent
-    // forward (fwd_mode 3, B ≤ 128) — the decoder step has no fused form
-    enc->var.fwd_mode = var.fwd_mode == 1 ? 3 : 0;
+    // the attention cell's fuse_fwd AV (bf16): bit 0 runs the encoder chain as the small-batch
+    // persistent forward (fwd_mode 3, B ≤ 128); bit 1 runs each decoder step's K-concatenated
+    // recurrent GEMM with the LSTM gate epilogue fused (lstm_rec_fwd_kernel, one launch per step —
+    // the attention sub-step between steps rules out a persistent decoder)
+    enc->var.fwd_mode = (var.fwd_mode & 1) ? 3 : 0;
   }
-  int fwd_fusions() const override { return (ot == OT::BF16 && lstm_fwd_persist_supported(B, Hp)) ? 2 : 1; }
+  // modes 0..3 (bit 0 is a no-op where the persistent encoder is unsupported: B > 128)
+  int fwd_fusions() const override { return ot == OT::BF16 ? 4 : 1; }
   // the encoder runs outside the decoder-chain region: the choice is judged on the whole step
   const char* fwd_fusion_metric() const override { return "t_step"; }
 
@@ -189,14 +192,55 @@ class AttnCell : public Cell {
     qg.A = mat(HC(0), Hp, B, 2L * Hp, T + 1, (long)B * 2 * Hp);
     qg.B = mat(MWq, Hp, Ap, Hp);
     qg.M = B; qg.N = Ap; qg.K = Hp;
+    // K2 fused decoder step (fuse_fwd bit 1): the same MMAs in the same K order as the K1 GEMM below
+    // and cell_math.cuh's gate arithmetic on the bf16 path, so the same bits (R17)
+    const bool fused_dec = ot == OT::BF16 && (var.fwd_mode & 2);
+    const bool dec_persist = fused_dec && lstm_fwd_persist_supported(B, Hp);   // B ≤ 128: 16-unit tiles
+    RecPersistArgs pa{};
+    if (dec_persist) {
+      pa.B = B; pa.H = H; pa.Hp = Hp; pa.NG = NG; pa.T = T;
+      pa.WX = WXd; pa.UH = UHd; pa.C = Cd; pa.Hb = (__nv_bfloat16*)HC(0);
+      pa.y = y; pa.ldy = ldy; pa.y_kind = y ? 1 : 0;
+      pa.gp = gp;
+      pa.flags = nullptr;   // one step per launch: no grid barrier, the counter is never touched
+      pa.K = 2 * Hp;
+      pa.max_resident = 0;
+      pa.b_old = 1;   // MUC is mirrored at the start of forward, many launches before the decoder chain
+    }
+    RecFwdArgs ra{};
+    const TcGemm* tg = nullptr;
+    if (fused_dec && !dec_persist) {
+      tg = &tc_get(2, rec, KCfg{256, 1, 1}, true);
+      ra.B = B; ra.H = H; ra.Hp = Hp; ra.NG = NG; ra.T = T;
+      ra.num_m = cdiv(B, TC_BM); ra.num_n = NG / 256;
+      ra.idesc = tg->args.idesc;
+      ra.WX = WXd; ra.UH = UHd; ra.C = Cd; ra.Hb = (__nv_bfloat16*)HC(0);
+      ra.y = y; ra.ldy = ldy; ra.y_kind = y ? 1 : 0;
+      ra.gp = gp;
+      ra.persistent = 0;
+      ra.K = 2 * Hp;
+      ra.ldh = 2L * Hp;
+    }
     for (int i = 0; i < T; ++i) {
       float* UHi = UHd + (long)i * B * NG;
-      run_gemm(2, rec, epi(UHi, NG, B, NG), i, 0, var.g[G_REC], st);
       const bool last = i == T - 1;
-      lstm_fwd_pointwise(K_LSTM, ot, B, H, Hp, WXd + (long)i * B * NG, UHi, gp, Cd + (long)i * B * Hp,
-                         Cd + (long)(i + 1) * B * Hp, HC(i + 1), 2L * Hp,
-                         y ? (char*)y + (size_t)i * B * ldy * e : nullptr, ldy, ot, last ? hT : nullptr,
-                         last ? cT : nullptr, st);
+      if (dec_persist) {
+        pa.t0 = i; pa.t1 = i + 1;
+        pa.hT = last ? hT : nullptr;
+        pa.cT = last ? cT : nullptr;
+        lstm_fwd_persist_launch(K_LSTM, HC(0), MUC, T, pa, st);
+      } else if (fused_dec) {
+        ra.t0 = i; ra.t1 = i + 1;
+        ra.hT = last ? hT : nullptr;
+        ra.cT = last ? cT : nullptr;
+        lstm_rec_fwd_launch(K_LSTM, tg->mapA, tg->mapB, ra, st);
+      } else {
+        run_gemm(2, rec, epi(UHi, NG, B, NG), i, 0, var.g[G_REC], st);
+        lstm_fwd_pointwise(K_LSTM, ot, B, H, Hp, WXd + (long)i * B * NG, UHi, gp, Cd + (long)i * B * Hp,
+                           Cd + (long)(i + 1) * B * Hp, HC(i + 1), 2L * Hp,
+                           y ? (char*)y + (size_t)i * B * ldy * e : nullptr, ldy, ot, last ? hT : nullptr,
+                           last ? cT : nullptr, st);
+      }
       float* Qi = Q + (long)i * B * Ap;
       run_gemm(3, qg, epi(Qi, Ap, B, Ap), i + 1, 0, var.g[G_REC], st);
       attn_fwd(ot, B, Ts, H, Hp, A, Ap, Qi, Keys, p("v"), Encf, Pr + (long)i * B * Ts, sc<float>(off_att), HC(i + 1) + (size_t)Hp * e,

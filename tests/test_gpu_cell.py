@@ -426,15 +426,26 @@ def _attn_check(Ts, Tt, B, I, H, A, dtype, seed, tol, variant=None):
     return got
 
 
-@pytest.mark.parametrize("Ts,Tt,B,H", [(6, 4, 128, 256), (5, 3, 37, 128)])
+@pytest.mark.parametrize("Ts,Tt,B,H", [(6, 4, 128, 256), (5, 3, 37, 128), (3, 5, 160, 192)])
 def test_attn_encoder_persistent_bitwise(Ts, Tt, B, H):
-    """The attention cell's fuse_fwd AV runs its encoder chain as the small-batch persistent forward
-    (fwd=1 → encoder fwd_mode 3): every output and gradient bitwise equal to the launched encoder
-    chain (fwd=0), both against the oracle."""
+    """The attention cell's fuse_fwd AV: bit 0 runs its encoder chain as the small-batch persistent
+    forward (encoder fwd_mode 3), bit 1 runs each decoder step's K-concatenated recurrent GEMM with
+    the gate epilogue fused (lstm_rec_fwd_kernel, K = 2Hp).  Every output and gradient of modes 1-3
+    bitwise equal to the launched chains (fwd=0), all against the oracle.  B = 160: two row tiles,
+    a ragged one, and no persistent encoder (bit 0 is then a no-op)."""
+    import paper_conf_asplos_sivathanucsz19_b200 as AS
+    n0 = AS.launch_count()
     ga = _attn_check(Ts, Tt, B, 64, H, H, "bf16", synth.config_seed(4) + 7, TOL_BF16, variant="fwd=0")
-    gb = _attn_check(Ts, Tt, B, 64, H, H, "bf16", synth.config_seed(4) + 7, TOL_BF16, variant="fwd=1")
-    for k in ga:
-        assert np.array_equal(ga[k], gb[k]), k
+    launches = {0: AS.launch_count() - n0}
+    for mode in (1, 2, 3):
+        n0 = AS.launch_count()
+        gb = _attn_check(Ts, Tt, B, 64, H, H, "bf16", synth.config_seed(4) + 7, TOL_BF16, variant=f"fwd={mode}")
+        launches[mode] = AS.launch_count() - n0
+        for k in ga:
+            assert np.array_equal(ga[k], gb[k]), (mode, k)
+    # the fused decoder really ran: one launch per decoder step instead of GEMM + pointwise
+    # (B ≤ 128: the small-batch kernel run one step per launch; B = 160: lstm_rec_fwd_kernel)
+    assert launches[2] <= launches[0] - Tt, launches
 
 
 @pytest.mark.parametrize("dtype,tol", [("fp32", TOL_FP32), ("bf16", TOL_BF16)])
