@@ -26,14 +26,14 @@ __device__ __forceinline__ void store2<__nv_bfloat16>(__nv_bfloat16* p, float a,
 // ============================================================================ mirrors
 template <typename T>
 __global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int H, int Hp, T* __restrict__ dst,
-                                      long ldd, long kcols) {
+                                      long ldd, long kcols, int gu) {
   // tile 32 (k) x 32 (internal rows r); dst[r][k] = src[k][ext(r)]
   __shared__ float tile[32][33];
   const int r0 = blockIdx.x * 32, k0 = blockIdx.y * 32;
   const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
   for (int i = ty; i < 32; i += 8) {
     const int k = k0 + i, r = r0 + tx;
-    const int tileu = r / (4 * GATE_U), g = (r % (4 * GATE_U)) / GATE_U, j = tileu * GATE_U + r % GATE_U;
+    const int tileu = r / (4 * gu), g = (r % (4 * gu)) / gu, j = tileu * gu + r % gu;
     float v = 0.f;
     if (k < K && j < H) v = src[(long)k * 4 * H + g * H + j];
     tile[i][tx] = v;
@@ -49,12 +49,12 @@ __global__ void mirror_gates_T_kernel(const float* __restrict__ src, int K, int 
 // a warp one 128-byte run of a dst row) instead of one 2-byte element.  Same per-element rounding.
 template <typename T>
 __global__ void mirror_gates_T2_kernel(const float* __restrict__ src, int K, int H, int Hp, T* __restrict__ dst,
-                                       long ldd, long kcols) {
+                                       long ldd, long kcols, int gu) {
   __shared__ float tile[64][33];
   const int r0 = blockIdx.x * 32, k0 = blockIdx.y * 64;
   const int tx = threadIdx.x, ty = threadIdx.y;  // 32 x 8
   const int r = r0 + tx;
-  const int tileu = r / (4 * GATE_U), g = (r % (4 * GATE_U)) / GATE_U, j = tileu * GATE_U + r % GATE_U;
+  const int tileu = r / (4 * gu), g = (r % (4 * gu)) / gu, j = tileu * gu + r % gu;
   for (int i = ty; i < 64; i += 8) {
     const int k = k0 + i;
     tile[i][tx] = (k < K && j < H) ? src[(long)k * 4 * H + g * H + j] : 0.f;
@@ -70,10 +70,11 @@ __global__ void mirror_gates_T2_kernel(const float* __restrict__ src, int K, int
 // consecutive source columns g·H + j0 … (H % 4 == 0), 4 consecutive k per thread on the store side.
 template <typename T>
 __global__ void __launch_bounds__(256) mirror_gates_T4_kernel(const float* __restrict__ src, int K, int H, int Hp,
-                                                              T* __restrict__ dst, long ldd, long kcols) {
+                                                              T* __restrict__ dst, long ldd, long kcols, int gu) {
   __shared__ float tile[64][65];
   const int rb = blockIdx.x, k0 = blockIdx.y * 64, tid = threadIdx.x;
-  const int tileu = rb / 4, g = rb % 4, r0 = rb * 64, j0 = tileu * GATE_U;
+  // a 64-row block lies inside one gate of one unit block (gu is a multiple of 64)
+  const int r0 = rb * 64, g = (r0 % (4 * gu)) / gu, j0 = (r0 / (4 * gu)) * gu + r0 % gu;
 #pragma unroll
   for (int jj = 0; jj < 4; ++jj) {
     const int kl = tid / 16 + 16 * jj, q = tid % 16, k = k0 + kl, j = j0 + 4 * q;
@@ -108,33 +109,35 @@ __global__ void __launch_bounds__(256) mirror_gates_T4_kernel(const float* __res
   }
 }
 
-void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st, long kcols) {
+void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st, long kcols,
+                    int gu) {
   if (kcols < 0) kcols = ldd;
+  ASTRA_CHECK_ARG(gu % 64 == 0 && gu > 0 && (gu == GATE_U || gu == Hp), "mirror_gates_T: gate layout must be GATE_U or Hp");
   const size_t e = ot == OT::BF16 ? 2 : 4;
   if (H % 4 == 0 && ldd % 4 == 0 && Hp % GATE_U == 0 && ((uintptr_t)src & 15) == 0 &&
       ((uintptr_t)dst & (4 * e - 1)) == 0) {
     dim3 grid(4 * Hp / 64, cdiv(kcols, 64));
     if (ot == OT::BF16)
-      mirror_gates_T4_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
+      mirror_gates_T4_kernel<__nv_bfloat16><<<grid, 256, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols, gu);
     else
-      mirror_gates_T4_kernel<float><<<grid, 256, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols);
+      mirror_gates_T4_kernel<float><<<grid, 256, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols, gu);
     LAUNCH_CHECK();
     return;
   }
   if (kcols % 2 == 0 && ldd % 2 == 0) {
     dim3 grid(cdiv(4L * Hp, 32), cdiv(kcols, 64)), block(32, 8);
     if (ot == OT::BF16)
-      mirror_gates_T2_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
+      mirror_gates_T2_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols, gu);
     else
-      mirror_gates_T2_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols);
+      mirror_gates_T2_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols, gu);
     LAUNCH_CHECK();
     return;
   }
   dim3 grid(cdiv(4L * Hp, 32), cdiv(kcols, 32)), block(32, 8);
   if (ot == OT::BF16)
-    mirror_gates_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols);
+    mirror_gates_T_kernel<__nv_bfloat16><<<grid, block, 0, st>>>(src, K, H, Hp, (__nv_bfloat16*)dst, ldd, kcols, gu);
   else
-    mirror_gates_T_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols);
+    mirror_gates_T_kernel<float><<<grid, block, 0, st>>>(src, K, H, Hp, (float*)dst, ldd, kcols, gu);
   LAUNCH_CHECK();
 }
 
@@ -305,6 +308,7 @@ constexpr int FB_STAGE = 2 * FB_SW + FB_UB * 4;
 
 struct FwdPwArgs {
   int B, H, Hp, nub, rstep;
+  int gu;                      // gate layout (cell_math.cuh gcol_u): GATE_U interleaved, Hp gate-blocked
   const float* WX;
   const float* UH;
   GateParams gp;
@@ -350,18 +354,29 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   // WX_t (the a1 GEMM's output) and c_{t-1} (the previous pointwise kernel's, complete before the
   // GEMM of this step released us) are older than the grid dependency: their copies for the first
   // stages go out before griddepcontrol.wait; UH_t (the GEMM's output) after it.
+  // interleaved layout: the CTA's units' four gates are one contiguous run of 4·nu columns; gate-
+  // blocked: four runs of nu columns (g·Hp + u0), landed at gate offsets g·FB_UB of the stage
+  const bool blk = a.gu != GATE_U;
+  auto load_gates = [&](uint32_t dst, const float* row, uint64_t* bar) {
+    if (!blk) {
+      sm100::bulk_load(dst, row + (long)u0 * 4, wbytes, bar);
+    } else {
+#pragma unroll
+      for (int g = 0; g < 4; ++g) sm100::bulk_load(dst + g * FB_UB * 4, row + (long)g * a.Hp + u0, cbytes, bar);
+    }
+  };
   auto issue_old = [&](int k) {
     const int s = k % FB_STAGES;
     const long b = b_first + (long)k * a.rstep;
     uint8_t* st = sm + s * FB_STAGE;
     sm100::mbar_arrive_expect_tx(&full[s], 2 * wbytes + cbytes);
-    sm100::bulk_load(sm100::smem_u32(st), a.WX + b * NG + (long)u0 * 4, wbytes, &full[s]);
+    load_gates(sm100::smem_u32(st), a.WX + b * NG, &full[s]);
     sm100::bulk_load(sm100::smem_u32(st + 2 * FB_SW), a.c_prev + b * a.Hp + u0, cbytes, &full[s]);
   };
   auto issue_new = [&](int k) {
     const int s = k % FB_STAGES;
     const long b = b_first + (long)k * a.rstep;
-    sm100::bulk_load(sm100::smem_u32(sm + s * FB_STAGE + FB_SW), a.UH + b * NG + (long)u0 * 4, wbytes, &full[s]);
+    load_gates(sm100::smem_u32(sm + s * FB_STAGE + FB_SW), a.UH + b * NG, &full[s]);
   };
   unsigned long long* tr = a.trace ? a.trace + (size_t)blockIdx.x * 34 : nullptr;
   if (tr && tid == 0) tr[0] = gtime_ns();
@@ -388,7 +403,8 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   __syncthreads();
   const int ul = 2 * tid;
   const bool act = ul < nu;
-  const int base = (ul / 64) * 256 + ul % 64;
+  const int base = blk ? ul : (ul / 64) * 256 + ul % 64;
+  const int gstride = blk ? FB_UB : 64;   // stage offset between a unit's gates
   const bool vh = (a.ldh & 1) == 0, vy = (a.ldy & 1) == 0;
   // this thread's units keep their gate parameters in registers for all its rows
   float pb[2][4], pal[2][4], pb1[2][4], pb2[2][4];
@@ -414,8 +430,8 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
       float2 wx[4], uh[4];
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
-        wx[g] = *reinterpret_cast<const float2*>(sw + base + g * 64);
-        uh[g] = *reinterpret_cast<const float2*>(su + base + g * 64);
+        wx[g] = *reinterpret_cast<const float2*>(sw + base + g * gstride);
+        uh[g] = *reinterpret_cast<const float2*>(su + base + g * gstride);
       }
       const float2 cp = *reinterpret_cast<const float2*>(sc + ul);
       float cv[2], hv[2];
@@ -461,9 +477,11 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
 template <int KIND, typename T>
 static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
                           const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, float* hT,
-                          float* cT, cudaStream_t st) {
+                          float* cT, cudaStream_t st, int gu) {
   FwdPwArgs a;
   a.B = B; a.H = H; a.Hp = Hp;
+  ASTRA_CHECK_ARG(gu == GATE_U || gu == Hp, "lstm_fwd_pointwise: gate layout must be GATE_U or Hp");
+  a.gu = gu;
   a.nub = cdiv(Hp, FB_UB);
   a.rstep = std::max(1, std::min(B, 2 * num_sms() / a.nub));
   a.WX = WX; a.UH = UH; a.gp = gp; a.c_prev = c_prev; a.c_new = c_new;
@@ -488,13 +506,13 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
 
 void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
                         const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, OT y_ot,
-                        float* hT, float* cT, cudaStream_t st) {
+                        float* hT, float* cT, cudaStream_t st, int gu) {
 #define FWD_CASE(K)                                                                                          \
   if (kind == K) {                                                                                           \
     if (ot == OT::BF16)                                                                                      \
-      fwd_pw_launch<K, __nv_bfloat16>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, ldh, y, ldy, hT, cT, st);  \
+      fwd_pw_launch<K, __nv_bfloat16>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, ldh, y, ldy, hT, cT, st, gu); \
     else                                                                                                     \
-      fwd_pw_launch<K, float>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, ldh, y, ldy, hT, cT, st);          \
+      fwd_pw_launch<K, float>(y_ot, B, H, Hp, WX, UH, gp, c_prev, c_new, h_op, ldh, y, ldy, hT, cT, st, gu);      \
     return;                                                                                                  \
   }
   FWD_CASE(K_LSTM)
@@ -524,7 +542,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
                        long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
                        const float* __restrict__ WX, const float* __restrict__ UH, const float* __restrict__ c_new,
                        const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
-                       T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
+                       T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first, int gu) {
   constexpr int NV = BwdNV<KIND>::value;
   constexpr int NP = KIND == K_MILSTM ? 4 : 1;   // gate parameter sets: b (and α, β1, β2)
   __shared__ float red[BWD_RY][NV][BWD_UX];
@@ -539,7 +557,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
-  const int c0 = gcol(0, j);
+  const int c0 = gcol_u(0, j, gu);   // gate g of unit j at c0 + g·gu (the `alloc` layout)
   // Operands of one row.  Only dh_rec is produced by the predecessor (the BPTT GEMM); WX, UH, the
   // cell states and dy are older, and dc was written by the pointwise kernel two launches back
   // (complete: the GEMM waits on it before triggering this launch).  So the first row is loaded
@@ -552,8 +570,8 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
     const float* uhp = UH + (long)b * NG + c0;
 #pragma unroll
     for (int g = 0; g < 4; ++g) {
-      w[g] = __ldcs(wxp + g * GATE_U);
-      h[g] = __ldcs(uhp + g * GATE_U);
+      w[g] = __ldcs(wxp + g * gu);
+      h[g] = __ldcs(uhp + g * gu);
     }
     const long ro = (long)b * Hp + j;
     dcv = dc[ro];
@@ -587,15 +605,15 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
         be2[g] = KIND == K_MILSTM ? sg[(NP > 3 ? 12 : 0) * BWD_UX + g * BWD_UX] : 0.f;
       }
       lstm_bwd_row<KIND, T>(w, h, dh, dcv, cp, cn, bb, al, be1, be2, acc, D_uh + (long)b * NG + c0,
-                            D_wx + (long)b * NG + c0);
+                            D_wx + (long)b * NG + c0, gu);
       dc[ro] = dcv;
     }
   } else if (j < Hp) {  // padding units: keep their gradients exactly zero
     for (int b = b0 + ty; b < b1; b += BWD_RY) {
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
-        D_uh[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
-        if (KIND == K_MILSTM) D_wx[(long)b * NG + gcol(g, j)] = from_f<T>(0.f);
+        D_uh[(long)b * NG + gcol_u(g, j, gu)] = from_f<T>(0.f);
+        if (KIND == K_MILSTM) D_wx[(long)b * NG + gcol_u(g, j, gu)] = from_f<T>(0.f);
       }
       dc[(long)b * Hp + j] = 0.f;
     }
@@ -604,7 +622,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   for (int i = 0; i < NV; ++i) red[ty][i][tx] = acc[i];
   __syncthreads();
   if (j >= Hp) return;
-  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, gcol(0, j), nq, first);
+  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, gcol_u(0, j, gu), nq, first, gu);
 }
 
 // K4 backward half, wide form (AV bwd_pw = 1; measured faster at small batch — B = 64: BPTT chain
@@ -667,7 +685,7 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
                         long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
                         const float* __restrict__ WX, const float* __restrict__ UH, const float* __restrict__ c_new,
                         const float* __restrict__ c_prev, GateParams gp, T* __restrict__ D_uh,
-                        T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first) {
+                        T* __restrict__ D_wx, float* __restrict__ partials, int nq, int first, int gu) {
   constexpr int NV = BwdNV<KIND>::value;
   constexpr int NP = KIND == K_MILSTM ? 4 : 1;
   constexpr int NC = KIND == K_MILSTM ? 3 : 1;    // per (row, unit, gate): da (, wx, uh)
@@ -687,7 +705,7 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
   }
   const bool rowok = b < B;
   const int nvalid = min(4, H - j0);            // units of this quad that exist (≤ 0: padding only)
-  const int c0 = gcol(0, j0);
+  const int c0 = gcol_u(0, j0, gu);   // gate g of the quad's units at c0 + g·gu
   const long ro = (long)b * Hp + j0;
   // everything except the GEMM's dh_rec is older than the grid dependency: loaded before the wait
   // (not at the first step, whose predecessor may have produced dy or initialised dc)
@@ -696,8 +714,8 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
   auto load_old = [&] {
 #pragma unroll
     for (int g = 0; g < 4; ++g) {
-      w4[g] = ld4cs(WX + (long)b * NG + c0 + g * GATE_U);
-      h4[g] = ld4cs(UH + (long)b * NG + c0 + g * GATE_U);
+      w4[g] = ld4cs(WX + (long)b * NG + c0 + g * gu);
+      h4[g] = ld4cs(UH + (long)b * NG + c0 + g * gu);
     }
     dc4 = ld4(dc + ro);
     cp4 = ld4cs(c_prev + ro);
@@ -785,10 +803,10 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
 #pragma unroll
     for (int g = 0; g < 4; ++g) {
       float v[4] = {duh4[0][g], duh4[1][g], duh4[2][g], duh4[3][g]};
-      store4<T>(D_uh + (long)b * NG + c0 + g * GATE_U, v);
+      store4<T>(D_uh + (long)b * NG + c0 + g * gu, v);
       if (KIND == K_MILSTM) {
         float x[4] = {dwx4[0][g], dwx4[1][g], dwx4[2][g], dwx4[3][g]};
-        store4<T>(D_wx + (long)b * NG + c0 + g * GATE_U, x);
+        store4<T>(D_wx + (long)b * NG + c0 + g * gu, x);
       }
     }
     *reinterpret_cast<float4*>(dc + ro) = make_float4(dcn[0], dcn[1], dcn[2], dcn[3]);
@@ -826,7 +844,7 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
     float v = 0.f;
 #pragma unroll
     for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[(y * NV + i) * BW2_UB + u]);
-    float* pp = partials + (long)chunk * nq * NG + (long)q * NG + gcol(g, j);
+    float* pp = partials + (long)chunk * nq * NG + (long)q * NG + gcol_u(g, j, gu);
     *pp = first ? v : __fadd_rn(*pp, v);
   }
 }
@@ -835,7 +853,7 @@ template <int KIND, typename T>
 static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32, const float* dh_rec,
                           long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH, const float* c_new,
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
-                          bool first, cudaStream_t st, int form) {
+                          bool first, cudaStream_t st, int form, int gu) {
   if (form == 1) {
     constexpr int NC = KIND == K_MILSTM ? 3 : 1, NP = KIND == K_MILSTM ? 4 : 1;
     const size_t smem = (size_t)(NC * 4 * BWD_RB * BW2_UB + NP * 4 * BW2_UB) * 4;
@@ -845,13 +863,13 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
       static bool attr = false;
       if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
       launch_pdl(k, grid2, dim3(BW2_THREADS), smem, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit,
-                 split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first);
+                 split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
     } else {
       auto k = lstm_bwd_pw2_kernel<KIND, T, __nv_bfloat16>;
       static bool attr = false;
       if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
       launch_pdl(k, grid2, dim3(BW2_THREADS), smem, st, 1, B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh,
-                 nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first);
+                 nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
     }
     LAUNCH_CHECK();
     return;
@@ -861,26 +879,27 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
   if (dy_f32 || dy_ot == OT::F32)
     launch_pdl(lstm_bwd_pw_kernel<KIND, T, float>, grid, block, 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec,
                ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq,
-               (int)first);
+               (int)first, gu);
   else
     launch_pdl(lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16>, grid, block, 0, st, 1, B, H, Hp,
                (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp,
-               (T*)D_uh, (T*)D_wx, partials, nq, (int)first);
+               (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
   LAUNCH_CHECK();
 }
 
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
                         const float* dh_rec, long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH,
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
-                        float* partials, int nq, bool first, cudaStream_t st, int form) {
+                        float* partials, int nq, bool first, cudaStream_t st, int form, int gu) {
+  ASTRA_CHECK_ARG(gu == GATE_U || gu == Hp, "lstm_bwd_pointwise: gate layout must be GATE_U or Hp");
 #define BWD_CASE(K)                                                                                            \
   if (kind == K) {                                                                                             \
     if (ot == OT::BF16)                                                                                        \
       bwd_pw_launch<K, __nv_bfloat16>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, \
-                                      gp, D_uh, D_wx, partials, nq, first, st, form);                          \
+                                      gp, D_uh, D_wx, partials, nq, first, st, form, gu);                          \
     else                                                                                                       \
       bwd_pw_launch<K, float>(B, H, Hp, dy, ldy, dy_ot, dy_f32, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp,  \
-                              D_uh, D_wx, partials, nq, first, st, form);                                      \
+                              D_uh, D_wx, partials, nq, first, st, form, gu);                                      \
     return;                                                                                                    \
   }
   BWD_CASE(K_LSTM)
@@ -893,24 +912,24 @@ void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, l
 struct GradPtrs { float* p[4]; };
 
 __global__ void reduce_gate_partials_kernel(const float* __restrict__ partials, int nchunk, int nq, int H, int Hp,
-                                            GradPtrs out) {
+                                            GradPtrs out, int gu) {
   const int e = blockIdx.x * blockDim.x + threadIdx.x;
   const int q = blockIdx.y;
   if (e >= 4 * H) return;
   const int g = e / H, j = e % H;
   const long NG = 4L * Hp;
-  const int col = gcol(g, j);
+  const int col = gcol_u(g, j, gu);
   float s = 0.f;
   for (int c = 0; c < nchunk; ++c) s = __fadd_rn(s, partials[((long)c * nq + q) * NG + col]);
   out.p[q][e] = s;
 }
 
 void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,
-                          cudaStream_t st) {
+                          cudaStream_t st, int gu) {
   GradPtrs gp{};
   for (int q = 0; q < nq; ++q) gp.p[q] = grads_q[q];
   dim3 grid(cdiv(4L * H, 256), nq);
-  reduce_gate_partials_kernel<<<grid, 256, 0, st>>>(partials, nchunk, nq, H, Hp, gp);
+  reduce_gate_partials_kernel<<<grid, 256, 0, st>>>(partials, nchunk, nq, H, Hp, gp, gu);
   LAUNCH_CHECK();
 }
 

@@ -10,6 +10,10 @@ namespace astra {
 // internal column of (gate g, unit j) = (j / 64)·256 + g·64 + (j % 64).
 constexpr int GATE_U = 64;
 __host__ __device__ __forceinline__ int gcol(int g, int j) { return (j / GATE_U) * (4 * GATE_U) + g * GATE_U + (j % GATE_U); }
+// The same order for a general unit block gu (a multiple of 64): gu = GATE_U is the interleaved layout
+// above, gu = Hp the gate-blocked one (column g·Hp + j) — the two layouts of the `alloc` fork (R38).
+// The gate stride of a unit's four columns is gu.
+__host__ __device__ __forceinline__ int gcol_u(int g, int j, int gu) { return (j / gu) * (4 * gu) + g * gu + (j % gu); }
 
 // Transcendentals.  fp32 path (F = false): IEEE-accurate expf / tanhf (the 1e-4 parity bar).  bf16
 // path (F = true, reading R3): the MUFU tanh.approx.f32 (rel. error ≈ 2^-11), σ(x) = ½·tanh(x/2) + ½ —

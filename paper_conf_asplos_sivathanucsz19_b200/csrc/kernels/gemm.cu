@@ -151,7 +151,8 @@ static int smem_for(int& stages, int cap) {
 }
 
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
-                     int cm, int cn, bool b_keep, int ksplit, int cg, int smem_cap, bool plain_maps) {
+                     int cm, int cn, bool b_keep, int ksplit, int cg, int smem_cap, bool plain_maps, int kperm) {
+  ASTRA_CHECK_ARG(kperm == 0 || (K == 4 * kperm * TC_BK), "tc_gemm: a gate-permuted K must be 4 gate blocks of kperm k-blocks");
   // BN = 224 (74 CTA pairs fill all 148 SMs on an 8192-column chain GEMM instead of 64 pairs of 256)
   // exists only for CTA pairs with a K-major B (each CTA holds 112 B rows); elsewhere the same tile
   // width is run as 256 — same bits (R1: every output element is one accumulation over K)
@@ -173,7 +174,7 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
     }();
     const int nk_all = cdiv(K, TC_BK), kper = cdiv(nk_all, ksplit);
     const bool kmaj_ok = (a_mn || K % TC_BK == 0) && (b_mn || K % TC_BK == 0);
-    if (cg == 1 && cm * cn == 1 && kmaj_ok && kb_env != 1 && !plain_maps) {
+    if (cg == 1 && cm * cn == 1 && kmaj_ok && kb_env != 1 && !plain_maps && kperm == 0) {
       int dev = 0, maxs = 0;
       CUDA_TRY(cudaGetDevice(&dev));
       CUDA_TRY(cudaDeviceGetAttribute(&maxs, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
@@ -218,6 +219,7 @@ void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_
   }
   g.args.kb = KB;
   g.args.a_rows = a_rows;
+  g.args.kperm = kperm;
   g.args.pf = L2Pf{};
   g.args.cg = cg;
   static const int gm_env = [] {

@@ -34,7 +34,7 @@ struct TcGemm {
 // another kernel (the fused recurrent / BPTT kernels load single k-block boxes through them).
 void tc_gemm_prepare(TcGemm& g, const Mat2& A, bool a_mn, const Mat2& B, bool b_mn, int M, int N, int K, int BN,
                      int cm = 1, int cn = 1, bool b_keep = false, int ksplit = 1, int cg = 1, int smem_cap = 0,
-                     bool plain_maps = false);
+                     bool plain_maps = false, int kperm = 0);
 // Launch with the given z-coordinates (time slices) and epilogue; grid ≤ #SMs (persistent).
 void tc_gemm_launch(const TcGemm& g, const EpiStore& epi, int az, int bz, cudaStream_t st, int max_ctas = 0,
                     const L2Pf* pf = nullptr);

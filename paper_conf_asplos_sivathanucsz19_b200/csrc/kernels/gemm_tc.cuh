@@ -73,7 +73,13 @@ struct TcArgs {
   // The pair kernel (tc_gemm2) ignores both (kb = 1, a_rows = 128).
   int kb;
   int a_rows;
+  // k-block order (the `alloc` fork, reading R38): 0 = ascending; P > 0 = the contraction runs over
+  // 4 gate blocks of P k-blocks each (a gate-blocked K = 4·Hp, P = Hp/64) in the canonical gate-
+  // interleaved order — canonical k-block c reads physical k-block (c % 4)·P + c / 4 — so the
+  // accumulation order, hence every bit, is the interleaved layout's.  Needs kb = 1.
+  int kperm;
 };
+__device__ __forceinline__ int tc_kphys(int kb, int kperm) { return kperm ? (kb & 3) * kperm + (kb >> 2) : kb; }
 
 // One warp of every CTA issues its slice of the prefetch ranges (cp.async.bulk.prefetch.L2, 16-byte
 // granules): range bytes split evenly over gridDim.x × 32 lanes.
@@ -379,7 +385,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           uint8_t* sa = smem + s * stage_bytes;
           uint8_t* sb = sa + KB * a_kb_bytes;
           sm100::mbar_arrive_expect_tx_warp(&full[s], stage_bytes);
-          const int k0 = kb * TC_BK;
+          const int k0 = tc_kphys(kb, args.kperm) * TC_BK;
           if (KB > 1) {   // (cs == 1) one box per operand for the KB k-blocks of the stage
             if (args.a_mn) {
               sm100::tma_load_3d_warp(sa, &mapA, &full[s], m0, k0, args.az);
@@ -616,7 +622,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           uint8_t* sa = smem + i * S::STAGE_BYTES;
           if (rank == 0) sm100::mbar_arrive_expect_tx(&full[i], 2 * S::STAGE_BYTES);
           load_b(sa + S::A_BYTES, sm100::mapa_shared(sm100::smem_u32(&full[i]), 0), ni * BN + rank * BH,
-                 (kb0 + i) * TC_BK);
+                 tc_kphys(kb0 + i, args.kperm) * TC_BK);
         }
       }
       pdl_wait();
@@ -636,7 +642,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
           uint8_t* sb = sa + S::A_BYTES;
           if (!early && rank == 0) sm100::mbar_arrive_expect_tx(&full[s], 2 * S::STAGE_BYTES);
           const uint32_t bar = sm100::mapa_shared(sm100::smem_u32(&full[s]), 0);
-          const int k0 = kb * TC_BK;
+          const int k0 = tc_kphys(kb, args.kperm) * TC_BK;
           if (args.a_mn) {
             sm100::tma_load_3d_cg2(sa, &mapA, bar, m0, k0, args.az);
             sm100::tma_load_3d_cg2(sa + 8192, &mapA, bar, m0 + 64, k0, args.az);

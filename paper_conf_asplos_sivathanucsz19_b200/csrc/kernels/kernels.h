@@ -22,10 +22,11 @@ struct GateParams {          // external-layout fp32 vectors of length 4H (may b
 };
 
 // ---- mirrors (K9): fp32 params → operand-type copies in the internal layout
-// dst[gcol(g, j)][k] = src[k][g*H + j] for the gate-blocked [K][4H] matrix `src`
-// (dst rows = 4*Hp, row stride ldd ≥ K; padding rows/cols zero).
+// dst[gcol_u(g, j, gu)][k] = src[k][g*H + j] for the gate-blocked [K][4H] matrix `src`
+// (dst rows = 4*Hp, row stride ldd ≥ K; padding rows/cols zero).  gu: the internal gate layout of
+// the `alloc` fork — 64 (GATE_U, gate-interleaved, the default) or Hp (gate-blocked), cell_math.cuh.
 void mirror_gates_T(OT ot, const float* src, int K, int H, int Hp, void* dst, long ldd, cudaStream_t st,
-                    long kcols = -1);
+                    long kcols = -1, int gu = 64);
 // dst[n][k] = src[k][n] (plain transpose), dst [Np][ldd], padding zero.
 void mirror_T(OT ot, const float* src, int K, int N, int Np, int Kp, void* dst, long ldd, cudaStream_t st);
 // Operand copy of an external [rows][cols] (OT or fp32 `src_ot`) into [rows][ldd] of type `ot`.
@@ -39,20 +40,20 @@ void copy_f32_pad(const float* src, long rows, int cols, long lds, float* dst, l
 // h_op: operand copy of h_t, row stride ldh (≥ Hp); y (type y_ot, row stride ldy) optional.
 void lstm_fwd_pointwise(int kind, OT ot, int B, int H, int Hp, const float* WX, const float* UH, GateParams gp,
                         const float* c_prev, float* c_new, void* h_op, long ldh, void* y, long ldy, OT y_ot,
-                        float* hT, float* cT, cudaStream_t st);
+                        float* hT, float* cT, cudaStream_t st, int gu = 64);
 // dy: row stride ldy of type dy_ot (or fp32); dh_rec: [B][ld_dh] fp32 or null (zeros).
 // dh_rec: nsplit fp32 partials (split-K) at stride split_stride elements, summed in order.
 void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32,
                         const float* dh_rec, long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH,
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
-                        float* partials, int nq, bool first, cudaStream_t st, int form = 0);
+                        float* partials, int nq, bool first, cudaStream_t st, int form = 0, int gu = 64);
 // form (AV "bwd_pw", bitwise interchangeable): 0 the row-lane kernel (thread = unit, rows walked 4
 // lanes x 8), 1 the wide kernel (thread = row x 4 units, all rows of a 32-row chunk in flight).
 int lstm_bwd_row_chunks(int B);
 constexpr int BWD_ROW_CHUNK = 32;   // rows per column-partial chunk of the backward pointwise kernels (R5)
 // grads_q[e] = Σ_chunk partials[chunk][q][gcol(e)] for q < nq (external e < 4H).
 void reduce_gate_partials(const float* partials, int nchunk, int nq, int H, int Hp, float* const* grads_q,
-                          cudaStream_t st);
+                          cudaStream_t st, int gu = 64);
 
 // ---- SCRN [22] / RHN [39] pointwise and scan halves (scrn_rhn_kernels.cu)
 int pw_row_chunks(int B);

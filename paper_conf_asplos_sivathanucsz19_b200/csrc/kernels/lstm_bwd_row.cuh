@@ -62,36 +62,36 @@ __device__ __forceinline__ void lstm_bwd_acc(float (&acc)[BwdNV<KIND>::value], i
 }
 
 // Both halves for one (row, unit) with the accumulation in this thread (the unfused kernel's and the
-// fused BPTT kernel's form): D_uh / D_wx stored at gate stride GATE_U.
+// fused BPTT kernel's form): D_uh / D_wx stored at gate stride gs (GATE_U, or Hp gate-blocked).
 template <int KIND, typename T>
 __device__ __forceinline__ void lstm_bwd_row(const float (&w)[4], const float (&h)[4], float dh, float& dcv, float cp,
                                              float cn, const float (&bb)[4], const float (&al)[4],
                                              const float (&be1)[4], const float (&be2)[4],
-                                             float (&acc)[BwdNV<KIND>::value], T* duhp, T* dwxp) {
+                                             float (&acc)[BwdNV<KIND>::value], T* duhp, T* dwxp, int gs = GATE_U) {
   constexpr bool F = FastMath<T>::value;   // bf16 path: fused multiply-adds (reading R27)
   float da[4], duh[4], dwx[4];
   lstm_bwd_da<KIND, F>(w, h, dh, dcv, cp, cn, bb, al, be1, be2, da, duh, dwx);
 #pragma unroll
   for (int g = 0; g < 4; ++g) {
     lstm_bwd_acc<KIND, F>(acc, g, da[g], w[g], h[g]);
-    duhp[g * GATE_U] = from_f<T>(duh[g]);
-    if (KIND == K_MILSTM) __stcs(dwxp + g * GATE_U, from_f<T>(dwx[g]));
+    duhp[g * gs] = from_f<T>(duh[g]);
+    if (KIND == K_MILSTM) __stcs(dwxp + g * gs, from_f<T>(dwx[g]));
   }
 }
 
 // After every thread of the chunk has stored red[ty][i][tx] = acc[i] and the caller synchronised:
 // thread (tx, ty) finalises quantities i = ty, ty + 4, ... for unit column `col` (gate g at col +
-// g·GATE_U) into the chunk's partials p[q·NG + ...].
+// g·gs) into the chunk's partials p[q·NG + ...].
 template <int NV>
 __device__ __forceinline__ void bwd_chunk_finalize(const float (*red)[NV][BWD_UX], int tx, int ty, float* p, long NG,
-                                                   int col0, int nq, int first) {
+                                                   int col0, int nq, int first, int gs = GATE_U) {
   for (int i = ty; i < NV; i += BWD_RY) {
     float v = 0.f;
 #pragma unroll
     for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[y][i][tx]);
     const int q = i / 4, g = i % 4;
     if (q >= nq) continue;
-    float* pp = p + (long)q * NG + col0 + g * GATE_U;
+    float* pp = p + (long)q * NG + col0 + g * gs;
     *pp = first ? v : __fadd_rn(*pp, v);
   }
 }

@@ -69,6 +69,11 @@ struct Variant {
                         // ranges, on GCHUNK_S[gchunk] streams (P:122 two streams vs one fused GEMM)
   int recomp = 0;       // alloc fork: 1 = the recurrent projection UH_t is not
                         // kept for BPTT but recomputed there from the saved h_{t-1} operands (same bits)
+  int gblk = 0;         // alloc fork (§8(a.9) `alloc`, reading R38): internal gate layout of the LSTM
+                        // family's mirrors and gate-column tensors, 0 gate-interleaved (64-unit blocks), 1 gate-
+                        // blocked ([K, G·Hp]); the GEMMs contracting over gates read k-blocks in the interleaved
+                        // order (TcArgs::kperm), so the same bits; the fused / persistent K2 / K4 forms need a
+                        // unit's four gates in one tile, so they exist only under the interleaved context
   Variant() { g[G_BPTT].bn = 128; }
   std::string str() const;                    // "a1=256.1.1,rec=...,wg_side=0"
   static Variant parse(const std::string& s); // inverse of str(); throws ASTRA_E_ARG
@@ -81,6 +86,7 @@ struct GemmSpec {
   bool b_keep = false;   // B is a weight re-read every step: keep it in L2 (evict_last)
   int ksplit = 1;        // fixed split-K (part of the canonical numerics: every variant uses it)
   int M = 0, N = 0, K = 0;
+  int kperm = 0;         // K over gate-blocked gate columns, read in the canonical interleaved order (TcArgs::kperm)
 };
 
 Mat2 mat(const void* p, long inner, long outer, long ld, long z = 1, long zstride = 0);
@@ -149,7 +155,7 @@ class Cell {
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
   // prepared GEMMs keyed by (gemm id, T, bn, cm, cn, cg, A, B, M, N, K): the tensor maps carry the
   // operand pointers and extents, so two row ranges of one role never share an entry
-  using TcKey = std::tuple<int, int, int, int, int, int, const void*, const void*, int, int, int, bool>;
+  using TcKey = std::tuple<int, int, int, int, int, int, const void*, const void*, int, int, int, bool, int>;
   std::map<TcKey, TcGemm> tc_cache;
 
   // Bucketed profiling: one independent exploration per active length T, the
@@ -204,6 +210,7 @@ class Cell {
   virtual bool lm_capable() const { return true; }
   virtual bool chain_prefetch() const { return false; }   // supports Variant::l2pf (tuner AVs pf_fwd / pf_bwd)
   virtual bool supports_recompute() const { return false; }   // Variant::recomp (tuner root fork "recomp")
+  virtual bool supports_gate_blocked() const { return false; }   // Variant::gblk (tuner root fork "alloc")
   virtual int fwd_fusions() const { return 1; }   // number of K2 fusion choices (tuner AV "fuse_fwd")
   virtual const char* fwd_fusion_metric() const { return "t_fwd"; }   // the region that judges it
   virtual int bwd_fusions() const { return 1; }   // number of K4 fusion choices (tuner AV "fuse_bwd")

@@ -25,6 +25,7 @@ std::string Variant::str() const {
   o << "wg_side=" << wg_side << ",fwd=" << fwd_mode << ",bwd=" << bwd_mode << ",pf=" << l2pf << ",hov=" << head_ov;
   if (lwf) o << ",lwf=" << lwf;
   if (recomp) o << ",rc=" << recomp;
+  if (gblk) o << ",gb=" << gblk;
   if (dpb) o << ",dpb=" << dpb;
   if (gchunk) o << ",gc=" << gchunk;
   if (wgs) o << ",wgs=" << wgs;
@@ -73,6 +74,11 @@ Variant Variant::parse(const std::string& s) {
     if (k == "gc") {
       v.gchunk = std::stoi(val);
       ASTRA_CHECK_ARG(v.gchunk >= 0 && v.gchunk <= 4, "variant: gc (gate_chunking) must be 0..4");
+      continue;
+    }
+    if (k == "gb") {
+      v.gblk = std::stoi(val);
+      ASTRA_CHECK_ARG(v.gblk == 0 || v.gblk == 1, "variant: gb must be 0 (gate-interleaved) or 1 (gate-blocked layout)");
       continue;
     }
     if (k == "rc") {
@@ -222,7 +228,7 @@ void Cell::mark(Region r, int which, cudaStream_t st) {
 TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k, bool plain_maps) {
   // split-K only runs without clusters; the cluster choice then falls back to 1x1 (same numerics)
   const int cm = s.ksplit > 1 ? 1 : k.cm, cn = s.ksplit > 1 ? 1 : k.cn;
-  const TcKey key{id, T, k.bn, cm, cn, k.cg, s.A.ptr, s.B.ptr, s.M, s.N, s.K, plain_maps};
+  const TcKey key{id, T, k.bn, cm, cn, k.cg, s.A.ptr, s.B.ptr, s.M, s.N, s.K, plain_maps, s.kperm};
   auto it = tc_cache.find(key);
   if (it == tc_cache.end()) {
     TcGemm g;
@@ -238,7 +244,7 @@ TcGemm& Cell::tc_get(int id, const GemmSpec& s, const KCfg& k, bool plain_maps) 
       return e ? std::atoi(e) * 1024 : 0;
     }();
     tc_gemm_prepare(g, s.A, s.a_mn, s.B, s.b_mn, s.M, s.N, s.K, k.bn, cm, cn, s.b_keep, s.ksplit, k.cg,
-                    id == 2 ? bptt_cap : id == 1 ? rec_cap : 0, plain_maps);
+                    id == 2 ? bptt_cap : id == 1 ? rec_cap : 0, plain_maps, s.kperm);
     it = tc_cache.emplace(key, g).first;
   }
   return it->second;
@@ -451,7 +457,12 @@ void Cell::tuner_setup() {
   // SURVEY §8(f) rank 4 / §8(a.9) `alloc`: store-vs-recompute of the recurrent projection is a
   // memory-allocation context: the whole tree is explored under each context, then
   // each context's best configuration is raced end to end, 3 steps each
-  if (ot == OT::BF16 && supports_recompute()) t = "(fork (leaf recomp 2 t_step) t_step " + t + " 3)";
+  // The gate layout (gate-interleaved vs gate-blocked, reading R38) is the other allocation context:
+  // with both, the fork leaf `alloc` has 4 contexts, option o = recompute (o & 1) × gate-blocked (o >> 1)
+  if (ot == OT::BF16 && supports_recompute() && supports_gate_blocked())
+    t = "(fork (leaf alloc 4 t_step) t_step " + t + " 3)";
+  else if (ot == OT::BF16 && supports_recompute())
+    t = "(fork (leaf recomp 2 t_step) t_step " + t + " 3)";
   tree.reset(new tuner::Tree(tuner::parse(t)));
   wirer.reset(new tuner::Wirer(tree.get()));
   wirer->index().bucket = T;
@@ -475,6 +486,7 @@ void Cell::apply_config(const tuner::Config& c) {
     if (n == "head_ov") { v.head_ov = o; continue; }
     if (n == "lwf") { v.lwf = o; continue; }
     if (n == "recomp") { v.recomp = o; continue; }
+    if (n == "alloc") { v.recomp = o & 1; v.gblk = o >> 1; continue; }
     if (n == "dp_bucket") { v.dpb = o; continue; }
     if (n == "gate_chunking") { v.gchunk = o; continue; }
     if (n == "wgrad_schedule") { v.wgs = o; continue; }

@@ -74,6 +74,12 @@ class LstmCell : public Cell {
     }
   }
   bool supports_recompute() const override { return true; }
+  bool supports_gate_blocked() const override { return ot == OT::BF16; }
+  // the `alloc` gate layout (Variant::gblk, reading R38): unit block of the gate order (cell_math.cuh
+  // gcol_u) and the k-block permutation the gate-contracting GEMMs read in the canonical order with
+  bool blocked() const { return var.gblk != 0 && ot == OT::BF16; }
+  int gate_u() const { return blocked() ? Hp : GATE_U; }
+  int kperm() const { return blocked() ? Hp / TC_BK : 0; }
 
   // Fixed split-K of the per-step BPTT GEMM (K = 4·Hp): with B rows the GEMM has few output tiles,
   // so each SM would stream a whole K-panel of Uᵀ; four K-chunks cut the bytes per SM 4× while the
@@ -166,8 +172,8 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   if (t0 == 0) {
     if (!lm_mode) mark(R_STEP, 0, st);   // an LM marks its step itself (embedding included)
     // K9 second half: operand mirrors in the internal gate-interleaved layout
-    mirror_gates_T(ot, p("W"), I, H, Hp, Wm, Ip, st);
-    mirror_gates_T(ot, p("U"), H, H, Hp, Um, Hp, st);
+    mirror_gates_T(ot, p("W"), I, H, Hp, Wm, Ip, st, -1, gate_u());
+    mirror_gates_T(ot, p("U"), H, H, Hp, Um, Hp, st, -1, gate_u());
     if (!lm_mode) copy_pad(ot, x, ot, TB, I, I, X, Ip, st);
     copy_pad(ot, h0, OT::F32, B, H, H, Hrow(0), Hp, st);
     copy_f32_pad(c0, B, H, H, Cb, Hp, H, st);
@@ -191,7 +197,10 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     CUDA_TRY(cudaStreamWaitEvent(side[0], ev_fork, 0));
   }
   for (int k = 0; k < nc; ++k) {
-    const int n0 = (int)((long)nblk * k / nc) * 4 * GATE_U, n1 = (int)((long)nblk * (k + 1) / nc) * 4 * GATE_U;
+    // gate-interleaved: ranges of whole 256-column unit blocks; gate-blocked: whole gates (nc ∈ {1, 2, 4}:
+    // G/nc gates per GEMM — the paper's G separate gate GEMMs, G/2, or one fused)
+    int n0 = (int)((long)nblk * k / nc) * 4 * GATE_U, n1 = (int)((long)nblk * (k + 1) / nc) * 4 * GATE_U;
+    if (blocked()) { n0 = (int)((long)NG * k / nc); n1 = (int)((long)NG * (k + 1) / nc); }
     GemmSpec a1;
     a1.A = mat((const char*)X + (size_t)t0 * B * Ip * e, I, rows, Ip);
     a1.B = mat((const char*)Wm + (size_t)n0 * Ip * e, I, n1 - n0, Ip);
@@ -213,7 +222,9 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
   rec.B = mat(Um, Hp, NG, Hp);
   rec.M = B; rec.N = NG; rec.K = Hp;
   rec.b_keep = true;
-  if (ot == OT::BF16 && var.fwd_mode == 1 && !y_f32) {
+  // the fused / persistent forms tile a unit's four gates together: gate-interleaved context only
+  const int fmode = blocked() ? 0 : var.fwd_mode;
+  if (ot == OT::BF16 && fmode == 1 && !y_f32) {
     // K2 fused, CTA-pair form: GEMM + gate epilogue with TMA-staged epilogue I/O, one launch per step
     const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1, 2}, true);
     if (fm_key != (const void*)y || fm_wx != (const void*)WX || fm_T != T) {
@@ -244,7 +255,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
       lstm_fwd_pair_launch(kind, fm, ra, st);
       fwd_step_done(t, st);
     }
-  } else if (ot == OT::BF16 && var.fwd_mode == 3 && lstm_fwd_persist_supported(B, Hp)) {
+  } else if (ot == OT::BF16 && fmode == 3 && lstm_fwd_persist_supported(B, Hp)) {
     // K2 small-batch persistent: the whole range in one cooperative launch, U slices resident
     RecPersistArgs pa{};
     pa.B = B; pa.H = H; pa.Hp = Hp; pa.NG = NG; pa.T = T; pa.t0 = t0; pa.t1 = t1;
@@ -258,7 +269,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     CUDA_TRY(cudaMemsetAsync(pa.flags, 0, 4096, st));
     lstm_fwd_persist_launch(kind, Hrow(0), Um, Tmax, pa, st);
     for (int t = t0; t < t1; ++t) fwd_step_done(t, st);   // one kernel: every step is done at its end
-  } else if (ot == OT::BF16 && var.fwd_mode > 0 && var.fwd_mode < 3) {
+  } else if (ot == OT::BF16 && fmode > 0 && fmode < 3) {
     // K2 fused: GEMM + gate epilogue in one kernel (per step, or persistent over all steps)
     const TcGemm& tg = tc_get(1, rec, KCfg{256, 1, 1}, true);
     RecFwdArgs ra;
@@ -271,7 +282,7 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
     else { ra.y = nullptr; ra.ldy = 0; ra.y_kind = 0; }
     ra.hT = hT; ra.cT = cT; ra.gp = gp;
     ra.flags = sc<unsigned>(off_flags);
-    const bool persistent = var.fwd_mode == 2 && ra.num_m * ra.num_n <= num_sms() && ra.num_m <= 1024;
+    const bool persistent = fmode == 2 && ra.num_m * ra.num_n <= num_sms() && ra.num_m <= 1024;
     if (persistent) {
       CUDA_TRY(cudaMemsetAsync(ra.flags, 0, 4096, st));
       ra.persistent = 1; ra.t0 = t0; ra.t1 = t1;
@@ -303,11 +314,11 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
         if (y_f32)
           lstm_fwd_pointwise(kind, ot, Bh, H, Hp, WX + rr * NG, UHt, gp, Cb + rr * Hp, Cb + (rr + B) * Hp,
                              (char*)Hrow(t + 1) + (size_t)r0 * Hp * e, Hp, y_f32 + (size_t)rr * Hp, Hp, OT::F32,
-                             last && hT ? hT + r0 * H : nullptr, last && cT ? cT + r0 * H : nullptr, S);
+                             last && hT ? hT + r0 * H : nullptr, last && cT ? cT + r0 * H : nullptr, S, gate_u());
         else
           lstm_fwd_pointwise(kind, ot, Bh, H, Hp, WX + rr * NG, UHt, gp, Cb + rr * Hp, Cb + (rr + B) * Hp,
                              (char*)Hrow(t + 1) + (size_t)r0 * Hp * e, Hp, y ? (char*)y + (size_t)rr * H * e : nullptr,
-                             H, ot, last && hT ? hT + r0 * H : nullptr, last && cT ? cT + r0 * H : nullptr, S);
+                             H, ot, last && hT ? hT + r0 * H : nullptr, last && cT ? cT + r0 * H : nullptr, S, gate_u());
       }
     }
     rs_join(st);
@@ -322,11 +333,11 @@ void LstmCell::forward(const void* x, const float* h0, const float* c0, void* y,
       if (y_f32)   // internal fp32 output (e.g. the encoder of LSTM-attention), row stride Hp
         lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
                            Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y_f32 + (size_t)t * B * Hp, Hp, OT::F32,
-                           last ? hT : nullptr, last ? cT : nullptr, st);
+                           last ? hT : nullptr, last ? cT : nullptr, st, gate_u());
       else
         lstm_fwd_pointwise(kind, ot, B, H, Hp, WX + (long)t * B * NG, UHt, gp, Cb + (long)t * B * Hp,
                            Cb + (long)(t + 1) * B * Hp, Hrow(t + 1), Hp, y ? (char*)y + (size_t)t * B * H * e : nullptr,
-                           H, ot, last ? hT : nullptr, last ? cT : nullptr, st);
+                           H, ot, last ? hT : nullptr, last ? cT : nullptr, st, gate_u());
       fwd_step_done(t, st);
     }
   }
@@ -373,13 +384,15 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   bp.b_mn = true;
   bp.M = B; bp.N = Hp; bp.K = NG;
   bp.b_keep = true;
+  bp.kperm = kperm();   // K over the gate columns: the canonical (interleaved) k-block order in any layout
   GemmSpec bp0 = bp;   // dh0 (once, no split)
   bp.ksplit = bptt_ksplit();
   // fused BPTT step (K4 fused): dy must be TMA-mappable (the LM's fp32 dY, or bf16 with H % 8 == 0)
-  const bool fuse = var.bwd_mode == 1 && lstm_bptt_fused_supported(B, Hp, bp.ksplit) && ot == OT::BF16 && T > 1 &&
+  const int bmode = blocked() ? 0 : var.bwd_mode;   // fused / persistent: gate-interleaved context only
+  const bool fuse = bmode == 1 && lstm_bptt_fused_supported(B, Hp, bp.ksplit) && ot == OT::BF16 && T > 1 &&
                     (lm_dy || (H % 8 == 0 && ((uintptr_t)dy & 15) == 0));
   // small-batch persistent BPTT chain (bptt_persist.cu): the whole range in one launch
-  const bool persist = !fuse && var.bwd_mode >= 2 && whole && var.recomp == 0 && bptt_persist_ok();
+  const bool persist = !fuse && bmode >= 2 && whole && var.recomp == 0 && bptt_persist_ok();
   BpttFusedArgs fa{};
   if (fuse) {
     const TcGemm& tg = tc_get(2, bp, KCfg{64, 1, 1}, true);
@@ -461,6 +474,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     gx.B = mat(Wm, I, NG, Ip);
     gx.b_mn = true;
     gx.M = (int)rows; gx.N = I; gx.K = NG;
+    gx.kperm = kperm();
     if (lm_mode)
       run_gemm(id, gx, epi((float*)dx + (size_t)r0 * B * Ip, Ip, (int)rows, I), 0, 0, var.g[G_DX], s_, nullptr, max_ctas);
     else
@@ -528,7 +542,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
         lstm_bwd_pointwise(kind, ot, Bh, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC + r0 * Hp,
                            WX + rr * NG, UH + rr * NG, Cb + (rr + B) * Hp, Cb + rr * Hp, gp,
                            Duh + (size_t)rr * NG * e, Dwx + (size_t)rr * NG * e,
-                           part + (size_t)(r0 / BWD_ROW_CHUNK) * nq * NG, nq, t == T - 1, S, var.bpw);
+                           part + (size_t)(r0 / BWD_ROW_CHUNK) * nq * NG, nq, t == T - 1, S, var.bpw, gate_u());
       }
     }
     rs_join(st);
@@ -570,7 +584,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
     }
     lstm_bwd_pointwise(kind, ot, B, H, Hp, dyt, ldy, ot, dyf32, dh_rec, ld_dh, nsplit, (long)B * Hp, dC, WX + (long)t * B * NG,
                        uh_of(t), Cb + (long)(t + 1) * B * Hp, Cb + (long)t * B * Hp, gp,
-                       Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st, var.bpw);
+                       Duh + (size_t)t * B * NG * e, Dwx + (size_t)t * B * NG * e, part, nq, t == T - 1, st, var.bpw, gate_u());
     if (rc && !fuse && t == chunk_lo(kc)) {   // chunk kc consumed: its slot takes chunk kc - 2
       if (rs != st) CUDA_TRY(cudaEventRecord(ev_rc_free[kc & 1], st));
       released[kc & 1] = true;
@@ -606,7 +620,8 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   gu.b_mn = true;
   gu.M = Hp; gu.N = NG; gu.K = (int)TB;
   if (st_u == st) mark(R_DU, 0, st);
-  run_gemm(4, gu, epi_perm(g("U"), 4L * H, H, NG, GATE_U, 0, H), 0, 0, var.g[G_DU], st_u);
+  run_gemm(4, gu, blocked() ? epi_perm(g("U"), 4L * H, H, NG, 0, Hp, H) : epi_perm(g("U"), 4L * H, H, NG, GATE_U, 0, H),
+           0, 0, var.g[G_DU], st_u);
   if (st_u == st) mark(R_DU, 1, st);
   grad_bucket(g("U"), (size_t)H * 4 * H, st_u);
 
@@ -617,7 +632,8 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   gw.b_mn = true;
   gw.M = I; gw.N = NG; gw.K = (int)TB;
   mark(R_DW, 0, st);
-  run_gemm(5, gw, epi_perm(g("W"), 4L * H, I, NG, GATE_U, 0, H), 0, 0, var.g[G_DW], st);
+  run_gemm(5, gw, blocked() ? epi_perm(g("W"), 4L * H, I, NG, 0, Hp, H) : epi_perm(g("W"), 4L * H, I, NG, GATE_U, 0, H),
+           0, 0, var.g[G_DW], st);
   mark(R_DW, 1, st);
   grad_bucket(g("W"), (size_t)I * 4 * H, st);
 
@@ -628,7 +644,7 @@ void LstmCell::backward(const void* dy, const float* dhT, const float* dcT, void
   }
   float* gq[4] = {g("b"), nullptr, nullptr, nullptr};
   if (kind == K_MILSTM) { gq[1] = g("alpha"); gq[2] = g("beta1"); gq[3] = g("beta2"); }
-  reduce_gate_partials(part, nchunk, nq, H, Hp, gq, st);
+  reduce_gate_partials(part, nchunk, nq, H, Hp, gq, st, gate_u());
   grad_bucket(g("b"), (size_t)(G + n_params - g("b")), st);   // b (and α, β1, β2): the tail of the cell block
   if (st_u != st) {
     CUDA_TRY(cudaEventRecord(ev_join, st_u));

@@ -255,6 +255,30 @@ def test_recompute_bitwise_and_parity(cell, dtype, tol, monkeypatch):
     _check(cell, T, B, I, H, dtype, 78, tol, variant="rc=1")
 
 
+@pytest.mark.parametrize("cell", ["lstm", "milstm", "sublstm"])
+@pytest.mark.parametrize("T,B,I,H", [(5, 72, 64, 96), (4, 160, 128, 192), (3, 64, 256, 1024)])
+def test_gate_blocked_alloc_bitwise(cell, T, B, I, H):
+    """The `alloc` fork's gate layout (reading R38): gate-blocked mirrors / gate tensors
+    (gb=1) with the gate-contracting GEMMs (per-step BPTT dh_rec = D_uh·Uᵀ, input dgrad D_wx·Wᵀ)
+    reading their k-blocks in the interleaved layout's order give the same bits as the gate-
+    interleaved layout for every output and gradient — with per-gate a1 GEMMs (gc=2: the paper's G
+    separate gate GEMMs; gc=4 on two streams), both backward pointwise forms, the chunked dX,
+    CTA-pair BPTT GEMMs, the recompute context, and at H = 1024 the 2-way split-K BPTT GEMM —
+    and match the oracle.  Hp > H (padding units) in the first case."""
+    p, inp, dY, dhT, dcT = make_cell_case(cell, T, B, I, H, 91, bf16=True)
+    out0, g0, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, "bf16", "fwd=0")
+    ref = {**out0, **g0}
+    vs = ["gb=1", "gb=1,gc=2,bpw=1", "gb=1,gc=4,wg_side=1,wgs=1",
+          "a1=256.1.1.2,rec=256.1.1.2,bptt=128.1.1.2,du=256.1.1.2,dw=256.1.1.2,dx=256.1.1.2,wg_side=0,fwd=0,gb=1",
+          "gb=1,rc=1", "gb=1,fwd=2,bwd=1"]
+    for v in vs:
+        out, g, _ = run_gpu_cell(cell, p, inp, dY, dhT, dcT, "bf16", v)
+        cur = {**out, **g}
+        for k in ref:
+            assert np.array_equal(ref[k], cur[k]), (v, k)
+    _check(cell, T, B, I, H, "bf16", 91, TOL_BF16, variant="gb=1,gc=2")
+
+
 def test_variants_bitwise():
     """Every tile-width / stream variant gives bitwise-identical outputs and gradients."""
     T, B, I, H = 6, 160, 128, 192

@@ -134,7 +134,7 @@ def _steps_params(variant, graph, steps=8):
 
 @pytest.mark.parametrize("variant", ["fwd=0", "a1=256.1.1.2,rec=256.1.1.2,bptt=128.1.1.2,du=256.1.1.2,dw=128.1.1.2,"
                                      "dx=256.1.1.2,head=256.1.1.2,wg_side=1,fwd=1",
-                                     "fwd=0,hov=1,wgs=2,gc=3,wg_side=1"])
+                                     "fwd=0,hov=1,wgs=2,gc=3,wg_side=1", "gb=1,gc=2,hov=1,bpw=1"])
 def test_graph_replay_bitwise(variant):
     """CUDA-graph replay of frozen steps (the bench path) is bitwise identical to kernel-by-kernel
     enqueueing, over 8 SGD steps (state carried between steps)."""
@@ -247,7 +247,8 @@ def test_profiling_switch():
     assert torch.equal(out[0], out[1])
 
 
-@pytest.mark.parametrize("variant", ["rc=1", "rc=1,fwd=1", "rc=1,fwd=2", "rc=1,bwd=1", "rc=1,wg_side=1,hov=1"])
+@pytest.mark.parametrize("variant", ["rc=1", "rc=1,fwd=1", "rc=1,fwd=2", "rc=1,bwd=1", "rc=1,wg_side=1,hov=1",
+                                     "gb=1", "gb=1,rc=1,gc=2,wgs=1"])
 def test_recompute_lm_bitwise(variant, monkeypatch):
     """SURVEY §8(f) rank 4, the alloc fork: recomputing UH_t = h_{t-1}·U in BPTT (ring of 2-step
     chunks on a side stream, 3 chunks at T = 5 so the ring wraps) gives the same bits as storing it,
@@ -262,12 +263,12 @@ def test_recompute_lm_bitwise(variant, monkeypatch):
 
 
 def test_tuner_fork_explores_both_allocation_contexts():
-    """The live update tree's root is the hierarchical alloc fork: both contexts are
+    """The live update tree's root is the hierarchical alloc fork: all four contexts are
     explored and raced end to end; the run stays bitwise equal to the default."""
     import paper_conf_asplos_sivathanucsz19_b200 as A
     T, B, I, H, V = 4, 64, 64, 64, 40
     res = []
-    n_steps = 600
+    n_steps = 1500
     for mode in (A.TUNE_ON, A.TUNE_OFF):
         p, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, synth.config_seed(5) + 60, True)
         c = A.Cell("milstm", H, I, B, T, dtype="bf16")
@@ -278,15 +279,17 @@ def test_tuner_fork_explores_both_allocation_contexts():
         seen = set()
         for i in range(n_steps):
             m.train_step(tokens, 0.05)
-            seen.add("rc=1" in c.tune_report()["variant"])
+            vr = c.tune_report()["variant"]
+            seen.add(("rc=1" in vr, "gb=1" in vr))
             if c.tune_next() == A.TUNE_CONVERGED:
                 n_steps = i + 1
                 break
         torch.cuda.synchronize()
         res.append((m.params.clone(), seen))
-    assert n_steps < 600, "the tuner did not converge"
+    assert n_steps < 1500, "the tuner did not converge"
     assert torch.equal(res[0][0], res[1][0])
-    assert res[0][1] == {False, True}, "the recompute context was never explored"
+    # the four allocation contexts: store / recompute UH × gate-interleaved / gate-blocked layout
+    assert res[0][1] == {(False, False), (True, False), (False, True), (True, True)}, res[0][1]
 
 
 @pytest.mark.parametrize("hov", [0, 1])
