@@ -256,6 +256,9 @@ def main():
     # ---- online exploration (work-conserving: every explored step is a real training step)
     tune_steps, tune_t0 = 0, time.perf_counter()
     tune_info = {"mode": "off"}
+    if args.no_tune and os.environ.get("ASTRA_VARIANT"):   # A/B runs: a forced variant, no exploration
+        cell.tune_mode(A.TUNE_FROZEN, os.environ["ASTRA_VARIANT"])
+        tune_info = {"mode": "frozen (ASTRA_VARIANT)", "variant": os.environ["ASTRA_VARIANT"]}
     if not args.no_tune:
         cell.tune_mode(A.TUNE_ON)
         while True:

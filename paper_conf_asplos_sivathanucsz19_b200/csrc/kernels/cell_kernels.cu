@@ -483,7 +483,11 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
   ASTRA_CHECK_ARG(gu == GATE_U || gu == Hp, "lstm_fwd_pointwise: gate layout must be GATE_U or Hp");
   a.gu = gu;
   a.nub = cdiv(Hp, FB_UB);
-  a.rstep = std::max(1, std::min(B, 2 * num_sms() / a.nub));
+  static const int cap = [] {   // A/B knob: CTAs of one launch (row_streams experiments)
+    const char* e = std::getenv("ASTRA_FWDPW_CTAS");
+    return e ? std::atoi(e) : 0;
+  }();
+  a.rstep = std::max(1, std::min(B, (cap > 0 ? cap : 2 * num_sms()) / a.nub));
   a.WX = WX; a.UH = UH; a.gp = gp; a.c_prev = c_prev; a.c_new = c_new;
   a.h_op = h_op; a.ldh = ldh; a.y = y; a.ldy = ldy; a.hT = hT; a.cT = cT;
   a.trace = trace_buffer(TRACE_FWD_PW);   // diagnostics only (null: no stamps)
