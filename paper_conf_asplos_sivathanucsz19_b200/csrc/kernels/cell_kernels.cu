@@ -8,6 +8,8 @@
 #include "sm100.cuh"
 #include <algorithm>
 #include <cstdlib>
+#include <map>
+#include <tuple>
 
 namespace astra {
 
@@ -853,11 +855,252 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
   }
 }
 
+// K4 backward half, TMA-tiled form (AV bwd_pw = 2; large batch).  The wide form's work split (CTA =
+// one 32-row partial chunk x 32 units, thread = row x 4 units) and arithmetic (lstm_bwd_da, then the
+// R5 column sums replayed in the row-lane kernel's order: the same bits), but every operand tile is
+// landed in shared memory by the copy engine — WX_t / UH_t (4 gate boxes each), c_t, c_{t-1}, dc,
+// dy (boxes of 32 rows x 32 units, fp32) and the nsplit dh_rec partials — so no register holds a
+// load in flight: 2 CTAs per SM, each CTA's whole tile (64 KB at cfg5) requested at once, all the
+// older operands (and the chunk's column-sum partials) before the grid dependency resolves.  The
+// replay reads w, h from the operand tiles (only da is staged).
+struct Bw3Maps {
+  CUtensorMap wx, uh, p, dc, cp, cn, dy;   // fp32 [rows][cols] boxes {32, 32}; p: z = split chunk
+};
+constexpr int BW3_TILE = BWD_RB * BW2_UB;   // floats of one [32 rows][32 units] box
+constexpr int BW3_FLOATS = (4 + 4 + SPLIT_MAX + 4 + 4) * BW3_TILE + 4 * 4 * BW2_UB;   // + params
+constexpr size_t BW3_SMEM = (size_t)BW3_FLOATS * 4 + 128 + 64;
+
+template <int KIND, typename T>
+__global__ void __launch_bounds__(BW2_THREADS, 2)
+    lstm_bwd_pw3_kernel(const __grid_constant__ Bw3Maps m, int B, int H, int Hp, int nsplit, int gu,
+                        float* __restrict__ dc, GateParams gp, T* __restrict__ D_uh, T* __restrict__ D_wx,
+                        float* __restrict__ partials, int nq, int first) {
+  constexpr int NV = BwdNV<KIND>::value;
+  constexpr int NP = KIND == K_MILSTM ? 4 : 1;
+  constexpr bool F = FastMath<T>::value;
+  extern __shared__ uint8_t sm3_raw[];
+  float* smf = reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(sm3_raw) + 127) & ~uintptr_t(127));
+  float* sWX = smf;                          // [4 gates][32 rows][32 units]
+  float* sUH = sWX + 4 * BW3_TILE;
+  float* sP = sUH + 4 * BW3_TILE;            // [nsplit][32][32]
+  float* sDC = sP + SPLIT_MAX * BW3_TILE;
+  float* sCP = sDC + BW3_TILE;
+  float* sCN = sCP + BW3_TILE;
+  float* sDY = sCN + BW3_TILE;
+  float* sDA = sDY + BW3_TILE;               // [4 gates][32][32] da; later the lane sums
+  float* sgp = sDA + 4 * BW3_TILE;           // [NP][4][32]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sgp + 4 * 4 * BW2_UB);   // [0] older operands, [1] dh_rec
+  const int tid = threadIdx.x;
+  const int qd = tid % (BW2_UB / 4), r = tid / (BW2_UB / 4);
+  const int u0 = blockIdx.x * BW2_UB, ul = 4 * qd, j0 = u0 + ul;
+  const int chunk = blockIdx.y, b0 = chunk * BWD_RB, b = b0 + r;
+  const long NG = 4L * Hp;
+  const int cg0 = gcol_u(0, u0, gu);         // gate g of the tile's 32 units: columns cg0 + g·gu ..
+  constexpr uint32_t BOX = BW3_TILE * 4;
+  auto issue_old = [&] {
+    sm100::mbar_arrive_expect_tx(&bar[0], 12 * BOX);
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      sm100::tma_load_3d(sWX + g * BW3_TILE, &m.wx, &bar[0], cg0 + g * gu, b0, 0);
+      sm100::tma_load_3d(sUH + g * BW3_TILE, &m.uh, &bar[0], cg0 + g * gu, b0, 0);
+    }
+    sm100::tma_load_3d(sDC, &m.dc, &bar[0], u0, b0, 0);
+    sm100::tma_load_3d(sCP, &m.cp, &bar[0], u0, b0, 0);
+    sm100::tma_load_3d(sCN, &m.cn, &bar[0], u0, b0, 0);
+    sm100::tma_load_3d(sDY, &m.dy, &bar[0], u0, b0, 0);
+  };
+  if (tid == 0) {
+    sm100::mbar_init(&bar[0], 1);
+    sm100::mbar_init(&bar[1], 1);
+    sm100::fence_barrier_init();
+    sm100::tma_prefetch(&m.wx); sm100::tma_prefetch(&m.uh); sm100::tma_prefetch(&m.p);
+  }
+  __syncthreads();
+  // the previous step's column-sum partials of this chunk (written two launches back: complete)
+  float pre[2] = {0.f, 0.f};
+  for (int k = 0, item = tid; item < NV * BW2_UB; item += BW2_THREADS, ++k) {
+    const int u = item % BW2_UB, i = item / BW2_UB, j = u0 + u, q = i / 4, g = i % 4;
+    if (!first && q < nq && j < Hp) pre[k] = partials[(long)chunk * nq * NG + (long)q * NG + gcol_u(g, j, gu)];
+  }
+  // operands older than the grid dependency: all but dh_rec (not at the first step, whose
+  // predecessor may have produced dy or initialised dc)
+  if (tid == 0 && !first) issue_old();
+  for (int i = tid; i < NP * 4 * BW2_UB; i += BW2_THREADS) {   // parameters: not written by the chain
+    const int pi = i / (4 * BW2_UB), g = (i / BW2_UB) % 4, u = i % BW2_UB, j = u0 + u;
+    const float* src = pi == 0 ? gp.b : pi == 1 ? gp.alpha : pi == 2 ? gp.beta1 : gp.beta2;
+    sgp[i] = j < H ? src[g * H + j] : 0.f;
+  }
+  pdl_wait();
+  pdl_trigger();
+  if (tid == 0) {
+    if (first) issue_old();
+    sm100::mbar_arrive_expect_tx(&bar[1], (uint32_t)nsplit * BOX);
+    for (int k = 0; k < nsplit; ++k) sm100::tma_load_3d(sP + k * BW3_TILE, &m.p, &bar[1], u0, b0, k);
+  }
+  __syncthreads();   // parameters staged
+  sm100::mbar_wait(&bar[0], 0);
+  sm100::mbar_wait(&bar[1], 0);
+  const bool rowok = b < B;
+  const int nvalid = min(4, H - j0);
+  const int c0 = gcol_u(0, j0, gu);
+  const long ro = (long)b * Hp + j0;
+  const int so = r * BW2_UB + ul;            // this thread's offset in a [32][32] tile
+  if (rowok) {
+    float duh4[4][4], dwx4[4][4], dcn[4];
+    if (nvalid > 0) {
+      float4 w4[4], h4[4];
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        w4[g] = *reinterpret_cast<const float4*>(sWX + g * BW3_TILE + so);
+        h4[g] = *reinterpret_cast<const float4*>(sUH + g * BW3_TILE + so);
+      }
+      const float4 dc4 = *reinterpret_cast<const float4*>(sDC + so);
+      const float4 cp4 = *reinterpret_cast<const float4*>(sCP + so);
+      const float4 cn4 = *reinterpret_cast<const float4*>(sCN + so);
+      const float4 dy4 = *reinterpret_cast<const float4*>(sDY + so);
+      float4 pv[SPLIT_MAX];
+#pragma unroll
+      for (int k = 0; k < SPLIT_MAX; ++k)
+        pv[k] = k < nsplit ? *reinterpret_cast<const float4*>(sP + k * BW3_TILE + so) : make_float4(0, 0, 0, 0);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        // split-K partials of dh_rec summed in chunk order, then added to dy (the other forms' order)
+        float sacc = f4(pv[0], u);
+#pragma unroll
+        for (int k = 1; k < SPLIT_MAX; ++k)
+          if (k < nsplit) sacc = __fadd_rn(sacc, f4(pv[k], u));
+        const float dh = __fadd_rn(f4(dy4, u), sacc);
+        float w[4], h[4], bb[4], al[4], be1[4], be2[4], da[4], duh[4], dwx[4];
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          w[g] = f4(w4[g], u);
+          h[g] = f4(h4[g], u);
+          bb[g] = sgp[g * BW2_UB + ul + u];
+          al[g] = KIND == K_MILSTM ? sgp[(NP > 1 ? 1 : 0) * 4 * BW2_UB + g * BW2_UB + ul + u] : 0.f;
+          be1[g] = KIND == K_MILSTM ? sgp[(NP > 2 ? 2 : 0) * 4 * BW2_UB + g * BW2_UB + ul + u] : 0.f;
+          be2[g] = KIND == K_MILSTM ? sgp[(NP > 3 ? 3 : 0) * 4 * BW2_UB + g * BW2_UB + ul + u] : 0.f;
+        }
+        float dcv = f4(dc4, u);
+        if (u < nvalid) {
+          lstm_bwd_da<KIND, F>(w, h, dh, dcv, f4(cp4, u), f4(cn4, u), bb, al, be1, be2, da, duh, dwx);
+        } else {   // padding units: exact zeros everywhere
+#pragma unroll
+          for (int g = 0; g < 4; ++g) { da[g] = 0.f; duh[g] = 0.f; dwx[g] = 0.f; }
+          dcv = 0.f;
+        }
+        dcn[u] = dcv;
+#pragma unroll
+        for (int g = 0; g < 4; ++g) {
+          sDA[g * BW3_TILE + so + u] = da[g];
+          duh4[u][g] = duh[g]; dwx4[u][g] = dwx[g];
+        }
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        dcn[u] = 0.f;
+#pragma unroll
+        for (int g = 0; g < 4; ++g) { sDA[g * BW3_TILE + so + u] = 0.f; duh4[u][g] = 0.f; dwx4[u][g] = 0.f; }
+      }
+    }
+#pragma unroll
+    for (int g = 0; g < 4; ++g) {
+      float v[4] = {duh4[0][g], duh4[1][g], duh4[2][g], duh4[3][g]};
+      store4<T>(D_uh + (long)b * NG + c0 + g * gu, v);
+      if (KIND == K_MILSTM) {
+        float x[4] = {dwx4[0][g], dwx4[1][g], dwx4[2][g], dwx4[3][g]};
+        store4<T>(D_wx + (long)b * NG + c0 + g * gu, x);
+      }
+    }
+    *reinterpret_cast<float4*>(dc + ro) = make_float4(dcn[0], dcn[1], dcn[2], dcn[3]);
+  }
+  __syncthreads();
+  // lane sums: thread (u, y) accumulates rows y, y+4, ... of the chunk in ascending order, every gate
+  // (lstm_bwd_pw2_kernel's replay; w, h of padding units are zero there, so here too)
+  const int nrows = min(BWD_RB, B - b0);
+  float acc[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) acc[i] = 0.f;
+  const int su = tid % BW2_UB, sy = tid / BW2_UB;
+  const bool uvalid = u0 + su < H;
+  if (tid < BWD_RY * BW2_UB) {
+    for (int rr = sy; rr < nrows; rr += BWD_RY) {
+#pragma unroll
+      for (int g = 0; g < 4; ++g) {
+        const int o = g * BW3_TILE + rr * BW2_UB + su;
+        const float da = sDA[o];
+        const float w = (KIND == K_MILSTM && uvalid) ? sWX[o] : 0.f;
+        const float h = (KIND == K_MILSTM && uvalid) ? sUH[o] : 0.f;
+        lstm_bwd_acc<KIND, F>(acc, g, da, w, h);
+      }
+    }
+  }
+  __syncthreads();   // contributions consumed: the same memory holds the lane sums
+  float* red = sDA;  // [4 lanes][NV][BW2_UB]
+  if (tid < BWD_RY * BW2_UB) {
+#pragma unroll
+    for (int i = 0; i < NV; ++i) red[(sy * NV + i) * BW2_UB + su] = acc[i];
+  }
+  __syncthreads();
+  for (int k = 0, item = tid; item < NV * BW2_UB; item += BW2_THREADS, ++k) {
+    const int u = item % BW2_UB, i = item / BW2_UB, j = u0 + u;
+    const int q = i / 4, g = i % 4;
+    if (q >= nq || j >= Hp) continue;
+    float v = 0.f;
+#pragma unroll
+    for (int y = 0; y < BWD_RY; ++y) v = __fadd_rn(v, red[(y * NV + i) * BW2_UB + u]);
+    partials[(long)chunk * nq * NG + (long)q * NG + gcol_u(g, j, gu)] = first ? v : __fadd_rn(pre[k], v);
+  }
+}
+
+// fp32 tile maps of the TMA-tiled form, cached by (pointer, shape): the per-step operand pointers
+// repeat every training step, so each map is encoded once
+static const CUtensorMap& bw3_map(const void* ptr, long inner, long rows, long z, long ld, long zstride) {
+  using Key = std::tuple<const void*, long, long, long, long, long>;
+  static std::map<Key, CUtensorMap> cache;
+  const Key k{ptr, inner, rows, z, ld, zstride};
+  auto it = cache.find(k);
+  if (it != cache.end()) return it->second;
+  if (cache.size() > 16384) cache.clear();
+  CUtensorMap mm;
+  make_tile_map(&mm, ptr, false, inner, rows, z, ld, zstride, 32, 32, 0);
+  return cache.emplace(k, mm).first->second;
+}
+
 template <int KIND, typename T>
 static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_ot, bool dy_f32, const float* dh_rec,
                           long ld_dh, int nsplit, long split_stride, float* dc, const float* WX, const float* UH, const float* c_new,
                           const float* c_prev, GateParams gp, void* D_uh, void* D_wx, float* partials, int nq,
                           bool first, cudaStream_t st, int form, int gu) {
+  // the TMA-tiled form needs fp32 dy (the LM's internal dY), split partials of dh_rec, 16-byte rows
+  if (form == 2) {
+    const bool ok = !first && dh_rec && nsplit >= 1 && nsplit <= SPLIT_MAX && (dy_f32 || dy_ot == OT::F32) && ld_dh % 4 == 0 &&
+                    split_stride % 4 == 0 && ldy % 4 == 0 && Hp % BW2_UB == 0 && ((uintptr_t)dh_rec & 15) == 0 &&
+                    ((uintptr_t)dy & 15) == 0 && ((uintptr_t)WX & 15) == 0 && ((uintptr_t)UH & 15) == 0 &&
+                    ((uintptr_t)c_new & 15) == 0 && ((uintptr_t)c_prev & 15) == 0 && ((uintptr_t)dc & 15) == 0;
+    if (!ok && !first && std::getenv("ASTRA_BPW2_STRICT"))   // tests: prove the tiled form runs
+      throw Error(ASTRA_E_UNSUPPORTED, "lstm_bwd_pointwise: the TMA-tiled form cannot run this step");
+    if (!ok) form = 1;
+  }
+  if (form == 2) {
+    const long NG = 4L * Hp;
+    Bw3Maps m;
+    m.wx = bw3_map(WX, NG, B, 1, NG, 0);
+    m.uh = bw3_map(UH, NG, B, 1, NG, 0);
+    m.p = bw3_map(dh_rec, Hp, B, nsplit, ld_dh, split_stride);
+    m.dc = bw3_map(dc, Hp, B, 1, Hp, 0);
+    m.cp = bw3_map(c_prev, Hp, B, 1, Hp, 0);
+    m.cn = bw3_map(c_new, Hp, B, 1, Hp, 0);
+    m.dy = bw3_map(dy, Hp, B, 1, ldy, 0);
+    auto k = lstm_bwd_pw3_kernel<KIND, T>;
+    static bool attr = false;
+    if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)BW3_SMEM)); attr = true; }
+    dim3 grid3(Hp / BW2_UB, lstm_bwd_row_chunks(B));
+    launch_pdl(k, grid3, dim3(BW2_THREADS), BW3_SMEM, st, 1, m, B, H, Hp, nsplit, gu, dc, gp, (T*)D_uh, (T*)D_wx,
+               partials, nq, (int)first);
+    LAUNCH_CHECK();
+    return;
+  }
   if (form == 1) {
     constexpr int NC = KIND == K_MILSTM ? 3 : 1, NP = KIND == K_MILSTM ? 4 : 1;
     const size_t smem = (size_t)(NC * 4 * BWD_RB * BW2_UB + NP * 4 * BW2_UB) * 4;

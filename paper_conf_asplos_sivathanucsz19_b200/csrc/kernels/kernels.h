@@ -48,7 +48,9 @@ void lstm_bwd_pointwise(int kind, OT ot, int B, int H, int Hp, const void* dy, l
                         const float* c_new, const float* c_prev, GateParams gp, void* D_uh, void* D_wx,
                         float* partials, int nq, bool first, cudaStream_t st, int form = 0, int gu = 64);
 // form (AV "bwd_pw", bitwise interchangeable): 0 the row-lane kernel (thread = unit, rows walked 4
-// lanes x 8), 1 the wide kernel (thread = row x 4 units, all rows of a 32-row chunk in flight).
+// lanes x 8), 1 the wide kernel (thread = row x 4 units, all rows of a 32-row chunk in flight), 2 the
+// wide kernel with its operand tiles landed in shared memory by TMA (fp32 dy and split dh_rec partials
+// only, not at the first step; otherwise it runs form 1).
 int lstm_bwd_row_chunks(int B);
 constexpr int BWD_ROW_CHUNK = 32;   // rows per column-partial chunk of the backward pointwise kernels (R5)
 // grads_q[e] = Σ_chunk partials[chunk][q][gcol(e)] for q < nq (external e < 4H).

@@ -61,7 +61,8 @@ struct Variant {
                         // independent chains on two streams (the sequences are independent), so one half's
                         // pointwise kernel overlaps the other half's recurrent GEMM (LSTM family, B ≥ 256)
   int bpw = 0;          // bwd_pw (§8(a.9) bwd_kernel / bwd_epilogue): backward pointwise form, 0 row-lane (unit per
-                        // thread, 8 rows walked), 1 wide (row x 4 units per thread, whole 32-row chunk in flight)
+                        // thread, 8 rows walked), 1 wide (row x 4 units per thread, whole 32-row chunk in flight),
+                        // 2 wide with every operand tile landed in shared memory by TMA (fp32 dY: LM mode)
   int wgs = 0;          // wgrad_schedule (§8(a.9)): the input dgrad dX in WGS_CHUNKS[wgs] time chunks,
                         // each issued on a side stream as soon as BPTT has produced its rows (0: after BPTT)
   int gchunk = 0;       // gate_chunking (§8(a.9), "chunking the fusion group", P:220 chunk sizes): the

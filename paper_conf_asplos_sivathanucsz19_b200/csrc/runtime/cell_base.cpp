@@ -63,7 +63,7 @@ Variant Variant::parse(const std::string& s) {
     }
     if (k == "bpw") {
       v.bpw = std::stoi(val);
-      ASTRA_CHECK_ARG(v.bpw == 0 || v.bpw == 1, "variant: bpw (backward pointwise form) must be 0 or 1");
+      ASTRA_CHECK_ARG(v.bpw >= 0 && v.bpw <= 2, "variant: bpw (backward pointwise form) must be 0..2");
       continue;
     }
     if (k == "wgs") {

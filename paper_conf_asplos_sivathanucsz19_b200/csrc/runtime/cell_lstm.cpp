@@ -90,7 +90,8 @@ class LstmCell : public Cell {
   // persistent (256-column tiles), 3 small-batch persistent with the U slice resident (B ≤ 128)
   int gate_chunkings() const override { return ot == OT::BF16 ? (side.empty() ? 3 : 5) : 1; }
   int wgrad_schedules() const override { return (ot == OT::BF16 && T >= 4) ? 3 : 1; }
-  int bwd_pw_forms() const override { return ot == OT::BF16 ? 2 : 1; }
+  // backward pointwise forms (AV bwd_pw): 0 row-lane, 1 wide, 2 wide with TMA-tiled operands (the LM's fp32 dY)
+  int bwd_pw_forms() const override { return ot == OT::BF16 ? (lm_mode ? 3 : 2) : 1; }
   int row_stream_options() const override { return (ot == OT::BF16 && B >= 256 && B % 64 == 0) ? 2 : 1; }
   cudaEvent_t ev_rs[2] = {nullptr, nullptr};   // row_streams fork / join
   // the two row halves of the chains as independent chains on (main, side[0]): value-preserving —

@@ -361,6 +361,34 @@ def test_tune_next_never_blocks():
     assert rep["configs_explored"] >= 10 and rep["converged"]
 
 
+@pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
+@pytest.mark.parametrize("T,B,H", [(4, 300, 192), (3, 512, 2048), (5, 40, 130)])
+def test_bwd_pointwise_tiled_lm_bitwise(cell, T, B, H, monkeypatch):
+    """The TMA-tiled backward pointwise form (bwd_pw = 2: operand tiles landed in shared memory, the
+    older ones before the grid dependency) gives the row-lane and wide forms' bits over 3 LM SGD
+    steps (graph replay) — ragged row chunks (B = 300, 40), padding units (H = 130), the R25 4-way
+    split at cfg5's H = 2048, the gate-blocked layout too.  ASTRA_BPW2_STRICT makes a fallback to the
+    wide form an error, so the tiled kernel really ran at every step but the first."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    monkeypatch.setenv("ASTRA_BPW2_STRICT", "1")
+    V = 64
+    out = {}
+    for v in ("bpw=0", "bpw=1", "bpw=2", "bpw=2,gb=1"):
+        p, tok, h0, c0 = _lm_case(cell, T, B, 64, H, V, synth.config_seed(5) + 31, True)
+        c = A.Cell(cell, H, 64, B, T, dtype="bf16")
+        m = A.LM(c, V)
+        m.load(p)
+        m.set_graph(True)
+        c.tune_mode(A.TUNE_FROZEN, v)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(3):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out[v] = (m.params.clone(), float(m.loss.item()))
+    for v in out:
+        assert torch.equal(out[v][0], out["bpw=0"][0]) and out[v][1] == out["bpw=0"][1], v
+
+
 @pytest.mark.parametrize("variant", ["hov=1,wgs=2,gc=3,wg_side=1", "wgs=1,gc=4,fwd=3", "gc=2,wgs=2,rc=1",
                                      "rsp=1,bpw=1,gc=3", "hdy=128.1.1.2,head=128.1.1", "hdy=64.2.1"])
 def test_stream_schedules_lm_bitwise(variant):
