@@ -542,7 +542,7 @@ int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 // rows b0 + ty, b0 + ty + 4, ...; a warp reads 128-byte runs of every gate's pre-activations.  The
 // row arithmetic and the column-sum order are lstm_bwd_row.cuh's, shared with the fused BPTT kernel.
 // 256-thread CTAs at <= 64 registers: one resident wave at B = 512.
-template <int KIND, typename T, typename TDY>
+template <int KIND, typename T, typename TDY, bool BLK>
 __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
     lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
                        long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
@@ -563,7 +563,16 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   const int chunk = blockIdx.y;
   const int NG = 4 * Hp;
   const int b0 = chunk * BWD_RB, b1 = min(B, b0 + BWD_RB);
-  const int c0 = gcol_u(0, j, gu);   // gate g of unit j at c0 + g·gu (the `alloc` layout)
+  // gate stride of the `alloc` layout: the interleaved one is a compile-time 64 (folded into the
+  // address offsets), the gate-blocked one Hp
+  const int gs = BLK ? gu : GATE_U;
+  const int c0 = BLK ? j : gcol(0, j);   // gate g of unit j at column c0 + g·gs
+  // Per-thread 32-bit element offsets of the first row (one step's tensors: B·4Hp < 2^31, checked by
+  // the launcher), advanced by BWD_RY rows per iteration: the row loop's address arithmetic is an
+  // add per operand instead of fresh 64-bit products, without holding nine 64-bit pointers
+  const int bf = b0 + ty;
+  int o_ng = bf * NG + c0, o_hp = bf * Hp + j, o_dy = bf * (int)ldy + j, o_dh = bf * (int)ld_dh + j;
+  const int st_ng = BWD_RY * NG, st_hp = BWD_RY * Hp, st_dy = BWD_RY * (int)ldy, st_dh = BWD_RY * (int)ld_dh;
   // Operands of one row.  Only dh_rec is produced by the predecessor (the BPTT GEMM); WX, UH, the
   // cell states and dy are older, and dc was written by the pointwise kernel two launches back
   // (complete: the GEMM waits on it before triggering this launch).  So the first row is loaded
@@ -571,21 +580,18 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   // first step (`first`): its predecessor may be the kernel that initialised dc or produced dy.
   const bool early = !first;
   float w[4], h[4], dcv = 0.f, cp = 0.f, cn = 0.f, dyv = 0.f;
-  auto load_row = [&](int b) {
-    const float* wxp = WX + (long)b * NG + c0;
-    const float* uhp = UH + (long)b * NG + c0;
+  auto load_row = [&] {
 #pragma unroll
     for (int g = 0; g < 4; ++g) {
-      w[g] = __ldcs(wxp + g * gu);
-      h[g] = __ldcs(uhp + g * gu);
+      w[g] = __ldcs(WX + o_ng + g * gs);
+      h[g] = __ldcs(UH + o_ng + g * gs);
     }
-    const long ro = (long)b * Hp + j;
-    dcv = dc[ro];
-    cp = c_prev[ro];
-    cn = c_new[ro];
-    dyv = to_f<TDY>(dy[(long)b * ldy + j]);
+    dcv = dc[o_hp];
+    cp = c_prev[o_hp];
+    cn = c_new[o_hp];
+    dyv = to_f<TDY>(dy[o_dy]);
   };
-  if (early && j < H && b0 + ty < b1) load_row(b0 + ty);
+  if (early && j < H && bf < b1) load_row();
   pdl_wait();
   pdl_trigger();
   __syncthreads();
@@ -594,13 +600,12 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   for (int i = 0; i < NV; ++i) acc[i] = 0.f;
   if (j < H) {
 #pragma unroll 1
-    for (int b = b0 + ty; b < b1; b += BWD_RY) {
+    for (int b = bf; b < b1; b += BWD_RY) {
       // every operand of the row is loaded before any arithmetic: one memory latency per row
-      if (!early || b != b0 + ty) load_row(b);
-      const long ro = (long)b * Hp + j;
+      if (!early || b != bf) load_row();
       float dh = dyv;
       if (dh_rec)   // split-K partials of dh_rec summed in chunk order, then added to dy
-        dh = __fadd_rn(dh, sum_split(dh_rec + (long)b * ld_dh + j, nsplit, split_stride));
+        dh = __fadd_rn(dh, sum_split(dh_rec + o_dh, nsplit, split_stride));
       float bb[4], al[4], be1[4], be2[4];
       const volatile float* sg = &sgp[0][0][tx];   // volatile: re-read each row, not hoisted into registers
 #pragma unroll
@@ -610,16 +615,16 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
         be1[g] = KIND == K_MILSTM ? sg[(NP > 2 ? 8 : 0) * BWD_UX + g * BWD_UX] : 0.f;
         be2[g] = KIND == K_MILSTM ? sg[(NP > 3 ? 12 : 0) * BWD_UX + g * BWD_UX] : 0.f;
       }
-      lstm_bwd_row<KIND, T>(w, h, dh, dcv, cp, cn, bb, al, be1, be2, acc, D_uh + (long)b * NG + c0,
-                            D_wx + (long)b * NG + c0, gu);
-      dc[ro] = dcv;
+      lstm_bwd_row<KIND, T>(w, h, dh, dcv, cp, cn, bb, al, be1, be2, acc, D_uh + o_ng, D_wx + o_ng, gs);
+      dc[o_hp] = dcv;
+      o_ng += st_ng; o_hp += st_hp; o_dy += st_dy; o_dh += st_dh;
     }
   } else if (j < Hp) {  // padding units: keep their gradients exactly zero
-    for (int b = b0 + ty; b < b1; b += BWD_RY) {
+    for (int b = bf; b < b1; b += BWD_RY) {
 #pragma unroll
       for (int g = 0; g < 4; ++g) {
-        D_uh[(long)b * NG + gcol_u(g, j, gu)] = from_f<T>(0.f);
-        if (KIND == K_MILSTM) D_wx[(long)b * NG + gcol_u(g, j, gu)] = from_f<T>(0.f);
+        D_uh[(long)b * NG + c0 + g * gs] = from_f<T>(0.f);
+        if (KIND == K_MILSTM) D_wx[(long)b * NG + c0 + g * gs] = from_f<T>(0.f);
       }
       dc[(long)b * Hp + j] = 0.f;
     }
@@ -628,7 +633,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   for (int i = 0; i < NV; ++i) red[ty][i][tx] = acc[i];
   __syncthreads();
   if (j >= Hp) return;
-  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, gcol_u(0, j, gu), nq, first, gu);
+  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, c0, nq, first, gs);
 }
 
 // K4 backward half, wide form (AV bwd_pw = 1; measured faster at small batch — B = 64: BPTT chain
@@ -1123,14 +1128,17 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
   }
   dim3 grid(cdiv(Hp, BWD_UX), lstm_bwd_row_chunks(B));
   dim3 block(BWD_UX, BWD_RY);
+  const bool blk = gu != GATE_U;
+  ASTRA_CHECK_ARG((long)B * 4 * Hp < (1L << 31) && (long)B * ldy < (1L << 31) && (long)B * ld_dh < (1L << 31),
+                  "lstm_bwd_pointwise: one step's tensors must have < 2^31 elements");
   if (dy_f32 || dy_ot == OT::F32)
-    launch_pdl(lstm_bwd_pw_kernel<KIND, T, float>, grid, block, 0, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec,
-               ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq,
-               (int)first, gu);
+    launch_pdl(blk ? lstm_bwd_pw_kernel<KIND, T, float, true> : lstm_bwd_pw_kernel<KIND, T, float, false>, grid, block,
+               0, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev,
+               gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
   else
-    launch_pdl(lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16>, grid, block, 0, st, 1, B, H, Hp,
-               (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev, gp,
-               (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
+    launch_pdl(blk ? lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16, true> : lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16, false>,
+               grid, block, 0, st, 1, B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc,
+               WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
   LAUNCH_CHECK();
 }
 
