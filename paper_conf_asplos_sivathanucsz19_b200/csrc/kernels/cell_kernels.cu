@@ -542,7 +542,7 @@ int lstm_bwd_row_chunks(int B) { return cdiv(B, BWD_RB); }
 // rows b0 + ty, b0 + ty + 4, ...; a warp reads 128-byte runs of every gate's pre-activations.  The
 // row arithmetic and the column-sum order are lstm_bwd_row.cuh's, shared with the fused BPTT kernel.
 // 256-thread CTAs at <= 64 registers: one resident wave at B = 512.
-template <int KIND, typename T, typename TDY, bool BLK>
+template <int KIND, typename T, typename TDY, bool BLK, int NS>
 __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
     lstm_bwd_pw_kernel(int B, int H, int Hp, const TDY* __restrict__ dy, long ldy, const float* __restrict__ dh_rec,
                        long ld_dh, int nsplit, long split_stride, float* __restrict__ dc,
@@ -605,7 +605,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
       if (!early || b != bf) load_row();
       float dh = dyv;
       if (dh_rec)   // split-K partials of dh_rec summed in chunk order, then added to dy
-        dh = __fadd_rn(dh, sum_split(dh_rec + o_dh, nsplit, split_stride));
+        dh = __fadd_rn(dh, sum_split_n<NS>(dh_rec + o_dh, nsplit, split_stride));
       float bb[4], al[4], be1[4], be2[4];
       const volatile float* sg = &sgp[0][0][tx];   // volatile: re-read each row, not hoisted into registers
 #pragma unroll
@@ -1131,14 +1131,21 @@ static void bwd_pw_launch(int B, int H, int Hp, const void* dy, long ldy, OT dy_
   const bool blk = gu != GATE_U;
   ASTRA_CHECK_ARG((long)B * 4 * Hp < (1L << 31) && (long)B * ldy < (1L << 31) && (long)B * ld_dh < (1L << 31),
                   "lstm_bwd_pointwise: one step's tensors must have < 2^31 elements");
-  if (dy_f32 || dy_ot == OT::F32)
-    launch_pdl(blk ? lstm_bwd_pw_kernel<KIND, T, float, true> : lstm_bwd_pw_kernel<KIND, T, float, false>, grid, block,
-               0, st, 1, B, H, Hp, (const float*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH, c_new, c_prev,
-               gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
-  else
-    launch_pdl(blk ? lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16, true> : lstm_bwd_pw_kernel<KIND, T, __nv_bfloat16, false>,
-               grid, block, 0, st, 1, B, H, Hp, (const __nv_bfloat16*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc,
-               WX, UH, c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
+  // compile-time split count for the R25 splits the chains use (4 at cfg5, 2, 1), else generic
+  const int ns = !dh_rec ? 1 : (nsplit == 4 || nsplit == 2 || nsplit == 1) ? nsplit : 0;
+  auto pick = [&](auto tdy) {
+    using TD = decltype(tdy);
+    void (*k)(int, int, int, const TD*, long, const float*, long, int, long, float*, const float*, const float*,
+              const float*, const float*, GateParams, T*, T*, float*, int, int, int) = nullptr;
+#define BWD_NS(N) \
+    if (ns == N) k = blk ? lstm_bwd_pw_kernel<KIND, T, TD, true, N> : lstm_bwd_pw_kernel<KIND, T, TD, false, N>;
+    BWD_NS(0) BWD_NS(1) BWD_NS(2) BWD_NS(4)
+#undef BWD_NS
+    launch_pdl(k, grid, block, 0, st, 1, B, H, Hp, (const TD*)dy, ldy, dh_rec, ld_dh, nsplit, split_stride, dc, WX, UH,
+               c_new, c_prev, gp, (T*)D_uh, (T*)D_wx, partials, nq, (int)first, gu);
+  };
+  if (dy_f32 || dy_ot == OT::F32) pick(float{});
+  else pick(__nv_bfloat16{});
   LAUNCH_CHECK();
 }
 

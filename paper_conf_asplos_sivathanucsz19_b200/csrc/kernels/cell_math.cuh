@@ -59,6 +59,23 @@ __device__ __forceinline__ float sum_split(const float* __restrict__ p, int n, l
   return r;
 }
 
+// The same sum with the chunk count fixed at compile time (NS > 0; NS = 0: sum_split): the loads
+// are unpredicated and the adds in the same order.
+template <int NS>
+__device__ __forceinline__ float sum_split_n(const float* __restrict__ p, int n, long s) {
+  if constexpr (NS == 0) {
+    return sum_split(p, n, s);
+  } else {
+    float v[NS];
+#pragma unroll
+    for (int k = 0; k < NS; ++k) v[k] = p[k * s];
+    float r = v[0];
+#pragma unroll
+    for (int k = 1; k < NS; ++k) r = __fadd_rn(r, v[k]);
+    return r;
+  }
+}
+
 enum CellKind { K_LSTM = 0, K_MILSTM = 1, K_SUBLSTM = 5 };
 
 // Pre-activation of one gate.  LSTM/subLSTM: a = wx + uh + b.
