@@ -269,6 +269,9 @@ def main():
                 break
         torch.cuda.synchronize()
         rep = cell.tune_report()
+        if os.environ.get("ASTRA_DUMP_REPORT"):   # diagnostics: the tuner's profile index
+            with open(os.environ["ASTRA_DUMP_REPORT"], "w") as f:
+                json.dump(rep, f)
         cell.tune_mode(A.TUNE_FROZEN, rep["variant"])
         tune_info = {"mode": "explored then frozen", "converged": s == A.TUNE_CONVERGED, "steps": tune_steps,
                      "configs_explored": rep.get("configs_explored"), "harvest_waits": rep.get("harvest_waits"),

@@ -133,6 +133,10 @@ class Cell {
   std::unique_ptr<tuner::Wirer> wirer;
   std::vector<Variant> configs_seen;
   int tune_reps = 3, rep_i = 0;
+  // measured steps left in flight when the host waits for a configuration's reps (1: the step just
+  // enqueued).  2 was measured at cfg5 (profiles/r2s5_tune_lag.txt): the same decisions, the same
+  // exploration-vs-frozen gap of the unfused forward chain (2.7 vs 3.1 ms), 20 % more steps — kept 1
+  int tune_lag = 1;
   tuner::Metrics rep_min;
   // Region events live in a ring of per-step slots, so the tuner can harvest a
   // measured step with cudaEventQuery some steps later instead of blocking on it (include/astra.h

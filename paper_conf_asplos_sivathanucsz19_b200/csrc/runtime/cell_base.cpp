@@ -541,7 +541,7 @@ void Cell::harvest(int wait) {
   for (; k < pending.size(); ++k) {
     const PendingRep& p = pending[k];
     cudaEvent_t end = evr[p.slot][R_STEP][1];
-    if (wait == 2 || (wait == 1 && k + 1 < pending.size())) {
+    if (wait == 2 || (wait == 1 && k + tune_lag < pending.size())) {
       if (cudaEventQuery(end) == cudaErrorNotReady) ++tune_blocks;
       CUDA_TRY(cudaEventSynchronize(end));
     } else {
@@ -573,9 +573,9 @@ void Cell::harvest(int wait) {
 // Never waits for the step just enqueued (include/astra.h): a measured step's events are harvested
 // with cudaEventQuery once the GPU has finished it; the configuration keeps running (real training
 // steps, so the exploration stays work-conserving) until tune_reps of its measured steps are in,
-// waiting at most for the steps BEFORE the newest one — the GPU is busy with the newest meanwhile,
-// so host and GPU stay pipelined and a configuration costs at most 1 warm-up + tune_reps + 1
-// steps.  With world > 1 every rank must decide at the same step (reading R29), so there the
+// waiting at most for the steps before the newest tune_lag (1) — the GPU is busy with those
+// meanwhile, so host and GPU stay pipelined and a configuration costs at most 1 warm-up + tune_reps
+// + tune_lag steps.  With world > 1 every rank must decide at the same step (reading R29), so there the
 // decision step is fixed — the tune_reps-th measured step — and waits for its events.
 int Cell::tune_next() {
   if (tune_mode != ASTRA_TUNE_ON) return tune_mode == ASTRA_TUNE_FROZEN ? ASTRA_TUNE_CONVERGED : ASTRA_TUNE_IDLE;
@@ -605,7 +605,7 @@ int Cell::tune_next() {
   // one rank: once tune_reps measured steps precede the newest, wait for those (the newest keeps
   // running on the GPU), else only fold in what has finished
   if (world > 1) harvest(rep_i > tune_reps ? 2 : 0);
-  else harvest(rep_i > tune_reps + 1 ? 1 : 0);
+  else harvest(rep_i > tune_reps + tune_lag ? 1 : 0);
   if (reps_harvested < tune_reps) {
     advance();
     return ASTRA_TUNE_EXPLORING;

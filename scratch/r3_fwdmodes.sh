@@ -1,0 +1,11 @@
+#!/bin/bash
+mkdir -p gpurun_out
+V="a1=256.1.1.2,rec=256.1.1,bptt=256.1.1.2,du=256.1.1.2,dw=256.1.1.2,dx=256.1.1.2,head=256.1.1,hdy=256.1.1,wg_side=1,bwd=0,pf=0,hov=0,gc=3,bpw=0"
+for r in 1 2; do for f in 0 1 2; do
+  echo "== fwd=$f" >> gpurun_out/r3f_ab.log
+  ASTRA_VARIANT="$V,fwd=$f" timeout 300 python bench.py --no-tune --no-cpu-baseline --steps 20 2>&1 | grep '^{' | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['ms_per_step'], d['regions_ms'], d['clocks'].get('sm_mhz'))" >> gpurun_out/r3f_ab.log 2>&1
+done; done
+for r in 1 2; do for b in 0 1; do
+  echo "== bwd=$b" >> gpurun_out/r3f_ab.log
+  ASTRA_VARIANT="$V,fwd=0,bwd=$b" timeout 300 python bench.py --no-tune --no-cpu-baseline --steps 20 2>&1 | grep '^{' | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['ms_per_step'], d['regions_ms'], d['clocks'].get('sm_mhz'))" >> gpurun_out/r3f_ab.log 2>&1
+done; done
