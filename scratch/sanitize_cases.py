@@ -34,6 +34,28 @@ elif case == "gemm_kb":        # K1 with multi-k-block stages (K-major and MN-ma
 elif case == "rhn_bptt":       # persistent RHN BPTT (bwd=1: clusters of 4, R33 split of 4)
     p, inp, dY, dhT, dcT = make_cell_case("rhn", 2, 16, 64, 512, 5, bf16=True, L=2)   # Hp 512: split of 4
     run_gpu_cell("rhn", p, inp, dY, dhT, dcT, "bf16", "bwd=1", depth=2)
+elif case == "bwd_pw3":        # TMA-tiled backward pointwise (bpw=2, LM mode: fp32 dY, 2-way split at H = 1024)
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    sys.path.insert(0, "/root/repo/tests")
+    from test_gpu_lm import _lm_case
+    import synth
+    for H in (130, 1024):
+        pa, tok, h0, c0 = _lm_case("milstm", 3, 40, 64, H, 64, synth.config_seed(5) + 31, True)
+        c = A.Cell("milstm", H, 64, 40, 3, dtype="bf16")
+        m = A.LM(c, 64)
+        m.load(pa)
+        c.tune_mode(A.TUNE_FROZEN, "bpw=2,gb=1" if H == 1024 else "bpw=2")
+        m.train_step(torch.as_tensor(tok, dtype=torch.int32, device=c.device), 0.1)
+elif case == "attn_dec_fused":  # attentive decoder's fused step: one-step persistent (B <= 128) and rec_fused (B > 128)
+    import synth
+    from test_gpu_cell import _attn_check
+    from helpers import TOL_BF16
+    for B in (37, 160):
+        _attn_check(3, 3, B, 64, 128, 128, "bf16", synth.config_seed(4) + 7, TOL_BF16, variant="fwd=3")
+elif case == "gate_blocked":   # gate-blocked layout (kperm GEMMs, per-gate a1, both pointwise forms)
+    p, inp, dY, dhT, dcT = make_cell_case("milstm", 3, 72, 64, 1024, 5, bf16=True)
+    for v in ("gb=1,gc=2", "gb=1,bpw=1,bptt=128.1.1.2"):
+        run_gpu_cell("milstm", p, inp, dY, dhT, dcT, "bf16", v)
 else:
     raise SystemExit(f"unknown case {case}")
 torch.cuda.synchronize()
