@@ -341,7 +341,7 @@ __device__ __forceinline__ void store_pair(T* p, bool vec, float a, float b, boo
   }
 }
 
-template <int KIND, typename T, typename TY>
+template <int KIND, typename T, typename TY, bool BLK>
 __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwArgs a) {
   constexpr int NP = KIND == K_MILSTM ? 4 : 1;
   extern __shared__ __align__(128) uint8_t sm[];
@@ -358,7 +358,7 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   // stages go out before griddepcontrol.wait; UH_t (the GEMM's output) after it.
   // interleaved layout: the CTA's units' four gates are one contiguous run of 4·nu columns; gate-
   // blocked: four runs of nu columns (g·Hp + u0), landed at gate offsets g·FB_UB of the stage
-  const bool blk = a.gu != GATE_U;
+  constexpr bool blk = BLK;   // the `alloc` layout at compile time (interleaved: folded offsets)
   auto load_gates = [&](uint32_t dst, const float* row, uint64_t* bar) {
     if (!blk) {
       sm100::bulk_load(dst, row + (long)u0 * 4, wbytes, bar);
@@ -453,17 +453,20 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
         }
       }
       const int j = u0 + ul;
-      *reinterpret_cast<float2*>(a.c_new + b * a.Hp + j) = make_float2(cv[0], cv[1]);
-      store_pair<T>(reinterpret_cast<T*>(a.h_op) + b * a.ldh + j, vh, hv[0], hv[1], true);
+      const int bi = (int)b;   // one step's rows: B·max(Hp, ldh, ldy) < 2^31 (checked by the launcher)
+      *reinterpret_cast<float2*>(a.c_new + (bi * a.Hp + j)) = make_float2(cv[0], cv[1]);
+      store_pair<T>(reinterpret_cast<T*>(a.h_op) + (bi * (int)a.ldh + j), vh, hv[0], hv[1], true);
       if (a.y) {
         const bool ok0 = j < a.H || a.ldy >= a.Hp, ok1 = j + 1 < a.H || a.ldy >= a.Hp;
-        if (ok0) store_pair<TY>(reinterpret_cast<TY*>(a.y) + b * a.ldy + j, vy && ok1, hv[0], hv[1], ok1);
+        if (ok0) store_pair<TY>(reinterpret_cast<TY*>(a.y) + (bi * (int)a.ldy + j), vy && ok1, hv[0], hv[1], ok1);
       }
+      if (a.hT || a.cT) {   // the last step only
 #pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        if (j + u >= a.H) break;
-        if (a.hT) a.hT[b * a.H + j + u] = hv[u];
-        if (a.cT) a.cT[b * a.H + j + u] = cv[u];
+        for (int u = 0; u < 2; ++u) {
+          if (j + u >= a.H) break;
+          if (a.hT) a.hT[(long)b * a.H + j + u] = hv[u];
+          if (a.cT) a.cT[(long)b * a.H + j + u] = cv[u];
+        }
       }
     }
     __syncthreads();   // stage s fully consumed
@@ -484,6 +487,8 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
   a.B = B; a.H = H; a.Hp = Hp;
   ASTRA_CHECK_ARG(gu == GATE_U || gu == Hp, "lstm_fwd_pointwise: gate layout must be GATE_U or Hp");
   a.gu = gu;
+  ASTRA_CHECK_ARG((long)B * std::max({(long)Hp, ldh, ldy}) < (1L << 31), "lstm_fwd_pointwise: one step's rows must have < 2^31 elements");
+  const bool blk = gu != GATE_U;
   a.nub = cdiv(Hp, FB_UB);
   static const int cap = [] {   // A/B knob: CTAs of one launch (row_streams experiments)
     const char* e = std::getenv("ASTRA_FWDPW_CTAS");
@@ -497,14 +502,14 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
   const size_t smem = (size_t)FB_STAGES * FB_STAGE + (size_t)np * 4 * FB_UB * 4 + FB_STAGES * 8;
   const dim3 grid(a.nub * a.rstep);
   if (y_ot == OT::BF16) {
-    auto k = lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16>;
-    static bool attr = false;
-    if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
+    auto k = blk ? lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16, true> : lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16, false>;
+    static bool attr[2] = {false, false};
+    if (!attr[blk]) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr[blk] = true; }
     launch_pdl(k, grid, dim3(FB_THREADS), smem, st, 1, a);
   } else {
-    auto k = lstm_fwd_pw_kernel<KIND, T, float>;
-    static bool attr = false;
-    if (!attr) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr = true; }
+    auto k = blk ? lstm_fwd_pw_kernel<KIND, T, float, true> : lstm_fwd_pw_kernel<KIND, T, float, false>;
+    static bool attr[2] = {false, false};
+    if (!attr[blk]) { CUDA_TRY(cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)); attr[blk] = true; }
     launch_pdl(k, grid, dim3(FB_THREADS), smem, st, 1, a);
   }
   LAUNCH_CHECK();
