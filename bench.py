@@ -170,6 +170,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="astra", choices=["astra", "reference"])
     ap.add_argument("--no-tune", action="store_true")
+    ap.add_argument("--tune-warmup", type=int, default=0,
+                    help="untimed steps before the exploration starts (settles the power-capped SM clock)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile", action="store_true", help="1 warm-up + --steps steps, nothing else (for ncu)")
     ap.add_argument("--batch", type=int, default=None, help="override the global batch (strong) / per-rank batch (weak)")
@@ -260,6 +262,8 @@ def main():
         cell.tune_mode(A.TUNE_FROZEN, os.environ["ASTRA_VARIANT"])
         tune_info = {"mode": "frozen (ASTRA_VARIANT)", "variant": os.environ["ASTRA_VARIANT"]}
     if not args.no_tune:
+        for _ in range(args.tune_warmup):   # real training steps at the default variant
+            lm.train_step(tokens, lr)
         cell.tune_mode(A.TUNE_ON)
         while True:
             lm.train_step(tokens, lr)
