@@ -362,12 +362,12 @@ def test_tune_next_never_blocks():
 
 
 @pytest.mark.parametrize("cell", ["milstm", "lstm", "sublstm"])
-@pytest.mark.parametrize("T,B,H", [(4, 300, 192), (3, 512, 2048), (5, 40, 130)])
+@pytest.mark.parametrize("T,B,H", [(4, 300, 192), (3, 512, 2048), (5, 40, 130), (4, 64, 1024)])
 def test_bwd_pointwise_tiled_lm_bitwise(cell, T, B, H, monkeypatch):
     """The TMA-tiled backward pointwise form (bwd_pw = 2: operand tiles landed in shared memory, the
     older ones before the grid dependency) gives the row-lane and wide forms' bits over 3 LM SGD
     steps (graph replay) — ragged row chunks (B = 300, 40), padding units (H = 130), the R25 4-way
-    split at cfg5's H = 2048, the gate-blocked layout too.  ASTRA_BPW2_STRICT makes a fallback to the
+    split at cfg5's H = 2048 and the 2-way split at H = 1024, the gate-blocked layout too.  ASTRA_BPW2_STRICT makes a fallback to the
     wide form an error, so the tiled kernel really ran at every step but the first."""
     import paper_conf_asplos_sivathanucsz19_b200 as A
     monkeypatch.setenv("ASTRA_BPW2_STRICT", "1")
