@@ -172,6 +172,8 @@ astra_status astra_tune_mode(astra_cell c, int mode, const char* forced) {
       cc.var = Variant::parse(forced);
     }
     cc.tune_mode = mode;
+    cc.racing = false;
+    cc.race_pending.clear();
   });
 }
 

@@ -156,6 +156,25 @@ class Cell {
   void use_slot(int s);
   tuner::Metrics read_metrics(int slot);
   void harvest(int wait);
+  // Final race (reading R41): once the wirer converges, the close alternatives of the chain-form
+  // AVs (fuse_fwd, fuse_bwd, bwd_pw, row_streams: options within 10 % of the chosen one in the
+  // profile index) are re-measured against the converged configuration in interleaved rounds
+  // (5 rounds of 1 warm-up + 1 measured step each) on t_step, and the fastest is kept.  The exploration
+  // measured them minutes apart while the power-capped SM clock drifted; interleaving
+  // removes the drift from the comparison.  One rank, no buckets; ASTRA_TUNE_RACE=0 disables it.
+  bool racing = false;
+  std::vector<tuner::Config> race_cfg;
+  std::vector<double> race_best;
+  std::vector<int> race_seq;
+  size_t race_pos = 0;
+  int race_sub = 0;
+  struct RacePend { int slot, cand; };
+  std::vector<RacePend> race_pending;
+  int race_winner = -1;
+  bool race_start();
+  int race_step();
+  void race_harvest(bool wait_all);
+  void race_advance();
   bool profiling = true;
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
   // prepared GEMMs keyed by (gemm id, T, bn, cm, cn, cg, A, B, M, N, K): the tensor maps carry the

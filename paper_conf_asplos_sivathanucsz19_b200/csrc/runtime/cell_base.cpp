@@ -582,6 +582,7 @@ int Cell::tune_next() {
   ASTRA_CHECK_STATE(world <= 1 || nccl_comm,
                     "tune_next: exploring with world > 1 needs astra_comm_init (cross-rank decisions, reading R29)");
   if (!wirer) tuner_setup();
+  if (racing) return race_step();
   if (wirer->converged()) return ASTRA_TUNE_CONVERGED;
   auto advance = [&] {   // the next step records into a slot no pending measurement uses
     int s = (ev_slot + 1) % EV_SLOTS;
@@ -632,6 +633,109 @@ int Cell::tune_next() {
   }
   apply_config(wirer->final_config());
   configs_seen.pop_back();
+  if (race_start()) return ASTRA_TUNE_EXPLORING;
+  return ASTRA_TUNE_CONVERGED;
+}
+
+bool Cell::race_start() {
+  race_winner = -1;
+  const char* e = std::getenv("ASTRA_TUNE_RACE");
+  if ((e && e[0] == '0') || world > 1 || !tune_ctx.empty() || !tree || !wirer) return false;
+  const tuner::Config fin = wirer->final_config();
+  int ctx = 0;   // the allocation context of the converged configuration: the fork leaf's option
+  for (const char* f : {"alloc", "recomp"}) {
+    const int i = tree->av_index(f);
+    if (i >= 0) { ctx = fin[i]; break; }
+  }
+  const char* me = std::getenv("ASTRA_TUNE_RACE_MARGIN");   // tests: widen the 10 % window
+  const double margin = me ? std::atof(me) : 0.10;
+  const auto& d = wirer->index().d;
+  race_cfg.assign(1, fin);
+  for (const char* a : {"fuse_fwd", "fuse_bwd", "bwd_pw", "row_streams"}) {
+    const int i = tree->av_index(a);
+    if (i < 0) continue;
+    auto key = [&](int k) { return tuner::ProfileIndex::key(ctx, a, std::to_string(k), wirer->index().bucket); };
+    const auto it = d.find(key(fin[i]));
+    if (it == d.end()) continue;
+    for (int k = 0; k < tree->av_n[i] && race_cfg.size() < 5; ++k) {
+      if (k == fin[i]) continue;
+      const auto jt = d.find(key(k));
+      if (jt == d.end() || jt->second > it->second * (1.0 + margin)) continue;
+      tuner::Config c = fin;
+      c[i] = k;
+      race_cfg.push_back(c);
+    }
+  }
+  if (race_cfg.size() < 2) return false;
+  constexpr int ROUNDS = 5;
+  race_seq.clear();
+  for (int r = 0; r < ROUNDS; ++r)
+    for (int c = 0; c < (int)race_cfg.size(); ++c) race_seq.push_back(c);
+  race_best.assign(race_cfg.size(), 1e30);
+  race_pending.clear();
+  race_pos = 0;
+  race_sub = 0;
+  racing = true;
+  apply_config(race_cfg[race_seq[0]]);   // the next step: warm-up of the first candidate
+  return true;
+}
+
+void Cell::race_harvest(bool wait_all) {
+  size_t k = 0;
+  for (; k < race_pending.size(); ++k) {
+    cudaEvent_t end = evr[race_pending[k].slot][R_STEP][1];
+    if (wait_all) {
+      if (cudaEventQuery(end) == cudaErrorNotReady) ++tune_blocks;
+      CUDA_TRY(cudaEventSynchronize(end));
+    } else {
+      const cudaError_t q = cudaEventQuery(end);
+      if (q == cudaErrorNotReady) break;
+      if (q != cudaSuccess) CUDA_TRY(q);
+    }
+    const int s = race_pending[k].slot;
+    const double v = elapsed(evr[s][R_STEP][0], evr[s][R_STEP][1]);
+    double& b = race_best[race_pending[k].cand];
+    b = std::min(b, v);
+  }
+  race_pending.erase(race_pending.begin(), race_pending.begin() + k);
+}
+
+void Cell::race_advance() {   // the next step records into a slot no pending race measurement uses
+  for (int tries = 0; tries < 2; ++tries) {
+    int s = (ev_slot + 1) % EV_SLOTS;
+    for (int n = 0; n < EV_SLOTS; ++n, s = (s + 1) % EV_SLOTS) {
+      bool busy = false;
+      for (const RacePend& p : race_pending) busy |= p.slot == s;
+      if (!busy) { use_slot(s); return; }
+    }
+    race_harvest(true);   // ring full: wait for the older measurements
+  }
+  use_slot((ev_slot + 1) % EV_SLOTS);
+}
+
+int Cell::race_step() {
+  if (race_sub == 0) {   // the warm-up step of race_seq[race_pos] ran: the next one is measured
+    race_sub = 1;
+    race_advance();
+    return ASTRA_TUNE_EXPLORING;
+  }
+  race_pending.push_back({ev_slot, race_seq[race_pos]});
+  ++race_pos;
+  race_sub = 0;
+  race_harvest(false);
+  if (race_pos < race_seq.size()) {
+    apply_config(race_cfg[race_seq[race_pos]]);
+    race_advance();
+    return ASTRA_TUNE_EXPLORING;
+  }
+  race_harvest(true);
+  int best = 0;   // an alternative replaces the converged configuration only if faster by > TOL
+  for (int c = 1; c < (int)race_cfg.size(); ++c)
+    if (race_best[c] < race_best[best] * (1.0 - tuner::TOL)) best = c;
+  race_winner = best;
+  apply_config(race_cfg[best]);
+  racing = false;
+  race_advance();
   return ASTRA_TUNE_CONVERGED;
 }
 
@@ -653,7 +757,25 @@ std::string Cell::report() {
       << ", \"index_entries\": "
       << wirer->index().d.size() << ", \"tree_avs\": [";
     for (size_t i = 0; i < tree->avs.size(); ++i) o << (i ? ", " : "") << "\"" << tree->avs[i] << "\"";
-    o << "], \"index\": {";
+    o << "]";
+    if (!race_cfg.empty() && race_cfg.size() == race_best.size()) {   // the final race (R41)
+      o << ", \"race\": {\"winner\": " << race_winner << ", \"candidates\": [";
+      for (size_t c = 0; c < race_cfg.size(); ++c) {
+        Variant v = var;
+        for (size_t i = 0; i < tree->avs.size() && i < race_cfg[c].size(); ++i) {
+          const std::string& n = tree->avs[i];
+          const int x = race_cfg[c][i];
+          if (n == "fuse_fwd") v.fwd_mode = x;
+          else if (n == "fuse_bwd") v.bwd_mode = x;
+          else if (n == "bwd_pw") v.bpw = x;
+          else if (n == "row_streams") v.rsp = x;
+        }
+        o << (c ? ", " : "") << "{\"fwd\": " << v.fwd_mode << ", \"bwd\": " << v.bwd_mode << ", \"bpw\": " << v.bpw
+          << ", \"rsp\": " << v.rsp << ", \"t_step_min\": " << race_best[c] << "}";
+      }
+      o << "]}";
+    }
+    o << ", \"index\": {";
     size_t k = 0;
     for (auto& kv : wirer->index().d) o << (k++ ? ", " : "") << "\"" << kv.first << "\": " << kv.second;
     o << "}";

@@ -244,7 +244,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   bool exploring = false;
   std::string vs;
   for (Cell* L : layers) {
-    exploring |= L->tune_mode == ASTRA_TUNE_ON && !(L->wirer && L->wirer->converged());
+    exploring |= L->tune_mode == ASTRA_TUNE_ON && (!(L->wirer && L->wirer->converged()) || L->racing);
     // a captured step records into the region-event slot current at capture time
     vs += L->var.str() + (L->profiling ? ";p" + std::to_string(L->ev_slot) + ";" : ";");
   }

@@ -334,6 +334,44 @@ def test_rhn_wg_side_lm_bitwise():
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
 
 
+def test_tuner_final_race(monkeypatch):
+    """Reading R41: after the wirer converges, the chain-form AVs' alternatives (here every one: the
+    margin widened to 1000 %) are re-measured interleaved with the converged configuration, 5
+    rounds of warm-up + measured step each; the report names the candidates, their min step times
+    and the winner, the run converges, and the parameters equal an untuned run's after as many SGD
+    steps (every variant is value-preserving)."""
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    monkeypatch.setenv("ASTRA_TUNE_RACE_MARGIN", "10")
+    T, B, I, H, V = 4, 64, 64, 64, 40
+
+    def lm():
+        p, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, synth.config_seed(5) + 61, True)
+        c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+        m = A.LM(c, V)
+        m.load(p)
+        return c, m, torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+
+    c, m, tokens = lm()
+    c.tune_mode(A.TUNE_ON)
+    n, state = 0, A.TUNE_EXPLORING
+    while state != A.TUNE_CONVERGED and n < 1500:
+        m.train_step(tokens, 0.05)
+        n += 1
+        state = c.tune_next()
+    m.train_step(tokens, 0.05)
+    torch.cuda.synchronize()
+    rep = c.tune_report()
+    assert state == A.TUNE_CONVERGED and "race" in rep, rep.keys()
+    race = rep["race"]
+    assert len(race["candidates"]) >= 2 and 0 <= race["winner"] < len(race["candidates"]), race
+    assert all(0 < x["t_step_min"] < 1e29 for x in race["candidates"]), race
+    c2, m2, tokens2 = lm()
+    for _ in range(n + 1):
+        m2.train_step(tokens2, 0.05)
+    torch.cuda.synchronize()
+    assert torch.equal(m.params, m2.params)
+
+
 def test_tune_next_never_blocks():
     """astra_tune_next harvests the measured steps' events with cudaEventQuery (include/astra.h):
     right after it returns, the step just enqueued is still running on the GPU — the host keeps
