@@ -157,8 +157,9 @@ class Cell {
   tuner::Metrics read_metrics(int slot);
   void harvest(int wait);
   // Final race (reading R41): once the wirer converges, the close alternatives of the chain-form
-  // AVs (fuse_fwd, fuse_bwd, bwd_pw, row_streams: options within 10 % of the chosen one in the
-  // profile index) are re-measured against the converged configuration in interleaved rounds
+  // AVs and of the per-step chain GEMMs' kernel choices (fuse_fwd, fuse_bwd, bwd_pw, row_streams,
+  // g_rec, g_bptt: options within 10 % of the chosen one in the profile index, the 5 closest) are
+  // re-measured against the converged configuration in interleaved rounds
   // (5 rounds of 1 warm-up + 1 measured step each) on t_step, and the fastest is kept.  The exploration
   // measured them minutes apart while the power-capped SM clock drifted; interleaving
   // removes the drift from the comparison.  One rank, no buckets; ASTRA_TUNE_RACE=0 disables it.

@@ -651,21 +651,28 @@ bool Cell::race_start() {
   const double margin = me ? std::atof(me) : 0.10;
   const auto& d = wirer->index().d;
   race_cfg.assign(1, fin);
-  for (const char* a : {"fuse_fwd", "fuse_bwd", "bwd_pw", "row_streams"}) {
+  // the alternatives (at most 5): the chain-form AVs' options, then the per-step chain GEMMs' kernel
+  // choices, closest first within each group, each within `margin` of the chosen one in the index
+  std::vector<std::pair<double, tuner::Config>> alts;
+  for (const char* a : {"fuse_fwd", "fuse_bwd", "bwd_pw", "row_streams", "g_rec", "g_bptt"}) {
     const int i = tree->av_index(a);
     if (i < 0) continue;
     auto key = [&](int k) { return tuner::ProfileIndex::key(ctx, a, std::to_string(k), wirer->index().bucket); };
     const auto it = d.find(key(fin[i]));
-    if (it == d.end()) continue;
-    for (int k = 0; k < tree->av_n[i] && race_cfg.size() < 5; ++k) {
+    if (it == d.end() || !(it->second > 0)) continue;
+    for (int k = 0; k < tree->av_n[i]; ++k) {
       if (k == fin[i]) continue;
       const auto jt = d.find(key(k));
       if (jt == d.end() || jt->second > it->second * (1.0 + margin)) continue;
       tuner::Config c = fin;
       c[i] = k;
-      race_cfg.push_back(c);
+      // the chain-form AVs first (their options differ most in clock sensitivity), then the kernels
+      const bool form = a[0] != 'g';
+      alts.push_back({jt->second / it->second + (form ? 0.0 : 10.0), c});
     }
   }
+  std::stable_sort(alts.begin(), alts.end(), [](const auto& x, const auto& y) { return x.first < y.first; });
+  for (size_t k = 0; k < alts.size() && race_cfg.size() < 6; ++k) race_cfg.push_back(alts[k].second);
   if (race_cfg.size() < 2) return false;
   constexpr int ROUNDS = 5;
   race_seq.clear();
@@ -769,9 +776,13 @@ std::string Cell::report() {
           else if (n == "fuse_bwd") v.bwd_mode = x;
           else if (n == "bwd_pw") v.bpw = x;
           else if (n == "row_streams") v.rsp = x;
+          else if (n == "g_rec" && x < (int)allowed[G_REC].size()) v.g[G_REC] = allowed[G_REC][x];
+          else if (n == "g_bptt" && x < (int)allowed[G_BPTT].size()) v.g[G_BPTT] = allowed[G_BPTT][x];
         }
         o << (c ? ", " : "") << "{\"fwd\": " << v.fwd_mode << ", \"bwd\": " << v.bwd_mode << ", \"bpw\": " << v.bpw
-          << ", \"rsp\": " << v.rsp << ", \"t_step_min\": " << race_best[c] << "}";
+          << ", \"rsp\": " << v.rsp << ", \"rec\": \"" << v.g[G_REC].bn << "." << v.g[G_REC].cm << "." << v.g[G_REC].cn
+          << "." << v.g[G_REC].cg << "\", \"bptt\": \"" << v.g[G_BPTT].bn << "." << v.g[G_BPTT].cm << "." << v.g[G_BPTT].cn
+          << "." << v.g[G_BPTT].cg << "\", \"t_step_min\": " << race_best[c] << "}";
       }
       o << "]}";
     }
