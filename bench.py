@@ -248,6 +248,7 @@ def main():
     if args.profile:
         if os.environ.get("ASTRA_VARIANT"):
             cell.tune_mode(A.TUNE_FROZEN, os.environ["ASTRA_VARIANT"])
+        cell.set_profiling(2)   # the phase regions too (diagnostics)
         lm.train_step(tokens, lr)
         torch.cuda.synchronize()
         for _ in range(args.steps):
@@ -393,6 +394,7 @@ def cell_region_ms(cell, lm, tokens, lr, steps=3):
     """Per-region device times from the library's own cudaEvent pairs, min over steps."""
     import torch
     out = {}
+    cell.set_profiling(2)   # phase regions for these diagnostic steps (the timed ones record the step only)
     keys = {"a1_ms": "t_a1", "fwd_chain_ms": "t_fwd", "bptt_chain_ms": "t_bptt", "head_ms": "t_head",
             "wgrad_ms": "t_se4", "step_ms": "t_step"}
     for _ in range(steps):
@@ -401,6 +403,7 @@ def cell_region_ms(cell, lm, tokens, lr, steps=3):
         r = region_times(cell)
         for k, v in r.items():
             out[k] = min(out.get(k, 1e30), v)
+    cell.set_profiling(1)   # back to the always-on level
     return out
 
 

@@ -132,9 +132,12 @@ astra_status astra_tune_next(astra_cell c, int* state);
  * (use `forced_variant`, a string from astra_tune_report's "variant" field, or the best
  * found so far when NULL).                                                                  */
 astra_status astra_tune_mode(astra_cell c, int mode, const char* forced_variant);
-/* Region events (cudaEvent pairs around the step phases) on (default) or off.  The
- * tuner harvests them, so on = 0 is refused with E_STATE while the mode is ASTRA_TUNE_ON; off is
- * for measuring the profiling overhead (< 0.5 %).                                   */
+/* Region events (cudaEvent pairs around the step phases).  on = 1 (default): the
+ * always-on level — the step region every step, the phase regions (a1, chains, head, SE4,
+ * dU / dW / dX) only while the tuner explores or races; on = 2: the phase regions every step
+ * (diagnostics: astra_region_times); on = 0: none.  The tuner harvests them, so on = 0 is refused
+ * with E_STATE while the mode is ASTRA_TUNE_ON; off is for measuring the profiling overhead
+ * (< 0.5 %).  Other values: E_ARG.                                                   */
 astra_status astra_set_profiling(astra_cell c, int on);
 /* JSON report (current variant, #configs explored, index size, trials).  Writes at most
  * len bytes including the NUL; *needed ← required length.                                  */

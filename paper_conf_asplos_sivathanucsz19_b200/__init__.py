@@ -208,9 +208,11 @@ class Cell:
         arr = (ctypes.c_void_p * max(1, n_side))(*[s.cuda_stream for s in self._side])
         _check(lib().astra_set_streams(self.h, _stream(), arr, n_side, None))
 
-    def set_profiling(self, on: bool):
-        """Region cudaEvent pairs on/off (astra_set_profiling; off only outside exploration)."""
-        _check(lib().astra_set_profiling(self.h, int(bool(on))))
+    def set_profiling(self, on):
+        """Region cudaEvent pairs (astra_set_profiling): False / 0 off (only outside exploration),
+        True / 1 the always-on level (step region; phase regions while exploring), 2 every phase
+        region every step (diagnostics)."""
+        _check(lib().astra_set_profiling(self.h, int(on)))
 
     def view(self, name, t=None):
         """View of parameter `name` inside the flat params (or grads) vector, external layout."""

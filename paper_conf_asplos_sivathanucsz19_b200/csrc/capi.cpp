@@ -182,7 +182,9 @@ astra_status astra_set_profiling(astra_cell c, int on) {
     NEED(c);
     Cell& cc = *c->c;
     ASTRA_CHECK_STATE(on || cc.tune_mode != ASTRA_TUNE_ON, "set_profiling: exploration needs the region events");
+    ASTRA_CHECK_ARG(on >= 0 && on <= 2, "set_profiling: on must be 0, 1 or 2");
     cc.profiling = on != 0;
+    cc.full_regions = on == 2;
   });
 }
 

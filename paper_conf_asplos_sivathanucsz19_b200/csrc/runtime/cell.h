@@ -177,6 +177,15 @@ class Cell {
   void race_harvest(bool wait_all);
   void race_advance();
   bool profiling = true;
+  // Profiling levels: the step region is always recorded; the phase regions
+  // (a1, chains, head, SE4, dU / dW / dX) only while the tuner needs them — exploring or racing —
+  // or when asked for (astra_set_profiling(c, 2): diagnostics such as bench.py's region table).  A
+  // frozen step then carries 2 event records instead of 18, each of which would otherwise sit
+  // between two chain kernels in the step graph and cost their programmatic overlap.
+  bool full_regions = false;
+  bool regions_needed() const {
+    return full_regions || (tune_mode == ASTRA_TUNE_ON && (!wirer || !wirer->converged() || racing));
+  }
   std::vector<KCfg> allowed[G_ROLES];  // statically pruned options per role (A19), default first
   // prepared GEMMs keyed by (gemm id, T, bn, cm, cn, cg, A, B, M, N, K): the tensor maps carry the
   // operand pointers and extents, so two row ranges of one role never share an entry

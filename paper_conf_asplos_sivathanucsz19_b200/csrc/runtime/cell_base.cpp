@@ -213,6 +213,10 @@ void Cell::bind(float* pp, float* gg, void* sv_p, void* sc_p) {
 
 void Cell::mark(Region r, int which, cudaStream_t st) {
   if (!profiling) return;
+  if (r != R_STEP && !regions_needed()) return;
+  if (r == R_STEP && which == 0 && !regions_needed())   // this step's phase regions are not recorded
+    for (int q = 0; q < R_COUNT; ++q)
+      if (q != R_STEP) region_used[q] = false;
   // External: inside a CUDA-graph capture this becomes a real event-record node (replays keep
   // timing the regions); outside a capture it is a plain record
   cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;

@@ -246,7 +246,7 @@ void LM::step(const int32_t* tokens, float lr, float* loss_dev, bool do_sgd) {
   for (Cell* L : layers) {
     exploring |= L->tune_mode == ASTRA_TUNE_ON && (!(L->wirer && L->wirer->converged()) || L->racing);
     // a captured step records into the region-event slot current at capture time
-    vs += L->var.str() + (L->profiling ? ";p" + std::to_string(L->ev_slot) + ";" : ";");
+    vs += L->var.str() + (L->profiling ? ";p" + std::to_string(L->ev_slot) + (L->regions_needed() ? "r;" : ";") : ";");
   }
   if (!use_graphs || !graphs_enabled() || exploring || c.ot != OT::BF16 ||
       (c.world > 1 && (!graph_nccl || c.peer))) {

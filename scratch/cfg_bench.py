@@ -35,6 +35,7 @@ def lm_run(name, cell, H, I, B, T, V, kw, steps=10):
     e1.record(); torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / steps
     import bench
+    c.set_profiling(2)   # phase regions for the diagnostic step
     m.set_graph(False)
     m.train_step(tok, 0.01); torch.cuda.synchronize()
     regions = {k: round(v, 3) for k, v in bench.region_times(c).items()}
@@ -85,6 +86,7 @@ def attn_run(name, H, I, A_, B, Ts, Tt, steps=10):
     e1.record(); torch.cuda.synchronize()
     ms = e0.elapsed_time(e1) / steps
     import bench
+    c.set_profiling(2)   # phase regions for the diagnostic step
     step(); torch.cuda.synchronize()
     regions = {k: round(v, 3) for k, v in bench.region_times(c).items()}
     print(json.dumps({"config": name, "samples_per_s": round(B / ms * 1e3, 1), "ms_per_step": round(ms, 3),

@@ -334,6 +334,44 @@ def test_rhn_wg_side_lm_bitwise():
     assert torch.equal(out[0][0], out[1][0]) and out[0][1] == out[1][1]
 
 
+def test_profiling_levels():
+    """The always-on profiling level records the step region every step and the phase
+    regions only while the tuner needs them; level 2 records every phase region (diagnostics);
+    neither changes a value (the step graph is re-captured per level)."""
+    import ctypes
+    import paper_conf_asplos_sivathanucsz19_b200 as A
+    T, B, I, H, V = 5, 64, 64, 64, 50
+
+    def regions(c):
+        buf = (ctypes.c_double * 16)()
+        n = ctypes.c_int()
+        A._check(A.lib().astra_region_times(c.h, buf, 16, ctypes.byref(n)))
+        return [buf[i] for i in range(n.value)]
+
+    out = []
+    for lvl in (1, 2, 0):
+        pa, tok, h0, c0 = _lm_case("milstm", T, B, I, H, V, synth.config_seed(5) + 71, True)
+        c = A.Cell("milstm", H, I, B, T, dtype="bf16")
+        m = A.LM(c, V)
+        m.load(pa)
+        c.tune_mode(A.TUNE_FROZEN, "fwd=0")
+        c.set_profiling(lvl)
+        tokens = torch.as_tensor(tok, dtype=torch.int32, device=c.device)
+        for _ in range(3):
+            m.train_step(tokens, 0.1)
+        torch.cuda.synchronize()
+        out.append(m.params.clone())
+        if lvl:
+            r = regions(c)
+            step = r[8]   # R_STEP
+            phases = [r[0], r[1], r[3]]   # a1, forward chain, BPTT chain
+            assert step > 0, r
+            assert all(x > 0 for x in phases) if lvl == 2 else all(x == 0 for x in phases), (lvl, r)
+    assert torch.equal(out[0], out[1]) and torch.equal(out[0], out[2])
+    with pytest.raises(A.AstraError):
+        c.set_profiling(3)
+
+
 def test_tuner_final_race(monkeypatch):
     """Reading R41: after the wirer converges, the chain-form AVs' alternatives (here every one: the
     margin widened to 1000 %) are re-measured interleaved with the converged configuration, 5
