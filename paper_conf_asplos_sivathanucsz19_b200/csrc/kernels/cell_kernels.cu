@@ -9,6 +9,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <map>
+#include <mutex>
 #include <tuple>
 
 namespace astra {
@@ -1065,9 +1066,11 @@ __global__ void __launch_bounds__(BW2_THREADS, 2)
 
 // fp32 tile maps of the TMA-tiled form, cached by (pointer, shape): the per-step operand pointers
 // repeat every training step, so each map is encoded once
-static const CUtensorMap& bw3_map(const void* ptr, long inner, long rows, long z, long ld, long zstride) {
+static CUtensorMap bw3_map(const void* ptr, long inner, long rows, long z, long ld, long zstride) {
   using Key = std::tuple<const void*, long, long, long, long, long>;
   static std::map<Key, CUtensorMap> cache;
+  static std::mutex mu;   // cells may enqueue from several host threads
+  std::lock_guard<std::mutex> lock(mu);
   const Key k{ptr, inner, rows, z, ld, zstride};
   auto it = cache.find(k);
   if (it != cache.end()) return it->second;
