@@ -127,13 +127,14 @@ void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q
 // Backward of one attention step (oracle/cells.py attn_backward):
 //   dctx = dy_ctx + dctx_rec;  dp_j = dctx·enc_j;  de_j = p_j (dp_j − Σ p dp);  denc_j += p_j dctx;
 //   u_j = tanh(q + k_j);  du_j = de_j v (1 − u_j²);  dq = Σ_j du_j;  dk_j += du_j;  dv_b += Σ_j de_j u_j
-// dctx_h of row b = dy_ctx + dctx_rec (0 past H)
+// dctx_h of row b = dy_ctx + dctx_rec (0 past H); dctx_rec may be the ns split-K partials of the
+// decoder's BPTT GEMM at stride ss (reading R42), summed in chunk order first
 template <typename TDY>
 __device__ __forceinline__ float attn_dctx(const TDY* __restrict__ dy_ctx, long ldy, const float* __restrict__ dctx_rec,
-                                           long ldr, int b, int h, int H) {
+                                           long ldr, int ns, long ss, int b, int h, int H) {
   if (h >= H) return 0.f;
   float d = dy_ctx ? to_f<TDY>(dy_ctx[(long)b * ldy + h]) : 0.f;
-  if (dctx_rec) d = __fadd_rn(d, dctx_rec[(long)b * ldr + h]);
+  if (dctx_rec) d = __fadd_rn(d, sum_split(dctx_rec + (long)b * ldr + h, ns, ss));
   return d;
 }
 
@@ -142,21 +143,24 @@ __device__ __forceinline__ float attn_dctx(const TDY* __restrict__ dy_ctx, long 
 template <typename TDY>
 __global__ void __launch_bounds__(ATT_THREADS)
     attn_dp_kernel(int B, int Ts, int H, int Hp, const TDY* __restrict__ dy_ctx, long ldy,
-                   const float* __restrict__ dctx_rec, long ldr, const float* __restrict__ enc, float* __restrict__ dp) {
+                   const float* __restrict__ dctx_rec, long ldr, int ns, long ss, const float* __restrict__ enc, float* __restrict__ dp) {
+  extern __shared__ float sdctx[];   // [Hp]: row b's dctx, formed once per CTA (its warps share b)
   pdl_wait();
   pdl_trigger();
   const int w = threadIdx.x / 32, l = threadIdx.x % 32;
   const int b = blockIdx.y, j = blockIdx.x * (ATT_THREADS / 32) + w;
+  for (int h = threadIdx.x; h < Hp; h += ATT_THREADS) sdctx[h] = attn_dctx(dy_ctx, ldy, dctx_rec, ldr, ns, ss, b, h, H);
+  __syncthreads();
   if (j >= Ts) return;
   const float4* ej = reinterpret_cast<const float4*>(enc + ((long)j * B + b) * Hp);
   float s = 0.f;
   for (int c = l; 4 * c < H; c += 32) {
     const float4 x = ej[c];
     const int h = 4 * c;
-    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h, H), x.x));
-    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h + 1, H), x.y));
-    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h + 2, H), x.z));
-    s = __fadd_rn(s, __fmul_rn(attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, h + 3, H), x.w));
+    s = __fadd_rn(s, __fmul_rn(sdctx[h], x.x));
+    s = __fadd_rn(s, __fmul_rn(sdctx[h + 1], x.y));
+    s = __fadd_rn(s, __fmul_rn(sdctx[h + 2], x.z));
+    s = __fadd_rn(s, __fmul_rn(sdctx[h + 3], x.w));
   }
 #pragma unroll
   for (int o = 16; o; o >>= 1) s = __fadd_rn(s, __shfl_xor_sync(0xffffffffu, s, o));
@@ -172,7 +176,7 @@ __global__ void __launch_bounds__(ATT_THREADS)
 template <typename T, typename TDY>
 __global__ void __launch_bounds__(ATT_THREADS)
     attn_bwd_kernel(int B, int Ts, int H, int Hp, int A, int Ap, const TDY* __restrict__ dy_ctx, long ldy,
-                    const float* __restrict__ dctx_rec, long ldr, const float* __restrict__ pr,
+                    const float* __restrict__ dctx_rec, long ldr, int ns, long ss, const float* __restrict__ pr,
                     const float* __restrict__ dpv, const float* __restrict__ q, const float* __restrict__ keys,
                     const float* __restrict__ v, T* __restrict__ dq_op, float* __restrict__ dctx_save,
                     float* __restrict__ de_save, float* __restrict__ dvb, int first) {
@@ -196,7 +200,7 @@ __global__ void __launch_bounds__(ATT_THREADS)
   if (blockIdx.x == 0)
     for (int j = threadIdx.x; j < Ts; j += ATT_THREADS) de_save[(long)b * Ts + j] = de[j];
   const int x = blockIdx.x * ATT_THREADS + threadIdx.x;
-  if (x < Hp) dctx_save[(long)b * Hp + x] = attn_dctx(dy_ctx, ldy, dctx_rec, ldr, b, x, H);
+  if (x < Hp) dctx_save[(long)b * Hp + x] = attn_dctx(dy_ctx, ldy, dctx_rec, ldr, ns, ss, b, x, H);
   if (x < Ap) {   // attention-width terms
     constexpr int JG = 10;
     const int a = x;
@@ -325,14 +329,14 @@ void attn_acc(OT ot, int T, int B, int Ts, int Hp, int A, int Ap, const float* p
 
 template <typename T, typename TDY>
 static void attn_bwd_launch(int B, int Ts, int H, int Hp, int A, int Ap, const TDY* dy_ctx, long ldy,
-                            const float* dctx_rec, long ldr, const float* pr, float* dp, const float* q,
+                            const float* dctx_rec, long ldr, int ns, long ss, const float* pr, float* dp, const float* q,
                             const float* keys, const float* v, const float* enc, T* dq_op, float* dctx_save,
                             float* de_save, float* dvb, bool first, cudaStream_t st) {
-  launch_pdl(attn_dp_kernel<TDY>, dim3(cdiv(Ts, ATT_THREADS / 32), B), dim3(ATT_THREADS), 0, st, 1, B, Ts, H, Hp,
-             dy_ctx, ldy, dctx_rec, ldr, enc, dp);
+  launch_pdl(attn_dp_kernel<TDY>, dim3(cdiv(Ts, ATT_THREADS / 32), B), dim3(ATT_THREADS), (size_t)Hp * sizeof(float), st, 1, B, Ts, H, Hp,
+             dy_ctx, ldy, dctx_rec, ldr, ns, ss, enc, dp);
   LAUNCH_CHECK();
   launch_pdl(attn_bwd_kernel<T, TDY>, dim3(cdiv(std::max(Hp, Ap), ATT_THREADS), B), dim3(ATT_THREADS),
-             (Ts + 8) * sizeof(float), st, 1, B, Ts, H, Hp, A, Ap, dy_ctx, ldy, dctx_rec, ldr, pr, (const float*)dp, q,
+             (Ts + 8) * sizeof(float), st, 1, B, Ts, H, Hp, A, Ap, dy_ctx, ldy, dctx_rec, ldr, ns, ss, pr, (const float*)dp, q,
              keys, v, dq_op, dctx_save, de_save, dvb, (int)first);
   LAUNCH_CHECK();
 }
@@ -340,19 +344,21 @@ static void attn_bwd_launch(int B, int Ts, int H, int Hp, int A, int Ap, const T
 void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
               const float* dctx_rec, long ldr, const float* pr, float* dpscratch, const float* q, const float* keys,
               const float* v, const float* enc, void* dq_op, float* dctx_save, float* de_save, float* dvb, bool first,
-              cudaStream_t st) {
+              cudaStream_t st, int ns, long ss) {
+  ASTRA_CHECK_ARG(ns >= 1, "attn_bwd: ns must be >= 1");
+  ASTRA_CHECK_ARG((size_t)Hp * sizeof(float) <= 48 * 1024, "attn_bwd: Hp too large for the staged dctx row");
   ASTRA_CHECK_ARG(Hp % 4 == 0 && ((uintptr_t)enc & 15) == 0, "attn_bwd: enc rows must be 16-byte aligned");
   if (ot == OT::BF16) {
     if (dy_f32 || !dy_ctx)
-      attn_bwd_launch<__nv_bfloat16, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, pr,
+      attn_bwd_launch<__nv_bfloat16, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, ns, ss, pr,
                                             dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op, dctx_save, de_save, dvb,
                                             first, st);
     else
       attn_bwd_launch<__nv_bfloat16, __nv_bfloat16>(B, Ts, H, Hp, A, Ap, (const __nv_bfloat16*)dy_ctx, ldy, dctx_rec,
-                                                    ldr, pr, dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op,
+                                                    ldr, ns, ss, pr, dpscratch, q, keys, v, enc, (__nv_bfloat16*)dq_op,
                                                     dctx_save, de_save, dvb, first, st);
   } else {
-    attn_bwd_launch<float, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, pr, dpscratch, q,
+    attn_bwd_launch<float, float>(B, Ts, H, Hp, A, Ap, (const float*)dy_ctx, ldy, dctx_rec, ldr, ns, ss, pr, dpscratch, q,
                                   keys, v, enc, (float*)dq_op, dctx_save, de_save, dvb, first, st);
   }
 }

@@ -90,7 +90,7 @@ void attn_fwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const float* q
 void attn_bwd(OT ot, int B, int Ts, int H, int Hp, int A, int Ap, const void* dy_ctx, long ldy, bool dy_f32,
               const float* dctx_rec, long ldr, const float* pr, float* dpscratch, const float* q, const float* keys,
               const float* v, const float* enc, void* dq_op, float* dctx_save, float* de_save, float* dvb, bool first,
-              cudaStream_t st);
+              cudaStream_t st, int ns = 1, long ss = 0);   // dctx_rec: ns split-K partials at stride ss
 // denc / dk ([Ts][B][Hp] / [Ts][B][Ap], overwritten) from the T steps' saved p, de, dctx and q
 void attn_acc(OT ot, int T, int B, int Ts, int Hp, int A, int Ap, const float* pr, const float* de_save,
               const float* dctx_save, const float* q, const float* keys, const float* v, float* denc, float* dk,

@@ -29,6 +29,13 @@ class AttnCell : public Cell {
   size_t off_DA, off_dHC, off_dC, off_DQ, off_denc, off_DKf, off_DK, off_dvb, off_part, off_dh0e, off_dc0e,
       off_colsum, off_att, off_dctxs, off_des;
 
+  // Reading R42: the decoder's per-step BPTT GEMM [dh | dctx]_rec = da·[U_d; C_d]ᵀ (M = B, K = 4Hp)
+  // gets a fixed split-K like R25 — K chunks accumulated from zero, summed in chunk order by the
+  // attention backward (ctx part) and the pointwise kernel (h part; the dq·W_qᵀ GEMM split the same
+  // way, chunk k accumulated into partial k) — at cfg4 (K = 4096) 4 chunks of 16 k-blocks on 4× the
+  // CTAs (bf16 path; the same for every variant)
+  int bptt_ksplit() const { return ot != OT::BF16 ? 1 : NG >= 4096 ? 4 : NG >= 2048 ? 2 : 1; }
+
   explicit AttnCell(const astra_cell_desc& dd) : Cell(dd) {
     Ts = d.src_seq;
     A = d.attn_dim;
@@ -76,7 +83,7 @@ class AttnCell : public Cell {
     Carve c;
     off_encscratch = c.take(enc->scratch_bytes);
     off_DA = c.take(TB * NG * e);
-    off_dHC = c.take((size_t)B * 2 * Hp * 4);
+    off_dHC = c.take((size_t)bptt_ksplit() * B * 2 * Hp * 4);   // the split-K partials of [dh | dctx]_rec
     off_dC = c.take((size_t)B * Hp * 4);
     off_DQ = c.take(TB * Ap * e);
     off_denc = c.take(SB * Hp * 4);
@@ -294,18 +301,35 @@ class AttnCell : public Cell {
     bp.b_mn = true;
     bp.M = B; bp.N = (int)ld2; bp.K = NG;
     bp.b_keep = true;
+    GemmSpec bp0 = bp;                 // the decoder's initial-state gradient (once, no split)
+    const int nsp = bptt_ksplit();
+    bp.ksplit = nsp;
+    const long sstr = (long)B * ld2;   // partial k of [dh | dctx]_rec at dHC + k·sstr
+    EpiStore ebp = epi(dHC, ld2, B, (int)ld2);
+    ebp.split_stride = sstr;
     GemmSpec dqw;                      // dh += dq·W_qᵀ
     dqw.A = mat(DQ, Ap, B, Ap, T, (long)B * Ap);
     dqw.B = mat(MWq, Hp, Ap, Hp);
     dqw.b_mn = true;
     dqw.M = B; dqw.N = Hp; dqw.K = Ap;
+    // R42: split like bp — K chunk k of dq·W_qᵀ accumulates into partial k of dh_rec, so partial k =
+    // bp_k + dqw_k and the pointwise kernel sums them in chunk order (the last step, which has no
+    // bp partials yet, runs it unsplit onto dhT)
+    GemmSpec dqw0 = dqw;
+    dqw.ksplit = nsp;
+    EpiStore edq = accum(epi(dHC, ld2, B, Hp));
+    edq.split_stride = sstr;
     for (int i = T - 1; i >= 0; --i) {
-      if (i < T - 1) run_gemm(4, bp, epi(dHC, ld2, B, (int)ld2), i + 1, 0, var.g[G_BPTT], st);
+      // the last step starts from dhT (one "partial": no GEMM yet), the others from the split GEMM
+      const int ns_i = i < T - 1 ? nsp : 1;
+      if (i < T - 1) run_gemm(4, bp, ebp, i + 1, 0, var.g[G_BPTT], st);
       attn_bwd(ot, B, Ts, H, Hp, A, Ap, (const char*)dy + ((size_t)i * B * ldy + H) * e, ldy, false, dHC + Hp, ld2,
                Pr + (long)i * B * Ts, sc<float>(off_att), Q + (long)i * B * Ap, Keys, p("v"), Encf, DQ + (size_t)i * B * Ap * e,
-               sc<float>(off_dctxs) + (long)i * B * Hp, sc<float>(off_des) + (long)i * B * Ts, dvb, i == T - 1, st);
-      run_gemm(5, dqw, accum(epi(dHC, ld2, B, Hp)), i, 0, var.g[G_BPTT], st);
-      lstm_bwd_pointwise(K_LSTM, ot, B, H, Hp, (const char*)dy + (size_t)i * B * ldy * e, ldy, ot, false, dHC, ld2, 1, 0,
+               sc<float>(off_dctxs) + (long)i * B * Hp, sc<float>(off_des) + (long)i * B * Ts, dvb, i == T - 1, st, ns_i,
+               sstr);
+      if (i < T - 1) run_gemm(5, dqw, edq, i, 0, var.g[G_BPTT], st);
+      else run_gemm(14, dqw0, accum(epi(dHC, ld2, B, Hp)), i, 0, var.g[G_BPTT], st);
+      lstm_bwd_pointwise(K_LSTM, ot, B, H, Hp, (const char*)dy + (size_t)i * B * ldy * e, ldy, ot, false, dHC, ld2, ns_i, sstr,
                          dC, WXd + (long)i * B * NG, UHd + (long)i * B * NG, Cd + (long)(i + 1) * B * Hp,
                          Cd + (long)i * B * Hp, gp, DA + (size_t)i * B * NG * e, DA + (size_t)i * B * NG * e, part, 1,
                          i == T - 1, st);
@@ -313,7 +337,7 @@ class AttnCell : public Cell {
     // encoder-side attention accumulators over the T steps (same per-element order as per-step updates)
     attn_acc(ot, T, B, Ts, Hp, A, Ap, Pr, sc<float>(off_des), sc<float>(off_dctxs), Q, Keys, p("v"), denc, DKf, st);
     // decoder initial-state gradient → encoder final-state gradient
-    run_gemm(4, bp, epi(dHC, ld2, B, (int)ld2), 0, 0, var.g[G_BPTT], st);
+    run_gemm(13, bp0, epi(dHC, ld2, B, (int)ld2), 0, 0, var.g[G_BPTT], st);
     copy_pad(OT::F32, dHC, OT::F32, B, H, ld2, dh0e, H, st);
     copy_pad(OT::F32, dC, OT::F32, B, H, Hp, dc0e, H, st);
     mark(R_BPTT, 1, st);
