@@ -84,7 +84,7 @@ class LstmCell : public Cell {
   // Fixed split-K of the per-step BPTT GEMM (K = 4·Hp): with B rows the GEMM has few output tiles,
   // so each SM would stream a whole K-panel of Uᵀ; four K-chunks cut the bytes per SM 4× while the
   // chunk partials are summed in a fixed order by the pointwise kernel (identical for every variant).
-  int bptt_ksplit() const { return (ot == OT::BF16 && NG >= 8192) ? 4 : (ot == OT::BF16 && NG >= 4096) ? 2 : 1; }
+  int bptt_ksplit() const { return (ot == OT::BF16 && NG >= 4096) ? 4 : (ot == OT::BF16 && NG >= 2048) ? 2 : 1; }
 
   // K2 fusion choices (AV fuse_fwd): 0 GEMM + pointwise, 1 fused per step (CTA pairs), 2 fused
   // persistent (256-column tiles), 3 small-batch persistent with the U slice resident (B ≤ 128)
