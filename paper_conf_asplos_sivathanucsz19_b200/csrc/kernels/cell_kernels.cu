@@ -559,6 +559,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   constexpr int NP = KIND == K_MILSTM ? 4 : 1;   // gate parameter sets: b (and α, β1, β2)
   __shared__ float red[BWD_RY][NV][BWD_UX];
   __shared__ float sgp[NP][4][BWD_UX];   // staged once; re-read per row so they hold no registers
+  __shared__ float spre[NV][BWD_UX];     // the chunk's old column-sum partials (prefetched)
   const int tx = threadIdx.x, ty = threadIdx.y;
   const int j = blockIdx.x * BWD_UX + tx;
   if (ty < NP) {   // parameters are not written by the chain: staged before the grid dependency
@@ -573,6 +574,11 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   // address offsets), the gate-blocked one Hp
   const int gs = BLK ? gu : GATE_U;
   const int c0 = BLK ? j : gcol(0, j);   // gate g of unit j at column c0 + g·gs
+  // the previous step's partials of this chunk (written two launches back: complete) — loaded now,
+  // so the final fold does not wait on a load after the row loop
+  if (!first && j < Hp)
+    for (int i = ty; i < NV; i += BWD_RY)
+      if (i / 4 < nq) spre[i][tx] = partials[(long)chunk * nq * NG + (long)(i / 4) * NG + c0 + (i % 4) * gs];
   // Per-thread 32-bit element offsets of the first row (one step's tensors: B·4Hp < 2^31, checked by
   // the launcher), advanced by BWD_RY rows per iteration: the row loop's address arithmetic is an
   // add per operand instead of fresh 64-bit products, without holding nine 64-bit pointers
@@ -639,7 +645,7 @@ __global__ void __launch_bounds__(BWD_UX * BWD_RY, 4)
   for (int i = 0; i < NV; ++i) red[ty][i][tx] = acc[i];
   __syncthreads();
   if (j >= Hp) return;
-  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, c0, nq, first, gs);
+  bwd_chunk_finalize<NV>(red, tx, ty, partials + (long)chunk * nq * NG, NG, c0, nq, first, gs, spre);
 }
 
 // K4 backward half, wide form (AV bwd_pw = 1; measured faster at small batch — B = 64: BPTT chain

@@ -82,9 +82,11 @@ __device__ __forceinline__ void lstm_bwd_row(const float (&w)[4], const float (&
 // After every thread of the chunk has stored red[ty][i][tx] = acc[i] and the caller synchronised:
 // thread (tx, ty) finalises quantities i = ty, ty + 4, ... for unit column `col` (gate g at col +
 // g·gs) into the chunk's partials p[q·NG + ...].
+// pre (optional): the old partials p[...] of these items, loaded earlier by the caller (pre[i][tx]).
 template <int NV>
 __device__ __forceinline__ void bwd_chunk_finalize(const float (*red)[NV][BWD_UX], int tx, int ty, float* p, long NG,
-                                                   int col0, int nq, int first, int gs = GATE_U) {
+                                                   int col0, int nq, int first, int gs = GATE_U,
+                                                   const float (*pre)[BWD_UX] = nullptr) {
   for (int i = ty; i < NV; i += BWD_RY) {
     float v = 0.f;
 #pragma unroll
@@ -92,7 +94,7 @@ __device__ __forceinline__ void bwd_chunk_finalize(const float (*red)[NV][BWD_UX
     const int q = i / 4, g = i % 4;
     if (q >= nq) continue;
     float* pp = p + (long)q * NG + col0 + g * gs;
-    *pp = first ? v : __fadd_rn(*pp, v);
+    *pp = first ? v : __fadd_rn(pre ? pre[i][tx] : *pp, v);
   }
 }
 
