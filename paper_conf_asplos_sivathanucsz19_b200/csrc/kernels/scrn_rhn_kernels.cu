@@ -97,12 +97,15 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
                        long ld_dh, int nsplit, long split_stride, const float* __restrict__ Hf, T* __restrict__ DZ,
                        long ldz,
                        float* __restrict__ part, int first) {
-  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
-  pdl_trigger();
   __shared__ float red[PW_RY][PW_UX];
   const int ux = threadIdx.x, ty = threadIdx.y;
   const int j = blockIdx.x * PW_UX + ux;
   const int chunk = blockIdx.y;
+  // the chunk's old db_h partial (the previous step's kernel, 2 launches back): loaded before the
+  // grid dependency so the final fold does not wait on a load
+  const float pold = (!first && ty == 0 && j < Hp) ? part[(long)chunk * Hp + j] : 0.f;
+  pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
+  pdl_trigger();
   const int b0 = chunk * PW_RB, b1 = min(B, b0 + PW_RB);
   float sacc = 0.f;
   if (j < Hp) {
@@ -126,8 +129,7 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
     float v = 0.f;
 #pragma unroll
     for (int y = 0; y < PW_RY; ++y) v = __fadd_rn(v, red[y][ux]);
-    float* p = part + (long)chunk * Hp + j;
-    *p = first ? v : __fadd_rn(*p, v);
+    part[(long)chunk * Hp + j] = first ? v : __fadd_rn(pold, v);
   }
 }
 
@@ -282,6 +284,10 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
   };
   const bool early = ds_part != nullptr;
   if (early) load_old();
+  // this chunk's old db partial (written by an earlier micro-step's kernel, ≥ 2 launches back):
+  // loaded now so the final fold does not wait on a load
+  float pold = 0.f;
+  if (!first && ty < 2 && j < Hp) pold = part[(long)chunk * 2 * Hp + ty * Hp + j];
   pdl_wait();   // chain kernel: launched with PDL (pdl.cuh)
   pdl_trigger();
   if (!early) load_old();
@@ -324,8 +330,7 @@ __global__ void __launch_bounds__(PW_UX * PW_RY)
     float v = 0.f;
 #pragma unroll
     for (int y = 0; y < PW_RY; ++y) v = __fadd_rn(v, red[y][ty][ux]);
-    float* p = part + (long)chunk * 2 * Hp + ty * Hp + j;
-    *p = first ? v : __fadd_rn(*p, v);
+    part[(long)chunk * 2 * Hp + ty * Hp + j] = first ? v : __fadd_rn(pold, v);
   }
 }
 
