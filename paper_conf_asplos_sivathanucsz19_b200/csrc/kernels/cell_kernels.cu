@@ -343,11 +343,10 @@ __device__ __forceinline__ void store_pair(T* p, bool vec, float a, float b, boo
 }
 
 template <int KIND, typename T, typename TY, bool BLK>
-__global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwArgs a) {
+__global__ void __launch_bounds__(FB_THREADS, 3) lstm_fwd_pw_kernel(const FwdPwArgs a) {
   constexpr int NP = KIND == K_MILSTM ? 4 : 1;
   extern __shared__ __align__(128) uint8_t sm[];
-  float* prm = reinterpret_cast<float*>(sm + FB_STAGES * FB_STAGE);   // [NP][4][FB_UB]
-  uint64_t* full = reinterpret_cast<uint64_t*>(prm + NP * 4 * FB_UB);
+  uint64_t* full = reinterpret_cast<uint64_t*>(sm + FB_STAGES * FB_STAGE);
   const int tid = threadIdx.x;
   const int ub = blockIdx.x % a.nub, b_first = blockIdx.x / a.nub;
   const int u0 = ub * FB_UB, nu = min(FB_UB, a.Hp - u0);   // nu: multiple of 64
@@ -393,33 +392,25 @@ __global__ void __launch_bounds__(FB_THREADS, 2) lstm_fwd_pw_kernel(const FwdPwA
   if (tr && tid == 0) tr[1] = gtime_ns();
   if (tid == 0)
     for (int k = 0; k < FB_STAGES && k < nitems; ++k) issue_new(k);
-  for (int i = tid; i < 4 * nu; i += FB_THREADS) {
-    const int g = i / nu, ul = i % nu, j = u0 + ul, e = g * a.H + j;
-    const bool ok = j < a.H;
-    prm[g * FB_UB + ul] = ok ? a.gp.b[e] : 0.f;
-    if (KIND == K_MILSTM) {
-      prm[(NP > 1 ? 1 : 0) * 4 * FB_UB + g * FB_UB + ul] = ok ? a.gp.alpha[e] : 0.f;
-      prm[(NP > 2 ? 2 : 0) * 4 * FB_UB + g * FB_UB + ul] = ok ? a.gp.beta1[e] : 0.f;
-      prm[(NP > 3 ? 3 : 0) * 4 * FB_UB + g * FB_UB + ul] = ok ? a.gp.beta2[e] : 0.f;
-    }
-  }
-  __syncthreads();
+  __syncthreads();   // the ring's barriers are initialised
   const int ul = 2 * tid;
   const bool act = ul < nu;
   const int base = blk ? ul : (ul / 64) * 256 + ul % 64;
   const int gstride = blk ? FB_UB : 64;   // stage offset between a unit's gates
   const bool vh = (a.ldh & 1) == 0, vy = (a.ldy & 1) == 0;
-  // this thread's units keep their gate parameters in registers for all its rows
+  // this thread's units keep their gate parameters in registers for all its rows (loaded straight
+  // from the external vectors: no shared staging, so three CTAs fit on an SM)
   float pb[2][4], pal[2][4], pb1[2][4], pb2[2][4];
 #pragma unroll
   for (int u = 0; u < 2; ++u)
 #pragma unroll
     for (int g = 0; g < 4; ++g) {
-      const int pi = act ? g * FB_UB + ul + u : 0;
-      pb[u][g] = prm[pi];
-      pal[u][g] = KIND == K_MILSTM ? prm[(NP > 1 ? 1 : 0) * 4 * FB_UB + pi] : 0.f;
-      pb1[u][g] = KIND == K_MILSTM ? prm[(NP > 2 ? 2 : 0) * 4 * FB_UB + pi] : 0.f;
-      pb2[u][g] = KIND == K_MILSTM ? prm[(NP > 3 ? 3 : 0) * 4 * FB_UB + pi] : 0.f;
+      const int j = u0 + ul + u, e = g * a.H + j;
+      const bool ok = act && j < a.H;
+      pb[u][g] = ok ? a.gp.b[e] : 0.f;
+      pal[u][g] = (ok && KIND == K_MILSTM) ? a.gp.alpha[e] : 0.f;
+      pb1[u][g] = (ok && KIND == K_MILSTM) ? a.gp.beta1[e] : 0.f;
+      pb2[u][g] = (ok && KIND == K_MILSTM) ? a.gp.beta2[e] : 0.f;
     }
   for (int k = 0; k < nitems; ++k) {
     const int s = k % FB_STAGES;
@@ -495,12 +486,13 @@ static void fwd_pw_launch(OT y_ot, int B, int H, int Hp, const float* WX, const 
     const char* e = std::getenv("ASTRA_FWDPW_CTAS");
     return e ? std::atoi(e) : 0;
   }();
-  a.rstep = std::max(1, std::min(B, (cap > 0 ? cap : 2 * num_sms()) / a.nub));
+  a.rstep = std::max(1, std::min(B, (cap > 0 ? cap : 3 * num_sms()) / a.nub));
   a.WX = WX; a.UH = UH; a.gp = gp; a.c_prev = c_prev; a.c_new = c_new;
   a.h_op = h_op; a.ldh = ldh; a.y = y; a.ldy = ldy; a.hT = hT; a.cT = cT;
   a.trace = trace_buffer(TRACE_FWD_PW);   // diagnostics only (null: no stamps)
   const int np = KIND == K_MILSTM ? 4 : 1;
-  const size_t smem = (size_t)FB_STAGES * FB_STAGE + (size_t)np * 4 * FB_UB * 4 + FB_STAGES * 8;
+  (void)np;
+  const size_t smem = (size_t)FB_STAGES * FB_STAGE + FB_STAGES * 8;
   const dim3 grid(a.nub * a.rstep);
   if (y_ot == OT::BF16) {
     auto k = blk ? lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16, true> : lstm_fwd_pw_kernel<KIND, T, __nv_bfloat16, false>;
