@@ -482,6 +482,14 @@ def test_attn_ragged(dtype, tol):
     _attn_check(7, 3, 20, 40, 100, 72, dtype, synth.config_seed(4) + 2, tol)
 
 
+@pytest.mark.parametrize("H,A", [(512, 256), (1024, 512)])
+def test_attn_split_bptt_vs_oracle(H, A):
+    """Reading R42: the decoder's per-step BPTT GEMMs split into 2 (4Hp = 2048) and 4 (4Hp = 4096)
+    K chunks — partials summed in chunk order by the attention backward and the pointwise kernel,
+    dq·W_qᵀ accumulated chunk by chunk — match the oracle, with a ragged batch."""
+    _attn_check(5, 4, 72, 64, H, A, "bf16", synth.config_seed(4) + 9, TOL_BF16)
+
+
 def test_attn_cfg4_reduced():
     """cfg4 reduced rung: H = A = I = 1024, B = 128, Ts = Tt = 8 (bf16)."""
     _attn_check(8, 8, 128, 1024, 1024, 1024, "bf16", synth.config_seed(4), TOL_BF16)
